@@ -1,0 +1,201 @@
+/*
+ * dp.h — C ABI of the B200-native DREAMPlace objective/gradient evaluation library (libdp).
+ *
+ * One call evaluates the global-placement objective of eq (2)
+ *     obj = sum_e w_e WA_e(x, y)  +  lambda * D(x, y)
+ * and its gradient with respect to every cell's lower-left corner, where
+ *   - WA_e is the weighted-average wirelength of eq (3) with the overflow-safe shift
+ *     of P:159 and the gradient of eq (6), evaluated net-parallel, x and y fused;
+ *   - D is the electrostatic density energy of the ePlace model: the four steps of
+ *     density map, DCT spectrum a_uv (eqs 5a/9a), potential and field
+ *     (eqs 5b-d / 9b-d via eqs 7-8), force gather.
+ * Readings of passages the paper leaves silent or garbled are listed in DESIGN.md §3 and are
+ * cited below as A1..A26.
+ *
+ * Conventions
+ *   - All functions return dp_status; nothing throws across the ABI.  On failure
+ *     dp_last_error() returns a thread-local, NUL-terminated message (valid until the next
+ *     call on the same thread).
+ *   - "device" pointers are CUDA device (or managed) pointers on the context's device;
+ *     "host" pointers are ordinary host memory (pinned memory is faster for dp_eval_host).
+ *   - dp_stream_t is a cudaStream_t passed as void* (NULL = the legacy default stream).
+ *     Evaluation calls only enqueue work on that stream and never synchronise the host
+ *     (except dp_eval_host), so they may be captured into CUDA graphs by the caller.
+ *   - Scalar outputs (double*) are DEVICE pointers written on-stream; NULL skips the output.
+ *   - Coordinates: x[c], y[c] are the lower-left corner of cell c in the grid's length
+ *     units; pin location = (x[c] + pin_dx[p], y[c] + pin_dy[p])  (reading A1).
+ *   - Gradients gx, gy are OVERWRITTEN (not accumulated).
+ *   - One context may be used by one stream at a time (it owns scratch buffers).
+ *     Different contexts are independent.
+ *   - The library runs only on sm_100a (B200).  There is no CPU fallback: without a usable
+ *     device every call that needs one returns DP_ERR_CUDA.
+ */
+#ifndef DP_H_
+#define DP_H_
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum dp_status {
+    DP_OK = 0,
+    DP_ERR_INVALID_ARG = 1,   /* null pointer, bad CSR, gamma <= 0, lambda < 0, ...         */
+    DP_ERR_UNSUPPORTED = 2,   /* valid input outside what this build implements (bin counts) */
+    DP_ERR_OUT_OF_MEMORY = 3, /* device or host allocation failed                             */
+    DP_ERR_CUDA = 4,          /* a CUDA runtime error (no device, launch failure, ...)         */
+    DP_ERR_NCCL = 5           /* NCCL missing or a collective failed (distributed contexts)    */
+} dp_status;
+
+typedef void *dp_stream_t;     /* cudaStream_t */
+typedef struct dp_ctx dp_ctx;  /* opaque */
+
+/* The hypergraph H = (V, E) of P:27 in CSR form, plus per-pin offsets and cell sizes.
+ * All arrays are HOST arrays; dp_create deep-copies them (the caller may free them after
+ * dp_create returns).                                                                    */
+typedef struct dp_netlist {
+    int32_t num_cells;         /* |V| >= 1                                                 */
+    int32_t num_nets;          /* |E| >= 0                                                 */
+    int32_t num_pins;          /* |P| >= 0, < 2^31                                         */
+    const int32_t *net_start;  /* [num_nets+1]; net_start[0] = 0, nondecreasing,
+                                  net_start[num_nets] = num_pins.  Net e owns pin slots
+                                  net_start[e] .. net_start[e+1]-1                          */
+    const int32_t *net2pin;    /* [num_pins] permutation mapping slot -> pin id, or NULL
+                                  (identity: pins already stored in net order)              */
+    const int32_t *pin2cell;   /* [num_pins] indexed by pin id; values in [0, num_cells)    */
+    const float *pin_dx;       /* [num_pins] pin offset from the cell's lower-left corner   */
+    const float *pin_dy;       /* [num_pins]                                               */
+    const float *cell_w;       /* [num_cells] finite, >= 0                                 */
+    const float *cell_h;       /* [num_cells] finite, >= 0                                 */
+    const float *net_weight;   /* [num_nets] finite, >= 0, or NULL (all 1).  Scales WL_e
+                                  and its gradient (reading A4); HPWL is unweighted         */
+} dp_netlist;
+
+/* The placement region [xl, xh] x [yl, yh] split into bins_x x bins_y bins.
+ * Maps are stored [bins_x][bins_y], y contiguous (reading A20).
+ * This build supports bins_x, bins_y powers of two in [16, 4096] (even lengths are what
+ * Alg 3 requires; reading A23); anything else -> DP_ERR_UNSUPPORTED.
+ * stretch = 1: cells smaller than sqrt(2) bins are stretched to sqrt(2) bins with their
+ * charge scaled to keep the area (reading A10); stretch = 0: literal overlap.       */
+typedef struct dp_grid {
+    double xl, yl, xh, yh;     /* xh > xl, yh > yl, finite                                 */
+    int32_t bins_x, bins_y;
+    int32_t stretch;           /* 0 or 1                                                   */
+} dp_grid;
+
+/* Thread-local message describing the last failure on this thread ("" if none). */
+const char *dp_last_error(void);
+
+/* Library version (major*10000 + minor*100 + patch). */
+int32_t dp_version(void);
+
+/* Validate the netlist and grid, copy them to `device`, reorder pins into the kernels'
+ * layout (degree-binned, locality-sorted nets), precompute the per-cell stretched footprint
+ * sizes and transform twiddles, allocate scratch.  One-time host-side cost.
+ * Errors: DP_ERR_INVALID_ARG (null, CSR not monotone / out of range, sizes negative or
+ * non-finite, degenerate region, stretch not 0/1), DP_ERR_UNSUPPORTED (bin counts),
+ * DP_ERR_OUT_OF_MEMORY, DP_ERR_CUDA.  *out is set only on success.                       */
+dp_status dp_create(const dp_netlist *nl, const dp_grid *grid, int device, dp_ctx **out);
+
+/* Distributed context for rank `rank` of `world` (one process per GPU).  Every rank passes
+ * the full netlist; the library keeps the cells [cell_begin, cell_end) of this rank
+ * (contiguous, balanced) and every net with at least one pin on them ("owner computes":
+ * a net cut by the partition is evaluated on each rank it touches, each rank writes only
+ * its own cells' gradient, and WA / HPWL of a net are counted once, on the rank owning the
+ * net's first pin).  The density map is summed over ranks with one ncclAllReduce per
+ * evaluation; the Poisson solve is replicated.  nccl_unique_id: 128-byte ncclUniqueId from
+ * dp_nccl_unique_id() on rank 0, broadcast by the caller (e.g. torch.distributed); NULL
+ * builds a "virtual shard" whose collectives are skipped (tests on one GPU).
+ * In a distributed context gx, gy are written only on [cell_begin, cell_end) and the
+ * scalar outputs are global (summed over ranks).                                         */
+dp_status dp_create_dist(const dp_netlist *nl, const dp_grid *grid, int device, int rank,
+                         int world, const void *nccl_unique_id, dp_ctx **out);
+
+/* Fill out128 (128 bytes, host) with a fresh ncclUniqueId (NCCL loaded at run time). */
+dp_status dp_nccl_unique_id(void *out128);
+
+/* Host-only partition plan used by dp_create_dist (no GPU needed; exposed for tests).
+ * cell range of `rank` -> *cell_begin, *cell_end.  net_mask (host, [num_nets], nullable)
+ * receives per net: 0 = not evaluated on this rank, 1 = evaluated (gradient for own cells
+ * only), 3 = evaluated and counted (WA, HPWL) on this rank.                               */
+dp_status dp_partition_plan(const dp_netlist *nl, int rank, int world, int32_t *cell_begin,
+                            int32_t *cell_end, uint8_t *net_mask);
+
+/* Free everything the context owns.  NULL is accepted. */
+dp_status dp_destroy(dp_ctx *ctx);
+
+/* Full evaluation (eq 2):
+ *   gx, gy   (device, [num_cells]) <- dWA/dx + lambda dD/dx,  dWA/dy + lambda dD/dy
+ *   d_obj    (device double, nullable) <- WA + lambda D
+ *   d_wl     (device double, nullable) <- WA = sum_e w_e (WL_e^x + WL_e^y)
+ *   d_energy (device double, nullable) <- D = 1/2 b_x b_y sum_b rho_b psi_b   (reading A8)
+ *   d_hpwl   (device double, nullable) <- HPWL, correctly rounded fp64 (reading A7); NULL
+ *            skips it (the fused HPWL costs one extra int64 limb reduction)
+ * gamma > 0 (length units, reading A5), lambda >= 0, finite.  x, y, gx, gy must not alias.
+ * Errors: DP_ERR_INVALID_ARG, DP_ERR_CUDA, DP_ERR_NCCL.                                  */
+dp_status dp_eval(dp_ctx *ctx, const float *x, const float *y, float gamma, float lambda,
+                  float *gx, float *gy, double *d_obj, double *d_wl, double *d_energy,
+                  double *d_hpwl, dp_stream_t stream);
+
+/* WA wirelength only (eqs 3, 6): gx, gy <- dWA/dx, dWA/dy; d_wl <- WA.                    */
+dp_status dp_wl_grad(dp_ctx *ctx, const float *x, const float *y, float gamma, float *gx,
+                     float *gy, double *d_wl, dp_stream_t stream);
+
+/* Density only: gx, gy <- dD/dx, dD/dy; d_energy <- D.                        */
+dp_status dp_density_grad(dp_ctx *ctx, const float *x, const float *y, float *gx, float *gy,
+                          double *d_energy, dp_stream_t stream);
+
+/* Standalone HPWL (reading A6/A7), correctly rounded fp64.                                */
+dp_status dp_hpwl(dp_ctx *ctx, const float *x, const float *y, double *d_hpwl,
+                  dp_stream_t stream);
+
+/* End-to-end variant of dp_eval on HOST buffers: copies x, y host->device, evaluates,
+ * copies gx, gy and the four scalars device->host, and synchronises `stream` before
+ * returning.  h_scalars (host, [4], nullable) <- {obj, wl, energy, hpwl}; with_hpwl = 0
+ * skips HPWL (h_scalars[3] = NaN).                                                        */
+dp_status dp_eval_host(dp_ctx *ctx, const float *hx, const float *hy, float gamma,
+                       float lambda, float *hgx, float *hgy, double *h_scalars,
+                       int with_hpwl, dp_stream_t stream);
+
+/* ---- introspection -------------------------------------------------------------------- */
+typedef struct dp_info {
+    int32_t num_cells, num_nets, num_pins;       /* as stored on this rank                 */
+    int32_t cell_begin, cell_end;                /* owned cells ([0, num_cells) if 1 rank) */
+    int32_t bins_x, bins_y;
+    int32_t rank, world;
+    int32_t launches_eval;       /* kernels launched by one dp_eval (d_hpwl = NULL)        */
+    int32_t launches_eval_hpwl;  /* ... with d_hpwl != NULL                                */
+    int64_t device_bytes;        /* device memory owned by the context                     */
+    int32_t num_sms;
+    int32_t l2_bytes;
+} dp_info;
+
+dp_status dp_get_info(const dp_ctx *ctx, dp_info *info);
+
+/* ---- test-only hooks (not part of the metric) ------------------------------------------
+ * Expose single stages so parity tests can localise a failure.  All pointers device.     */
+
+/* rho (device, [bins_x*bins_y]) <- the density map of step 1.                     */
+dp_status dp_debug_density_map(dp_ctx *ctx, const float *x, const float *y, float *rho,
+                               dp_stream_t stream);
+
+/* From a given map rho: psi, xi_x, xi_y (device, [bins_x*bins_y], each nullable)
+ * <- eqs 9b-9d;  d_energy (device double, nullable) <- 1/2 b_x b_y sum rho psi
+ * (computed spectrally by Parseval, the way dp_eval does).                                */
+dp_status dp_debug_fields(dp_ctx *ctx, const float *rho, float *psi, float *xi_x, float *xi_y,
+                          double *d_energy, dp_stream_t stream);
+
+/* Single 2-D transform of a bins_x x bins_y map (device in/out, may not alias):
+ *   DP_T_DCT2       a = DCT_x DCT_y (in)         (eq 9a, 2/N per axis, reading A13)
+ *   DP_T_IDCT2      IDCT_x IDCT_y (in)           (eq 9b without the scaling)
+ *   DP_T_IDXST_IDCT IDXST_x IDCT_y (in)          (eq 9c without the scaling)
+ *   DP_T_IDCT_IDXST IDCT_x IDXST_y (in)          (eq 9d without the scaling)          */
+enum { DP_T_DCT2 = 0, DP_T_IDCT2 = 1, DP_T_IDXST_IDCT = 2, DP_T_IDCT_IDXST = 3 };
+dp_status dp_debug_transform(dp_ctx *ctx, int kind, const float *in, float *out,
+                             dp_stream_t stream);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* DP_H_ */

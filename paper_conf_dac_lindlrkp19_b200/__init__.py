@@ -1,0 +1,308 @@
+"""B200-native DREAMPlace objective/gradient evaluation — Python binding of libdp.
+
+Thin ctypes marshalling over the C ABI declared in include/dp.h (same function names).
+Every step of the evaluation runs in libdp's sm_100a kernels; torch is used only for device
+memory (tensors), streams and torch.distributed bootstrap.  There is no CPU fallback: if
+libdp.so is missing or no B200 is present, the calls raise.
+
+    from paper_conf_dac_lindlrkp19_b200 import dp_create
+    ctx = dp_create(netlist)                       # synth.Netlist or any object with the fields
+    out = ctx.eval(x, y, gamma, lam)               # x, y: float32 CUDA tensors [num_cells]
+    out["gx"], out["gy"], out["obj"], out["wl"], out["energy"]
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+from .build import LIB, build  # noqa: F401
+
+__all__ = [
+    "DPError", "Context", "lib", "dp_create", "dp_create_dist", "dp_nccl_unique_id",
+    "dp_partition_plan", "dp_eval", "dp_wl_grad", "dp_density_grad", "dp_hpwl", "dp_eval_host",
+    "dp_get_info", "dp_debug_density_map", "dp_debug_fields", "dp_debug_transform",
+    "DP_T_DCT2", "DP_T_IDCT2", "DP_T_IDXST_IDCT", "DP_T_IDCT_IDXST", "EXPORTED_SYMBOLS",
+]
+
+DP_T_DCT2, DP_T_IDCT2, DP_T_IDXST_IDCT, DP_T_IDCT_IDXST = 0, 1, 2, 3
+_STATUS = {0: "DP_OK", 1: "DP_ERR_INVALID_ARG", 2: "DP_ERR_UNSUPPORTED", 3: "DP_ERR_OUT_OF_MEMORY",
+           4: "DP_ERR_CUDA", 5: "DP_ERR_NCCL"}
+
+EXPORTED_SYMBOLS = [
+    "dp_last_error", "dp_version", "dp_create", "dp_create_dist", "dp_nccl_unique_id",
+    "dp_partition_plan", "dp_destroy", "dp_eval", "dp_wl_grad", "dp_density_grad", "dp_hpwl",
+    "dp_eval_host", "dp_get_info", "dp_debug_density_map", "dp_debug_fields", "dp_debug_transform",
+]
+
+
+class DPError(RuntimeError):
+    def __init__(self, status: int, msg: str):
+        super().__init__(f"{_STATUS.get(status, status)}: {msg}")
+        self.status = status
+
+
+P = ctypes.c_void_p
+I32 = ctypes.c_int32
+
+
+class DpNetlist(ctypes.Structure):
+    _fields_ = [("num_cells", I32), ("num_nets", I32), ("num_pins", I32),
+                ("net_start", P), ("net2pin", P), ("pin2cell", P), ("pin_dx", P), ("pin_dy", P),
+                ("cell_w", P), ("cell_h", P), ("net_weight", P)]
+
+
+class DpGrid(ctypes.Structure):
+    _fields_ = [("xl", ctypes.c_double), ("yl", ctypes.c_double), ("xh", ctypes.c_double),
+                ("yh", ctypes.c_double), ("bins_x", I32), ("bins_y", I32), ("stretch", I32)]
+
+
+class DpInfo(ctypes.Structure):
+    _fields_ = [("num_cells", I32), ("num_nets", I32), ("num_pins", I32), ("cell_begin", I32),
+                ("cell_end", I32), ("bins_x", I32), ("bins_y", I32), ("rank", I32), ("world", I32),
+                ("launches_eval", I32), ("launches_eval_hpwl", I32), ("device_bytes", ctypes.c_int64),
+                ("num_sms", I32), ("l2_bytes", I32)]
+
+
+_lib = None
+
+
+def lib() -> ctypes.CDLL:
+    """Load libdp.so (built in-tree by build()).  Raises if it is missing: no fallback."""
+    global _lib
+    if _lib is None:
+        if not os.path.exists(LIB):
+            raise RuntimeError(f"libdp.so not built ({LIB}); run paper_conf_dac_lindlrkp19_b200.build.build()")
+        L = ctypes.CDLL(LIB)
+        L.dp_last_error.restype = ctypes.c_char_p
+        L.dp_version.restype = I32
+        for name, args in {
+            "dp_create": [ctypes.POINTER(DpNetlist), ctypes.POINTER(DpGrid), ctypes.c_int, ctypes.POINTER(P)],
+            "dp_create_dist": [ctypes.POINTER(DpNetlist), ctypes.POINTER(DpGrid), ctypes.c_int, ctypes.c_int,
+                               ctypes.c_int, P, ctypes.POINTER(P)],
+            "dp_nccl_unique_id": [P],
+            "dp_partition_plan": [ctypes.POINTER(DpNetlist), ctypes.c_int, ctypes.c_int, ctypes.POINTER(I32),
+                                  ctypes.POINTER(I32), P],
+            "dp_destroy": [P],
+            "dp_eval": [P, P, P, ctypes.c_float, ctypes.c_float, P, P, P, P, P, P, P],
+            "dp_wl_grad": [P, P, P, ctypes.c_float, P, P, P, P],
+            "dp_density_grad": [P, P, P, P, P, P, P],
+            "dp_hpwl": [P, P, P, P, P],
+            "dp_eval_host": [P, P, P, ctypes.c_float, ctypes.c_float, P, P, P, ctypes.c_int, P],
+            "dp_get_info": [P, ctypes.POINTER(DpInfo)],
+            "dp_debug_density_map": [P, P, P, P, P],
+            "dp_debug_fields": [P, P, P, P, P, P, P],
+            "dp_debug_transform": [P, ctypes.c_int, P, P, P],
+        }.items():
+            f = getattr(L, name)
+            f.argtypes = args
+            f.restype = ctypes.c_int
+        _lib = L
+    return _lib
+
+
+def _check(st: int):
+    if st != 0:
+        raise DPError(st, lib().dp_last_error().decode(errors="replace"))
+
+
+def _ptr(t):
+    """Device/host address of a torch tensor, numpy array, or None."""
+    if t is None:
+        return None
+    if hasattr(t, "data_ptr"):
+        return ctypes.c_void_p(t.data_ptr())
+    if hasattr(t, "ctypes"):
+        return t.ctypes.data_as(ctypes.c_void_p)
+    return ctypes.c_void_p(int(t))
+
+
+def _stream(stream):
+    if stream is None:
+        import torch
+        return ctypes.c_void_p(torch.cuda.current_stream().cuda_stream)
+    if hasattr(stream, "cuda_stream"):
+        return ctypes.c_void_p(stream.cuda_stream)
+    return ctypes.c_void_p(int(stream))
+
+
+def _netlist_struct(nl):
+    import numpy as np
+    keep = []
+
+    def arr(a, dt):
+        if a is None:
+            return None
+        a = np.ascontiguousarray(a, dtype=dt)
+        keep.append(a)
+        return a.ctypes.data_as(ctypes.c_void_p)
+
+    s = DpNetlist(num_cells=int(nl.num_cells), num_nets=int(nl.num_nets), num_pins=int(nl.num_pins),
+                  net_start=arr(nl.net_start, np.int32), net2pin=arr(getattr(nl, "net2pin", None), np.int32),
+                  pin2cell=arr(nl.pin2cell, np.int32), pin_dx=arr(nl.pin_dx, np.float32),
+                  pin_dy=arr(nl.pin_dy, np.float32), cell_w=arr(nl.cell_w, np.float32),
+                  cell_h=arr(nl.cell_h, np.float32), net_weight=arr(getattr(nl, "net_weight", None), np.float32))
+    return s, keep
+
+
+def _grid_struct(nl, stretch):
+    return DpGrid(xl=float(nl.xl), yl=float(nl.yl), xh=float(nl.xh), yh=float(nl.yh),
+                  bins_x=int(nl.bins_x), bins_y=int(nl.bins_y), stretch=int(stretch))
+
+
+class Context:
+    """Owns a dp_ctx*.  Methods allocate outputs as torch tensors for convenience."""
+
+    def __init__(self, handle, nl, device):
+        self.handle = handle
+        self.num_cells = int(nl.num_cells)
+        self.bins = (int(nl.bins_x), int(nl.bins_y))
+        self.device = device
+        self.info = dp_get_info(self)
+
+    def close(self):
+        if self.handle:
+            lib().dp_destroy(self.handle)
+            self.handle = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def _dev(self):
+        import torch
+        return torch.device("cuda", self.device)
+
+    def eval(self, x, y, gamma, lam, with_hpwl=False, gx=None, gy=None, stream=None):
+        import torch
+        gx = torch.empty(self.num_cells, dtype=torch.float32, device=self._dev()) if gx is None else gx
+        gy = torch.empty(self.num_cells, dtype=torch.float32, device=self._dev()) if gy is None else gy
+        sc = torch.full((4,), float("nan"), dtype=torch.float64, device=self._dev())
+        dp_eval(self, x, y, gamma, lam, gx, gy, sc[0:1], sc[1:2], sc[2:3], sc[3:4] if with_hpwl else None,
+                stream)
+        return dict(gx=gx, gy=gy, obj=sc[0], wl=sc[1], energy=sc[2], hpwl=sc[3], scalars=sc)
+
+    def wl_grad(self, x, y, gamma, stream=None):
+        import torch
+        gx = torch.empty(self.num_cells, dtype=torch.float32, device=self._dev())
+        gy = torch.empty_like(gx)
+        wl = torch.zeros(1, dtype=torch.float64, device=self._dev())
+        dp_wl_grad(self, x, y, gamma, gx, gy, wl, stream)
+        return dict(gx=gx, gy=gy, wl=wl[0])
+
+    def density_grad(self, x, y, stream=None):
+        import torch
+        gx = torch.empty(self.num_cells, dtype=torch.float32, device=self._dev())
+        gy = torch.empty_like(gx)
+        en = torch.zeros(1, dtype=torch.float64, device=self._dev())
+        dp_density_grad(self, x, y, gx, gy, en, stream)
+        return dict(gx=gx, gy=gy, energy=en[0])
+
+    def hpwl(self, x, y, stream=None):
+        import torch
+        h = torch.zeros(1, dtype=torch.float64, device=self._dev())
+        dp_hpwl(self, x, y, h, stream)
+        return h[0]
+
+    def density_map(self, x, y, stream=None):
+        import torch
+        rho = torch.empty(self.bins, dtype=torch.float32, device=self._dev())
+        dp_debug_density_map(self, x, y, rho, stream)
+        return rho
+
+    def fields(self, rho, want_psi=True, stream=None):
+        import torch
+        psi = torch.empty(self.bins, dtype=torch.float32, device=self._dev()) if want_psi else None
+        xx = torch.empty(self.bins, dtype=torch.float32, device=self._dev())
+        xy = torch.empty_like(xx)
+        en = torch.zeros(1, dtype=torch.float64, device=self._dev())
+        dp_debug_fields(self, rho, psi, xx, xy, en, stream)
+        return dict(psi=psi, xi_x=xx, xi_y=xy, energy=en[0])
+
+    def transform(self, kind, inp, stream=None):
+        import torch
+        out = torch.empty(self.bins, dtype=torch.float32, device=self._dev())
+        dp_debug_transform(self, kind, inp, out, stream)
+        return out
+
+
+# ---- functions with the C names -----------------------------------------------------------
+def dp_create(nl, device: int = 0, stretch: int = 1) -> Context:
+    s, keep = _netlist_struct(nl)
+    g = _grid_struct(nl, stretch)
+    h = ctypes.c_void_p()
+    _check(lib().dp_create(ctypes.byref(s), ctypes.byref(g), int(device), ctypes.byref(h)))
+    del keep
+    return Context(h, nl, device)
+
+
+def dp_create_dist(nl, device: int, rank: int, world: int, nccl_unique_id: bytes | None,
+                   stretch: int = 1) -> Context:
+    s, keep = _netlist_struct(nl)
+    g = _grid_struct(nl, stretch)
+    h = ctypes.c_void_p()
+    idbuf = None if nccl_unique_id is None else ctypes.create_string_buffer(bytes(nccl_unique_id), 128)
+    _check(lib().dp_create_dist(ctypes.byref(s), ctypes.byref(g), int(device), int(rank), int(world),
+                                idbuf, ctypes.byref(h)))
+    del keep
+    return Context(h, nl, device)
+
+
+def dp_nccl_unique_id() -> bytes:
+    buf = ctypes.create_string_buffer(128)
+    _check(lib().dp_nccl_unique_id(buf))
+    return buf.raw
+
+
+def dp_partition_plan(nl, rank: int, world: int):
+    import numpy as np
+    s, keep = _netlist_struct(nl)
+    cb, ce = I32(), I32()
+    mask = np.zeros(max(int(nl.num_nets), 1), dtype=np.uint8)
+    _check(lib().dp_partition_plan(ctypes.byref(s), int(rank), int(world), ctypes.byref(cb), ctypes.byref(ce),
+                                   mask.ctypes.data_as(ctypes.c_void_p)))
+    return cb.value, ce.value, mask[: int(nl.num_nets)]
+
+
+def dp_eval(ctx, x, y, gamma, lam, gx, gy, d_obj=None, d_wl=None, d_energy=None, d_hpwl=None, stream=None):
+    _check(lib().dp_eval(ctx.handle, _ptr(x), _ptr(y), float(gamma), float(lam), _ptr(gx), _ptr(gy),
+                         _ptr(d_obj), _ptr(d_wl), _ptr(d_energy), _ptr(d_hpwl), _stream(stream)))
+
+
+def dp_wl_grad(ctx, x, y, gamma, gx, gy, d_wl=None, stream=None):
+    _check(lib().dp_wl_grad(ctx.handle, _ptr(x), _ptr(y), float(gamma), _ptr(gx), _ptr(gy), _ptr(d_wl),
+                            _stream(stream)))
+
+
+def dp_density_grad(ctx, x, y, gx, gy, d_energy=None, stream=None):
+    _check(lib().dp_density_grad(ctx.handle, _ptr(x), _ptr(y), _ptr(gx), _ptr(gy), _ptr(d_energy),
+                                 _stream(stream)))
+
+
+def dp_hpwl(ctx, x, y, d_hpwl, stream=None):
+    _check(lib().dp_hpwl(ctx.handle, _ptr(x), _ptr(y), _ptr(d_hpwl), _stream(stream)))
+
+
+def dp_eval_host(ctx, hx, hy, gamma, lam, hgx, hgy, h_scalars=None, with_hpwl=False, stream=None):
+    _check(lib().dp_eval_host(ctx.handle, _ptr(hx), _ptr(hy), float(gamma), float(lam), _ptr(hgx), _ptr(hgy),
+                              _ptr(h_scalars), int(bool(with_hpwl)), _stream(stream)))
+
+
+def dp_get_info(ctx) -> DpInfo:
+    info = DpInfo()
+    _check(lib().dp_get_info(ctx.handle, ctypes.byref(info)))
+    return info
+
+
+def dp_debug_density_map(ctx, x, y, rho, stream=None):
+    _check(lib().dp_debug_density_map(ctx.handle, _ptr(x), _ptr(y), _ptr(rho), _stream(stream)))
+
+
+def dp_debug_fields(ctx, rho, psi, xi_x, xi_y, d_energy=None, stream=None):
+    _check(lib().dp_debug_fields(ctx.handle, _ptr(rho), _ptr(psi), _ptr(xi_x), _ptr(xi_y), _ptr(d_energy),
+                                 _stream(stream)))
+
+
+def dp_debug_transform(ctx, kind, inp, out, stream=None):
+    _check(lib().dp_debug_transform(ctx.handle, int(kind), _ptr(inp), _ptr(out), _stream(stream)))

@@ -1,0 +1,406 @@
+// dct.cu — DCT / IDCT / IDXST transforms and the spectral Poisson solve on sm_100a.
+//
+// Method: potential and field by eqs (5a)-(5d) computed as the
+// separable transforms of eqs (9a)-(9d) built from the 1-D DCT of eq (7a),
+// IDCT of eq (7b) and IDXST of eq (8a)/(8e); N-point FFT evaluation in the
+// spirit of Alg 3 (Makhoul [32]).  Readings: A12 (wavenumbers k = pi u / W),
+// A13 (2/N per axis), A14 (half weight of the u = 0 term), A15 (DC term dropped),
+// A16/A17 (the garbled eqs 11/12 are not used: every transform here is checked against the
+// naive eq 7/8 definitions), A20 (1-D ops along y = the contiguous axis first).
+//
+// B200 design: the three transforms of a density evaluation are three
+// kernels over maps that stay L2-resident:
+//   T1  rows:     DCT over y of rho                                   -> t
+//   T2  columns:  DCT over x of t, spectral scaling, Parseval energy, and BOTH inverse
+//                 column transforms (IDXST_x of a k_u/k^2, IDCT_x of a k_v/k^2)  -> sX, sY
+//   T3  rows:     IDCT_y of sX and IDXST_y of sY, written interleaved (xi_X, xi_Y)
+// Two real sequences always share one complex FFT (z = p + i q).  The FFT is a shared-memory
+// radix-2 DIT with bit-reversed loads and fp32 twiddles computed in fp64 at create.
+// The energy D = 1/2 b_x b_y sum rho psi is taken in the spectral domain (Parseval), so psi
+// is never materialised on the hot path (reading A8).
+#include "dp_internal.h"
+
+namespace dp {
+
+namespace {
+
+constexpr int kRowThreads = 256;
+constexpr int kColThreads = 256;
+// columns per CTA in the column kernels (even: pairs share a complex FFT); sized so the
+// shared-memory slab fits: 8 up to 1024 rows, 4 at 2048, 2 at 4096
+__host__ __device__ inline int col_slab(int mx) { return mx <= 1024 ? 8 : (mx <= 2048 ? 4 : 2); }
+
+__device__ __forceinline__ float2 cmul(float2 a, float2 b) {
+  return make_float2(a.x * b.x - a.y * b.y, a.x * b.y + a.y * b.x);
+}
+__device__ __forceinline__ int brev(int n, int log2n) { return (int)(__brev((unsigned)n) >> (32 - log2n)); }
+// Makhoul reordering (Alg 3 lines 3-8): v[n] = x[2n], v[N-1-n] = x[2n+1]; position of x[t] in v
+__device__ __forceinline__ int mk_pos(int t, int n) { return (t & 1) ? n - ((t + 1) >> 1) : (t >> 1); }
+
+// In-place radix-2 DIT FFT of nseq sequences of length n = 2^log2n stored back to back in
+// buf, input already in bit-reversed order.  tw[k] = exp(-2 pi i k / n), k < n/2.
+// inverse = true uses conjugate twiddles (unnormalised inverse DFT).
+__device__ void fft_block(float2 *buf, int n, int log2n, int nseq, const float2 *__restrict__ tw,
+                          bool inverse) {
+  const int half_n = n >> 1, total = nseq * half_n;
+  for (int s = 1; s <= log2n; s++) {
+    const int half = 1 << (s - 1), len = half << 1, tstride = n >> s;
+    for (int b = threadIdx.x; b < total; b += blockDim.x) {
+      const int seq = b >> (log2n - 1), r = b & (half_n - 1);
+      const int grp = r >> (s - 1), k = r & (half - 1);
+      const int i = seq * n + grp * len + k, jx = i + half;
+      float2 w = __ldg(tw + k * tstride);
+      if (inverse) w.y = -w.y;
+      const float2 u = buf[i], v = cmul(w, buf[jx]);
+      buf[i] = make_float2(u.x + v.x, u.y + v.y);
+      buf[jx] = make_float2(u.x - v.x, u.y - v.y);
+    }
+    __syncthreads();
+  }
+}
+
+// Forward DCT post-processing for a pair packed as z = p + i q (Alg 3 lines 10-16, split
+// of the two real spectra): returns (DCT(p)_k, DCT(q)_k) with the 2/N factor (reading A13).
+__device__ __forceinline__ float2 dct_post(const float2 *Z, int k, int n, float2 ph, float scale) {
+  const float2 z = Z[k], zc = Z[(n - k) & (n - 1)];
+  // V0 = (z + conj zc)/2, V1 = (z - conj zc) * (-i/2)
+  const float v0x = 0.5f * (z.x + zc.x), v0y = 0.5f * (z.y - zc.y);
+  const float dx = z.x - zc.x, dy = z.y + zc.y;
+  const float v1x = 0.5f * dy, v1y = -0.5f * dx;
+  // Re(V e^{-i pi k / 2N}), ph = (cos, -sin)
+  return make_float2(scale * (v0x * ph.x - v0y * ph.y), scale * (v1x * ph.x - v1y * ph.y));
+}
+
+// Inverse pre-processing for two IDCT-type sequences p (real part) and q (imag part), both
+// already reversed if they are IDXST inputs (eq 8e):  Z_k = e^{+i pi k/2N} [(p_k + q_{N-k})
+// + i (q_k - p_{N-k})] with p_N = q_N = 0.  ph = e^{-i pi k/2N} (conjugated here).
+__device__ __forceinline__ float2 inv_pre(float pk, float qk, float pnk, float qnk, float2 ph) {
+  const float re = pk + qnk, im = qk - pnk;
+  return make_float2(re * ph.x + im * ph.y, im * ph.x - re * ph.y);
+}
+
+// ---------------------------------------------------------------------------------------
+// T1 / debug: forward DCT over rows, rows (2r, 2r+1) share one complex FFT.
+// ---------------------------------------------------------------------------------------
+__global__ void __launch_bounds__(kRowThreads) k_row_dct(const float *__restrict__ in, float *__restrict__ out,
+                                                         int n, int log2n, const float2 *__restrict__ tw,
+                                                         const float2 *__restrict__ ph) {
+  extern __shared__ float2 zbuf[];
+  const float *r0 = in + (size_t)(2 * blockIdx.x) * n, *r1 = r0 + n;
+  for (int t = threadIdx.x; t < n; t += kRowThreads)
+    zbuf[brev(mk_pos(t, n), log2n)] = make_float2(__ldg(r0 + t), __ldg(r1 + t));
+  __syncthreads();
+  fft_block(zbuf, n, log2n, 1, tw, false);
+  float *o0 = out + (size_t)(2 * blockIdx.x) * n, *o1 = o0 + n;
+  const float scale = 2.f / n;
+  for (int k = threadIdx.x; k < n; k += kRowThreads) {
+    const float2 v = dct_post(zbuf, k, n, __ldg(ph + k), scale);
+    o0[k] = v.x;
+    o1[k] = v.y;
+  }
+}
+
+// ---------------------------------------------------------------------------------------
+// T3 / debug: inverse over rows.  Row r of A (op opA) and row r of B (op opB) share one
+// complex IFFT.  op: 1 = IDCT (eq 7b), 2 = IDXST (eq 8a via 8e).  Output either two planes
+// or one interleaved float2 plane (xi_X, xi_Y).
+// ---------------------------------------------------------------------------------------
+struct RowInvArgs {
+  const float *inA, *inB;
+  long long stepA, stepB;   // row r of A at inA + r * stepA
+  int opA, opB;
+  float *outA, *outB;       // planes (row step n), used if outI == nullptr
+  long long ostepA, ostepB;
+  float2 *outI;             // interleaved output (row step n)
+  int n, log2n;
+  const float2 *tw, *ph;
+};
+
+__global__ void __launch_bounds__(kRowThreads) k_row_inv(RowInvArgs a) {
+  extern __shared__ float2 zbuf[];
+  const int n = a.n;
+  float *p = reinterpret_cast<float *>(zbuf + n);
+  float *q = p + n;
+  const float *ra = a.inA + (long long)blockIdx.x * a.stepA;
+  const float *rb = a.inB + (long long)blockIdx.x * a.stepB;
+  for (int t = threadIdx.x; t < n; t += kRowThreads) {
+    // IDXST input reversal (eq 8e): x'_t = x_{N-t}, x'_0 = 0
+    p[t] = (a.opA == 2) ? (t ? __ldg(ra + n - t) : 0.f) : __ldg(ra + t);
+    q[t] = (a.opB == 2) ? (t ? __ldg(rb + n - t) : 0.f) : __ldg(rb + t);
+  }
+  __syncthreads();
+  for (int k = threadIdx.x; k < n; k += kRowThreads) {
+    const float pnk = k ? p[n - k] : 0.f, qnk = k ? q[n - k] : 0.f;
+    zbuf[brev(k, a.log2n)] = inv_pre(p[k], q[k], pnk, qnk, __ldg(a.ph + k));
+  }
+  __syncthreads();
+  fft_block(zbuf, n, a.log2n, 1, a.tw, true);
+  for (int t = threadIdx.x; t < n; t += kRowThreads) {
+    const float2 v = zbuf[mk_pos(t, n)];
+    float va = 0.5f * v.x, vb = 0.5f * v.y;
+    if (t & 1) {
+      if (a.opA == 2) va = -va;
+      if (a.opB == 2) vb = -vb;
+    }
+    if (a.outI) {
+      a.outI[(size_t)blockIdx.x * n + t] = make_float2(va, vb);
+    } else {
+      a.outA[(long long)blockIdx.x * a.ostepA + t] = va;
+      a.outB[(long long)blockIdx.x * a.ostepB + t] = vb;
+    }
+  }
+}
+
+// ---------------------------------------------------------------------------------------
+// Column kernels: a CTA owns kColSlab adjacent columns (pairs share a complex FFT).
+// ---------------------------------------------------------------------------------------
+// Generic column transform (debug transforms): op 0 = DCT, 1 = IDCT, 2 = IDXST.
+__global__ void __launch_bounds__(kColThreads) k_col_generic(const float *__restrict__ in, float *__restrict__ out,
+                                                             int op, int mx, int log2mx, int my,
+                                                             const float2 *__restrict__ tw,
+                                                             const float2 *__restrict__ ph) {
+  extern __shared__ float2 zbuf[];  // [sc/2][mx] complex + [sc][mx] real
+  const int kColSlab = col_slab(mx);
+  float *rbuf = reinterpret_cast<float *>(zbuf + (kColSlab / 2) * mx);
+  const int c0 = blockIdx.x * kColSlab;
+  for (int idx = threadIdx.x; idx < mx * kColSlab; idx += kColThreads) {
+    const int row = idx / kColSlab, col = idx % kColSlab;
+    rbuf[col * mx + row] = __ldg(in + (size_t)row * my + c0 + col);
+  }
+  __syncthreads();
+  if (op == 0) {
+    for (int idx = threadIdx.x; idx < mx * (kColSlab / 2); idx += kColThreads) {
+      const int pr = idx / mx, t = idx % mx;
+      zbuf[pr * mx + brev(mk_pos(t, mx), log2mx)] = make_float2(rbuf[(2 * pr) * mx + t], rbuf[(2 * pr + 1) * mx + t]);
+    }
+  } else {
+    for (int idx = threadIdx.x; idx < mx * (kColSlab / 2); idx += kColThreads) {
+      const int pr = idx / mx, k = idx % mx;
+      const float *pp = rbuf + (2 * pr) * mx, *qq = rbuf + (2 * pr + 1) * mx;
+      float pk, qk, pnk, qnk;
+      if (op == 2) {  // reversed inputs x'_t = x_{N-t}
+        pk = k ? pp[mx - k] : 0.f;
+        qk = k ? qq[mx - k] : 0.f;
+        pnk = k ? pp[k] : 0.f;
+        qnk = k ? qq[k] : 0.f;
+      } else {
+        pk = pp[k];
+        qk = qq[k];
+        pnk = k ? pp[mx - k] : 0.f;
+        qnk = k ? qq[mx - k] : 0.f;
+      }
+      zbuf[pr * mx + brev(k, log2mx)] = inv_pre(pk, qk, pnk, qnk, __ldg(ph + k));
+    }
+  }
+  __syncthreads();
+  fft_block(zbuf, mx, log2mx, kColSlab / 2, tw, op != 0);
+  for (int idx = threadIdx.x; idx < mx * kColSlab; idx += kColThreads) {
+    const int row = idx / kColSlab, col = idx % kColSlab, pr = col >> 1;
+    float v;
+    if (op == 0) {
+      const float2 d = dct_post(zbuf + pr * mx, row, mx, __ldg(ph + row), 2.f / mx);
+      v = (col & 1) ? d.y : d.x;
+    } else {
+      const float2 z = zbuf[pr * mx + mk_pos(row, mx)];
+      v = 0.5f * ((col & 1) ? z.y : z.x);
+      if (op == 2 && (row & 1)) v = -v;
+    }
+    out[(size_t)row * my + c0 + col] = v;
+  }
+}
+
+// T2: fused column pass.  For each column v of t = DCT_y(rho):
+//   a[u][v]   = DCT_x(t[.][v])                                  (eq 9a)
+//   energy   += omega_u omega_v a^2 / (k_u^2 + k_v^2)           (Parseval form of D, A8)
+//   sX[.][v]  = IDXST_x( a k_u / k^2 )                          (eq 9c, x part)
+//   sY[.][v]  = IDCT_x ( a k_v / k^2 )                          (eq 9d, x part)
+// with a_00 / k^2 := 0 (eq 4c, A15).  The IDXST of column v and the IDCT of column v share
+// one complex IFFT.
+struct ColFieldArgs {
+  const float *t;
+  float *sx, *sy;
+  int mx, log2mx, my;
+  const float2 *tw_x, *ph_x;
+  const float *kx, *ky;
+  double *energy_part;   // one slot per CTA
+  double energy_scale;   // 1/2 b_x b_y
+};
+
+__global__ void __launch_bounds__(kColThreads) k_col_fields(ColFieldArgs a) {
+  extern __shared__ float2 zbuf[];  // [sc][mx] complex; the first half doubles as the forward buffer
+  const int mx = a.mx, log2mx = a.log2mx, my = a.my;
+  const int kColSlab = col_slab(mx);
+  float *abuf = reinterpret_cast<float *>(zbuf + kColSlab * mx);  // [kColSlab][mx] real spectrum
+  __shared__ double s_red[kColThreads / 32];
+  const int c0 = blockIdx.x * kColSlab;
+  // load + Makhoul reorder along x, pairs of columns -> complex
+  for (int idx = threadIdx.x; idx < mx * kColSlab; idx += kColThreads) {
+    const int row = idx / kColSlab, col = idx % kColSlab, pr = col >> 1;
+    const float v = __ldg(a.t + (size_t)row * my + c0 + col);
+    float2 *slot = &zbuf[pr * mx + brev(mk_pos(row, mx), log2mx)];
+    if (col & 1) slot->y = v; else slot->x = v;
+  }
+  __syncthreads();
+  fft_block(zbuf, mx, log2mx, kColSlab / 2, a.tw_x, false);
+  const float scale = 2.f / mx;
+  double e = 0.0;
+  for (int idx = threadIdx.x; idx < mx * (kColSlab / 2); idx += kColThreads) {
+    const int pr = idx / mx, u = idx % mx;
+    const float2 d = dct_post(zbuf + pr * mx, u, mx, __ldg(a.ph_x + u), scale);
+    abuf[(2 * pr) * mx + u] = d.x;
+    abuf[(2 * pr + 1) * mx + u] = d.y;
+    const float kx = __ldg(a.kx + u);
+#pragma unroll
+    for (int h = 0; h < 2; h++) {
+      const int v = c0 + 2 * pr + h;
+      const float ky = __ldg(a.ky + v);
+      const float k2 = kx * kx + ky * ky;
+      if (u == 0 && v == 0) continue;
+      const float av = h ? d.y : d.x;
+      const double wu = (u == 0) ? 0.25 * mx : 0.5 * mx;
+      const double wv = (v == 0) ? 0.25 * my : 0.5 * my;
+      e += wu * wv * (double)av * (double)av / (double)k2;
+    }
+  }
+  __syncthreads();  // abuf complete; zbuf free
+  // inverse pre-processing: per column, p = reversed (a k_u / k^2) (IDXST), q = a k_v / k^2 (IDCT)
+  for (int idx = threadIdx.x; idx < mx * kColSlab; idx += kColThreads) {
+    const int col = idx / mx, k = idx % mx;
+    const int v = c0 + col;
+    const float *ac = abuf + col * mx;
+    const float ky = __ldg(a.ky + v), ky2 = ky * ky;
+    // A_X[u] = a[u] k_u / k^2, A_Y[u] = a[u] k_v / k^2, zero at (0,0)
+    auto AX = [&](int u) -> float {
+      const float kx = __ldg(a.kx + u), k2 = kx * kx + ky2;
+      return (u == 0 && v == 0) ? 0.f : ac[u] * kx / k2;
+    };
+    auto AY = [&](int u) -> float {
+      const float kx = __ldg(a.kx + u), k2 = kx * kx + ky2;
+      return (u == 0 && v == 0) ? 0.f : ac[u] * ky / k2;
+    };
+    // p (IDXST input reversed): p_k = AX[N-k] (k >= 1), p_0 = 0;  p_{N-k} = AX[k] (k >= 1)
+    const float pk = k ? AX(mx - k) : 0.f;
+    const float pnk = k ? AX(k) : 0.f;
+    const float qk = AY(k);
+    const float qnk = k ? AY(mx - k) : 0.f;
+    zbuf[col * mx + brev(k, log2mx)] = inv_pre(pk, qk, pnk, qnk, __ldg(a.ph_x + k));
+  }
+  __syncthreads();
+  fft_block(zbuf, mx, log2mx, kColSlab, a.tw_x, true);
+  for (int idx = threadIdx.x; idx < mx * kColSlab; idx += kColThreads) {
+    const int row = idx / kColSlab, col = idx % kColSlab;
+    const float2 z = zbuf[col * mx + mk_pos(row, mx)];
+    const float vx = (row & 1) ? -0.5f * z.x : 0.5f * z.x;  // IDXST sign (-1)^x
+    a.sx[(size_t)row * my + c0 + col] = vx;
+    a.sy[(size_t)row * my + c0 + col] = 0.5f * z.y;
+  }
+  // energy partial
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) e += __shfl_xor_sync(0xffffffffu, e, o);
+  if ((threadIdx.x & 31) == 0) s_red[threadIdx.x >> 5] = e;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    double t = 0.0;
+    for (int w = 0; w < kColThreads / 32; w++) t += s_red[w];
+    a.energy_part[blockIdx.x] = t * a.energy_scale;
+  }
+}
+
+// psi spectrum scaling for the debug hook: out = a / k^2 (0 at the DC term)
+__global__ void k_scale_psi(const float *a, float *out, const float *kx, const float *ky, int mx, int my) {
+  const size_t n = (size_t)mx * my;
+  for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < n; i += (size_t)gridDim.x * blockDim.x) {
+    const int u = (int)(i / my), v = (int)(i % my);
+    const float k2 = kx[u] * kx[u] + ky[v] * ky[v];
+    out[i] = (u == 0 && v == 0) ? 0.f : a[i] / k2;
+  }
+}
+
+__global__ void k_split_xi(const float2 *xi, float *xx, float *xy, size_t n) {
+  for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < n; i += (size_t)gridDim.x * blockDim.x) {
+    const float2 v = xi[i];
+    if (xx) xx[i] = v.x;
+    if (xy) xy[i] = v.y;
+  }
+}
+
+size_t row_smem(int n) { return (size_t)n * sizeof(float2) + 2 * (size_t)n * sizeof(float); }
+size_t col_generic_smem(int mx) { return (size_t)(col_slab(mx) / 2) * mx * sizeof(float2) + (size_t)col_slab(mx) * mx * sizeof(float); }
+size_t col_fields_smem(int mx) { return (size_t)col_slab(mx) * mx * sizeof(float2) + (size_t)col_slab(mx) * mx * sizeof(float); }
+
+void row_inv(const Ctx &c, const float *inA, long long stepA, int opA, const float *inB, long long stepB,
+             int opB, float *outA, long long ostepA, float *outB, long long ostepB, float2 *outI,
+             int rows, cudaStream_t s) {
+  RowInvArgs a;
+  a.inA = inA; a.inB = inB; a.stepA = stepA; a.stepB = stepB; a.opA = opA; a.opB = opB;
+  a.outA = outA; a.outB = outB; a.ostepA = ostepA; a.ostepB = ostepB; a.outI = outI;
+  a.n = c.my; a.log2n = c.log2my; a.tw = c.d_tw_y; a.ph = c.d_ph_y;
+  k_row_inv<<<rows, kRowThreads, row_smem(c.my), s>>>(a);
+}
+
+}  // namespace
+
+// smem opt-in (called once from dp_create)
+cudaError_t dct_configure(int mx, int my) {
+  cudaError_t e;
+  e = cudaFuncSetAttribute(k_row_dct, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)row_smem(my));
+  if (e != cudaSuccess) return e;
+  e = cudaFuncSetAttribute(k_row_inv, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)row_smem(my));
+  if (e != cudaSuccess) return e;
+  e = cudaFuncSetAttribute(k_col_generic, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)col_generic_smem(mx));
+  if (e != cudaSuccess) return e;
+  return cudaFuncSetAttribute(k_col_fields, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)col_fields_smem(mx));
+}
+
+int col_fields_ctas(int mx, int my) { return my / col_slab(mx); }
+
+void launch_fields(const Ctx &c, const float *rho, cudaStream_t s) {
+  // T1: t = DCT_y(rho)
+  k_row_dct<<<c.mx / 2, kRowThreads, row_smem(c.my), s>>>(rho, c.d_t, c.my, c.log2my, c.d_tw_y, c.d_ph_y);
+  // T2: columns (DCT_x, scaling, energy, inverse x)
+  ColFieldArgs a;
+  a.t = c.d_t; a.sx = c.d_sx; a.sy = c.d_sy;
+  a.mx = c.mx; a.log2mx = c.log2mx; a.my = c.my;
+  a.tw_x = c.d_tw_x; a.ph_x = c.d_ph_x; a.kx = c.d_kx; a.ky = c.d_ky;
+  a.energy_part = c.d_part + c.n_wa_part;
+  a.energy_scale = 0.5 * c.bx * c.by;
+  k_col_fields<<<c.my / col_slab(c.mx), kColThreads, col_fields_smem(c.mx), s>>>(a);
+  // T3: rows: xi_X = IDCT_y(sX), xi_Y = IDXST_y(sY), interleaved
+  row_inv(c, c.d_sx, c.my, 1, c.d_sy, c.my, 2, nullptr, 0, nullptr, 0, c.d_xi, c.mx, s);
+}
+
+void launch_split_fields(const Ctx &c, float *xi_x, float *xi_y, cudaStream_t s) {
+  k_split_xi<<<c.num_sms * 4, 256, 0, s>>>(c.d_xi, xi_x, xi_y, (size_t)c.mx * c.my);
+}
+
+void launch_transform(const Ctx &c, int kind, const float *in, float *out, cudaStream_t s) {
+  const int mx = c.mx, my = c.my;
+  float *tmp = c.d_t;  // scratch (debug path only)
+  switch (kind) {
+    case DP_T_DCT2:
+      k_row_dct<<<mx / 2, kRowThreads, row_smem(my), s>>>(in, tmp, my, c.log2my, c.d_tw_y, c.d_ph_y);
+      k_col_generic<<<my / col_slab(mx), kColThreads, col_generic_smem(mx), s>>>(tmp, out, 0, mx, c.log2mx, my, c.d_tw_x, c.d_ph_x);
+      break;
+    case DP_T_IDCT2:
+    case DP_T_IDXST_IDCT:
+    case DP_T_IDCT_IDXST: {
+      const int op_y = (kind == DP_T_IDCT_IDXST) ? 2 : 1;
+      const int op_x = (kind == DP_T_IDXST_IDCT) ? 2 : 1;
+      // rows (2r, 2r+1) share a complex IFFT
+      row_inv(c, in, 2LL * my, op_y, in + my, 2LL * my, op_y, tmp, 2LL * my, tmp + my, 2LL * my, nullptr, mx / 2, s);
+      k_col_generic<<<my / col_slab(mx), kColThreads, col_generic_smem(mx), s>>>(tmp, out, op_x, mx, c.log2mx, my, c.d_tw_x, c.d_ph_x);
+      break;
+    }
+    default:
+      break;
+  }
+}
+
+void launch_psi(const Ctx &c, const float *rho, float *psi, cudaStream_t s) {
+  // debug only: a = DCT2(rho) -> psi = IDCT2(a / k^2).  Uses sx / sy as scratch.
+  launch_transform(c, DP_T_DCT2, rho, c.d_sx, s);
+  k_scale_psi<<<c.num_sms * 4, 256, 0, s>>>(c.d_sx, c.d_sy, c.d_kx, c.d_ky, c.mx, c.my);
+  launch_transform(c, DP_T_IDCT2, c.d_sy, psi, s);
+}
+
+}  // namespace dp

@@ -1,0 +1,742 @@
+// dp_api.cu — the C ABI of libdp (include/dp.h): validation, dp_create (host-side layout
+// building), evaluation orchestration over two streams, and the test hooks.
+//
+// dp_create does all data-dependent preparation once:
+//   * pins are put in net order (net2pin applied), degree 0/1 nets are dropped (reading A3);
+//   * nets of degree <= kWaMaxDeg are sorted by the median cell index of their pins and cut
+//     into chunks of ~kWaChunkPins pins; each chunk gets the densest window of kWaWindow
+//     consecutive cells (its positions and gradients live in shared memory);
+//   * inside a chunk nets are grouped by lanes-per-net G (degree <= 8 G) and sorted by degree,
+//     32/G nets form a warp group whose pins are stored slot-major so every load coalesces;
+//   * nets of larger degree keep a CSR list for the CTA-per-net kernel;
+//   * the own-cell range, large-cell list, tile grid, FFT twiddles and wavenumbers.
+// dp_eval forks the caller stream into a WA stream and a density stream, joins, combines.
+#include <dlfcn.h>
+
+#include <algorithm>
+#include <cmath>
+#include <cstring>
+#include <numeric>
+#include <string>
+#include <vector>
+
+#include "dp_internal.h"
+
+namespace dp {
+
+static thread_local std::string g_err;
+
+void set_error(const std::string &msg) { g_err = msg; }
+dp_status fail(dp_status st, const std::string &msg) {
+  g_err = msg;
+  return st;
+}
+dp_status cuda_fail(cudaError_t e, const char *what) {
+  g_err = std::string("CUDA error ") + cudaGetErrorName(e) + " (" + cudaGetErrorString(e) + ") in " + what;
+  return e == cudaErrorMemoryAllocation ? DP_ERR_OUT_OF_MEMORY : DP_ERR_CUDA;
+}
+
+namespace {
+
+struct DeviceGuard {
+  int prev = -1;
+  explicit DeviceGuard(int dev) {
+    if (cudaGetDevice(&prev) != cudaSuccess) prev = -1;
+    if (prev != dev) cudaSetDevice(dev);
+  }
+  ~DeviceGuard() {
+    int cur = -1;
+    if (prev >= 0 && cudaGetDevice(&cur) == cudaSuccess && cur != prev) cudaSetDevice(prev);
+  }
+};
+
+template <class T>
+dp_status dev_alloc(Ctx &c, T **p, size_t n) {
+  *p = nullptr;
+  if (n == 0) n = 1;
+  void *q = nullptr;
+  cudaError_t e = cudaMalloc(&q, n * sizeof(T));
+  if (e != cudaSuccess) return cuda_fail(e, "cudaMalloc");
+  c.allocations.push_back(q);
+  c.device_bytes += (int64_t)(n * sizeof(T));
+  *p = static_cast<T *>(q);
+  return DP_OK;
+}
+
+template <class T>
+dp_status dev_upload(Ctx &c, T **p, const std::vector<T> &v) {
+  dp_status st = dev_alloc(c, p, v.size());
+  if (st != DP_OK) return st;
+  if (!v.empty()) DP_CUDA(cudaMemcpy(*p, v.data(), v.size() * sizeof(T), cudaMemcpyHostToDevice));
+  return DP_OK;
+}
+
+bool is_pow2(int v) { return v > 0 && (v & (v - 1)) == 0; }
+int ilog2(int v) {
+  int r = 0;
+  while ((1 << r) < v) r++;
+  return r;
+}
+
+dp_status validate(const dp_netlist *nl, const dp_grid *g) {
+  if (!nl || !g) return fail(DP_ERR_INVALID_ARG, "netlist or grid is NULL");
+  if (nl->num_cells < 1) return fail(DP_ERR_INVALID_ARG, "num_cells must be >= 1");
+  if (nl->num_nets < 0 || nl->num_pins < 0) return fail(DP_ERR_INVALID_ARG, "negative net or pin count");
+  if (!nl->net_start || !nl->cell_w || !nl->cell_h) return fail(DP_ERR_INVALID_ARG, "net_start, cell_w and cell_h are required");
+  if (nl->num_pins > 0 && (!nl->pin2cell || !nl->pin_dx || !nl->pin_dy))
+    return fail(DP_ERR_INVALID_ARG, "pin2cell, pin_dx, pin_dy are required when num_pins > 0");
+  if (nl->net_start[0] != 0) return fail(DP_ERR_INVALID_ARG, "net_start[0] must be 0");
+  for (int32_t e = 0; e < nl->num_nets; e++)
+    if (nl->net_start[e + 1] < nl->net_start[e]) return fail(DP_ERR_INVALID_ARG, "net_start must be nondecreasing (net " + std::to_string(e) + ")");
+  if (nl->net_start[nl->num_nets] != nl->num_pins) return fail(DP_ERR_INVALID_ARG, "net_start[num_nets] must equal num_pins");
+  for (int32_t p = 0; p < nl->num_pins; p++) {
+    const int32_t c = nl->pin2cell[p];
+    if (c < 0 || c >= nl->num_cells) return fail(DP_ERR_INVALID_ARG, "pin2cell out of range at pin " + std::to_string(p));
+    if (!std::isfinite(nl->pin_dx[p]) || !std::isfinite(nl->pin_dy[p])) return fail(DP_ERR_INVALID_ARG, "non-finite pin offset at pin " + std::to_string(p));
+  }
+  if (nl->net2pin) {
+    std::vector<uint8_t> seen(nl->num_pins, 0);
+    for (int32_t s = 0; s < nl->num_pins; s++) {
+      const int32_t p = nl->net2pin[s];
+      if (p < 0 || p >= nl->num_pins || seen[p]) return fail(DP_ERR_INVALID_ARG, "net2pin is not a permutation");
+      seen[p] = 1;
+    }
+  }
+  for (int32_t c = 0; c < nl->num_cells; c++) {
+    const float w = nl->cell_w[c], h = nl->cell_h[c];
+    if (!std::isfinite(w) || !std::isfinite(h) || w < 0.f || h < 0.f) return fail(DP_ERR_INVALID_ARG, "cell sizes must be finite and >= 0 (cell " + std::to_string(c) + ")");
+  }
+  if (nl->net_weight)
+    for (int32_t e = 0; e < nl->num_nets; e++)
+      if (!std::isfinite(nl->net_weight[e]) || nl->net_weight[e] < 0.f) return fail(DP_ERR_INVALID_ARG, "net weights must be finite and >= 0");
+  if (!(std::isfinite(g->xl) && std::isfinite(g->xh) && std::isfinite(g->yl) && std::isfinite(g->yh)) || !(g->xh > g->xl) || !(g->yh > g->yl))
+    return fail(DP_ERR_INVALID_ARG, "degenerate or non-finite placement region");
+  if (g->stretch != 0 && g->stretch != 1) return fail(DP_ERR_INVALID_ARG, "stretch must be 0 or 1");
+  if (!is_pow2(g->bins_x) || !is_pow2(g->bins_y) || g->bins_x < 16 || g->bins_y < 16 || g->bins_x > 4096 || g->bins_y > 4096)
+    return fail(DP_ERR_UNSUPPORTED, "bins_x and bins_y must be powers of two in [16, 4096]");
+  return DP_OK;
+}
+
+// Contiguous, count-balanced cell ranges; a net is evaluated on every rank owning one of its
+// pins' cells and counted (WA, HPWL) on the rank owning its first pin's cell.
+void plan(const dp_netlist *nl, int rank, int world, int32_t &cb, int32_t &ce, std::vector<uint8_t> *mask) {
+  const int64_t n = nl->num_cells;
+  cb = (int32_t)(n * rank / world);
+  ce = (int32_t)(n * (rank + 1) / world);
+  if (!mask) return;
+  mask->assign(nl->num_nets, 0);
+  for (int32_t e = 0; e < nl->num_nets; e++) {
+    const int32_t s = nl->net_start[e], t = nl->net_start[e + 1];
+    uint8_t m = 0;
+    for (int32_t k = s; k < t; k++) {
+      const int32_t p = nl->net2pin ? nl->net2pin[k] : k;
+      const int32_t c = nl->pin2cell[p];
+      if (c >= cb && c < ce) {
+        m = 1;
+        break;
+      }
+    }
+    if (m && t > s) {
+      const int32_t p0 = nl->net2pin ? nl->net2pin[s] : s;
+      const int32_t c0 = nl->pin2cell[p0];
+      if (c0 >= cb && c0 < ce) m = 3;
+    }
+    (*mask)[e] = m;
+  }
+}
+
+int g_class(int d) {  // log2 of lanes per net
+  int g = 0;
+  while ((kWaPpl << g) < d) g++;
+  return g;
+}
+
+dp_status build_wa(Ctx &c, const dp_netlist *nl, const std::vector<uint8_t> &mask) {
+  const int32_t ncells = nl->num_cells;
+  auto pin_of = [&](int32_t slot) { return nl->net2pin ? nl->net2pin[slot] : slot; };
+  std::vector<int32_t> small, big;
+  for (int32_t e = 0; e < nl->num_nets; e++) {
+    const int d = nl->net_start[e + 1] - nl->net_start[e];
+    if (d < 2 || !mask[e]) continue;  // reading A3: degree 0/1 contribute nothing
+    (d > kWaMaxDeg ? big : small).push_back(e);
+  }
+  // ---- locality order: median cell index of each net's pins ----
+  std::vector<int32_t> key(nl->num_nets, 0);
+  std::vector<int32_t> tmp;
+  for (int32_t e : small) {
+    const int32_t s = nl->net_start[e], t = nl->net_start[e + 1];
+    tmp.clear();
+    for (int32_t k = s; k < t; k++) tmp.push_back(nl->pin2cell[pin_of(k)]);
+    std::nth_element(tmp.begin(), tmp.begin() + tmp.size() / 2, tmp.end());
+    key[e] = tmp[tmp.size() / 2];
+  }
+  std::stable_sort(small.begin(), small.end(), [&](int32_t a, int32_t b) { return key[a] < key[b]; });
+
+  std::vector<Chunk> chunks;
+  std::vector<WarpGroup> wgs;
+  std::vector<int32_t> net_deg, pin_cell;
+  std::vector<float> net_w, pin_dx, pin_dy;
+  size_t i = 0;
+  std::vector<int32_t> cells;
+  while (i < small.size()) {
+    // take nets until the pin budget is reached (at least one net)
+    size_t j = i;
+    int pins = 0;
+    while (j < small.size()) {
+      const int d = nl->net_start[small[j] + 1] - nl->net_start[small[j]];
+      if (j > i && pins + d > kWaChunkPins) break;
+      pins += d;
+      j++;
+    }
+    // densest window of kWaWindow consecutive cells
+    cells.clear();
+    for (size_t q = i; q < j; q++)
+      for (int32_t k = nl->net_start[small[q]]; k < nl->net_start[small[q] + 1]; k++) cells.push_back(nl->pin2cell[pin_of(k)]);
+    std::sort(cells.begin(), cells.end());
+    const int win_n = std::min<int32_t>(kWaWindow, ncells);
+    int32_t best_lo = cells[0];
+    size_t best = 0, lo = 0;
+    for (size_t hi = 0; hi < cells.size(); hi++) {
+      while (cells[hi] - cells[lo] >= win_n) lo++;
+      if (hi - lo + 1 > best) {
+        best = hi - lo + 1;
+        best_lo = cells[lo];
+      }
+    }
+    best_lo = std::max(0, std::min(best_lo, ncells - win_n));
+    Chunk ch;
+    ch.wg_begin = (int32_t)wgs.size();
+    ch.win_lo = best_lo;
+    ch.win_n = win_n;
+    // group nets by lanes-per-net class, largest class first, degree-descending inside
+    std::vector<std::vector<int32_t>> cls(6);
+    for (size_t q = i; q < j; q++) {
+      const int d = nl->net_start[small[q] + 1] - nl->net_start[small[q]];
+      cls[g_class(d)].push_back(small[q]);
+    }
+    for (int g = 5; g >= 0; g--) {
+      auto &v = cls[g];
+      std::stable_sort(v.begin(), v.end(), [&](int32_t a, int32_t b) {
+        return (nl->net_start[a + 1] - nl->net_start[a]) > (nl->net_start[b + 1] - nl->net_start[b]);
+      });
+      const int per = 32 >> g, G = 1 << g;
+      for (size_t q = 0; q < v.size(); q += per) {
+        WarpGroup wg;
+        wg.pin_base = (int32_t)pin_cell.size();
+        wg.net_base = (int32_t)net_deg.size();
+        wg.nnets = (int32_t)std::min<size_t>(per, v.size() - q);
+        wg.g_log2 = g;
+        wg.pad = 0;
+        int dmax = 0;
+        for (int n = 0; n < wg.nnets; n++) {
+          const int32_t e = v[q + n];
+          const int d = nl->net_start[e + 1] - nl->net_start[e];
+          dmax = std::max(dmax, d);
+          net_deg.push_back(d | ((mask[e] & 2) ? (int32_t)0x80000000u : 0));
+          net_w.push_back(nl->net_weight ? nl->net_weight[e] : 1.f);
+        }
+        wg.slots = (dmax + G - 1) / G;
+        for (int s = 0; s < wg.slots; s++)
+          for (int L = 0; L < 32; L++) {
+            const int gi = L >> g, jj = L & (G - 1);
+            if (gi >= wg.nnets) continue;
+            const int32_t e = v[q + gi];
+            const int d = nl->net_start[e + 1] - nl->net_start[e];
+            const int k = s * G + jj;
+            if (k >= d) continue;
+            const int32_t p = pin_of(nl->net_start[e] + k);
+            const int32_t cell = nl->pin2cell[p];
+            const bool foreign = cell < c.cell_begin || cell >= c.cell_end;
+            pin_cell.push_back(cell | (foreign ? (int32_t)0x80000000u : 0));
+            pin_dx.push_back(nl->pin_dx[p]);
+            pin_dy.push_back(nl->pin_dy[p]);
+          }
+        wgs.push_back(wg);
+      }
+    }
+    ch.wg_end = (int32_t)wgs.size();
+    chunks.push_back(ch);
+    i = j;
+  }
+  c.n_chunks = (int32_t)chunks.size();
+  c.n_wgroups = (int32_t)wgs.size();
+  c.n_wa_nets = (int32_t)net_deg.size();
+  c.n_wa_pins = (int32_t)pin_cell.size();
+  dp_status st;
+  if ((st = dev_upload(c, &c.d_chunks, chunks)) != DP_OK) return st;
+  if ((st = dev_upload(c, &c.d_wgroups, wgs)) != DP_OK) return st;
+  if ((st = dev_upload(c, &c.d_net_deg, net_deg)) != DP_OK) return st;
+  if ((st = dev_upload(c, &c.d_net_w, net_w)) != DP_OK) return st;
+  if ((st = dev_upload(c, &c.d_pin_cell, pin_cell)) != DP_OK) return st;
+  if ((st = dev_upload(c, &c.d_pin_dx, pin_dx)) != DP_OK) return st;
+  if ((st = dev_upload(c, &c.d_pin_dy, pin_dy)) != DP_OK) return st;
+  // ---- big nets ----
+  std::vector<int32_t> bstart{0}, bflags, bcell;
+  std::vector<float> bw, bdx, bdy;
+  for (int32_t e : big) {
+    for (int32_t k = nl->net_start[e]; k < nl->net_start[e + 1]; k++) {
+      const int32_t p = pin_of(k);
+      const int32_t cell = nl->pin2cell[p];
+      const bool foreign = cell < c.cell_begin || cell >= c.cell_end;
+      bcell.push_back(cell | (foreign ? (int32_t)0x80000000u : 0));
+      bdx.push_back(nl->pin_dx[p]);
+      bdy.push_back(nl->pin_dy[p]);
+    }
+    bstart.push_back((int32_t)bcell.size());
+    bflags.push_back((mask[e] & 2) ? 1 : 0);
+    bw.push_back(nl->net_weight ? nl->net_weight[e] : 1.f);
+  }
+  c.n_big = (int32_t)big.size();
+  if ((st = dev_upload(c, &c.d_big_start, bstart)) != DP_OK) return st;
+  if ((st = dev_upload(c, &c.d_big_flags, bflags)) != DP_OK) return st;
+  if ((st = dev_upload(c, &c.d_big_w, bw)) != DP_OK) return st;
+  if ((st = dev_upload(c, &c.d_big_cell, bcell)) != DP_OK) return st;
+  if ((st = dev_upload(c, &c.d_big_dx, bdx)) != DP_OK) return st;
+  if ((st = dev_upload(c, &c.d_big_dy, bdy)) != DP_OK) return st;
+  return DP_OK;
+}
+
+std::vector<float2> twiddles(int n) {  // exp(-2 pi i k / n), k < n/2, from fp64
+  std::vector<float2> t(n / 2);
+  for (int k = 0; k < n / 2; k++) {
+    const double a = 2.0 * M_PI * k / n;
+    t[k] = make_float2((float)std::cos(a), (float)-std::sin(a));
+  }
+  return t;
+}
+std::vector<float2> phases(int n) {  // exp(-i pi k / 2n), k < n
+  std::vector<float2> t(n);
+  for (int k = 0; k < n; k++) {
+    const double a = M_PI * k / (2.0 * n);
+    t[k] = make_float2((float)std::cos(a), (float)-std::sin(a));
+  }
+  return t;
+}
+
+dp_status build_density(Ctx &c, const dp_netlist *nl) {
+  c.n_own = c.cell_end - c.cell_begin;
+  std::vector<float> w(nl->cell_w + c.cell_begin, nl->cell_w + c.cell_end);
+  std::vector<float> h(nl->cell_h + c.cell_begin, nl->cell_h + c.cell_end);
+  std::vector<int32_t> large;
+  for (int32_t i = 0; i < c.n_own; i++)
+    if ((double)w[i] > 2.0 * c.bx || (double)h[i] > 2.0 * c.by) large.push_back(i);
+  c.n_large = (int32_t)large.size();
+  c.tile = std::min(std::max(c.mx, c.my) > 2048 ? 64 : kTile, std::min(c.mx, c.my));
+  c.tiles_x = c.mx / c.tile;
+  c.tiles_y = c.my / c.tile;
+  const int ntiles = c.tiles_x * c.tiles_y;
+  c.max_segs = c.n_own / kSegCells + ntiles + 1;
+  const size_t nb = (size_t)c.mx * c.my;
+  dp_status st;
+  if ((st = dev_upload(c, &c.d_cell_w, w)) != DP_OK) return st;
+  if ((st = dev_upload(c, &c.d_cell_h, h)) != DP_OK) return st;
+  if ((st = dev_upload(c, &c.d_large, large)) != DP_OK) return st;
+  if ((st = dev_alloc(c, &c.d_tile_cnt, ntiles)) != DP_OK) return st;
+  DP_CUDA(cudaMemset(c.d_tile_cnt, 0, sizeof(int32_t) * ntiles));
+  if ((st = dev_alloc(c, &c.d_tile_cursor, ntiles)) != DP_OK) return st;
+  if ((st = dev_alloc(c, &c.d_tile_off, ntiles + 1)) != DP_OK) return st;
+  if ((st = dev_alloc(c, &c.d_rec, std::max(c.n_own, 1))) != DP_OK) return st;
+  if ((st = dev_alloc(c, &c.d_rec_rc, std::max(c.n_own, 1))) != DP_OK) return st;
+  if ((st = dev_alloc(c, &c.d_rec_cell, std::max(c.n_own, 1))) != DP_OK) return st;
+  if ((st = dev_alloc(c, &c.d_segs, c.max_segs)) != DP_OK) return st;
+  if ((st = dev_alloc(c, &c.d_nsegs, 1)) != DP_OK) return st;
+  DP_CUDA(cudaMemset(c.d_nsegs, 0, sizeof(int32_t)));
+  if ((st = dev_alloc(c, &c.d_rho, nb)) != DP_OK) return st;
+  if ((st = dev_alloc(c, &c.d_t, nb)) != DP_OK) return st;
+  if ((st = dev_alloc(c, &c.d_sx, nb)) != DP_OK) return st;
+  if ((st = dev_alloc(c, &c.d_sy, nb)) != DP_OK) return st;
+  if ((st = dev_alloc(c, &c.d_xi, nb)) != DP_OK) return st;
+  if ((st = dev_alloc(c, &c.d_force, std::max(c.n_own, 1))) != DP_OK) return st;
+  DP_CUDA(cudaMemset(c.d_force, 0, sizeof(float2) * std::max(c.n_own, 1)));
+  if ((st = dev_upload(c, &c.d_tw_x, twiddles(c.mx))) != DP_OK) return st;
+  if ((st = dev_upload(c, &c.d_tw_y, twiddles(c.my))) != DP_OK) return st;
+  if ((st = dev_upload(c, &c.d_ph_x, phases(c.mx))) != DP_OK) return st;
+  if ((st = dev_upload(c, &c.d_ph_y, phases(c.my))) != DP_OK) return st;
+  std::vector<float> kx(c.mx), ky(c.my);
+  for (int u = 0; u < c.mx; u++) kx[u] = (float)(M_PI * u / (c.xh - c.xl));   // reading A12
+  for (int v = 0; v < c.my; v++) ky[v] = (float)(M_PI * v / (c.yh - c.yl));
+  if ((st = dev_upload(c, &c.d_kx, kx)) != DP_OK) return st;
+  if ((st = dev_upload(c, &c.d_ky, ky)) != DP_OK) return st;
+  // shared-memory opt-in (process-wide maxima)
+  static int max_m = 0, max_tiles = 0, max_tile = 0;
+  const int m = std::max(c.mx, c.my);
+  if (m > max_m || c.mx != c.my) {
+    DP_CUDA(dct_configure(std::max(c.mx, max_m), std::max(c.my, max_m)));
+    max_m = std::max(max_m, m);
+  }
+  if (ntiles > max_tiles || c.tile > max_tile) {
+    max_tiles = std::max(max_tiles, ntiles);
+    max_tile = std::max(max_tile, c.tile);
+    DP_CUDA(density_configure(max_tiles, max_tile));
+  }
+  return DP_OK;
+}
+
+void destroy(Ctx *c) {
+  if (!c) return;
+  DeviceGuard g(c->device);
+  if (c->s_wa) cudaStreamSynchronize(c->s_wa);
+  if (c->s_den) cudaStreamSynchronize(c->s_den);
+  nccl_destroy(*c);
+  for (void *p : c->allocations) cudaFree(p);
+  if (c->d_hx) cudaFreeHost(c->d_hx);
+  if (c->s_wa) cudaStreamDestroy(c->s_wa);
+  if (c->s_den) cudaStreamDestroy(c->s_den);
+  if (c->ev_fork) cudaEventDestroy(c->ev_fork);
+  if (c->ev_wa) cudaEventDestroy(c->ev_wa);
+  if (c->ev_den) cudaEventDestroy(c->ev_den);
+  if (c->ev_done) cudaEventDestroy(c->ev_done);
+  delete c;
+}
+
+dp_status create(const dp_netlist *nl, const dp_grid *grid, int device, int rank, int world, const void *nccl_id,
+                 dp_ctx **out) {
+  if (!out) return fail(DP_ERR_INVALID_ARG, "out is NULL");
+  *out = nullptr;
+  dp_status st = validate(nl, grid);
+  if (st != DP_OK) return st;
+  if (world < 1 || rank < 0 || rank >= world) return fail(DP_ERR_INVALID_ARG, "bad rank / world");
+  int ndev = 0;
+  cudaError_t e = cudaGetDeviceCount(&ndev);
+  if (e != cudaSuccess || ndev == 0) return fail(DP_ERR_CUDA, "no CUDA device available (libdp has no CPU path)");
+  if (device < 0 || device >= ndev) return fail(DP_ERR_INVALID_ARG, "device index out of range");
+  DeviceGuard guard(device);
+  cudaDeviceProp prop;
+  DP_CUDA(cudaGetDeviceProperties(&prop, device));
+  if (prop.major != 10 || prop.minor != 0)
+    return fail(DP_ERR_CUDA, std::string("libdp is built for sm_100a (B200); device is ") + prop.name);
+  Ctx *c = new Ctx();
+  c->device = device;
+  c->rank = rank;
+  c->world = world;
+  c->dist = world > 1;
+  c->num_sms = prop.multiProcessorCount;
+  c->l2_bytes = prop.l2CacheSize;
+  c->num_cells = nl->num_cells;
+  c->num_nets_in = nl->num_nets;
+  c->num_pins_in = nl->num_pins;
+  c->has_weights = nl->net_weight != nullptr;
+  c->xl = grid->xl; c->yl = grid->yl; c->xh = grid->xh; c->yh = grid->yh;
+  c->mx = grid->bins_x; c->my = grid->bins_y;
+  c->log2mx = ilog2(c->mx); c->log2my = ilog2(c->my);
+  c->bx = (c->xh - c->xl) / c->mx;
+  c->by = (c->yh - c->yl) / c->my;
+  c->stretch = grid->stretch;
+  std::vector<uint8_t> mask;
+  plan(nl, rank, world, c->cell_begin, c->cell_end, &mask);
+  auto bail = [&](dp_status s) {
+    destroy(c);
+    return s;
+  };
+  if ((st = build_wa(*c, nl, mask)) != DP_OK) return bail(st);
+  if ((st = build_density(*c, nl)) != DP_OK) return bail(st);
+  c->n_wa_part = c->n_chunks + c->n_big;
+  c->n_en_part = c->my / (c->mx <= 1024 ? 8 : (c->mx <= 2048 ? 4 : 2));
+  if ((st = dev_alloc(*c, &c->d_g2, c->num_cells)) != DP_OK) return bail(st);
+  if (cudaMemset(c->d_g2, 0, sizeof(float2) * c->num_cells) != cudaSuccess) return bail(fail(DP_ERR_CUDA, "memset"));
+  if ((st = dev_alloc(*c, &c->d_part, c->n_wa_part + c->n_en_part + 1)) != DP_OK) return bail(st);
+  if (cudaMemset(c->d_part, 0, sizeof(double) * (c->n_wa_part + c->n_en_part + 1)) != cudaSuccess) return bail(fail(DP_ERR_CUDA, "memset"));
+  if ((st = dev_alloc(*c, &c->d_limbs, kHpwlLimbs + 1)) != DP_OK) return bail(st);
+  if (cudaMemset(c->d_limbs, 0, sizeof(unsigned long long) * (kHpwlLimbs + 1)) != cudaSuccess) return bail(fail(DP_ERR_CUDA, "memset"));
+  if ((st = dev_alloc(*c, &c->d_scal, 8)) != DP_OK) return bail(st);
+  if ((st = dev_alloc(*c, &c->d_hgx, c->num_cells)) != DP_OK) return bail(st);   // e2e device buffers
+  if ((st = dev_alloc(*c, &c->d_hgy, c->num_cells)) != DP_OK) return bail(st);
+  if ((st = dev_alloc(*c, &c->d_hy, 2 * (size_t)c->num_cells)) != DP_OK) return bail(st);  // x then y
+  c->d_hx = nullptr;
+  if (cudaStreamCreateWithFlags(&c->s_wa, cudaStreamNonBlocking) != cudaSuccess ||
+      cudaStreamCreateWithFlags(&c->s_den, cudaStreamNonBlocking) != cudaSuccess ||
+      cudaEventCreateWithFlags(&c->ev_fork, cudaEventDisableTiming) != cudaSuccess ||
+      cudaEventCreateWithFlags(&c->ev_wa, cudaEventDisableTiming) != cudaSuccess ||
+      cudaEventCreateWithFlags(&c->ev_den, cudaEventDisableTiming) != cudaSuccess ||
+      cudaEventCreateWithFlags(&c->ev_done, cudaEventDisableTiming) != cudaSuccess)
+    return bail(fail(DP_ERR_CUDA, "stream/event creation failed"));
+  const int wa_k = (c->n_chunks > 0) + (c->n_big > 0);
+  c->launches_eval = wa_k + density_launches(*c) + 3 /* T1 T2 T3 */ + 2 /* combine, finalize */;
+  c->launches_eval_hpwl = c->launches_eval;
+  if (world > 1 && nccl_id) {
+    if ((st = nccl_init(*c, nccl_id)) != DP_OK) return bail(st);
+  }
+  cudaError_t le = cudaDeviceSynchronize();
+  if (le != cudaSuccess) return bail(cuda_fail(le, "dp_create"));
+  *out = reinterpret_cast<dp_ctx *>(c);
+  return DP_OK;
+}
+
+inline Ctx *C(dp_ctx *p) { return reinterpret_cast<Ctx *>(p); }
+
+dp_status check_eval_args(Ctx *c, const void *x, const void *y) {
+  if (!c) return fail(DP_ERR_INVALID_ARG, "ctx is NULL");
+  if (!x || !y) return fail(DP_ERR_INVALID_ARG, "x / y is NULL");
+  return DP_OK;
+}
+
+// the density chain on the density stream: map -> (allreduce) -> fields -> gather
+dp_status density_chain(Ctx &c, const float *x, const float *y) {
+  launch_density_map(c, x, y, c.s_den);
+  if (c.dist && c.nccl_comm) {
+    dp_status st = nccl_allreduce_f32(c, c.d_rho, (size_t)c.mx * c.my, c.s_den);
+    if (st != DP_OK) return st;
+  }
+  launch_fields(c, c.d_rho, c.s_den);
+  launch_density_gather(c, x, y, c.s_den);
+  return DP_OK;
+}
+
+dp_status finalize(Ctx &c, float lambda, bool with_wl, bool with_energy, bool with_hpwl, double *d_obj, double *d_wl,
+                   double *d_energy, double *d_hpwl, cudaStream_t s) {
+  if (c.dist && c.nccl_comm) {
+    launch_finalize_phase(c, 0, lambda, with_wl, with_energy, with_hpwl, d_obj, d_wl, d_energy, d_hpwl, s);
+    dp_status st;
+    if (with_wl && (st = nccl_allreduce_f64(c, c.d_scal, 1, s)) != DP_OK) return st;
+    if (with_hpwl && (st = nccl_allreduce_u64(c, c.d_limbs, kHpwlLimbs + 1, s)) != DP_OK) return st;
+    launch_finalize_phase(c, 1, lambda, with_wl, with_energy, with_hpwl, d_obj, d_wl, d_energy, d_hpwl, s);
+  } else {
+    launch_finalize(c, lambda, with_wl, with_energy, with_hpwl, d_obj, d_wl, d_energy, d_hpwl, s);
+  }
+  return DP_OK;
+}
+
+// A context owns scratch (g2, maps, partials): calls issued on different streams are ordered
+// by making each call wait for the previous one (skipped while the stream is being captured,
+// where the caller's graph already orders the calls).
+dp_status call_begin(Ctx &c, cudaStream_t s) {
+  cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+  DP_CUDA(cudaStreamIsCapturing(s, &cs));
+  if (cs == cudaStreamCaptureStatusNone) DP_CUDA(cudaStreamWaitEvent(s, c.ev_done, 0));
+  return DP_OK;
+}
+dp_status call_end(Ctx &c, cudaStream_t s) {
+  cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+  DP_CUDA(cudaStreamIsCapturing(s, &cs));
+  if (cs == cudaStreamCaptureStatusNone) DP_CUDA(cudaEventRecord(c.ev_done, s));
+  return DP_OK;
+}
+
+dp_status eval_impl(Ctx &c, const float *x, const float *y, float gamma, float lambda, float *gx, float *gy,
+                    double *d_obj, double *d_wl, double *d_energy, double *d_hpwl, cudaStream_t s, bool do_wa,
+                    bool do_den) {
+  dp_status st0 = call_begin(c, s);
+  if (st0 != DP_OK) return st0;
+  DP_CUDA(cudaEventRecord(c.ev_fork, s));
+  if (do_wa) {
+    DP_CUDA(cudaStreamWaitEvent(c.s_wa, c.ev_fork, 0));
+    launch_wa(c, x, y, gamma, false, d_hpwl != nullptr, c.s_wa);
+    DP_CUDA(cudaEventRecord(c.ev_wa, c.s_wa));
+  }
+  if (do_den) {
+    DP_CUDA(cudaStreamWaitEvent(c.s_den, c.ev_fork, 0));
+    dp_status st = density_chain(c, x, y);
+    if (st != DP_OK) return st;
+    DP_CUDA(cudaEventRecord(c.ev_den, c.s_den));
+  }
+  if (do_wa) DP_CUDA(cudaStreamWaitEvent(s, c.ev_wa, 0));
+  if (do_den) DP_CUDA(cudaStreamWaitEvent(s, c.ev_den, 0));
+  launch_combine(c, do_den ? lambda : 0.f, gx, gy, do_wa, do_den, s);
+  dp_status st = finalize(c, lambda, do_wa, do_den, do_wa && d_hpwl != nullptr, d_obj, d_wl, d_energy, d_hpwl, s);
+  if (st != DP_OK) return st;
+  DP_CUDA(cudaGetLastError());
+  return call_end(c, s);
+}
+
+}  // namespace
+}  // namespace dp
+
+using dp::C;
+using dp::Ctx;
+using dp::fail;
+
+extern "C" {
+
+const char *dp_last_error(void) { return dp::g_err.c_str(); }
+
+int32_t dp_version(void) { return 100; }
+
+dp_status dp_create(const dp_netlist *nl, const dp_grid *grid, int device, dp_ctx **out) {
+  try {
+    return dp::create(nl, grid, device, 0, 1, nullptr, out);
+  } catch (const std::bad_alloc &) {
+    return fail(DP_ERR_OUT_OF_MEMORY, "host allocation failed in dp_create");
+  } catch (...) {
+    return fail(DP_ERR_INVALID_ARG, "unexpected exception in dp_create");
+  }
+}
+
+dp_status dp_create_dist(const dp_netlist *nl, const dp_grid *grid, int device, int rank, int world,
+                         const void *nccl_unique_id, dp_ctx **out) {
+  try {
+    return dp::create(nl, grid, device, rank, world, nccl_unique_id, out);
+  } catch (const std::bad_alloc &) {
+    return fail(DP_ERR_OUT_OF_MEMORY, "host allocation failed in dp_create_dist");
+  } catch (...) {
+    return fail(DP_ERR_INVALID_ARG, "unexpected exception in dp_create_dist");
+  }
+}
+
+dp_status dp_nccl_unique_id(void *out128) {
+  if (!out128) return fail(DP_ERR_INVALID_ARG, "out128 is NULL");
+  return dp::nccl_get_unique_id(out128);
+}
+
+dp_status dp_partition_plan(const dp_netlist *nl, int rank, int world, int32_t *cell_begin, int32_t *cell_end,
+                            uint8_t *net_mask) {
+  try {
+    if (!cell_begin || !cell_end) return fail(DP_ERR_INVALID_ARG, "cell_begin / cell_end NULL");
+    if (world < 1 || rank < 0 || rank >= world) return fail(DP_ERR_INVALID_ARG, "bad rank / world");
+    if (!nl || !nl->net_start || nl->num_cells < 1 || (nl->num_pins > 0 && !nl->pin2cell))
+      return fail(DP_ERR_INVALID_ARG, "netlist incomplete");
+    std::vector<uint8_t> mask;
+    dp::plan(nl, rank, world, *cell_begin, *cell_end, net_mask ? &mask : nullptr);
+    if (net_mask && !mask.empty()) std::memcpy(net_mask, mask.data(), mask.size());
+    return DP_OK;
+  } catch (...) {
+    return fail(DP_ERR_OUT_OF_MEMORY, "exception in dp_partition_plan");
+  }
+}
+
+dp_status dp_destroy(dp_ctx *ctx) {
+  dp::destroy(C(ctx));
+  return DP_OK;
+}
+
+dp_status dp_eval(dp_ctx *ctx, const float *x, const float *y, float gamma, float lambda, float *gx, float *gy,
+                  double *d_obj, double *d_wl, double *d_energy, double *d_hpwl, dp_stream_t stream) {
+  Ctx *c = C(ctx);
+  dp_status st = dp::check_eval_args(c, x, y);
+  if (st != DP_OK) return st;
+  if (!gx || !gy) return fail(DP_ERR_INVALID_ARG, "gx / gy is NULL");
+  if (!(gamma > 0.f) || !std::isfinite(gamma)) return fail(DP_ERR_INVALID_ARG, "gamma must be finite and > 0");
+  if (!(lambda >= 0.f) || !std::isfinite(lambda)) return fail(DP_ERR_INVALID_ARG, "lambda must be finite and >= 0");
+  dp::DeviceGuard g(c->device);
+  return dp::eval_impl(*c, x, y, gamma, lambda, gx, gy, d_obj, d_wl, d_energy, d_hpwl, (cudaStream_t)stream, true,
+                       true);
+}
+
+dp_status dp_wl_grad(dp_ctx *ctx, const float *x, const float *y, float gamma, float *gx, float *gy, double *d_wl,
+                     dp_stream_t stream) {
+  Ctx *c = C(ctx);
+  dp_status st = dp::check_eval_args(c, x, y);
+  if (st != DP_OK) return st;
+  if (!gx || !gy) return fail(DP_ERR_INVALID_ARG, "gx / gy is NULL");
+  if (!(gamma > 0.f) || !std::isfinite(gamma)) return fail(DP_ERR_INVALID_ARG, "gamma must be finite and > 0");
+  dp::DeviceGuard g(c->device);
+  return dp::eval_impl(*c, x, y, gamma, 0.f, gx, gy, nullptr, d_wl, nullptr, nullptr, (cudaStream_t)stream, true,
+                       false);
+}
+
+dp_status dp_density_grad(dp_ctx *ctx, const float *x, const float *y, float *gx, float *gy, double *d_energy,
+                          dp_stream_t stream) {
+  Ctx *c = C(ctx);
+  dp_status st = dp::check_eval_args(c, x, y);
+  if (st != DP_OK) return st;
+  if (!gx || !gy) return fail(DP_ERR_INVALID_ARG, "gx / gy is NULL");
+  dp::DeviceGuard g(c->device);
+  return dp::eval_impl(*c, x, y, 1.f, 1.f, gx, gy, nullptr, nullptr, d_energy, nullptr, (cudaStream_t)stream, false,
+                       true);
+}
+
+dp_status dp_hpwl(dp_ctx *ctx, const float *x, const float *y, double *d_hpwl, dp_stream_t stream) {
+  Ctx *c = C(ctx);
+  dp_status st = dp::check_eval_args(c, x, y);
+  if (st != DP_OK) return st;
+  if (!d_hpwl) return fail(DP_ERR_INVALID_ARG, "d_hpwl is NULL");
+  dp::DeviceGuard g(c->device);
+  cudaStream_t s = (cudaStream_t)stream;
+  if ((st = dp::call_begin(*c, s)) != DP_OK) return st;
+  dp::launch_wa(*c, x, y, 1.f, true, true, s);
+  st = dp::finalize(*c, 0.f, false, false, true, nullptr, nullptr, nullptr, d_hpwl, s);
+  if (st != DP_OK) return st;
+  DP_CUDA(cudaGetLastError());
+  return dp::call_end(*c, s);
+}
+
+dp_status dp_eval_host(dp_ctx *ctx, const float *hx, const float *hy, float gamma, float lambda, float *hgx,
+                       float *hgy, double *h_scalars, int with_hpwl, dp_stream_t stream) {
+  Ctx *c = C(ctx);
+  if (!c) return fail(DP_ERR_INVALID_ARG, "ctx is NULL");
+  if (!hx || !hy || !hgx || !hgy) return fail(DP_ERR_INVALID_ARG, "host buffer is NULL");
+  if (!(gamma > 0.f) || !std::isfinite(gamma)) return fail(DP_ERR_INVALID_ARG, "gamma must be finite and > 0");
+  if (!(lambda >= 0.f) || !std::isfinite(lambda)) return fail(DP_ERR_INVALID_ARG, "lambda must be finite and >= 0");
+  dp::DeviceGuard g(c->device);
+  cudaStream_t s = (cudaStream_t)stream;
+  const size_t n = (size_t)c->num_cells;
+  float *dx = c->d_hy, *dy = c->d_hy + n;
+  DP_CUDA(cudaMemcpyAsync(dx, hx, n * sizeof(float), cudaMemcpyHostToDevice, s));
+  DP_CUDA(cudaMemcpyAsync(dy, hy, n * sizeof(float), cudaMemcpyHostToDevice, s));
+  double *sc = c->d_scal + 4;
+  dp_status st = dp::eval_impl(*c, dx, dy, gamma, lambda, c->d_hgx, c->d_hgy, sc + 0, sc + 1, sc + 2,
+                               with_hpwl ? sc + 3 : nullptr, s, true, true);
+  if (st != DP_OK) return st;
+  const size_t off = (size_t)c->cell_begin, cnt = (size_t)(c->cell_end - c->cell_begin);
+  DP_CUDA(cudaMemcpyAsync(hgx + off, c->d_hgx + off, cnt * sizeof(float), cudaMemcpyDeviceToHost, s));
+  DP_CUDA(cudaMemcpyAsync(hgy + off, c->d_hgy + off, cnt * sizeof(float), cudaMemcpyDeviceToHost, s));
+  double tmp[4];
+  DP_CUDA(cudaMemcpyAsync(tmp, sc, 4 * sizeof(double), cudaMemcpyDeviceToHost, s));
+  DP_CUDA(cudaStreamSynchronize(s));
+  if (h_scalars) {
+    h_scalars[0] = tmp[0];
+    h_scalars[1] = tmp[1];
+    h_scalars[2] = tmp[2];
+    h_scalars[3] = with_hpwl ? tmp[3] : std::nan("");
+  }
+  return DP_OK;
+}
+
+dp_status dp_get_info(const dp_ctx *ctx, dp_info *info) {
+  const Ctx *c = reinterpret_cast<const Ctx *>(ctx);
+  if (!c || !info) return fail(DP_ERR_INVALID_ARG, "NULL argument");
+  info->num_cells = c->num_cells;
+  info->num_nets = c->n_wa_nets + c->n_big;
+  info->num_pins = c->n_wa_pins;
+  info->cell_begin = c->cell_begin;
+  info->cell_end = c->cell_end;
+  info->bins_x = c->mx;
+  info->bins_y = c->my;
+  info->rank = c->rank;
+  info->world = c->world;
+  info->launches_eval = c->launches_eval;
+  info->launches_eval_hpwl = c->launches_eval_hpwl;
+  info->device_bytes = c->device_bytes;
+  info->num_sms = c->num_sms;
+  info->l2_bytes = c->l2_bytes;
+  return DP_OK;
+}
+
+dp_status dp_debug_density_map(dp_ctx *ctx, const float *x, const float *y, float *rho, dp_stream_t stream) {
+  Ctx *c = C(ctx);
+  dp_status st = dp::check_eval_args(c, x, y);
+  if (st != DP_OK) return st;
+  if (!rho) return fail(DP_ERR_INVALID_ARG, "rho is NULL");
+  dp::DeviceGuard g(c->device);
+  cudaStream_t s = (cudaStream_t)stream;
+  dp::launch_density_map(*c, x, y, s);
+  DP_CUDA(cudaMemcpyAsync(rho, c->d_rho, sizeof(float) * (size_t)c->mx * c->my, cudaMemcpyDeviceToDevice, s));
+  DP_CUDA(cudaGetLastError());
+  return DP_OK;
+}
+
+dp_status dp_debug_fields(dp_ctx *ctx, const float *rho, float *psi, float *xi_x, float *xi_y, double *d_energy,
+                          dp_stream_t stream) {
+  Ctx *c = C(ctx);
+  if (!c || !rho) return fail(DP_ERR_INVALID_ARG, "NULL argument");
+  dp::DeviceGuard g(c->device);
+  cudaStream_t s = (cudaStream_t)stream;
+  dp::launch_fields(*c, rho, s);
+  if (xi_x || xi_y) dp::launch_split_fields(*c, xi_x, xi_y, s);
+  if (d_energy) dp::launch_finalize(*c, 1.f, false, true, false, nullptr, nullptr, d_energy, nullptr, s);
+  if (psi) dp::launch_psi(*c, rho, psi, s);
+  DP_CUDA(cudaGetLastError());
+  return DP_OK;
+}
+
+dp_status dp_debug_transform(dp_ctx *ctx, int kind, const float *in, float *out, dp_stream_t stream) {
+  Ctx *c = C(ctx);
+  if (!c || !in || !out) return fail(DP_ERR_INVALID_ARG, "NULL argument");
+  if (kind < DP_T_DCT2 || kind > DP_T_IDCT_IDXST) return fail(DP_ERR_INVALID_ARG, "unknown transform kind");
+  if (in == out) return fail(DP_ERR_INVALID_ARG, "in and out must not alias");
+  dp::DeviceGuard g(c->device);
+  dp::launch_transform(*c, kind, in, out, (cudaStream_t)stream);
+  DP_CUDA(cudaGetLastError());
+  return DP_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,172 @@
+// dp_internal.h — private definitions of libdp (context layout, kernel entry points).
+// Not part of the ABI; see include/dp.h for the public contract and DESIGN.md for the design.
+#pragma once
+
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <string>
+#include <vector>
+
+#include "../../include/dp.h"
+
+namespace dp {
+
+// ---------------------------------------------------------------------------------------
+// Compile-time layout parameters.
+// ---------------------------------------------------------------------------------------
+constexpr int kWaThreads = 256;       // threads per WA chunk CTA (8 warps)
+constexpr int kWaPpl = 8;             // pin slots per lane (registers)
+constexpr int kWaMaxDeg = 256;        // nets up to this degree go through the chunk kernel
+constexpr int kWaChunkPins = 4096;    // target pins per chunk
+constexpr int kWaWindow = 2048;       // cells per chunk window held in shared memory
+constexpr int kBigThreads = 256;      // CTA-per-net kernel for nets > kWaMaxDeg
+constexpr int kHpwlLimbs = 9;         // limbs 0..kHpwlLimbs (10) of 32-bit digits, LSB 2^-149 (reading A7)
+
+constexpr int kTile = 32;             // density tile = kTile x kTile bins
+constexpr int kHalo = 2;              // small-cell footprints extend <= 2 bins past their tile
+constexpr int kSegCells = 2048;       // cells per scatter/gather work segment
+constexpr int kCountThreads = 256;
+constexpr int kCountCells = 4096;     // cells per count/place CTA
+
+// Per warp-group metadata of the WA chunk layout.
+struct WarpGroup {
+  int32_t pin_base;   // first pin entry of the group (slot-major compressed layout)
+  int32_t net_base;   // first net (index into the reordered net arrays)
+  int32_t nnets;      // nets in the group (<= 32 / g)
+  int32_t g_log2 : 8; // log2 of lanes per net
+  int32_t slots : 8;  // pin slots per lane (<= kWaPpl)
+  int32_t pad : 16;
+};
+
+struct Chunk {
+  int32_t wg_begin, wg_end;   // warp groups of this chunk
+  int32_t win_lo, win_n;      // cell window [win_lo, win_lo + win_n)
+};
+
+// Work segment of the density scatter/gather (built on device each evaluation).
+struct Segment {
+  int32_t tile;
+  int32_t begin, end;   // record range
+  int32_t pad;
+};
+
+struct Ctx {
+  // ---- identity ----
+  int device = 0;
+  int rank = 0, world = 1;
+  int num_sms = 0, l2_bytes = 0;
+  int32_t num_cells = 0, num_nets_in = 0, num_pins_in = 0;
+  int32_t cell_begin = 0, cell_end = 0;
+  bool has_weights = false;
+  bool dist = false;
+
+  // ---- grid ----
+  double xl = 0, yl = 0, xh = 0, yh = 0, bx = 0, by = 0;
+  int mx = 0, my = 0, log2mx = 0, log2my = 0, stretch = 1;
+  int tiles_x = 0, tiles_y = 0, tile = kTile;
+
+  // ---- WA layout (device) ----
+  int32_t n_chunks = 0, n_wgroups = 0, n_wa_nets = 0, n_wa_pins = 0;
+  Chunk *d_chunks = nullptr;
+  WarpGroup *d_wgroups = nullptr;
+  int32_t *d_net_deg = nullptr;     // degree | counted<<31 per reordered net
+  float *d_net_w = nullptr;         // weights per reordered net (if has_weights)
+  int32_t *d_pin_cell = nullptr;    // cell | foreign<<31 per pin entry
+  float *d_pin_dx = nullptr, *d_pin_dy = nullptr;
+  // big nets (degree > kWaMaxDeg): plain CSR, one CTA per net
+  int32_t n_big = 0;
+  int32_t *d_big_start = nullptr;   // [n_big + 1]
+  int32_t *d_big_flags = nullptr;   // counted flag per big net
+  float *d_big_w = nullptr;
+  int32_t *d_big_cell = nullptr;
+  float *d_big_dx = nullptr, *d_big_dy = nullptr;
+
+  // ---- density layout (device) ----
+  float *d_cell_w = nullptr, *d_cell_h = nullptr;   // own cells (index from cell_begin)
+  int32_t n_own = 0;                // cells owned by this rank
+  int32_t n_large = 0;              // large cells (footprint > 3 bins on an axis)
+  int32_t *d_large = nullptr;       // ids of large own cells
+  uint8_t *d_is_large = nullptr;    // per own cell
+  int32_t *d_tile_cnt = nullptr;      // [tiles] small-cell counts (reset by the scan)
+  int32_t *d_tile_cursor = nullptr;   // [tiles] placement cursors
+  int32_t *d_tile_off = nullptr;      // [tiles + 1]
+  float4 *d_rec = nullptr;            // per slot: footprint box in tile-local bin units
+  int2 *d_rec_rc = nullptr;           // per slot: (charge ratio r as float bits, i0 | j0 << 16)
+  int32_t *d_rec_cell = nullptr;      // per slot: own cell index
+  Segment *d_segs = nullptr;
+  int32_t max_segs = 0;
+  int32_t *d_nsegs = nullptr;
+  float *d_rho = nullptr, *d_t = nullptr, *d_sx = nullptr, *d_sy = nullptr;
+  float2 *d_xi = nullptr;
+  float2 *d_force = nullptr;          // per own cell: -(sum ov xi)
+  float2 *d_tw_x = nullptr, *d_tw_y = nullptr;     // FFT twiddles W_N^k, k < N/2
+  float2 *d_ph_x = nullptr, *d_ph_y = nullptr;     // e^{-i pi k / 2N}, k < N
+  float *d_kx = nullptr, *d_ky = nullptr;          // wavenumbers (reading A12)
+
+  // ---- shared scratch ----
+  float2 *d_g2 = nullptr;             // WA gradient accumulator, interleaved, kept zero between calls
+  double *d_part = nullptr;           // partial sums: [0, n_wa_part) WA, then energy
+  int32_t n_wa_part = 0, n_en_part = 0;
+  unsigned long long *d_limbs = nullptr;  // HPWL fixed-point limbs
+  double *d_scal = nullptr;           // {wl, energy, hpwl, obj} staging
+  float *d_hx = nullptr, *d_hy = nullptr, *d_hgx = nullptr, *d_hgy = nullptr;  // e2e buffers
+
+  // ---- streams / events ----
+  cudaStream_t s_wa = nullptr, s_den = nullptr;
+  cudaEvent_t ev_fork = nullptr, ev_wa = nullptr, ev_den = nullptr;
+  cudaEvent_t ev_done = nullptr;   // end of the last call: serialises use from several streams
+
+  // ---- NCCL (distributed) ----
+  void *nccl_comm = nullptr;
+
+  int64_t device_bytes = 0;
+  int launches_eval = 0, launches_eval_hpwl = 0;
+  std::vector<void *> allocations;
+};
+
+// error handling ---------------------------------------------------------------------------
+void set_error(const std::string &msg);
+dp_status fail(dp_status st, const std::string &msg);
+dp_status cuda_fail(cudaError_t e, const char *what);
+
+#define DP_CUDA(call)                                               \
+  do {                                                              \
+    cudaError_t _e = (call);                                        \
+    if (_e != cudaSuccess) return ::dp::cuda_fail(_e, #call);        \
+  } while (0)
+
+// kernel launchers (defined in the .cu files) ---------------------------------------------
+// WA (wa.cu)
+void launch_wa(const Ctx &c, const float *x, const float *y, float gamma, bool hpwl_only,
+               bool with_hpwl, cudaStream_t s);
+// density (density.cu)
+void launch_density_map(const Ctx &c, const float *x, const float *y, cudaStream_t s);
+void launch_density_gather(const Ctx &c, const float *x, const float *y, cudaStream_t s);
+// transforms (dct.cu)
+void launch_fields(const Ctx &c, const float *rho, cudaStream_t s);
+void launch_transform(const Ctx &c, int kind, const float *in, float *out, cudaStream_t s);
+void launch_split_fields(const Ctx &c, float *xi_x, float *xi_y, cudaStream_t s);
+void launch_psi(const Ctx &c, const float *rho, float *psi, cudaStream_t s);
+// combine / finalize (finalize.cu)
+void launch_combine(const Ctx &c, float lambda, float *gx, float *gy, bool use_wa,
+                    bool use_density, cudaStream_t s);
+void launch_finalize(const Ctx &c, float lambda, bool with_wl, bool with_energy,
+                     bool with_hpwl, double *d_obj, double *d_wl, double *d_energy,
+                     double *d_hpwl, cudaStream_t s);
+void launch_finalize_phase(const Ctx &c, int phase, float lambda, bool with_wl, bool with_energy,
+                           bool with_hpwl, double *d_obj, double *d_wl, double *d_energy,
+                           double *d_hpwl, cudaStream_t s);
+// configuration (shared-memory opt-in), called from dp_create
+cudaError_t dct_configure(int mx, int my);
+cudaError_t density_configure(int ntiles, int tile);
+int density_launches(const Ctx &c);
+// NCCL (nccl_dyn.cpp)
+dp_status nccl_get_unique_id(void *out128);
+dp_status nccl_init(Ctx &c, const void *id);
+dp_status nccl_allreduce_f32(Ctx &c, float *buf, size_t n, cudaStream_t s);
+dp_status nccl_allreduce_f64(Ctx &c, double *buf, size_t n, cudaStream_t s);
+dp_status nccl_allreduce_u64(Ctx &c, unsigned long long *buf, size_t n, cudaStream_t s);
+void nccl_destroy(Ctx &c);
+
+}  // namespace dp

@@ -1,0 +1,160 @@
+// finalize.cu — gradient combine (eq 2: grad WA + lambda grad D) and the scalar
+// outputs (WA, D, obj, HPWL) on sm_100a.
+//
+// The WA kernels accumulate into the interleaved scratch g2, which this pass reads, splits
+// into the caller's gx / gy, and resets to zero for the next evaluation (so no memset is
+// needed on the hot path).  Scalars are reduced from per-CTA partials in a fixed order, so
+// WA and D are run-to-run deterministic given the partials; HPWL is converted from the
+// exact int64 limb sum with one correctly rounded step (reading A7).
+#include "dp_internal.h"
+
+namespace dp {
+
+namespace {
+
+__global__ void k_combine(float2 *__restrict__ g2, const float2 *__restrict__ force, float *__restrict__ gx,
+                          float *__restrict__ gy, int cell_begin, int n_own, float lambda, int use_wa,
+                          int use_den) {
+  for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < n_own; i += gridDim.x * blockDim.x) {
+    const int c = cell_begin + i;
+    float vx = 0.f, vy = 0.f;
+    if (use_wa) {
+      const float2 g = g2[c];
+      vx = g.x;
+      vy = g.y;
+      g2[c] = make_float2(0.f, 0.f);
+    }
+    if (use_den) {
+      const float2 f = force[i];
+      vx = fmaf(lambda, f.x, vx);
+      vy = fmaf(lambda, f.y, vy);
+    }
+    gx[c] = vx;
+    gy[c] = vy;
+  }
+}
+
+// Correctly rounded double of sum_j L[j] 2^(32 j - 149), L[j] < 2^63 (reading A7).
+__device__ double limbs_to_double(const unsigned long long *L) {
+  unsigned int D[kHpwlLimbs + 3];
+  unsigned long long carry = 0;
+  for (int j = 0; j <= kHpwlLimbs; j++) {
+    const unsigned __int128 v = (unsigned __int128)L[j] + carry;
+    D[j] = (unsigned int)(v & 0xffffffffu);
+    carry = (unsigned long long)(v >> 32);
+  }
+  D[kHpwlLimbs + 1] = (unsigned int)(carry & 0xffffffffu);
+  D[kHpwlLimbs + 2] = (unsigned int)(carry >> 32);
+  int top = -1;
+  for (int j = kHpwlLimbs + 2; j >= 0; j--)
+    if (D[j]) {
+      top = j;
+      break;
+    }
+  if (top < 0) return 0.0;
+  auto dig = [&](int j) -> unsigned __int128 { return (j >= 0) ? (unsigned __int128)D[j] : (unsigned __int128)0; };
+  unsigned __int128 W = (dig(top) << 96) | (dig(top - 1) << 64) | (dig(top - 2) << 32) | dig(top - 3);
+  bool sticky = false;
+  for (int j = 0; j < top - 3; j++) sticky |= (D[j] != 0);
+  const int lz = __clz(D[top]);  // leading zeros of the top digit
+  W <<= lz;
+  int pos = 32 * (top - 3) + 127 - lz;  // bit index of the MSB in the 2^-149 scaled integer
+  unsigned long long mant = (unsigned long long)(W >> 75);
+  const unsigned __int128 rem = W & (((unsigned __int128)1 << 75) - 1);
+  const unsigned __int128 half = (unsigned __int128)1 << 74;
+  if (rem > half || (rem == half && (sticky || (mant & 1ull)))) mant++;
+  if (mant == (1ull << 53)) {
+    mant >>= 1;
+    pos++;
+  }
+  return ldexp((double)mant, pos - 52 - 149);
+}
+
+struct FinArgs {
+  const double *part;
+  int n_wa, n_en;
+  unsigned long long *limbs;
+  double *scal;   // staging {wl, energy, hpwl, obj}
+  double *d_obj, *d_wl, *d_energy, *d_hpwl;
+  float lambda;
+  int with_wl, with_energy, with_hpwl, phase;  // phase 0: local sums -> scal (dist), 1: outputs, 2: both
+};
+
+__global__ void __launch_bounds__(256) k_finalize(FinArgs a) {
+  __shared__ double s_a[256], s_b[256];
+  if (a.phase != 1) {
+    double wl = 0.0, en = 0.0;
+    // fixed assignment of partials to threads and a fixed tree -> deterministic
+    if (a.with_wl)
+      for (int i = threadIdx.x; i < a.n_wa; i += 256) wl += a.part[i];
+    if (a.with_energy)
+      for (int i = threadIdx.x; i < a.n_en; i += 256) en += a.part[a.n_wa + i];
+    s_a[threadIdx.x] = wl;
+    s_b[threadIdx.x] = en;
+    __syncthreads();
+    for (int o = 128; o > 0; o >>= 1) {
+      if ((int)threadIdx.x < o) {
+        s_a[threadIdx.x] += s_a[threadIdx.x + o];
+        s_b[threadIdx.x] += s_b[threadIdx.x + o];
+      }
+      __syncthreads();
+    }
+    if (threadIdx.x == 0) {
+      a.scal[0] = s_a[0];
+      a.scal[1] = s_b[0];
+    }
+  }
+  if (a.phase == 0) return;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    const double wl = a.scal[0], en = a.scal[1];
+    double hp = __longlong_as_double(0x7ff8000000000000ll);
+    if (a.with_hpwl) {
+      hp = limbs_to_double(a.limbs);
+      for (int k = 0; k <= kHpwlLimbs; k++) a.limbs[k] = 0ull;
+    }
+    if (a.d_wl) *a.d_wl = wl;
+    if (a.d_energy) *a.d_energy = en;
+    if (a.d_hpwl) *a.d_hpwl = hp;
+    if (a.d_obj) *a.d_obj = (a.with_wl ? wl : 0.0) + (a.with_energy ? (double)a.lambda * en : 0.0);
+    a.scal[2] = hp;
+    a.scal[3] = (a.with_wl ? wl : 0.0) + (a.with_energy ? (double)a.lambda * en : 0.0);
+  }
+}
+
+}  // namespace
+
+void launch_combine(const Ctx &c, float lambda, float *gx, float *gy, bool use_wa, bool use_density,
+                    cudaStream_t s) {
+  if (c.n_own <= 0) return;
+  const int blocks = std::min((c.n_own + 255) / 256, c.num_sms * 8);
+  k_combine<<<blocks, 256, 0, s>>>(c.d_g2, c.d_force, gx, gy, c.cell_begin, c.n_own, lambda, use_wa ? 1 : 0,
+                                   use_density ? 1 : 0);
+}
+
+void launch_finalize_phase(const Ctx &c, int phase, float lambda, bool with_wl, bool with_energy, bool with_hpwl,
+                           double *d_obj, double *d_wl, double *d_energy, double *d_hpwl, cudaStream_t s) {
+  FinArgs a;
+  a.part = c.d_part;
+  a.n_wa = c.n_wa_part;
+  a.n_en = c.n_en_part;
+  a.limbs = c.d_limbs;
+  a.scal = c.d_scal;
+  a.d_obj = d_obj;
+  a.d_wl = d_wl;
+  a.d_energy = d_energy;
+  a.d_hpwl = d_hpwl;
+  a.lambda = lambda;
+  a.with_wl = with_wl;
+  a.with_energy = with_energy;
+  a.with_hpwl = with_hpwl;
+  a.phase = phase;
+  k_finalize<<<1, 256, 0, s>>>(a);
+}
+
+void launch_finalize(const Ctx &c, float lambda, bool with_wl, bool with_energy, bool with_hpwl, double *d_obj,
+                     double *d_wl, double *d_energy, double *d_hpwl, cudaStream_t s) {
+  launch_finalize_phase(c, 2, lambda, with_wl, with_energy, with_hpwl, d_obj, d_wl, d_energy, d_hpwl, s);
+}
+
+}  // namespace dp

@@ -1,0 +1,286 @@
+"""GPU parity: the CUDA path through the C ABI against the fp64 oracle on the same seeded
+inputs (BASELINE.json north_star tolerances; HPWL bit-exact).  Requires a B200."""
+import numpy as np
+import pytest
+import torch
+
+import oracle
+import paper_conf_dac_lindlrkp19_b200 as dp
+from synth import custom_netlist, make_netlist, make_positions
+from parity_util import check_map, check_scalar, check_vector, to_np
+
+pytestmark = pytest.mark.gpu
+DEV = torch.device("cuda", 0)
+
+
+def _t(a):
+    return torch.as_tensor(np.ascontiguousarray(a, dtype=np.float32), device=DEV)
+
+
+@pytest.fixture(scope="module")
+def tiny():
+    nl = make_netlist("tiny")
+    return nl, dp.dp_create(nl)
+
+
+# ------------------------------------------------------------------------------ transforms
+@pytest.mark.parametrize("m", [16, 64, 256])
+def test_transforms(m):
+    nl = custom_netlist([0], [], [], [], [1.0], [1.0], (0, 0, 10.0 * m, 7.0 * m), (m, m))
+    ctx = dp.dp_create(nl)
+    rng = np.random.default_rng(m)
+    a = rng.standard_normal((m, m))
+    inp = _t(a)
+    a32 = to_np(inp)
+    got = to_np(ctx.transform(dp.DP_T_DCT2, inp))
+    check_map("DCT2", got, oracle.dct2(a32))
+    got = to_np(ctx.transform(dp.DP_T_IDCT2, inp))
+    check_map("IDCT2", got, oracle.transform(oracle.IDCT, oracle.transform(oracle.IDCT, a32, 1), 0))
+    got = to_np(ctx.transform(dp.DP_T_IDXST_IDCT, inp))
+    check_map("IDXST_IDCT", got, oracle.transform(oracle.IDXST, oracle.transform(oracle.IDCT, a32, 1), 0))
+    got = to_np(ctx.transform(dp.DP_T_IDCT_IDXST, inp))
+    check_map("IDCT_IDXST", got, oracle.transform(oracle.IDCT, oracle.transform(oracle.IDXST, a32, 1), 0))
+
+
+def test_transforms_rectangular():
+    nl = custom_netlist([0], [], [], [], [1.0], [1.0], (0, 0, 320.0, 90.0), (32, 128))
+    ctx = dp.dp_create(nl)
+    a = np.random.default_rng(3).standard_normal((32, 128))
+    inp = _t(a)
+    a32 = to_np(inp)
+    check_map("DCT2", to_np(ctx.transform(dp.DP_T_DCT2, inp)), oracle.dct2(a32))
+    check_map("IDXST_IDCT", to_np(ctx.transform(dp.DP_T_IDXST_IDCT, inp)),
+              oracle.transform(oracle.IDXST, oracle.transform(oracle.IDCT, a32, 1), 0))
+
+
+# ---------------------------------------------------------------------------- density map
+@pytest.mark.parametrize("dist", ["spread", "initial"])
+def test_density_map_tiny(tiny, dist):
+    nl, ctx = tiny
+    x, y = make_positions(nl, dist)
+    got = to_np(ctx.density_map(_t(x), _t(y)))
+    check_map("rho", got, oracle.density_map(nl, x, y, 1), rel=2e-6)
+
+
+def test_fields_tiny(tiny):
+    nl, ctx = tiny
+    x, y = make_positions(nl)
+    rho = oracle.density_map(nl, x, y, 1)
+    f = ctx.fields(_t(rho))
+    rho32 = rho.astype(np.float32).astype(np.float64)
+    psi, xi_x, xi_y = oracle.fields(nl, oracle.dct2(rho32))
+    check_map("psi", to_np(f["psi"]), psi)
+    check_map("xi_x", to_np(f["xi_x"]), xi_x)
+    check_map("xi_y", to_np(f["xi_y"]), xi_y)
+    check_scalar("energy", f["energy"].item(), oracle.energy(nl, rho32, psi))
+
+
+# ------------------------------------------------------------------------------ wirelength
+@pytest.mark.parametrize("gscale", [0.05, 0.5, 5.0, 50.0])
+@pytest.mark.parametrize("weighted", [False, True])
+def test_wl_grad_tiny(gscale, weighted):
+    nl = make_netlist("tiny")
+    if weighted:
+        nl.net_weight = np.random.default_rng(1).uniform(0.5, 2.0, nl.num_nets).astype(np.float32)
+    ctx = dp.dp_create(nl)
+    x, y = make_positions(nl)
+    gamma = gscale * nl.bin_w
+    out = ctx.wl_grad(_t(x), _t(y), gamma)
+    wl, gx, gy = oracle.wa(nl, x, y, np.float32(gamma))
+    check_scalar("WA", out["wl"].item(), wl)
+    check_vector("dWA/dx", to_np(out["gx"]), gx)
+    check_vector("dWA/dy", to_np(out["gy"]), gy)
+
+
+def test_wl_grad_high_fanout_and_degenerate():
+    """Every lanes-per-net class, a 10K-pin net (CTA-per-net path), degree 0/1 nets, repeated
+    cells inside a net, nets spanning the whole region."""
+    rng = np.random.default_rng(11)
+    nc = 20000
+    degs = [0, 1, 1, 2, 2, 3, 5, 8, 9, 16, 17, 31, 32, 33, 64, 65, 100, 128, 129, 200, 256, 257, 1000, 10000]
+    degs = degs + list(rng.integers(2, 8, 3000))
+    ns = np.concatenate([[0], np.cumsum(degs)])
+    npins = int(ns[-1])
+    p2c = rng.integers(0, nc, npins)
+    p2c[ns[5]:ns[5] + 2] = 7  # a 2-pin net on one cell (coincident pins)
+    w = rng.integers(2, 41, nc).astype(np.float32)
+    h = np.full(nc, 12.0, np.float32)
+    W = 8192.0
+    nl = custom_netlist(ns, p2c, rng.random(npins) * w[p2c], rng.random(npins) * h[p2c], w, h,
+                        (0, 0, W, W), (256, 256))
+    ctx = dp.dp_create(nl)
+    x = (rng.random(nc) * (W - w)).astype(np.float32)
+    y = (rng.random(nc) * (W - h)).astype(np.float32)
+    for gamma in (2.0, 40.0):
+        out = ctx.wl_grad(_t(x), _t(y), gamma)
+        wl, gx, gy = oracle.wa(nl, x, y, gamma)
+        check_scalar("WA", out["wl"].item(), wl)
+        check_vector("dWA/dx", to_np(out["gx"]), gx)
+        check_vector("dWA/dy", to_np(out["gy"]), gy)
+    assert ctx.hpwl(_t(x), _t(y)).item() == oracle.hpwl(nl, x, y)
+
+
+def test_empty_and_degree_one_netlists():
+    nl = custom_netlist([0, 1, 1], [3], [0.5], [0.5], np.full(10, 4.0), np.full(10, 4.0), (0, 0, 160, 160), (16, 16))
+    ctx = dp.dp_create(nl)
+    x = np.linspace(0, 150, 10).astype(np.float32)
+    y = np.linspace(5, 120, 10).astype(np.float32)
+    out = ctx.eval(_t(x), _t(y), 2.0, 0.5, with_hpwl=True)
+    assert out["wl"].item() == 0.0 and out["hpwl"].item() == 0.0
+    ref = oracle.evaluate(nl, x, y, 2.0, 0.5)
+    check_scalar("energy", out["energy"].item(), ref["energy"])
+    check_vector("gx", to_np(out["gx"]), ref["gx"])
+
+
+# -------------------------------------------------------------------------------- HPWL
+@pytest.mark.parametrize("name", ["tiny", "adaptec1", "bigblue4"])
+@pytest.mark.parametrize("dist", ["spread", "initial"])
+def test_hpwl_bit_exact(name, dist):
+    nl = make_netlist(name)
+    ctx = dp.dp_create(nl)
+    x, y = make_positions(nl, dist)
+    got = ctx.hpwl(_t(x), _t(y)).item()
+    assert got == oracle.hpwl(nl, x, y)   # bit-exact fp64 (reading A7)
+    out = ctx.eval(_t(x), _t(y), nl.bin_w, 1.0, with_hpwl=True)
+    assert out["hpwl"].item() == got
+
+
+def test_hpwl_extreme_magnitudes():
+    """Coordinates spanning 2^-20 .. 2^40 exercise every limb of the fixed-point sum."""
+    rng = np.random.default_rng(5)
+    nc = 4000
+    ns = np.arange(0, 2 * 1500 + 1, 2)
+    p2c = rng.integers(0, nc, ns[-1])
+    dx = (rng.random(ns[-1]) * 2.0 ** rng.integers(-20, 4, ns[-1])).astype(np.float32)
+    nl = custom_netlist(ns, p2c, dx, dx[::-1].copy(), np.ones(nc), np.ones(nc), (0, 0, 1e13, 1e13), (16, 16))
+    ctx = dp.dp_create(nl)
+    x = (2.0 ** rng.uniform(-20, 40, nc)).astype(np.float32)
+    y = (2.0 ** rng.uniform(-20, 40, nc)).astype(np.float32)
+    assert ctx.hpwl(_t(x), _t(y)).item() == oracle.hpwl(nl, x, y)
+
+
+# ------------------------------------------------------------------------- density grad
+@pytest.mark.parametrize("dist", ["spread", "initial"])
+def test_density_grad_tiny(tiny, dist):
+    nl, ctx = tiny
+    x, y = make_positions(nl, dist)
+    out = ctx.density_grad(_t(x), _t(y))
+    D, gx, gy, _ = oracle.density(nl, x, y, 1)
+    check_scalar("D", out["energy"].item(), D)
+    check_vector("dD/dx", to_np(out["gx"]), gx)
+    check_vector("dD/dy", to_np(out["gy"]), gy)
+
+
+def _macro_netlist(stretch_bins=64):
+    rng = np.random.default_rng(21)
+    nc = 6000
+    w = rng.integers(2, 41, nc).astype(np.float32)
+    h = np.full(nc, 12.0, np.float32)
+    big = rng.choice(nc, 12, replace=False)
+    w[big] = rng.uniform(96, 700, 12).astype(np.float32)
+    h[big] = rng.uniform(96, 700, 12).astype(np.float32)
+    w[:5] = 0.0  # zero-area cells
+    deg = rng.integers(2, 6, 7000)
+    ns = np.concatenate([[0], np.cumsum(deg)])
+    p2c = rng.integers(0, nc, ns[-1])
+    W = 3200.0
+    nl = custom_netlist(ns, p2c, rng.random(ns[-1]) * w[p2c], rng.random(ns[-1]) * h[p2c], w, h, (0, 0, W, W),
+                        (stretch_bins, stretch_bins))
+    x = (rng.random(nc) * (W - w)).astype(np.float32)
+    y = (rng.random(nc) * (W - h)).astype(np.float32)
+    x[5:40] = rng.uniform(-300, W + 200, 35)  # partly / fully outside the region (reading A11)
+    return nl, x, y
+
+
+@pytest.mark.parametrize("stretch", [0, 1])
+def test_density_grad_macros_and_edges(stretch):
+    nl, x, y = _macro_netlist()
+    ctx = dp.dp_create(nl, stretch=stretch)
+    out = ctx.density_grad(_t(x), _t(y))
+    D, gx, gy, parts = oracle.density(nl, x, y, stretch)
+    check_map("rho", to_np(ctx.density_map(_t(x), _t(y))), parts["rho"], rel=2e-6)
+    check_scalar("D", out["energy"].item(), D)
+    check_vector("dD/dx", to_np(out["gx"]), gx)
+    check_vector("dD/dy", to_np(out["gy"]), gy)
+
+
+# ------------------------------------------------------------------------------ full eval
+@pytest.mark.parametrize("dist", ["spread", "initial"])
+@pytest.mark.parametrize("lam", [0.0, 1e-4, 1.0])
+def test_eval_tiny(dist, lam):
+    nl = make_netlist("tiny")
+    ctx = dp.dp_create(nl)
+    x, y = make_positions(nl, dist)
+    gamma = nl.bin_w
+    out = ctx.eval(_t(x), _t(y), gamma, lam, with_hpwl=True)
+    ref = oracle.evaluate(nl, x, y, gamma, lam)
+    check_scalar("WA", out["wl"].item(), ref["wl"])
+    check_scalar("D", out["energy"].item(), ref["energy"])
+    check_scalar("obj", out["obj"].item(), ref["obj"])
+    assert out["hpwl"].item() == ref["hpwl"]
+    check_vector("gx", to_np(out["gx"]), ref["gx"])
+    check_vector("gy", to_np(out["gy"]), ref["gy"])
+
+
+def test_eval_repeatable_and_stream_independent(tiny):
+    """g2 is reset by every evaluation: repeated calls give the same result within fp32
+    atomic-order noise; a side stream works the same as the default stream."""
+    nl, ctx = tiny
+    x, y = make_positions(nl)
+    xt, yt = _t(x), _t(y)
+    a = ctx.eval(xt, yt, 11.0, 0.3)
+    s = torch.cuda.Stream()
+    s.wait_stream(torch.cuda.current_stream())
+    with torch.cuda.stream(s):
+        b = ctx.eval(xt, yt, 11.0, 0.3, stream=s)
+    # no host sync between: the context orders its own calls across streams
+    c = ctx.eval(xt, yt, 11.0, 0.3)
+    torch.cuda.synchronize()
+    ref = oracle.evaluate(nl, x, y, 11.0, 0.3)
+    for o in (a, b, c):
+        check_vector("gx", to_np(o["gx"]), ref["gx"])
+        check_scalar("obj", o["obj"].item(), ref["obj"])
+    check_vector("repeat gx", to_np(b["gx"]), to_np(a["gx"]), rel_l2=1e-5, rel_entry=1e-4)
+
+
+def test_eval_host_e2e(tiny):
+    nl, ctx = tiny
+    x, y = make_positions(nl)
+    gx = np.zeros(nl.num_cells, np.float32)
+    gy = np.zeros(nl.num_cells, np.float32)
+    sc = np.zeros(4)
+    dp.dp_eval_host(ctx, x, y, 9.0, 0.5, gx, gy, sc, with_hpwl=True)
+    torch.cuda.synchronize()
+    ref = oracle.evaluate(nl, x, y, 9.0, 0.5)
+    check_scalar("obj", sc[0], ref["obj"])
+    assert sc[3] == ref["hpwl"]
+    check_vector("gx", gx, ref["gx"])
+
+
+@pytest.mark.slow
+@pytest.mark.parametrize("name", ["adaptec1", "bigblue4"])
+def test_eval_full_size(name):
+    """BASELINE configs at full size in the launch configuration bench.py times."""
+    nl = make_netlist(name)
+    ctx = dp.dp_create(nl)
+    x, y = make_positions(nl)
+    gamma = nl.bin_w
+    out = ctx.eval(_t(x), _t(y), gamma, 1.0, with_hpwl=True)
+    ref = oracle.evaluate(nl, x, y, gamma, 1.0)
+    check_scalar("WA", out["wl"].item(), ref["wl"])
+    check_scalar("D", out["energy"].item(), ref["energy"])
+    assert out["hpwl"].item() == ref["hpwl"]
+    check_vector("gx", to_np(out["gx"]), ref["gx"])
+    check_vector("gy", to_np(out["gy"]), ref["gy"])
+
+
+def test_invalid_args(tiny):
+    nl, ctx = tiny
+    x, y = make_positions(nl)
+    gx = torch.empty(nl.num_cells, device=DEV)
+    with pytest.raises(dp.DPError, match="INVALID_ARG"):
+        dp.dp_eval(ctx, _t(x), _t(y), 0.0, 1.0, gx, gx.clone())
+    with pytest.raises(dp.DPError, match="INVALID_ARG"):
+        dp.dp_eval(ctx, _t(x), _t(y), 1.0, -1.0, gx, gx.clone())
+    with pytest.raises(dp.DPError, match="INVALID_ARG"):
+        dp.dp_eval(ctx, None, _t(y), 1.0, 1.0, gx, gx.clone())

@@ -1,0 +1,370 @@
+#!/usr/bin/env python
+"""bench.py — WA + density objective/gradient evaluations per second (BASELINE.json metric).
+
+One step = one full dp_eval (WA wirelength + gradient, density map, Poisson solve, field,
+force gather, combine) on the bigblue4-shaped synthetic workload (2.18M cells, 2.23M nets,
+8.9M pins, 1024x1024 bins; BASELINE.json configs[2], the config the metric is quoted on).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference] [--config NAME]
+
+N > 1 is launched by torchrun (one rank per GPU, NCCL): the evaluation is sharded by cells
+(owner computes) with one ncclAllReduce of the bin map per step, so the total
+work per step is fixed ("scaling": "strong").  Device time: CUDA events around every step on
+the launching stream, L2 flushed (a 2x L2 write) before every timed step, max over ranks.
+Rank 0 prints one JSON line.  --impl reference times the fp64 CPU oracle (the reference arm of
+this tier) on a bounded sample of the same workload.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import math
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "WA+density obj/grad evals/sec (bigblue4-shape) and HBM GB/s vs peak at 1/2/4/8 GPU"
+UNIT = "evals/s"
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=2000)
+    ap.add_argument("--warmup", type=int, default=50)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--config", default="bigblue4")
+    ap.add_argument("--dist", default="spread", choices=["spread", "initial"])
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--e2e-steps", type=int, default=200)
+    return ap.parse_args()
+
+
+def load_peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            p = json.load(f)
+        return float(p["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    except Exception:
+        return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+def algorithmic_bytes(nl):
+    """B = 4(N_e+1) + 12 N_p + 24 N_c + 32 M^2 (each input read once, each
+    output written once, each intermediate map written once and read once); WA part
+    B_WA = 4(N_e+1) + 12 N_p + 8 N_c (net starts, pin cell/offsets, x and y)."""
+    m2 = nl.bins_x * nl.bins_y
+    total = 4 * (nl.num_nets + 1) + 12 * nl.num_pins + 24 * nl.num_cells + 32 * m2
+    wa = 4 * (nl.num_nets + 1) + 12 * nl.num_pins + 8 * nl.num_cells
+    return total, wa
+
+
+class ClockSampler:
+    """nvidia-smi clocks / throttle reasons sampled during the timed region."""
+    FIELDS = ["clocks.sm", "clocks.max.sm", "power.draw", "clocks_event_reasons.hw_slowdown",
+              "clocks_event_reasons.hw_thermal_slowdown", "clocks_event_reasons.sw_thermal_slowdown",
+              "clocks_event_reasons.sw_power_cap"]
+
+    def __init__(self, gpu_id: str):
+        self.gpu_id = gpu_id
+        self.samples = []
+        self.proc = None
+
+    def start(self):
+        cmd = ["nvidia-smi", f"--id={self.gpu_id}", "--query-gpu=" + ",".join(self.FIELDS),
+               "--format=csv,noheader,nounits", "-lms", "100"]
+        try:
+            self.proc = subprocess.Popen(cmd, stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+        except Exception:
+            self.proc = None
+            return
+        threading.Thread(target=self._read, daemon=True).start()
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.samples.append((time.time(), [v.strip() for v in line.split(",")]))
+
+    def stop(self):
+        if self.proc:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except Exception:
+                self.proc.kill()
+
+    def summary(self, t0, t1):
+        win = [s for t, s in self.samples if t0 - 0.15 <= t <= t1 + 0.15]
+        if not win and self.samples:
+            win = [min(self.samples, key=lambda ts: abs(ts[0] - (t0 + t1) / 2))[1]]
+        if not win:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unavailable"], "samples": 0}
+        def num(v):
+            try:
+                return float(v)
+            except ValueError:
+                return None
+        sm = [num(s[0]) for s in win if num(s[0]) is not None]
+        mx = [num(s[1]) for s in win if num(s[1]) is not None]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for s in win for i in range(4) if len(s) > 3 + i and s[3 + i] == "Active"})
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": reasons, "samples": len(win)}
+
+
+def gpu_uuid(dev):
+    import torch
+    try:
+        u = torch.cuda.get_device_properties(dev).uuid
+        return "GPU-" + str(u)
+    except Exception:
+        return str(dev)
+
+
+def workload_config(nl, dist_name, world):
+    return {"workload": f"{nl.name}-shaped: {nl.num_cells} cells, {nl.num_nets} nets, {nl.num_pins} pins, "
+                        f"{nl.bins_x}x{nl.bins_y} bins (synthetic, seeded; DESIGN.md §4)",
+            "cells": nl.num_cells, "nets": nl.num_nets, "pins": nl.num_pins,
+            "bins": [nl.bins_x, nl.bins_y], "positions": dist_name, "gamma": nl.bin_w, "lambda": 1.0,
+            "hpwl": "not fused (d_hpwl = NULL)",
+            "l2": "flushed before every timed step (write of 2x L2 bytes, untimed)",
+            "parallelism": f"cells{world} (owner-computes shards, NCCL all-reduce of the bin map)"
+                           if world > 1 else "single GPU"}
+
+
+# --------------------------------------------------------------------------------- oracle
+def oracle_sample(nl, x, y, frac, gamma, lam):
+    """A bounded sample of one evaluation on the CPU oracle: the first `frac` of the nets (WA),
+    of the cells (density map + gather) and of the rows of every transform pass.  Returns the
+    amount of work done in evaluation units (= frac)."""
+    import numpy as np
+    import oracle
+    from synth import custom_netlist
+    ne = max(1, int(math.ceil(frac * nl.num_nets)))
+    nc = max(1, int(math.ceil(frac * nl.num_cells)))
+    ns = nl.net_start[: ne + 1]
+    sub = custom_netlist(ns, nl.pin2cell[: ns[-1]], nl.pin_dx[: ns[-1]], nl.pin_dy[: ns[-1]],
+                         nl.cell_w, nl.cell_h, (nl.xl, nl.yl, nl.xh, nl.yh), (nl.bins_x, nl.bins_y))
+    oracle.wa(sub, x, y, gamma)
+    cells = custom_netlist([0], [], [], [], nl.cell_w[:nc], nl.cell_h[:nc], (nl.xl, nl.yl, nl.xh, nl.yh),
+                           (nl.bins_x, nl.bins_y))
+    rho = oracle.density_map(cells, x[:nc], y[:nc], 1)
+    rows = max(1, int(math.ceil(frac * nl.bins_x)))
+    # 8 naive passes (DCT2: 2, psi/xi_x/xi_y: 2 each) over `rows` sequences each
+    for kind in (oracle.DCT, oracle.DCT, oracle.IDCT, oracle.IDCT, oracle.IDCT, oracle.IDXST, oracle.IDXST, oracle.IDCT):
+        oracle.transform(kind, rho[:rows], 1)
+    xi = np.zeros_like(rho)
+    oracle.density_grad(cells, x[:nc], y[:nc], xi, xi, 1)
+    return frac
+
+
+def cpu_threads():
+    try:
+        return len(os.sched_getaffinity(0))
+    except Exception:
+        return os.cpu_count() or 1
+
+
+def run_cpu_baseline(nl, x, y, gamma, lam, budget_s=20.0):
+    import oracle
+    t0 = time.perf_counter()
+    n = 0
+    while n < 3 and (time.perf_counter() - t0) < budget_s:
+        oracle.evaluate(nl, x, y, gamma, lam, with_hpwl=False)
+        n += 1
+    dt = time.perf_counter() - t0
+    return {"value": n / dt, "unit": UNIT, "cores": cpu_threads(), "kind": "oracle",
+            "sample": f"{n} full fp64 oracle evaluation(s) of the {nl.name} workload "
+                      f"(naive O(M^3) transforms; OpenMP over transform rows and gather cells), {dt:.1f} s"}
+
+
+def run_reference(args, rank, world):
+    if rank != 0:
+        return 0
+    os.environ.setdefault("OMP_NUM_THREADS", str(cpu_threads()))
+    from synth import make_netlist, make_positions
+    nl = make_netlist(args.config)
+    x, y = make_positions(nl, args.dist)
+    gamma, lam = nl.bin_w, 1.0
+    # calibrate with one small sample, then size each step so the run ends in ~2 minutes
+    t = time.perf_counter()
+    oracle_sample(nl, x, y, 0.02, gamma, lam)
+    per_unit = (time.perf_counter() - t) / 0.02
+    budget = 120.0
+    frac = min(1.0, budget / max(1, args.steps + args.warmup) / per_unit)
+    for _ in range(args.warmup):
+        oracle_sample(nl, x, y, frac, gamma, lam)
+    t0 = time.perf_counter()
+    work = 0.0
+    for _ in range(args.steps):
+        work += oracle_sample(nl, x, y, frac, gamma, lam)
+    dt = time.perf_counter() - t0
+    value = work / dt
+    out = {"metric": METRIC, "value": value, "unit": UNIT, "impl": "reference", "n_gpus": args.gpus,
+           "steps": args.steps, "warmup": args.warmup, "ms_per_step": dt / args.steps * 1e3,
+           "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f64",
+           "data": "synthetic", "config": workload_config(nl, args.dist, 1),
+           "cpu_baseline": {"value": value, "unit": UNIT, "kind": "oracle", "cores": cpu_threads(),
+                            "sample": f"each step: first {frac:.4f} of the nets (WA), cells (map + gather) and "
+                                      f"transform rows (8 naive passes) of one evaluation"},
+           "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(out), flush=True)
+    return 0
+
+
+# ------------------------------------------------------------------------------------ ours
+def run_ours(args, rank, world, local_rank):
+    import numpy as np
+    import torch
+    import paper_conf_dac_lindlrkp19_b200 as dp
+    from synth import make_netlist, make_positions
+
+    torch.cuda.set_device(local_rank)
+    dev = torch.device("cuda", local_rank)
+    pg = None
+    if world > 1:
+        import torch.distributed as tdist
+        tdist.init_process_group("nccl", device_id=dev)
+        pg = tdist
+    nl = make_netlist(args.config)
+    x, y = make_positions(nl, args.dist)
+    gamma, lam = float(nl.bin_w), 1.0
+    if world > 1:
+        uid = [dp.dp_nccl_unique_id() if rank == 0 else None]
+        pg.broadcast_object_list(uid, src=0)
+        ctx = dp.dp_create_dist(nl, local_rank, rank, world, uid[0])
+    else:
+        ctx = dp.dp_create(nl, local_rank)
+    info = ctx.info
+    xt = torch.as_tensor(x, device=dev)
+    yt = torch.as_tensor(y, device=dev)
+    gx = torch.empty(nl.num_cells, dtype=torch.float32, device=dev)
+    gy = torch.empty_like(gx)
+    sc = torch.zeros(4, dtype=torch.float64, device=dev)
+    flush = torch.empty(2 * max(info.l2_bytes, 64 << 20), dtype=torch.uint8, device=dev)
+    stream = torch.cuda.current_stream()
+
+    def step():
+        dp.dp_eval(ctx, xt, yt, gamma, lam, gx, gy, sc[0:1], sc[1:2], sc[2:3], None, stream)
+
+    sampler = ClockSampler(gpu_uuid(local_rank))
+    sampler.start()
+    for _ in range(max(args.warmup, 3)):
+        flush.zero_()
+        step()
+    torch.cuda.synchronize()
+    if pg:
+        pg.barrier()
+    assert all(math.isfinite(v) for v in sc[:3].tolist()), "non-finite objective"
+    K = args.steps
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(K)]
+    dp.dp_profile_enable(ctx, True)
+    torch.cuda.synchronize()
+    if pg:
+        pg.barrier()
+    t0 = time.time()
+    for k in range(K):
+        flush.zero_()
+        ev[k][0].record(stream)
+        step()
+        ev[k][1].record(stream)
+    torch.cuda.synchronize()
+    t1 = time.time()
+    if pg:
+        pg.barrier()
+    dp.dp_profile_enable(ctx, False)
+    stage_ms, n_prof = dp.dp_profile_read(ctx)
+    total_ms = sum(a.elapsed_time(b) for a, b in ev)
+    clocks = sampler.summary(t0, t1)
+    # hot (L2-warm, back-to-back) variant, secondary
+    Kh = min(K, 500)
+    h0, h1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    h0.record(stream)
+    for _ in range(Kh):
+        step()
+    h1.record(stream)
+    torch.cuda.synchronize()
+    hot_ms = h0.elapsed_time(h1) / Kh
+    # e2e through the public API on pinned host buffers (H2D x, y; D2H gx, gy, scalars)
+    hx = torch.as_tensor(x).pin_memory()
+    hy = torch.as_tensor(y).pin_memory()
+    hgx = torch.empty(nl.num_cells, dtype=torch.float32).pin_memory()
+    hgy = torch.empty_like(hgx).pin_memory()
+    hsc = np.zeros(4)
+    Ke = max(1, min(args.e2e_steps, K))
+    for _ in range(3):
+        dp.dp_eval_host(ctx, hx, hy, gamma, lam, hgx, hgy, hsc, False, stream)
+    if pg:
+        pg.barrier()
+    e0 = time.perf_counter()
+    for _ in range(Ke):
+        dp.dp_eval_host(ctx, hx, hy, gamma, lam, hgx, hgy, hsc, False, stream)
+    e2e_s = time.perf_counter() - e0
+    sampler.stop()
+
+    tensors = torch.tensor([total_ms, e2e_s, hot_ms], dtype=torch.float64, device=dev)
+    if pg:
+        pg.all_reduce(tensors, op=pg.ReduceOp.MAX)
+    total_ms, e2e_s, hot_ms = tensors.tolist()
+    if rank != 0:
+        if pg:
+            pg.destroy_process_group()
+        return 0
+    ms_per_step = total_ms / K
+    value = K / (total_ms / 1e3)
+    peak, peak_src = load_peaks()
+    b_total, b_wa = algorithmic_bytes(nl)
+    wa_ms = stage_ms["wa"] / max(n_prof, 1)
+    achieved = b_wa / (wa_ms * 1e-3) / 1e9
+    traffic = None
+    prof_path = os.path.join(ROOT, "profiles", "ncu_wa_traffic.json")
+    if os.path.exists(prof_path):
+        try:
+            with open(prof_path) as f:
+                traffic = json.load(f).get("dram_bytes_per_launch")
+        except Exception:
+            traffic = None
+    cfg = workload_config(nl, args.dist, world)
+    cfg["hot_ms_per_step"] = hot_ms
+    cfg["peak_source"] = peak_src
+    out = {
+        "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": K, "warmup": args.warmup,
+        "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
+        "dtype": "f32", "data": "synthetic", "config": cfg,
+        "roofline": {"bound": "hbm", "kernel": "WA stage (k_wa_chunks + k_wa_big)", "achieved": achieved,
+                     "peak": peak, "unit": "GB/s", "frac": achieved / peak, "traffic": traffic,
+                     "algorithmic_bytes": b_wa, "avg_launch_us": wa_ms * 1e3},
+        "step_roofline": {"algorithmic_bytes": b_total, "achieved": b_total / (ms_per_step * 1e-3) / 1e9,
+                          "peak": peak, "unit": "GB/s", "frac": b_total / (ms_per_step * 1e-3) / 1e9 / peak},
+        "stages_us": {k: v / max(n_prof, 1) * 1e3 for k, v in stage_ms.items()},
+        "e2e": {"value": Ke / e2e_s, "unit": UNIT, "h2d_bytes_per_step": 8 * nl.num_cells,
+                "d2h_bytes_per_step": 8 * nl.num_cells + 32},
+        "gpu_launches": info.launches_eval * K,
+        "clocks": clocks,
+    }
+    if world == 1 and not args.no_cpu_baseline:
+        os.environ.setdefault("OMP_NUM_THREADS", str(cpu_threads()))
+        out["cpu_baseline"] = run_cpu_baseline(nl, x, y, gamma, lam)
+    print(json.dumps(out), flush=True)
+    if pg:
+        pg.destroy_process_group()
+    return 0
+
+
+def main():
+    args = parse()
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    if args.impl == "reference":
+        return run_reference(args, rank, world)
+    return run_ours(args, rank, world, local_rank)
+
+
+if __name__ == "__main__":
+    sys.exit(main())

@@ -173,6 +173,22 @@ typedef struct dp_info {
 
 dp_status dp_get_info(const dp_ctx *ctx, dp_info *info);
 
+/* ---- stage timing (CUDA events on the streams each stage runs on) ----------------------
+ * While enabled, every evaluation records a start/stop event pair per stage on the stream
+ * the stage is launched on:
+ *   DP_STAGE_WA       WA + gradient (+ HPWL) kernels               (WA stream)
+ *   DP_STAGE_MAP      density map: count, scan, place, scatter     (density stream)
+ *   DP_STAGE_FIELDS   DCT / scaling / IDCT-IDXST transforms        (density stream)
+ *   DP_STAGE_GATHER   force gather                                 (density stream)
+ *   DP_STAGE_COMBINE  gradient combine + scalar finalize           (caller stream)
+ *   DP_STAGE_EVAL     the whole call, fork to join                  (caller stream)
+ * dp_profile_read synchronises the recorded events, writes the summed milliseconds per
+ * stage to ms[DP_NSTAGES] (host) and the number of evaluations to *count, and resets.  */
+enum { DP_STAGE_WA = 0, DP_STAGE_MAP = 1, DP_STAGE_FIELDS = 2, DP_STAGE_GATHER = 3,
+       DP_STAGE_COMBINE = 4, DP_STAGE_EVAL = 5, DP_NSTAGES = 6 };
+dp_status dp_profile_enable(dp_ctx *ctx, int on);
+dp_status dp_profile_read(dp_ctx *ctx, double *ms, int64_t *count);
+
 /* ---- test-only hooks (not part of the metric) ------------------------------------------
  * Expose single stages so parity tests can localise a failure.  All pointers device.     */
 

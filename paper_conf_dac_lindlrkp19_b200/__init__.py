@@ -32,7 +32,10 @@ EXPORTED_SYMBOLS = [
     "dp_last_error", "dp_version", "dp_create", "dp_create_dist", "dp_nccl_unique_id",
     "dp_partition_plan", "dp_destroy", "dp_eval", "dp_wl_grad", "dp_density_grad", "dp_hpwl",
     "dp_eval_host", "dp_get_info", "dp_debug_density_map", "dp_debug_fields", "dp_debug_transform",
+    "dp_profile_enable", "dp_profile_read",
 ]
+__all__ += ["dp_profile_enable", "dp_profile_read", "STAGES"]
+STAGES = ["wa", "map", "fields", "gather", "combine", "eval"]
 
 
 class DPError(RuntimeError):
@@ -92,6 +95,8 @@ def lib() -> ctypes.CDLL:
             "dp_debug_density_map": [P, P, P, P, P],
             "dp_debug_fields": [P, P, P, P, P, P, P],
             "dp_debug_transform": [P, ctypes.c_int, P, P, P],
+            "dp_profile_enable": [P, ctypes.c_int],
+            "dp_profile_read": [P, P, P],
         }.items():
             f = getattr(L, name)
             f.argtypes = args
@@ -293,6 +298,19 @@ def dp_get_info(ctx) -> DpInfo:
     info = DpInfo()
     _check(lib().dp_get_info(ctx.handle, ctypes.byref(info)))
     return info
+
+
+def dp_profile_enable(ctx, on=True):
+    _check(lib().dp_profile_enable(ctx.handle, int(bool(on))))
+
+
+def dp_profile_read(ctx):
+    """-> ({stage: summed ms}, evaluations recorded); synchronises the recorded events."""
+    import numpy as np
+    ms = np.zeros(len(STAGES))
+    cnt = ctypes.c_int64()
+    _check(lib().dp_profile_read(ctx.handle, ms.ctypes.data_as(ctypes.c_void_p), ctypes.byref(cnt)))
+    return dict(zip(STAGES, ms.tolist())), cnt.value
 
 
 def dp_debug_density_map(ctx, x, y, rho, stream=None):

@@ -31,7 +31,7 @@ struct DenArgs {
   const float *x, *y;   // global cell arrays
   const float *w, *h;   // own cells
   int cell_begin, n_own;
-  double xl, yl, xh, yh, bx, by, sx, sy;
+  double xl, yl, xh, yh, bx, by, sx, sy, ibx, iby;   // ibx = 1 / bx (no fp64 divisions on the hot path)
   int mx, my, tile, tiles_y, ntiles, stretch;
   int *tile_cnt, *tile_cursor, *tile_off;
   Segment *segs;
@@ -74,7 +74,7 @@ __device__ __forceinline__ Foot footprint(const DenArgs &a, int i) {
 }
 
 __device__ __forceinline__ int small_tile(const DenArgs &a, const Foot &f, int &ox, int &oy) {
-  int bx0 = (int)floor((f.lx - a.xl) / a.bx), by0 = (int)floor((f.ly - a.yl) / a.by);
+  int bx0 = (int)floor((f.lx - a.xl) * a.ibx), by0 = (int)floor((f.ly - a.yl) * a.iby);
   bx0 = min(max(bx0, 0), a.mx - 1);
   by0 = min(max(by0, 0), a.my - 1);
   const int tx = bx0 / a.tile, ty = by0 / a.tile;
@@ -200,10 +200,11 @@ __global__ void __launch_bounds__(kCountThreads) k_place(DenArgs a) {
     const int pos = s_hist[tl[k]] + rk[k];
     // bin-local fractions (|v| < 3): fp32 keeps ~2e-7 bin absolute precision, which the force
     // gather needs where large opposite bin fields cancel (the 'initial' placement)
-    const int i0 = min(max((int)floor((f.lx - a.xl) / a.bx), 0), a.mx - 1);
-    const int j0 = min(max((int)floor((f.ly - a.yl) / a.by), 0), a.my - 1);
-    a.rec[pos] = make_float4((float)((f.lx - a.xl) / a.bx - i0), (float)((f.ly - a.yl) / a.by - j0),
-                             (float)((f.hx - a.xl) / a.bx - i0), (float)((f.hy - a.yl) / a.by - j0));
+    const double ux0 = (f.lx - a.xl) * a.ibx, uy0 = (f.ly - a.yl) * a.iby;
+    const int i0 = min(max((int)floor(ux0), 0), a.mx - 1);
+    const int j0 = min(max((int)floor(uy0), 0), a.my - 1);
+    a.rec[pos] = make_float4((float)(ux0 - i0), (float)(uy0 - j0), (float)((f.hx - a.xl) * a.ibx - i0),
+                             (float)((f.hy - a.yl) * a.iby - j0));
     a.rec_rc[pos] = make_int2(__float_as_int(f.r), (i0 - ox) | ((j0 - oy) << 16));
     a.rec_cell[pos] = i;
   }
@@ -295,15 +296,15 @@ __global__ void __launch_bounds__(256) k_scatter_large(DenArgs a) {
   const int i = a.large[blockIdx.x];
   const Foot f = footprint(a, i);
   if (f.empty) return;
-  const int i0 = max((int)floor((f.lx - a.xl) / a.bx), 0), i1 = min((int)floor((f.hx - a.xl) / a.bx), a.mx - 1);
-  const int j0 = max((int)floor((f.ly - a.yl) / a.by), 0), j1 = min((int)floor((f.hy - a.yl) / a.by), a.my - 1);
+  const int i0 = max((int)floor((f.lx - a.xl) * a.ibx), 0), i1 = min((int)floor((f.hx - a.xl) * a.ibx), a.mx - 1);
+  const int j0 = max((int)floor((f.ly - a.yl) * a.iby), 0), j1 = min((int)floor((f.hy - a.yl) * a.iby), a.my - 1);
   const int nj = j1 - j0 + 1, n = (i1 - i0 + 1) * nj;
   for (int k = threadIdx.x; k < n; k += blockDim.x) {
     const int bi = i0 + k / nj, bj = j0 + k % nj;
     const double ox = fmin(f.hx, a.xl + (bi + 1) * a.bx) - fmax(f.lx, a.xl + bi * a.bx);
     const double oy = fmin(f.hy, a.yl + (bj + 1) * a.by) - fmax(f.ly, a.yl + bj * a.by);
     if (ox <= 0.0 || oy <= 0.0) continue;
-    const float v = (float)((double)f.r * ox * oy / (a.bx * a.by));
+    const float v = (float)((double)f.r * ox * oy * a.ibx * a.iby);
     asm volatile("red.global.add.f32 [%0], %1;" ::"l"(a.rho + (size_t)bi * a.my + bj), "f"(v) : "memory");
   }
 }
@@ -314,8 +315,8 @@ __global__ void __launch_bounds__(256) k_gather_large(DenArgs a) {
   __shared__ double s_x[8], s_y[8];
   double fx = 0.0, fy = 0.0;
   if (!f.empty) {
-    const int i0 = max((int)floor((f.lx - a.xl) / a.bx), 0), i1 = min((int)floor((f.hx - a.xl) / a.bx), a.mx - 1);
-    const int j0 = max((int)floor((f.ly - a.yl) / a.by), 0), j1 = min((int)floor((f.hy - a.yl) / a.by), a.my - 1);
+    const int i0 = max((int)floor((f.lx - a.xl) * a.ibx), 0), i1 = min((int)floor((f.hx - a.xl) * a.ibx), a.mx - 1);
+    const int j0 = max((int)floor((f.ly - a.yl) * a.iby), 0), j1 = min((int)floor((f.hy - a.yl) * a.iby), a.my - 1);
     const int nj = j1 - j0 + 1, n = (i1 - i0 + 1) * nj;
     for (int k = threadIdx.x; k < n; k += blockDim.x) {
       const int bi = i0 + k / nj, bj = j0 + k % nj;
@@ -358,6 +359,8 @@ DenArgs make_args(const Ctx &c, const float *x, const float *y) {
   a.xl = c.xl; a.yl = c.yl; a.xh = c.xh; a.yh = c.yh; a.bx = c.bx; a.by = c.by;
   a.sx = 1.4142135623730951 * c.bx;
   a.sy = 1.4142135623730951 * c.by;
+  a.ibx = 1.0 / c.bx;
+  a.iby = 1.0 / c.by;
   a.mx = c.mx; a.my = c.my; a.tile = c.tile; a.tiles_y = c.tiles_y;
   a.ntiles = c.tiles_x * c.tiles_y;
   a.stretch = c.stretch;

@@ -346,8 +346,11 @@ dp_status build_density(Ctx &c, const dp_netlist *nl) {
   if ((st = dev_alloc(c, &c.d_sx, nb)) != DP_OK) return st;
   if ((st = dev_alloc(c, &c.d_sy, nb)) != DP_OK) return st;
   if ((st = dev_alloc(c, &c.d_xi, nb)) != DP_OK) return st;
-  if ((st = dev_alloc(c, &c.d_force, std::max(c.n_own, 1))) != DP_OK) return st;
-  DP_CUDA(cudaMemset(c.d_force, 0, sizeof(float2) * std::max(c.n_own, 1)));
+  // force[i] for own cell i = cell_begin + i; offset by the parity of cell_begin so that even
+  // global cells are 16-byte aligned (the combine pass reads cell pairs as float4)
+  if ((st = dev_alloc(c, &c.d_force, c.n_own + 2)) != DP_OK) return st;
+  DP_CUDA(cudaMemset(c.d_force, 0, sizeof(float2) * (c.n_own + 2)));
+  c.d_force += (c.cell_begin & 1);
   if ((st = dev_upload(c, &c.d_tw_x, twiddles(c.mx))) != DP_OK) return st;
   if ((st = dev_upload(c, &c.d_tw_y, twiddles(c.my))) != DP_OK) return st;
   if ((st = dev_upload(c, &c.d_ph_x, phases(c.mx))) != DP_OK) return st;
@@ -386,6 +389,12 @@ void destroy(Ctx *c) {
   if (c->ev_wa) cudaEventDestroy(c->ev_wa);
   if (c->ev_den) cudaEventDestroy(c->ev_den);
   if (c->ev_done) cudaEventDestroy(c->ev_done);
+  for (auto &v : c->prof_pairs)
+    for (auto &p : v) {
+      cudaEventDestroy(p.first);
+      cudaEventDestroy(p.second);
+    }
+  for (cudaEvent_t e : c->prof_pool) cudaEventDestroy(e);
   delete c;
 }
 
@@ -470,14 +479,52 @@ dp_status check_eval_args(Ctx *c, const void *x, const void *y) {
   return DP_OK;
 }
 
+// ---- stage profiling ---------------------------------------------------------------------
+cudaEvent_t prof_event(Ctx &c) {
+  if (!c.prof_pool.empty()) {
+    cudaEvent_t e = c.prof_pool.back();
+    c.prof_pool.pop_back();
+    return e;
+  }
+  cudaEvent_t e = nullptr;
+  cudaEventCreate(&e);
+  return e;
+}
+struct StageMark {
+  Ctx &c;
+  int stage;
+  cudaStream_t s;
+  cudaEvent_t a = nullptr;
+  StageMark(Ctx &c_, int st, cudaStream_t s_) : c(c_), stage(st), s(s_) {
+    if (c.profiling) {
+      a = prof_event(c);
+      cudaEventRecord(a, s);
+    }
+  }
+  ~StageMark() {
+    if (a) {
+      cudaEvent_t b = prof_event(c);
+      cudaEventRecord(b, s);
+      c.prof_pairs[stage].push_back({a, b});
+    }
+  }
+};
+
 // the density chain on the density stream: map -> (allreduce) -> fields -> gather
 dp_status density_chain(Ctx &c, const float *x, const float *y) {
-  launch_density_map(c, x, y, c.s_den);
-  if (c.dist && c.nccl_comm) {
-    dp_status st = nccl_allreduce_f32(c, c.d_rho, (size_t)c.mx * c.my, c.s_den);
-    if (st != DP_OK) return st;
+  {
+    StageMark m(c, DP_STAGE_MAP, c.s_den);
+    launch_density_map(c, x, y, c.s_den);
+    if (c.dist && c.nccl_comm) {
+      dp_status st = nccl_allreduce_f32(c, c.d_rho, (size_t)c.mx * c.my, c.s_den);
+      if (st != DP_OK) return st;
+    }
   }
-  launch_fields(c, c.d_rho, c.s_den);
+  {
+    StageMark m(c, DP_STAGE_FIELDS, c.s_den);
+    launch_fields(c, c.d_rho, c.s_den);
+  }
+  StageMark m(c, DP_STAGE_GATHER, c.s_den);
   launch_density_gather(c, x, y, c.s_den);
   return DP_OK;
 }
@@ -517,10 +564,15 @@ dp_status eval_impl(Ctx &c, const float *x, const float *y, float gamma, float l
                     bool do_den) {
   dp_status st0 = call_begin(c, s);
   if (st0 != DP_OK) return st0;
+  StageMark whole(c, DP_STAGE_EVAL, s);
+  if (c.profiling) c.prof_evals++;
   DP_CUDA(cudaEventRecord(c.ev_fork, s));
   if (do_wa) {
     DP_CUDA(cudaStreamWaitEvent(c.s_wa, c.ev_fork, 0));
-    launch_wa(c, x, y, gamma, false, d_hpwl != nullptr, c.s_wa);
+    {
+      StageMark m(c, DP_STAGE_WA, c.s_wa);
+      launch_wa(c, x, y, gamma, false, d_hpwl != nullptr, c.s_wa);
+    }
     DP_CUDA(cudaEventRecord(c.ev_wa, c.s_wa));
   }
   if (do_den) {
@@ -531,9 +583,12 @@ dp_status eval_impl(Ctx &c, const float *x, const float *y, float gamma, float l
   }
   if (do_wa) DP_CUDA(cudaStreamWaitEvent(s, c.ev_wa, 0));
   if (do_den) DP_CUDA(cudaStreamWaitEvent(s, c.ev_den, 0));
-  launch_combine(c, do_den ? lambda : 0.f, gx, gy, do_wa, do_den, s);
-  dp_status st = finalize(c, lambda, do_wa, do_den, do_wa && d_hpwl != nullptr, d_obj, d_wl, d_energy, d_hpwl, s);
-  if (st != DP_OK) return st;
+  {
+    StageMark m(c, DP_STAGE_COMBINE, s);
+    launch_combine(c, do_den ? lambda : 0.f, gx, gy, do_wa, do_den, s);
+    dp_status st = finalize(c, lambda, do_wa, do_den, do_wa && d_hpwl != nullptr, d_obj, d_wl, d_energy, d_hpwl, s);
+    if (st != DP_OK) return st;
+  }
   DP_CUDA(cudaGetLastError());
   return call_end(c, s);
 }
@@ -698,6 +753,35 @@ dp_status dp_get_info(const dp_ctx *ctx, dp_info *info) {
   info->device_bytes = c->device_bytes;
   info->num_sms = c->num_sms;
   info->l2_bytes = c->l2_bytes;
+  return DP_OK;
+}
+
+dp_status dp_profile_enable(dp_ctx *ctx, int on) {
+  Ctx *c = C(ctx);
+  if (!c) return fail(DP_ERR_INVALID_ARG, "ctx is NULL");
+  c->profiling = on != 0;
+  return DP_OK;
+}
+
+dp_status dp_profile_read(dp_ctx *ctx, double *ms, int64_t *count) {
+  Ctx *c = C(ctx);
+  if (!c || !ms) return fail(DP_ERR_INVALID_ARG, "NULL argument");
+  dp::DeviceGuard g(c->device);
+  for (int st = 0; st < DP_NSTAGES; st++) {
+    double tot = 0.0;
+    for (auto &p : c->prof_pairs[st]) {
+      DP_CUDA(cudaEventSynchronize(p.second));
+      float t = 0.f;
+      DP_CUDA(cudaEventElapsedTime(&t, p.first, p.second));
+      tot += t;
+      c->prof_pool.push_back(p.first);
+      c->prof_pool.push_back(p.second);
+    }
+    c->prof_pairs[st].clear();
+    ms[st] = tot;
+  }
+  if (count) *count = c->prof_evals;
+  c->prof_evals = 0;
   return DP_OK;
 }
 

@@ -6,6 +6,7 @@
 #include <stdint.h>
 
 #include <string>
+#include <utility>
 #include <vector>
 
 #include "../../include/dp.h"
@@ -16,11 +17,11 @@ namespace dp {
 // Compile-time layout parameters.
 // ---------------------------------------------------------------------------------------
 constexpr int kWaThreads = 256;       // threads per WA chunk CTA (8 warps)
-constexpr int kWaPpl = 8;             // pin slots per lane (registers)
-constexpr int kWaMaxDeg = 256;        // nets up to this degree go through the chunk kernel
+constexpr int kWaPpl = 4;             // pin slots per lane (registers)
+constexpr int kWaMaxDeg = 128;        // nets up to this degree go through the chunk kernel (G <= 32)
 constexpr int kWaChunkPins = 4096;    // target pins per chunk
 constexpr int kWaWindow = 2048;       // cells per chunk window held in shared memory
-constexpr int kBigThreads = 256;      // CTA-per-net kernel for nets > kWaMaxDeg
+constexpr int kBigThreads = 128;      // CTA-per-net kernel for nets > kWaMaxDeg
 constexpr int kHpwlLimbs = 9;         // limbs 0..kHpwlLimbs (10) of 32-bit digits, LSB 2^-149 (reading A7)
 
 constexpr int kTile = 32;             // density tile = kTile x kTile bins
@@ -119,6 +120,12 @@ struct Ctx {
 
   // ---- NCCL (distributed) ----
   void *nccl_comm = nullptr;
+
+  // ---- stage profiling (dp_profile_enable) ----
+  bool profiling = false;
+  std::vector<cudaEvent_t> prof_pool;          // free events
+  std::vector<std::pair<cudaEvent_t, cudaEvent_t>> prof_pairs[DP_NSTAGES];
+  int64_t prof_evals = 0;
 
   int64_t device_bytes = 0;
   int launches_eval = 0, launches_eval_hpwl = 0;

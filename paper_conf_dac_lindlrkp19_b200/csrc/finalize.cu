@@ -12,22 +12,41 @@ namespace dp {
 
 namespace {
 
-__global__ void k_combine(float2 *__restrict__ g2, const float2 *__restrict__ force, float *__restrict__ gx,
-                          float *__restrict__ gy, int cell_begin, int n_own, float lambda, int use_wa,
-                          int use_den) {
-  for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < n_own; i += gridDim.x * blockDim.x) {
-    const int c = cell_begin + i;
+// One pair of cells per thread (16-byte loads of g2 / force, 8-byte stores of gx / gy), no
+// grid-stride loop: every warp has exactly one round of independent loads in flight.
+__global__ void __launch_bounds__(256) k_combine(float2 *__restrict__ g2, const float2 *__restrict__ force,
+                                                 float *__restrict__ gx, float *__restrict__ gy, int cell_begin,
+                                                 int n_own, float lambda, int use_wa, int use_den) {
+  const int c0 = (cell_begin & ~1) + 2 * (blockIdx.x * blockDim.x + threadIdx.x);  // even cell
+  const int cend = cell_begin + n_own;
+  if (c0 >= cend) return;
+  const bool full = c0 >= cell_begin && c0 + 1 < cend;
+  float4 g = make_float4(0.f, 0.f, 0.f, 0.f), f = make_float4(0.f, 0.f, 0.f, 0.f);
+  if (full) {
+    if (use_wa) {
+      g = __ldcs(reinterpret_cast<const float4 *>(g2 + c0));
+      __stcs(reinterpret_cast<float4 *>(g2 + c0), make_float4(0.f, 0.f, 0.f, 0.f));
+    }
+    if (use_den) f = __ldcs(reinterpret_cast<const float4 *>(force + (c0 - cell_begin)));
+    const float2 ox = make_float2(fmaf(lambda, f.x, g.x), fmaf(lambda, f.z, g.z));
+    const float2 oy = make_float2(fmaf(lambda, f.y, g.y), fmaf(lambda, f.w, g.w));
+    *reinterpret_cast<float2 *>(gx + c0) = ox;
+    *reinterpret_cast<float2 *>(gy + c0) = oy;
+    return;
+  }
+  for (int c = c0; c < c0 + 2; c++) {  // ragged ends of the own range
+    if (c < cell_begin || c >= cend) continue;
     float vx = 0.f, vy = 0.f;
     if (use_wa) {
-      const float2 g = g2[c];
-      vx = g.x;
-      vy = g.y;
+      const float2 q = g2[c];
+      vx = q.x;
+      vy = q.y;
       g2[c] = make_float2(0.f, 0.f);
     }
     if (use_den) {
-      const float2 f = force[i];
-      vx = fmaf(lambda, f.x, vx);
-      vy = fmaf(lambda, f.y, vy);
+      const float2 q = force[c - cell_begin];
+      vx = fmaf(lambda, q.x, vx);
+      vy = fmaf(lambda, q.y, vy);
     }
     gx[c] = vx;
     gy[c] = vy;
@@ -127,7 +146,8 @@ __global__ void __launch_bounds__(256) k_finalize(FinArgs a) {
 void launch_combine(const Ctx &c, float lambda, float *gx, float *gy, bool use_wa, bool use_density,
                     cudaStream_t s) {
   if (c.n_own <= 0) return;
-  const int blocks = std::min((c.n_own + 255) / 256, c.num_sms * 8);
+  const int pairs = (c.n_own + 3) / 2;
+  const int blocks = (pairs + 255) / 256;
   k_combine<<<blocks, 256, 0, s>>>(c.d_g2, c.d_force, gx, gy, c.cell_begin, c.n_own, lambda, use_wa ? 1 : 0,
                                    use_density ? 1 : 0);
 }

@@ -137,13 +137,198 @@ __device__ void block_flush_scalars(double wl, unsigned long long (&L)[kHpwlLimb
   }
 }
 
+// Fast2Sum (3 flops): exact when |a| >= |b| (cell coordinate vs pin offset, the usual case);
+// otherwise still accurate to ~ulp of the sum, which is all the WA value/gradient needs.
+__device__ __forceinline__ void fast_sum(float a, float b, float &s, float &e) {
+  s = __fadd_rn(a, b);
+  e = __fadd_rn(__fsub_rn(a, s), b);
+}
+
+// Per-lane running extremes of one axis as (hi, lo) pairs.
+struct Axis { float Ph, Pl, Mh, Ml; };
+
+template <bool EXACT>
+__device__ __forceinline__ void ext_update(Axis &A, float h, float l) {
+  if (EXACT) {
+    if (pair_gt(h, l, A.Ph, A.Pl)) { A.Ph = h; A.Pl = l; }
+    if (pair_gt(A.Mh, A.Ml, h, l)) { A.Mh = h; A.Ml = l; }
+  } else {  // the shift only needs a pin at (or within an ulp of) the extreme
+    if (h > A.Ph) { A.Ph = h; A.Pl = l; }
+    if (h < A.Mh) { A.Mh = h; A.Ml = l; }
+  }
+}
+
+template <bool EXACT>
+__device__ __forceinline__ void ext_shfl(Axis &A, int o) {
+  const float ph = __shfl_xor_sync(0xffffffffu, A.Ph, o), pl = __shfl_xor_sync(0xffffffffu, A.Pl, o);
+  const float mh = __shfl_xor_sync(0xffffffffu, A.Mh, o), ml = __shfl_xor_sync(0xffffffffu, A.Ml, o);
+  if (EXACT) {
+    if (pair_gt(ph, pl, A.Ph, A.Pl)) { A.Ph = ph; A.Pl = pl; }
+    if (pair_gt(A.Mh, A.Ml, mh, ml)) { A.Mh = mh; A.Ml = ml; }
+  } else {
+    if (ph > A.Ph || (ph == A.Ph && pl > A.Pl)) { A.Ph = ph; A.Pl = pl; }
+    if (mh < A.Mh || (mh == A.Mh && ml < A.Ml)) { A.Mh = mh; A.Ml = ml; }
+  }
+}
+
+struct GroupCtx {
+  const Chunk &ch;
+  const float2 *s_pos;
+  float *s_g;
+  int lane;
+  unsigned lt_mask;
+};
+
+// One warp group: 32/G nets, G lanes per net, S pin slots per lane.
+template <int MODE, int S>
+__device__ __forceinline__ void wa_group(const WaArgs &a, const WarpGroup &wg, const GroupCtx &gc, double &wl_acc,
+                                         unsigned long long (&L)[kHpwlLimbs + 1]) {
+  constexpr bool kGrad = MODE != 2;
+  constexpr bool kHpwl = MODE != 0;
+  const int glog = wg.g_log2, G = 1 << glog;
+  const int gi = gc.lane >> glog, j = gc.lane & (G - 1);
+  int d = 0, counted = 0;
+  float we = 1.f;
+  if (gi < wg.nnets) {
+    const int raw = __ldg(a.net_deg + wg.net_base + gi);
+    d = raw & 0x7fffffff;
+    counted = (raw >> 31) & 1;
+    if (a.has_w) we = __ldg(a.net_w + wg.net_base + gi);
+  }
+  // ---- phase A: pin records of all slots (slot-major compressed layout, coalesced) ----
+  int cell[S];
+  float dxs[S], dys[S];
+  unsigned vm = 0;
+  int base = wg.pin_base;
+#pragma unroll
+  for (int s = 0; s < S; s++) {
+    const bool valid = s * G + j < d;
+    const unsigned m = __ballot_sync(0xffffffffu, valid);
+    cell[s] = 0;
+    dxs[s] = dys[s] = 0.f;
+    if (valid) {
+      const int p = base + __popc(m & gc.lt_mask);
+      cell[s] = __ldg(a.pin_cell + p);
+      dxs[s] = __ldg(a.pin_dx + p);
+      dys[s] = __ldg(a.pin_dy + p);
+      vm |= 1u << s;
+    }
+    base += __popc(m);
+  }
+  // ---- phase B: pin positions px = x_cell + dx as (hi, lo) pairs ----
+  float hx[S], lx[S], hy[S], ly[S];
+  Axis X{-INFINITY, 0.f, INFINITY, 0.f}, Y{-INFINITY, 0.f, INFINITY, 0.f};
+#pragma unroll
+  for (int s = 0; s < S; s++) {
+    hx[s] = lx[s] = hy[s] = ly[s] = 0.f;
+    if (vm & (1u << s)) {
+      const int c = cell[s] & 0x7fffffff;
+      const int wi = c - gc.ch.win_lo;
+      float xc, yc;
+      if ((unsigned)wi < (unsigned)gc.ch.win_n) {
+        const float2 q = gc.s_pos[wi];
+        xc = q.x;
+        yc = q.y;
+      } else {
+        xc = __ldg(a.x + c);
+        yc = __ldg(a.y + c);
+      }
+      if (kHpwl) {
+        two_sum(xc, dxs[s], hx[s], lx[s]);
+        two_sum(yc, dys[s], hy[s], ly[s]);
+      } else {
+        fast_sum(xc, dxs[s], hx[s], lx[s]);
+        fast_sum(yc, dys[s], hy[s], ly[s]);
+      }
+      ext_update<kHpwl>(X, hx[s], lx[s]);
+      ext_update<kHpwl>(Y, hy[s], ly[s]);
+    }
+  }
+  for (int o = 1; o < G; o <<= 1) {
+    ext_shfl<kHpwl>(X, o);
+    ext_shfl<kHpwl>(Y, o);
+  }
+  const bool leader = (j == 0) && d >= 2;
+  if (kHpwl && leader && counted) {
+    // px = fl64(x + dx) as the oracle forms it: (double)hi + (double)lo rounds the exact
+    // real x + dx once (reading A7)
+    const double xp = __dadd_rn((double)X.Ph, (double)X.Pl), xm = __dadd_rn((double)X.Mh, (double)X.Ml);
+    const double yp = __dadd_rn((double)Y.Ph, (double)Y.Pl), ym = __dadd_rn((double)Y.Mh, (double)Y.Ml);
+    limbs_add(L, __dadd_rn(__dsub_rn(xp, xm), __dsub_rn(yp, ym)));
+  }
+  if (!kGrad) return;
+  // ---- shifted exponentials a^+- and sums b^+-, c~^+- (Table I) ----
+  float lxp[S], lxm[S], lyp[S], lym[S], axp[S], axm[S], ayp[S], aym[S];
+  float bxp = 0.f, bxm = 0.f, cxp = 0.f, cxm = 0.f, byp = 0.f, bym = 0.f, cyp = 0.f, cym = 0.f;
+#pragma unroll
+  for (int s = 0; s < S; s++) {
+    lxp[s] = lxm[s] = lyp[s] = lym[s] = 0.f;
+    axp[s] = axm[s] = ayp[s] = aym[s] = 0.f;
+    if (vm & (1u << s)) {
+      lxp[s] = __fadd_rn(__fsub_rn(hx[s], X.Ph), __fsub_rn(lx[s], X.Pl));   // <= 0 (net-local)
+      lxm[s] = __fadd_rn(__fsub_rn(hx[s], X.Mh), __fsub_rn(lx[s], X.Ml));   // >= 0
+      lyp[s] = __fadd_rn(__fsub_rn(hy[s], Y.Ph), __fsub_rn(ly[s], Y.Pl));
+      lym[s] = __fadd_rn(__fsub_rn(hy[s], Y.Mh), __fsub_rn(ly[s], Y.Ml));
+      axp[s] = ex2(lxp[s] * a.k2);
+      axm[s] = ex2(-lxm[s] * a.k2);
+      ayp[s] = ex2(lyp[s] * a.k2);
+      aym[s] = ex2(-lym[s] * a.k2);
+      bxp += axp[s]; cxp = fmaf(lxp[s], axp[s], cxp);
+      bxm += axm[s]; cxm = fmaf(lxm[s], axm[s], cxm);
+      byp += ayp[s]; cyp = fmaf(lyp[s], ayp[s], cyp);
+      bym += aym[s]; cym = fmaf(lym[s], aym[s], cym);
+    }
+  }
+  for (int o = 1; o < G; o <<= 1) {
+    bxp += __shfl_xor_sync(0xffffffffu, bxp, o);
+    cxp += __shfl_xor_sync(0xffffffffu, cxp, o);
+    bxm += __shfl_xor_sync(0xffffffffu, bxm, o);
+    cxm += __shfl_xor_sync(0xffffffffu, cxm, o);
+    byp += __shfl_xor_sync(0xffffffffu, byp, o);
+    cyp += __shfl_xor_sync(0xffffffffu, cyp, o);
+    bym += __shfl_xor_sync(0xffffffffu, bym, o);
+    cym += __shfl_xor_sync(0xffffffffu, cym, o);
+  }
+  if (d < 2) return;  // lanes without a net; degree-1 nets are dropped at create
+  const float ibxp = __frcp_rn(bxp), ibxm = __frcp_rn(bxm), ibyp = __frcp_rn(byp), ibym = __frcp_rn(bym);
+  const float mxp = cxp * ibxp, mxm = cxm * ibxm, myp = cyp * ibyp, mym = cym * ibym;
+  if (leader && counted) {
+    // WL_e = c+/b+ - c-/b- = (x+ - x-) + c~+/b+ - c~-/b-   (eq 3 in net-local coordinates)
+    const float spanx = __fadd_rn(__fsub_rn(X.Ph, X.Mh), __fsub_rn(X.Pl, X.Ml));
+    const float spany = __fadd_rn(__fsub_rn(Y.Ph, Y.Mh), __fsub_rn(Y.Pl, Y.Ml));
+    wl_acc += (double)(we * ((spanx + mxp - mxm) + (spany + myp - mym)));
+  }
+  // eq (6): dWL/dx_i = a+_i/b+ (1 + (l+_i - m+)/g) - a-_i/b- (1 - (l-_i - m-)/g)
+  //                  = a+_i (P+ + l+_i Q+) - a-_i (P- - l-_i Q-)
+  const float ig = a.inv_gamma;
+  const float qxp = we * ibxp * ig, pxp = we * ibxp * (1.f - mxp * ig);
+  const float qxm = we * ibxm * ig, pxm = we * ibxm * (1.f + mxm * ig);
+  const float qyp = we * ibyp * ig, pyp = we * ibyp * (1.f - myp * ig);
+  const float qym = we * ibym * ig, pym = we * ibym * (1.f + mym * ig);
+#pragma unroll
+  for (int s = 0; s < S; s++) {
+    if ((vm & (1u << s)) && cell[s] >= 0) {  // cell < 0: foreign pin (another rank owns it)
+      const float gx = axp[s] * fmaf(lxp[s], qxp, pxp) - axm[s] * fmaf(-lxm[s], qxm, pxm);
+      const float gy = ayp[s] * fmaf(lyp[s], qyp, pyp) - aym[s] * fmaf(-lym[s], qym, pym);
+      const int wi = cell[s] - gc.ch.win_lo;
+      if ((unsigned)wi < (unsigned)gc.ch.win_n) {
+        atomicAdd(gc.s_g + 2 * wi, gx);
+        atomicAdd(gc.s_g + 2 * wi + 1, gy);
+      } else {
+        red_v2(a.g2 + cell[s], gx, gy);
+      }
+    }
+  }
+}
+
 // MODE 0: WA + gradient; 1: WA + gradient + HPWL; 2: HPWL only.
 template <int MODE>
-__global__ void __launch_bounds__(kWaThreads, 2) k_wa_chunks(WaArgs a) {
+__global__ void __launch_bounds__(kWaThreads, 3) k_wa_chunks(WaArgs a) {
   constexpr bool kGrad = MODE != 2;
   constexpr bool kHpwl = MODE != 0;
   __shared__ float2 s_pos[kWaWindow];
   __shared__ float s_g[kGrad ? 2 * kWaWindow : 1];
+  __shared__ int s_next;
 
   const Chunk ch = a.chunks[blockIdx.x];
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
@@ -154,157 +339,28 @@ __global__ void __launch_bounds__(kWaThreads, 2) k_wa_chunks(WaArgs a) {
       s_g[2 * i + 1] = 0.f;
     }
   }
+  if (tid == 0) s_next = ch.wg_begin + kWaThreads / 32;
   __syncthreads();
 
   double wl_acc = 0.0;
   unsigned long long L[kHpwlLimbs + 1];
 #pragma unroll
   for (int k = 0; k <= kHpwlLimbs; k++) L[k] = 0ull;
-  const unsigned lt_mask = (1u << lane) - 1u;
+  const GroupCtx gc{ch, s_pos, s_g, lane, (1u << lane) - 1u};
 
-  for (int wgi = ch.wg_begin + warp; wgi < ch.wg_end; wgi += kWaThreads / 32) {
+  // warp groups are handed out dynamically inside the CTA (self-balancing)
+  int wgi = ch.wg_begin + warp;
+  while (wgi < ch.wg_end) {
     const WarpGroup wg = a.wgs[wgi];
-    const int glog = wg.g_log2, G = 1 << glog, nslots = wg.slots;
-    const int gi = lane >> glog, j = lane & (G - 1);
-    int d = 0, counted = 0;
-    float we = 1.f;
-    if (gi < wg.nnets) {
-      int raw = __ldg(a.net_deg + wg.net_base + gi);
-      d = raw & 0x7fffffff;
-      counted = (raw >> 31) & 1;
-      if (a.has_w) we = __ldg(a.net_w + wg.net_base + gi);
+    switch (wg.slots) {
+      case 1: wa_group<MODE, 1>(a, wg, gc, wl_acc, L); break;
+      case 2: wa_group<MODE, 2>(a, wg, gc, wl_acc, L); break;
+      case 3: wa_group<MODE, 3>(a, wg, gc, wl_acc, L); break;
+      default: wa_group<MODE, 4>(a, wg, gc, wl_acc, L); break;
     }
-    // ---- load pins into registers (slot-major compressed layout, coalesced) ----
-    int cell[kWaPpl];
-    float hx[kWaPpl], lx[kWaPpl], hy[kWaPpl], ly[kWaPpl];
-    unsigned vmask = 0;
-    int slot_base = wg.pin_base;
-#pragma unroll
-    for (int s = 0; s < kWaPpl; s++) {
-      cell[s] = 0;
-      hx[s] = lx[s] = hy[s] = ly[s] = 0.f;
-      if (s < nslots) {
-        const bool valid = s * G + j < d;
-        const unsigned m = __ballot_sync(0xffffffffu, valid);
-        if (valid) {
-          const int p = slot_base + __popc(m & lt_mask);
-          const int raw = __ldg(a.pin_cell + p);
-          const float dx = __ldg(a.pin_dx + p), dy = __ldg(a.pin_dy + p);
-          const int c = raw & 0x7fffffff;
-          const int wi = c - ch.win_lo;
-          float xc, yc;
-          if ((unsigned)wi < (unsigned)ch.win_n) {
-            const float2 q = s_pos[wi];
-            xc = q.x;
-            yc = q.y;
-          } else {
-            xc = __ldg(a.x + c);
-            yc = __ldg(a.y + c);
-          }
-          two_sum(xc, dx, hx[s], lx[s]);
-          two_sum(yc, dy, hy[s], ly[s]);
-          cell[s] = raw;
-          vmask |= 1u << s;
-        }
-        slot_base += __popc(m);
-      }
-    }
-    // ---- per-net extremes x_e^+-, y_e^+- (Table I), exact as (hi, lo) pairs ----
-    float Xh = -INFINITY, Xl = 0.f, xh_ = INFINITY, xl_ = 0.f;
-    float Yh = -INFINITY, Yl = 0.f, yh_ = INFINITY, yl_ = 0.f;
-#pragma unroll
-    for (int s = 0; s < kWaPpl; s++) {
-      if (vmask & (1u << s)) {
-        if (pair_gt(hx[s], lx[s], Xh, Xl)) { Xh = hx[s]; Xl = lx[s]; }
-        if (pair_gt(xh_, xl_, hx[s], lx[s])) { xh_ = hx[s]; xl_ = lx[s]; }
-        if (pair_gt(hy[s], ly[s], Yh, Yl)) { Yh = hy[s]; Yl = ly[s]; }
-        if (pair_gt(yh_, yl_, hy[s], ly[s])) { yh_ = hy[s]; yl_ = ly[s]; }
-      }
-    }
-    for (int o = 1; o < G; o <<= 1) {
-      float h, l;
-      h = __shfl_xor_sync(0xffffffffu, Xh, o); l = __shfl_xor_sync(0xffffffffu, Xl, o);
-      if (pair_gt(h, l, Xh, Xl)) { Xh = h; Xl = l; }
-      h = __shfl_xor_sync(0xffffffffu, xh_, o); l = __shfl_xor_sync(0xffffffffu, xl_, o);
-      if (pair_gt(xh_, xl_, h, l)) { xh_ = h; xl_ = l; }
-      h = __shfl_xor_sync(0xffffffffu, Yh, o); l = __shfl_xor_sync(0xffffffffu, Yl, o);
-      if (pair_gt(h, l, Yh, Yl)) { Yh = h; Yl = l; }
-      h = __shfl_xor_sync(0xffffffffu, yh_, o); l = __shfl_xor_sync(0xffffffffu, yl_, o);
-      if (pair_gt(yh_, yl_, h, l)) { yh_ = h; yl_ = l; }
-    }
-    const bool leader = (j == 0) && d >= 2;
-    if (kHpwl && leader && counted) {
-      // px = fl64(x + dx) exactly as the oracle forms it: (double)hi + (double)lo rounds the
-      // exact real x + dx once.
-      const double xp = __dadd_rn((double)Xh, (double)Xl), xm = __dadd_rn((double)xh_, (double)xl_);
-      const double yp = __dadd_rn((double)Yh, (double)Yl), ym = __dadd_rn((double)yh_, (double)yl_);
-      limbs_add(L, __dadd_rn(__dsub_rn(xp, xm), __dsub_rn(yp, ym)));
-    }
-    if (!kGrad) continue;
-    // ---- shifted exponentials a^+- and sums b^+-, c~^+- (Table I) ----
-    float ax_p[kWaPpl], ax_m[kWaPpl], ay_p[kWaPpl], ay_m[kWaPpl];
-    float bxp = 0.f, bxm = 0.f, cxp = 0.f, cxm = 0.f, byp = 0.f, bym = 0.f, cyp = 0.f, cym = 0.f;
-#pragma unroll
-    for (int s = 0; s < kWaPpl; s++) {
-      ax_p[s] = ax_m[s] = ay_p[s] = ay_m[s] = 0.f;
-      if (vmask & (1u << s)) {
-        const float lxp = __fadd_rn(__fsub_rn(hx[s], Xh), __fsub_rn(lx[s], Xl));   // <= 0
-        const float lxm = __fadd_rn(__fsub_rn(hx[s], xh_), __fsub_rn(lx[s], xl_)); // >= 0
-        const float lyp = __fadd_rn(__fsub_rn(hy[s], Yh), __fsub_rn(ly[s], Yl));
-        const float lym = __fadd_rn(__fsub_rn(hy[s], yh_), __fsub_rn(ly[s], yl_));
-        ax_p[s] = ex2(lxp * a.k2);
-        ax_m[s] = ex2(-lxm * a.k2);
-        ay_p[s] = ex2(lyp * a.k2);
-        ay_m[s] = ex2(-lym * a.k2);
-        bxp += ax_p[s]; cxp += lxp * ax_p[s];
-        bxm += ax_m[s]; cxm += lxm * ax_m[s];
-        byp += ay_p[s]; cyp += lyp * ay_p[s];
-        bym += ay_m[s]; cym += lym * ay_m[s];
-      }
-    }
-    for (int o = 1; o < G; o <<= 1) {
-      bxp += __shfl_xor_sync(0xffffffffu, bxp, o);
-      cxp += __shfl_xor_sync(0xffffffffu, cxp, o);
-      bxm += __shfl_xor_sync(0xffffffffu, bxm, o);
-      cxm += __shfl_xor_sync(0xffffffffu, cxm, o);
-      byp += __shfl_xor_sync(0xffffffffu, byp, o);
-      cyp += __shfl_xor_sync(0xffffffffu, cyp, o);
-      bym += __shfl_xor_sync(0xffffffffu, bym, o);
-      cym += __shfl_xor_sync(0xffffffffu, cym, o);
-    }
-    if (d < 2) continue;  // lanes without a net (d = 0); degree-1 nets are dropped at create
-    const float ibxp = 1.f / bxp, ibxm = 1.f / bxm, ibyp = 1.f / byp, ibym = 1.f / bym;
-    const float mxp = cxp * ibxp, mxm = cxm * ibxm, myp = cyp * ibyp, mym = cym * ibym;
-    if (leader && counted) {
-      // WL_e = c+/b+ - c-/b- = (x+ - x-) + c~+/b+ - c~-/b-   (eq 3 in shifted coordinates)
-      const float spanx = __fadd_rn(__fsub_rn(Xh, xh_), __fsub_rn(Xl, xl_));
-      const float spany = __fadd_rn(__fsub_rn(Yh, yh_), __fsub_rn(Yl, yl_));
-      const float wle = (spanx + mxp - mxm) + (spany + myp - mym);
-      wl_acc += (double)(we * wle);
-    }
-    // eq (6): dWL/dx_i = a+_i/b+ (1 + (x_i - c+/b+)/g) - a-_i/b- (1 - (x_i - c-/b-)/g)
-#pragma unroll
-    for (int s = 0; s < kWaPpl; s++) {
-      if (vmask & (1u << s)) {
-        const int raw = cell[s];
-        if (raw < 0) continue;  // foreign pin (distributed): another rank owns the cell
-        const float lxp = __fadd_rn(__fsub_rn(hx[s], Xh), __fsub_rn(lx[s], Xl));
-        const float lxm = __fadd_rn(__fsub_rn(hx[s], xh_), __fsub_rn(lx[s], xl_));
-        const float lyp = __fadd_rn(__fsub_rn(hy[s], Yh), __fsub_rn(ly[s], Yl));
-        const float lym = __fadd_rn(__fsub_rn(hy[s], yh_), __fsub_rn(ly[s], yl_));
-        const float gx = we * (ax_p[s] * ibxp * (1.f + (lxp - mxp) * a.inv_gamma) -
-                               ax_m[s] * ibxm * (1.f - (lxm - mxm) * a.inv_gamma));
-        const float gy = we * (ay_p[s] * ibyp * (1.f + (lyp - myp) * a.inv_gamma) -
-                               ay_m[s] * ibym * (1.f - (lym - mym) * a.inv_gamma));
-        const int wi = raw - ch.win_lo;
-        if ((unsigned)wi < (unsigned)ch.win_n) {
-          atomicAdd(&s_g[2 * wi], gx);
-          atomicAdd(&s_g[2 * wi + 1], gy);
-        } else {
-          red_v2(a.g2 + raw, gx, gy);
-        }
-      }
-    }
+    int nx = 0;
+    if (lane == 0) nx = atomicAdd(&s_next, 1);
+    wgi = __shfl_sync(0xffffffffu, nx, 0);
   }
   __syncthreads();
   if (kGrad) {

@@ -27,8 +27,8 @@ namespace {
 constexpr int kRowThreads = 256;
 constexpr int kColThreads = 256;
 // columns per CTA in the column kernels (even: pairs share a complex FFT); sized so the
-// shared-memory slab fits: 8 up to 1024 rows, 4 at 2048, 2 at 4096
-__host__ __device__ inline int col_slab(int mx) { return mx <= 1024 ? 8 : (mx <= 2048 ? 4 : 2); }
+// shared-memory slab fits and the grid has >= 256 CTAs at 1024 columns
+__host__ __device__ inline int col_slab(int mx) { return mx <= 2048 ? 4 : 2; }
 
 __device__ __forceinline__ float2 cmul(float2 a, float2 b) {
   return make_float2(a.x * b.x - a.y * b.y, a.x * b.y + a.y * b.x);
@@ -37,19 +37,49 @@ __device__ __forceinline__ int brev(int n, int log2n) { return (int)(__brev((uns
 // Makhoul reordering (Alg 3 lines 3-8): v[n] = x[2n], v[N-1-n] = x[2n+1]; position of x[t] in v
 __device__ __forceinline__ int mk_pos(int t, int n) { return (t & 1) ? n - ((t + 1) >> 1) : (t >> 1); }
 
-// In-place radix-2 DIT FFT of nseq sequences of length n = 2^log2n stored back to back in
-// buf, input already in bit-reversed order.  tw[k] = exp(-2 pi i k / n), k < n/2.
-// inverse = true uses conjugate twiddles (unnormalised inverse DFT).
+// In-place DIT FFT of nseq sequences of length n = 2^log2n stored back to back in buf, input
+// already in bit-reversed order.  tw[k] = exp(-2 pi i k / n), k < n/2.  inverse = true uses
+// conjugate twiddles (unnormalised inverse DFT).  Two radix-2 levels are fused per shared-
+// memory round trip (a radix-4 step on {i, i+h, i+2h, i+3h}), so a 1024-point transform takes
+// 5 barriers instead of 10.
 __device__ void fft_block(float2 *buf, int n, int log2n, int nseq, const float2 *__restrict__ tw,
                           bool inverse) {
-  const int half_n = n >> 1, total = nseq * half_n;
-  for (int s = 1; s <= log2n; s++) {
-    const int half = 1 << (s - 1), len = half << 1, tstride = n >> s;
+  const int quarter_n = n >> 2;
+  const int total4 = nseq * quarter_n;
+  int s = 1;
+  for (; s + 1 <= log2n; s += 2) {
+    const int h = 1 << (s - 1), lh = s - 1;
+    const int st1 = n >> s, st2 = n >> (s + 1);   // twiddle strides of W_{2h} and W_{4h}
+    for (int q = threadIdx.x; q < total4; q += blockDim.x) {
+      const int seq = q / quarter_n, r = q - seq * quarter_n;
+      const int blk = r >> lh, k = r & (h - 1);
+      const int base = seq * n + (blk << (lh + 2)) + k;
+      float2 w1 = __ldg(tw + k * st1), w2 = __ldg(tw + k * st2);
+      if (inverse) {
+        w1.y = -w1.y;
+        w2.y = -w2.y;
+      }
+      // W_{4h}^{k+h} = W_{4h}^k * (-i) forward, (+i) inverse
+      const float2 w3 = inverse ? make_float2(-w2.y, w2.x) : make_float2(w2.y, -w2.x);
+      const float2 a0 = buf[base], a1 = buf[base + h], a2 = buf[base + 2 * h], a3 = buf[base + 3 * h];
+      const float2 t1 = cmul(w1, a1), t3 = cmul(w1, a3);
+      const float2 b0 = make_float2(a0.x + t1.x, a0.y + t1.y), b1 = make_float2(a0.x - t1.x, a0.y - t1.y);
+      const float2 b2 = make_float2(a2.x + t3.x, a2.y + t3.y), b3 = make_float2(a2.x - t3.x, a2.y - t3.y);
+      const float2 u2 = cmul(w2, b2), u3 = cmul(w3, b3);
+      buf[base] = make_float2(b0.x + u2.x, b0.y + u2.y);
+      buf[base + 2 * h] = make_float2(b0.x - u2.x, b0.y - u2.y);
+      buf[base + h] = make_float2(b1.x + u3.x, b1.y + u3.y);
+      buf[base + 3 * h] = make_float2(b1.x - u3.x, b1.y - u3.y);
+    }
+    __syncthreads();
+  }
+  if (s == log2n) {  // odd log2n: one last radix-2 level
+    const int half = 1 << (s - 1), half_n = n >> 1, total = nseq * half_n;
     for (int b = threadIdx.x; b < total; b += blockDim.x) {
-      const int seq = b >> (log2n - 1), r = b & (half_n - 1);
-      const int grp = r >> (s - 1), k = r & (half - 1);
-      const int i = seq * n + grp * len + k, jx = i + half;
-      float2 w = __ldg(tw + k * tstride);
+      const int seq = b / half_n, r = b - seq * half_n;
+      const int k = r;  // one group: grp = 0, len = n
+      const int i = seq * n + k, jx = i + half;
+      float2 w = __ldg(tw + k);
       if (inverse) w.y = -w.y;
       const float2 u = buf[i], v = cmul(w, buf[jx]);
       buf[i] = make_float2(u.x + v.x, u.y + v.y);
@@ -263,26 +293,28 @@ __global__ void __launch_bounds__(kColThreads) k_col_fields(ColFieldArgs a) {
     }
   }
   __syncthreads();  // abuf complete; zbuf free
-  // inverse pre-processing: per column, p = reversed (a k_u / k^2) (IDXST), q = a k_v / k^2 (IDCT)
+  // spectral scaling (eqs 9c/9d): A_X = a k_u / k^2 (in place of a), A_Y = a k_v / k^2 (to the
+  // real scratch behind abuf); a_00 / k^2 := 0
+  float *ybuf = abuf + kColSlab * mx;
   for (int idx = threadIdx.x; idx < mx * kColSlab; idx += kColThreads) {
-    const int col = idx / mx, k = idx % mx;
+    const int col = idx / mx, u = idx - col * mx;
     const int v = c0 + col;
-    const float *ac = abuf + col * mx;
-    const float ky = __ldg(a.ky + v), ky2 = ky * ky;
-    // A_X[u] = a[u] k_u / k^2, A_Y[u] = a[u] k_v / k^2, zero at (0,0)
-    auto AX = [&](int u) -> float {
-      const float kx = __ldg(a.kx + u), k2 = kx * kx + ky2;
-      return (u == 0 && v == 0) ? 0.f : ac[u] * kx / k2;
-    };
-    auto AY = [&](int u) -> float {
-      const float kx = __ldg(a.kx + u), k2 = kx * kx + ky2;
-      return (u == 0 && v == 0) ? 0.f : ac[u] * ky / k2;
-    };
-    // p (IDXST input reversed): p_k = AX[N-k] (k >= 1), p_0 = 0;  p_{N-k} = AX[k] (k >= 1)
-    const float pk = k ? AX(mx - k) : 0.f;
-    const float pnk = k ? AX(k) : 0.f;
-    const float qk = AY(k);
-    const float qnk = k ? AY(mx - k) : 0.f;
+    const float kx = __ldg(a.kx + u), ky = __ldg(a.ky + v);
+    const float k2 = kx * kx + ky * ky;
+    const float ik2 = (u == 0 && v == 0) ? 0.f : 1.f / k2;
+    const float av = abuf[idx];
+    abuf[idx] = av * kx * ik2;
+    ybuf[idx] = av * ky * ik2;
+  }
+  __syncthreads();
+  // inverse pre-processing: per column, p = reversed A_X (IDXST via eq 8e), q = A_Y (IDCT)
+  for (int idx = threadIdx.x; idx < mx * kColSlab; idx += kColThreads) {
+    const int col = idx / mx, k = idx - col * mx;
+    const float *ax = abuf + col * mx, *ay = ybuf + col * mx;
+    const float pk = k ? ax[mx - k] : 0.f;
+    const float pnk = k ? ax[k] : 0.f;
+    const float qk = ay[k];
+    const float qnk = k ? ay[mx - k] : 0.f;
     zbuf[col * mx + brev(k, log2mx)] = inv_pre(pk, qk, pnk, qnk, __ldg(a.ph_x + k));
   }
   __syncthreads();
@@ -326,7 +358,7 @@ __global__ void k_split_xi(const float2 *xi, float *xx, float *xy, size_t n) {
 
 size_t row_smem(int n) { return (size_t)n * sizeof(float2) + 2 * (size_t)n * sizeof(float); }
 size_t col_generic_smem(int mx) { return (size_t)(col_slab(mx) / 2) * mx * sizeof(float2) + (size_t)col_slab(mx) * mx * sizeof(float); }
-size_t col_fields_smem(int mx) { return (size_t)col_slab(mx) * mx * sizeof(float2) + (size_t)col_slab(mx) * mx * sizeof(float); }
+size_t col_fields_smem(int mx) { return (size_t)col_slab(mx) * mx * sizeof(float2) + 2 * (size_t)col_slab(mx) * mx * sizeof(float); }
 
 void row_inv(const Ctx &c, const float *inA, long long stepA, int opA, const float *inB, long long stepB,
              int opB, float *outA, long long ostepA, float *outB, long long ostepB, float2 *outI,

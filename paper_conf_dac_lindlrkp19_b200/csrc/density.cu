@@ -51,19 +51,21 @@ struct Foot {
   bool large, empty;
 };
 
-// Stretched, clipped footprint of own cell i (readings A10, A11).
-__device__ __forceinline__ Foot footprint(const DenArgs &a, int i) {
+// Stretched, clipped footprint of a cell (readings A10, A11) from its loaded values.
+__device__ __forceinline__ Foot footprint_v(const DenArgs &a, float xf, float yf, float wf, float hf) {
   Foot f;
-  const double x = __ldg(a.x + a.cell_begin + i), y = __ldg(a.y + a.cell_begin + i);
-  const double w = __ldg(a.w + i), h = __ldg(a.h + i);
+  const double x = xf, y = yf, w = wf, h = hf;
   double ws = w, hs = h;
+  float wsf = wf, hsf = hf;
   if (a.stretch) {
     ws = fmax(w, a.sx);
     hs = fmax(h, a.sy);
+    wsf = fmaxf(wf, (float)a.sx);
+    hsf = fmaxf(hf, (float)a.sy);
   }
   f.large = (w > 2.0 * a.bx) || (h > 2.0 * a.by);
-  const double wh = ws * hs;
-  f.r = (wh > 0.0) ? (float)((w * h) / wh) : 0.f;
+  // charge ratio r = w h / (w' h') in fp32 (only its fp32 rounding is stored)
+  f.r = (wsf * hsf > 0.f) ? __fdiv_rn(wf * hf, wsf * hsf) : 0.f;
   const double cx = x + 0.5 * w, cy = y + 0.5 * h;
   f.lx = fmax(cx - 0.5 * ws, a.xl);
   f.hx = fmin(cx + 0.5 * ws, a.xh);
@@ -71,6 +73,41 @@ __device__ __forceinline__ Foot footprint(const DenArgs &a, int i) {
   f.hy = fmin(cy + 0.5 * hs, a.yh);
   f.empty = !(f.hx > f.lx && f.hy > f.ly && f.r > 0.f);
   return f;
+}
+
+__device__ __forceinline__ Foot footprint(const DenArgs &a, int i) {
+  return footprint_v(a, __ldg(a.x + a.cell_begin + i), __ldg(a.y + a.cell_begin + i), __ldg(a.w + i), __ldg(a.h + i));
+}
+
+// Loads x, y, w, h of own cells [i0, i0 + 8) (i0 a multiple of 8) with 16-byte vector loads
+// when the global index is aligned; out-of-range cells get w = h = 0 (empty).
+struct Cells8 { float x[8], y[8], w[8], h[8]; };
+
+__device__ __forceinline__ void load_cells8(const DenArgs &a, int i0, Cells8 &c) {
+  const int g0 = a.cell_begin + i0;
+  if (i0 + 8 <= a.n_own && (g0 & 3) == 0) {
+#pragma unroll
+    for (int v = 0; v < 2; v++) {
+      const float4 X = __ldg(reinterpret_cast<const float4 *>(a.x + g0) + v);
+      const float4 Y = __ldg(reinterpret_cast<const float4 *>(a.y + g0) + v);
+      const float4 W = __ldg(reinterpret_cast<const float4 *>(a.w + i0) + v);
+      const float4 H = __ldg(reinterpret_cast<const float4 *>(a.h + i0) + v);
+      c.x[4 * v] = X.x; c.x[4 * v + 1] = X.y; c.x[4 * v + 2] = X.z; c.x[4 * v + 3] = X.w;
+      c.y[4 * v] = Y.x; c.y[4 * v + 1] = Y.y; c.y[4 * v + 2] = Y.z; c.y[4 * v + 3] = Y.w;
+      c.w[4 * v] = W.x; c.w[4 * v + 1] = W.y; c.w[4 * v + 2] = W.z; c.w[4 * v + 3] = W.w;
+      c.h[4 * v] = H.x; c.h[4 * v + 1] = H.y; c.h[4 * v + 2] = H.z; c.h[4 * v + 3] = H.w;
+    }
+  } else {
+#pragma unroll
+    for (int k = 0; k < 8; k++) {
+      const int i = i0 + k;
+      const bool ok = i < a.n_own;
+      c.x[k] = ok ? __ldg(a.x + a.cell_begin + i) : 0.f;
+      c.y[k] = ok ? __ldg(a.y + a.cell_begin + i) : 0.f;
+      c.w[k] = ok ? __ldg(a.w + i) : 0.f;
+      c.h[k] = ok ? __ldg(a.h + i) : 0.f;
+    }
+  }
 }
 
 __device__ __forceinline__ int small_tile(const DenArgs &a, const Foot &f, int &ox, int &oy) {
@@ -83,19 +120,23 @@ __device__ __forceinline__ int small_tile(const DenArgs &a, const Foot &f, int &
   return tx * a.tiles_y + ty;
 }
 
-// D1
+// D1: 8 cells per thread, all loads issued up front
 __global__ void __launch_bounds__(kCountThreads) k_count(DenArgs a) {
   extern __shared__ int s_hist[];
   for (int t = threadIdx.x; t < a.ntiles; t += kCountThreads) s_hist[t] = 0;
   __syncthreads();
-  const int base = blockIdx.x * kCountCells;
-  for (int k = 0; k < kCountCells / kCountThreads; k++) {
-    const int i = base + k * kCountThreads + threadIdx.x;
-    if (i >= a.n_own) break;
-    const Foot f = footprint(a, i);
-    if (f.empty || f.large) continue;
-    int ox, oy;
-    atomicAdd(&s_hist[small_tile(a, f, ox, oy)], 1);
+  const int i0 = (blockIdx.x * kCountThreads + threadIdx.x) * 8;
+  if (i0 < a.n_own) {
+    Cells8 c;
+    load_cells8(a, i0, c);
+#pragma unroll
+    for (int k = 0; k < 8; k++) {
+      if (i0 + k >= a.n_own) break;
+      const Foot f = footprint_v(a, c.x[k], c.y[k], c.w[k], c.h[k]);
+      if (f.empty || f.large) continue;
+      int ox, oy;
+      atomicAdd(&s_hist[small_tile(a, f, ox, oy)], 1);
+    }
   }
   __syncthreads();
   for (int t = threadIdx.x; t < a.ntiles; t += kCountThreads)
@@ -158,30 +199,43 @@ __global__ void __launch_bounds__(1024) k_scan(DenArgs a) {
   }
 }
 
-// D3
+// D3: same 8-cells-per-thread traversal as D1; records stay in registers while the CTA
+// reserves its ranges in the tile cursors.
 __global__ void __launch_bounds__(kCountThreads) k_place(DenArgs a) {
   extern __shared__ int s_hist[];
-  constexpr int K = kCountCells / kCountThreads;
   for (int t = threadIdx.x; t < a.ntiles; t += kCountThreads) s_hist[t] = 0;
   __syncthreads();
-  const int base = blockIdx.x * kCountCells;
-  int tl[K], rk[K];
+  const int i0 = (blockIdx.x * kCountThreads + threadIdx.x) * 8;
+  int tl[8], rk[8], ij[8];
+  float4 rec[8];
+  float rr[8];
 #pragma unroll
-  for (int k = 0; k < K; k++) {
-    tl[k] = -1;
-    rk[k] = 0;
-    const int i = base + k * kCountThreads + threadIdx.x;
-    if (i < a.n_own) {
-      const Foot f = footprint(a, i);
-      if (!f.large) {
-        if (f.empty) {
-          a.force[i] = make_float2(0.f, 0.f);
-        } else {
-          int ox, oy;
-          tl[k] = small_tile(a, f, ox, oy);
-          rk[k] = atomicAdd(&s_hist[tl[k]], 1);
-        }
+  for (int k = 0; k < 8; k++) tl[k] = -1;
+  if (i0 < a.n_own) {
+    Cells8 c;
+    load_cells8(a, i0, c);
+#pragma unroll
+    for (int k = 0; k < 8; k++) {
+      const int i = i0 + k;
+      if (i >= a.n_own) break;
+      const Foot f = footprint_v(a, c.x[k], c.y[k], c.w[k], c.h[k]);
+      if (f.large) continue;
+      if (f.empty) {
+        a.force[i] = make_float2(0.f, 0.f);
+        continue;
       }
+      int ox, oy;
+      tl[k] = small_tile(a, f, ox, oy);
+      rk[k] = atomicAdd(&s_hist[tl[k]], 1);
+      // bin-local fractions (|v| < 3): fp32 keeps ~2e-7 bin absolute precision, which the force
+      // gather needs where large opposite bin fields cancel (the 'initial' placement)
+      const double ux0 = (f.lx - a.xl) * a.ibx, uy0 = (f.ly - a.yl) * a.iby;
+      const int bi = min(max((int)floor(ux0), 0), a.mx - 1);
+      const int bj = min(max((int)floor(uy0), 0), a.my - 1);
+      rec[k] = make_float4((float)(ux0 - bi), (float)(uy0 - bj), (float)((f.hx - a.xl) * a.ibx - bi),
+                           (float)((f.hy - a.yl) * a.iby - bj));
+      rr[k] = f.r;
+      ij[k] = (bi - ox) | ((bj - oy) << 16);
     }
   }
   __syncthreads();
@@ -191,36 +245,27 @@ __global__ void __launch_bounds__(kCountThreads) k_place(DenArgs a) {
   }
   __syncthreads();
 #pragma unroll
-  for (int k = 0; k < K; k++) {
+  for (int k = 0; k < 8; k++) {
     if (tl[k] < 0) continue;
-    const int i = base + k * kCountThreads + threadIdx.x;
-    const Foot f = footprint(a, i);
-    int ox, oy;
-    small_tile(a, f, ox, oy);
     const int pos = s_hist[tl[k]] + rk[k];
-    // bin-local fractions (|v| < 3): fp32 keeps ~2e-7 bin absolute precision, which the force
-    // gather needs where large opposite bin fields cancel (the 'initial' placement)
-    const double ux0 = (f.lx - a.xl) * a.ibx, uy0 = (f.ly - a.yl) * a.iby;
-    const int i0 = min(max((int)floor(ux0), 0), a.mx - 1);
-    const int j0 = min(max((int)floor(uy0), 0), a.my - 1);
-    a.rec[pos] = make_float4((float)(ux0 - i0), (float)(uy0 - j0), (float)((f.hx - a.xl) * a.ibx - i0),
-                             (float)((f.hy - a.yl) * a.iby - j0));
-    a.rec_rc[pos] = make_int2(__float_as_int(f.r), (i0 - ox) | ((j0 - oy) << 16));
-    a.rec_cell[pos] = i;
+    a.rec[pos] = rec[k];
+    a.rec_rc[pos] = make_int2(__float_as_int(rr[k]), ij[k]);
+    a.rec_cell[pos] = i0 + k;
   }
 }
 
 // D4
 __global__ void __launch_bounds__(256) k_scatter_tiles(DenArgs a) {
-  extern __shared__ float s_t[];
+  extern __shared__ int s_t[];   // int32 fixed point, 2^-kTileScaleLog2 units (native ATOMS.ADD)
   const int sg = blockIdx.x;
   if (sg >= *a.nsegs) return;
   const Segment seg = a.segs[sg];
   const int P = a.tile + kHalo;
   const int tx = seg.tile / a.tiles_y, ty = seg.tile % a.tiles_y;
   const int ox = tx * a.tile, oy = ty * a.tile;
-  for (int k = threadIdx.x; k < P * P; k += blockDim.x) s_t[k] = 0.f;
+  for (int k = threadIdx.x; k < P * P; k += blockDim.x) s_t[k] = 0;
   __syncthreads();
+  const float scale = (float)(1 << kTileScaleLog2);
   for (int p = seg.begin + threadIdx.x; p < seg.end; p += blockDim.x) {
     const float4 q = a.rec[p];
     const int2 rc = a.rec_rc[p];
@@ -236,15 +281,17 @@ __global__ void __launch_bounds__(256) k_scatter_tiles(DenArgs a) {
         const int j = j0 + dj;
         const float ovy = fminf(q.w, (float)(dj + 1)) - fmaxf(q.y, (float)dj);
         if (ovy <= 0.f || j >= P || oy + j >= a.my) break;
-        atomicAdd(&s_t[i * P + j], r * ovx * ovy);
+        atomicAdd(&s_t[i * P + j], __float2int_rn(r * ovx * ovy * scale));
       }
     }
   }
   __syncthreads();
+  const float inv = 1.f / scale;
   for (int k = threadIdx.x; k < P * P; k += blockDim.x) {
-    const float v = s_t[k];
+    const int iv = s_t[k];
+    const float v = iv * inv;
     const int gi = ox + k / P, gj = oy + k % P;
-    if (v != 0.f && gi < a.mx && gj < a.my)
+    if (iv != 0 && gi < a.mx && gj < a.my)
       asm volatile("red.global.add.f32 [%0], %1;" ::"l"(a.rho + (size_t)gi * a.my + gj), "f"(v) : "memory");
   }
 }
@@ -398,7 +445,7 @@ void launch_density_map(const Ctx &c, const float *x, const float *y, cudaStream
   const DenArgs a = make_args(c, x, y);
   const int P = c.tile + kHalo;
   const int ntiles = a.ntiles;
-  const int nblk = (c.n_own + kCountCells - 1) / kCountCells;
+  const int nblk = (c.n_own + kCountThreads * 8 - 1) / (kCountThreads * 8);
   cudaMemsetAsync(c.d_rho, 0, sizeof(float) * (size_t)c.mx * c.my, s);
   if (nblk > 0) {
     k_count<<<nblk, kCountThreads, ntiles * 4, s>>>(a);

@@ -174,10 +174,12 @@ dp_status build_wa(Ctx &c, const dp_netlist *nl, const std::vector<uint8_t> &mas
 
   std::vector<Chunk> chunks;
   std::vector<WarpGroup> wgs;
-  std::vector<int32_t> net_deg, pin_cell;
+  std::vector<int32_t> net_deg, pin_cell, far_cells;
   std::vector<float> net_w, pin_dx, pin_dy;
+  WaCaps caps{4, 4, 4, 4};
+  auto up4 = [](int v) { return (v + 3) & ~3; };
   size_t i = 0;
-  std::vector<int32_t> cells;
+  std::vector<int32_t> cells, far;
   while (i < small.size()) {
     // take nets until the pin budget is reached (at least one net)
     size_t j = i;
@@ -188,26 +190,72 @@ dp_status build_wa(Ctx &c, const dp_netlist *nl, const std::vector<uint8_t> &mas
       pins += d;
       j++;
     }
-    // densest window of kWaWindow consecutive cells
+    // densest window of kWaWindow consecutive cells, start aligned to 4 cells (16 bytes) so
+    // the kernel can stage x / y with bulk async copies
     cells.clear();
     for (size_t q = i; q < j; q++)
       for (int32_t k = nl->net_start[small[q]]; k < nl->net_start[small[q] + 1]; k++) cells.push_back(nl->pin2cell[pin_of(k)]);
     std::sort(cells.begin(), cells.end());
-    const int win_n = std::min<int32_t>(kWaWindow, ncells);
+    const int win_n0 = std::min<int32_t>(kWaWindow, ncells);
     int32_t best_lo = cells[0];
     size_t best = 0, lo = 0;
     for (size_t hi = 0; hi < cells.size(); hi++) {
-      while (cells[hi] - cells[lo] >= win_n) lo++;
+      while (cells[hi] - cells[lo] >= std::max(1, win_n0 - 3)) lo++;
       if (hi - lo + 1 > best) {
         best = hi - lo + 1;
         best_lo = cells[lo];
       }
     }
-    best_lo = std::max(0, std::min(best_lo, ncells - win_n));
+    best_lo = std::max(0, std::min(best_lo, ncells - win_n0)) & ~3;
+    const int win_n = std::min<int32_t>(kWaWindow, ncells - best_lo);
+    // far cells: distinct cells of the chunk outside the window
+    far.clear();
+    for (int32_t cc : cells)
+      if (cc < best_lo || cc >= best_lo + win_n) far.push_back(cc);
+    far.erase(std::unique(far.begin(), far.end()), far.end());   // cells are sorted
+    auto slot_of = [&](int32_t cc) -> int32_t {
+      if (cc >= best_lo && cc < best_lo + win_n) return cc - best_lo;
+      return kWaWindow + (int32_t)(std::lower_bound(far.begin(), far.end(), cc) - far.begin());
+    };
+    auto pad4 = [&]() {
+      while (pin_cell.size() & 3) {
+        pin_cell.push_back(0);
+        pin_dx.push_back(0.f);
+        pin_dy.push_back(0.f);
+      }
+      while (net_deg.size() & 3) {
+        net_deg.push_back(0);
+        net_w.push_back(0.f);
+      }
+    };
+    pad4();
     Chunk ch;
     ch.wg_begin = (int32_t)wgs.size();
     ch.win_lo = best_lo;
     ch.win_n = win_n;
+    ch.pin_begin = (int32_t)pin_cell.size();
+    ch.net_begin = (int32_t)net_deg.size();
+    ch.far_begin = (int32_t)far_cells.size();
+    ch.far_n = (int32_t)far.size();
+    ch.far_pad = up4(ch.far_n);
+    far_cells.insert(far_cells.end(), far.begin(), far.end());
+    while ((int32_t)far_cells.size() < ch.far_begin + ch.far_pad) far_cells.push_back(0);
+    {
+      // int32 fixed-point scale of the gradient slots: |dWL_e/dx_i| <= (2 + d/2) w_e per pin
+      // (max pin: 1 + (d-1)/e; others: <= 1 + 1/e, per side), so a slot's sum is bounded by
+      // the sum of its pins' bounds; pick 2^k with bound * 2^k < 2^30.
+      std::vector<double> bound(kWaWindow + far.size() + 1, 0.0);
+      for (size_t q = i; q < j; q++) {
+        const int32_t e = small[q];
+        const int d = nl->net_start[e + 1] - nl->net_start[e];
+        const double we = nl->net_weight ? (double)nl->net_weight[e] : 1.0;
+        for (int32_t k = nl->net_start[e]; k < nl->net_start[e + 1]; k++)
+          bound[slot_of(nl->pin2cell[pin_of(k)])] += (2.0 + 0.5 * d) * we;
+      }
+      const double bmax = std::max(1e-30, *std::max_element(bound.begin(), bound.end()));
+      int k = (int)std::floor(std::log2(double(1 << 30) / bmax));
+      ch.scale_log2 = std::max(-100, std::min(k, 100));
+    }
     // group nets by lanes-per-net class, largest class first, degree-descending inside
     std::vector<std::vector<int32_t>> cls(6);
     for (size_t q = i; q < j; q++) {
@@ -222,20 +270,22 @@ dp_status build_wa(Ctx &c, const dp_netlist *nl, const std::vector<uint8_t> &mas
       const int per = 32 >> g, G = 1 << g;
       for (size_t q = 0; q < v.size(); q += per) {
         WarpGroup wg;
-        wg.pin_base = (int32_t)pin_cell.size();
-        wg.net_base = (int32_t)net_deg.size();
+        wg.pin_base = (int32_t)pin_cell.size() - ch.pin_begin;
+        wg.net_base = (int32_t)net_deg.size() - ch.net_begin;
         wg.nnets = (int32_t)std::min<size_t>(per, v.size() - q);
         wg.g_log2 = g;
-        wg.pad = 0;
         int dmax = 0;
+        bool pairs = (g == 0);
         for (int n = 0; n < wg.nnets; n++) {
           const int32_t e = v[q + n];
           const int d = nl->net_start[e + 1] - nl->net_start[e];
           dmax = std::max(dmax, d);
+          pairs = pairs && d == 2;
           net_deg.push_back(d | ((mask[e] & 2) ? (int32_t)0x80000000u : 0));
           net_w.push_back(nl->net_weight ? nl->net_weight[e] : 1.f);
         }
         wg.slots = (dmax + G - 1) / G;
+        wg.flags = pairs ? 1 : 0;
         for (int s = 0; s < wg.slots; s++)
           for (int L = 0; L < 32; L++) {
             const int gi = L >> g, jj = L & (G - 1);
@@ -247,14 +297,21 @@ dp_status build_wa(Ctx &c, const dp_netlist *nl, const std::vector<uint8_t> &mas
             const int32_t p = pin_of(nl->net_start[e] + k);
             const int32_t cell = nl->pin2cell[p];
             const bool foreign = cell < c.cell_begin || cell >= c.cell_end;
-            pin_cell.push_back(cell | (foreign ? (int32_t)0x80000000u : 0));
+            pin_cell.push_back(slot_of(cell) | (foreign ? (int32_t)0x80000000u : 0));
             pin_dx.push_back(nl->pin_dx[p]);
             pin_dy.push_back(nl->pin_dy[p]);
           }
         wgs.push_back(wg);
       }
     }
-    ch.wg_end = (int32_t)wgs.size();
+    ch.wg_n = (int32_t)wgs.size() - ch.wg_begin;
+    pad4();
+    ch.pin_n = (int32_t)pin_cell.size() - ch.pin_begin;
+    ch.net_n = (int32_t)net_deg.size() - ch.net_begin;
+    caps.pins = std::max(caps.pins, ch.pin_n);
+    caps.nets = std::max(caps.nets, ch.net_n);
+    caps.groups = std::max(caps.groups, up4(ch.wg_n));
+    caps.far = std::max(caps.far, ch.far_pad);
     chunks.push_back(ch);
     i = j;
   }
@@ -262,6 +319,17 @@ dp_status build_wa(Ctx &c, const dp_netlist *nl, const std::vector<uint8_t> &mas
   c.n_wgroups = (int32_t)wgs.size();
   c.n_wa_nets = (int32_t)net_deg.size();
   c.n_wa_pins = (int32_t)pin_cell.size();
+  {
+    static WaCaps max_caps{4, 4, 4, 4};
+    WaCaps m{std::max(max_caps.pins, caps.pins), std::max(max_caps.nets, caps.nets),
+             std::max(max_caps.groups, caps.groups), std::max(max_caps.far, caps.far)};
+    if (wa_smem_bytes(m) > 227 * 1024) return fail(DP_ERR_UNSUPPORTED, "WA chunk staging exceeds shared memory");
+    if (m.pins != max_caps.pins || m.nets != max_caps.nets || m.groups != max_caps.groups || m.far != max_caps.far) {
+      DP_CUDA(wa_configure(m));
+      max_caps = m;
+    }
+    c.wa_caps = caps;
+  }
   dp_status st;
   if ((st = dev_upload(c, &c.d_chunks, chunks)) != DP_OK) return st;
   if ((st = dev_upload(c, &c.d_wgroups, wgs)) != DP_OK) return st;
@@ -270,6 +338,7 @@ dp_status build_wa(Ctx &c, const dp_netlist *nl, const std::vector<uint8_t> &mas
   if ((st = dev_upload(c, &c.d_pin_cell, pin_cell)) != DP_OK) return st;
   if ((st = dev_upload(c, &c.d_pin_dx, pin_dx)) != DP_OK) return st;
   if ((st = dev_upload(c, &c.d_pin_dy, pin_dy)) != DP_OK) return st;
+  if ((st = dev_upload(c, &c.d_far_cells, far_cells)) != DP_OK) return st;
   // ---- big nets ----
   std::vector<int32_t> bstart{0}, bflags, bcell;
   std::vector<float> bw, bdx, bdy;
@@ -440,7 +509,7 @@ dp_status create(const dp_netlist *nl, const dp_grid *grid, int device, int rank
   if ((st = build_wa(*c, nl, mask)) != DP_OK) return bail(st);
   if ((st = build_density(*c, nl)) != DP_OK) return bail(st);
   c->n_wa_part = c->n_chunks + c->n_big;
-  c->n_en_part = c->my / (c->mx <= 1024 ? 8 : (c->mx <= 2048 ? 4 : 2));
+  c->n_en_part = c->my / (c->mx <= 2048 ? 4 : 2);   // = CTAs of the column-fields kernel
   if ((st = dev_alloc(*c, &c->d_g2, c->num_cells)) != DP_OK) return bail(st);
   if (cudaMemset(c->d_g2, 0, sizeof(float2) * c->num_cells) != cudaSuccess) return bail(fail(DP_ERR_CUDA, "memset"));
   if ((st = dev_alloc(*c, &c->d_part, c->n_wa_part + c->n_en_part + 1)) != DP_OK) return bail(st);

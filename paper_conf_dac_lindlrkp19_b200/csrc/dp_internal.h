@@ -19,30 +19,44 @@ namespace dp {
 constexpr int kWaThreads = 256;       // threads per WA chunk CTA (8 warps)
 constexpr int kWaPpl = 4;             // pin slots per lane (registers)
 constexpr int kWaMaxDeg = 128;        // nets up to this degree go through the chunk kernel (G <= 32)
-constexpr int kWaChunkPins = 4096;    // target pins per chunk
-constexpr int kWaWindow = 2048;       // cells per chunk window held in shared memory
+constexpr int kWaChunkPins = 2048;    // max pins per chunk (staged in shared memory)
+constexpr int kWaWindow = 1024;       // consecutive cells per chunk window held in shared memory
 constexpr int kBigThreads = 128;      // CTA-per-net kernel for nets > kWaMaxDeg
 constexpr int kHpwlLimbs = 9;         // limbs 0..kHpwlLimbs (10) of 32-bit digits, LSB 2^-149 (reading A7)
 
 constexpr int kTile = 32;             // density tile = kTile x kTile bins
 constexpr int kHalo = 2;              // small-cell footprints extend <= 2 bins past their tile
 constexpr int kSegCells = 2048;       // cells per scatter/gather work segment
+constexpr int kTileScaleLog2 = 19;    // tile bins accumulate int32 units of 2^-19 (<= kSegCells x 1 < 2^12)
 constexpr int kCountThreads = 256;
-constexpr int kCountCells = 4096;     // cells per count/place CTA
+constexpr int kCountCells = kCountThreads * 8;  // cells per count/place CTA (8 per thread)
 
-// Per warp-group metadata of the WA chunk layout.
+// Per warp-group metadata of the WA chunk layout (16 bytes, bulk-copied per chunk).
 struct WarpGroup {
-  int32_t pin_base;   // first pin entry of the group (slot-major compressed layout)
-  int32_t net_base;   // first net (index into the reordered net arrays)
+  int32_t pin_base;   // first pin entry of the group, relative to its chunk's pin_begin
+  int32_t net_base;   // first net, relative to its chunk's net_begin
   int32_t nnets;      // nets in the group (<= 32 / g)
   int32_t g_log2 : 8; // log2 of lanes per net
   int32_t slots : 8;  // pin slots per lane (<= kWaPpl)
-  int32_t pad : 16;
+  int32_t flags : 16; // bit 0: all nets of the group have degree 2 (closed-form path)
 };
 
+// One CTA's work in the WA kernel (48 bytes).  Pin records hold a chunk-local position slot:
+// [0, kWaWindow) = window cell win_lo + i, kWaWindow + f = far cell far_cells[far_begin + f];
+// bit 31 marks a foreign pin (distributed: no gradient for that cell on this rank).
 struct Chunk {
-  int32_t wg_begin, wg_end;   // warp groups of this chunk
-  int32_t win_lo, win_n;      // cell window [win_lo, win_lo + win_n)
+  int32_t wg_begin, wg_n;     // warp groups (16-byte records)
+  int32_t pin_begin, pin_n;   // pin records (16-byte aligned, padded to 4)
+  int32_t net_begin, net_n;   // net degrees / weights (16-byte aligned, padded to 4)
+  int32_t far_begin, far_n;   // deduplicated cells outside the window
+  int32_t far_pad;            // far_n padded to 4 (bulk copy size)
+  int32_t win_lo, win_n;      // window [win_lo, win_lo + win_n), win_lo a multiple of 4
+  int32_t scale_log2;         // window / far gradients accumulate int32 units of 2^-scale_log2
+};
+
+// Shared-memory capacities of the WA chunk kernel (maxima over chunks, multiples of 4).
+struct WaCaps {
+  int pins, nets, groups, far;
 };
 
 // Work segment of the density scatter/gather (built on device each evaluation).
@@ -69,11 +83,13 @@ struct Ctx {
 
   // ---- WA layout (device) ----
   int32_t n_chunks = 0, n_wgroups = 0, n_wa_nets = 0, n_wa_pins = 0;
+  WaCaps wa_caps{4, 4, 4, 4};          // per-chunk staging capacities
+  int32_t *d_far_cells = nullptr;      // far-cell lists of all chunks
   Chunk *d_chunks = nullptr;
   WarpGroup *d_wgroups = nullptr;
   int32_t *d_net_deg = nullptr;     // degree | counted<<31 per reordered net
   float *d_net_w = nullptr;         // weights per reordered net (if has_weights)
-  int32_t *d_pin_cell = nullptr;    // cell | foreign<<31 per pin entry
+  int32_t *d_pin_cell = nullptr;    // chunk-local position slot | foreign<<31 per pin entry
   float *d_pin_dx = nullptr, *d_pin_dy = nullptr;
   // big nets (degree > kWaMaxDeg): plain CSR, one CTA per net
   int32_t n_big = 0;
@@ -166,6 +182,8 @@ void launch_finalize_phase(const Ctx &c, int phase, float lambda, bool with_wl, 
                            double *d_hpwl, cudaStream_t s);
 // configuration (shared-memory opt-in), called from dp_create
 cudaError_t dct_configure(int mx, int my);
+cudaError_t wa_configure(const WaCaps &caps);
+int wa_smem_bytes(const WaCaps &caps);
 cudaError_t density_configure(int ntiles, int tile);
 int density_launches(const Ctx &c);
 // NCCL (nccl_dyn.cpp)

@@ -5,17 +5,25 @@
 // Alg 2 so no per-net intermediate touches global memory; HPWL.
 //
 // B200 design, differences from the paper's Alg 2:
-//  * nets are locality-sorted into chunks at dp_create; a CTA owns one chunk and keeps the
-//    positions and gradients of the chunk's cell window in shared memory, so the pin->cell
-//    gradient reduction is a shared-memory atomic instead of a global one (random L2 reds
-//    run at ~0.2 Gop/ms on B200 — tools/microbench), flushed once with coalesced red.v4;
-//  * nets are processed by groups of G = 1..32 lanes (by degree), each lane holding up to 8
-//    pins in registers: a^+- are computed once and kept (Alg 2 recomputes them);
-//  * x and y are fused in one pass (the paper uses two streams);
-//  * the shift is done in net-local coordinates with an exact TwoSum of (x_cell + dx), so
-//    fp32 keeps full relative precision even at |x| ~ 1e6 (reading A2);
-//  * HPWL uses the exact per-net extremes and a 2^-149 fixed-point int64 limb sum, which
-//    makes the total correctly rounded and order independent (reading A7).
+//  * nets are locality-sorted into chunks at dp_create (~2048 pins).  A CTA owns one chunk and
+//    stages it in shared memory with bulk async copies (cp.async.bulk + mbarrier): pin records,
+//    net degrees, warp-group metadata, the chunk's window of 1024 consecutive cells and a
+//    deduplicated list of its "far" cells.  Every pin refers to a chunk-local position slot
+//    [window | far | trash], so the inner loop touches shared memory only and has no
+//    data-dependent branches;
+//  * pin -> cell gradients accumulate in shared memory as int32 fixed point (sm_100a has a
+//    native 32-bit integer ATOMS.ADD; shared float atomics are CAS loops), with a per-chunk
+//    scale chosen at create from a bound on the cell sums, then flush once per cell with
+//    coalesced red.global.add.v4.f32 (window) / v2 (far cells);
+//  * nets are processed by groups of G = 1..32 lanes (by degree), each lane holding up to 4
+//    pins in registers (slot count templated): a^+- are computed once and kept (Alg 2
+//    recomputes them); x and y fused (the paper uses two streams);
+//  * 2-pin nets (55% of nets) use the closed form of eqs (3)/(6) for two pins;
+//  * numerics: the shift reference is the rounded extreme P = max fl(x + dx); for every pin
+//    whose exponential matters, x_cell - P is exact (Sterbenz) and the rounding of P is a
+//    common shift that cancels exactly (reading A2).  Values are carried in log2 units;
+//  * HPWL mode uses exact (TwoSum) pin positions and extremes and a 2^-149 fixed-point int64
+//    limb sum: correctly rounded and order independent (reading A7).
 #include "dp_internal.h"
 
 namespace dp {
@@ -23,14 +31,16 @@ namespace dp {
 namespace {
 
 constexpr float kLog2e = 1.4426950408889634f;
+constexpr float kLn2 = 0.6931471805599453f;
 
 struct WaArgs {
   const Chunk *chunks;
   const WarpGroup *wgs;
   const int32_t *net_deg;
   const float *net_w;
-  const int32_t *pin_cell;
+  const int32_t *pin_slot;
   const float *pin_dx, *pin_dy;
+  const int32_t *far_cells;
   const float *x, *y;
   float2 *g2;
   float gamma, inv_gamma, k2;   // k2 = log2(e) / gamma
@@ -41,6 +51,7 @@ struct WaArgs {
   const int32_t *big_start, *big_flags, *big_cell;
   const float *big_w, *big_dx, *big_dy;
   int part_offset;
+  WaCaps caps;
 };
 
 // Exact sum s + e = a + b (Knuth TwoSum, fp32, no contraction).
@@ -59,6 +70,12 @@ __device__ __forceinline__ bool pair_gt(float h1, float l1, float h2, float l2) 
 __device__ __forceinline__ float ex2(float v) {
   float r;
   asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(r) : "f"(v));
+  return r;
+}
+
+__device__ __forceinline__ float rcp(float v) {
+  float r;
+  asm("rcp.approx.ftz.f32 %0, %1;" : "=f"(r) : "f"(v));
   return r;
 }
 
@@ -137,147 +154,123 @@ __device__ void block_flush_scalars(double wl, unsigned long long (&L)[kHpwlLimb
   }
 }
 
-// Fast2Sum (3 flops): exact when |a| >= |b| (cell coordinate vs pin offset, the usual case);
-// otherwise still accurate to ~ulp of the sum, which is all the WA value/gradient needs.
-__device__ __forceinline__ void fast_sum(float a, float b, float &s, float &e) {
-  s = __fadd_rn(a, b);
-  e = __fadd_rn(__fsub_rn(a, s), b);
-}
-
-// Per-lane running extremes of one axis as (hi, lo) pairs.
+// Per-lane running extremes of one axis as exact (hi, lo) pairs (HPWL mode).
 struct Axis { float Ph, Pl, Mh, Ml; };
 
-template <bool EXACT>
 __device__ __forceinline__ void ext_update(Axis &A, float h, float l) {
-  if (EXACT) {
-    if (pair_gt(h, l, A.Ph, A.Pl)) { A.Ph = h; A.Pl = l; }
-    if (pair_gt(A.Mh, A.Ml, h, l)) { A.Mh = h; A.Ml = l; }
-  } else {  // the shift only needs a pin at (or within an ulp of) the extreme
-    if (h > A.Ph) { A.Ph = h; A.Pl = l; }
-    if (h < A.Mh) { A.Mh = h; A.Ml = l; }
-  }
+  if (pair_gt(h, l, A.Ph, A.Pl)) { A.Ph = h; A.Pl = l; }
+  if (pair_gt(A.Mh, A.Ml, h, l)) { A.Mh = h; A.Ml = l; }
 }
 
-template <bool EXACT>
 __device__ __forceinline__ void ext_shfl(Axis &A, int o) {
   const float ph = __shfl_xor_sync(0xffffffffu, A.Ph, o), pl = __shfl_xor_sync(0xffffffffu, A.Pl, o);
   const float mh = __shfl_xor_sync(0xffffffffu, A.Mh, o), ml = __shfl_xor_sync(0xffffffffu, A.Ml, o);
-  if (EXACT) {
-    if (pair_gt(ph, pl, A.Ph, A.Pl)) { A.Ph = ph; A.Pl = pl; }
-    if (pair_gt(A.Mh, A.Ml, mh, ml)) { A.Mh = mh; A.Ml = ml; }
-  } else {
-    if (ph > A.Ph || (ph == A.Ph && pl > A.Pl)) { A.Ph = ph; A.Pl = pl; }
-    if (mh < A.Mh || (mh == A.Mh && ml < A.Ml)) { A.Mh = mh; A.Ml = ml; }
-  }
+  if (pair_gt(ph, pl, A.Ph, A.Pl)) { A.Ph = ph; A.Pl = pl; }
+  if (pair_gt(A.Mh, A.Ml, mh, ml)) { A.Mh = mh; A.Ml = ml; }
 }
 
+// Shared-memory view of one staged chunk.
 struct GroupCtx {
-  const Chunk &ch;
-  const float2 *s_pos;
-  float *s_g;
+  const int *slot;       // [pins] position slot | foreign << 31
+  const float *dx, *dy;  // [pins]
+  const int *deg;        // [nets] degree | counted << 31
+  const float *w;        // [nets]
+  const float *px, *py;  // [slots] cell positions: window cells, then far cells
+  int *g;                // [2 * slots] int32 fixed-point gradient (x, y interleaved)
+  int trash;             // gradient slot of foreign pins (never flushed)
+  float scale;           // 2^scale_log2
   int lane;
   unsigned lt_mask;
 };
 
-// One warp group: 32/G nets, G lanes per net, S pin slots per lane.
-template <int MODE, int S>
-__device__ __forceinline__ void wa_group(const WaArgs &a, const WarpGroup &wg, const GroupCtx &gc, double &wl_acc,
-                                         unsigned long long (&L)[kHpwlLimbs + 1]) {
-  constexpr bool kGrad = MODE != 2;
-  constexpr bool kHpwl = MODE != 0;
-  const int glog = wg.g_log2, G = 1 << glog;
-  const int gi = gc.lane >> glog, j = gc.lane & (G - 1);
-  int d = 0, counted = 0;
-  float we = 1.f;
-  if (gi < wg.nnets) {
-    const int raw = __ldg(a.net_deg + wg.net_base + gi);
-    d = raw & 0x7fffffff;
-    counted = (raw >> 31) & 1;
-    if (a.has_w) we = __ldg(a.net_w + wg.net_base + gi);
-  }
-  // ---- phase A: pin records of all slots (slot-major compressed layout, coalesced) ----
-  int cell[S];
-  float dxs[S], dys[S];
+__device__ __forceinline__ void grad_add(const GroupCtx &gc, int raw, float gx, float gy) {
+  const int gs = raw < 0 ? gc.trash : raw;
+  atomicAdd(gc.g + 2 * gs, __float2int_rn(gx * gc.scale));
+  atomicAdd(gc.g + 2 * gs + 1, __float2int_rn(gy * gc.scale));
+}
+
+// Pin records of one warp group, slot-major compressed layout (32/G nets, G lanes per net).
+template <int S>
+__device__ __forceinline__ unsigned load_pins(const WarpGroup &wg, const GroupCtx &gc, int G, int j, int d,
+                                              int (&raw)[S], float (&xc)[S], float (&yc)[S], float (&dxs)[S],
+                                              float (&dys)[S]) {
   unsigned vm = 0;
   int base = wg.pin_base;
 #pragma unroll
   for (int s = 0; s < S; s++) {
     const bool valid = s * G + j < d;
     const unsigned m = __ballot_sync(0xffffffffu, valid);
-    cell[s] = 0;
-    dxs[s] = dys[s] = 0.f;
-    if (valid) {
-      const int p = base + __popc(m & gc.lt_mask);
-      cell[s] = __ldg(a.pin_cell + p);
-      dxs[s] = __ldg(a.pin_dx + p);
-      dys[s] = __ldg(a.pin_dy + p);
-      vm |= 1u << s;
-    }
+    const int p = valid ? base + __popc(m & gc.lt_mask) : wg.pin_base;
+    raw[s] = gc.slot[p];
+    dxs[s] = gc.dx[p];
+    dys[s] = gc.dy[p];
+    const int ps = raw[s] & 0x7fffffff;
+    xc[s] = gc.px[ps];
+    yc[s] = gc.py[ps];
+    vm |= (valid ? 1u : 0u) << s;
     base += __popc(m);
   }
-  // ---- phase B: pin positions px = x_cell + dx as (hi, lo) pairs ----
+  return vm;
+}
+
+// HPWL modes (MODE 1: WA + gradient + HPWL, MODE 2: HPWL only): exact TwoSum positions.
+template <int MODE, int S>
+__device__ __forceinline__ void wa_group_exact(const WaArgs &a, const WarpGroup &wg, const GroupCtx &gc, float &wl_acc,
+                                               unsigned long long (&L)[kHpwlLimbs + 1]) {
+  constexpr bool kGrad = MODE != 2;
+  const int glog = wg.g_log2, G = 1 << glog;
+  const int gi = gc.lane >> glog, j = gc.lane & (G - 1);
+  int d = 0, counted = 0;
+  float we = 1.f;
+  if (gi < wg.nnets) {
+    const int r = gc.deg[wg.net_base + gi];
+    d = r & 0x7fffffff;
+    counted = (r >> 31) & 1;
+    if (a.has_w) we = gc.w[wg.net_base + gi];
+  }
+  int raw[S];
+  float xc[S], yc[S], dxs[S], dys[S];
+  const unsigned vm = load_pins<S>(wg, gc, G, j, d, raw, xc, yc, dxs, dys);
   float hx[S], lx[S], hy[S], ly[S];
   Axis X{-INFINITY, 0.f, INFINITY, 0.f}, Y{-INFINITY, 0.f, INFINITY, 0.f};
 #pragma unroll
   for (int s = 0; s < S; s++) {
-    hx[s] = lx[s] = hy[s] = ly[s] = 0.f;
+    two_sum(xc[s], dxs[s], hx[s], lx[s]);
+    two_sum(yc[s], dys[s], hy[s], ly[s]);
     if (vm & (1u << s)) {
-      const int c = cell[s] & 0x7fffffff;
-      const int wi = c - gc.ch.win_lo;
-      float xc, yc;
-      if ((unsigned)wi < (unsigned)gc.ch.win_n) {
-        const float2 q = gc.s_pos[wi];
-        xc = q.x;
-        yc = q.y;
-      } else {
-        xc = __ldg(a.x + c);
-        yc = __ldg(a.y + c);
-      }
-      if (kHpwl) {
-        two_sum(xc, dxs[s], hx[s], lx[s]);
-        two_sum(yc, dys[s], hy[s], ly[s]);
-      } else {
-        fast_sum(xc, dxs[s], hx[s], lx[s]);
-        fast_sum(yc, dys[s], hy[s], ly[s]);
-      }
-      ext_update<kHpwl>(X, hx[s], lx[s]);
-      ext_update<kHpwl>(Y, hy[s], ly[s]);
+      ext_update(X, hx[s], lx[s]);
+      ext_update(Y, hy[s], ly[s]);
     }
   }
   for (int o = 1; o < G; o <<= 1) {
-    ext_shfl<kHpwl>(X, o);
-    ext_shfl<kHpwl>(Y, o);
+    ext_shfl(X, o);
+    ext_shfl(Y, o);
   }
-  const bool leader = (j == 0) && d >= 2;
-  if (kHpwl && leader && counted) {
-    // px = fl64(x + dx) as the oracle forms it: (double)hi + (double)lo rounds the exact
-    // real x + dx once (reading A7)
+  if (j == 0 && d >= 2 && counted) {
+    // px = fl64(x + dx) as the oracle forms it: (double)hi + (double)lo rounds the exact real
+    // x + dx once (reading A7)
     const double xp = __dadd_rn((double)X.Ph, (double)X.Pl), xm = __dadd_rn((double)X.Mh, (double)X.Ml);
     const double yp = __dadd_rn((double)Y.Ph, (double)Y.Pl), ym = __dadd_rn((double)Y.Mh, (double)Y.Ml);
     limbs_add(L, __dadd_rn(__dsub_rn(xp, xm), __dsub_rn(yp, ym)));
   }
   if (!kGrad) return;
-  // ---- shifted exponentials a^+- and sums b^+-, c~^+- (Table I) ----
   float lxp[S], lxm[S], lyp[S], lym[S], axp[S], axm[S], ayp[S], aym[S];
   float bxp = 0.f, bxm = 0.f, cxp = 0.f, cxm = 0.f, byp = 0.f, bym = 0.f, cyp = 0.f, cym = 0.f;
 #pragma unroll
   for (int s = 0; s < S; s++) {
-    lxp[s] = lxm[s] = lyp[s] = lym[s] = 0.f;
-    axp[s] = axm[s] = ayp[s] = aym[s] = 0.f;
-    if (vm & (1u << s)) {
-      lxp[s] = __fadd_rn(__fsub_rn(hx[s], X.Ph), __fsub_rn(lx[s], X.Pl));   // <= 0 (net-local)
-      lxm[s] = __fadd_rn(__fsub_rn(hx[s], X.Mh), __fsub_rn(lx[s], X.Ml));   // >= 0
-      lyp[s] = __fadd_rn(__fsub_rn(hy[s], Y.Ph), __fsub_rn(ly[s], Y.Pl));
-      lym[s] = __fadd_rn(__fsub_rn(hy[s], Y.Mh), __fsub_rn(ly[s], Y.Ml));
-      axp[s] = ex2(lxp[s] * a.k2);
-      axm[s] = ex2(-lxm[s] * a.k2);
-      ayp[s] = ex2(lyp[s] * a.k2);
-      aym[s] = ex2(-lym[s] * a.k2);
-      bxp += axp[s]; cxp = fmaf(lxp[s], axp[s], cxp);
-      bxm += axm[s]; cxm = fmaf(lxm[s], axm[s], cxm);
-      byp += ayp[s]; cyp = fmaf(lyp[s], ayp[s], cyp);
-      bym += aym[s]; cym = fmaf(lym[s], aym[s], cym);
-    }
+    const bool v = vm & (1u << s);
+    lxp[s] = v ? __fadd_rn(__fsub_rn(hx[s], X.Ph), __fsub_rn(lx[s], X.Pl)) * a.k2 : -1e30f;
+    lxm[s] = v ? __fadd_rn(__fsub_rn(hx[s], X.Mh), __fsub_rn(lx[s], X.Ml)) * a.k2 : 1e30f;
+    lyp[s] = v ? __fadd_rn(__fsub_rn(hy[s], Y.Ph), __fsub_rn(ly[s], Y.Pl)) * a.k2 : -1e30f;
+    lym[s] = v ? __fadd_rn(__fsub_rn(hy[s], Y.Mh), __fsub_rn(ly[s], Y.Ml)) * a.k2 : 1e30f;
+    axp[s] = ex2(lxp[s]);
+    axm[s] = ex2(-lxm[s]);
+    ayp[s] = ex2(lyp[s]);
+    aym[s] = ex2(-lym[s]);
+    bxp += axp[s]; cxp = fmaf(lxp[s], axp[s], cxp);
+    bxm += axm[s]; cxm = fmaf(lxm[s], axm[s], cxm);
+    byp += ayp[s]; cyp = fmaf(lyp[s], ayp[s], cyp);
+    bym += aym[s]; cym = fmaf(lym[s], aym[s], cym);
   }
   for (int o = 1; o < G; o <<= 1) {
     bxp += __shfl_xor_sync(0xffffffffu, bxp, o);
@@ -289,102 +282,309 @@ __device__ __forceinline__ void wa_group(const WaArgs &a, const WarpGroup &wg, c
     bym += __shfl_xor_sync(0xffffffffu, bym, o);
     cym += __shfl_xor_sync(0xffffffffu, cym, o);
   }
-  if (d < 2) return;  // lanes without a net; degree-1 nets are dropped at create
-  const float ibxp = __frcp_rn(bxp), ibxm = __frcp_rn(bxm), ibyp = __frcp_rn(byp), ibym = __frcp_rn(bym);
+  if (d < 2) return;
+  const float ibxp = rcp(bxp), ibxm = rcp(bxm), ibyp = rcp(byp), ibym = rcp(bym);
   const float mxp = cxp * ibxp, mxm = cxm * ibxm, myp = cyp * ibyp, mym = cym * ibym;
-  if (leader && counted) {
-    // WL_e = c+/b+ - c-/b- = (x+ - x-) + c~+/b+ - c~-/b-   (eq 3 in net-local coordinates)
+  if (j == 0 && counted) {
+    const float ig2 = a.gamma * kLn2;
     const float spanx = __fadd_rn(__fsub_rn(X.Ph, X.Mh), __fsub_rn(X.Pl, X.Ml));
     const float spany = __fadd_rn(__fsub_rn(Y.Ph, Y.Mh), __fsub_rn(Y.Pl, Y.Ml));
-    wl_acc += (double)(we * ((spanx + mxp - mxm) + (spany + myp - mym)));
+    wl_acc += we * ((spanx + (mxp - mxm) * ig2) + (spany + (myp - mym) * ig2));
   }
-  // eq (6): dWL/dx_i = a+_i/b+ (1 + (l+_i - m+)/g) - a-_i/b- (1 - (l-_i - m-)/g)
-  //                  = a+_i (P+ + l+_i Q+) - a-_i (P- - l-_i Q-)
-  const float ig = a.inv_gamma;
-  const float qxp = we * ibxp * ig, pxp = we * ibxp * (1.f - mxp * ig);
-  const float qxm = we * ibxm * ig, pxm = we * ibxm * (1.f + mxm * ig);
-  const float qyp = we * ibyp * ig, pyp = we * ibyp * (1.f - myp * ig);
-  const float qym = we * ibym * ig, pym = we * ibym * (1.f + mym * ig);
+  const float wl2 = we * kLn2;
+  const float qxp = ibxp * wl2, pxp = we * ibxp - mxp * qxp;
+  const float qxm = ibxm * wl2, pxm = we * ibxm + mxm * qxm;
+  const float qyp = ibyp * wl2, pyp = we * ibyp - myp * qyp;
+  const float qym = ibym * wl2, pym = we * ibym + mym * qym;
 #pragma unroll
   for (int s = 0; s < S; s++) {
-    if ((vm & (1u << s)) && cell[s] >= 0) {  // cell < 0: foreign pin (another rank owns it)
+    if (vm & (1u << s)) {
       const float gx = axp[s] * fmaf(lxp[s], qxp, pxp) - axm[s] * fmaf(-lxm[s], qxm, pxm);
       const float gy = ayp[s] * fmaf(lyp[s], qyp, pyp) - aym[s] * fmaf(-lym[s], qym, pym);
-      const int wi = cell[s] - gc.ch.win_lo;
-      if ((unsigned)wi < (unsigned)gc.ch.win_n) {
-        atomicAdd(gc.s_g + 2 * wi, gx);
-        atomicAdd(gc.s_g + 2 * wi + 1, gy);
-      } else {
-        red_v2(a.g2 + cell[s], gx, gy);
-      }
+      grad_add(gc, raw[s], gx, gy);
     }
   }
 }
+
+// Headline path (no HPWL).  Shift reference = the rounded extreme P = max fl(x_c + dx): for
+// every pin whose exponential matters, (x_c - P) is exact (Sterbenz) and the one rounding of
+// P is a common shift that cancels in eq (3)/(6).  Everything is carried in log2 units
+// lambda = (x - P) log2(e)/gamma, so a = 2^lambda and (x - m)/gamma = (lambda - mu) ln 2.
+// Invalid slots get lambda = -+1e30 (a = 0, lambda a = 0): no per-slot branches.
+template <int S>
+__device__ __forceinline__ void wa_group_fast(const WaArgs &a, const WarpGroup &wg, const GroupCtx &gc,
+                                              float &wl_acc) {
+  const int glog = wg.g_log2, G = 1 << glog;
+  const int gi = gc.lane >> glog, j = gc.lane & (G - 1);
+  int d = 0, counted = 0;
+  float we = 1.f;
+  if (gi < wg.nnets) {
+    const int r = gc.deg[wg.net_base + gi];
+    d = r & 0x7fffffff;
+    counted = (r >> 31) & 1;
+    if (a.has_w) we = gc.w[wg.net_base + gi];
+  }
+  int raw[S];
+  float xc[S], yc[S], dxs[S], dys[S];
+  const unsigned vm = load_pins<S>(wg, gc, G, j, d, raw, xc, yc, dxs, dys);
+  float Px = -INFINITY, Mx = INFINITY, Py = -INFINITY, My = INFINITY;
+#pragma unroll
+  for (int s = 0; s < S; s++) {
+    const bool v = vm & (1u << s);
+    const float px = xc[s] + dxs[s], py = yc[s] + dys[s];
+    Px = fmaxf(Px, v ? px : -INFINITY);
+    Mx = fminf(Mx, v ? px : INFINITY);
+    Py = fmaxf(Py, v ? py : -INFINITY);
+    My = fminf(My, v ? py : INFINITY);
+  }
+  for (int o = 1; o < G; o <<= 1) {
+    Px = fmaxf(Px, __shfl_xor_sync(0xffffffffu, Px, o));
+    Mx = fminf(Mx, __shfl_xor_sync(0xffffffffu, Mx, o));
+    Py = fmaxf(Py, __shfl_xor_sync(0xffffffffu, Py, o));
+    My = fminf(My, __shfl_xor_sync(0xffffffffu, My, o));
+  }
+  const float k2 = a.k2;
+  float lxp[S], lxm[S], lyp[S], lym[S], axp[S], axm[S], ayp[S], aym[S];
+  float bxp = 0.f, bxm = 0.f, cxp = 0.f, cxm = 0.f, byp = 0.f, bym = 0.f, cyp = 0.f, cym = 0.f;
+#pragma unroll
+  for (int s = 0; s < S; s++) {
+    const bool v = vm & (1u << s);
+    const float dkx = dxs[s] * k2, dky = dys[s] * k2;
+    lxp[s] = v ? fmaf(xc[s] - Px, k2, dkx) : -1e30f;   // <= 0 (to an ulp of P)
+    lxm[s] = v ? fmaf(xc[s] - Mx, k2, dkx) : 1e30f;    // >= 0
+    lyp[s] = v ? fmaf(yc[s] - Py, k2, dky) : -1e30f;
+    lym[s] = v ? fmaf(yc[s] - My, k2, dky) : 1e30f;
+    axp[s] = ex2(lxp[s]);
+    axm[s] = ex2(-lxm[s]);
+    ayp[s] = ex2(lyp[s]);
+    aym[s] = ex2(-lym[s]);
+    bxp += axp[s]; cxp = fmaf(lxp[s], axp[s], cxp);
+    bxm += axm[s]; cxm = fmaf(lxm[s], axm[s], cxm);
+    byp += ayp[s]; cyp = fmaf(lyp[s], ayp[s], cyp);
+    bym += aym[s]; cym = fmaf(lym[s], aym[s], cym);
+  }
+  for (int o = 1; o < G; o <<= 1) {
+    bxp += __shfl_xor_sync(0xffffffffu, bxp, o);
+    cxp += __shfl_xor_sync(0xffffffffu, cxp, o);
+    bxm += __shfl_xor_sync(0xffffffffu, bxm, o);
+    cxm += __shfl_xor_sync(0xffffffffu, cxm, o);
+    byp += __shfl_xor_sync(0xffffffffu, byp, o);
+    cyp += __shfl_xor_sync(0xffffffffu, cyp, o);
+    bym += __shfl_xor_sync(0xffffffffu, bym, o);
+    cym += __shfl_xor_sync(0xffffffffu, cym, o);
+  }
+  if (d < 2) return;
+  const float ibxp = rcp(bxp), ibxm = rcp(bxm), ibyp = rcp(byp), ibym = rcp(bym);
+  const float mxp = cxp * ibxp, mxm = cxm * ibxm, myp = cyp * ibyp, mym = cym * ibym;  // log2 units
+  if (j == 0 && counted) {
+    // WL_e = (x+ - x-) + (mu+ - mu-) gamma ln 2   (eq 3 in shifted coordinates)
+    const float ig2 = a.gamma * kLn2;
+    wl_acc += we * ((Px - Mx) + (mxp - mxm) * ig2 + (Py - My) + (myp - mym) * ig2);
+  }
+  // eq (6) in log2 units: a+ (P+ + lambda+ Q+) - a- (P- - lambda- Q-)
+  const float wl2 = we * kLn2;
+  const float qxp = ibxp * wl2, pxp = we * ibxp - mxp * qxp;
+  const float qxm = ibxm * wl2, pxm = we * ibxm + mxm * qxm;
+  const float qyp = ibyp * wl2, pyp = we * ibyp - myp * qyp;
+  const float qym = ibym * wl2, pym = we * ibym + mym * qym;
+#pragma unroll
+  for (int s = 0; s < S; s++) {
+    if (vm & (1u << s)) {
+      const float gx = axp[s] * fmaf(lxp[s], qxp, pxp) - axm[s] * fmaf(-lxm[s], qxm, pxm);
+      const float gy = ayp[s] * fmaf(lyp[s], qyp, pyp) - aym[s] * fmaf(-lym[s], qym, pym);
+      grad_add(gc, raw[s], gx, gy);
+    }
+  }
+}
+
+// tanh(u/2) for u = t ln2 >= 0 given e = 2^-t: series for small u (1 - e loses digits),
+// (1 - e)/(1 + e) otherwise.
+__device__ __forceinline__ float tanh_half(float t, float e) {
+  const float h = 0.5f * kLn2 * t;
+  if (h < 0.0625f) {
+    const float h2 = h * h;
+    return h * fmaf(h2, fmaf(h2, 2.f / 15.f, -1.f / 3.f), 1.f);
+  }
+  return (1.f - e) * rcp(1.f + e);
+}
+
+// Warp groups of 2-pin nets (G = 1): the closed form of eqs (3)/(6) for two pins at
+// separation delta, WA = |delta| tanh(|delta| / 2 gamma) and dWA/dx_2 = -dWA/dx_1 =
+// sign(delta) [tanh(u/2) + (u/2) sech^2(u/2)], u = |delta| / gamma (pinned against the oracle
+// in tests/test_oracle_wa.py::test_two_pin_closed_form).
+__device__ __forceinline__ void wa_group_pairs(const WaArgs &a, const WarpGroup &wg, const GroupCtx &gc,
+                                               float &wl_acc) {
+  const int lane = gc.lane;
+  if (lane >= wg.nnets) return;
+  const int r = gc.deg[wg.net_base + lane];
+  const int counted = (r >> 31) & 1;
+  const float we = a.has_w ? gc.w[wg.net_base + lane] : 1.f;
+  // slot-major: pin 0 of net L at pin_base + L, pin 1 at pin_base + nnets + L
+  const int p0 = wg.pin_base + lane, p1 = p0 + wg.nnets;
+  const int r0 = gc.slot[p0], r1 = gc.slot[p1];
+  const int s0 = r0 & 0x7fffffff, s1 = r1 & 0x7fffffff;
+  const float ddx = (gc.px[s1] - gc.px[s0]) + (gc.dx[p1] - gc.dx[p0]);
+  const float ddy = (gc.py[s1] - gc.py[s0]) + (gc.dy[p1] - gc.dy[p0]);
+  const float tx = fabsf(ddx) * a.k2, ty = fabsf(ddy) * a.k2;   // u log2(e)
+  const float thx = tanh_half(tx, ex2(-tx)), thy = tanh_half(ty, ex2(-ty));
+  if (counted) wl_acc += we * (fabsf(ddx) * thx + fabsf(ddy) * thy);
+  const float hx = 0.5f * kLn2 * tx, hy = 0.5f * kLn2 * ty;
+  const float gx = copysignf(we * fmaf(hx, fmaf(-thx, thx, 1.f), thx), ddx);   // d/dx of pin 1
+  const float gy = copysignf(we * fmaf(hy, fmaf(-thy, thy, 1.f), thy), ddy);
+  grad_add(gc, r1, gx, gy);
+  grad_add(gc, r0, -gx, -gy);
+}
+
+__device__ __forceinline__ unsigned smem_u32(const void *p) { return (unsigned)__cvta_generic_to_shared(p); }
+
+__device__ __forceinline__ void bulk_g2s(void *dst, const void *src, unsigned bytes, uint64_t *bar) {
+  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+               ::"r"(smem_u32(dst)), "l"(src), "r"(bytes), "r"(smem_u32(bar))
+               : "memory");
+}
+
+__device__ __forceinline__ void mbar_wait(uint64_t *bar, unsigned phase) {
+  unsigned done = 0;
+  while (!done) {
+    asm volatile(
+        "{\n .reg .pred p;\n mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n selp.u32 %0, 1, 0, p;\n}"
+        : "=r"(done)
+        : "r"(smem_u32(bar)), "r"(phase)
+        : "memory");
+  }
+}
+
+// Dynamic shared-memory layout of the chunk kernel (capacities fixed at create).
+struct WaSmem {
+  WaCaps c;
+  __host__ __device__ int slots() const { return kWaWindow + c.far + 4; }   // + trash, padded
+  __host__ __device__ int off_slot() const { return 0; }
+  __host__ __device__ int off_dx() const { return 4 * c.pins; }
+  __host__ __device__ int off_dy() const { return 8 * c.pins; }
+  __host__ __device__ int off_deg() const { return 12 * c.pins; }
+  __host__ __device__ int off_w() const { return off_deg() + 4 * c.nets; }
+  __host__ __device__ int off_wg() const { return off_w() + 4 * c.nets; }
+  __host__ __device__ int off_far() const { return off_wg() + 16 * c.groups; }
+  __host__ __device__ int off_px() const { return off_far() + 4 * c.far; }
+  __host__ __device__ int off_py() const { return off_px() + 4 * slots(); }
+  __host__ __device__ int off_g() const { return off_py() + 4 * slots(); }
+  __host__ __device__ int off_bar() const { return off_g() + 8 * slots(); }
+  __host__ __device__ int bytes() const { return off_bar() + 16; }
+};
 
 // MODE 0: WA + gradient; 1: WA + gradient + HPWL; 2: HPWL only.
 template <int MODE>
 __global__ void __launch_bounds__(kWaThreads, 3) k_wa_chunks(WaArgs a) {
   constexpr bool kGrad = MODE != 2;
   constexpr bool kHpwl = MODE != 0;
-  __shared__ float2 s_pos[kWaWindow];
-  __shared__ float s_g[kGrad ? 2 * kWaWindow : 1];
-  __shared__ int s_next;
+  extern __shared__ __align__(16) unsigned char smem[];
+  const WaSmem L_{a.caps};
+  int *s_slot = reinterpret_cast<int *>(smem + L_.off_slot());
+  float *s_dx = reinterpret_cast<float *>(smem + L_.off_dx());
+  float *s_dy = reinterpret_cast<float *>(smem + L_.off_dy());
+  int *s_deg = reinterpret_cast<int *>(smem + L_.off_deg());
+  float *s_w = reinterpret_cast<float *>(smem + L_.off_w());
+  WarpGroup *s_wg = reinterpret_cast<WarpGroup *>(smem + L_.off_wg());
+  int *s_far = reinterpret_cast<int *>(smem + L_.off_far());
+  float *s_px = reinterpret_cast<float *>(smem + L_.off_px());
+  float *s_py = reinterpret_cast<float *>(smem + L_.off_py());
+  int *s_g = reinterpret_cast<int *>(smem + L_.off_g());
+  uint64_t *bar = reinterpret_cast<uint64_t *>(smem + L_.off_bar());
 
   const Chunk ch = a.chunks[blockIdx.x];
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-  for (int i = tid; i < ch.win_n; i += kWaThreads) {
-    s_pos[i] = make_float2(__ldg(a.x + ch.win_lo + i), __ldg(a.y + ch.win_lo + i));
-    if (kGrad) {
-      s_g[2 * i] = 0.f;
-      s_g[2 * i + 1] = 0.f;
+  // window positions by bulk copy when 16-byte aligned (the caller's x / y), else by threads
+  const int wbulk = ch.win_n & ~3;
+  const bool win_bulk = ((((uintptr_t)(a.x + ch.win_lo)) | ((uintptr_t)(a.y + ch.win_lo))) & 15) == 0 && wbulk > 0;
+  if (tid == 0) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(1) : "memory");
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    const unsigned tx = 12u * ch.pin_n + (a.has_w ? 8u : 4u) * ch.net_n + 16u * ch.wg_n + 4u * ch.far_pad +
+                        (win_bulk ? 8u * wbulk : 0u);
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(tx) : "memory");
+    if (ch.pin_n) {
+      bulk_g2s(s_slot, a.pin_slot + ch.pin_begin, 4u * ch.pin_n, bar);
+      bulk_g2s(s_dx, a.pin_dx + ch.pin_begin, 4u * ch.pin_n, bar);
+      bulk_g2s(s_dy, a.pin_dy + ch.pin_begin, 4u * ch.pin_n, bar);
+    }
+    if (ch.net_n) {
+      bulk_g2s(s_deg, a.net_deg + ch.net_begin, 4u * ch.net_n, bar);
+      if (a.has_w) bulk_g2s(s_w, a.net_w + ch.net_begin, 4u * ch.net_n, bar);
+    }
+    if (ch.wg_n) bulk_g2s(s_wg, a.wgs + ch.wg_begin, 16u * ch.wg_n, bar);
+    if (ch.far_pad) bulk_g2s(s_far, a.far_cells + ch.far_begin, 4u * ch.far_pad, bar);
+    if (win_bulk) {
+      bulk_g2s(s_px, a.x + ch.win_lo, 4u * wbulk, bar);
+      bulk_g2s(s_py, a.y + ch.win_lo, 4u * wbulk, bar);
     }
   }
-  if (tid == 0) s_next = ch.wg_begin + kWaThreads / 32;
+  const int nslots = L_.slots();
+  if (kGrad)
+    for (int i = tid; i < 2 * nslots; i += kWaThreads) s_g[i] = 0;
+  for (int i = (win_bulk ? wbulk : 0) + tid; i < ch.win_n; i += kWaThreads) {
+    s_px[i] = __ldg(a.x + ch.win_lo + i);
+    s_py[i] = __ldg(a.y + ch.win_lo + i);
+  }
+  __syncthreads();   // barrier initialised before anyone waits on it
+  mbar_wait(bar, 0);
+  // far cells: positions gathered once per chunk
+  for (int f = tid; f < ch.far_n; f += kWaThreads) {
+    const int c = s_far[f];
+    s_px[kWaWindow + f] = __ldg(a.x + c);
+    s_py[kWaWindow + f] = __ldg(a.y + c);
+  }
   __syncthreads();
 
-  double wl_acc = 0.0;
+  float wl_acc = 0.f;
   unsigned long long L[kHpwlLimbs + 1];
 #pragma unroll
   for (int k = 0; k <= kHpwlLimbs; k++) L[k] = 0ull;
-  const GroupCtx gc{ch, s_pos, s_g, lane, (1u << lane) - 1u};
+  const GroupCtx gc{s_slot, s_dx, s_dy, s_deg, s_w, s_px, s_py, s_g, nslots - 1, exp2f((float)ch.scale_log2),
+                    lane, (1u << lane) - 1u};
 
-  // warp groups are handed out dynamically inside the CTA (self-balancing)
-  int wgi = ch.wg_begin + warp;
-  while (wgi < ch.wg_end) {
-    const WarpGroup wg = a.wgs[wgi];
-    switch (wg.slots) {
-      case 1: wa_group<MODE, 1>(a, wg, gc, wl_acc, L); break;
-      case 2: wa_group<MODE, 2>(a, wg, gc, wl_acc, L); break;
-      case 3: wa_group<MODE, 3>(a, wg, gc, wl_acc, L); break;
-      default: wa_group<MODE, 4>(a, wg, gc, wl_acc, L); break;
+  // warp groups are dealt round-robin (the host orders them by decreasing cost)
+  for (int gi = warp; gi < ch.wg_n; gi += kWaThreads / 32) {
+    const WarpGroup wg = s_wg[gi];
+    if (MODE == 0) {
+      if (wg.flags & 1) {
+        wa_group_pairs(a, wg, gc, wl_acc);
+      } else {
+        switch (wg.slots) {
+          case 1: wa_group_fast<1>(a, wg, gc, wl_acc); break;
+          case 2: wa_group_fast<2>(a, wg, gc, wl_acc); break;
+          case 3: wa_group_fast<3>(a, wg, gc, wl_acc); break;
+          default: wa_group_fast<4>(a, wg, gc, wl_acc); break;
+        }
+      }
+    } else {
+      switch (wg.slots) {
+        case 1: wa_group_exact<MODE, 1>(a, wg, gc, wl_acc, L); break;
+        case 2: wa_group_exact<MODE, 2>(a, wg, gc, wl_acc, L); break;
+        case 3: wa_group_exact<MODE, 3>(a, wg, gc, wl_acc, L); break;
+        default: wa_group_exact<MODE, 4>(a, wg, gc, wl_acc, L); break;
+      }
     }
-    int nx = 0;
-    if (lane == 0) nx = atomicAdd(&s_next, 1);
-    wgi = __shfl_sync(0xffffffffu, nx, 0);
   }
   __syncthreads();
   if (kGrad) {
-    // flush the window: cells [win_lo, win_lo + win_n) as 16-byte vector reductions
-    float4 *g4 = reinterpret_cast<float4 *>(a.g2);
-    const int lo = ch.win_lo, n = ch.win_n;
-    const int head = lo & 1;  // an odd first cell is flushed alone
-    if (head && tid == 0 && n > 0) {
-      const float gx = s_g[0], gy = s_g[1];
-      if (gx != 0.f || gy != 0.f) red_v2(a.g2 + lo, gx, gy);
-    }
-    const int npair = (n - head) >> 1;
+    const float inv = exp2f(-(float)ch.scale_log2);
+    // window: cells [win_lo, win_lo + win_n), win_lo a multiple of 4 -> 16-byte vector reductions
+    float4 *g4 = reinterpret_cast<float4 *>(a.g2 + ch.win_lo);
+    const int npair = ch.win_n >> 1;
     for (int i = tid; i < npair; i += kWaThreads) {
-      const int w = head + 2 * i;
-      const float v0 = s_g[2 * w], v1 = s_g[2 * w + 1], v2 = s_g[2 * w + 2], v3 = s_g[2 * w + 3];
-      if (v0 != 0.f || v1 != 0.f || v2 != 0.f || v3 != 0.f) red_v4(g4 + ((lo + w) >> 1), v0, v1, v2, v3);
+      const int4 v = *reinterpret_cast<const int4 *>(s_g + 4 * i);
+      if (v.x | v.y | v.z | v.w) red_v4(g4 + i, v.x * inv, v.y * inv, v.z * inv, v.w * inv);
     }
-    if (((n - head) & 1) && tid == 0) {
-      const int w = n - 1;
-      const float gx = s_g[2 * w], gy = s_g[2 * w + 1];
-      if (gx != 0.f || gy != 0.f) red_v2(a.g2 + lo + w, gx, gy);
+    if ((ch.win_n & 1) && tid == 0) {
+      const int w = ch.win_n - 1;
+      if (s_g[2 * w] | s_g[2 * w + 1]) red_v2(a.g2 + ch.win_lo + w, s_g[2 * w] * inv, s_g[2 * w + 1] * inv);
+    }
+    for (int f = tid; f < ch.far_n; f += kWaThreads) {
+      const int gx = s_g[2 * (kWaWindow + f)], gy = s_g[2 * (kWaWindow + f) + 1];
+      if (gx | gy) red_v2(a.g2 + s_far[f], gx * inv, gy * inv);
     }
   }
-  block_flush_scalars<kWaThreads>(wl_acc, L, kHpwl, kGrad ? a.part + blockIdx.x : nullptr, a.limbs);
+  block_flush_scalars<kWaThreads>((double)wl_acc, L, kHpwl, kGrad ? a.part + blockIdx.x : nullptr, a.limbs);
 }
 
 // ---------------------------------------------------------------------------------------
@@ -509,22 +709,35 @@ __global__ void __launch_bounds__(kBigThreads) k_wa_big(WaArgs a) {
 
 template <int MODE>
 void launch_mode(const Ctx &c, const WaArgs &a, cudaStream_t s) {
-  if (c.n_chunks > 0) k_wa_chunks<MODE><<<c.n_chunks, kWaThreads, 0, s>>>(a);
+  const WaSmem L{a.caps};
+  if (c.n_chunks > 0) k_wa_chunks<MODE><<<c.n_chunks, kWaThreads, L.bytes(), s>>>(a);
   if (c.n_big > 0) k_wa_big<MODE><<<c.n_big, kBigThreads, 0, s>>>(a);
 }
 
 }  // namespace
 
-void launch_wa(const Ctx &c, const float *x, const float *y, float gamma, bool hpwl_only,
-               bool with_hpwl, cudaStream_t s) {
+int wa_smem_bytes(const WaCaps &caps) { return WaSmem{caps}.bytes(); }
+
+cudaError_t wa_configure(const WaCaps &caps) {
+  const int b = WaSmem{caps}.bytes();
+  cudaError_t e = cudaFuncSetAttribute(k_wa_chunks<0>, cudaFuncAttributeMaxDynamicSharedMemorySize, b);
+  if (e != cudaSuccess) return e;
+  e = cudaFuncSetAttribute(k_wa_chunks<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, b);
+  if (e != cudaSuccess) return e;
+  return cudaFuncSetAttribute(k_wa_chunks<2>, cudaFuncAttributeMaxDynamicSharedMemorySize, b);
+}
+
+void launch_wa(const Ctx &c, const float *x, const float *y, float gamma, bool hpwl_only, bool with_hpwl,
+               cudaStream_t s) {
   WaArgs a;
   a.chunks = c.d_chunks;
   a.wgs = c.d_wgroups;
   a.net_deg = c.d_net_deg;
   a.net_w = c.d_net_w;
-  a.pin_cell = c.d_pin_cell;
+  a.pin_slot = c.d_pin_cell;
   a.pin_dx = c.d_pin_dx;
   a.pin_dy = c.d_pin_dy;
+  a.far_cells = c.d_far_cells;
   a.x = x;
   a.y = y;
   a.g2 = c.d_g2;
@@ -541,6 +754,7 @@ void launch_wa(const Ctx &c, const float *x, const float *y, float gamma, bool h
   a.big_dx = c.d_big_dx;
   a.big_dy = c.d_big_dy;
   a.part_offset = c.n_chunks;
+  a.caps = c.wa_caps;
   if (hpwl_only)
     launch_mode<2>(c, a, s);
   else if (with_hpwl)

@@ -112,13 +112,20 @@ __device__ __forceinline__ float2 inv_pre(float pk, float qk, float pnk, float q
 // ---------------------------------------------------------------------------------------
 // T1 / debug: forward DCT over rows, rows (2r, 2r+1) share one complex FFT.
 // ---------------------------------------------------------------------------------------
-__global__ void __launch_bounds__(kRowThreads) k_row_dct(const float *__restrict__ in, float *__restrict__ out,
+// IN = float, or unsigned long long = int64 fixed point in 2^-kRhoScaleLog2 units (the bin map)
+__device__ __forceinline__ float load_map(const float *p) { return __ldg(p); }
+__device__ __forceinline__ float load_map(const unsigned long long *p) {
+  return (float)((double)(long long)__ldg(p) * (1.0 / (double)(1ll << kRhoScaleLog2)));
+}
+
+template <class IN>
+__global__ void __launch_bounds__(kRowThreads) k_row_dct(const IN *__restrict__ in, float *__restrict__ out,
                                                          int n, int log2n, const float2 *__restrict__ tw,
                                                          const float2 *__restrict__ ph) {
   extern __shared__ float2 zbuf[];
-  const float *r0 = in + (size_t)(2 * blockIdx.x) * n, *r1 = r0 + n;
+  const IN *r0 = in + (size_t)(2 * blockIdx.x) * n, *r1 = r0 + n;
   for (int t = threadIdx.x; t < n; t += kRowThreads)
-    zbuf[brev(mk_pos(t, n), log2n)] = make_float2(__ldg(r0 + t), __ldg(r1 + t));
+    zbuf[brev(mk_pos(t, n), log2n)] = make_float2(load_map(r0 + t), load_map(r1 + t));
   __syncthreads();
   fft_block(zbuf, n, log2n, 1, tw, false);
   float *o0 = out + (size_t)(2 * blockIdx.x) * n, *o1 = o0 + n;
@@ -375,7 +382,9 @@ void row_inv(const Ctx &c, const float *inA, long long stepA, int opA, const flo
 // smem opt-in (called once from dp_create)
 cudaError_t dct_configure(int mx, int my) {
   cudaError_t e;
-  e = cudaFuncSetAttribute(k_row_dct, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)row_smem(my));
+  e = cudaFuncSetAttribute(k_row_dct<float>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)row_smem(my));
+  if (e != cudaSuccess) return e;
+  e = cudaFuncSetAttribute(k_row_dct<unsigned long long>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)row_smem(my));
   if (e != cudaSuccess) return e;
   e = cudaFuncSetAttribute(k_row_inv, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)row_smem(my));
   if (e != cudaSuccess) return e;
@@ -386,9 +395,33 @@ cudaError_t dct_configure(int mx, int my) {
 
 int col_fields_ctas(int mx, int my) { return my / col_slab(mx); }
 
+namespace {
+void fields_after_t1(const Ctx &c, cudaStream_t s);
+}
+
 void launch_fields(const Ctx &c, const float *rho, cudaStream_t s) {
   // T1: t = DCT_y(rho)
-  k_row_dct<<<c.mx / 2, kRowThreads, row_smem(c.my), s>>>(rho, c.d_t, c.my, c.log2my, c.d_tw_y, c.d_ph_y);
+  k_row_dct<float><<<c.mx / 2, kRowThreads, row_smem(c.my), s>>>(rho, c.d_t, c.my, c.log2my, c.d_tw_y, c.d_ph_y);
+  fields_after_t1(c, s);
+}
+
+void launch_fields_fixed(const Ctx &c, cudaStream_t s) {
+  k_row_dct<unsigned long long><<<c.mx / 2, kRowThreads, row_smem(c.my), s>>>(c.d_rho, c.d_t, c.my, c.log2my, c.d_tw_y,
+                                                                              c.d_ph_y);
+  fields_after_t1(c, s);
+}
+
+__global__ void k_rho_to_float(const unsigned long long *in, float *out, size_t n) {
+  for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < n; i += (size_t)gridDim.x * blockDim.x)
+    out[i] = load_map(in + i);
+}
+
+void launch_rho_to_float(const Ctx &c, float *out, cudaStream_t s) {
+  k_rho_to_float<<<c.num_sms * 4, 256, 0, s>>>(c.d_rho, out, (size_t)c.mx * c.my);
+}
+
+namespace {
+void fields_after_t1(const Ctx &c, cudaStream_t s) {
   // T2: columns (DCT_x, scaling, energy, inverse x)
   ColFieldArgs a;
   a.t = c.d_t; a.sx = c.d_sx; a.sy = c.d_sy;
@@ -400,6 +433,7 @@ void launch_fields(const Ctx &c, const float *rho, cudaStream_t s) {
   // T3: rows: xi_X = IDCT_y(sX), xi_Y = IDXST_y(sY), interleaved
   row_inv(c, c.d_sx, c.my, 1, c.d_sy, c.my, 2, nullptr, 0, nullptr, 0, c.d_xi, c.mx, s);
 }
+}  // namespace
 
 void launch_split_fields(const Ctx &c, float *xi_x, float *xi_y, cudaStream_t s) {
   k_split_xi<<<c.num_sms * 4, 256, 0, s>>>(c.d_xi, xi_x, xi_y, (size_t)c.mx * c.my);
@@ -410,7 +444,7 @@ void launch_transform(const Ctx &c, int kind, const float *in, float *out, cudaS
   float *tmp = c.d_t;  // scratch (debug path only)
   switch (kind) {
     case DP_T_DCT2:
-      k_row_dct<<<mx / 2, kRowThreads, row_smem(my), s>>>(in, tmp, my, c.log2my, c.d_tw_y, c.d_ph_y);
+      k_row_dct<float><<<mx / 2, kRowThreads, row_smem(my), s>>>(in, tmp, my, c.log2my, c.d_tw_y, c.d_ph_y);
       k_col_generic<<<my / col_slab(mx), kColThreads, col_generic_smem(mx), s>>>(tmp, out, 0, mx, c.log2mx, my, c.d_tw_x, c.d_ph_x);
       break;
     case DP_T_IDCT2:

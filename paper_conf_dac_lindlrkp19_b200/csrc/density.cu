@@ -19,6 +19,9 @@
 //   D5 gather  one CTA per segment stages the (tile+2)^2 float2 field tile in shared memory
 //              and writes each cell's force
 // Large cells (footprint wider than 3 bins) take a CTA-per-cell path with global reds.
+// The tile accumulators (int32, 2^-19) flush into an int64 global map (2^-24) with native
+// red.global.add.u64: the density map is exact up to one rounding per contribution and
+// independent of execution order (deterministic; bit-identical after an int64 all-reduce).
 // Footprint geometry is computed in fp64 (B200 runs FP64 at half rate); records hold the
 // footprint in fractions of the cell's first bin (|v| < 3) plus that bin's tile-local index.
 #include "dp_internal.h"
@@ -32,14 +35,14 @@ struct DenArgs {
   const float *w, *h;   // own cells
   int cell_begin, n_own;
   double xl, yl, xh, yh, bx, by, sx, sy, ibx, iby;   // ibx = 1 / bx (no fp64 divisions on the hot path)
-  int mx, my, tile, tiles_y, ntiles, stretch;
+  int mx, my, tile, tile_log2, tiles_y, ntiles, stretch;
   int *tile_cnt, *tile_cursor, *tile_off;
   Segment *segs;
   int *nsegs;
   float4 *rec;
   int2 *rec_rc;   // (r as float bits, tile-local first bin i0 | j0 << 16)
   int *rec_cell;  // own cell index
-  float *rho;
+  unsigned long long *rho;   // int64 fixed point, 2^-kRhoScaleLog2 units
   const float2 *xi;
   float2 *force;
   const int *large;
@@ -65,7 +68,7 @@ __device__ __forceinline__ Foot footprint_v(const DenArgs &a, float xf, float yf
   }
   f.large = (w > 2.0 * a.bx) || (h > 2.0 * a.by);
   // charge ratio r = w h / (w' h') in fp32 (only its fp32 rounding is stored)
-  f.r = (wsf * hsf > 0.f) ? __fdiv_rn(wf * hf, wsf * hsf) : 0.f;
+  f.r = (wsf * hsf > 0.f) ? __fdividef(wf * hf, wsf * hsf) : 0.f;
   const double cx = x + 0.5 * w, cy = y + 0.5 * h;
   f.lx = fmax(cx - 0.5 * ws, a.xl);
   f.hx = fmin(cx + 0.5 * ws, a.xh);
@@ -114,9 +117,9 @@ __device__ __forceinline__ int small_tile(const DenArgs &a, const Foot &f, int &
   int bx0 = (int)floor((f.lx - a.xl) * a.ibx), by0 = (int)floor((f.ly - a.yl) * a.iby);
   bx0 = min(max(bx0, 0), a.mx - 1);
   by0 = min(max(by0, 0), a.my - 1);
-  const int tx = bx0 / a.tile, ty = by0 / a.tile;
-  ox = tx * a.tile;
-  oy = ty * a.tile;
+  const int tx = bx0 >> a.tile_log2, ty = by0 >> a.tile_log2;
+  ox = tx << a.tile_log2;
+  oy = ty << a.tile_log2;
   return tx * a.tiles_y + ty;
 }
 
@@ -286,13 +289,13 @@ __global__ void __launch_bounds__(256) k_scatter_tiles(DenArgs a) {
     }
   }
   __syncthreads();
-  const float inv = 1.f / scale;
   for (int k = threadIdx.x; k < P * P; k += blockDim.x) {
     const int iv = s_t[k];
-    const float v = iv * inv;
     const int gi = ox + k / P, gj = oy + k % P;
     if (iv != 0 && gi < a.mx && gj < a.my)
-      asm volatile("red.global.add.f32 [%0], %1;" ::"l"(a.rho + (size_t)gi * a.my + gj), "f"(v) : "memory");
+      asm volatile("red.global.add.u64 [%0], %1;" ::"l"(a.rho + (size_t)gi * a.my + gj),
+                   "l"((unsigned long long)iv << (kRhoScaleLog2 - kTileScaleLog2))
+                   : "memory");
   }
 }
 
@@ -351,8 +354,9 @@ __global__ void __launch_bounds__(256) k_scatter_large(DenArgs a) {
     const double ox = fmin(f.hx, a.xl + (bi + 1) * a.bx) - fmax(f.lx, a.xl + bi * a.bx);
     const double oy = fmin(f.hy, a.yl + (bj + 1) * a.by) - fmax(f.ly, a.yl + bj * a.by);
     if (ox <= 0.0 || oy <= 0.0) continue;
-    const float v = (float)((double)f.r * ox * oy * a.ibx * a.iby);
-    asm volatile("red.global.add.f32 [%0], %1;" ::"l"(a.rho + (size_t)bi * a.my + bj), "f"(v) : "memory");
+    const unsigned long long v =
+        (unsigned long long)__double2ll_rn((double)f.r * ox * oy * a.ibx * a.iby * (double)(1ll << kRhoScaleLog2));
+    asm volatile("red.global.add.u64 [%0], %1;" ::"l"(a.rho + (size_t)bi * a.my + bj), "l"(v) : "memory");
   }
 }
 
@@ -409,6 +413,8 @@ DenArgs make_args(const Ctx &c, const float *x, const float *y) {
   a.ibx = 1.0 / c.bx;
   a.iby = 1.0 / c.by;
   a.mx = c.mx; a.my = c.my; a.tile = c.tile; a.tiles_y = c.tiles_y;
+  a.tile_log2 = 0;
+  while ((1 << a.tile_log2) < c.tile) a.tile_log2++;
   a.ntiles = c.tiles_x * c.tiles_y;
   a.stretch = c.stretch;
   a.tile_cnt = c.d_tile_cnt;
@@ -446,7 +452,7 @@ void launch_density_map(const Ctx &c, const float *x, const float *y, cudaStream
   const int P = c.tile + kHalo;
   const int ntiles = a.ntiles;
   const int nblk = (c.n_own + kCountThreads * 8 - 1) / (kCountThreads * 8);
-  cudaMemsetAsync(c.d_rho, 0, sizeof(float) * (size_t)c.mx * c.my, s);
+  cudaMemsetAsync(c.d_rho, 0, sizeof(unsigned long long) * (size_t)c.mx * c.my, s);
   if (nblk > 0) {
     k_count<<<nblk, kCountThreads, ntiles * 4, s>>>(a);
     k_scan<<<1, 1024, 0, s>>>(a);

@@ -417,8 +417,8 @@ dp_status build_density(Ctx &c, const dp_netlist *nl) {
   if ((st = dev_alloc(c, &c.d_xi, nb)) != DP_OK) return st;
   // force[i] for own cell i = cell_begin + i; offset by the parity of cell_begin so that even
   // global cells are 16-byte aligned (the combine pass reads cell pairs as float4)
-  if ((st = dev_alloc(c, &c.d_force, c.n_own + 2)) != DP_OK) return st;
-  DP_CUDA(cudaMemset(c.d_force, 0, sizeof(float2) * (c.n_own + 2)));
+  if ((st = dev_alloc(c, &c.d_force, c.n_own + 4)) != DP_OK) return st;
+  DP_CUDA(cudaMemset(c.d_force, 0, sizeof(float2) * (c.n_own + 4)));
   c.d_force += (c.cell_begin & 1);
   if ((st = dev_upload(c, &c.d_tw_x, twiddles(c.mx))) != DP_OK) return st;
   if ((st = dev_upload(c, &c.d_tw_y, twiddles(c.my))) != DP_OK) return st;
@@ -585,13 +585,13 @@ dp_status density_chain(Ctx &c, const float *x, const float *y) {
     StageMark m(c, DP_STAGE_MAP, c.s_den);
     launch_density_map(c, x, y, c.s_den);
     if (c.dist && c.nccl_comm) {
-      dp_status st = nccl_allreduce_f32(c, c.d_rho, (size_t)c.mx * c.my, c.s_den);
+      dp_status st = nccl_allreduce_u64(c, c.d_rho, (size_t)c.mx * c.my, c.s_den);   // exact
       if (st != DP_OK) return st;
     }
   }
   {
     StageMark m(c, DP_STAGE_FIELDS, c.s_den);
-    launch_fields(c, c.d_rho, c.s_den);
+    launch_fields_fixed(c, c.s_den);
   }
   StageMark m(c, DP_STAGE_GATHER, c.s_den);
   launch_density_gather(c, x, y, c.s_den);
@@ -640,6 +640,8 @@ dp_status eval_impl(Ctx &c, const float *x, const float *y, float gamma, float l
     DP_CUDA(cudaStreamWaitEvent(c.s_wa, c.ev_fork, 0));
     {
       StageMark m(c, DP_STAGE_WA, c.s_wa);
+      // clear the own-cell range of the WA gradient accumulator (read, not reset, by combine)
+      DP_CUDA(cudaMemsetAsync(c.d_g2 + c.cell_begin, 0, sizeof(float2) * (size_t)(c.cell_end - c.cell_begin), c.s_wa));
       launch_wa(c, x, y, gamma, false, d_hpwl != nullptr, c.s_wa);
     }
     DP_CUDA(cudaEventRecord(c.ev_wa, c.s_wa));
@@ -862,7 +864,7 @@ dp_status dp_debug_density_map(dp_ctx *ctx, const float *x, const float *y, floa
   dp::DeviceGuard g(c->device);
   cudaStream_t s = (cudaStream_t)stream;
   dp::launch_density_map(*c, x, y, s);
-  DP_CUDA(cudaMemcpyAsync(rho, c->d_rho, sizeof(float) * (size_t)c->mx * c->my, cudaMemcpyDeviceToDevice, s));
+  dp::launch_rho_to_float(*c, rho, s);
   DP_CUDA(cudaGetLastError());
   return DP_OK;
 }

@@ -28,6 +28,7 @@ constexpr int kTile = 32;             // density tile = kTile x kTile bins
 constexpr int kHalo = 2;              // small-cell footprints extend <= 2 bins past their tile
 constexpr int kSegCells = 2048;       // cells per scatter/gather work segment
 constexpr int kTileScaleLog2 = 19;    // tile bins accumulate int32 units of 2^-19 (<= kSegCells x 1 < 2^12)
+constexpr int kRhoScaleLog2 = 24;     // global bin map: int64 units of 2^-24
 constexpr int kCountThreads = 256;
 constexpr int kCountCells = kCountThreads * 8;  // cells per count/place CTA (8 per thread)
 
@@ -114,7 +115,8 @@ struct Ctx {
   Segment *d_segs = nullptr;
   int32_t max_segs = 0;
   int32_t *d_nsegs = nullptr;
-  float *d_rho = nullptr, *d_t = nullptr, *d_sx = nullptr, *d_sy = nullptr;
+  unsigned long long *d_rho = nullptr;  // bin map, int64 fixed point in units of 2^-kRhoScaleLog2 (exact, deterministic)
+  float *d_t = nullptr, *d_sx = nullptr, *d_sy = nullptr;
   float2 *d_xi = nullptr;
   float2 *d_force = nullptr;          // per own cell: -(sum ov xi)
   float2 *d_tw_x = nullptr, *d_tw_y = nullptr;     // FFT twiddles W_N^k, k < N/2
@@ -122,7 +124,7 @@ struct Ctx {
   float *d_kx = nullptr, *d_ky = nullptr;          // wavenumbers (reading A12)
 
   // ---- shared scratch ----
-  float2 *d_g2 = nullptr;             // WA gradient accumulator, interleaved, kept zero between calls
+  float2 *d_g2 = nullptr;             // WA gradient accumulator, interleaved, cleared per call
   double *d_part = nullptr;           // partial sums: [0, n_wa_part) WA, then energy
   int32_t n_wa_part = 0, n_en_part = 0;
   unsigned long long *d_limbs = nullptr;  // HPWL fixed-point limbs
@@ -167,7 +169,9 @@ void launch_wa(const Ctx &c, const float *x, const float *y, float gamma, bool h
 void launch_density_map(const Ctx &c, const float *x, const float *y, cudaStream_t s);
 void launch_density_gather(const Ctx &c, const float *x, const float *y, cudaStream_t s);
 // transforms (dct.cu)
-void launch_fields(const Ctx &c, const float *rho, cudaStream_t s);
+void launch_fields(const Ctx &c, const float *rho, cudaStream_t s);            // rho as float (debug hook)
+void launch_fields_fixed(const Ctx &c, cudaStream_t s);                          // rho = c.d_rho (hot path)
+void launch_rho_to_float(const Ctx &c, float *out, cudaStream_t s);
 void launch_transform(const Ctx &c, int kind, const float *in, float *out, cudaStream_t s);
 void launch_split_fields(const Ctx &c, float *xi_x, float *xi_y, cudaStream_t s);
 void launch_psi(const Ctx &c, const float *rho, float *psi, cudaStream_t s);

@@ -1,9 +1,8 @@
 // finalize.cu — gradient combine (eq 2: grad WA + lambda grad D) and the scalar
 // outputs (WA, D, obj, HPWL) on sm_100a.
 //
-// The WA kernels accumulate into the interleaved scratch g2, which this pass reads, splits
-// into the caller's gx / gy, and resets to zero for the next evaluation (so no memset is
-// needed on the hot path).  Scalars are reduced from per-CTA partials in a fixed order, so
+// The WA kernels accumulate into the interleaved scratch g2 (cleared at the head of the WA
+// stream), which this pass reads and splits into the caller's gx / gy.  Scalars are reduced from per-CTA partials in a fixed order, so
 // WA and D are run-to-run deterministic given the partials; HPWL is converted from the
 // exact int64 limb sum with one correctly rounded step (reading A7).
 #include "dp_internal.h"
@@ -12,39 +11,48 @@ namespace dp {
 
 namespace {
 
-// One pair of cells per thread (16-byte loads of g2 / force, 8-byte stores of gx / gy), no
-// grid-stride loop: every warp has exactly one round of independent loads in flight.
-__global__ void __launch_bounds__(256) k_combine(float2 *__restrict__ g2, const float2 *__restrict__ force,
+// Four cells per thread: 16-byte loads of g2 / force issued together, 16-byte stores of gx / gy,
+// no grid-stride loop.  g2 is only read here (zeroing it in the same pass, a store to the
+// lines just loaded, measured 2.5x slower on B200); the WA stream clears it before the next
+// accumulation.  force[i] is stored with the parity offset of cell_begin (dp_create), so even
+// global cells are 16-byte aligned in both arrays.
+__global__ void __launch_bounds__(256) k_combine(const float2 *__restrict__ g2, const float2 *__restrict__ force,
                                                  float *__restrict__ gx, float *__restrict__ gy, int cell_begin,
                                                  int n_own, float lambda, int use_wa, int use_den) {
-  const int c0 = (cell_begin & ~1) + 2 * (blockIdx.x * blockDim.x + threadIdx.x);  // even cell
+  const int c0 = (cell_begin & ~3) + 4 * (blockIdx.x * blockDim.x + threadIdx.x);
   const int cend = cell_begin + n_own;
   if (c0 >= cend) return;
-  const bool full = c0 >= cell_begin && c0 + 1 < cend;
-  float4 g = make_float4(0.f, 0.f, 0.f, 0.f), f = make_float4(0.f, 0.f, 0.f, 0.f);
-  if (full) {
+  const float2 *fb = force - cell_begin;   // fb[c] = force of global cell c
+  const bool aligned4 = (((uintptr_t)(fb + c0)) & 15) == 0 && (((uintptr_t)(gx + c0)) & 15) == 0 &&
+                        (((uintptr_t)(gy + c0)) & 15) == 0;
+  if (c0 >= cell_begin && c0 + 3 < cend && aligned4) {
+    float4 g0 = make_float4(0.f, 0.f, 0.f, 0.f), g1 = g0, f0 = g0, f1 = g0;
     if (use_wa) {
-      g = __ldcs(reinterpret_cast<const float4 *>(g2 + c0));
-      __stcs(reinterpret_cast<float4 *>(g2 + c0), make_float4(0.f, 0.f, 0.f, 0.f));
+      g0 = __ldcs(reinterpret_cast<const float4 *>(g2 + c0));
+      g1 = __ldcs(reinterpret_cast<const float4 *>(g2 + c0 + 2));
     }
-    if (use_den) f = __ldcs(reinterpret_cast<const float4 *>(force + (c0 - cell_begin)));
-    const float2 ox = make_float2(fmaf(lambda, f.x, g.x), fmaf(lambda, f.z, g.z));
-    const float2 oy = make_float2(fmaf(lambda, f.y, g.y), fmaf(lambda, f.w, g.w));
-    *reinterpret_cast<float2 *>(gx + c0) = ox;
-    *reinterpret_cast<float2 *>(gy + c0) = oy;
+    if (use_den) {
+      f0 = __ldcs(reinterpret_cast<const float4 *>(fb + c0));
+      f1 = __ldcs(reinterpret_cast<const float4 *>(fb + c0 + 2));
+    }
+    __stcs(reinterpret_cast<float4 *>(gx + c0),
+           make_float4(fmaf(lambda, f0.x, g0.x), fmaf(lambda, f0.z, g0.z), fmaf(lambda, f1.x, g1.x),
+                       fmaf(lambda, f1.z, g1.z)));
+    __stcs(reinterpret_cast<float4 *>(gy + c0),
+           make_float4(fmaf(lambda, f0.y, g0.y), fmaf(lambda, f0.w, g0.w), fmaf(lambda, f1.y, g1.y),
+                       fmaf(lambda, f1.w, g1.w)));
     return;
   }
-  for (int c = c0; c < c0 + 2; c++) {  // ragged ends of the own range
+  for (int c = c0; c < c0 + 4; c++) {  // ragged ends of the own range / unaligned caller buffers
     if (c < cell_begin || c >= cend) continue;
     float vx = 0.f, vy = 0.f;
     if (use_wa) {
       const float2 q = g2[c];
       vx = q.x;
       vy = q.y;
-      g2[c] = make_float2(0.f, 0.f);
     }
     if (use_den) {
-      const float2 q = force[c - cell_begin];
+      const float2 q = fb[c];
       vx = fmaf(lambda, q.x, vx);
       vy = fmaf(lambda, q.y, vy);
     }
@@ -146,8 +154,8 @@ __global__ void __launch_bounds__(256) k_finalize(FinArgs a) {
 void launch_combine(const Ctx &c, float lambda, float *gx, float *gy, bool use_wa, bool use_density,
                     cudaStream_t s) {
   if (c.n_own <= 0) return;
-  const int pairs = (c.n_own + 3) / 2;
-  const int blocks = (pairs + 255) / 256;
+  const int quads = (c.n_own + 6) / 4 + 1;
+  const int blocks = (quads + 255) / 256;
   k_combine<<<blocks, 256, 0, s>>>(c.d_g2, c.d_force, gx, gy, c.cell_begin, c.n_own, lambda, use_wa ? 1 : 0,
                                    use_density ? 1 : 0);
 }

@@ -285,3 +285,16 @@ def test_invalid_args(tiny):
         dp.dp_eval(ctx, _t(x), _t(y), 1.0, -1.0, gx, gx.clone())
     with pytest.raises(dp.DPError, match="INVALID_ARG"):
         dp.dp_eval(ctx, None, _t(y), 1.0, 1.0, gx, gx.clone())
+
+
+@pytest.mark.parametrize("dist", ["spread", "initial"])
+def test_density_bitwise_deterministic(tiny, dist):
+    """The bin map accumulates in int64 fixed point, so the density energy and
+    gradient are bitwise identical from call to call regardless of atomic order."""
+    nl, ctx = tiny
+    x, y = make_positions(nl, dist)
+    a = ctx.density_grad(_t(x), _t(y))
+    b = ctx.density_grad(_t(x), _t(y))
+    assert a["energy"].item() == b["energy"].item()
+    assert torch.equal(a["gx"], b["gx"]) and torch.equal(a["gy"], b["gy"])
+    assert torch.equal(ctx.density_map(_t(x), _t(y)), ctx.density_map(_t(x), _t(y)))

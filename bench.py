@@ -9,8 +9,10 @@ force gather, combine) on the bigblue4-shaped synthetic workload (2.18M cells, 2
 
 N > 1 is launched by torchrun (one rank per GPU, NCCL): the evaluation is sharded by cells
 (owner computes) with one ncclAllReduce of the bin map per step, so the total
-work per step is fixed ("scaling": "strong").  Device time: CUDA events around every step on
-the launching stream, L2 flushed (a 2x L2 write) before every timed step, max over ranks.
+work per step is fixed ("scaling": "strong").  Device time: one CUDA event pair around the K
+timed steps on the launching stream (barrier + synchronize on both sides), max over ranks; the
+per-step working set (~280 MB) exceeds L2, so no flush is inserted (the contract's "inputs larger
+than L2"); an L2-flushed per-step time is reported beside it.
 Rank 0 prints one JSON line.  --impl reference times the fp64 CPU oracle (the reference arm of
 this tier) on a bounded sample of the same workload.
 """
@@ -132,7 +134,8 @@ def workload_config(nl, dist_name, world):
             "cells": nl.num_cells, "nets": nl.num_nets, "pins": nl.num_pins,
             "bins": [nl.bins_x, nl.bins_y], "positions": dist_name, "gamma": nl.bin_w, "lambda": 1.0,
             "hpwl": "not fused (d_hpwl = NULL)",
-            "l2": "flushed before every timed step (write of 2x L2 bytes, untimed)",
+            "l2": "not flushed: per-step working set ~280 MB > 126 MB L2 (inputs larger than L2); "
+                  "l2_flushed_ms_per_step = same step after an untimed 2x-L2 write",
             "parallelism": f"cells{world} (owner-computes shards, NCCL all-reduce of the bin map)"
                            if world > 1 else "single GPU"}
 
@@ -262,34 +265,37 @@ def run_ours(args, rank, world, local_rank):
         pg.barrier()
     assert all(math.isfinite(v) for v in sc[:3].tolist()), "non-finite objective"
     K = args.steps
-    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(K)]
+    # headline: K back-to-back steps bracketed by one event pair (barrier + sync on both sides).
+    # The per-step working set (pins 107 MB, nets 9 MB, cells 35 MB, sort records 61 MB, maps
+    # and scratch ~65 MB at bigblue4) exceeds the 126 MB L2, so no flush is inserted.
     dp.dp_profile_enable(ctx, True)
     torch.cuda.synchronize()
     if pg:
         pg.barrier()
     t0 = time.time()
-    for k in range(K):
-        flush.zero_()
-        ev[k][0].record(stream)
+    h0, h1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    h0.record(stream)
+    for _ in range(K):
         step()
-        ev[k][1].record(stream)
+    h1.record(stream)
     torch.cuda.synchronize()
     t1 = time.time()
     if pg:
         pg.barrier()
     dp.dp_profile_enable(ctx, False)
     stage_ms, n_prof = dp.dp_profile_read(ctx)
-    total_ms = sum(a.elapsed_time(b) for a, b in ev)
+    total_ms = h0.elapsed_time(h1)
     clocks = sampler.summary(t0, t1)
-    # hot (L2-warm, back-to-back) variant, secondary
-    Kh = min(K, 500)
-    h0, h1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    h0.record(stream)
-    for _ in range(Kh):
+    # secondary: L2 flushed (2x L2 bytes written, untimed) before every timed step
+    Kf = min(K, 200)
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(Kf)]
+    for k in range(Kf):
+        flush.zero_()
+        ev[k][0].record(stream)
         step()
-    h1.record(stream)
+        ev[k][1].record(stream)
     torch.cuda.synchronize()
-    hot_ms = h0.elapsed_time(h1) / Kh
+    flushed_ms = sum(a.elapsed_time(b) for a, b in ev) / Kf
     # e2e through the public API on pinned host buffers (H2D x, y; D2H gx, gy, scalars)
     hx = torch.as_tensor(x).pin_memory()
     hy = torch.as_tensor(y).pin_memory()
@@ -307,10 +313,10 @@ def run_ours(args, rank, world, local_rank):
     e2e_s = time.perf_counter() - e0
     sampler.stop()
 
-    tensors = torch.tensor([total_ms, e2e_s, hot_ms], dtype=torch.float64, device=dev)
+    tensors = torch.tensor([total_ms, e2e_s, flushed_ms], dtype=torch.float64, device=dev)
     if pg:
         pg.all_reduce(tensors, op=pg.ReduceOp.MAX)
-    total_ms, e2e_s, hot_ms = tensors.tolist()
+    total_ms, e2e_s, flushed_ms = tensors.tolist()
     if rank != 0:
         if pg:
             pg.destroy_process_group()
@@ -330,7 +336,7 @@ def run_ours(args, rank, world, local_rank):
         except Exception:
             traffic = None
     cfg = workload_config(nl, args.dist, world)
-    cfg["hot_ms_per_step"] = hot_ms
+    cfg["l2_flushed_ms_per_step"] = flushed_ms
     cfg["peak_source"] = peak_src
     out = {
         "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": K, "warmup": args.warmup,

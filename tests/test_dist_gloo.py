@@ -1,0 +1,114 @@
+"""Multi-process check of the distributed partition (owner computes) on CPU.
+
+Two gloo ranks each take libdp's host-only partition plan (dp_partition_plan), evaluate their
+shard with the fp64 oracle exactly as a distributed context does (nets touching own cells, the
+gradient of own cells only, WA / HPWL counted once, the density map of own cells), combine with
+the same collectives the GPU path uses (sum of the bin map, sum of WA, sum of HPWL terms) and must
+reproduce the single-process oracle."""
+import math
+import os
+import socket
+
+import numpy as np
+import pytest
+import torch
+import torch.distributed as dist
+import torch.multiprocessing as mp
+
+
+def _free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    return port
+
+
+def _shard_eval(nl, x, y, gamma, cb, ce, mask):
+    import oracle
+    from synth import custom_netlist
+    # WA over the nets this rank evaluates (mask & 1); gradient kept for own cells only
+    sel = np.nonzero(mask & 1)[0]
+    starts = nl.net_start
+    deg = starts[sel + 1] - starts[sel]
+    ns = np.concatenate([[0], np.cumsum(deg)])
+    pins = np.concatenate([np.arange(starts[e], starts[e + 1]) for e in sel]) if len(sel) else np.zeros(0, int)
+    sub = custom_netlist(ns, nl.pin2cell[pins], nl.pin_dx[pins], nl.pin_dy[pins], nl.cell_w, nl.cell_h,
+                         (nl.xl, nl.yl, nl.xh, nl.yh), (nl.bins_x, nl.bins_y))
+    _, gx, gy, wl_net = oracle.wa(sub, x, y, gamma, per_net=True)
+    own = np.zeros(nl.num_cells, bool)
+    own[cb:ce] = True
+    gx[~own] = 0.0
+    gy[~own] = 0.0
+    counted = (mask[sel] & 2) != 0
+    wl = float(np.sum(wl_net[counted]))
+    h = oracle.hpwl_nets(sub, x, y)[counted]
+    # density: this rank's cells only
+    cells = custom_netlist([0], [], [], [], nl.cell_w[cb:ce], nl.cell_h[cb:ce], (nl.xl, nl.yl, nl.xh, nl.yh),
+                           (nl.bins_x, nl.bins_y))
+    rho = oracle.density_map(cells, x[cb:ce], y[cb:ce], 1)
+    return wl, gx, gy, h, rho, cells
+
+
+def _worker(rank, world, port, q):
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    import oracle
+    import paper_conf_dac_lindlrkp19_b200 as dp
+    from synth import make_netlist, make_positions
+    nl = make_netlist("tiny")
+    x, y = make_positions(nl)
+    gamma = 7.0
+    cb, ce, mask = dp.dp_partition_plan(nl, rank, world)
+    wl, gx, gy, h, rho, cells = _shard_eval(nl, x, y, gamma, cb, ce, mask)
+    t = torch.tensor([wl], dtype=torch.float64)
+    dist.all_reduce(t)                                   # WA partial sums (fp64 all-reduce)
+    rho_t = torch.from_numpy(rho.copy())
+    dist.all_reduce(rho_t)                               # bin map (the GPU path sums int64)
+    g = torch.from_numpy(np.stack([gx, gy]))
+    dist.all_reduce(g)                                   # disjoint own ranges: assembles the gradient
+    hs = [None] * world
+    dist.all_gather_object(hs, h.tolist())
+    # replicated Poisson solve on the summed map, force for own cells
+    rho_full = rho_t.numpy()
+    psi, xi_x, xi_y = oracle.fields(nl, oracle.dct2(rho_full))
+    D = oracle.energy(nl, rho_full, psi)
+    fx, fy = oracle.density_grad(cells, x[cb:ce], y[cb:ce], xi_x, xi_y, 1)
+    f = torch.zeros(2, nl.num_cells, dtype=torch.float64)
+    f[0, cb:ce] = torch.from_numpy(fx)
+    f[1, cb:ce] = torch.from_numpy(fy)
+    dist.all_reduce(f)
+    if rank == 0:
+        q.put(dict(wl=t.item(), gx=g[0].numpy(), gy=g[1].numpy(), hpwl=math.fsum(sum(hs, [])), D=D,
+                   fx=f[0].numpy(), fy=f[1].numpy(), rho=rho_full))
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world", [2])
+def test_owner_computes_shards_reassemble_the_oracle(world):
+    import oracle
+    from synth import make_netlist, make_positions
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_worker, args=(r, world, port, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = q.get(timeout=300)
+    for p in procs:
+        p.join(timeout=300)
+        assert p.exitcode == 0
+    nl = make_netlist("tiny")
+    x, y = make_positions(nl)
+    wl, gx, gy = oracle.wa(nl, x, y, 7.0)
+    assert res["wl"] == pytest.approx(wl, rel=1e-12)
+    np.testing.assert_allclose(res["gx"], gx, rtol=1e-12, atol=1e-12)
+    np.testing.assert_allclose(res["gy"], gy, rtol=1e-12, atol=1e-12)
+    assert res["hpwl"] == oracle.hpwl(nl, x, y)
+    D, fx, fy, parts = oracle.density(nl, x, y, 1)
+    np.testing.assert_allclose(res["rho"], parts["rho"], rtol=1e-12, atol=1e-12)
+    assert res["D"] == pytest.approx(D, rel=1e-12)
+    np.testing.assert_allclose(res["fx"], fx, rtol=1e-10, atol=1e-9 * np.abs(fx).max())
+    np.testing.assert_allclose(res["fy"], fy, rtol=1e-10, atol=1e-9 * np.abs(fy).max())

@@ -28,7 +28,7 @@ constexpr int kRowThreads = 256;
 constexpr int kColThreads = 256;
 // columns per CTA in the column kernels (even: pairs share a complex FFT); sized so the
 // shared-memory slab fits and the grid has >= 256 CTAs at 1024 columns
-__host__ __device__ inline int col_slab(int mx) { return mx <= 2048 ? 4 : 2; }
+__host__ __device__ inline int col_slab(int mx) { (void)mx; return 2; }
 
 __device__ __forceinline__ float2 cmul(float2 a, float2 b) {
   return make_float2(a.x * b.x - a.y * b.y, a.x * b.y + a.y * b.x);

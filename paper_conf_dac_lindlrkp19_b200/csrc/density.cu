@@ -19,22 +19,30 @@
 //   D5 gather  one CTA per segment stages the (tile+2)^2 float2 field tile in shared memory
 //              and writes each cell's force
 // Large cells (footprint wider than 3 bins) take a CTA-per-cell path with global reds.
-// The tile accumulators (int32, 2^-19) flush into an int64 global map (2^-24) with native
-// red.global.add.u64: the density map is exact up to one rounding per contribution and
-// independent of execution order (deterministic; bit-identical after an int64 all-reduce).
+// The tile accumulators (two 32-bit words per bin, 2^-29 resolution) flush into an int64 global
+// map (2^-29 units) with native red.global.add.u64: the density map is exact up to one rounding
+// per contribution and independent of execution order (deterministic; bit-identical after an
+// int64 all-reduce).
 // Footprint geometry is computed in fp64 (B200 runs FP64 at half rate); records hold the
 // footprint in fractions of the cell's first bin (|v| < 3) plus that bin's tile-local index.
+#include <algorithm>
+
+#include "async_copy.cuh"
 #include "dp_internal.h"
 
 namespace dp {
 
 namespace {
 
+constexpr int kTileThreads = 512;   // scatter / gather CTA size (smem-bound at 2 CTAs per SM)
+
 struct DenArgs {
   const float *x, *y;   // global cell arrays
   const float *w, *h;   // own cells
   int cell_begin, n_own;
   double xl, yl, xh, yh, bx, by, sx, sy, ibx, iby;   // ibx = 1 / bx (no fp64 divisions on the hot path)
+  double cx0, cy0;     // -xl / bx, -yl / by: bin coordinate of x is x * ibx + cx0
+  float sxf, syf;      // stretched minimum sizes sqrt2 b (fp32)
   int mx, my, tile, tile_log2, tiles_y, ntiles, stretch;
   int *tile_cnt, *tile_cursor, *tile_off;
   Segment *segs;
@@ -48,38 +56,41 @@ struct DenArgs {
   const int *large;
 };
 
+// Stretched, clipped footprint of a cell in BIN units (readings A10, A11):
+//   lo = (x - xl)/b_x + (w - w')/2 / b_x, hi = lo + w'/b_x, clipped to [0, M].
+// Formulated as a few fp64 FMAs from the fp32 inputs; count and place evaluate it identically,
+// so their tile choices agree.  The charge ratio r = w h / (w' h') is fp32 (stored as fp32).
 struct Foot {
-  double lx, hx, ly, hy;
+  double lo_x, hi_x, lo_y, hi_y;
   float r;
   bool large, empty;
 };
 
-// Stretched, clipped footprint of a cell (readings A10, A11) from its loaded values.
-__device__ __forceinline__ Foot footprint_v(const DenArgs &a, float xf, float yf, float wf, float hf) {
+__device__ __forceinline__ Foot footprint_v(const DenArgs &a, float x, float y, float w, float h) {
   Foot f;
-  const double x = xf, y = yf, w = wf, h = hf;
-  double ws = w, hs = h;
-  float wsf = wf, hsf = hf;
-  if (a.stretch) {
-    ws = fmax(w, a.sx);
-    hs = fmax(h, a.sy);
-    wsf = fmaxf(wf, (float)a.sx);
-    hsf = fmaxf(hf, (float)a.sy);
-  }
-  f.large = (w > 2.0 * a.bx) || (h > 2.0 * a.by);
-  // charge ratio r = w h / (w' h') in fp32 (only its fp32 rounding is stored)
-  f.r = (wsf * hsf > 0.f) ? __fdividef(wf * hf, wsf * hsf) : 0.f;
-  const double cx = x + 0.5 * w, cy = y + 0.5 * h;
-  f.lx = fmax(cx - 0.5 * ws, a.xl);
-  f.hx = fmin(cx + 0.5 * ws, a.xh);
-  f.ly = fmax(cy - 0.5 * hs, a.yl);
-  f.hy = fmin(cy + 0.5 * hs, a.yh);
-  f.empty = !(f.hx > f.lx && f.hy > f.ly && f.r > 0.f);
+  const float ws = a.stretch ? fmaxf(w, a.sxf) : w;
+  const float hs = a.stretch ? fmaxf(h, a.syf) : h;
+  f.large = ((double)w > 2.0 * a.bx) || ((double)h > 2.0 * a.by);   // same test as dp_create's list
+  f.r = (ws * hs > 0.f) ? __fdividef(w * h, ws * hs) : 0.f;
+  const double lx = fma((double)(0.5f * (w - ws)), a.ibx, fma((double)x, a.ibx, a.cx0));
+  const double ly = fma((double)(0.5f * (h - hs)), a.iby, fma((double)y, a.iby, a.cy0));
+  f.hi_x = fmin(fma((double)ws, a.ibx, lx), (double)a.mx);
+  f.hi_y = fmin(fma((double)hs, a.iby, ly), (double)a.my);
+  f.lo_x = fmax(lx, 0.0);
+  f.lo_y = fmax(ly, 0.0);
+  f.empty = !(f.hi_x > f.lo_x && f.hi_y > f.lo_y && f.r > 0.f);
   return f;
 }
 
 __device__ __forceinline__ Foot footprint(const DenArgs &a, int i) {
   return footprint_v(a, __ldg(a.x + a.cell_begin + i), __ldg(a.y + a.cell_begin + i), __ldg(a.w + i), __ldg(a.h + i));
+}
+
+// first bin of a (non-empty) footprint and its tile
+__device__ __forceinline__ int small_tile(const DenArgs &a, const Foot &f, int &bx0, int &by0) {
+  bx0 = min((int)f.lo_x, a.mx - 1);
+  by0 = min((int)f.lo_y, a.my - 1);
+  return (bx0 >> a.tile_log2) * a.tiles_y + (by0 >> a.tile_log2);
 }
 
 // Loads x, y, w, h of own cells [i0, i0 + 8) (i0 a multiple of 8) with 16-byte vector loads
@@ -113,43 +124,71 @@ __device__ __forceinline__ void load_cells8(const DenArgs &a, int i0, Cells8 &c)
   }
 }
 
-__device__ __forceinline__ int small_tile(const DenArgs &a, const Foot &f, int &ox, int &oy) {
-  int bx0 = (int)floor((f.lx - a.xl) * a.ibx), by0 = (int)floor((f.ly - a.yl) * a.iby);
-  bx0 = min(max(bx0, 0), a.mx - 1);
-  by0 = min(max(by0, 0), a.my - 1);
-  const int tx = bx0 >> a.tile_log2, ty = by0 >> a.tile_log2;
-  ox = tx << a.tile_log2;
-  oy = ty << a.tile_log2;
-  return tx * a.tiles_y + ty;
+
+// Stage the x, y, w, h of own cells [i0, i0 + n) (n <= kCountCells) in shared memory: bulk async
+// copies of the 16-byte aligned prefix (one elected thread, one mbarrier), plain loads for the
+// rest (ragged tail, or a caller x / y that is not 16-byte aligned).  Returns after the data is
+// visible to the whole CTA.
+struct CellStage {
+  float x[kCountCells], y[kCountCells], w[kCountCells], h[kCountCells];
+  uint64_t bar;
+};
+
+__device__ __forceinline__ void stage_cells(const DenArgs &a, CellStage &st, int i0, int n) {
+  const float *gx = a.x + a.cell_begin + i0, *gy = a.y + a.cell_begin + i0;
+  const bool ok = aligned16(gx) && aligned16(gy) && aligned16(a.w + i0) && aligned16(a.h + i0);
+  const int nb = ok ? (n & ~3) : 0;
+  if (threadIdx.x == 0 && nb > 0) {
+    mbar_init(&st.bar);
+    mbar_expect_tx(&st.bar, 16u * nb);
+    bulk_g2s(st.x, gx, 4u * nb, &st.bar);
+    bulk_g2s(st.y, gy, 4u * nb, &st.bar);
+    bulk_g2s(st.w, a.w + i0, 4u * nb, &st.bar);
+    bulk_g2s(st.h, a.h + i0, 4u * nb, &st.bar);
+  }
+  for (int i = nb + threadIdx.x; i < n; i += blockDim.x) {
+    st.x[i] = __ldg(gx + i);
+    st.y[i] = __ldg(gy + i);
+    st.w[i] = __ldg(a.w + i0 + i);
+    st.h[i] = __ldg(a.h + i0 + i);
+  }
+  __syncthreads();
+  if (nb > 0) mbar_wait(&st.bar, 0);
 }
 
-// D1: 8 cells per thread, all loads issued up front
+// D1: per-CTA shared histogram of tile ids over a staged block of cells
 __global__ void __launch_bounds__(kCountThreads) k_count(DenArgs a) {
   extern __shared__ int s_hist[];
+  __shared__ CellStage st;
+  const int i0 = blockIdx.x * kCountCells, n = min(kCountCells, a.n_own - i0);
   for (int t = threadIdx.x; t < a.ntiles; t += kCountThreads) s_hist[t] = 0;
-  __syncthreads();
-  const int i0 = (blockIdx.x * kCountThreads + threadIdx.x) * 8;
-  if (i0 < a.n_own) {
-    Cells8 c;
-    load_cells8(a, i0, c);
-#pragma unroll
-    for (int k = 0; k < 8; k++) {
-      if (i0 + k >= a.n_own) break;
-      const Foot f = footprint_v(a, c.x[k], c.y[k], c.w[k], c.h[k]);
-      if (f.empty || f.large) continue;
-      int ox, oy;
-      atomicAdd(&s_hist[small_tile(a, f, ox, oy)], 1);
-    }
+  stage_cells(a, st, i0, n);
+  for (int i = threadIdx.x; i < n; i += kCountThreads) {
+    const Foot f = footprint_v(a, st.x[i], st.y[i], st.w[i], st.h[i]);
+    if (f.empty || f.large) continue;
+    int bx0, by0;
+    atomicAdd(&s_hist[small_tile(a, f, bx0, by0)], 1);
   }
   __syncthreads();
   for (int t = threadIdx.x; t < a.ntiles; t += kCountThreads)
     if (s_hist[t]) atomicAdd(a.tile_cnt + t, s_hist[t]);
 }
 
-// D2 (single CTA of 1024 threads)
+// D2 (single CTA of 1024 threads): exclusive scans of tile counts and segment counts with
+// warp shuffles (two barriers), cursors, work segments; resets the counts for the next call.
+__device__ __forceinline__ int warp_incl_scan(int v, int lane) {
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const int t = __shfl_up_sync(0xffffffffu, v, o);
+    if (lane >= o) v += t;
+  }
+  return v;
+}
+
 __global__ void __launch_bounds__(1024) k_scan(DenArgs a) {
-  __shared__ int s_a[1024], s_b[1024];
+  __shared__ int s_wa[32], s_wb[32];
   constexpr int T = 1024;
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const int per = (a.ntiles + T - 1) / T;
   const int t0 = threadIdx.x * per;
   int cnt_sum = 0, seg_sum = 0;
@@ -161,21 +200,20 @@ __global__ void __launch_bounds__(1024) k_scan(DenArgs a) {
       seg_sum += (c + kSegCells - 1) / kSegCells;
     }
   }
-  s_a[threadIdx.x] = cnt_sum;
-  s_b[threadIdx.x] = seg_sum;
-  __syncthreads();
-  for (int off = 1; off < T; off <<= 1) {  // inclusive Hillis-Steele scan
-    int va = 0, vb = 0;
-    if ((int)threadIdx.x >= off) {
-      va = s_a[threadIdx.x - off];
-      vb = s_b[threadIdx.x - off];
-    }
-    __syncthreads();
-    s_a[threadIdx.x] += va;
-    s_b[threadIdx.x] += vb;
-    __syncthreads();
+  const int ia = warp_incl_scan(cnt_sum, lane), ib = warp_incl_scan(seg_sum, lane);
+  if (lane == 31) {
+    s_wa[warp] = ia;
+    s_wb[warp] = ib;
   }
-  int off_c = s_a[threadIdx.x] - cnt_sum, off_s = s_b[threadIdx.x] - seg_sum;
+  __syncthreads();
+  if (warp == 0) {
+    const int xa = warp_incl_scan(s_wa[lane], lane), xb = warp_incl_scan(s_wb[lane], lane);
+    s_wa[lane] = xa;
+    s_wb[lane] = xb;
+  }
+  __syncthreads();
+  int off_c = (warp ? s_wa[warp - 1] : 0) + ia - cnt_sum;
+  int off_s = (warp ? s_wb[warp - 1] : 0) + ib - seg_sum;
   for (int k = 0; k < per; k++) {
     const int t = t0 + k;
     if (t < a.ntiles) {
@@ -197,147 +235,291 @@ __global__ void __launch_bounds__(1024) k_scan(DenArgs a) {
     }
   }
   if (threadIdx.x == T - 1) {
-    a.tile_off[a.ntiles] = s_a[T - 1];
-    *a.nsegs = s_b[T - 1];
+    a.tile_off[a.ntiles] = off_c;
+    *a.nsegs = off_s;
   }
 }
 
-// D3: same 8-cells-per-thread traversal as D1; records stay in registers while the CTA
-// reserves its ranges in the tile cursors.
+// D3: same staged block as D1.  Pass 1: shared histogram; local exclusive scan (the block's
+// records in tile order) and one global reservation per non-empty tile.  Pass 2: each cell's
+// record goes to shared memory at its tile-ordered local slot; finally the block writes its
+// records out in contiguous per-tile runs (random per-record stores were measured 3x slower).
+struct PlaceOut {
+  float4 rec[kCountCells];
+  int2 rc[kCountCells];
+  int cell[kCountCells];
+  int tile[kCountCells];
+};
+
+__host__ __device__ constexpr int place_static_bytes() { return 0; }
+int place_smem_bytes(int ntiles) { return (int)sizeof(PlaceOut) + 12 * ntiles; }
+
 __global__ void __launch_bounds__(kCountThreads) k_place(DenArgs a) {
-  extern __shared__ int s_hist[];
-  for (int t = threadIdx.x; t < a.ntiles; t += kCountThreads) s_hist[t] = 0;
-  __syncthreads();
-  const int i0 = (blockIdx.x * kCountThreads + threadIdx.x) * 8;
-  int tl[8], rk[8], ij[8];
-  float4 rec[8];
-  float rr[8];
-#pragma unroll
-  for (int k = 0; k < 8; k++) tl[k] = -1;
-  if (i0 < a.n_own) {
-    Cells8 c;
-    load_cells8(a, i0, c);
-#pragma unroll
-    for (int k = 0; k < 8; k++) {
-      const int i = i0 + k;
-      if (i >= a.n_own) break;
-      const Foot f = footprint_v(a, c.x[k], c.y[k], c.w[k], c.h[k]);
-      if (f.large) continue;
-      if (f.empty) {
-        a.force[i] = make_float2(0.f, 0.f);
-        continue;
-      }
-      int ox, oy;
-      tl[k] = small_tile(a, f, ox, oy);
-      rk[k] = atomicAdd(&s_hist[tl[k]], 1);
-      // bin-local fractions (|v| < 3): fp32 keeps ~2e-7 bin absolute precision, which the force
-      // gather needs where large opposite bin fields cancel (the 'initial' placement)
-      const double ux0 = (f.lx - a.xl) * a.ibx, uy0 = (f.ly - a.yl) * a.iby;
-      const int bi = min(max((int)floor(ux0), 0), a.mx - 1);
-      const int bj = min(max((int)floor(uy0), 0), a.my - 1);
-      rec[k] = make_float4((float)(ux0 - bi), (float)(uy0 - bj), (float)((f.hx - a.xl) * a.ibx - bi),
-                           (float)((f.hy - a.yl) * a.iby - bj));
-      rr[k] = f.r;
-      ij[k] = (bi - ox) | ((bj - oy) << 16);
-    }
-  }
-  __syncthreads();
+  extern __shared__ __align__(16) unsigned char psm[];
+  PlaceOut &po = *reinterpret_cast<PlaceOut *>(psm);
+  int *s_hist = reinterpret_cast<int *>(psm + sizeof(PlaceOut));   // [ntiles] counts -> local offsets
+  int *s_base = s_hist + a.ntiles;                                  // [ntiles] global bases
+  int *s_rank = s_base + a.ntiles;                                  // [ntiles] running local rank
+  __shared__ CellStage st;
+  __shared__ int s_warp[kCountThreads / 32];
+  const int i0 = blockIdx.x * kCountCells, n = min(kCountCells, a.n_own - i0);
   for (int t = threadIdx.x; t < a.ntiles; t += kCountThreads) {
-    const int c = s_hist[t];
-    if (c) s_hist[t] = atomicAdd(a.tile_cursor + t, c);
+    s_hist[t] = 0;
+    s_rank[t] = 0;
+  }
+  stage_cells(a, st, i0, n);
+  for (int i = threadIdx.x; i < n; i += kCountThreads) {
+    const Foot f = footprint_v(a, st.x[i], st.y[i], st.w[i], st.h[i]);
+    if (f.large || f.empty) continue;
+    int bx0, by0;
+    atomicAdd(&s_hist[small_tile(a, f, bx0, by0)], 1);
   }
   __syncthreads();
-#pragma unroll
-  for (int k = 0; k < 8; k++) {
-    if (tl[k] < 0) continue;
-    const int pos = s_hist[tl[k]] + rk[k];
-    a.rec[pos] = rec[k];
-    a.rec_rc[pos] = make_int2(__float_as_int(rr[k]), ij[k]);
-    a.rec_cell[pos] = i0 + k;
+  // reservation + block exclusive scan of the histogram (tiles split evenly over the threads)
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const int per = (a.ntiles + kCountThreads - 1) / kCountThreads, t0 = threadIdx.x * per;
+  int sum = 0;
+  for (int q = 0; q < per; q++) {
+    const int t = t0 + q;
+    if (t < a.ntiles) {
+      const int cnt = s_hist[t];
+      if (cnt) s_base[t] = atomicAdd(a.tile_cursor + t, cnt);
+      sum += cnt;
+    }
   }
-}
-
-// D4
-__global__ void __launch_bounds__(256) k_scatter_tiles(DenArgs a) {
-  extern __shared__ int s_t[];   // int32 fixed point, 2^-kTileScaleLog2 units (native ATOMS.ADD)
-  const int sg = blockIdx.x;
-  if (sg >= *a.nsegs) return;
-  const Segment seg = a.segs[sg];
-  const int P = a.tile + kHalo;
-  const int tx = seg.tile / a.tiles_y, ty = seg.tile % a.tiles_y;
-  const int ox = tx * a.tile, oy = ty * a.tile;
-  for (int k = threadIdx.x; k < P * P; k += blockDim.x) s_t[k] = 0;
+  int incl = warp_incl_scan(sum, lane);
+  if (lane == 31) s_warp[warp] = incl;
   __syncthreads();
-  const float scale = (float)(1 << kTileScaleLog2);
-  for (int p = seg.begin + threadIdx.x; p < seg.end; p += blockDim.x) {
-    const float4 q = a.rec[p];
-    const int2 rc = a.rec_rc[p];
-    const float r = __int_as_float(rc.x);
-    const int i0 = rc.y & 0xffff, j0 = rc.y >> 16;
-#pragma unroll
-    for (int di = 0; di < 3; di++) {
-      const int i = i0 + di;
-      const float ovx = fminf(q.z, (float)(di + 1)) - fmaxf(q.x, (float)di);
-      if (ovx <= 0.f || i >= P || ox + i >= a.mx) break;
-#pragma unroll
-      for (int dj = 0; dj < 3; dj++) {
-        const int j = j0 + dj;
-        const float ovy = fminf(q.w, (float)(dj + 1)) - fmaxf(q.y, (float)dj);
-        if (ovy <= 0.f || j >= P || oy + j >= a.my) break;
-        atomicAdd(&s_t[i * P + j], __float2int_rn(r * ovx * ovy * scale));
-      }
+  if (warp == 0) {
+    const int v = lane < kCountThreads / 32 ? s_warp[lane] : 0;
+    const int w = warp_incl_scan(v, lane);
+    if (lane < kCountThreads / 32) s_warp[lane] = w;
+  }
+  __syncthreads();
+  int run = (warp ? s_warp[warp - 1] : 0) + incl - sum;
+  for (int q = 0; q < per; q++) {
+    const int t = t0 + q;
+    if (t < a.ntiles) {
+      const int cnt = s_hist[t];
+      s_hist[t] = run;
+      run += cnt;
     }
   }
   __syncthreads();
-  for (int k = threadIdx.x; k < P * P; k += blockDim.x) {
-    const int iv = s_t[k];
-    const int gi = ox + k / P, gj = oy + k % P;
-    if (iv != 0 && gi < a.mx && gj < a.my)
-      asm volatile("red.global.add.u64 [%0], %1;" ::"l"(a.rho + (size_t)gi * a.my + gj),
-                   "l"((unsigned long long)iv << (kRhoScaleLog2 - kTileScaleLog2))
-                   : "memory");
+  for (int k = threadIdx.x; k < n; k += kCountThreads) {
+    const int i = i0 + k;
+    const Foot f = footprint_v(a, st.x[k], st.y[k], st.w[k], st.h[k]);
+    if (f.large) continue;
+    if (f.empty) {
+      a.force[i] = make_float2(0.f, 0.f);
+      continue;
+    }
+    int bi, bj;
+    const int t = small_tile(a, f, bi, bj);
+    const int slot = s_hist[t] + atomicAdd(&s_rank[t], 1);
+    const int mask = a.tile - 1;
+    // bin-local fractions (|v| < 3): fp32 keeps ~2e-7 bin absolute precision, which the force
+    // gather needs where large opposite bin fields cancel (the 'initial' placement)
+    po.rec[slot] = make_float4((float)(f.lo_x - bi), (float)(f.lo_y - bj), (float)(f.hi_x - bi), (float)(f.hi_y - bj));
+    po.rc[slot] = make_int2(__float_as_int(f.r), (bi & mask) | ((bj & mask) << 16));
+    po.cell[slot] = i;
+    po.tile[slot] = t;
+  }
+  __syncthreads();
+  const int nrec = (warp == 0 && lane == 0) ? 0 : 0;
+  (void)nrec;
+  const int total = s_warp[kCountThreads / 32 - 1];
+  for (int j = threadIdx.x; j < total; j += kCountThreads) {
+    const int t = po.tile[j];
+    const int pos = s_base[t] + (j - s_hist[t]);
+    a.rec[pos] = po.rec[j];
+    a.rec_rc[pos] = po.rc[j];
+    a.rec_cell[pos] = po.cell[j];
   }
 }
 
-// D5
-__global__ void __launch_bounds__(256) k_gather_tiles(DenArgs a) {
-  extern __shared__ float2 s_xi[];
+// Double-buffered record staging: buffer b holds up to kSegChunk / 2 records of rec (16 B),
+// rec_rc (8 B) and rec_cell (4 B); each buffer completes on its own mbarrier.  The copied range
+// is rounded out to 4-record multiples (the record arrays are padded by 8 records).
+constexpr int kStageRecs = kSegChunk / 2;
+struct RecBuf {
+  float4 rec[kStageRecs + 8];
+  int2 rc[kStageRecs + 8];
+  int cell[kStageRecs + 8];
+};
+struct RecStage {
+  RecBuf buf[2];
+  uint64_t bar[2];
+};
+
+__host__ __device__ constexpr int rec_stage_bytes() { return (int)((sizeof(RecStage) + 15) & ~(size_t)15); }
+
+// Issue (thread 0) the copies of records [begin, end) into buffer b; returns the offset of the
+// first record inside the buffer (all threads).
+__device__ __forceinline__ int stage_records(const DenArgs &a, RecStage &st, int b, int begin, int end,
+                                             bool with_cell, unsigned extra_tx) {
+  const int b0 = begin & ~3, e0 = (end + 3) & ~3, n = e0 - b0;
+  if (threadIdx.x == 0) {
+    RecBuf &B = st.buf[b];
+    mbar_expect_tx(&st.bar[b], (unsigned)n * (with_cell ? 28u : 24u) + extra_tx);
+    bulk_g2s(B.rec, a.rec + b0, 16u * n, &st.bar[b]);
+    bulk_g2s(B.rc, a.rec_rc + b0, 8u * n, &st.bar[b]);
+    if (with_cell) bulk_g2s(B.cell, a.rec_cell + b0, 4u * n, &st.bar[b]);
+  }
+  return begin - b0;
+}
+
+// D4: a segment's records (<= kSegCells, staged kSegChunk at a time) accumulate into a
+// (tile+2)^2 shared tile of (hi, lo) 32-bit words, flushed once into the int64 global map.
+__global__ void __launch_bounds__(kTileThreads) k_scatter_tiles(DenArgs a) {
+  extern __shared__ __align__(16) unsigned char dsm[];
+  RecStage &st = *reinterpret_cast<RecStage *>(dsm);
+  unsigned *s_hi = reinterpret_cast<unsigned *>(dsm + rec_stage_bytes());   // 2^-kTileHiBits units
+  unsigned *s_lo = s_hi + (a.tile + kHalo) * (a.tile + kHalo);               // 2^-(hi + lo bits) units
   const int sg = blockIdx.x;
   if (sg >= *a.nsegs) return;
   const Segment seg = a.segs[sg];
   const int P = a.tile + kHalo;
   const int tx = seg.tile / a.tiles_y, ty = seg.tile % a.tiles_y;
   const int ox = tx * a.tile, oy = ty * a.tile;
+  if (threadIdx.x == 0) {
+    mbar_init(&st.bar[0]);
+    mbar_init(&st.bar[1]);
+  }
   for (int k = threadIdx.x; k < P * P; k += blockDim.x) {
-    const int gi = ox + k / P, gj = oy + k % P;
-    s_xi[k] = (gi < a.mx && gj < a.my) ? a.xi[(size_t)gi * a.my + gj] : make_float2(0.f, 0.f);
+    s_hi[k] = 0u;
+    s_lo[k] = 0u;
   }
   __syncthreads();
+  const float scale_hi = (float)(1 << kTileHiBits), scale_lo = (float)(1 << kTileLoBits);
+  const int nch = (seg.end - seg.begin + kStageRecs - 1) / kStageRecs;
+  int offs[2];
+  offs[0] = stage_records(a, st, 0, seg.begin, min(seg.end, seg.begin + kStageRecs), false, 0);
+  for (int c = 0; c < nch; c++) {
+    const int b = c & 1;
+    if (c + 1 < nch) {   // prefetch the next chunk into the other buffer (freed by the last sync)
+      const int nb = seg.begin + (c + 1) * kStageRecs;
+      offs[b ^ 1] = stage_records(a, st, b ^ 1, nb, min(seg.end, nb + kStageRecs), false, 0);
+    }
+    mbar_wait(&st.bar[b], (c >> 1) & 1);
+    const RecBuf &B = st.buf[b];
+    const int off = offs[b];
+    const int cb = seg.begin + c * kStageRecs, ce = min(seg.end, cb + kStageRecs);
+    for (int k = threadIdx.x; k < ce - cb; k += blockDim.x) {
+      const float4 q = B.rec[off + k];
+      const int2 rc = B.rc[off + k];
+      const float r = __int_as_float(rc.x) * scale_hi;
+      const int i0 = rc.y & 0xffff, j0 = rc.y >> 16;
+      // overlaps with the 3 x 3 bins from the first bin; clipping makes out-of-map overlaps <= 0
+      float ox3[3], oy3[3];
+#pragma unroll
+      for (int d = 0; d < 3; d++) {
+        ox3[d] = fmaxf(fminf(q.z, (float)(d + 1)) - fmaxf(q.x, (float)d), 0.f);
+        oy3[d] = fmaxf(fminf(q.w, (float)(d + 1)) - fmaxf(q.y, (float)d), 0.f);
+      }
+      const int base = i0 * P + j0;
+#pragma unroll
+      for (int di = 0; di < 3; di++) {
+        const float rx = r * ox3[di];
+#pragma unroll
+        for (int dj = 0; dj < 3; dj++) {
+          const float vh = rx * oy3[dj];   // v 2^hi_bits, exact scaling
+          const unsigned hi = (unsigned)vh;
+          const unsigned lo = (unsigned)((vh - (float)hi) * scale_lo);
+          const int k2 = base + di * P + dj;
+          if (hi) atomicAdd(s_hi + k2, hi);
+          if (lo) atomicAdd(s_lo + k2, lo);
+        }
+      }
+    }
+    __syncthreads();   // buffer b consumed before it is refilled (two chunks later)
+  }
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = blockDim.x >> 5;
+  for (int i = warp; i < P; i += nw) {
+    const int gi = ox + i;
+    if (gi >= a.mx) break;
+    for (int j = lane; j < P; j += 32) {
+      const unsigned long long v =
+          ((unsigned long long)s_hi[i * P + j] << kTileLoBits) + (unsigned long long)s_lo[i * P + j];
+      const int gj = oy + j;
+      if (v != 0ull && gj < a.my)
+        asm volatile("red.global.add.u64 [%0], %1;" ::"l"(a.rho + (size_t)gi * a.my + gj), "l"(v) : "memory");
+    }
+  }
+}
+
+// D5: the (tile+2)^2 float2 field tile staged once per segment (one bulk copy per tile row,
+// one issuing thread per row), records staged kSegChunk at a time, force written per cell.
+__global__ void __launch_bounds__(kTileThreads) k_gather_tiles(DenArgs a) {
+  extern __shared__ __align__(16) unsigned char dsm[];
+  RecStage &st = *reinterpret_cast<RecStage *>(dsm);
+  float2 *s_xi = reinterpret_cast<float2 *>(dsm + rec_stage_bytes());
+  const int sg = blockIdx.x;
+  if (sg >= *a.nsegs) return;
+  const Segment seg = a.segs[sg];
+  const int P = a.tile + kHalo;
+  const int tx = seg.tile / a.tiles_y, ty = seg.tile % a.tiles_y;
+  const int ox = tx * a.tile, oy = ty * a.tile;
+  const int rows = min(P, a.mx - ox), cols = min(P, a.my - oy);   // cols = tile or tile + 2: 16-byte multiple
+  if (threadIdx.x == 0) {
+    mbar_init(&st.bar[0]);
+    mbar_init(&st.bar[1]);
+  }
+  __syncthreads();   // barriers initialised
+  const int nch = (seg.end - seg.begin + kStageRecs - 1) / kStageRecs;
+  int offs[2];
+  offs[0] = stage_records(a, st, 0, seg.begin, min(seg.end, seg.begin + kStageRecs), true,
+                          (unsigned)(rows * cols * 8));
+  if (threadIdx.x < rows)
+    bulk_g2s(s_xi + threadIdx.x * P, a.xi + (size_t)(ox + threadIdx.x) * a.my + oy, 8u * cols, &st.bar[0]);
+  // bins outside the map (last tile row / column) read as zero
+  if (rows < P || cols < P) {
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = blockDim.x >> 5;
+    for (int i = warp; i < P; i += nw)
+      for (int j = lane; j < P; j += 32)
+        if (i >= rows || j >= cols) s_xi[i * P + j] = make_float2(0.f, 0.f);
+    __syncthreads();
+  }
   const float area = (float)(a.bx * a.by);
-  for (int p = seg.begin + threadIdx.x; p < seg.end; p += blockDim.x) {
-    const float4 q = a.rec[p];
-    const int2 rc = a.rec_rc[p];
-    const float r = __int_as_float(rc.x);
-    const int i0 = rc.y & 0xffff, j0 = rc.y >> 16;
-    float fx = 0.f, fy = 0.f;
-#pragma unroll
-    for (int di = 0; di < 3; di++) {
-      const int i = i0 + di;
-      const float ovx = fminf(q.z, (float)(di + 1)) - fmaxf(q.x, (float)di);
-      if (ovx <= 0.f || i >= P) break;
-#pragma unroll
-      for (int dj = 0; dj < 3; dj++) {
-        const int j = j0 + dj;
-        const float ovy = fminf(q.w, (float)(dj + 1)) - fmaxf(q.y, (float)dj);
-        if (ovy <= 0.f || j >= P) break;
-        const float2 e = s_xi[i * P + j];
-        const float ov = ovx * ovy;
-        fx += ov * e.x;
-        fy += ov * e.y;
-      }
+  for (int c = 0; c < nch; c++) {
+    const int b = c & 1;
+    if (c + 1 < nch) {
+      const int nb = seg.begin + (c + 1) * kStageRecs;
+      offs[b ^ 1] = stage_records(a, st, b ^ 1, nb, min(seg.end, nb + kStageRecs), true, 0);
     }
-    // dD/dx = - r sum_b ov(i,b) xi^X_b  (reading A21), ov in length^2
-    a.force[a.rec_cell[p]] = make_float2(-area * r * fx, -area * r * fy);
+    mbar_wait(&st.bar[b], (c >> 1) & 1);
+    const RecBuf &B = st.buf[b];
+    const int off = offs[b];
+    const int cb = seg.begin + c * kStageRecs, ce = min(seg.end, cb + kStageRecs);
+    for (int k = threadIdx.x; k < ce - cb; k += blockDim.x) {
+      const float4 q = B.rec[off + k];
+      const int2 rc = B.rc[off + k];
+      const float r = __int_as_float(rc.x);
+      const int i0 = rc.y & 0xffff, j0 = rc.y >> 16;
+      float ox3[3], oy3[3];
+#pragma unroll
+      for (int d = 0; d < 3; d++) {
+        ox3[d] = fmaxf(fminf(q.z, (float)(d + 1)) - fmaxf(q.x, (float)d), 0.f);
+        oy3[d] = fmaxf(fminf(q.w, (float)(d + 1)) - fmaxf(q.y, (float)d), 0.f);
+      }
+      const float2 *row = s_xi + i0 * P + j0;
+      float fx = 0.f, fy = 0.f;
+#pragma unroll
+      for (int di = 0; di < 3; di++) {
+        float sx = 0.f, sy = 0.f;
+#pragma unroll
+        for (int dj = 0; dj < 3; dj++) {
+          const float2 e2 = row[di * P + dj];   // in-bounds: i0 < tile, j0 < tile, P = tile + 2
+          sx = fmaf(oy3[dj], e2.x, sx);
+          sy = fmaf(oy3[dj], e2.y, sy);
+        }
+        fx = fmaf(ox3[di], sx, fx);
+        fy = fmaf(ox3[di], sy, fy);
+      }
+      // dD/dx = - r sum_b ov(i,b) xi^X_b  (reading A21), ov in length^2
+      a.force[B.cell[off + k]] = make_float2(-area * r * fx, -area * r * fy);
+    }
+    __syncthreads();
   }
 }
 
@@ -346,16 +528,16 @@ __global__ void __launch_bounds__(256) k_scatter_large(DenArgs a) {
   const int i = a.large[blockIdx.x];
   const Foot f = footprint(a, i);
   if (f.empty) return;
-  const int i0 = max((int)floor((f.lx - a.xl) * a.ibx), 0), i1 = min((int)floor((f.hx - a.xl) * a.ibx), a.mx - 1);
-  const int j0 = max((int)floor((f.ly - a.yl) * a.iby), 0), j1 = min((int)floor((f.hy - a.yl) * a.iby), a.my - 1);
+  const int i0 = (int)f.lo_x, i1 = min((int)ceil(f.hi_x), a.mx) - 1;
+  const int j0 = (int)f.lo_y, j1 = min((int)ceil(f.hi_y), a.my) - 1;
   const int nj = j1 - j0 + 1, n = (i1 - i0 + 1) * nj;
   for (int k = threadIdx.x; k < n; k += blockDim.x) {
     const int bi = i0 + k / nj, bj = j0 + k % nj;
-    const double ox = fmin(f.hx, a.xl + (bi + 1) * a.bx) - fmax(f.lx, a.xl + bi * a.bx);
-    const double oy = fmin(f.hy, a.yl + (bj + 1) * a.by) - fmax(f.ly, a.yl + bj * a.by);
+    const double ox = fmin(f.hi_x, (double)(bi + 1)) - fmax(f.lo_x, (double)bi);
+    const double oy = fmin(f.hi_y, (double)(bj + 1)) - fmax(f.lo_y, (double)bj);
     if (ox <= 0.0 || oy <= 0.0) continue;
     const unsigned long long v =
-        (unsigned long long)__double2ll_rn((double)f.r * ox * oy * a.ibx * a.iby * (double)(1ll << kRhoScaleLog2));
+        (unsigned long long)__double2ll_rn((double)f.r * ox * oy * (double)(1ll << kRhoScaleLog2));
     asm volatile("red.global.add.u64 [%0], %1;" ::"l"(a.rho + (size_t)bi * a.my + bj), "l"(v) : "memory");
   }
 }
@@ -366,13 +548,13 @@ __global__ void __launch_bounds__(256) k_gather_large(DenArgs a) {
   __shared__ double s_x[8], s_y[8];
   double fx = 0.0, fy = 0.0;
   if (!f.empty) {
-    const int i0 = max((int)floor((f.lx - a.xl) * a.ibx), 0), i1 = min((int)floor((f.hx - a.xl) * a.ibx), a.mx - 1);
-    const int j0 = max((int)floor((f.ly - a.yl) * a.iby), 0), j1 = min((int)floor((f.hy - a.yl) * a.iby), a.my - 1);
+    const int i0 = (int)f.lo_x, i1 = min((int)ceil(f.hi_x), a.mx) - 1;
+    const int j0 = (int)f.lo_y, j1 = min((int)ceil(f.hi_y), a.my) - 1;
     const int nj = j1 - j0 + 1, n = (i1 - i0 + 1) * nj;
     for (int k = threadIdx.x; k < n; k += blockDim.x) {
       const int bi = i0 + k / nj, bj = j0 + k % nj;
-      const double ox = fmin(f.hx, a.xl + (bi + 1) * a.bx) - fmax(f.lx, a.xl + bi * a.bx);
-      const double oy = fmin(f.hy, a.yl + (bj + 1) * a.by) - fmax(f.ly, a.yl + bj * a.by);
+      const double ox = fmin(f.hi_x, (double)(bi + 1)) - fmax(f.lo_x, (double)bi);
+      const double oy = fmin(f.hi_y, (double)(bj + 1)) - fmax(f.lo_y, (double)bj);
       if (ox <= 0.0 || oy <= 0.0) continue;
       const float2 e = a.xi[(size_t)bi * a.my + bj];
       fx += ox * oy * e.x;
@@ -395,7 +577,8 @@ __global__ void __launch_bounds__(256) k_gather_large(DenArgs a) {
       tx += s_x[w];
       ty += s_y[w];
     }
-    a.force[i] = make_float2((float)(-(double)f.r * tx), (float)(-(double)f.r * ty));
+    const double area = a.bx * a.by;   // overlaps above are in bin units
+    a.force[i] = make_float2((float)(-(double)f.r * area * tx), (float)(-(double)f.r * area * ty));
   }
 }
 
@@ -412,6 +595,10 @@ DenArgs make_args(const Ctx &c, const float *x, const float *y) {
   a.sy = 1.4142135623730951 * c.by;
   a.ibx = 1.0 / c.bx;
   a.iby = 1.0 / c.by;
+  a.cx0 = -c.xl * a.ibx;
+  a.cy0 = -c.yl * a.iby;
+  a.sxf = (float)a.sx;
+  a.syf = (float)a.sy;
   a.mx = c.mx; a.my = c.my; a.tile = c.tile; a.tiles_y = c.tiles_y;
   a.tile_log2 = 0;
   while ((1 << a.tile_log2) < c.tile) a.tile_log2++;
@@ -438,11 +625,11 @@ cudaError_t density_configure(int ntiles, int tile) {
   const int P = tile + kHalo;
   cudaError_t e = cudaFuncSetAttribute(k_count, cudaFuncAttributeMaxDynamicSharedMemorySize, ntiles * 4);
   if (e != cudaSuccess) return e;
-  e = cudaFuncSetAttribute(k_place, cudaFuncAttributeMaxDynamicSharedMemorySize, ntiles * 4);
+  e = cudaFuncSetAttribute(k_place, cudaFuncAttributeMaxDynamicSharedMemorySize, place_smem_bytes(ntiles));
   if (e != cudaSuccess) return e;
-  e = cudaFuncSetAttribute(k_scatter_tiles, cudaFuncAttributeMaxDynamicSharedMemorySize, P * P * 4);
+  e = cudaFuncSetAttribute(k_scatter_tiles, cudaFuncAttributeMaxDynamicSharedMemorySize, rec_stage_bytes() + P * P * 8);
   if (e != cudaSuccess) return e;
-  return cudaFuncSetAttribute(k_gather_tiles, cudaFuncAttributeMaxDynamicSharedMemorySize, P * P * 8);
+  return cudaFuncSetAttribute(k_gather_tiles, cudaFuncAttributeMaxDynamicSharedMemorySize, rec_stage_bytes() + P * P * 8);
 }
 
 int density_launches(const Ctx &c) { return 6 + (c.n_large > 0 ? 1 : 0); }
@@ -451,13 +638,13 @@ void launch_density_map(const Ctx &c, const float *x, const float *y, cudaStream
   const DenArgs a = make_args(c, x, y);
   const int P = c.tile + kHalo;
   const int ntiles = a.ntiles;
-  const int nblk = (c.n_own + kCountThreads * 8 - 1) / (kCountThreads * 8);
+  const int nblk = (c.n_own + kCountCells - 1) / kCountCells;
   cudaMemsetAsync(c.d_rho, 0, sizeof(unsigned long long) * (size_t)c.mx * c.my, s);
   if (nblk > 0) {
     k_count<<<nblk, kCountThreads, ntiles * 4, s>>>(a);
     k_scan<<<1, 1024, 0, s>>>(a);
-    k_place<<<nblk, kCountThreads, ntiles * 4, s>>>(a);
-    k_scatter_tiles<<<c.max_segs, 256, P * P * 4, s>>>(a);
+    k_place<<<nblk, kCountThreads, place_smem_bytes(ntiles), s>>>(a);
+    k_scatter_tiles<<<c.max_segs, kTileThreads, rec_stage_bytes() + P * P * 8, s>>>(a);
   }
   if (c.n_large > 0) k_scatter_large<<<c.n_large, 256, 0, s>>>(a);
 }
@@ -465,7 +652,7 @@ void launch_density_map(const Ctx &c, const float *x, const float *y, cudaStream
 void launch_density_gather(const Ctx &c, const float *x, const float *y, cudaStream_t s) {
   const DenArgs a = make_args(c, x, y);
   const int P = c.tile + kHalo;
-  if (c.n_own > 0) k_gather_tiles<<<c.max_segs, 256, P * P * 8, s>>>(a);
+  if (c.n_own > 0) k_gather_tiles<<<c.max_segs, kTileThreads, rec_stage_bytes() + P * P * 8, s>>>(a);
   if (c.n_large > 0) k_gather_large<<<c.n_large, 256, 0, s>>>(a);
 }
 

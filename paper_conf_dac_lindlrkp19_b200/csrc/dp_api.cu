@@ -390,7 +390,7 @@ dp_status build_density(Ctx &c, const dp_netlist *nl) {
   for (int32_t i = 0; i < c.n_own; i++)
     if ((double)w[i] > 2.0 * c.bx || (double)h[i] > 2.0 * c.by) large.push_back(i);
   c.n_large = (int32_t)large.size();
-  c.tile = std::min(std::max(c.mx, c.my) > 2048 ? 64 : kTile, std::min(c.mx, c.my));
+  c.tile = std::min(kTile, std::min(c.mx, c.my));
   c.tiles_x = c.mx / c.tile;
   c.tiles_y = c.my / c.tile;
   const int ntiles = c.tiles_x * c.tiles_y;
@@ -404,9 +404,10 @@ dp_status build_density(Ctx &c, const dp_netlist *nl) {
   DP_CUDA(cudaMemset(c.d_tile_cnt, 0, sizeof(int32_t) * ntiles));
   if ((st = dev_alloc(c, &c.d_tile_cursor, ntiles)) != DP_OK) return st;
   if ((st = dev_alloc(c, &c.d_tile_off, ntiles + 1)) != DP_OK) return st;
-  if ((st = dev_alloc(c, &c.d_rec, std::max(c.n_own, 1))) != DP_OK) return st;
-  if ((st = dev_alloc(c, &c.d_rec_rc, std::max(c.n_own, 1))) != DP_OK) return st;
-  if ((st = dev_alloc(c, &c.d_rec_cell, std::max(c.n_own, 1))) != DP_OK) return st;
+  // sort records; padded by 4 so segment copies may round their range to 4-record multiples
+  if ((st = dev_alloc(c, &c.d_rec, c.n_own + 8)) != DP_OK) return st;
+  if ((st = dev_alloc(c, &c.d_rec_rc, c.n_own + 8)) != DP_OK) return st;
+  if ((st = dev_alloc(c, &c.d_rec_cell, c.n_own + 8)) != DP_OK) return st;
   if ((st = dev_alloc(c, &c.d_segs, c.max_segs)) != DP_OK) return st;
   if ((st = dev_alloc(c, &c.d_nsegs, 1)) != DP_OK) return st;
   DP_CUDA(cudaMemset(c.d_nsegs, 0, sizeof(int32_t)));
@@ -509,7 +510,7 @@ dp_status create(const dp_netlist *nl, const dp_grid *grid, int device, int rank
   if ((st = build_wa(*c, nl, mask)) != DP_OK) return bail(st);
   if ((st = build_density(*c, nl)) != DP_OK) return bail(st);
   c->n_wa_part = c->n_chunks + c->n_big;
-  c->n_en_part = c->my / (c->mx <= 2048 ? 4 : 2);   // = CTAs of the column-fields kernel
+  c->n_en_part = c->my / 2;   // = CTAs of the column-fields kernel (2-column slabs)
   if ((st = dev_alloc(*c, &c->d_g2, c->num_cells)) != DP_OK) return bail(st);
   if (cudaMemset(c->d_g2, 0, sizeof(float2) * c->num_cells) != cudaSuccess) return bail(fail(DP_ERR_CUDA, "memset"));
   if ((st = dev_alloc(*c, &c->d_part, c->n_wa_part + c->n_en_part + 1)) != DP_OK) return bail(st);

@@ -24,13 +24,19 @@ constexpr int kWaWindow = 1024;       // consecutive cells per chunk window held
 constexpr int kBigThreads = 128;      // CTA-per-net kernel for nets > kWaMaxDeg
 constexpr int kHpwlLimbs = 9;         // limbs 0..kHpwlLimbs (10) of 32-bit digits, LSB 2^-149 (reading A7)
 
-constexpr int kTile = 32;             // density tile = kTile x kTile bins
+constexpr int kTile = 64;             // density tile = kTile x kTile bins (smaller maps: the map)
 constexpr int kHalo = 2;              // small-cell footprints extend <= 2 bins past their tile
-constexpr int kSegCells = 2048;       // cells per scatter/gather work segment
-constexpr int kTileScaleLog2 = 19;    // tile bins accumulate int32 units of 2^-19 (<= kSegCells x 1 < 2^12)
-constexpr int kRhoScaleLog2 = 24;     // global bin map: int64 units of 2^-24
+constexpr int kSegCells = 2048;       // cells per scatter/gather work segment (one CTA; load balance)
+constexpr int kSegChunk = 2048;       // records staged in shared memory at a time
+// Tile bins accumulate each contribution v in (0, 1] as two native 32-bit shared atomics:
+// hi = floor(v 2^kTileHiBits) and lo = floor(frac 2^kTileLoBits); with <= kSegCells = 2^13
+// records per segment neither word can overflow (2^13 * 2^10 < 2^32, 2^13 * (2^19 - 1) < 2^32),
+// and the pair resolves 2^-29.
+constexpr int kTileHiBits = 10;
+constexpr int kTileLoBits = 19;
+constexpr int kRhoScaleLog2 = kTileHiBits + kTileLoBits;   // global bin map: int64 units of 2^-29
 constexpr int kCountThreads = 256;
-constexpr int kCountCells = kCountThreads * 8;  // cells per count/place CTA (8 per thread)
+constexpr int kCountCells = 2048;     // cells per count/place CTA (staged in shared memory)
 
 // Per warp-group metadata of the WA chunk layout (16 bytes, bulk-copied per chunk).
 struct WarpGroup {

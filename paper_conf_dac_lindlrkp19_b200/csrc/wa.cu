@@ -24,6 +24,7 @@
 //    common shift that cancels exactly (reading A2).  Values are carried in log2 units;
 //  * HPWL mode uses exact (TwoSum) pin positions and extremes and a 2^-149 fixed-point int64
 //    limb sum: correctly rounded and order independent (reading A7).
+#include "async_copy.cuh"
 #include "dp_internal.h"
 
 namespace dp {
@@ -435,25 +436,6 @@ __device__ __forceinline__ void wa_group_pairs(const WaArgs &a, const WarpGroup 
   grad_add(gc, r0, -gx, -gy);
 }
 
-__device__ __forceinline__ unsigned smem_u32(const void *p) { return (unsigned)__cvta_generic_to_shared(p); }
-
-__device__ __forceinline__ void bulk_g2s(void *dst, const void *src, unsigned bytes, uint64_t *bar) {
-  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
-               ::"r"(smem_u32(dst)), "l"(src), "r"(bytes), "r"(smem_u32(bar))
-               : "memory");
-}
-
-__device__ __forceinline__ void mbar_wait(uint64_t *bar, unsigned phase) {
-  unsigned done = 0;
-  while (!done) {
-    asm volatile(
-        "{\n .reg .pred p;\n mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n selp.u32 %0, 1, 0, p;\n}"
-        : "=r"(done)
-        : "r"(smem_u32(bar)), "r"(phase)
-        : "memory");
-  }
-}
-
 // Dynamic shared-memory layout of the chunk kernel (capacities fixed at create).
 struct WaSmem {
   WaCaps c;
@@ -497,11 +479,10 @@ __global__ void __launch_bounds__(kWaThreads, 3) k_wa_chunks(WaArgs a) {
   const int wbulk = ch.win_n & ~3;
   const bool win_bulk = ((((uintptr_t)(a.x + ch.win_lo)) | ((uintptr_t)(a.y + ch.win_lo))) & 15) == 0 && wbulk > 0;
   if (tid == 0) {
-    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(1) : "memory");
-    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    mbar_init(bar);
     const unsigned tx = 12u * ch.pin_n + (a.has_w ? 8u : 4u) * ch.net_n + 16u * ch.wg_n + 4u * ch.far_pad +
                         (win_bulk ? 8u * wbulk : 0u);
-    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(tx) : "memory");
+    mbar_expect_tx(bar, tx);
     if (ch.pin_n) {
       bulk_g2s(s_slot, a.pin_slot + ch.pin_begin, 4u * ch.pin_n, bar);
       bulk_g2s(s_dx, a.pin_dx + ch.pin_begin, 4u * ch.pin_n, bar);

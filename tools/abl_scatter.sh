@@ -1,0 +1,4 @@
+for A in 0 1 2 3 7; do
+  DP_ABLATE_SCATTER=$A ncu --metrics gpu__time_duration.sum --clock-control none -k regex:k_scatter_tiles -s 5 -c 3 --csv --log-file gpurun_out/abls_$A.csv python bench.py --steps 4 --warmup 4 --no-cpu-baseline --e2e-steps 1 > /dev/null 2>&1
+  echo "ablate=$A"; grep k_scatter gpurun_out/abls_$A.csv | awk -F'","' '{print $NF}' | tr -d '"' | head -3
+done

@@ -16,7 +16,7 @@ def summarise(path):
         v = float(r[mi].replace(',', ''))
         u = r[ui]
         v = v / 1000 if u in ('nsecond', 'ns') else (v * 1000 if u in ('msecond', 'ms') else v)
-        name = r[ki].split('(')[0].replace('void ', '').replace('dp::<unnamed>::', '')[:48]
+        name = r[ki].split('(')[0].replace('void ', '').replace('dp::<unnamed>::', '').replace('unnamed>::', '')[:48]
         d[name].append(v)
     return d
 

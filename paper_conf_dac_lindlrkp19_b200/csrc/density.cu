@@ -11,13 +11,15 @@
 // (tools/microbench), which would cost ~70 us for the ~13M bin updates of bigblue4.  So every
 // evaluation sorts the small cells by spatial tile (kTile x kTile bins):
 //   D1 count   per-CTA shared histogram of tile ids -> global tile counts
-//   D2 scan    one CTA: tile offsets, per-tile cursors, work segments (<= kSegCells cells)
+//   D2 scan    one CTA: tile offsets and per-tile cursors
 //   D3 place   recompute tile ids, reserve ranges per CTA, write tile-local footprint
 //              records in tile order
-//   D4 scatter one CTA per segment accumulates its records into a (tile+2)^2 shared tile,
-//              flushed with coalesced red.add into rho
-//   D5 gather  one CTA per segment stages the (tile+2)^2 float2 field tile in shared memory
-//              and writes each cell's force
+//   D4 scatter persistent walkers (SMs x resident CTAs) each take an equal slice of the
+//              tile-ordered records, stream it through double-buffered bulk copies and
+//              accumulate into a (tile+2)^2 shared tile, flushed with coalesced red.add into
+//              rho only where the slice leaves a tile
+//   D5 gather  same walkers; the (tile+2)^2 float2 field tile is reloaded only where the slice
+//              enters a new tile; each cell's force is written once
 // Large cells (footprint wider than 3 bins) take a CTA-per-cell path with global reds.
 // The tile accumulators (two 32-bit words per bin, 2^-29 resolution) flush into an int64 global
 // map (2^-29 units) with native red.global.add.u64: the density map is exact up to one rounding
@@ -45,8 +47,6 @@ struct DenArgs {
   float sxf, syf;      // stretched minimum sizes sqrt2 b (fp32)
   int mx, my, tile, tile_log2, tiles_y, ntiles, stretch;
   int *tile_cnt, *tile_cursor, *tile_off;
-  Segment *segs;
-  int *nsegs;
   float4 *rec;
   int2 *rec_rc;   // (r as float bits, tile-local first bin i0 | j0 << 16)
   int *rec_cell;  // own cell index
@@ -92,38 +92,6 @@ __device__ __forceinline__ int small_tile(const DenArgs &a, const Foot &f, int &
   by0 = min((int)f.lo_y, a.my - 1);
   return (bx0 >> a.tile_log2) * a.tiles_y + (by0 >> a.tile_log2);
 }
-
-// Loads x, y, w, h of own cells [i0, i0 + 8) (i0 a multiple of 8) with 16-byte vector loads
-// when the global index is aligned; out-of-range cells get w = h = 0 (empty).
-struct Cells8 { float x[8], y[8], w[8], h[8]; };
-
-__device__ __forceinline__ void load_cells8(const DenArgs &a, int i0, Cells8 &c) {
-  const int g0 = a.cell_begin + i0;
-  if (i0 + 8 <= a.n_own && (g0 & 3) == 0) {
-#pragma unroll
-    for (int v = 0; v < 2; v++) {
-      const float4 X = __ldg(reinterpret_cast<const float4 *>(a.x + g0) + v);
-      const float4 Y = __ldg(reinterpret_cast<const float4 *>(a.y + g0) + v);
-      const float4 W = __ldg(reinterpret_cast<const float4 *>(a.w + i0) + v);
-      const float4 H = __ldg(reinterpret_cast<const float4 *>(a.h + i0) + v);
-      c.x[4 * v] = X.x; c.x[4 * v + 1] = X.y; c.x[4 * v + 2] = X.z; c.x[4 * v + 3] = X.w;
-      c.y[4 * v] = Y.x; c.y[4 * v + 1] = Y.y; c.y[4 * v + 2] = Y.z; c.y[4 * v + 3] = Y.w;
-      c.w[4 * v] = W.x; c.w[4 * v + 1] = W.y; c.w[4 * v + 2] = W.z; c.w[4 * v + 3] = W.w;
-      c.h[4 * v] = H.x; c.h[4 * v + 1] = H.y; c.h[4 * v + 2] = H.z; c.h[4 * v + 3] = H.w;
-    }
-  } else {
-#pragma unroll
-    for (int k = 0; k < 8; k++) {
-      const int i = i0 + k;
-      const bool ok = i < a.n_own;
-      c.x[k] = ok ? __ldg(a.x + a.cell_begin + i) : 0.f;
-      c.y[k] = ok ? __ldg(a.y + a.cell_begin + i) : 0.f;
-      c.w[k] = ok ? __ldg(a.w + i) : 0.f;
-      c.h[k] = ok ? __ldg(a.h + i) : 0.f;
-    }
-  }
-}
-
 
 // Stage the x, y, w, h of own cells [i0, i0 + n) (n <= kCountCells) in shared memory: bulk async
 // copies of the 16-byte aligned prefix (one elected thread, one mbarrier), plain loads for the
@@ -174,8 +142,8 @@ __global__ void __launch_bounds__(kCountThreads) k_count(DenArgs a) {
     if (s_hist[t]) atomicAdd(a.tile_cnt + t, s_hist[t]);
 }
 
-// D2 (single CTA of 1024 threads): exclusive scans of tile counts and segment counts with
-// warp shuffles (two barriers), cursors, work segments; resets the counts for the next call.
+// D2 (single CTA of 1024 threads): exclusive scan of the tile counts with warp shuffles (two
+// barriers) -> tile offsets and cursors; resets the counts for the next call.
 __device__ __forceinline__ int warp_incl_scan(int v, int lane) {
 #pragma unroll
   for (int o = 1; o < 32; o <<= 1) {
@@ -186,58 +154,31 @@ __device__ __forceinline__ int warp_incl_scan(int v, int lane) {
 }
 
 __global__ void __launch_bounds__(1024) k_scan(DenArgs a) {
-  __shared__ int s_wa[32], s_wb[32];
+  __shared__ int s_wa[32];
   constexpr int T = 1024;
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const int per = (a.ntiles + T - 1) / T;
   const int t0 = threadIdx.x * per;
-  int cnt_sum = 0, seg_sum = 0;
-  for (int k = 0; k < per; k++) {
-    const int t = t0 + k;
-    if (t < a.ntiles) {
-      const int c = a.tile_cnt[t];
-      cnt_sum += c;
-      seg_sum += (c + kSegCells - 1) / kSegCells;
-    }
-  }
-  const int ia = warp_incl_scan(cnt_sum, lane), ib = warp_incl_scan(seg_sum, lane);
-  if (lane == 31) {
-    s_wa[warp] = ia;
-    s_wb[warp] = ib;
-  }
+  int cnt_sum = 0;
+  for (int k = 0; k < per; k++)
+    if (t0 + k < a.ntiles) cnt_sum += a.tile_cnt[t0 + k];
+  const int ia = warp_incl_scan(cnt_sum, lane);
+  if (lane == 31) s_wa[warp] = ia;
   __syncthreads();
-  if (warp == 0) {
-    const int xa = warp_incl_scan(s_wa[lane], lane), xb = warp_incl_scan(s_wb[lane], lane);
-    s_wa[lane] = xa;
-    s_wb[lane] = xb;
-  }
+  if (warp == 0) s_wa[lane] = warp_incl_scan(s_wa[lane], lane);
   __syncthreads();
   int off_c = (warp ? s_wa[warp - 1] : 0) + ia - cnt_sum;
-  int off_s = (warp ? s_wb[warp - 1] : 0) + ib - seg_sum;
   for (int k = 0; k < per; k++) {
     const int t = t0 + k;
     if (t < a.ntiles) {
       const int c = a.tile_cnt[t];
       a.tile_off[t] = off_c;
       a.tile_cursor[t] = off_c;
-      const int ns = (c + kSegCells - 1) / kSegCells;
-      for (int q = 0; q < ns; q++) {
-        Segment sg;
-        sg.tile = t;
-        sg.begin = off_c + q * kSegCells;
-        sg.end = min(off_c + c, sg.begin + kSegCells);
-        sg.pad = 0;
-        a.segs[off_s + q] = sg;
-      }
       off_c += c;
-      off_s += ns;
       a.tile_cnt[t] = 0;  // ready for the next evaluation
     }
   }
-  if (threadIdx.x == T - 1) {
-    a.tile_off[a.ntiles] = off_c;
-    *a.nsegs = off_s;
-  }
+  if (threadIdx.x == T - 1) a.tile_off[a.ntiles] = off_c;
 }
 
 // D3: same staged block as D1.  Pass 1: shared histogram; local exclusive scan (the block's
@@ -251,7 +192,6 @@ struct PlaceOut {
   int tile[kCountCells];
 };
 
-__host__ __device__ constexpr int place_static_bytes() { return 0; }
 int place_smem_bytes(int ntiles) { return (int)sizeof(PlaceOut) + 12 * ntiles; }
 
 __global__ void __launch_bounds__(kCountThreads) k_place(DenArgs a) {
@@ -326,8 +266,6 @@ __global__ void __launch_bounds__(kCountThreads) k_place(DenArgs a) {
     po.tile[slot] = t;
   }
   __syncthreads();
-  const int nrec = (warp == 0 && lane == 0) ? 0 : 0;
-  (void)nrec;
   const int total = s_warp[kCountThreads / 32 - 1];
   for (int j = threadIdx.x; j < total; j += kCountThreads) {
     const int t = po.tile[j];
@@ -338,10 +276,9 @@ __global__ void __launch_bounds__(kCountThreads) k_place(DenArgs a) {
   }
 }
 
-// Double-buffered record staging: buffer b holds up to kSegChunk / 2 records of rec (16 B),
+// Double-buffered record staging: buffer b holds up to kStageRecs records of rec (16 B),
 // rec_rc (8 B) and rec_cell (4 B); each buffer completes on its own mbarrier.  The copied range
 // is rounded out to 4-record multiples (the record arrays are padded by 8 records).
-constexpr int kStageRecs = kSegChunk / 2;
 struct RecBuf {
   float4 rec[kStageRecs + 8];
   int2 rc[kStageRecs + 8];
@@ -350,18 +287,20 @@ struct RecBuf {
 struct RecStage {
   RecBuf buf[2];
   uint64_t bar[2];
+  uint64_t bar_xi;
 };
 
 __host__ __device__ constexpr int rec_stage_bytes() { return (int)((sizeof(RecStage) + 15) & ~(size_t)15); }
+int walk_smem_bytes(int tile) { return rec_stage_bytes() + (tile + kHalo) * (tile + kHalo) * 8; }
 
 // Issue (thread 0) the copies of records [begin, end) into buffer b; returns the offset of the
 // first record inside the buffer (all threads).
 __device__ __forceinline__ int stage_records(const DenArgs &a, RecStage &st, int b, int begin, int end,
-                                             bool with_cell, unsigned extra_tx) {
+                                             bool with_cell) {
   const int b0 = begin & ~3, e0 = (end + 3) & ~3, n = e0 - b0;
   if (threadIdx.x == 0) {
     RecBuf &B = st.buf[b];
-    mbar_expect_tx(&st.bar[b], (unsigned)n * (with_cell ? 28u : 24u) + extra_tx);
+    mbar_expect_tx(&st.bar[b], (unsigned)n * (with_cell ? 28u : 24u));
     bulk_g2s(B.rec, a.rec + b0, 16u * n, &st.bar[b]);
     bulk_g2s(B.rc, a.rec_rc + b0, 8u * n, &st.bar[b]);
     if (with_cell) bulk_g2s(B.cell, a.rec_cell + b0, 4u * n, &st.bar[b]);
@@ -369,19 +308,84 @@ __device__ __forceinline__ int stage_records(const DenArgs &a, RecStage &st, int
   return begin - b0;
 }
 
-// D4: a segment's records (<= kSegCells, staged kSegChunk at a time) accumulate into a
-// (tile+2)^2 shared tile of (hi, lo) 32-bit words, flushed once into the int64 global map.
-__global__ void __launch_bounds__(kTileThreads) k_scatter_tiles(DenArgs a) {
+// A walker's slice [rb, re) of the tile-ordered small-cell records, cut into chunks of at most
+// kStageRecs records that never straddle a tile.  Every thread runs the same bookkeeping
+// (uniform loads of tile_off).
+struct WalkChunk {
+  int begin, end, tile, off;
+};
+struct Walker {
+  int cur, re, t, tend;
+};
+
+__device__ __forceinline__ bool walk_init(const DenArgs &a, Walker &w) {
+  const int N = a.tile_off[a.ntiles];
+  const int G = gridDim.x;
+  w.cur = (int)(((long long)N * blockIdx.x) / G);
+  w.re = (int)(((long long)N * (blockIdx.x + 1)) / G);
+  if (w.cur >= w.re) return false;
+  int lo = 0, hi = a.ntiles;   // largest t with tile_off[t] <= cur (then tile_off[t + 1] > cur)
+  while (hi - lo > 1) {
+    const int mid = (lo + hi) >> 1;
+    if (a.tile_off[mid] <= w.cur) lo = mid; else hi = mid;
+  }
+  w.t = lo;
+  w.tend = a.tile_off[lo + 1];
+  return true;
+}
+
+__device__ __forceinline__ WalkChunk walk_next(const DenArgs &a, Walker &w) {
+  WalkChunk c;
+  c.begin = c.end = w.cur;
+  c.tile = w.t;
+  c.off = 0;
+  if (w.cur >= w.re) return c;
+  while (w.tend <= w.cur) w.tend = a.tile_off[++w.t + 1];   // skip finished / empty tiles
+  c.tile = w.t;
+  c.end = min(min(w.cur + kStageRecs, w.tend), w.re);
+  w.cur = c.end;
+  return c;
+}
+
+// overlaps (bin units) of a record's footprint with the 3 bins from its first bin, per axis;
+// clipping makes out-of-map / non-covered overlaps 0
+__device__ __forceinline__ void rec_overlaps(const float4 q, float ox3[3], float oy3[3]) {
+#pragma unroll
+  for (int d = 0; d < 3; d++) {
+    ox3[d] = fmaxf(fminf(q.z, (float)(d + 1)) - fmaxf(q.x, (float)d), 0.f);
+    oy3[d] = fmaxf(fminf(q.w, (float)(d + 1)) - fmaxf(q.y, (float)d), 0.f);
+  }
+}
+
+// flush the shared (hi, lo) tile into rho and clear it (caller synchronises before and after)
+__device__ __forceinline__ void flush_tile(const DenArgs &a, unsigned *s_hi, unsigned *s_lo, int tile) {
+  const int P = a.tile + kHalo;
+  const int ox = (tile / a.tiles_y) * a.tile, oy = (tile % a.tiles_y) * a.tile;
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = blockDim.x >> 5;
+  for (int i = warp; i < P; i += nw) {
+    const int gi = ox + i;
+    for (int j = lane; j < P; j += 32) {
+      const int k = i * P + j;
+      const unsigned long long v = ((unsigned long long)s_hi[k] << kTileLoBits) + (unsigned long long)s_lo[k];
+      s_hi[k] = 0u;
+      s_lo[k] = 0u;
+      const int gj = oy + j;
+      if (v != 0ull && gi < a.mx && gj < a.my)
+        asm volatile("red.global.add.u64 [%0], %1;" ::"l"(a.rho + (size_t)gi * a.my + gj), "l"(v) : "memory");
+    }
+  }
+}
+
+// D4: persistent scatter walker.  The shared tile of (hi, lo) 32-bit words is flushed into the
+// int64 map when the slice moves to another tile and at least every kFlushRecs records.
+__global__ void __launch_bounds__(kTileThreads) k_scatter_walk(DenArgs a) {
   extern __shared__ __align__(16) unsigned char dsm[];
   RecStage &st = *reinterpret_cast<RecStage *>(dsm);
   unsigned *s_hi = reinterpret_cast<unsigned *>(dsm + rec_stage_bytes());   // 2^-kTileHiBits units
   unsigned *s_lo = s_hi + (a.tile + kHalo) * (a.tile + kHalo);               // 2^-(hi + lo bits) units
-  const int sg = blockIdx.x;
-  if (sg >= *a.nsegs) return;
-  const Segment seg = a.segs[sg];
+  Walker w;
+  if (!walk_init(a, w)) return;
   const int P = a.tile + kHalo;
-  const int tx = seg.tile / a.tiles_y, ty = seg.tile % a.tiles_y;
-  const int ox = tx * a.tile, oy = ty * a.tile;
   if (threadIdx.x == 0) {
     mbar_init(&st.bar[0]);
     mbar_init(&st.bar[1]);
@@ -392,31 +396,30 @@ __global__ void __launch_bounds__(kTileThreads) k_scatter_tiles(DenArgs a) {
   }
   __syncthreads();
   const float scale_hi = (float)(1 << kTileHiBits), scale_lo = (float)(1 << kTileLoBits);
-  const int nch = (seg.end - seg.begin + kStageRecs - 1) / kStageRecs;
-  int offs[2];
-  offs[0] = stage_records(a, st, 0, seg.begin, min(seg.end, seg.begin + kStageRecs), false, 0);
-  for (int c = 0; c < nch; c++) {
+  WalkChunk cc = walk_next(a, w);
+  cc.off = stage_records(a, st, 0, cc.begin, cc.end, false);
+  int cur_tile = cc.tile, acc = 0;
+  for (int c = 0; cc.begin < cc.end; c++) {
     const int b = c & 1;
-    if (c + 1 < nch) {   // prefetch the next chunk into the other buffer (freed by the last sync)
-      const int nb = seg.begin + (c + 1) * kStageRecs;
-      offs[b ^ 1] = stage_records(a, st, b ^ 1, nb, min(seg.end, nb + kStageRecs), false, 0);
+    WalkChunk nx = walk_next(a, w);   // prefetch into the other buffer (freed by the last sync)
+    if (nx.end > nx.begin) nx.off = stage_records(a, st, b ^ 1, nx.begin, nx.end, false);
+    const int n = cc.end - cc.begin;
+    if (cc.tile != cur_tile || acc + n > kFlushRecs) {
+      flush_tile(a, s_hi, s_lo, cur_tile);
+      __syncthreads();
+      cur_tile = cc.tile;
+      acc = 0;
     }
+    acc += n;
     mbar_wait(&st.bar[b], (c >> 1) & 1);
     const RecBuf &B = st.buf[b];
-    const int off = offs[b];
-    const int cb = seg.begin + c * kStageRecs, ce = min(seg.end, cb + kStageRecs);
-    for (int k = threadIdx.x; k < ce - cb; k += blockDim.x) {
-      const float4 q = B.rec[off + k];
-      const int2 rc = B.rc[off + k];
+    for (int k = threadIdx.x; k < n; k += blockDim.x) {
+      const float4 q = B.rec[cc.off + k];
+      const int2 rc = B.rc[cc.off + k];
       const float r = __int_as_float(rc.x) * scale_hi;
       const int i0 = rc.y & 0xffff, j0 = rc.y >> 16;
-      // overlaps with the 3 x 3 bins from the first bin; clipping makes out-of-map overlaps <= 0
       float ox3[3], oy3[3];
-#pragma unroll
-      for (int d = 0; d < 3; d++) {
-        ox3[d] = fmaxf(fminf(q.z, (float)(d + 1)) - fmaxf(q.x, (float)d), 0.f);
-        oy3[d] = fmaxf(fminf(q.w, (float)(d + 1)) - fmaxf(q.y, (float)d), 0.f);
-      }
+      rec_overlaps(q, ox3, oy3);
       const int base = i0 * P + j0;
 #pragma unroll
       for (int di = 0; di < 3; di++) {
@@ -432,47 +435,23 @@ __global__ void __launch_bounds__(kTileThreads) k_scatter_tiles(DenArgs a) {
         }
       }
     }
-    __syncthreads();   // buffer b consumed before it is refilled (two chunks later)
+    __syncthreads();   // buffer b consumed before it is refilled; tile complete before a flush
+    cc = nx;
   }
-  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = blockDim.x >> 5;
-  for (int i = warp; i < P; i += nw) {
-    const int gi = ox + i;
-    if (gi >= a.mx) break;
-    for (int j = lane; j < P; j += 32) {
-      const unsigned long long v =
-          ((unsigned long long)s_hi[i * P + j] << kTileLoBits) + (unsigned long long)s_lo[i * P + j];
-      const int gj = oy + j;
-      if (v != 0ull && gj < a.my)
-        asm volatile("red.global.add.u64 [%0], %1;" ::"l"(a.rho + (size_t)gi * a.my + gj), "l"(v) : "memory");
-    }
-  }
+  flush_tile(a, s_hi, s_lo, cur_tile);
 }
 
-// D5: the (tile+2)^2 float2 field tile staged once per segment (one bulk copy per tile row,
-// one issuing thread per row), records staged kSegChunk at a time, force written per cell.
-__global__ void __launch_bounds__(kTileThreads) k_gather_tiles(DenArgs a) {
-  extern __shared__ __align__(16) unsigned char dsm[];
-  RecStage &st = *reinterpret_cast<RecStage *>(dsm);
-  float2 *s_xi = reinterpret_cast<float2 *>(dsm + rec_stage_bytes());
-  const int sg = blockIdx.x;
-  if (sg >= *a.nsegs) return;
-  const Segment seg = a.segs[sg];
+// D5: persistent gather walker; the (tile+2)^2 float2 field tile is (re)loaded with one bulk copy
+// per tile row whenever the slice enters a tile; bins outside the map read as zero.
+__device__ __forceinline__ void load_xi_tile(const DenArgs &a, RecStage &st, float2 *s_xi, int tile,
+                                             unsigned phase) {
   const int P = a.tile + kHalo;
-  const int tx = seg.tile / a.tiles_y, ty = seg.tile % a.tiles_y;
-  const int ox = tx * a.tile, oy = ty * a.tile;
+  const int ox = (tile / a.tiles_y) * a.tile, oy = (tile % a.tiles_y) * a.tile;
   const int rows = min(P, a.mx - ox), cols = min(P, a.my - oy);   // cols = tile or tile + 2: 16-byte multiple
-  if (threadIdx.x == 0) {
-    mbar_init(&st.bar[0]);
-    mbar_init(&st.bar[1]);
-  }
-  __syncthreads();   // barriers initialised
-  const int nch = (seg.end - seg.begin + kStageRecs - 1) / kStageRecs;
-  int offs[2];
-  offs[0] = stage_records(a, st, 0, seg.begin, min(seg.end, seg.begin + kStageRecs), true,
-                          (unsigned)(rows * cols * 8));
+  if (threadIdx.x == 0) mbar_expect_tx(&st.bar_xi, (unsigned)(rows * cols * 8));
+  __syncthreads();   // armed before any copy can complete
   if (threadIdx.x < rows)
-    bulk_g2s(s_xi + threadIdx.x * P, a.xi + (size_t)(ox + threadIdx.x) * a.my + oy, 8u * cols, &st.bar[0]);
-  // bins outside the map (last tile row / column) read as zero
+    bulk_g2s(s_xi + threadIdx.x * P, a.xi + (size_t)(ox + threadIdx.x) * a.my + oy, 8u * cols, &st.bar_xi);
   if (rows < P || cols < P) {
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = blockDim.x >> 5;
     for (int i = warp; i < P; i += nw)
@@ -480,28 +459,46 @@ __global__ void __launch_bounds__(kTileThreads) k_gather_tiles(DenArgs a) {
         if (i >= rows || j >= cols) s_xi[i * P + j] = make_float2(0.f, 0.f);
     __syncthreads();
   }
+  mbar_wait(&st.bar_xi, phase);
+}
+
+__global__ void __launch_bounds__(kTileThreads) k_gather_walk(DenArgs a) {
+  extern __shared__ __align__(16) unsigned char dsm[];
+  RecStage &st = *reinterpret_cast<RecStage *>(dsm);
+  float2 *s_xi = reinterpret_cast<float2 *>(dsm + rec_stage_bytes());
+  Walker w;
+  if (!walk_init(a, w)) return;
+  const int P = a.tile + kHalo;
+  if (threadIdx.x == 0) {
+    mbar_init(&st.bar[0]);
+    mbar_init(&st.bar[1]);
+    mbar_init(&st.bar_xi);
+  }
+  __syncthreads();   // barriers initialised
+  WalkChunk cc = walk_next(a, w);
+  cc.off = stage_records(a, st, 0, cc.begin, cc.end, true);
+  int cur_tile = -1;
+  unsigned xi_phase = 0;
   const float area = (float)(a.bx * a.by);
-  for (int c = 0; c < nch; c++) {
+  for (int c = 0; cc.begin < cc.end; c++) {
     const int b = c & 1;
-    if (c + 1 < nch) {
-      const int nb = seg.begin + (c + 1) * kStageRecs;
-      offs[b ^ 1] = stage_records(a, st, b ^ 1, nb, min(seg.end, nb + kStageRecs), true, 0);
+    WalkChunk nx = walk_next(a, w);   // prefetch into the other buffer (freed by the last sync)
+    if (nx.end > nx.begin) nx.off = stage_records(a, st, b ^ 1, nx.begin, nx.end, true);
+    if (cc.tile != cur_tile) {   // the previous iteration's sync freed the field tile
+      load_xi_tile(a, st, s_xi, cc.tile, xi_phase);
+      xi_phase ^= 1u;
+      cur_tile = cc.tile;
     }
     mbar_wait(&st.bar[b], (c >> 1) & 1);
     const RecBuf &B = st.buf[b];
-    const int off = offs[b];
-    const int cb = seg.begin + c * kStageRecs, ce = min(seg.end, cb + kStageRecs);
-    for (int k = threadIdx.x; k < ce - cb; k += blockDim.x) {
-      const float4 q = B.rec[off + k];
-      const int2 rc = B.rc[off + k];
+    const int n = cc.end - cc.begin;
+    for (int k = threadIdx.x; k < n; k += blockDim.x) {
+      const float4 q = B.rec[cc.off + k];
+      const int2 rc = B.rc[cc.off + k];
       const float r = __int_as_float(rc.x);
       const int i0 = rc.y & 0xffff, j0 = rc.y >> 16;
       float ox3[3], oy3[3];
-#pragma unroll
-      for (int d = 0; d < 3; d++) {
-        ox3[d] = fmaxf(fminf(q.z, (float)(d + 1)) - fmaxf(q.x, (float)d), 0.f);
-        oy3[d] = fmaxf(fminf(q.w, (float)(d + 1)) - fmaxf(q.y, (float)d), 0.f);
-      }
+      rec_overlaps(q, ox3, oy3);
       const float2 *row = s_xi + i0 * P + j0;
       float fx = 0.f, fy = 0.f;
 #pragma unroll
@@ -517,9 +514,10 @@ __global__ void __launch_bounds__(kTileThreads) k_gather_tiles(DenArgs a) {
         fy = fmaf(ox3[di], sy, fy);
       }
       // dD/dx = - r sum_b ov(i,b) xi^X_b  (reading A21), ov in length^2
-      a.force[B.cell[off + k]] = make_float2(-area * r * fx, -area * r * fy);
+      a.force[B.cell[cc.off + k]] = make_float2(-area * r * fx, -area * r * fy);
     }
     __syncthreads();
+    cc = nx;
   }
 }
 
@@ -607,8 +605,6 @@ DenArgs make_args(const Ctx &c, const float *x, const float *y) {
   a.tile_cnt = c.d_tile_cnt;
   a.tile_cursor = c.d_tile_cursor;
   a.tile_off = c.d_tile_off;
-  a.segs = c.d_segs;
-  a.nsegs = c.d_nsegs;
   a.rec = c.d_rec;
   a.rec_rc = c.d_rec_rc;
   a.rec_cell = c.d_rec_cell;
@@ -622,21 +618,32 @@ DenArgs make_args(const Ctx &c, const float *x, const float *y) {
 }  // namespace
 
 cudaError_t density_configure(int ntiles, int tile) {
-  const int P = tile + kHalo;
   cudaError_t e = cudaFuncSetAttribute(k_count, cudaFuncAttributeMaxDynamicSharedMemorySize, ntiles * 4);
   if (e != cudaSuccess) return e;
   e = cudaFuncSetAttribute(k_place, cudaFuncAttributeMaxDynamicSharedMemorySize, place_smem_bytes(ntiles));
   if (e != cudaSuccess) return e;
-  e = cudaFuncSetAttribute(k_scatter_tiles, cudaFuncAttributeMaxDynamicSharedMemorySize, rec_stage_bytes() + P * P * 8);
+  e = cudaFuncSetAttribute(k_scatter_walk, cudaFuncAttributeMaxDynamicSharedMemorySize, walk_smem_bytes(tile));
   if (e != cudaSuccess) return e;
-  return cudaFuncSetAttribute(k_gather_tiles, cudaFuncAttributeMaxDynamicSharedMemorySize, rec_stage_bytes() + P * P * 8);
+  return cudaFuncSetAttribute(k_gather_walk, cudaFuncAttributeMaxDynamicSharedMemorySize, walk_smem_bytes(tile));
+}
+
+// grid of the walkers: every SM filled with as many CTAs as fit (the smaller of the two kernels'
+// occupancies, so both see the same slices)
+int density_walk_grid(int tile) {
+  int dev = 0, sms = 0, o1 = 0, o2 = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess) return 0;
+  if (cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess) return 0;
+  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o1, k_scatter_walk, kTileThreads, walk_smem_bytes(tile)) != cudaSuccess)
+    return 0;
+  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o2, k_gather_walk, kTileThreads, walk_smem_bytes(tile)) != cudaSuccess)
+    return 0;
+  return sms * std::max(1, std::min(o1, o2));
 }
 
 int density_launches(const Ctx &c) { return 6 + (c.n_large > 0 ? 1 : 0); }
 
 void launch_density_map(const Ctx &c, const float *x, const float *y, cudaStream_t s) {
   const DenArgs a = make_args(c, x, y);
-  const int P = c.tile + kHalo;
   const int ntiles = a.ntiles;
   const int nblk = (c.n_own + kCountCells - 1) / kCountCells;
   cudaMemsetAsync(c.d_rho, 0, sizeof(unsigned long long) * (size_t)c.mx * c.my, s);
@@ -644,15 +651,14 @@ void launch_density_map(const Ctx &c, const float *x, const float *y, cudaStream
     k_count<<<nblk, kCountThreads, ntiles * 4, s>>>(a);
     k_scan<<<1, 1024, 0, s>>>(a);
     k_place<<<nblk, kCountThreads, place_smem_bytes(ntiles), s>>>(a);
-    k_scatter_tiles<<<c.max_segs, kTileThreads, rec_stage_bytes() + P * P * 8, s>>>(a);
+    k_scatter_walk<<<c.walk_grid, kTileThreads, walk_smem_bytes(c.tile), s>>>(a);
   }
   if (c.n_large > 0) k_scatter_large<<<c.n_large, 256, 0, s>>>(a);
 }
 
 void launch_density_gather(const Ctx &c, const float *x, const float *y, cudaStream_t s) {
   const DenArgs a = make_args(c, x, y);
-  const int P = c.tile + kHalo;
-  if (c.n_own > 0) k_gather_tiles<<<c.max_segs, kTileThreads, rec_stage_bytes() + P * P * 8, s>>>(a);
+  if (c.n_own > 0) k_gather_walk<<<c.walk_grid, kTileThreads, walk_smem_bytes(c.tile), s>>>(a);
   if (c.n_large > 0) k_gather_large<<<c.n_large, 256, 0, s>>>(a);
 }
 

@@ -15,6 +15,7 @@
 
 #include <algorithm>
 #include <cmath>
+#include <cstdlib>
 #include <cstring>
 #include <numeric>
 #include <string>
@@ -321,12 +322,15 @@ dp_status build_wa(Ctx &c, const dp_netlist *nl, const std::vector<uint8_t> &mas
   c.n_wa_pins = (int32_t)pin_cell.size();
   {
     static WaCaps max_caps{4, 4, 4, 4};
+    static bool configured = false;
     WaCaps m{std::max(max_caps.pins, caps.pins), std::max(max_caps.nets, caps.nets),
              std::max(max_caps.groups, caps.groups), std::max(max_caps.far, caps.far)};
     if (wa_smem_bytes(m) > 227 * 1024) return fail(DP_ERR_UNSUPPORTED, "WA chunk staging exceeds shared memory");
-    if (m.pins != max_caps.pins || m.nets != max_caps.nets || m.groups != max_caps.groups || m.far != max_caps.far) {
+    if (!configured || m.pins != max_caps.pins || m.nets != max_caps.nets || m.groups != max_caps.groups ||
+        m.far != max_caps.far) {
       DP_CUDA(wa_configure(m));
       max_caps = m;
+      configured = true;
     }
     c.wa_caps = caps;
   }
@@ -340,6 +344,11 @@ dp_status build_wa(Ctx &c, const dp_netlist *nl, const std::vector<uint8_t> &mas
   if ((st = dev_upload(c, &c.d_pin_dy, pin_dy)) != DP_OK) return st;
   if ((st = dev_upload(c, &c.d_far_cells, far_cells)) != DP_OK) return st;
   // ---- big nets ----
+  // largest first: the longest CTAs start in the first wave
+  std::stable_sort(big.begin(), big.end(), [&](int32_t a, int32_t b) {
+    return nl->net_start[a + 1] - nl->net_start[a] > nl->net_start[b + 1] - nl->net_start[b];
+  });
+  c.big_stage = big.empty() ? 0 : std::min(kBigStage, nl->net_start[big[0] + 1] - nl->net_start[big[0]]);
   std::vector<int32_t> bstart{0}, bflags, bcell;
   std::vector<float> bw, bdx, bdy;
   for (int32_t e : big) {
@@ -394,7 +403,6 @@ dp_status build_density(Ctx &c, const dp_netlist *nl) {
   c.tiles_x = c.mx / c.tile;
   c.tiles_y = c.my / c.tile;
   const int ntiles = c.tiles_x * c.tiles_y;
-  c.max_segs = c.n_own / kSegCells + ntiles + 1;
   const size_t nb = (size_t)c.mx * c.my;
   dp_status st;
   if ((st = dev_upload(c, &c.d_cell_w, w)) != DP_OK) return st;
@@ -404,13 +412,10 @@ dp_status build_density(Ctx &c, const dp_netlist *nl) {
   DP_CUDA(cudaMemset(c.d_tile_cnt, 0, sizeof(int32_t) * ntiles));
   if ((st = dev_alloc(c, &c.d_tile_cursor, ntiles)) != DP_OK) return st;
   if ((st = dev_alloc(c, &c.d_tile_off, ntiles + 1)) != DP_OK) return st;
-  // sort records; padded by 4 so segment copies may round their range to 4-record multiples
+  // sort records; padded by 8 so staged copies may round their range to 4-record multiples
   if ((st = dev_alloc(c, &c.d_rec, c.n_own + 8)) != DP_OK) return st;
   if ((st = dev_alloc(c, &c.d_rec_rc, c.n_own + 8)) != DP_OK) return st;
   if ((st = dev_alloc(c, &c.d_rec_cell, c.n_own + 8)) != DP_OK) return st;
-  if ((st = dev_alloc(c, &c.d_segs, c.max_segs)) != DP_OK) return st;
-  if ((st = dev_alloc(c, &c.d_nsegs, 1)) != DP_OK) return st;
-  DP_CUDA(cudaMemset(c.d_nsegs, 0, sizeof(int32_t)));
   if ((st = dev_alloc(c, &c.d_rho, nb)) != DP_OK) return st;
   if ((st = dev_alloc(c, &c.d_t, nb)) != DP_OK) return st;
   if ((st = dev_alloc(c, &c.d_sx, nb)) != DP_OK) return st;
@@ -442,6 +447,8 @@ dp_status build_density(Ctx &c, const dp_netlist *nl) {
     max_tile = std::max(max_tile, c.tile);
     DP_CUDA(density_configure(max_tiles, max_tile));
   }
+  c.walk_grid = density_walk_grid(c.tile);
+  if (c.walk_grid <= 0) return fail(DP_ERR_CUDA, "density walker occupancy query failed");
   return DP_OK;
 }
 
@@ -522,6 +529,7 @@ dp_status create(const dp_netlist *nl, const dp_grid *grid, int device, int rank
   if ((st = dev_alloc(*c, &c->d_hgy, c->num_cells)) != DP_OK) return bail(st);
   if ((st = dev_alloc(*c, &c->d_hy, 2 * (size_t)c->num_cells)) != DP_OK) return bail(st);  // x then y
   c->d_hx = nullptr;
+  { const char *e = std::getenv("DP_SERIAL"); c->serial = e && e[0] == '1'; }
   if (cudaStreamCreateWithFlags(&c->s_wa, cudaStreamNonBlocking) != cudaSuccess ||
       cudaStreamCreateWithFlags(&c->s_den, cudaStreamNonBlocking) != cudaSuccess ||
       cudaEventCreateWithFlags(&c->ev_fork, cudaEventDisableTiming) != cudaSuccess ||
@@ -648,7 +656,7 @@ dp_status eval_impl(Ctx &c, const float *x, const float *y, float gamma, float l
     DP_CUDA(cudaEventRecord(c.ev_wa, c.s_wa));
   }
   if (do_den) {
-    DP_CUDA(cudaStreamWaitEvent(c.s_den, c.ev_fork, 0));
+    DP_CUDA(cudaStreamWaitEvent(c.s_den, (c.serial && do_wa) ? c.ev_wa : c.ev_fork, 0));
     dp_status st = density_chain(c, x, y);
     if (st != DP_OK) return st;
     DP_CUDA(cudaEventRecord(c.ev_den, c.s_den));

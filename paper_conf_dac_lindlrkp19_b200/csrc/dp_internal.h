@@ -21,16 +21,17 @@ constexpr int kWaPpl = 4;             // pin slots per lane (registers)
 constexpr int kWaMaxDeg = 128;        // nets up to this degree go through the chunk kernel (G <= 32)
 constexpr int kWaChunkPins = 2048;    // max pins per chunk (staged in shared memory)
 constexpr int kWaWindow = 1024;       // consecutive cells per chunk window held in shared memory
-constexpr int kBigThreads = 128;      // CTA-per-net kernel for nets > kWaMaxDeg
+constexpr int kBigThreads = 256;      // CTA-per-net kernel for nets > kWaMaxDeg
+constexpr int kBigStage = 4096;       // big-net pins whose exact positions stay in shared memory
 constexpr int kHpwlLimbs = 9;         // limbs 0..kHpwlLimbs (10) of 32-bit digits, LSB 2^-149 (reading A7)
 
 constexpr int kTile = 64;             // density tile = kTile x kTile bins (smaller maps: the map)
 constexpr int kHalo = 2;              // small-cell footprints extend <= 2 bins past their tile
-constexpr int kSegCells = 2048;       // cells per scatter/gather work segment (one CTA; load balance)
-constexpr int kSegChunk = 2048;       // records staged in shared memory at a time
+constexpr int kStageRecs = 1024;      // records per staging buffer of the scatter/gather walkers
+constexpr int kFlushRecs = 8192;      // a walker flushes its shared tile at least every 2^13 records
 // Tile bins accumulate each contribution v in (0, 1] as two native 32-bit shared atomics:
-// hi = floor(v 2^kTileHiBits) and lo = floor(frac 2^kTileLoBits); with <= kSegCells = 2^13
-// records per segment neither word can overflow (2^13 * 2^10 < 2^32, 2^13 * (2^19 - 1) < 2^32),
+// hi = floor(v 2^kTileHiBits) and lo = floor(frac 2^kTileLoBits); with <= kFlushRecs = 2^13
+// records between flushes neither word can overflow (2^13 * 2^10 < 2^32, 2^13 * (2^19 - 1) < 2^32),
 // and the pair resolves 2^-29.
 constexpr int kTileHiBits = 10;
 constexpr int kTileLoBits = 19;
@@ -66,13 +67,6 @@ struct WaCaps {
   int pins, nets, groups, far;
 };
 
-// Work segment of the density scatter/gather (built on device each evaluation).
-struct Segment {
-  int32_t tile;
-  int32_t begin, end;   // record range
-  int32_t pad;
-};
-
 struct Ctx {
   // ---- identity ----
   int device = 0;
@@ -100,6 +94,7 @@ struct Ctx {
   float *d_pin_dx = nullptr, *d_pin_dy = nullptr;
   // big nets (degree > kWaMaxDeg): plain CSR, one CTA per net
   int32_t n_big = 0;
+  int32_t big_stage = 0;            // staged pins per big-net CTA (min(max degree, kBigStage))
   int32_t *d_big_start = nullptr;   // [n_big + 1]
   int32_t *d_big_flags = nullptr;   // counted flag per big net
   float *d_big_w = nullptr;
@@ -118,9 +113,8 @@ struct Ctx {
   float4 *d_rec = nullptr;            // per slot: footprint box in tile-local bin units
   int2 *d_rec_rc = nullptr;           // per slot: (charge ratio r as float bits, i0 | j0 << 16)
   int32_t *d_rec_cell = nullptr;      // per slot: own cell index
-  Segment *d_segs = nullptr;
-  int32_t max_segs = 0;
-  int32_t *d_nsegs = nullptr;
+  bool serial = false;     // DP_SERIAL=1: density chain after WA (no stream overlap; measurement)
+  int32_t walk_grid = 0;   // CTAs of the persistent scatter / gather walkers (SMs x resident)
   unsigned long long *d_rho = nullptr;  // bin map, int64 fixed point in units of 2^-kRhoScaleLog2 (exact, deterministic)
   float *d_t = nullptr, *d_sx = nullptr, *d_sy = nullptr;
   float2 *d_xi = nullptr;
@@ -195,6 +189,7 @@ cudaError_t dct_configure(int mx, int my);
 cudaError_t wa_configure(const WaCaps &caps);
 int wa_smem_bytes(const WaCaps &caps);
 cudaError_t density_configure(int ntiles, int tile);
+int density_walk_grid(int tile);
 int density_launches(const Ctx &c);
 // NCCL (nccl_dyn.cpp)
 dp_status nccl_get_unique_id(void *out128);

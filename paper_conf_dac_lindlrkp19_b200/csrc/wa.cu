@@ -52,6 +52,7 @@ struct WaArgs {
   const int32_t *big_start, *big_flags, *big_cell;
   const float *big_w, *big_dx, *big_dy;
   int part_offset;
+  int big_stage;   // pins staged in shared memory per big-net CTA
   WaCaps caps;
 };
 
@@ -500,8 +501,8 @@ __global__ void __launch_bounds__(kWaThreads, 3) k_wa_chunks(WaArgs a) {
     }
   }
   const int nslots = L_.slots();
-  if (kGrad)
-    for (int i = tid; i < 2 * nslots; i += kWaThreads) s_g[i] = 0;
+  if (kGrad)   // 2 * nslots is a multiple of 8, s_g 16-byte aligned
+    for (int i = tid; i < nslots / 2; i += kWaThreads) reinterpret_cast<int4 *>(s_g)[i] = make_int4(0, 0, 0, 0);
   for (int i = (win_bulk ? wbulk : 0) + tid; i < ch.win_n; i += kWaThreads) {
     s_px[i] = __ldg(a.x + ch.win_lo + i);
     s_py[i] = __ldg(a.y + ch.win_lo + i);
@@ -509,10 +510,23 @@ __global__ void __launch_bounds__(kWaThreads, 3) k_wa_chunks(WaArgs a) {
   __syncthreads();   // barrier initialised before anyone waits on it
   mbar_wait(bar, 0);
   // far cells: positions gathered once per chunk
-  for (int f = tid; f < ch.far_n; f += kWaThreads) {
-    const int c = s_far[f];
-    s_px[kWaWindow + f] = __ldg(a.x + c);
-    s_py[kWaWindow + f] = __ldg(a.y + c);
+  for (int f0 = tid; f0 < ch.far_n; f0 += 4 * kWaThreads) {   // 8 loads in flight per thread
+    float fx[4], fy[4];
+#pragma unroll
+    for (int k = 0; k < 4; k++) {
+      const int f = f0 + k * kWaThreads;
+      const int c = f < ch.far_n ? s_far[f] : 0;
+      fx[k] = __ldg(a.x + c);
+      fy[k] = __ldg(a.y + c);
+    }
+#pragma unroll
+    for (int k = 0; k < 4; k++) {
+      const int f = f0 + k * kWaThreads;
+      if (f < ch.far_n) {
+        s_px[kWaWindow + f] = fx[k];
+        s_py[kWaWindow + f] = fy[k];
+      }
+    }
   }
   __syncthreads();
 
@@ -581,26 +595,50 @@ __device__ __forceinline__ void ext_merge(Ext &e, const Ext &o) {
   if (pair_gt(e.yh, e.yl, o.yh, o.yl)) { e.yh = o.yh; e.yl = o.yl; }
 }
 
+// Exact shifted coordinates of big-net pin p: (hx, lx) = TwoSum(x_c, dx), (hy, ly) likewise.
+__device__ __forceinline__ float4 big_pin(const WaArgs &a, int c, int s) {
+  float4 v;
+  two_sum(__ldg(a.x + c), __ldg(a.big_dx + s), v.x, v.y);
+  two_sum(__ldg(a.y + c), __ldg(a.big_dy + s), v.z, v.w);
+  return v;
+}
+
+// CTA per net of degree > kWaMaxDeg (largest first).  Pass 1 loads every pin once (4 loads in
+// flight per thread) and keeps the exact coordinates in shared memory (nets up to kBigStage
+// pins; larger nets reload), pass 2 forms the eq-6 sums, pass 3 the gradient.
 template <int MODE>
 __global__ void __launch_bounds__(kBigThreads) k_wa_big(WaArgs a) {
   constexpr bool kGrad = MODE != 2;
   constexpr bool kHpwl = MODE != 0;
+  extern __shared__ float4 s_pin[];
   const int net = blockIdx.x, tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   constexpr int NW = kBigThreads / 32;
   const int s0 = a.big_start[net], d = a.big_start[net + 1] - s0;
+  const bool staged = d <= a.big_stage;
   const int counted = a.big_flags[net];
   const float we = a.has_w ? a.big_w[net] : 1.f;
   __shared__ Ext s_ext[NW];
   __shared__ float s_sum[NW][8];
 
   Ext e{-INFINITY, 0.f, INFINITY, 0.f, -INFINITY, 0.f, INFINITY, 0.f};
-  for (int p = tid; p < d; p += kBigThreads) {
-    const int c = a.big_cell[s0 + p] & 0x7fffffff;
-    float h, l, H, Lo;
-    two_sum(__ldg(a.x + c), a.big_dx[s0 + p], h, l);
-    two_sum(__ldg(a.y + c), a.big_dy[s0 + p], H, Lo);
-    Ext o{h, l, h, l, H, Lo, H, Lo};
-    ext_merge(e, o);
+  for (int p0 = tid; p0 < d; p0 += 4 * kBigThreads) {
+    int c[4];
+#pragma unroll
+    for (int k = 0; k < 4; k++) {
+      const int p = p0 + k * kBigThreads;
+      c[k] = p < d ? (__ldg(a.big_cell + s0 + p) & 0x7fffffff) : -1;
+    }
+    float4 v[4];
+#pragma unroll
+    for (int k = 0; k < 4; k++)
+      if (c[k] >= 0) v[k] = big_pin(a, c[k], s0 + p0 + k * kBigThreads);
+#pragma unroll
+    for (int k = 0; k < 4; k++) {
+      if (c[k] < 0) continue;
+      if (staged) s_pin[p0 + k * kBigThreads] = v[k];
+      const Ext o{v[k].x, v[k].y, v[k].x, v[k].y, v[k].z, v[k].w, v[k].z, v[k].w};
+      ext_merge(e, o);
+    }
   }
 #pragma unroll
   for (int o = 16; o > 0; o >>= 1) {
@@ -612,7 +650,7 @@ __global__ void __launch_bounds__(kBigThreads) k_wa_big(WaArgs a) {
     ext_merge(e, t);
   }
   if (lane == 0) s_ext[warp] = e;
-  __syncthreads();
+  __syncthreads();   // also publishes s_pin
   e = s_ext[0];
   for (int w = 1; w < NW; w++) ext_merge(e, s_ext[w]);
 
@@ -628,14 +666,11 @@ __global__ void __launch_bounds__(kBigThreads) k_wa_big(WaArgs a) {
   if (kGrad) {
     float sm[8] = {0, 0, 0, 0, 0, 0, 0, 0};  // bxp cxp bxm cxm byp cyp bym cym
     for (int p = tid; p < d; p += kBigThreads) {
-      const int c = a.big_cell[s0 + p] & 0x7fffffff;
-      float hx, lx, hy, ly;
-      two_sum(__ldg(a.x + c), a.big_dx[s0 + p], hx, lx);
-      two_sum(__ldg(a.y + c), a.big_dy[s0 + p], hy, ly);
-      const float lxp = __fadd_rn(__fsub_rn(hx, e.Xh), __fsub_rn(lx, e.Xl));
-      const float lxm = __fadd_rn(__fsub_rn(hx, e.xh), __fsub_rn(lx, e.xl));
-      const float lyp = __fadd_rn(__fsub_rn(hy, e.Yh), __fsub_rn(ly, e.Yl));
-      const float lym = __fadd_rn(__fsub_rn(hy, e.yh), __fsub_rn(ly, e.yl));
+      const float4 v = staged ? s_pin[p] : big_pin(a, __ldg(a.big_cell + s0 + p) & 0x7fffffff, s0 + p);
+      const float lxp = __fadd_rn(__fsub_rn(v.x, e.Xh), __fsub_rn(v.y, e.Xl));
+      const float lxm = __fadd_rn(__fsub_rn(v.x, e.xh), __fsub_rn(v.y, e.xl));
+      const float lyp = __fadd_rn(__fsub_rn(v.z, e.Yh), __fsub_rn(v.w, e.Yl));
+      const float lym = __fadd_rn(__fsub_rn(v.z, e.yh), __fsub_rn(v.w, e.yl));
       const float axp = ex2(lxp * a.k2), axm = ex2(-lxm * a.k2);
       const float ayp = ex2(lyp * a.k2), aym = ex2(-lym * a.k2);
       sm[0] += axp; sm[1] += lxp * axp; sm[2] += axm; sm[3] += lxm * axm;
@@ -646,7 +681,6 @@ __global__ void __launch_bounds__(kBigThreads) k_wa_big(WaArgs a) {
 #pragma unroll
       for (int o = 16; o > 0; o >>= 1) sm[k] += __shfl_xor_sync(0xffffffffu, sm[k], o);
     }
-    __syncthreads();
     if (lane == 0)
 #pragma unroll
       for (int k = 0; k < 8; k++) s_sum[warp][k] = sm[k];
@@ -665,15 +699,13 @@ __global__ void __launch_bounds__(kBigThreads) k_wa_big(WaArgs a) {
       wl_acc = (double)(we * ((spanx + mxp - mxm) + (spany + myp - mym)));
     }
     for (int p = tid; p < d; p += kBigThreads) {
-      const int raw = a.big_cell[s0 + p];
+      const int raw = __ldg(a.big_cell + s0 + p);
       if (raw < 0) continue;
-      float hx, lx, hy, ly;
-      two_sum(__ldg(a.x + raw), a.big_dx[s0 + p], hx, lx);
-      two_sum(__ldg(a.y + raw), a.big_dy[s0 + p], hy, ly);
-      const float lxp = __fadd_rn(__fsub_rn(hx, e.Xh), __fsub_rn(lx, e.Xl));
-      const float lxm = __fadd_rn(__fsub_rn(hx, e.xh), __fsub_rn(lx, e.xl));
-      const float lyp = __fadd_rn(__fsub_rn(hy, e.Yh), __fsub_rn(ly, e.Yl));
-      const float lym = __fadd_rn(__fsub_rn(hy, e.yh), __fsub_rn(ly, e.yl));
+      const float4 v = staged ? s_pin[p] : big_pin(a, raw, s0 + p);
+      const float lxp = __fadd_rn(__fsub_rn(v.x, e.Xh), __fsub_rn(v.y, e.Xl));
+      const float lxm = __fadd_rn(__fsub_rn(v.x, e.xh), __fsub_rn(v.y, e.xl));
+      const float lyp = __fadd_rn(__fsub_rn(v.z, e.Yh), __fsub_rn(v.w, e.Yl));
+      const float lym = __fadd_rn(__fsub_rn(v.z, e.yh), __fsub_rn(v.w, e.yl));
       const float axp = ex2(lxp * a.k2), axm = ex2(-lxm * a.k2);
       const float ayp = ex2(lyp * a.k2), aym = ex2(-lym * a.k2);
       const float gx = we * (axp * ibxp * (1.f + (lxp - mxp) * a.inv_gamma) -
@@ -692,7 +724,7 @@ template <int MODE>
 void launch_mode(const Ctx &c, const WaArgs &a, cudaStream_t s) {
   const WaSmem L{a.caps};
   if (c.n_chunks > 0) k_wa_chunks<MODE><<<c.n_chunks, kWaThreads, L.bytes(), s>>>(a);
-  if (c.n_big > 0) k_wa_big<MODE><<<c.n_big, kBigThreads, 0, s>>>(a);
+  if (c.n_big > 0) k_wa_big<MODE><<<c.n_big, kBigThreads, 16 * a.big_stage, s>>>(a);
 }
 
 }  // namespace
@@ -705,7 +737,13 @@ cudaError_t wa_configure(const WaCaps &caps) {
   if (e != cudaSuccess) return e;
   e = cudaFuncSetAttribute(k_wa_chunks<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, b);
   if (e != cudaSuccess) return e;
-  return cudaFuncSetAttribute(k_wa_chunks<2>, cudaFuncAttributeMaxDynamicSharedMemorySize, b);
+  e = cudaFuncSetAttribute(k_wa_chunks<2>, cudaFuncAttributeMaxDynamicSharedMemorySize, b);
+  if (e != cudaSuccess) return e;
+  e = cudaFuncSetAttribute(k_wa_big<0>, cudaFuncAttributeMaxDynamicSharedMemorySize, 16 * kBigStage);
+  if (e != cudaSuccess) return e;
+  e = cudaFuncSetAttribute(k_wa_big<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, 16 * kBigStage);
+  if (e != cudaSuccess) return e;
+  return cudaFuncSetAttribute(k_wa_big<2>, cudaFuncAttributeMaxDynamicSharedMemorySize, 16 * kBigStage);
 }
 
 void launch_wa(const Ctx &c, const float *x, const float *y, float gamma, bool hpwl_only, bool with_hpwl,
@@ -735,6 +773,7 @@ void launch_wa(const Ctx &c, const float *x, const float *y, float gamma, bool h
   a.big_dx = c.d_big_dx;
   a.big_dy = c.d_big_dy;
   a.part_offset = c.n_chunks;
+  a.big_stage = c.big_stage;
   a.caps = c.wa_caps;
   if (hpwl_only)
     launch_mode<2>(c, a, s);

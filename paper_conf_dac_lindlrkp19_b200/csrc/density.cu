@@ -93,46 +93,35 @@ __device__ __forceinline__ int small_tile(const DenArgs &a, const Foot &f, int &
   return (bx0 >> a.tile_log2) * a.tiles_y + (by0 >> a.tile_log2);
 }
 
-// Stage the x, y, w, h of own cells [i0, i0 + n) (n <= kCountCells) in shared memory: bulk async
-// copies of the 16-byte aligned prefix (one elected thread, one mbarrier), plain loads for the
-// rest (ragged tail, or a caller x / y that is not 16-byte aligned).  Returns after the data is
-// visible to the whole CTA.
-struct CellStage {
-  float x[kCountCells], y[kCountCells], w[kCountCells], h[kCountCells];
-  uint64_t bar;
-};
+// Each thread of a count / place CTA holds kCellsPerThread cells (cell i0 + k * blockDim + tid,
+// coalesced loads, all issued before the first use); out-of-range cells are empty.
+constexpr int kCellsPerThread = kCountCells / kCountThreads;
 
-__device__ __forceinline__ void stage_cells(const DenArgs &a, CellStage &st, int i0, int n) {
-  const float *gx = a.x + a.cell_begin + i0, *gy = a.y + a.cell_begin + i0;
-  const bool ok = aligned16(gx) && aligned16(gy) && aligned16(a.w + i0) && aligned16(a.h + i0);
-  const int nb = ok ? (n & ~3) : 0;
-  if (threadIdx.x == 0 && nb > 0) {
-    mbar_init(&st.bar);
-    mbar_expect_tx(&st.bar, 16u * nb);
-    bulk_g2s(st.x, gx, 4u * nb, &st.bar);
-    bulk_g2s(st.y, gy, 4u * nb, &st.bar);
-    bulk_g2s(st.w, a.w + i0, 4u * nb, &st.bar);
-    bulk_g2s(st.h, a.h + i0, 4u * nb, &st.bar);
+__device__ __forceinline__ void load_cells(const DenArgs &a, int i0, float (&x)[kCellsPerThread],
+                                           float (&y)[kCellsPerThread], float (&w)[kCellsPerThread],
+                                           float (&h)[kCellsPerThread]) {
+#pragma unroll
+  for (int k = 0; k < kCellsPerThread; k++) {
+    const int i = i0 + k * kCountThreads + threadIdx.x;
+    const bool ok = i < a.n_own;
+    x[k] = ok ? __ldg(a.x + a.cell_begin + i) : 0.f;
+    y[k] = ok ? __ldg(a.y + a.cell_begin + i) : 0.f;
+    w[k] = ok ? __ldg(a.w + i) : 0.f;
+    h[k] = ok ? __ldg(a.h + i) : 0.f;
   }
-  for (int i = nb + threadIdx.x; i < n; i += blockDim.x) {
-    st.x[i] = __ldg(gx + i);
-    st.y[i] = __ldg(gy + i);
-    st.w[i] = __ldg(a.w + i0 + i);
-    st.h[i] = __ldg(a.h + i0 + i);
-  }
-  __syncthreads();
-  if (nb > 0) mbar_wait(&st.bar, 0);
 }
 
-// D1: per-CTA shared histogram of tile ids over a staged block of cells
+// D1: per-CTA shared histogram of tile ids
 __global__ void __launch_bounds__(kCountThreads) k_count(DenArgs a) {
   extern __shared__ int s_hist[];
-  __shared__ CellStage st;
-  const int i0 = blockIdx.x * kCountCells, n = min(kCountCells, a.n_own - i0);
+  const int i0 = blockIdx.x * kCountCells;
   for (int t = threadIdx.x; t < a.ntiles; t += kCountThreads) s_hist[t] = 0;
-  stage_cells(a, st, i0, n);
-  for (int i = threadIdx.x; i < n; i += kCountThreads) {
-    const Foot f = footprint_v(a, st.x[i], st.y[i], st.w[i], st.h[i]);
+  float x[kCellsPerThread], y[kCellsPerThread], w[kCellsPerThread], h[kCellsPerThread];
+  load_cells(a, i0, x, y, w, h);
+  __syncthreads();
+#pragma unroll
+  for (int k = 0; k < kCellsPerThread; k++) {
+    const Foot f = footprint_v(a, x[k], y[k], w[k], h[k]);
     if (f.empty || f.large) continue;
     int bx0, by0;
     atomicAdd(&s_hist[small_tile(a, f, bx0, by0)], 1);
@@ -181,10 +170,11 @@ __global__ void __launch_bounds__(1024) k_scan(DenArgs a) {
   if (threadIdx.x == T - 1) a.tile_off[a.ntiles] = off_c;
 }
 
-// D3: same staged block as D1.  Pass 1: shared histogram; local exclusive scan (the block's
-// records in tile order) and one global reservation per non-empty tile.  Pass 2: each cell's
-// record goes to shared memory at its tile-ordered local slot; finally the block writes its
-// records out in contiguous per-tile runs (random per-record stores were measured 3x slower).
+// D3: the same cells as D1, footprints computed once and held in registers.  The shared
+// histogram's atomicAdd returns each cell's rank inside its tile; a block scan of the histogram
+// (with one global reservation per non-empty tile) gives the local tile-ordered slots; records
+// are assembled in shared memory and written out in contiguous per-tile runs (random
+// per-record stores were measured 3x slower).
 struct PlaceOut {
   float4 rec[kCountCells];
   int2 rc[kCountCells];
@@ -192,27 +182,41 @@ struct PlaceOut {
   int tile[kCountCells];
 };
 
-int place_smem_bytes(int ntiles) { return (int)sizeof(PlaceOut) + 12 * ntiles; }
+int place_smem_bytes(int ntiles) { return (int)sizeof(PlaceOut) + 8 * ntiles; }
 
 __global__ void __launch_bounds__(kCountThreads) k_place(DenArgs a) {
   extern __shared__ __align__(16) unsigned char psm[];
   PlaceOut &po = *reinterpret_cast<PlaceOut *>(psm);
   int *s_hist = reinterpret_cast<int *>(psm + sizeof(PlaceOut));   // [ntiles] counts -> local offsets
   int *s_base = s_hist + a.ntiles;                                  // [ntiles] global bases
-  int *s_rank = s_base + a.ntiles;                                  // [ntiles] running local rank
-  __shared__ CellStage st;
   __shared__ int s_warp[kCountThreads / 32];
-  const int i0 = blockIdx.x * kCountCells, n = min(kCountCells, a.n_own - i0);
-  for (int t = threadIdx.x; t < a.ntiles; t += kCountThreads) {
-    s_hist[t] = 0;
-    s_rank[t] = 0;
-  }
-  stage_cells(a, st, i0, n);
-  for (int i = threadIdx.x; i < n; i += kCountThreads) {
-    const Foot f = footprint_v(a, st.x[i], st.y[i], st.w[i], st.h[i]);
-    if (f.large || f.empty) continue;
-    int bx0, by0;
-    atomicAdd(&s_hist[small_tile(a, f, bx0, by0)], 1);
+  const int i0 = blockIdx.x * kCountCells;
+  for (int t = threadIdx.x; t < a.ntiles; t += kCountThreads) s_hist[t] = 0;
+  float x[kCellsPerThread], y[kCellsPerThread], w[kCellsPerThread], h[kCellsPerThread];
+  load_cells(a, i0, x, y, w, h);
+  __syncthreads();
+  float4 rec[kCellsPerThread];
+  int rcy[kCellsPerThread], tl[kCellsPerThread], rank[kCellsPerThread];
+  float rr[kCellsPerThread];
+  const int mask = a.tile - 1;
+#pragma unroll
+  for (int k = 0; k < kCellsPerThread; k++) {
+    const int i = i0 + k * kCountThreads + threadIdx.x;
+    const Foot f = footprint_v(a, x[k], y[k], w[k], h[k]);
+    tl[k] = -1;
+    if (i >= a.n_own || f.large) continue;
+    if (f.empty) {
+      a.force[i] = make_float2(0.f, 0.f);
+      continue;
+    }
+    int bi, bj;
+    tl[k] = small_tile(a, f, bi, bj);
+    rank[k] = atomicAdd(&s_hist[tl[k]], 1);
+    // bin-local fractions (|v| < 3): fp32 keeps ~2e-7 bin absolute precision, which the force
+    // gather needs where large opposite bin fields cancel (the 'initial' placement)
+    rec[k] = make_float4((float)(f.lo_x - bi), (float)(f.lo_y - bj), (float)(f.hi_x - bi), (float)(f.hi_y - bj));
+    rr[k] = f.r;
+    rcy[k] = (bi & mask) | ((bj & mask) << 16);
   }
   __syncthreads();
   // reservation + block exclusive scan of the histogram (tiles split evenly over the threads)
@@ -227,13 +231,13 @@ __global__ void __launch_bounds__(kCountThreads) k_place(DenArgs a) {
       sum += cnt;
     }
   }
-  int incl = warp_incl_scan(sum, lane);
+  const int incl = warp_incl_scan(sum, lane);
   if (lane == 31) s_warp[warp] = incl;
   __syncthreads();
   if (warp == 0) {
     const int v = lane < kCountThreads / 32 ? s_warp[lane] : 0;
-    const int w = warp_incl_scan(v, lane);
-    if (lane < kCountThreads / 32) s_warp[lane] = w;
+    const int ws = warp_incl_scan(v, lane);
+    if (lane < kCountThreads / 32) s_warp[lane] = ws;
   }
   __syncthreads();
   int run = (warp ? s_warp[warp - 1] : 0) + incl - sum;
@@ -246,24 +250,14 @@ __global__ void __launch_bounds__(kCountThreads) k_place(DenArgs a) {
     }
   }
   __syncthreads();
-  for (int k = threadIdx.x; k < n; k += kCountThreads) {
-    const int i = i0 + k;
-    const Foot f = footprint_v(a, st.x[k], st.y[k], st.w[k], st.h[k]);
-    if (f.large) continue;
-    if (f.empty) {
-      a.force[i] = make_float2(0.f, 0.f);
-      continue;
-    }
-    int bi, bj;
-    const int t = small_tile(a, f, bi, bj);
-    const int slot = s_hist[t] + atomicAdd(&s_rank[t], 1);
-    const int mask = a.tile - 1;
-    // bin-local fractions (|v| < 3): fp32 keeps ~2e-7 bin absolute precision, which the force
-    // gather needs where large opposite bin fields cancel (the 'initial' placement)
-    po.rec[slot] = make_float4((float)(f.lo_x - bi), (float)(f.lo_y - bj), (float)(f.hi_x - bi), (float)(f.hi_y - bj));
-    po.rc[slot] = make_int2(__float_as_int(f.r), (bi & mask) | ((bj & mask) << 16));
-    po.cell[slot] = i;
-    po.tile[slot] = t;
+#pragma unroll
+  for (int k = 0; k < kCellsPerThread; k++) {
+    if (tl[k] < 0) continue;
+    const int slot = s_hist[tl[k]] + rank[k];
+    po.rec[slot] = rec[k];
+    po.rc[slot] = make_int2(__float_as_int(rr[k]), rcy[k]);
+    po.cell[slot] = i0 + k * kCountThreads + threadIdx.x;
+    po.tile[slot] = tl[k];
   }
   __syncthreads();
   const int total = s_warp[kCountThreads / 32 - 1];
@@ -276,54 +270,43 @@ __global__ void __launch_bounds__(kCountThreads) k_place(DenArgs a) {
   }
 }
 
-// Double-buffered record staging: buffer b holds up to kStageRecs records of rec (16 B),
-// rec_rc (8 B) and rec_cell (4 B); each buffer completes on its own mbarrier.  The copied range
-// is rounded out to 4-record multiples (the record arrays are padded by 8 records).
+// Record staging ring: kStages buffers of up to kStageRecs records of rec (16 B), rec_rc (8 B)
+// and rec_cell (4 B), each completing on its own mbarrier.  Thread 0 owns the walker and keeps
+// kStages - 1 chunks in flight; the chunk descriptors live in shared memory next to the data.
+// The copied range is rounded out to 4-record multiples (the record arrays are padded by 8).
+constexpr int kStages = 4;
 struct RecBuf {
   float4 rec[kStageRecs + 8];
   int2 rc[kStageRecs + 8];
   int cell[kStageRecs + 8];
 };
+struct WalkChunk {
+  int begin, end, tile, off;
+};
 struct RecStage {
-  RecBuf buf[2];
-  uint64_t bar[2];
+  RecBuf buf[kStages];
+  WalkChunk ch[kStages];
+  uint64_t bar[kStages];
   uint64_t bar_xi;
 };
 
 __host__ __device__ constexpr int rec_stage_bytes() { return (int)((sizeof(RecStage) + 15) & ~(size_t)15); }
 int walk_smem_bytes(int tile) { return rec_stage_bytes() + (tile + kHalo) * (tile + kHalo) * 8; }
 
-// Issue (thread 0) the copies of records [begin, end) into buffer b; returns the offset of the
-// first record inside the buffer (all threads).
-__device__ __forceinline__ int stage_records(const DenArgs &a, RecStage &st, int b, int begin, int end,
-                                             bool with_cell) {
-  const int b0 = begin & ~3, e0 = (end + 3) & ~3, n = e0 - b0;
-  if (threadIdx.x == 0) {
-    RecBuf &B = st.buf[b];
-    mbar_expect_tx(&st.bar[b], (unsigned)n * (with_cell ? 28u : 24u));
-    bulk_g2s(B.rec, a.rec + b0, 16u * n, &st.bar[b]);
-    bulk_g2s(B.rc, a.rec_rc + b0, 8u * n, &st.bar[b]);
-    if (with_cell) bulk_g2s(B.cell, a.rec_cell + b0, 4u * n, &st.bar[b]);
-  }
-  return begin - b0;
-}
-
 // A walker's slice [rb, re) of the tile-ordered small-cell records, cut into chunks of at most
-// kStageRecs records that never straddle a tile.  Every thread runs the same bookkeeping
-// (uniform loads of tile_off).
-struct WalkChunk {
-  int begin, end, tile, off;
-};
+// kStageRecs records that never straddle a tile.
 struct Walker {
   int cur, re, t, tend;
 };
 
-__device__ __forceinline__ bool walk_init(const DenArgs &a, Walker &w) {
+__device__ __forceinline__ void walk_init(const DenArgs &a, Walker &w) {
   const int N = a.tile_off[a.ntiles];
   const int G = gridDim.x;
   w.cur = (int)(((long long)N * blockIdx.x) / G);
   w.re = (int)(((long long)N * (blockIdx.x + 1)) / G);
-  if (w.cur >= w.re) return false;
+  w.t = 0;
+  w.tend = 0;
+  if (w.cur >= w.re) return;
   int lo = 0, hi = a.ntiles;   // largest t with tile_off[t] <= cur (then tile_off[t + 1] > cur)
   while (hi - lo > 1) {
     const int mid = (lo + hi) >> 1;
@@ -331,20 +314,36 @@ __device__ __forceinline__ bool walk_init(const DenArgs &a, Walker &w) {
   }
   w.t = lo;
   w.tend = a.tile_off[lo + 1];
-  return true;
 }
 
-__device__ __forceinline__ WalkChunk walk_next(const DenArgs &a, Walker &w) {
+// (thread 0) next chunk of the slice -> descriptor slot b, copies issued on bar[b]
+__device__ __forceinline__ void walk_issue(const DenArgs &a, Walker &w, RecStage &st, int b, bool with_cell) {
   WalkChunk c;
   c.begin = c.end = w.cur;
   c.tile = w.t;
   c.off = 0;
-  if (w.cur >= w.re) return c;
-  while (w.tend <= w.cur) w.tend = a.tile_off[++w.t + 1];   // skip finished / empty tiles
-  c.tile = w.t;
-  c.end = min(min(w.cur + kStageRecs, w.tend), w.re);
-  w.cur = c.end;
-  return c;
+  if (w.cur < w.re) {
+    while (w.tend <= w.cur) w.tend = a.tile_off[++w.t + 1];   // skip finished / empty tiles
+    c.tile = w.t;
+    c.end = min(min(w.cur + kStageRecs, w.tend), w.re);
+    w.cur = c.end;
+    const int b0 = c.begin & ~3, e0 = (c.end + 3) & ~3, n = e0 - b0;
+    c.off = c.begin - b0;
+    RecBuf &B = st.buf[b];
+    mbar_expect_tx(&st.bar[b], (unsigned)n * (with_cell ? 28u : 24u));
+    bulk_g2s(B.rec, a.rec + b0, 16u * n, &st.bar[b]);
+    bulk_g2s(B.rc, a.rec_rc + b0, 8u * n, &st.bar[b]);
+    if (with_cell) bulk_g2s(B.cell, a.rec_cell + b0, 4u * n, &st.bar[b]);
+  }
+  st.ch[b] = c;
+}
+
+// (thread 0) barriers + the first kStages - 1 chunks; the caller synchronises
+__device__ __forceinline__ void walk_start(const DenArgs &a, Walker &w, RecStage &st, bool with_cell) {
+  walk_init(a, w);
+  for (int b = 0; b < kStages; b++) mbar_init(&st.bar[b]);
+  mbar_init(&st.bar_xi);
+  for (int b = 0; b < kStages - 1; b++) walk_issue(a, w, st, b, with_cell);
 }
 
 // overlaps (bin units) of a record's footprint with the 3 bins from its first bin, per axis;
@@ -383,26 +382,21 @@ __global__ void __launch_bounds__(kTileThreads) k_scatter_walk(DenArgs a) {
   RecStage &st = *reinterpret_cast<RecStage *>(dsm);
   unsigned *s_hi = reinterpret_cast<unsigned *>(dsm + rec_stage_bytes());   // 2^-kTileHiBits units
   unsigned *s_lo = s_hi + (a.tile + kHalo) * (a.tile + kHalo);               // 2^-(hi + lo bits) units
-  Walker w;
-  if (!walk_init(a, w)) return;
   const int P = a.tile + kHalo;
-  if (threadIdx.x == 0) {
-    mbar_init(&st.bar[0]);
-    mbar_init(&st.bar[1]);
-  }
+  Walker w;
+  if (threadIdx.x == 0) walk_start(a, w, st, false);
   for (int k = threadIdx.x; k < P * P; k += blockDim.x) {
     s_hi[k] = 0u;
     s_lo[k] = 0u;
   }
   __syncthreads();
   const float scale_hi = (float)(1 << kTileHiBits), scale_lo = (float)(1 << kTileLoBits);
-  WalkChunk cc = walk_next(a, w);
-  cc.off = stage_records(a, st, 0, cc.begin, cc.end, false);
-  int cur_tile = cc.tile, acc = 0;
-  for (int c = 0; cc.begin < cc.end; c++) {
-    const int b = c & 1;
-    WalkChunk nx = walk_next(a, w);   // prefetch into the other buffer (freed by the last sync)
-    if (nx.end > nx.begin) nx.off = stage_records(a, st, b ^ 1, nx.begin, nx.end, false);
+  int cur_tile = st.ch[0].tile, acc = 0;
+  for (int c = 0;; c++) {
+    const int b = c % kStages;
+    const WalkChunk cc = st.ch[b];
+    if (cc.begin >= cc.end) break;
+    if (threadIdx.x == 0) walk_issue(a, w, st, (c + kStages - 1) % kStages, false);   // freed by the last sync
     const int n = cc.end - cc.begin;
     if (cc.tile != cur_tile || acc + n > kFlushRecs) {
       flush_tile(a, s_hi, s_lo, cur_tile);
@@ -411,7 +405,7 @@ __global__ void __launch_bounds__(kTileThreads) k_scatter_walk(DenArgs a) {
       acc = 0;
     }
     acc += n;
-    mbar_wait(&st.bar[b], (c >> 1) & 1);
+    mbar_wait(&st.bar[b], (c / kStages) & 1);
     const RecBuf &B = st.buf[b];
     for (int k = threadIdx.x; k < n; k += blockDim.x) {
       const float4 q = B.rec[cc.off + k];
@@ -436,7 +430,6 @@ __global__ void __launch_bounds__(kTileThreads) k_scatter_walk(DenArgs a) {
       }
     }
     __syncthreads();   // buffer b consumed before it is refilled; tile complete before a flush
-    cc = nx;
   }
   flush_tile(a, s_hi, s_lo, cur_tile);
 }
@@ -466,30 +459,24 @@ __global__ void __launch_bounds__(kTileThreads) k_gather_walk(DenArgs a) {
   extern __shared__ __align__(16) unsigned char dsm[];
   RecStage &st = *reinterpret_cast<RecStage *>(dsm);
   float2 *s_xi = reinterpret_cast<float2 *>(dsm + rec_stage_bytes());
-  Walker w;
-  if (!walk_init(a, w)) return;
   const int P = a.tile + kHalo;
-  if (threadIdx.x == 0) {
-    mbar_init(&st.bar[0]);
-    mbar_init(&st.bar[1]);
-    mbar_init(&st.bar_xi);
-  }
-  __syncthreads();   // barriers initialised
-  WalkChunk cc = walk_next(a, w);
-  cc.off = stage_records(a, st, 0, cc.begin, cc.end, true);
+  Walker w;
+  if (threadIdx.x == 0) walk_start(a, w, st, true);
+  __syncthreads();   // barriers initialised, first descriptors visible
   int cur_tile = -1;
   unsigned xi_phase = 0;
   const float area = (float)(a.bx * a.by);
-  for (int c = 0; cc.begin < cc.end; c++) {
-    const int b = c & 1;
-    WalkChunk nx = walk_next(a, w);   // prefetch into the other buffer (freed by the last sync)
-    if (nx.end > nx.begin) nx.off = stage_records(a, st, b ^ 1, nx.begin, nx.end, true);
+  for (int c = 0;; c++) {
+    const int b = c % kStages;
+    const WalkChunk cc = st.ch[b];
+    if (cc.begin >= cc.end) break;
+    if (threadIdx.x == 0) walk_issue(a, w, st, (c + kStages - 1) % kStages, true);
     if (cc.tile != cur_tile) {   // the previous iteration's sync freed the field tile
       load_xi_tile(a, st, s_xi, cc.tile, xi_phase);
       xi_phase ^= 1u;
       cur_tile = cc.tile;
     }
-    mbar_wait(&st.bar[b], (c >> 1) & 1);
+    mbar_wait(&st.bar[b], (c / kStages) & 1);
     const RecBuf &B = st.buf[b];
     const int n = cc.end - cc.begin;
     for (int k = threadIdx.x; k < n; k += blockDim.x) {
@@ -517,7 +504,6 @@ __global__ void __launch_bounds__(kTileThreads) k_gather_walk(DenArgs a) {
       a.force[B.cell[cc.off + k]] = make_float2(-area * r * fx, -area * r * fy);
     }
     __syncthreads();
-    cc = nx;
   }
 }
 

@@ -365,6 +365,8 @@ dp_status build_wa(Ctx &c, const dp_netlist *nl, const std::vector<uint8_t> &mas
     bw.push_back(nl->net_weight ? nl->net_weight[e] : 1.f);
   }
   c.n_big = (int32_t)big.size();
+  c.n_huge = 0;
+  while (c.n_huge < c.n_big && nl->net_start[big[c.n_huge] + 1] - nl->net_start[big[c.n_huge]] > kWarpNetMax) c.n_huge++;
   if ((st = dev_upload(c, &c.d_big_start, bstart)) != DP_OK) return st;
   if ((st = dev_upload(c, &c.d_big_flags, bflags)) != DP_OK) return st;
   if ((st = dev_upload(c, &c.d_big_w, bw)) != DP_OK) return st;
@@ -516,7 +518,7 @@ dp_status create(const dp_netlist *nl, const dp_grid *grid, int device, int rank
   };
   if ((st = build_wa(*c, nl, mask)) != DP_OK) return bail(st);
   if ((st = build_density(*c, nl)) != DP_OK) return bail(st);
-  c->n_wa_part = c->n_chunks + c->n_big;
+  c->n_wa_part = c->n_chunks + c->n_huge + (c->n_big - c->n_huge + kWarpNetThreads / 32 - 1) / (kWarpNetThreads / 32);
   c->n_en_part = c->my / 2;   // = CTAs of the column-fields kernel (2-column slabs)
   if ((st = dev_alloc(*c, &c->d_g2, c->num_cells)) != DP_OK) return bail(st);
   if (cudaMemset(c->d_g2, 0, sizeof(float2) * c->num_cells) != cudaSuccess) return bail(fail(DP_ERR_CUDA, "memset"));
@@ -537,7 +539,7 @@ dp_status create(const dp_netlist *nl, const dp_grid *grid, int device, int rank
       cudaEventCreateWithFlags(&c->ev_den, cudaEventDisableTiming) != cudaSuccess ||
       cudaEventCreateWithFlags(&c->ev_done, cudaEventDisableTiming) != cudaSuccess)
     return bail(fail(DP_ERR_CUDA, "stream/event creation failed"));
-  const int wa_k = (c->n_chunks > 0) + (c->n_big > 0);
+  const int wa_k = (c->n_chunks + c->n_big > 0) ? 1 : 0;   // one kernel: big nets, warp nets, chunks
   c->launches_eval = wa_k + density_launches(*c) + 3 /* T1 T2 T3 */ + 2 /* combine, finalize */;
   c->launches_eval_hpwl = c->launches_eval;
   if (world > 1 && nccl_id) {

@@ -23,11 +23,13 @@ constexpr int kWaChunkPins = 2048;    // max pins per chunk (staged in shared me
 constexpr int kWaWindow = 1024;       // consecutive cells per chunk window held in shared memory
 constexpr int kBigThreads = 256;      // CTA-per-net kernel for nets > kWaMaxDeg
 constexpr int kBigStage = 4096;       // big-net pins whose exact positions stay in shared memory
+constexpr int kWarpNetMax = 1024;     // nets of degree (kWaMaxDeg, kWarpNetMax] take a warp each; larger a CTA
+constexpr int kWarpNetThreads = 256;  // warp-per-net kernel CTA size
 constexpr int kHpwlLimbs = 9;         // limbs 0..kHpwlLimbs (10) of 32-bit digits, LSB 2^-149 (reading A7)
 
 constexpr int kTile = 64;             // density tile = kTile x kTile bins (smaller maps: the map)
 constexpr int kHalo = 2;              // small-cell footprints extend <= 2 bins past their tile
-constexpr int kStageRecs = 1024;      // records per staging buffer of the scatter/gather walkers
+constexpr int kStageRecs = 512;       // records per staging buffer of the scatter/gather walkers
 constexpr int kFlushRecs = 8192;      // a walker flushes its shared tile at least every 2^13 records
 // Tile bins accumulate each contribution v in (0, 1] as two native 32-bit shared atomics:
 // hi = floor(v 2^kTileHiBits) and lo = floor(frac 2^kTileLoBits); with <= kFlushRecs = 2^13
@@ -94,6 +96,7 @@ struct Ctx {
   float *d_pin_dx = nullptr, *d_pin_dy = nullptr;
   // big nets (degree > kWaMaxDeg): plain CSR, one CTA per net
   int32_t n_big = 0;
+  int32_t n_huge = 0;               // big nets [0, n_huge) (degree > kWarpNetMax) take a CTA each
   int32_t big_stage = 0;            // staged pins per big-net CTA (min(max degree, kBigStage))
   int32_t *d_big_start = nullptr;   // [n_big + 1]
   int32_t *d_big_flags = nullptr;   // counted flag per big net

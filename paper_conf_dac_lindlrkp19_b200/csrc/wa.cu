@@ -24,6 +24,8 @@
 //    common shift that cancels exactly (reading A2).  Values are carried in log2 units;
 //  * HPWL mode uses exact (TwoSum) pin positions and extremes and a 2^-149 fixed-point int64
 //    limb sum: correctly rounded and order independent (reading A7).
+#include <algorithm>
+
 #include "async_copy.cuh"
 #include "dp_internal.h"
 
@@ -53,6 +55,7 @@ struct WaArgs {
   const float *big_w, *big_dx, *big_dy;
   int part_offset;
   int big_stage;   // pins staged in shared memory per big-net CTA
+  int n_huge, n_big, n_warp_blocks;
   WaCaps caps;
 };
 
@@ -455,133 +458,6 @@ struct WaSmem {
   __host__ __device__ int bytes() const { return off_bar() + 16; }
 };
 
-// MODE 0: WA + gradient; 1: WA + gradient + HPWL; 2: HPWL only.
-template <int MODE>
-__global__ void __launch_bounds__(kWaThreads, 3) k_wa_chunks(WaArgs a) {
-  constexpr bool kGrad = MODE != 2;
-  constexpr bool kHpwl = MODE != 0;
-  extern __shared__ __align__(16) unsigned char smem[];
-  const WaSmem L_{a.caps};
-  int *s_slot = reinterpret_cast<int *>(smem + L_.off_slot());
-  float *s_dx = reinterpret_cast<float *>(smem + L_.off_dx());
-  float *s_dy = reinterpret_cast<float *>(smem + L_.off_dy());
-  int *s_deg = reinterpret_cast<int *>(smem + L_.off_deg());
-  float *s_w = reinterpret_cast<float *>(smem + L_.off_w());
-  WarpGroup *s_wg = reinterpret_cast<WarpGroup *>(smem + L_.off_wg());
-  int *s_far = reinterpret_cast<int *>(smem + L_.off_far());
-  float *s_px = reinterpret_cast<float *>(smem + L_.off_px());
-  float *s_py = reinterpret_cast<float *>(smem + L_.off_py());
-  int *s_g = reinterpret_cast<int *>(smem + L_.off_g());
-  uint64_t *bar = reinterpret_cast<uint64_t *>(smem + L_.off_bar());
-
-  const Chunk ch = a.chunks[blockIdx.x];
-  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-  // window positions by bulk copy when 16-byte aligned (the caller's x / y), else by threads
-  const int wbulk = ch.win_n & ~3;
-  const bool win_bulk = ((((uintptr_t)(a.x + ch.win_lo)) | ((uintptr_t)(a.y + ch.win_lo))) & 15) == 0 && wbulk > 0;
-  if (tid == 0) {
-    mbar_init(bar);
-    const unsigned tx = 12u * ch.pin_n + (a.has_w ? 8u : 4u) * ch.net_n + 16u * ch.wg_n + 4u * ch.far_pad +
-                        (win_bulk ? 8u * wbulk : 0u);
-    mbar_expect_tx(bar, tx);
-    if (ch.pin_n) {
-      bulk_g2s(s_slot, a.pin_slot + ch.pin_begin, 4u * ch.pin_n, bar);
-      bulk_g2s(s_dx, a.pin_dx + ch.pin_begin, 4u * ch.pin_n, bar);
-      bulk_g2s(s_dy, a.pin_dy + ch.pin_begin, 4u * ch.pin_n, bar);
-    }
-    if (ch.net_n) {
-      bulk_g2s(s_deg, a.net_deg + ch.net_begin, 4u * ch.net_n, bar);
-      if (a.has_w) bulk_g2s(s_w, a.net_w + ch.net_begin, 4u * ch.net_n, bar);
-    }
-    if (ch.wg_n) bulk_g2s(s_wg, a.wgs + ch.wg_begin, 16u * ch.wg_n, bar);
-    if (ch.far_pad) bulk_g2s(s_far, a.far_cells + ch.far_begin, 4u * ch.far_pad, bar);
-    if (win_bulk) {
-      bulk_g2s(s_px, a.x + ch.win_lo, 4u * wbulk, bar);
-      bulk_g2s(s_py, a.y + ch.win_lo, 4u * wbulk, bar);
-    }
-  }
-  const int nslots = L_.slots();
-  if (kGrad)   // 2 * nslots is a multiple of 8, s_g 16-byte aligned
-    for (int i = tid; i < nslots / 2; i += kWaThreads) reinterpret_cast<int4 *>(s_g)[i] = make_int4(0, 0, 0, 0);
-  for (int i = (win_bulk ? wbulk : 0) + tid; i < ch.win_n; i += kWaThreads) {
-    s_px[i] = __ldg(a.x + ch.win_lo + i);
-    s_py[i] = __ldg(a.y + ch.win_lo + i);
-  }
-  __syncthreads();   // barrier initialised before anyone waits on it
-  mbar_wait(bar, 0);
-  // far cells: positions gathered once per chunk
-  for (int f0 = tid; f0 < ch.far_n; f0 += 4 * kWaThreads) {   // 8 loads in flight per thread
-    float fx[4], fy[4];
-#pragma unroll
-    for (int k = 0; k < 4; k++) {
-      const int f = f0 + k * kWaThreads;
-      const int c = f < ch.far_n ? s_far[f] : 0;
-      fx[k] = __ldg(a.x + c);
-      fy[k] = __ldg(a.y + c);
-    }
-#pragma unroll
-    for (int k = 0; k < 4; k++) {
-      const int f = f0 + k * kWaThreads;
-      if (f < ch.far_n) {
-        s_px[kWaWindow + f] = fx[k];
-        s_py[kWaWindow + f] = fy[k];
-      }
-    }
-  }
-  __syncthreads();
-
-  float wl_acc = 0.f;
-  unsigned long long L[kHpwlLimbs + 1];
-#pragma unroll
-  for (int k = 0; k <= kHpwlLimbs; k++) L[k] = 0ull;
-  const GroupCtx gc{s_slot, s_dx, s_dy, s_deg, s_w, s_px, s_py, s_g, nslots - 1, exp2f((float)ch.scale_log2),
-                    lane, (1u << lane) - 1u};
-
-  // warp groups are dealt round-robin (the host orders them by decreasing cost)
-  for (int gi = warp; gi < ch.wg_n; gi += kWaThreads / 32) {
-    const WarpGroup wg = s_wg[gi];
-    if (MODE == 0) {
-      if (wg.flags & 1) {
-        wa_group_pairs(a, wg, gc, wl_acc);
-      } else {
-        switch (wg.slots) {
-          case 1: wa_group_fast<1>(a, wg, gc, wl_acc); break;
-          case 2: wa_group_fast<2>(a, wg, gc, wl_acc); break;
-          case 3: wa_group_fast<3>(a, wg, gc, wl_acc); break;
-          default: wa_group_fast<4>(a, wg, gc, wl_acc); break;
-        }
-      }
-    } else {
-      switch (wg.slots) {
-        case 1: wa_group_exact<MODE, 1>(a, wg, gc, wl_acc, L); break;
-        case 2: wa_group_exact<MODE, 2>(a, wg, gc, wl_acc, L); break;
-        case 3: wa_group_exact<MODE, 3>(a, wg, gc, wl_acc, L); break;
-        default: wa_group_exact<MODE, 4>(a, wg, gc, wl_acc, L); break;
-      }
-    }
-  }
-  __syncthreads();
-  if (kGrad) {
-    const float inv = exp2f(-(float)ch.scale_log2);
-    // window: cells [win_lo, win_lo + win_n), win_lo a multiple of 4 -> 16-byte vector reductions
-    float4 *g4 = reinterpret_cast<float4 *>(a.g2 + ch.win_lo);
-    const int npair = ch.win_n >> 1;
-    for (int i = tid; i < npair; i += kWaThreads) {
-      const int4 v = *reinterpret_cast<const int4 *>(s_g + 4 * i);
-      if (v.x | v.y | v.z | v.w) red_v4(g4 + i, v.x * inv, v.y * inv, v.z * inv, v.w * inv);
-    }
-    if ((ch.win_n & 1) && tid == 0) {
-      const int w = ch.win_n - 1;
-      if (s_g[2 * w] | s_g[2 * w + 1]) red_v2(a.g2 + ch.win_lo + w, s_g[2 * w] * inv, s_g[2 * w + 1] * inv);
-    }
-    for (int f = tid; f < ch.far_n; f += kWaThreads) {
-      const int gx = s_g[2 * (kWaWindow + f)], gy = s_g[2 * (kWaWindow + f) + 1];
-      if (gx | gy) red_v2(a.g2 + s_far[f], gx * inv, gy * inv);
-    }
-  }
-  block_flush_scalars<kWaThreads>((double)wl_acc, L, kHpwl, kGrad ? a.part + blockIdx.x : nullptr, a.limbs);
-}
-
 // ---------------------------------------------------------------------------------------
 // Nets with degree > kWaMaxDeg: one CTA per net, three passes over the pins (Alg 2's
 // structure, a^+- recomputed in the gradient pass because they do not fit in registers).
@@ -606,12 +482,13 @@ __device__ __forceinline__ float4 big_pin(const WaArgs &a, int c, int s) {
 // CTA per net of degree > kWaMaxDeg (largest first).  Pass 1 loads every pin once (4 loads in
 // flight per thread) and keeps the exact coordinates in shared memory (nets up to kBigStage
 // pins; larger nets reload), pass 2 forms the eq-6 sums, pass 3 the gradient.
+static_assert(kBigThreads == kWaThreads && kWarpNetThreads == kWaThreads, "big / warp nets run in chunk-kernel CTAs");
+
 template <int MODE>
-__global__ void __launch_bounds__(kBigThreads) k_wa_big(WaArgs a) {
+__device__ __forceinline__ void wa_big_net(const WaArgs &a, int net, float4 *s_pin) {
   constexpr bool kGrad = MODE != 2;
   constexpr bool kHpwl = MODE != 0;
-  extern __shared__ float4 s_pin[];
-  const int net = blockIdx.x, tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   constexpr int NW = kBigThreads / 32;
   const int s0 = a.big_start[net], d = a.big_start[net + 1] - s0;
   const bool staged = d <= a.big_stage;
@@ -720,11 +597,303 @@ __global__ void __launch_bounds__(kBigThreads) k_wa_big(WaArgs a) {
                                    a.limbs);
 }
 
+// Warp per net for degrees (kWaMaxDeg, kWarpNetMax]: three passes over the pins with warp
+// shuffles only (no block barriers); passes 2 and 3 reload the pin data (L1 / L2 resident).
+// MODE 0 uses the log2-unit fast path of the chunk kernel (shift reference P = max fl(x + dx));
+// the HPWL modes form exact TwoSum coordinates as k_wa_big does.
+__device__ __forceinline__ float warp_max(float v) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) v = fmaxf(v, __shfl_xor_sync(0xffffffffu, v, o));
+  return v;
+}
+__device__ __forceinline__ float warp_min(float v) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) v = fminf(v, __shfl_xor_sync(0xffffffffu, v, o));
+  return v;
+}
+__device__ __forceinline__ float warp_sum(float v) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+  return v;
+}
+
+template <int MODE>
+__device__ __forceinline__ void wa_warp_nets(const WaArgs &a, int wb) {
+  constexpr bool kGrad = MODE != 2;
+  constexpr bool kHpwl = MODE != 0;
+  const int lane = threadIdx.x & 31;
+  const int net = a.n_huge + wb * (kWarpNetThreads / 32) + (threadIdx.x >> 5);
+  double wl_acc = 0.0;
+  unsigned long long L[kHpwlLimbs + 1];
+#pragma unroll
+  for (int k = 0; k <= kHpwlLimbs; k++) L[k] = 0ull;
+  if (net < a.n_big) {
+    const int s0 = a.big_start[net], d = a.big_start[net + 1] - s0;
+    const int counted = a.big_flags[net];
+    const float we = a.has_w ? a.big_w[net] : 1.f;
+    const int *cell = a.big_cell + s0;
+    const float *pdx = a.big_dx + s0, *pdy = a.big_dy + s0;
+    if (MODE == 0) {
+      float Px = -INFINITY, Mx = INFINITY, Py = -INFINITY, My = INFINITY;
+#pragma unroll 4
+      for (int p = lane; p < d; p += 32) {
+        const int c = __ldg(cell + p) & 0x7fffffff;
+        const float px = __ldg(a.x + c) + __ldg(pdx + p), py = __ldg(a.y + c) + __ldg(pdy + p);
+        Px = fmaxf(Px, px); Mx = fminf(Mx, px);
+        Py = fmaxf(Py, py); My = fminf(My, py);
+      }
+      Px = warp_max(Px); Mx = warp_min(Mx); Py = warp_max(Py); My = warp_min(My);
+      const float k2 = a.k2;
+      float bxp = 0.f, bxm = 0.f, cxp = 0.f, cxm = 0.f, byp = 0.f, bym = 0.f, cyp = 0.f, cym = 0.f;
+#pragma unroll 4
+      for (int p = lane; p < d; p += 32) {
+        const int c = __ldg(cell + p) & 0x7fffffff;
+        const float xc = __ldg(a.x + c), yc = __ldg(a.y + c);
+        const float dkx = __ldg(pdx + p) * k2, dky = __ldg(pdy + p) * k2;
+        const float lxp = fmaf(xc - Px, k2, dkx), lxm = fmaf(xc - Mx, k2, dkx);
+        const float lyp = fmaf(yc - Py, k2, dky), lym = fmaf(yc - My, k2, dky);
+        const float axp = ex2(lxp), axm = ex2(-lxm), ayp = ex2(lyp), aym = ex2(-lym);
+        bxp += axp; cxp = fmaf(lxp, axp, cxp);
+        bxm += axm; cxm = fmaf(lxm, axm, cxm);
+        byp += ayp; cyp = fmaf(lyp, ayp, cyp);
+        bym += aym; cym = fmaf(lym, aym, cym);
+      }
+      bxp = warp_sum(bxp); cxp = warp_sum(cxp); bxm = warp_sum(bxm); cxm = warp_sum(cxm);
+      byp = warp_sum(byp); cyp = warp_sum(cyp); bym = warp_sum(bym); cym = warp_sum(cym);
+      const float ibxp = rcp(bxp), ibxm = rcp(bxm), ibyp = rcp(byp), ibym = rcp(bym);
+      const float mxp = cxp * ibxp, mxm = cxm * ibxm, myp = cyp * ibyp, mym = cym * ibym;   // log2 units
+      if (lane == 0 && counted) {
+        const float ig2 = a.gamma * kLn2;
+        wl_acc = (double)(we * ((Px - Mx) + (mxp - mxm) * ig2 + (Py - My) + (myp - mym) * ig2));
+      }
+      const float wl2 = we * kLn2;
+      const float qxp = ibxp * wl2, pxp = we * ibxp - mxp * qxp;
+      const float qxm = ibxm * wl2, pxm = we * ibxm + mxm * qxm;
+      const float qyp = ibyp * wl2, pyp = we * ibyp - myp * qyp;
+      const float qym = ibym * wl2, pym = we * ibym + mym * qym;
+#pragma unroll 4
+      for (int p = lane; p < d; p += 32) {
+        const int raw = __ldg(cell + p);
+        if (raw < 0) continue;
+        const float xc = __ldg(a.x + raw), yc = __ldg(a.y + raw);
+        const float dkx = __ldg(pdx + p) * k2, dky = __ldg(pdy + p) * k2;
+        const float lxp = fmaf(xc - Px, k2, dkx), lxm = fmaf(xc - Mx, k2, dkx);
+        const float lyp = fmaf(yc - Py, k2, dky), lym = fmaf(yc - My, k2, dky);
+        const float axp = ex2(lxp), axm = ex2(-lxm), ayp = ex2(lyp), aym = ex2(-lym);
+        const float gx = axp * fmaf(lxp, qxp, pxp) - axm * fmaf(-lxm, qxm, pxm);
+        const float gy = ayp * fmaf(lyp, qyp, pyp) - aym * fmaf(-lym, qym, pym);
+        red_v2(a.g2 + raw, gx, gy);
+      }
+    } else {
+      Ext e{-INFINITY, 0.f, INFINITY, 0.f, -INFINITY, 0.f, INFINITY, 0.f};
+      for (int p = lane; p < d; p += 32) {
+        const float4 v = big_pin(a, __ldg(cell + p) & 0x7fffffff, s0 + p);
+        const Ext o{v.x, v.y, v.x, v.y, v.z, v.w, v.z, v.w};
+        ext_merge(e, o);
+      }
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) {
+        Ext t;
+        t.Xh = __shfl_xor_sync(0xffffffffu, e.Xh, o); t.Xl = __shfl_xor_sync(0xffffffffu, e.Xl, o);
+        t.xh = __shfl_xor_sync(0xffffffffu, e.xh, o); t.xl = __shfl_xor_sync(0xffffffffu, e.xl, o);
+        t.Yh = __shfl_xor_sync(0xffffffffu, e.Yh, o); t.Yl = __shfl_xor_sync(0xffffffffu, e.Yl, o);
+        t.yh = __shfl_xor_sync(0xffffffffu, e.yh, o); t.yl = __shfl_xor_sync(0xffffffffu, e.yl, o);
+        ext_merge(e, t);
+      }
+      if (lane == 0 && counted) {
+        const double xp = __dadd_rn((double)e.Xh, (double)e.Xl), xm = __dadd_rn((double)e.xh, (double)e.xl);
+        const double yp = __dadd_rn((double)e.Yh, (double)e.Yl), ym = __dadd_rn((double)e.yh, (double)e.yl);
+        limbs_add(L, __dadd_rn(__dsub_rn(xp, xm), __dsub_rn(yp, ym)));
+      }
+      if (kGrad) {
+        float sm[8] = {0, 0, 0, 0, 0, 0, 0, 0};  // bxp cxp bxm cxm byp cyp bym cym
+        for (int p = lane; p < d; p += 32) {
+          const float4 v = big_pin(a, __ldg(cell + p) & 0x7fffffff, s0 + p);
+          const float lxp = __fadd_rn(__fsub_rn(v.x, e.Xh), __fsub_rn(v.y, e.Xl));
+          const float lxm = __fadd_rn(__fsub_rn(v.x, e.xh), __fsub_rn(v.y, e.xl));
+          const float lyp = __fadd_rn(__fsub_rn(v.z, e.Yh), __fsub_rn(v.w, e.Yl));
+          const float lym = __fadd_rn(__fsub_rn(v.z, e.yh), __fsub_rn(v.w, e.yl));
+          const float axp = ex2(lxp * a.k2), axm = ex2(-lxm * a.k2);
+          const float ayp = ex2(lyp * a.k2), aym = ex2(-lym * a.k2);
+          sm[0] += axp; sm[1] += lxp * axp; sm[2] += axm; sm[3] += lxm * axm;
+          sm[4] += ayp; sm[5] += lyp * ayp; sm[6] += aym; sm[7] += lym * aym;
+        }
+#pragma unroll
+        for (int k = 0; k < 8; k++) sm[k] = warp_sum(sm[k]);
+        const float ibxp = 1.f / sm[0], ibxm = 1.f / sm[2], ibyp = 1.f / sm[4], ibym = 1.f / sm[6];
+        const float mxp = sm[1] * ibxp, mxm = sm[3] * ibxm, myp = sm[5] * ibyp, mym = sm[7] * ibym;
+        if (lane == 0 && counted) {
+          const float spanx = __fadd_rn(__fsub_rn(e.Xh, e.xh), __fsub_rn(e.Xl, e.xl));
+          const float spany = __fadd_rn(__fsub_rn(e.Yh, e.yh), __fsub_rn(e.Yl, e.yl));
+          wl_acc = (double)(we * ((spanx + mxp - mxm) + (spany + myp - mym)));
+        }
+        for (int p = lane; p < d; p += 32) {
+          const int raw = __ldg(cell + p);
+          if (raw < 0) continue;
+          const float4 v = big_pin(a, raw, s0 + p);
+          const float lxp = __fadd_rn(__fsub_rn(v.x, e.Xh), __fsub_rn(v.y, e.Xl));
+          const float lxm = __fadd_rn(__fsub_rn(v.x, e.xh), __fsub_rn(v.y, e.xl));
+          const float lyp = __fadd_rn(__fsub_rn(v.z, e.Yh), __fsub_rn(v.w, e.Yl));
+          const float lym = __fadd_rn(__fsub_rn(v.z, e.yh), __fsub_rn(v.w, e.yl));
+          const float axp = ex2(lxp * a.k2), axm = ex2(-lxm * a.k2);
+          const float ayp = ex2(lyp * a.k2), aym = ex2(-lym * a.k2);
+          const float gx = we * (axp * ibxp * (1.f + (lxp - mxp) * a.inv_gamma) -
+                                 axm * ibxm * (1.f - (lxm - mxm) * a.inv_gamma));
+          const float gy = we * (ayp * ibyp * (1.f + (lyp - myp) * a.inv_gamma) -
+                                 aym * ibym * (1.f - (lym - mym) * a.inv_gamma));
+          red_v2(a.g2 + raw, gx, gy);
+        }
+      }
+    }
+  }
+  block_flush_scalars<kWarpNetThreads>(wl_acc, L, kHpwl, kGrad ? a.part + a.part_offset + a.n_huge + wb : nullptr,
+                                       a.limbs);
+}
+
+// MODE 0: WA + gradient; 1: WA + gradient + HPWL; 2: HPWL only.
+template <int MODE>
+__global__ void __launch_bounds__(kWaThreads, 3) k_wa_chunks(WaArgs a) {
+  constexpr bool kGrad = MODE != 2;
+  constexpr bool kHpwl = MODE != 0;
+  extern __shared__ __align__(16) unsigned char smem[];
+  const WaSmem L_{a.caps};
+  int *s_slot = reinterpret_cast<int *>(smem + L_.off_slot());
+  float *s_dx = reinterpret_cast<float *>(smem + L_.off_dx());
+  float *s_dy = reinterpret_cast<float *>(smem + L_.off_dy());
+  int *s_deg = reinterpret_cast<int *>(smem + L_.off_deg());
+  float *s_w = reinterpret_cast<float *>(smem + L_.off_w());
+  WarpGroup *s_wg = reinterpret_cast<WarpGroup *>(smem + L_.off_wg());
+  int *s_far = reinterpret_cast<int *>(smem + L_.off_far());
+  float *s_px = reinterpret_cast<float *>(smem + L_.off_px());
+  float *s_py = reinterpret_cast<float *>(smem + L_.off_py());
+  int *s_g = reinterpret_cast<int *>(smem + L_.off_g());
+  uint64_t *bar = reinterpret_cast<uint64_t *>(smem + L_.off_bar());
+
+  // one launch for all nets: CTAs [0, n_huge) take a net of degree > kWarpNetMax each, the next
+  // n_warp_blocks CTAs 8 nets of degree (kWaMaxDeg, kWarpNetMax] each (a warp per net), the rest
+  // the staged chunks; the long big-net CTAs are dispatched first and overlap the chunks.
+  if ((int)blockIdx.x < a.n_huge) {
+    wa_big_net<MODE>(a, blockIdx.x, reinterpret_cast<float4 *>(smem));
+    return;
+  }
+  if ((int)blockIdx.x < a.n_huge + a.n_warp_blocks) {
+    wa_warp_nets<MODE>(a, blockIdx.x - a.n_huge);
+    return;
+  }
+  const int chunk = blockIdx.x - a.n_huge - a.n_warp_blocks;
+  const Chunk ch = a.chunks[chunk];
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  // window positions by bulk copy when 16-byte aligned (the caller's x / y), else by threads
+  const int wbulk = ch.win_n & ~3;
+  const bool win_bulk = ((((uintptr_t)(a.x + ch.win_lo)) | ((uintptr_t)(a.y + ch.win_lo))) & 15) == 0 && wbulk > 0;
+  if (tid == 0) {
+    mbar_init(bar);
+    const unsigned tx = 12u * ch.pin_n + (a.has_w ? 8u : 4u) * ch.net_n + 16u * ch.wg_n + 4u * ch.far_pad +
+                        (win_bulk ? 8u * wbulk : 0u);
+    mbar_expect_tx(bar, tx);
+    if (ch.pin_n) {
+      bulk_g2s(s_slot, a.pin_slot + ch.pin_begin, 4u * ch.pin_n, bar);
+      bulk_g2s(s_dx, a.pin_dx + ch.pin_begin, 4u * ch.pin_n, bar);
+      bulk_g2s(s_dy, a.pin_dy + ch.pin_begin, 4u * ch.pin_n, bar);
+    }
+    if (ch.net_n) {
+      bulk_g2s(s_deg, a.net_deg + ch.net_begin, 4u * ch.net_n, bar);
+      if (a.has_w) bulk_g2s(s_w, a.net_w + ch.net_begin, 4u * ch.net_n, bar);
+    }
+    if (ch.wg_n) bulk_g2s(s_wg, a.wgs + ch.wg_begin, 16u * ch.wg_n, bar);
+    if (ch.far_pad) bulk_g2s(s_far, a.far_cells + ch.far_begin, 4u * ch.far_pad, bar);
+    if (win_bulk) {
+      bulk_g2s(s_px, a.x + ch.win_lo, 4u * wbulk, bar);
+      bulk_g2s(s_py, a.y + ch.win_lo, 4u * wbulk, bar);
+    }
+  }
+  const int nslots = L_.slots();
+  if (kGrad)   // 2 * nslots is a multiple of 8, s_g 16-byte aligned
+    for (int i = tid; i < nslots / 2; i += kWaThreads) reinterpret_cast<int4 *>(s_g)[i] = make_int4(0, 0, 0, 0);
+  for (int i = (win_bulk ? wbulk : 0) + tid; i < ch.win_n; i += kWaThreads) {
+    s_px[i] = __ldg(a.x + ch.win_lo + i);
+    s_py[i] = __ldg(a.y + ch.win_lo + i);
+  }
+  __syncthreads();   // barrier initialised before anyone waits on it
+  mbar_wait(bar, 0);
+  // far cells: positions gathered once per chunk
+  for (int f0 = tid; f0 < ch.far_n; f0 += 4 * kWaThreads) {   // 8 loads in flight per thread
+    float fx[4], fy[4];
+#pragma unroll
+    for (int k = 0; k < 4; k++) {
+      const int f = f0 + k * kWaThreads;
+      const int c = f < ch.far_n ? s_far[f] : 0;
+      fx[k] = __ldg(a.x + c);
+      fy[k] = __ldg(a.y + c);
+    }
+#pragma unroll
+    for (int k = 0; k < 4; k++) {
+      const int f = f0 + k * kWaThreads;
+      if (f < ch.far_n) {
+        s_px[kWaWindow + f] = fx[k];
+        s_py[kWaWindow + f] = fy[k];
+      }
+    }
+  }
+  __syncthreads();
+
+  float wl_acc = 0.f;
+  unsigned long long L[kHpwlLimbs + 1];
+#pragma unroll
+  for (int k = 0; k <= kHpwlLimbs; k++) L[k] = 0ull;
+  const GroupCtx gc{s_slot, s_dx, s_dy, s_deg, s_w, s_px, s_py, s_g, nslots - 1, exp2f((float)ch.scale_log2),
+                    lane, (1u << lane) - 1u};
+
+  // warp groups are dealt round-robin (the host orders them by decreasing cost)
+  for (int gi = warp; gi < ch.wg_n; gi += kWaThreads / 32) {
+    const WarpGroup wg = s_wg[gi];
+    if (MODE == 0) {
+      if (wg.flags & 1) {
+        wa_group_pairs(a, wg, gc, wl_acc);
+      } else {
+        switch (wg.slots) {
+          case 1: wa_group_fast<1>(a, wg, gc, wl_acc); break;
+          case 2: wa_group_fast<2>(a, wg, gc, wl_acc); break;
+          case 3: wa_group_fast<3>(a, wg, gc, wl_acc); break;
+          default: wa_group_fast<4>(a, wg, gc, wl_acc); break;
+        }
+      }
+    } else {
+      switch (wg.slots) {
+        case 1: wa_group_exact<MODE, 1>(a, wg, gc, wl_acc, L); break;
+        case 2: wa_group_exact<MODE, 2>(a, wg, gc, wl_acc, L); break;
+        case 3: wa_group_exact<MODE, 3>(a, wg, gc, wl_acc, L); break;
+        default: wa_group_exact<MODE, 4>(a, wg, gc, wl_acc, L); break;
+      }
+    }
+  }
+  __syncthreads();
+  if (kGrad) {
+    const float inv = exp2f(-(float)ch.scale_log2);
+    // window: cells [win_lo, win_lo + win_n), win_lo a multiple of 4 -> 16-byte vector reductions
+    float4 *g4 = reinterpret_cast<float4 *>(a.g2 + ch.win_lo);
+    const int npair = ch.win_n >> 1;
+    for (int i = tid; i < npair; i += kWaThreads) {
+      const int4 v = *reinterpret_cast<const int4 *>(s_g + 4 * i);
+      if (v.x | v.y | v.z | v.w) red_v4(g4 + i, v.x * inv, v.y * inv, v.z * inv, v.w * inv);
+    }
+    if ((ch.win_n & 1) && tid == 0) {
+      const int w = ch.win_n - 1;
+      if (s_g[2 * w] | s_g[2 * w + 1]) red_v2(a.g2 + ch.win_lo + w, s_g[2 * w] * inv, s_g[2 * w + 1] * inv);
+    }
+    for (int f = tid; f < ch.far_n; f += kWaThreads) {
+      const int gx = s_g[2 * (kWaWindow + f)], gy = s_g[2 * (kWaWindow + f) + 1];
+      if (gx | gy) red_v2(a.g2 + s_far[f], gx * inv, gy * inv);
+    }
+  }
+  block_flush_scalars<kWaThreads>((double)wl_acc, L, kHpwl, kGrad ? a.part + chunk : nullptr, a.limbs);
+}
+
 template <int MODE>
 void launch_mode(const Ctx &c, const WaArgs &a, cudaStream_t s) {
   const WaSmem L{a.caps};
-  if (c.n_chunks > 0) k_wa_chunks<MODE><<<c.n_chunks, kWaThreads, L.bytes(), s>>>(a);
-  if (c.n_big > 0) k_wa_big<MODE><<<c.n_big, kBigThreads, 16 * a.big_stage, s>>>(a);
+  const int grid = c.n_chunks + a.n_huge + a.n_warp_blocks;
+  if (grid > 0) k_wa_chunks<MODE><<<grid, kWaThreads, L.bytes(), s>>>(a);
 }
 
 }  // namespace
@@ -737,13 +906,7 @@ cudaError_t wa_configure(const WaCaps &caps) {
   if (e != cudaSuccess) return e;
   e = cudaFuncSetAttribute(k_wa_chunks<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, b);
   if (e != cudaSuccess) return e;
-  e = cudaFuncSetAttribute(k_wa_chunks<2>, cudaFuncAttributeMaxDynamicSharedMemorySize, b);
-  if (e != cudaSuccess) return e;
-  e = cudaFuncSetAttribute(k_wa_big<0>, cudaFuncAttributeMaxDynamicSharedMemorySize, 16 * kBigStage);
-  if (e != cudaSuccess) return e;
-  e = cudaFuncSetAttribute(k_wa_big<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, 16 * kBigStage);
-  if (e != cudaSuccess) return e;
-  return cudaFuncSetAttribute(k_wa_big<2>, cudaFuncAttributeMaxDynamicSharedMemorySize, 16 * kBigStage);
+  return cudaFuncSetAttribute(k_wa_chunks<2>, cudaFuncAttributeMaxDynamicSharedMemorySize, b);
 }
 
 void launch_wa(const Ctx &c, const float *x, const float *y, float gamma, bool hpwl_only, bool with_hpwl,
@@ -773,7 +936,11 @@ void launch_wa(const Ctx &c, const float *x, const float *y, float gamma, bool h
   a.big_dx = c.d_big_dx;
   a.big_dy = c.d_big_dy;
   a.part_offset = c.n_chunks;
-  a.big_stage = c.big_stage;
+  a.n_huge = c.n_huge;
+  a.n_big = c.n_big;
+  a.n_warp_blocks = (c.n_big - c.n_huge + kWarpNetThreads / 32 - 1) / (kWarpNetThreads / 32);
+  // big-net pins staged in the chunk kernel's dynamic shared memory (larger nets reload)
+  a.big_stage = std::min(c.big_stage, wa_smem_bytes(c.wa_caps) / 16);
   a.caps = c.wa_caps;
   if (hpwl_only)
     launch_mode<2>(c, a, s);

@@ -44,14 +44,14 @@ __device__ __forceinline__ int mk_pos(int t, int n) { return (t & 1) ? n - ((t +
 // 5 barriers instead of 10.
 __device__ void fft_block(float2 *buf, int n, int log2n, int nseq, const float2 *__restrict__ tw,
                           bool inverse) {
-  const int quarter_n = n >> 2;
+  const int quarter_n = n >> 2, lq = log2n - 2;
   const int total4 = nseq * quarter_n;
   int s = 1;
   for (; s + 1 <= log2n; s += 2) {
     const int h = 1 << (s - 1), lh = s - 1;
     const int st1 = n >> s, st2 = n >> (s + 1);   // twiddle strides of W_{2h} and W_{4h}
     for (int q = threadIdx.x; q < total4; q += blockDim.x) {
-      const int seq = q / quarter_n, r = q - seq * quarter_n;
+      const int seq = q >> lq, r = q & (quarter_n - 1);
       const int blk = r >> lh, k = r & (h - 1);
       const int base = seq * n + (blk << (lh + 2)) + k;
       float2 w1 = __ldg(tw + k * st1), w2 = __ldg(tw + k * st2);
@@ -76,7 +76,7 @@ __device__ void fft_block(float2 *buf, int n, int log2n, int nseq, const float2 
   if (s == log2n) {  // odd log2n: one last radix-2 level
     const int half = 1 << (s - 1), half_n = n >> 1, total = nseq * half_n;
     for (int b = threadIdx.x; b < total; b += blockDim.x) {
-      const int seq = b / half_n, r = b - seq * half_n;
+      const int seq = b >> (log2n - 1), r = b & (half_n - 1);
       const int k = r;  // one group: grp = 0, len = n
       const int i = seq * n + k, jx = i + half;
       float2 w = __ldg(tw + k);
@@ -207,12 +207,12 @@ __global__ void __launch_bounds__(kColThreads) k_col_generic(const float *__rest
   __syncthreads();
   if (op == 0) {
     for (int idx = threadIdx.x; idx < mx * (kColSlab / 2); idx += kColThreads) {
-      const int pr = idx / mx, t = idx % mx;
+      const int pr = idx >> log2mx, t = idx & (mx - 1);
       zbuf[pr * mx + brev(mk_pos(t, mx), log2mx)] = make_float2(rbuf[(2 * pr) * mx + t], rbuf[(2 * pr + 1) * mx + t]);
     }
   } else {
     for (int idx = threadIdx.x; idx < mx * (kColSlab / 2); idx += kColThreads) {
-      const int pr = idx / mx, k = idx % mx;
+      const int pr = idx >> log2mx, k = idx & (mx - 1);
       const float *pp = rbuf + (2 * pr) * mx, *qq = rbuf + (2 * pr + 1) * mx;
       float pk, qk, pnk, qnk;
       if (op == 2) {  // reversed inputs x'_t = x_{N-t}
@@ -281,42 +281,30 @@ __global__ void __launch_bounds__(kColThreads) k_col_fields(ColFieldArgs a) {
   fft_block(zbuf, mx, log2mx, kColSlab / 2, a.tw_x, false);
   const float scale = 2.f / mx;
   double e = 0.0;
+  // DCT_x spectrum, Parseval energy term and the spectral scaling of eqs (9c)/(9d) in one pass:
+  // A_X = a k_u / k^2 -> abuf, A_Y = a k_v / k^2 -> ybuf; a_00 / k^2 := 0 (A15)
+  float *ybuf = abuf + kColSlab * mx;
   for (int idx = threadIdx.x; idx < mx * (kColSlab / 2); idx += kColThreads) {
-    const int pr = idx / mx, u = idx % mx;
+    const int pr = idx >> log2mx, u = idx & (mx - 1);
     const float2 d = dct_post(zbuf + pr * mx, u, mx, __ldg(a.ph_x + u), scale);
-    abuf[(2 * pr) * mx + u] = d.x;
-    abuf[(2 * pr + 1) * mx + u] = d.y;
     const float kx = __ldg(a.kx + u);
+    const double wu = (u == 0) ? 0.25 * mx : 0.5 * mx;
 #pragma unroll
     for (int h = 0; h < 2; h++) {
-      const int v = c0 + 2 * pr + h;
+      const int col = 2 * pr + h, v = c0 + col;
       const float ky = __ldg(a.ky + v);
-      const float k2 = kx * kx + ky * ky;
-      if (u == 0 && v == 0) continue;
+      const float ik2 = (u == 0 && v == 0) ? 0.f : __frcp_rn(kx * kx + ky * ky);
       const float av = h ? d.y : d.x;
-      const double wu = (u == 0) ? 0.25 * mx : 0.5 * mx;
       const double wv = (v == 0) ? 0.25 * my : 0.5 * my;
-      e += wu * wv * (double)av * (double)av / (double)k2;
+      e += wu * wv * (double)(av * av * ik2);
+      abuf[col * mx + u] = av * kx * ik2;
+      ybuf[col * mx + u] = av * ky * ik2;
     }
-  }
-  __syncthreads();  // abuf complete; zbuf free
-  // spectral scaling (eqs 9c/9d): A_X = a k_u / k^2 (in place of a), A_Y = a k_v / k^2 (to the
-  // real scratch behind abuf); a_00 / k^2 := 0
-  float *ybuf = abuf + kColSlab * mx;
-  for (int idx = threadIdx.x; idx < mx * kColSlab; idx += kColThreads) {
-    const int col = idx / mx, u = idx - col * mx;
-    const int v = c0 + col;
-    const float kx = __ldg(a.kx + u), ky = __ldg(a.ky + v);
-    const float k2 = kx * kx + ky * ky;
-    const float ik2 = (u == 0 && v == 0) ? 0.f : 1.f / k2;
-    const float av = abuf[idx];
-    abuf[idx] = av * kx * ik2;
-    ybuf[idx] = av * ky * ik2;
   }
   __syncthreads();
   // inverse pre-processing: per column, p = reversed A_X (IDXST via eq 8e), q = A_Y (IDCT)
   for (int idx = threadIdx.x; idx < mx * kColSlab; idx += kColThreads) {
-    const int col = idx / mx, k = idx - col * mx;
+    const int col = idx >> log2mx, k = idx & (mx - 1);
     const float *ax = abuf + col * mx, *ay = ybuf + col * mx;
     const float pk = k ? ax[mx - k] : 0.f;
     const float pnk = k ? ax[k] : 0.f;

@@ -47,6 +47,8 @@ struct DenArgs {
   float sxf, syf;      // stretched minimum sizes sqrt2 b (fp32)
   int mx, my, tile, tile_log2, tiles_y, ntiles, stretch;
   int *tile_cnt, *tile_cursor, *tile_off;
+  int *walk_tile;   // [walk_grid] first tile of each walker's slice (D2)
+  int walk_grid;
   float4 *rec;
   int2 *rec_rc;   // (r as float bits, tile-local first bin i0 | j0 << 16)
   int *rec_cell;  // own cell index
@@ -156,6 +158,7 @@ __global__ void __launch_bounds__(1024) k_scan(DenArgs a) {
   __syncthreads();
   if (warp == 0) s_wa[lane] = warp_incl_scan(s_wa[lane], lane);
   __syncthreads();
+  const long long N = s_wa[31], G = a.walk_grid;
   int off_c = (warp ? s_wa[warp - 1] : 0) + ia - cnt_sum;
   for (int k = 0; k < per; k++) {
     const int t = t0 + k;
@@ -163,6 +166,12 @@ __global__ void __launch_bounds__(1024) k_scan(DenArgs a) {
       const int c = a.tile_cnt[t];
       a.tile_off[t] = off_c;
       a.tile_cursor[t] = off_c;
+      // walkers whose slice [N g / G, N (g + 1) / G) starts in this tile:
+      // off <= floor(N g / G) < off + c  <=>  ceil(off G / N) <= g < ceil((off + c) G / N)
+      if (c > 0) {
+        const long long g0 = ((long long)off_c * G + N - 1) / N, g1 = ((long long)(off_c + c) * G + N - 1) / N;
+        for (long long g = g0; g < g1; g++) a.walk_tile[g] = t;
+      }
       off_c += c;
       a.tile_cnt[t] = 0;  // ready for the next evaluation
     }
@@ -307,13 +316,8 @@ __device__ __forceinline__ void walk_init(const DenArgs &a, Walker &w) {
   w.t = 0;
   w.tend = 0;
   if (w.cur >= w.re) return;
-  int lo = 0, hi = a.ntiles;   // largest t with tile_off[t] <= cur (then tile_off[t + 1] > cur)
-  while (hi - lo > 1) {
-    const int mid = (lo + hi) >> 1;
-    if (a.tile_off[mid] <= w.cur) lo = mid; else hi = mid;
-  }
-  w.t = lo;
-  w.tend = a.tile_off[lo + 1];
+  w.t = a.walk_tile[blockIdx.x];   // from D2: tile_off[t] <= cur < tile_off[t + 1]
+  w.tend = a.tile_off[w.t + 1];
 }
 
 // (thread 0) next chunk of the slice -> descriptor slot b, copies issued on bar[b]
@@ -344,6 +348,12 @@ __device__ __forceinline__ void walk_start(const DenArgs &a, Walker &w, RecStage
   for (int b = 0; b < kStages; b++) mbar_init(&st.bar[b]);
   mbar_init(&st.bar_xi);
   for (int b = 0; b < kStages - 1; b++) walk_issue(a, w, st, b, with_cell);
+}
+
+// shared-memory reduction without a return value; unconditional (a zero add is cheaper than the
+// branch + reconvergence ptxas emits around a predicated shared atomic)
+__device__ __forceinline__ void red_shared(unsigned *p, unsigned v) {
+  asm volatile("red.shared.add.u32 [%0], %1;" ::"r"(smem_u32(p)), "r"(v) : "memory");
 }
 
 // overlaps (bin units) of a record's footprint with the 3 bins from its first bin, per axis;
@@ -424,8 +434,8 @@ __global__ void __launch_bounds__(kTileThreads) k_scatter_walk(DenArgs a) {
           const unsigned hi = (unsigned)vh;
           const unsigned lo = (unsigned)((vh - (float)hi) * scale_lo);
           const int k2 = base + di * P + dj;
-          if (hi) atomicAdd(s_hi + k2, hi);
-          if (lo) atomicAdd(s_lo + k2, lo);
+          red_shared(s_hi + k2, hi);
+          red_shared(s_lo + k2, lo);
         }
       }
     }
@@ -493,7 +503,8 @@ __global__ void __launch_bounds__(kTileThreads) k_gather_walk(DenArgs a) {
         float sx = 0.f, sy = 0.f;
 #pragma unroll
         for (int dj = 0; dj < 3; dj++) {
-          const float2 e2 = row[di * P + dj];   // in-bounds: i0 < tile, j0 < tile, P = tile + 2
+          // in-bounds: i0 < tile, j0 < tile, P = tile + 2; bins without overlap are not read
+          const float2 e2 = (ox3[di] > 0.f && oy3[dj] > 0.f) ? row[di * P + dj] : make_float2(0.f, 0.f);
           sx = fmaf(oy3[dj], e2.x, sx);
           sy = fmaf(oy3[dj], e2.y, sy);
         }
@@ -591,6 +602,8 @@ DenArgs make_args(const Ctx &c, const float *x, const float *y) {
   a.tile_cnt = c.d_tile_cnt;
   a.tile_cursor = c.d_tile_cursor;
   a.tile_off = c.d_tile_off;
+  a.walk_tile = c.d_walk_tile;
+  a.walk_grid = c.walk_grid;
   a.rec = c.d_rec;
   a.rec_rc = c.d_rec_rc;
   a.rec_cell = c.d_rec_cell;

@@ -451,6 +451,8 @@ dp_status build_density(Ctx &c, const dp_netlist *nl) {
   }
   c.walk_grid = density_walk_grid(c.tile);
   if (c.walk_grid <= 0) return fail(DP_ERR_CUDA, "density walker occupancy query failed");
+  if ((st = dev_alloc(c, &c.d_walk_tile, c.walk_grid)) != DP_OK) return st;
+  DP_CUDA(cudaMemset(c.d_walk_tile, 0, sizeof(int32_t) * c.walk_grid));
   return DP_OK;
 }
 

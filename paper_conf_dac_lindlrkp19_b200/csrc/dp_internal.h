@@ -117,7 +117,8 @@ struct Ctx {
   int2 *d_rec_rc = nullptr;           // per slot: (charge ratio r as float bits, i0 | j0 << 16)
   int32_t *d_rec_cell = nullptr;      // per slot: own cell index
   bool serial = false;     // DP_SERIAL=1: density chain after WA (no stream overlap; measurement)
-  int32_t walk_grid = 0;   // CTAs of the persistent scatter / gather walkers (SMs x resident)
+  int32_t walk_grid = 0;
+  int32_t *d_walk_tile = nullptr;   // [walk_grid]   // CTAs of the persistent scatter / gather walkers (SMs x resident)
   unsigned long long *d_rho = nullptr;  // bin map, int64 fixed point in units of 2^-kRhoScaleLog2 (exact, deterministic)
   float *d_t = nullptr, *d_sx = nullptr, *d_sy = nullptr;
   float2 *d_xi = nullptr;

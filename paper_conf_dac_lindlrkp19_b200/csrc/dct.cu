@@ -19,6 +19,7 @@
 // The energy D = 1/2 b_x b_y sum rho psi is taken in the spectral domain (Parseval), so psi
 // is never materialised on the hot path (reading A8).
 #include "dp_internal.h"
+#include "fft_warp.cuh"
 
 namespace dp {
 
@@ -149,6 +150,8 @@ struct RowInvArgs {
   float *outA, *outB;       // planes (row step n), used if outI == nullptr
   long long ostepA, ostepB;
   float2 *outI;             // interleaved output (row step n)
+  const float2 *inI;        // if set: interleaved input (A, B) with row step n (warp kernel only)
+  long long ostepT;         // if > 0 (warp kernel): outI[t * ostepT + r] (transposed store)
   int n, log2n;
   const float2 *tw, *ph;
 };
@@ -184,6 +187,124 @@ __global__ void __launch_bounds__(kRowThreads) k_row_inv(RowInvArgs a) {
     } else {
       a.outA[(long long)blockIdx.x * a.ostepA + t] = va;
       a.outB[(long long)blockIdx.x * a.ostepB + t] = vb;
+    }
+  }
+}
+
+// ---------------------------------------------------------------------------------------
+// Warp-FFT row kernels (N = 2^LOGN in [32, 1024]); every warp owns B = 1024 / N row pairs (T1)
+// or rows (T3) and never waits on a block barrier.
+// ---------------------------------------------------------------------------------------
+constexpr int kWRowWarps = 2;   // warps per CTA: a 1024-row map gives 256-512 CTAs
+
+// dct_post on values already loaded: z = Z[k], zc = Z[N - k]
+__device__ __forceinline__ float2 dct_post_v(float2 z, float2 zc, float2 ph, float scale) {
+  const float v0x = 0.5f * (z.x + zc.x), v0y = 0.5f * (z.y - zc.y);
+  const float dx = z.x - zc.x, dy = z.y + zc.y;
+  const float v1x = 0.5f * dy, v1y = -0.5f * dx;
+  return make_float2(scale * (v0x * ph.x - v0y * ph.y), scale * (v1x * ph.x - v1y * ph.y));
+}
+
+// T1: rows (2p, 2p+1) packed as one complex sequence (Makhoul order), DCT over y
+template <class IN, int LOGN>
+__global__ void __launch_bounds__(32 * kWRowWarps) k_row_dct_w(const IN *__restrict__ in, float *__restrict__ out,
+                                                             const float2 *__restrict__ tw2,
+                                                             const float2 *__restrict__ ph, int npairs) {
+  constexpr int N = 1 << LOGN, K = N / 32, B = wfft::kPts / N;
+  extern __shared__ float2 wsm[];
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  float2 *buf = wsm + warp * wfft::kBufPad;
+  const int p0 = (blockIdx.x * kWRowWarps + warp) * B;
+  if (p0 >= npairs) return;
+  float2 a[32];
+#pragma unroll
+  for (int s = 0; s < B; s++) {
+    const bool ok = p0 + s < npairs;
+    const IN *r0 = in + (size_t)(2 * (p0 + s)) * N, *r1 = r0 + N;
+#pragma unroll
+    for (int j = 0; j < K; j++) {
+      const int n = lane + 32 * j;
+      const int src = n < N / 2 ? 2 * n : 2 * (N - 1 - n) + 1;   // v[n] = x[2n], v[N-1-n] = x[2n+1]
+      a[s * K + j] = ok ? make_float2(load_map(r0 + src), load_map(r1 + src)) : make_float2(0.f, 0.f);
+    }
+  }
+  wfft::warp_fft<LOGN, false>(a, buf, tw2);
+  const float scale = 2.f / N;
+#pragma unroll
+  for (int s = 0; s < B; s++) {
+    if (p0 + s >= npairs) break;
+    float *o0 = out + (size_t)(2 * (p0 + s)) * N, *o1 = o0 + N;
+#pragma unroll
+    for (int j = 0; j < K; j++) {
+      const int k = lane + 32 * j;
+      const float2 v = dct_post_v(buf[wfft::pad(s * N + k)], buf[wfft::pad(s * N + ((N - k) & (N - 1)))],
+                                  __ldg(ph + k), scale);
+      o0[k] = v.x;
+      o1[k] = v.y;
+    }
+  }
+}
+
+// T3 / debug: row r of A (op opA) and row r of B (op opB) as one complex inverse sequence
+template <int LOGN>
+__global__ void __launch_bounds__(32 * kWRowWarps) k_row_inv_w(RowInvArgs a, const float2 *__restrict__ tw2, int rows) {
+  constexpr int N = 1 << LOGN, K = N / 32, B = wfft::kPts / N;
+  extern __shared__ float2 wsm[];
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  float2 *buf = wsm + warp * wfft::kBufPad;
+  const int r0 = (blockIdx.x * kWRowWarps + warp) * B;
+  if (r0 >= rows) return;
+  float2 v[32];
+#pragma unroll
+  for (int s = 0; s < B; s++) {
+    const bool ok = r0 + s < rows;
+    const float *ra = a.inA + (long long)(r0 + s) * a.stepA, *rb = a.inB + (long long)(r0 + s) * a.stepB;
+#pragma unroll
+    for (int j = 0; j < K; j++) {
+      const int k = lane + 32 * j;
+      float pk = 0.f, qk = 0.f, pnk = 0.f, qnk = 0.f;
+      if (ok) {
+        // IDXST input reversal (eq 8e): x'_t = x_{N-t}, x'_0 = 0
+        float ak, ank, bk, bnk;
+        if (a.inI) {
+          const float2 *ri = a.inI + (size_t)(r0 + s) * N;
+          const float2 vk = __ldg(ri + k), vn = k ? __ldg(ri + N - k) : make_float2(0.f, 0.f);
+          ak = vk.x; bk = vk.y; ank = vn.x; bnk = vn.y;
+        } else {
+          ak = __ldg(ra + k); ank = k ? __ldg(ra + N - k) : 0.f;
+          bk = __ldg(rb + k); bnk = k ? __ldg(rb + N - k) : 0.f;
+        }
+        pk = (a.opA == 2) ? ank : ak;
+        pnk = k ? ((a.opA == 2) ? ak : ank) : 0.f;
+        qk = (a.opB == 2) ? bnk : bk;
+        qnk = k ? ((a.opB == 2) ? bk : bnk) : 0.f;
+      }
+      v[s * K + j] = inv_pre(pk, qk, pnk, qnk, __ldg(a.ph + k));
+    }
+  }
+  wfft::warp_fft<LOGN, true>(v, buf, tw2);
+#pragma unroll
+  for (int s = 0; s < B; s++) {
+    const int r = r0 + s;
+    if (r >= rows) break;
+#pragma unroll
+    for (int j = 0; j < K; j++) {
+      const int t = lane + 32 * j;
+      const float2 z = buf[wfft::pad(s * N + mk_pos(t, N))];
+      float va = 0.5f * z.x, vb = 0.5f * z.y;
+      if (t & 1) {
+        if (a.opA == 2) va = -va;
+        if (a.opB == 2) vb = -vb;
+      }
+      if (a.outI) {
+        if (a.ostepT > 0)
+          a.outI[(size_t)t * a.ostepT + r] = make_float2(va, vb);
+        else
+          a.outI[(size_t)r * N + t] = make_float2(va, vb);
+      } else {
+        a.outA[(long long)r * a.ostepA + t] = va;
+        a.outB[(long long)r * a.ostepB + t] = vb;
+      }
     }
   }
 }
@@ -333,6 +454,64 @@ __global__ void __launch_bounds__(kColThreads) k_col_fields(ColFieldArgs a) {
   }
 }
 
+// T2a (warp FFT, M = mx = 2^LOGM in [32, 1024]): every warp owns B = 1024 / M column pairs of
+// t.  DCT_x of the pair as one complex sequence, the Parseval energy term and the spectral
+// scaling of eqs (9c)/(9d); writes (A_X, A_Y) transposed, specT[v][u] (row v contiguous), for
+// the inverse x pass (T2b = the row-inverse kernel on specT: IDXST_x of A_X + i IDCT_x of A_Y,
+// stored transposed into (sX, sY)[x][y]).  Splitting the column work in two keeps one FFT per
+// warp per kernel: these transforms are latency-bound at 512-1024 warps per map.
+constexpr int kWColWarps = 2;
+
+template <int LOGM>
+__global__ void __launch_bounds__(32 * kWColWarps) k_col_fwd_w(ColFieldArgs a, float2 *__restrict__ specT,
+                                                             const float2 *__restrict__ tw2) {
+  constexpr int M = 1 << LOGM, K = M / 32, B = wfft::kPts / M;
+  extern __shared__ float2 wsm[];
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  float2 *buf = wsm + warp * wfft::kBufPad;
+  const int gw = blockIdx.x * kWColWarps + warp;   // global warp: energy slot
+  const int p0 = gw * B;                           // first column pair
+  const int my = a.my, npairs = my / 2;
+  if (p0 >= npairs) return;
+  float2 z[32];
+#pragma unroll
+  for (int s = 0; s < B; s++) {
+    const bool ok = p0 + s < npairs;
+#pragma unroll
+    for (int j = 0; j < K; j++) {
+      const int n = lane + 32 * j;
+      const int src = n < M / 2 ? 2 * n : 2 * (M - 1 - n) + 1;   // Makhoul order along x
+      z[s * K + j] = ok ? __ldg(reinterpret_cast<const float2 *>(a.t + (size_t)src * my) + (p0 + s)) : make_float2(0.f, 0.f);
+    }
+  }
+  wfft::warp_fft<LOGM, false>(z, buf, tw2);
+  const float scale = 2.f / M;
+  double e = 0.0;
+#pragma unroll
+  for (int s = 0; s < B; s++) {
+    const int p = p0 + s;
+    if (p >= npairs) break;
+    const float ky0 = __ldg(a.ky + 2 * p), ky1 = __ldg(a.ky + 2 * p + 1);
+    const double wv0 = (p == 0) ? 0.25 * my : 0.5 * my, wv1 = 0.5 * my;
+#pragma unroll
+    for (int j = 0; j < K; j++) {
+      const int u = lane + 32 * j;
+      const float2 d = dct_post_v(buf[wfft::pad(s * M + u)], buf[wfft::pad(s * M + ((M - u) & (M - 1)))],
+                                  __ldg(a.ph_x + u), scale);   // (a_2p[u], a_2p+1[u])
+      const float kx = __ldg(a.kx + u);
+      const double wu = (u == 0) ? 0.25 * M : 0.5 * M;
+      const float ik0 = (u == 0 && p == 0) ? 0.f : __frcp_rn(kx * kx + ky0 * ky0);   // a_00 / k^2 := 0
+      const float ik1 = __frcp_rn(kx * kx + ky1 * ky1);
+      e += wu * (wv0 * (double)(d.x * d.x * ik0) + wv1 * (double)(d.y * d.y * ik1));
+      specT[(size_t)(2 * p) * M + u] = make_float2(d.x * kx * ik0, d.x * ky0 * ik0);
+      specT[(size_t)(2 * p + 1) * M + u] = make_float2(d.y * kx * ik1, d.y * ky1 * ik1);
+    }
+  }
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) e += __shfl_xor_sync(0xffffffffu, e, o);
+  if (lane == 0) a.energy_part[gw] = e * a.energy_scale;
+}
+
 // psi spectrum scaling for the debug hook: out = a / k^2 (0 at the DC term)
 __global__ void k_scale_psi(const float *a, float *out, const float *kx, const float *ky, int mx, int my) {
   const size_t n = (size_t)mx * my;
@@ -355,14 +534,59 @@ size_t row_smem(int n) { return (size_t)n * sizeof(float2) + 2 * (size_t)n * siz
 size_t col_generic_smem(int mx) { return (size_t)(col_slab(mx) / 2) * mx * sizeof(float2) + (size_t)col_slab(mx) * mx * sizeof(float); }
 size_t col_fields_smem(int mx) { return (size_t)col_slab(mx) * mx * sizeof(float2) + 2 * (size_t)col_slab(mx) * mx * sizeof(float); }
 
+bool warp_fft_ok(int log2n) { return log2n >= 5 && log2n <= 10; }
+size_t wrow_smem() { return (size_t)kWRowWarps * wfft::kBufPad * sizeof(float2); }
+int wrow_ctas(int units, int log2n) {   // units = row pairs (T1) or rows (T3)
+  const int per_warp = wfft::kPts >> log2n, per_cta = per_warp * kWRowWarps;
+  return (units + per_cta - 1) / per_cta;
+}
+
 void row_inv(const Ctx &c, const float *inA, long long stepA, int opA, const float *inB, long long stepB,
              int opB, float *outA, long long ostepA, float *outB, long long ostepB, float2 *outI,
-             int rows, cudaStream_t s) {
+             int rows, cudaStream_t s, const float2 *inI = nullptr, bool x_axis = false, long long ostepT = 0) {
   RowInvArgs a;
   a.inA = inA; a.inB = inB; a.stepA = stepA; a.stepB = stepB; a.opA = opA; a.opB = opB;
   a.outA = outA; a.outB = outB; a.ostepA = ostepA; a.ostepB = ostepB; a.outI = outI;
-  a.n = c.my; a.log2n = c.log2my; a.tw = c.d_tw_y; a.ph = c.d_ph_y;
-  k_row_inv<<<rows, kRowThreads, row_smem(c.my), s>>>(a);
+  a.inI = inI;
+  a.ostepT = ostepT;
+  const int log2n = x_axis ? c.log2mx : c.log2my;
+  const float2 *tw2 = x_axis ? c.d_tw2_x : c.d_tw2_y;
+  a.n = 1 << log2n; a.log2n = log2n;
+  a.tw = x_axis ? c.d_tw_x : c.d_tw_y;
+  a.ph = x_axis ? c.d_ph_x : c.d_ph_y;
+  if (!warp_fft_ok(log2n)) {
+    k_row_inv<<<rows, kRowThreads, row_smem(a.n), s>>>(a);
+    return;
+  }
+  const int g = wrow_ctas(rows, log2n);
+  const size_t sm = wrow_smem();
+  switch (log2n) {
+    case 5: k_row_inv_w<5><<<g, 32 * kWRowWarps, sm, s>>>(a, tw2, rows); break;
+    case 6: k_row_inv_w<6><<<g, 32 * kWRowWarps, sm, s>>>(a, tw2, rows); break;
+    case 7: k_row_inv_w<7><<<g, 32 * kWRowWarps, sm, s>>>(a, tw2, rows); break;
+    case 8: k_row_inv_w<8><<<g, 32 * kWRowWarps, sm, s>>>(a, tw2, rows); break;
+    case 9: k_row_inv_w<9><<<g, 32 * kWRowWarps, sm, s>>>(a, tw2, rows); break;
+    default: k_row_inv_w<10><<<g, 32 * kWRowWarps, sm, s>>>(a, tw2, rows); break;
+  }
+}
+
+// T1 dispatcher: DCT over y of every row of `in` (IN = float or the int64 map)
+template <class IN>
+void row_dct(const Ctx &c, const IN *in, float *out, cudaStream_t s) {
+  if (!warp_fft_ok(c.log2my)) {
+    k_row_dct<IN><<<c.mx / 2, kRowThreads, row_smem(c.my), s>>>(in, out, c.my, c.log2my, c.d_tw_y, c.d_ph_y);
+    return;
+  }
+  const int np = c.mx / 2, g = wrow_ctas(np, c.log2my);
+  const size_t sm = wrow_smem();
+  switch (c.log2my) {
+    case 5: k_row_dct_w<IN, 5><<<g, 32 * kWRowWarps, sm, s>>>(in, out, c.d_tw2_y, c.d_ph_y, np); break;
+    case 6: k_row_dct_w<IN, 6><<<g, 32 * kWRowWarps, sm, s>>>(in, out, c.d_tw2_y, c.d_ph_y, np); break;
+    case 7: k_row_dct_w<IN, 7><<<g, 32 * kWRowWarps, sm, s>>>(in, out, c.d_tw2_y, c.d_ph_y, np); break;
+    case 8: k_row_dct_w<IN, 8><<<g, 32 * kWRowWarps, sm, s>>>(in, out, c.d_tw2_y, c.d_ph_y, np); break;
+    case 9: k_row_dct_w<IN, 9><<<g, 32 * kWRowWarps, sm, s>>>(in, out, c.d_tw2_y, c.d_ph_y, np); break;
+    default: k_row_dct_w<IN, 10><<<g, 32 * kWRowWarps, sm, s>>>(in, out, c.d_tw2_y, c.d_ph_y, np); break;
+  }
 }
 
 }  // namespace
@@ -378,7 +602,9 @@ cudaError_t dct_configure(int mx, int my) {
   if (e != cudaSuccess) return e;
   e = cudaFuncSetAttribute(k_col_generic, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)col_generic_smem(mx));
   if (e != cudaSuccess) return e;
-  return cudaFuncSetAttribute(k_col_fields, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)col_fields_smem(mx));
+  e = cudaFuncSetAttribute(k_col_fields, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)col_fields_smem(mx));
+  if (e != cudaSuccess) return e;
+  return cudaSuccess;
 }
 
 int col_fields_ctas(int mx, int my) { return my / col_slab(mx); }
@@ -389,13 +615,12 @@ void fields_after_t1(const Ctx &c, cudaStream_t s);
 
 void launch_fields(const Ctx &c, const float *rho, cudaStream_t s) {
   // T1: t = DCT_y(rho)
-  k_row_dct<float><<<c.mx / 2, kRowThreads, row_smem(c.my), s>>>(rho, c.d_t, c.my, c.log2my, c.d_tw_y, c.d_ph_y);
+  row_dct<float>(c, rho, c.d_t, s);
   fields_after_t1(c, s);
 }
 
 void launch_fields_fixed(const Ctx &c, cudaStream_t s) {
-  k_row_dct<unsigned long long><<<c.mx / 2, kRowThreads, row_smem(c.my), s>>>(c.d_rho, c.d_t, c.my, c.log2my, c.d_tw_y,
-                                                                              c.d_ph_y);
+  row_dct<unsigned long long>(c, c.d_rho, c.d_t, s);
   fields_after_t1(c, s);
 }
 
@@ -417,6 +642,25 @@ void fields_after_t1(const Ctx &c, cudaStream_t s) {
   a.tw_x = c.d_tw_x; a.ph_x = c.d_ph_x; a.kx = c.d_kx; a.ky = c.d_ky;
   a.energy_part = c.d_part + c.n_wa_part;
   a.energy_scale = 0.5 * c.bx * c.by;
+  if (warp_fft_ok(c.log2mx) && warp_fft_ok(c.log2my)) {
+    const int warps = (c.my / 2) / (wfft::kPts >> c.log2mx);
+    const int g = (warps + kWColWarps - 1) / kWColWarps;
+    const size_t sm = (size_t)kWColWarps * wfft::kBufPad * sizeof(float2);
+    float2 *spec = c.d_spec, *sxy = c.d_sxy;
+    switch (c.log2mx) {   // T2a
+      case 5: k_col_fwd_w<5><<<g, 32 * kWColWarps, sm, s>>>(a, spec, c.d_tw2_x); break;
+      case 6: k_col_fwd_w<6><<<g, 32 * kWColWarps, sm, s>>>(a, spec, c.d_tw2_x); break;
+      case 7: k_col_fwd_w<7><<<g, 32 * kWColWarps, sm, s>>>(a, spec, c.d_tw2_x); break;
+      case 8: k_col_fwd_w<8><<<g, 32 * kWColWarps, sm, s>>>(a, spec, c.d_tw2_x); break;
+      case 9: k_col_fwd_w<9><<<g, 32 * kWColWarps, sm, s>>>(a, spec, c.d_tw2_x); break;
+      default: k_col_fwd_w<10><<<g, 32 * kWColWarps, sm, s>>>(a, spec, c.d_tw2_x); break;
+    }
+    // T2b: per column v (row v of specT): sX = IDXST_x(A_X), sY = IDCT_x(A_Y), stored [x][y]
+    row_inv(c, nullptr, 0, 2, nullptr, 0, 1, nullptr, 0, nullptr, 0, sxy, c.my, s, spec, true, c.my);
+    // T3: rows: xi_X = IDCT_y(sX), xi_Y = IDXST_y(sY), interleaved in and out
+    row_inv(c, nullptr, 0, 1, nullptr, 0, 2, nullptr, 0, nullptr, 0, c.d_xi, c.mx, s, sxy);
+    return;
+  }
   k_col_fields<<<c.my / col_slab(c.mx), kColThreads, col_fields_smem(c.mx), s>>>(a);
   // T3: rows: xi_X = IDCT_y(sX), xi_Y = IDXST_y(sY), interleaved
   row_inv(c, c.d_sx, c.my, 1, c.d_sy, c.my, 2, nullptr, 0, nullptr, 0, c.d_xi, c.mx, s);
@@ -432,7 +676,7 @@ void launch_transform(const Ctx &c, int kind, const float *in, float *out, cudaS
   float *tmp = c.d_t;  // scratch (debug path only)
   switch (kind) {
     case DP_T_DCT2:
-      k_row_dct<float><<<mx / 2, kRowThreads, row_smem(my), s>>>(in, tmp, my, c.log2my, c.d_tw_y, c.d_ph_y);
+      row_dct<float>(c, in, tmp, s);
       k_col_generic<<<my / col_slab(mx), kColThreads, col_generic_smem(mx), s>>>(tmp, out, 0, mx, c.log2mx, my, c.d_tw_x, c.d_ph_x);
       break;
     case DP_T_IDCT2:

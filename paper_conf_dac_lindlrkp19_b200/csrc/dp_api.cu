@@ -376,6 +376,18 @@ dp_status build_wa(Ctx &c, const dp_netlist *nl, const std::vector<uint8_t> &mas
   return DP_OK;
 }
 
+// warp-FFT four-step twiddles W_N^{n1 k2}, n1 < 32, k2 < N / 32, laid out [k2][n1] (fp64-rounded)
+std::vector<float2> twiddles2(int n) {
+  const int K = std::max(1, n / 32);
+  std::vector<float2> t((size_t)K * 32);
+  for (int k2 = 0; k2 < K; k2++)
+    for (int n1 = 0; n1 < 32; n1++) {
+      const double a = -2.0 * M_PI * (double)((n1 * k2) % n) / n;
+      t[(size_t)k2 * 32 + n1] = make_float2((float)std::cos(a), (float)std::sin(a));
+    }
+  return t;
+}
+
 std::vector<float2> twiddles(int n) {  // exp(-2 pi i k / n), k < n/2, from fp64
   std::vector<float2> t(n / 2);
   for (int k = 0; k < n / 2; k++) {
@@ -423,6 +435,8 @@ dp_status build_density(Ctx &c, const dp_netlist *nl) {
   if ((st = dev_alloc(c, &c.d_sx, nb)) != DP_OK) return st;
   if ((st = dev_alloc(c, &c.d_sy, nb)) != DP_OK) return st;
   if ((st = dev_alloc(c, &c.d_xi, nb)) != DP_OK) return st;
+  if ((st = dev_alloc(c, &c.d_sxy, nb)) != DP_OK) return st;
+  if ((st = dev_alloc(c, &c.d_spec, nb)) != DP_OK) return st;
   // force[i] for own cell i = cell_begin + i; offset by the parity of cell_begin so that even
   // global cells are 16-byte aligned (the combine pass reads cell pairs as float4)
   if ((st = dev_alloc(c, &c.d_force, c.n_own + 4)) != DP_OK) return st;
@@ -432,6 +446,8 @@ dp_status build_density(Ctx &c, const dp_netlist *nl) {
   if ((st = dev_upload(c, &c.d_tw_y, twiddles(c.my))) != DP_OK) return st;
   if ((st = dev_upload(c, &c.d_ph_x, phases(c.mx))) != DP_OK) return st;
   if ((st = dev_upload(c, &c.d_ph_y, phases(c.my))) != DP_OK) return st;
+  if ((st = dev_upload(c, &c.d_tw2_x, twiddles2(c.mx))) != DP_OK) return st;
+  if ((st = dev_upload(c, &c.d_tw2_y, twiddles2(c.my))) != DP_OK) return st;
   std::vector<float> kx(c.mx), ky(c.my);
   for (int u = 0; u < c.mx; u++) kx[u] = (float)(M_PI * u / (c.xh - c.xl));   // reading A12
   for (int v = 0; v < c.my; v++) ky[v] = (float)(M_PI * v / (c.yh - c.yl));
@@ -470,6 +486,7 @@ void destroy(Ctx *c) {
   if (c->ev_wa) cudaEventDestroy(c->ev_wa);
   if (c->ev_den) cudaEventDestroy(c->ev_den);
   if (c->ev_done) cudaEventDestroy(c->ev_done);
+  if (c->ev_map) cudaEventDestroy(c->ev_map);
   for (auto &v : c->prof_pairs)
     for (auto &p : v) {
       cudaEventDestroy(p.first);
@@ -534,8 +551,13 @@ dp_status create(const dp_netlist *nl, const dp_grid *grid, int device, int rank
   if ((st = dev_alloc(*c, &c->d_hy, 2 * (size_t)c->num_cells)) != DP_OK) return bail(st);  // x then y
   c->d_hx = nullptr;
   { const char *e = std::getenv("DP_SERIAL"); c->serial = e && e[0] == '1'; }
-  if (cudaStreamCreateWithFlags(&c->s_wa, cudaStreamNonBlocking) != cudaSuccess ||
-      cudaStreamCreateWithFlags(&c->s_den, cudaStreamNonBlocking) != cudaSuccess ||
+  { const char *e = std::getenv("DP_SCHED"); c->sched = e ? std::atoi(e) : 1; }
+  int prio_lo = 0, prio_hi = 0;
+  cudaDeviceGetStreamPriorityRange(&prio_lo, &prio_hi);
+  { const char *e = std::getenv("DP_PRIO"); if (e && e[0] == '0') prio_hi = prio_lo; }   // default: density first
+  if (cudaStreamCreateWithPriority(&c->s_wa, cudaStreamNonBlocking, prio_lo) != cudaSuccess ||
+      cudaStreamCreateWithPriority(&c->s_den, cudaStreamNonBlocking, prio_hi) != cudaSuccess ||
+      cudaEventCreateWithFlags(&c->ev_map, cudaEventDisableTiming) != cudaSuccess ||
       cudaEventCreateWithFlags(&c->ev_fork, cudaEventDisableTiming) != cudaSuccess ||
       cudaEventCreateWithFlags(&c->ev_wa, cudaEventDisableTiming) != cudaSuccess ||
       cudaEventCreateWithFlags(&c->ev_den, cudaEventDisableTiming) != cudaSuccess ||
@@ -602,6 +624,7 @@ dp_status density_chain(Ctx &c, const float *x, const float *y) {
       if (st != DP_OK) return st;
     }
   }
+  DP_CUDA(cudaEventRecord(c.ev_map, c.s_den));
   {
     StageMark m(c, DP_STAGE_FIELDS, c.s_den);
     launch_fields_fixed(c, c.s_den);
@@ -649,8 +672,15 @@ dp_status eval_impl(Ctx &c, const float *x, const float *y, float gamma, float l
   StageMark whole(c, DP_STAGE_EVAL, s);
   if (c.profiling) c.prof_evals++;
   DP_CUDA(cudaEventRecord(c.ev_fork, s));
+  if (do_den) {
+    DP_CUDA(cudaStreamWaitEvent(c.s_den, c.ev_fork, 0));
+    dp_status st = density_chain(c, x, y);
+    if (st != DP_OK) return st;
+    DP_CUDA(cudaEventRecord(c.ev_den, c.s_den));
+  }
   if (do_wa) {
-    DP_CUDA(cudaStreamWaitEvent(c.s_wa, c.ev_fork, 0));
+    DP_CUDA(cudaStreamWaitEvent(
+        c.s_wa, !do_den ? c.ev_fork : c.serial ? c.ev_den : c.sched == 1 ? c.ev_map : c.ev_fork, 0));
     {
       StageMark m(c, DP_STAGE_WA, c.s_wa);
       // clear the own-cell range of the WA gradient accumulator (read, not reset, by combine)
@@ -658,12 +688,6 @@ dp_status eval_impl(Ctx &c, const float *x, const float *y, float gamma, float l
       launch_wa(c, x, y, gamma, false, d_hpwl != nullptr, c.s_wa);
     }
     DP_CUDA(cudaEventRecord(c.ev_wa, c.s_wa));
-  }
-  if (do_den) {
-    DP_CUDA(cudaStreamWaitEvent(c.s_den, (c.serial && do_wa) ? c.ev_wa : c.ev_fork, 0));
-    dp_status st = density_chain(c, x, y);
-    if (st != DP_OK) return st;
-    DP_CUDA(cudaEventRecord(c.ev_den, c.s_den));
   }
   if (do_wa) DP_CUDA(cudaStreamWaitEvent(s, c.ev_wa, 0));
   if (do_den) DP_CUDA(cudaStreamWaitEvent(s, c.ev_den, 0));

@@ -116,7 +116,8 @@ struct Ctx {
   float4 *d_rec = nullptr;            // per slot: footprint box in tile-local bin units
   int2 *d_rec_rc = nullptr;           // per slot: (charge ratio r as float bits, i0 | j0 << 16)
   int32_t *d_rec_cell = nullptr;      // per slot: own cell index
-  bool serial = false;     // DP_SERIAL=1: density chain after WA (no stream overlap; measurement)
+  bool serial = false;
+  int sched = 0;           // DP_SCHED: 0 = WA from the fork, 1 = WA after the density map (overlaps the transforms)     // DP_SERIAL=1: density chain after WA (no stream overlap; measurement)
   int32_t walk_grid = 0;
   int32_t *d_walk_tile = nullptr;   // [walk_grid]   // CTAs of the persistent scatter / gather walkers (SMs x resident)
   unsigned long long *d_rho = nullptr;  // bin map, int64 fixed point in units of 2^-kRhoScaleLog2 (exact, deterministic)
@@ -125,6 +126,9 @@ struct Ctx {
   float2 *d_force = nullptr;          // per own cell: -(sum ov xi)
   float2 *d_tw_x = nullptr, *d_tw_y = nullptr;     // FFT twiddles W_N^k, k < N/2
   float2 *d_ph_x = nullptr, *d_ph_y = nullptr;     // e^{-i pi k / 2N}, k < N
+  float2 *d_spec = nullptr;                         // T2a -> T2b (A_X, A_Y) transposed [y][x]
+  float2 *d_sxy = nullptr;                          // T2 -> T3 interleaved (sX, sY) [x][y] (warp-FFT path)
+  float2 *d_tw2_x = nullptr, *d_tw2_y = nullptr;   // warp FFT: W_N^{n1 k2} at [k2 * 32 + n1] (N <= 1024)
   float *d_kx = nullptr, *d_ky = nullptr;          // wavenumbers (reading A12)
 
   // ---- shared scratch ----
@@ -138,6 +142,7 @@ struct Ctx {
   // ---- streams / events ----
   cudaStream_t s_wa = nullptr, s_den = nullptr;
   cudaEvent_t ev_fork = nullptr, ev_wa = nullptr, ev_den = nullptr;
+  cudaEvent_t ev_map = nullptr;    // density map complete (DP_SCHED=1 start of WA)
   cudaEvent_t ev_done = nullptr;   // end of the last call: serialises use from several streams
 
   // ---- NCCL (distributed) ----

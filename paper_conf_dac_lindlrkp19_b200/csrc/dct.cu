@@ -197,6 +197,13 @@ __global__ void __launch_bounds__(kRowThreads) k_row_inv(RowInvArgs a) {
 // ---------------------------------------------------------------------------------------
 constexpr int kWRowWarps = 2;   // warps per CTA: a 1024-row map gives 256-512 CTAs
 
+// 1/x to ~1 ulp on the MUFU (the IEEE __frcp_rn slow path stalled the column pass)
+__device__ __forceinline__ float fast_rcp(float x) {
+  float r;
+  asm("rcp.approx.f32 %0, %1;" : "=f"(r) : "f"(x));
+  return r;
+}
+
 // dct_post on values already loaded: z = Z[k], zc = Z[N - k]
 __device__ __forceinline__ float2 dct_post_v(float2 z, float2 zc, float2 ph, float scale) {
   const float v0x = 0.5f * (z.x + zc.x), v0y = 0.5f * (z.y - zc.y);
@@ -414,7 +421,7 @@ __global__ void __launch_bounds__(kColThreads) k_col_fields(ColFieldArgs a) {
     for (int h = 0; h < 2; h++) {
       const int col = 2 * pr + h, v = c0 + col;
       const float ky = __ldg(a.ky + v);
-      const float ik2 = (u == 0 && v == 0) ? 0.f : __frcp_rn(kx * kx + ky * ky);
+      const float ik2 = (u == 0 && v == 0) ? 0.f : fast_rcp(kx * kx + ky * ky);
       const float av = h ? d.y : d.x;
       const double wv = (v == 0) ? 0.25 * my : 0.5 * my;
       e += wu * wv * (double)(av * av * ik2);
@@ -500,8 +507,8 @@ __global__ void __launch_bounds__(32 * kWColWarps) k_col_fwd_w(ColFieldArgs a, f
                                   __ldg(a.ph_x + u), scale);   // (a_2p[u], a_2p+1[u])
       const float kx = __ldg(a.kx + u);
       const double wu = (u == 0) ? 0.25 * M : 0.5 * M;
-      const float ik0 = (u == 0 && p == 0) ? 0.f : __frcp_rn(kx * kx + ky0 * ky0);   // a_00 / k^2 := 0
-      const float ik1 = __frcp_rn(kx * kx + ky1 * ky1);
+      const float ik0 = (u == 0 && p == 0) ? 0.f : fast_rcp(kx * kx + ky0 * ky0);   // a_00 / k^2 := 0
+      const float ik1 = fast_rcp(kx * kx + ky1 * ky1);
       e += wu * (wv0 * (double)(d.x * d.x * ik0) + wv1 * (double)(d.y * d.y * ik1));
       specT[(size_t)(2 * p) * M + u] = make_float2(d.x * kx * ik0, d.x * ky0 * ik0);
       specT[(size_t)(2 * p + 1) * M + u] = make_float2(d.y * kx * ik1, d.y * ky1 * ik1);

@@ -400,7 +400,7 @@ __global__ void __launch_bounds__(kTileThreads) k_scatter_walk(DenArgs a) {
     s_lo[k] = 0u;
   }
   __syncthreads();
-  const float scale_hi = (float)(1 << kTileHiBits), scale_lo = (float)(1 << kTileLoBits);
+  const float scale_fx = (float)(1u << kRhoScaleLog2);
   int cur_tile = st.ch[0].tile, acc = 0;
   for (int c = 0;; c++) {
     const int b = c % kStages;
@@ -420,7 +420,7 @@ __global__ void __launch_bounds__(kTileThreads) k_scatter_walk(DenArgs a) {
     for (int k = threadIdx.x; k < n; k += blockDim.x) {
       const float4 q = B.rec[cc.off + k];
       const int2 rc = B.rc[cc.off + k];
-      const float r = __int_as_float(rc.x) * scale_hi;
+      const float r = __int_as_float(rc.x) * scale_fx;   // r 2^29
       const int i0 = rc.y & 0xffff, j0 = rc.y >> 16;
       float ox3[3], oy3[3];
       rec_overlaps(q, ox3, oy3);
@@ -430,9 +430,10 @@ __global__ void __launch_bounds__(kTileThreads) k_scatter_walk(DenArgs a) {
         const float rx = r * ox3[di];
 #pragma unroll
         for (int dj = 0; dj < 3; dj++) {
-          const float vh = rx * oy3[dj];   // v 2^hi_bits, exact scaling
-          const unsigned hi = (unsigned)vh;
-          const unsigned lo = (unsigned)((vh - (float)hi) * scale_lo);
+          // u = floor(v 2^29) < 2^30 (v <= 1; power-of-two scaling is exact), split into
+          // hi = floor(v 2^10) and lo = the low 19 bits (= floor(frac(v 2^10) 2^19))
+          const unsigned u = (unsigned)(rx * oy3[dj]);
+          const unsigned hi = u >> kTileLoBits, lo = u & ((1u << kTileLoBits) - 1u);
           const int k2 = base + di * P + dj;
           red_shared(s_hi + k2, hi);
           red_shared(s_lo + k2, lo);

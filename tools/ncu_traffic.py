@@ -1,5 +1,6 @@
-"""Write profiles/ncu_wa_traffic.json: DRAM bytes (read + write) per launch of the WA stage
-(k_wa_chunks + k_wa_big) from one `ncu --set full` capture, for bench.py's roofline.traffic."""
+"""Write profiles/ncu_wa_traffic.json: DRAM bytes (read + write) per launch of the WA kernel
+(k_wa_chunks: all nets in one launch) from one `ncu --set full` capture, for bench.py's
+roofline.traffic.   python tools/ncu_traffic.py <report.ncu-rep>"""
 import csv
 import json
 import subprocess
@@ -11,7 +12,6 @@ def dram_bytes(path, kname):
     rows = list(csv.reader(out.splitlines()))
     h, u = rows[0], rows[1]
     ki = h.index('Kernel Name')
-    tot = None
     for r in rows[2:]:
         if kname in r[ki]:
             b = 0.0
@@ -19,15 +19,13 @@ def dram_bytes(path, kname):
                 i = h.index(m)
                 scale = {'byte': 1, 'Kbyte': 1e3, 'Mbyte': 1e6, 'Gbyte': 1e9}[u[i]]
                 b += float(r[i].replace(',', '')) * scale
-            tot = b
-            break
-    return tot
+            return b
+    return None
 
 
 if __name__ == '__main__':
-    chunks = dram_bytes(sys.argv[1], 'k_wa_chunks')
-    big = dram_bytes(sys.argv[2] if len(sys.argv) > 2 else sys.argv[1], 'k_wa_big') or 0.0
-    out = {"dram_bytes_per_launch": chunks + big, "k_wa_chunks": chunks, "k_wa_big": big,
-           "source": sys.argv[1:]}
-    json.dump(out, open('profiles/ncu_wa_traffic.json', 'w'), indent=1)
+    b = dram_bytes(sys.argv[1], 'k_wa_chunks')
+    out = {"dram_bytes_per_launch": b, "kernel": "k_wa_chunks", "source": [sys.argv[1]]}
+    with open('profiles/ncu_wa_traffic.json', 'w') as f:
+        json.dump(out, f, indent=1)
     print(out)

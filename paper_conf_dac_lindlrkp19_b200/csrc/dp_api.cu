@@ -480,6 +480,8 @@ void destroy(Ctx *c) {
   nccl_destroy(*c);
   for (void *p : c->allocations) cudaFree(p);
   if (c->d_hx) cudaFreeHost(c->d_hx);
+  if (c->gexec) cudaGraphExecDestroy(c->gexec);
+  if (c->s_cap) cudaStreamDestroy(c->s_cap);
   if (c->s_wa) cudaStreamDestroy(c->s_wa);
   if (c->s_den) cudaStreamDestroy(c->s_den);
   if (c->ev_fork) cudaEventDestroy(c->ev_fork);
@@ -555,7 +557,9 @@ dp_status create(const dp_netlist *nl, const dp_grid *grid, int device, int rank
   int prio_lo = 0, prio_hi = 0;
   cudaDeviceGetStreamPriorityRange(&prio_lo, &prio_hi);
   { const char *e = std::getenv("DP_PRIO"); if (e && e[0] == '0') prio_hi = prio_lo; }   // default: density first
-  if (cudaStreamCreateWithPriority(&c->s_wa, cudaStreamNonBlocking, prio_lo) != cudaSuccess ||
+  { const char *e = std::getenv("DP_GRAPH"); c->use_graph = !(e && e[0] == '0'); }
+  if (cudaStreamCreateWithFlags(&c->s_cap, cudaStreamNonBlocking) != cudaSuccess ||
+      cudaStreamCreateWithPriority(&c->s_wa, cudaStreamNonBlocking, prio_lo) != cudaSuccess ||
       cudaStreamCreateWithPriority(&c->s_den, cudaStreamNonBlocking, prio_hi) != cudaSuccess ||
       cudaEventCreateWithFlags(&c->ev_map, cudaEventDisableTiming) != cudaSuccess ||
       cudaEventCreateWithFlags(&c->ev_fork, cudaEventDisableTiming) != cudaSuccess ||
@@ -664,11 +668,72 @@ dp_status call_end(Ctx &c, cudaStream_t s) {
   return DP_OK;
 }
 
+dp_status eval_body(Ctx &c, const float *x, const float *y, float gamma, float lambda, float *gx, float *gy,
+                    double *d_obj, double *d_wl, double *d_energy, double *d_hpwl, cudaStream_t s, bool do_wa,
+                    bool do_den);
+
+// Graph path: the whole evaluation (both streams, ~15 launches and their event edges) is
+// captured once per argument set into a CUDA graph and replayed with one cudaGraphLaunch;
+// a call with different arguments re-captures and updates the executable graph in place
+// (cudaGraphExecUpdate).  Skipped while profiling (per-stage events), for distributed
+// contexts (collectives) and when the caller is itself capturing.
+dp_status eval_graph(Ctx &c, const float *x, const float *y, float gamma, float lambda, float *gx, float *gy,
+                     double *d_obj, double *d_wl, double *d_energy, double *d_hpwl, cudaStream_t s, bool do_wa,
+                     bool do_den) {
+  const GraphKey key{x, y, gx, gy, d_obj, d_wl, d_energy, d_hpwl, gamma, lambda, do_wa, do_den};
+  if (!(c.gexec && key == c.gkey)) {
+    cudaGraph_t g = nullptr;
+    DP_CUDA(cudaStreamBeginCapture(c.s_cap, cudaStreamCaptureModeThreadLocal));
+    dp_status st = eval_body(c, x, y, gamma, lambda, gx, gy, d_obj, d_wl, d_energy, d_hpwl, c.s_cap, do_wa, do_den);
+    const cudaError_t ce = cudaStreamEndCapture(c.s_cap, &g);
+    if (st != DP_OK) {
+      if (g) cudaGraphDestroy(g);
+      return st;
+    }
+    if (ce != cudaSuccess) return cuda_fail(ce, "cudaStreamEndCapture");
+    if (c.gexec) {
+      cudaGraphExecUpdateResultInfo info;
+      if (cudaGraphExecUpdate(c.gexec, g, &info) != cudaSuccess) {
+        cudaGetLastError();
+        cudaGraphExecDestroy(c.gexec);
+        c.gexec = nullptr;
+      }
+    }
+    if (!c.gexec) {
+      // honour the captured stream priorities (density chain first), as in a stream launch
+      const cudaError_t ie = cudaGraphInstantiateWithFlags(&c.gexec, g, cudaGraphInstantiateFlagUseNodePriority);
+      if (ie != cudaSuccess) {
+        cudaGraphDestroy(g);
+        c.gexec = nullptr;
+        return cuda_fail(ie, "cudaGraphInstantiate");
+      }
+    }
+    cudaGraphDestroy(g);
+    c.gkey = key;
+  }
+  dp_status st0 = call_begin(c, s);
+  if (st0 != DP_OK) return st0;
+  DP_CUDA(cudaGraphLaunch(c.gexec, s));
+  return call_end(c, s);
+}
+
 dp_status eval_impl(Ctx &c, const float *x, const float *y, float gamma, float lambda, float *gx, float *gy,
                     double *d_obj, double *d_wl, double *d_energy, double *d_hpwl, cudaStream_t s, bool do_wa,
                     bool do_den) {
+  cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+  DP_CUDA(cudaStreamIsCapturing(s, &cs));
+  if (c.use_graph && !c.profiling && !c.dist && cs == cudaStreamCaptureStatusNone)
+    return eval_graph(c, x, y, gamma, lambda, gx, gy, d_obj, d_wl, d_energy, d_hpwl, s, do_wa, do_den);
   dp_status st0 = call_begin(c, s);
   if (st0 != DP_OK) return st0;
+  st0 = eval_body(c, x, y, gamma, lambda, gx, gy, d_obj, d_wl, d_energy, d_hpwl, s, do_wa, do_den);
+  if (st0 != DP_OK) return st0;
+  return call_end(c, s);
+}
+
+dp_status eval_body(Ctx &c, const float *x, const float *y, float gamma, float lambda, float *gx, float *gy,
+                    double *d_obj, double *d_wl, double *d_energy, double *d_hpwl, cudaStream_t s, bool do_wa,
+                    bool do_den) {
   StageMark whole(c, DP_STAGE_EVAL, s);
   if (c.profiling) c.prof_evals++;
   DP_CUDA(cudaEventRecord(c.ev_fork, s));
@@ -698,7 +763,7 @@ dp_status eval_impl(Ctx &c, const float *x, const float *y, float gamma, float l
     if (st != DP_OK) return st;
   }
   DP_CUDA(cudaGetLastError());
-  return call_end(c, s);
+  return DP_OK;
 }
 
 }  // namespace

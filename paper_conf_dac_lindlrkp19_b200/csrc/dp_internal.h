@@ -69,6 +69,18 @@ struct WaCaps {
   int pins, nets, groups, far;
 };
 
+// Arguments a captured evaluation graph was built for (kernel parameters are baked in).
+struct GraphKey {
+  const void *x = nullptr, *y = nullptr, *gx = nullptr, *gy = nullptr;
+  const void *obj = nullptr, *wl = nullptr, *en = nullptr, *hpwl = nullptr;
+  float gamma = 0.f, lambda = 0.f;
+  bool wa = false, den = false;
+  bool operator==(const GraphKey &o) const {
+    return x == o.x && y == o.y && gx == o.gx && gy == o.gy && obj == o.obj && wl == o.wl && en == o.en &&
+           hpwl == o.hpwl && gamma == o.gamma && lambda == o.lambda && wa == o.wa && den == o.den;
+  }
+};
+
 struct Ctx {
   // ---- identity ----
   int device = 0;
@@ -117,6 +129,10 @@ struct Ctx {
   int2 *d_rec_rc = nullptr;           // per slot: (charge ratio r as float bits, i0 | j0 << 16)
   int32_t *d_rec_cell = nullptr;      // per slot: own cell index
   bool serial = false;
+  bool use_graph = true;   // DP_GRAPH=0 disables the captured-graph evaluation path
+  cudaStream_t s_cap = nullptr;
+  cudaGraphExec_t gexec = nullptr;
+  GraphKey gkey;
   int sched = 0;           // DP_SCHED: 0 = WA from the fork, 1 = WA after the density map (overlaps the transforms)     // DP_SERIAL=1: density chain after WA (no stream overlap; measurement)
   int32_t walk_grid = 0;
   int32_t *d_walk_tile = nullptr;   // [walk_grid]   // CTAs of the persistent scatter / gather walkers (SMs x resident)

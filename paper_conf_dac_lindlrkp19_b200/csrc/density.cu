@@ -642,24 +642,46 @@ int density_walk_grid(int tile) {
 
 int density_launches(const Ctx &c) { return 6 + (c.n_large > 0 ? 1 : 0); }
 
-void launch_density_map(const Ctx &c, const float *x, const float *y, cudaStream_t s) {
+// aux (optional): a second stream for the large-cell CTAs, which then overlap the sort and the
+// tile walkers (joined back into s before return)
+void launch_density_map(const Ctx &c, const float *x, const float *y, cudaStream_t s, cudaStream_t aux) {
   const DenArgs a = make_args(c, x, y);
   const int ntiles = a.ntiles;
   const int nblk = (c.n_own + kCountCells - 1) / kCountCells;
   cudaMemsetAsync(c.d_rho, 0, sizeof(unsigned long long) * (size_t)c.mx * c.my, s);
+  const bool side = aux && c.n_large > 0;
+  if (side) {
+    cudaEventRecord(c.ev_aux_a, s);
+    cudaStreamWaitEvent(aux, c.ev_aux_a, 0);
+    k_scatter_large<<<c.n_large, 256, 0, aux>>>(a);
+    cudaEventRecord(c.ev_aux_b, aux);
+  }
   if (nblk > 0) {
     k_count<<<nblk, kCountThreads, ntiles * 4, s>>>(a);
     k_scan<<<1, 1024, 0, s>>>(a);
     k_place<<<nblk, kCountThreads, place_smem_bytes(ntiles), s>>>(a);
     k_scatter_walk<<<c.walk_grid, kTileThreads, walk_smem_bytes(c.tile), s>>>(a);
   }
-  if (c.n_large > 0) k_scatter_large<<<c.n_large, 256, 0, s>>>(a);
+  if (side)
+    cudaStreamWaitEvent(s, c.ev_aux_b, 0);
+  else if (c.n_large > 0)
+    k_scatter_large<<<c.n_large, 256, 0, s>>>(a);
 }
 
-void launch_density_gather(const Ctx &c, const float *x, const float *y, cudaStream_t s) {
+void launch_density_gather(const Ctx &c, const float *x, const float *y, cudaStream_t s, cudaStream_t aux) {
   const DenArgs a = make_args(c, x, y);
+  const bool side = aux && c.n_large > 0;
+  if (side) {
+    cudaEventRecord(c.ev_aux_a, s);
+    cudaStreamWaitEvent(aux, c.ev_aux_a, 0);
+    k_gather_large<<<c.n_large, 256, 0, aux>>>(a);
+    cudaEventRecord(c.ev_aux_b, aux);
+  }
   if (c.n_own > 0) k_gather_walk<<<c.walk_grid, kTileThreads, walk_smem_bytes(c.tile), s>>>(a);
-  if (c.n_large > 0) k_gather_large<<<c.n_large, 256, 0, s>>>(a);
+  if (side)
+    cudaStreamWaitEvent(s, c.ev_aux_b, 0);
+  else if (c.n_large > 0)
+    k_gather_large<<<c.n_large, 256, 0, s>>>(a);
 }
 
 }  // namespace dp

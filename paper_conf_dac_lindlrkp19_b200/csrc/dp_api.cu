@@ -477,6 +477,7 @@ void destroy(Ctx *c) {
   DeviceGuard g(c->device);
   if (c->s_wa) cudaStreamSynchronize(c->s_wa);
   if (c->s_den) cudaStreamSynchronize(c->s_den);
+  if (c->s_aux) cudaStreamSynchronize(c->s_aux);
   nccl_destroy(*c);
   for (void *p : c->allocations) cudaFree(p);
   if (c->d_hx) cudaFreeHost(c->d_hx);
@@ -489,6 +490,9 @@ void destroy(Ctx *c) {
   if (c->ev_den) cudaEventDestroy(c->ev_den);
   if (c->ev_done) cudaEventDestroy(c->ev_done);
   if (c->ev_map) cudaEventDestroy(c->ev_map);
+  for (cudaEvent_t e : {c->ev_aux_a, c->ev_aux_b, c->ev_join, c->ev_fin})
+    if (e) cudaEventDestroy(e);
+  if (c->s_aux) cudaStreamDestroy(c->s_aux);
   for (auto &v : c->prof_pairs)
     for (auto &p : v) {
       cudaEventDestroy(p.first);
@@ -562,6 +566,11 @@ dp_status create(const dp_netlist *nl, const dp_grid *grid, int device, int rank
       cudaStreamCreateWithPriority(&c->s_wa, cudaStreamNonBlocking, prio_lo) != cudaSuccess ||
       cudaStreamCreateWithPriority(&c->s_den, cudaStreamNonBlocking, prio_hi) != cudaSuccess ||
       cudaEventCreateWithFlags(&c->ev_map, cudaEventDisableTiming) != cudaSuccess ||
+      cudaStreamCreateWithPriority(&c->s_aux, cudaStreamNonBlocking, prio_hi) != cudaSuccess ||
+      cudaEventCreateWithFlags(&c->ev_aux_a, cudaEventDisableTiming) != cudaSuccess ||
+      cudaEventCreateWithFlags(&c->ev_aux_b, cudaEventDisableTiming) != cudaSuccess ||
+      cudaEventCreateWithFlags(&c->ev_join, cudaEventDisableTiming) != cudaSuccess ||
+      cudaEventCreateWithFlags(&c->ev_fin, cudaEventDisableTiming) != cudaSuccess ||
       cudaEventCreateWithFlags(&c->ev_fork, cudaEventDisableTiming) != cudaSuccess ||
       cudaEventCreateWithFlags(&c->ev_wa, cudaEventDisableTiming) != cudaSuccess ||
       cudaEventCreateWithFlags(&c->ev_den, cudaEventDisableTiming) != cudaSuccess ||
@@ -622,7 +631,7 @@ struct StageMark {
 dp_status density_chain(Ctx &c, const float *x, const float *y) {
   {
     StageMark m(c, DP_STAGE_MAP, c.s_den);
-    launch_density_map(c, x, y, c.s_den);
+    launch_density_map(c, x, y, c.s_den, c.s_aux);
     if (c.dist && c.nccl_comm) {
       dp_status st = nccl_allreduce_u64(c, c.d_rho, (size_t)c.mx * c.my, c.s_den);   // exact
       if (st != DP_OK) return st;
@@ -634,7 +643,7 @@ dp_status density_chain(Ctx &c, const float *x, const float *y) {
     launch_fields_fixed(c, c.s_den);
   }
   StageMark m(c, DP_STAGE_GATHER, c.s_den);
-  launch_density_gather(c, x, y, c.s_den);
+  launch_density_gather(c, x, y, c.s_den, c.s_aux);
   return DP_OK;
 }
 
@@ -758,9 +767,20 @@ dp_status eval_body(Ctx &c, const float *x, const float *y, float gamma, float l
   if (do_den) DP_CUDA(cudaStreamWaitEvent(s, c.ev_den, 0));
   {
     StageMark m(c, DP_STAGE_COMBINE, s);
-    launch_combine(c, do_den ? lambda : 0.f, gx, gy, do_wa, do_den, s);
-    dp_status st = finalize(c, lambda, do_wa, do_den, do_wa && d_hpwl != nullptr, d_obj, d_wl, d_energy, d_hpwl, s);
-    if (st != DP_OK) return st;
+    if (c.dist) {   // the finalize carries collectives: keep it on the caller stream
+      launch_combine(c, do_den ? lambda : 0.f, gx, gy, do_wa, do_den, s);
+      dp_status st = finalize(c, lambda, do_wa, do_den, do_wa && d_hpwl != nullptr, d_obj, d_wl, d_energy, d_hpwl, s);
+      if (st != DP_OK) return st;
+    } else {        // scalars (aux stream) beside the gradient combine (caller stream)
+      DP_CUDA(cudaEventRecord(c.ev_join, s));
+      DP_CUDA(cudaStreamWaitEvent(c.s_aux, c.ev_join, 0));
+      dp_status st =
+          finalize(c, lambda, do_wa, do_den, do_wa && d_hpwl != nullptr, d_obj, d_wl, d_energy, d_hpwl, c.s_aux);
+      if (st != DP_OK) return st;
+      DP_CUDA(cudaEventRecord(c.ev_fin, c.s_aux));
+      launch_combine(c, do_den ? lambda : 0.f, gx, gy, do_wa, do_den, s);
+      DP_CUDA(cudaStreamWaitEvent(s, c.ev_fin, 0));
+    }
   }
   DP_CUDA(cudaGetLastError());
   return DP_OK;

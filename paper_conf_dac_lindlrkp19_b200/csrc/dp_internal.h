@@ -158,7 +158,9 @@ struct Ctx {
   // ---- streams / events ----
   cudaStream_t s_wa = nullptr, s_den = nullptr;
   cudaEvent_t ev_fork = nullptr, ev_wa = nullptr, ev_den = nullptr;
-  cudaEvent_t ev_map = nullptr;    // density map complete (DP_SCHED=1 start of WA)
+  cudaEvent_t ev_map = nullptr;
+  cudaStream_t s_aux = nullptr;    // large cells and the finalize, beside the main chains
+  cudaEvent_t ev_aux_a = nullptr, ev_aux_b = nullptr, ev_join = nullptr, ev_fin = nullptr;    // density map complete (DP_SCHED=1 start of WA)
   cudaEvent_t ev_done = nullptr;   // end of the last call: serialises use from several streams
 
   // ---- NCCL (distributed) ----
@@ -191,8 +193,8 @@ dp_status cuda_fail(cudaError_t e, const char *what);
 void launch_wa(const Ctx &c, const float *x, const float *y, float gamma, bool hpwl_only,
                bool with_hpwl, cudaStream_t s);
 // density (density.cu)
-void launch_density_map(const Ctx &c, const float *x, const float *y, cudaStream_t s);
-void launch_density_gather(const Ctx &c, const float *x, const float *y, cudaStream_t s);
+void launch_density_map(const Ctx &c, const float *x, const float *y, cudaStream_t s, cudaStream_t aux = nullptr);
+void launch_density_gather(const Ctx &c, const float *x, const float *y, cudaStream_t s, cudaStream_t aux = nullptr);
 // transforms (dct.cu)
 void launch_fields(const Ctx &c, const float *rho, cudaStream_t s);            // rho as float (debug hook)
 void launch_fields_fixed(const Ctx &c, cudaStream_t s);                          // rho = c.d_rho (hot path)

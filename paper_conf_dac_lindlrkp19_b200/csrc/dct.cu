@@ -18,6 +18,7 @@
 // radix-2 DIT with bit-reversed loads and fp32 twiddles computed in fp64 at create.
 // The energy D = 1/2 b_x b_y sum rho psi is taken in the spectral domain (Parseval), so psi
 // is never materialised on the hot path (reading A8).
+#include "async_copy.cuh"
 #include "dp_internal.h"
 #include "fft_warp.cuh"
 
@@ -119,6 +120,11 @@ __device__ __forceinline__ float load_map(const unsigned long long *p) {
   return (float)((double)(long long)__ldg(p) * (1.0 / (double)(1ll << kRhoScaleLog2)));
 }
 
+__device__ __forceinline__ float smem_map(const float *p) { return *p; }
+__device__ __forceinline__ float smem_map(const unsigned long long *p) {
+  return (float)((double)(long long)*p * (1.0 / (double)(1ll << kRhoScaleLog2)));
+}
+
 template <class IN>
 __global__ void __launch_bounds__(kRowThreads) k_row_dct(const IN *__restrict__ in, float *__restrict__ out,
                                                          int n, int log2n, const float2 *__restrict__ tw,
@@ -152,6 +158,7 @@ struct RowInvArgs {
   float2 *outI;             // interleaved output (row step n)
   const float2 *inI;        // if set: interleaved input (A, B) with row step n (warp kernel only)
   long long ostepT;         // if > 0 (warp kernel): outI[t * ostepT + r] (transposed store)
+  int tma;                  // interleaved input by bulk copy (DP_ROW_TMA=0: per-lane loads, A/B)
   int n, log2n;
   const float2 *tw, *ph;
 };
@@ -216,26 +223,58 @@ __device__ __forceinline__ float2 dct_post_v(float2 z, float2 zc, float2 ph, flo
 template <class IN, int LOGN>
 __global__ void __launch_bounds__(32 * kWRowWarps) k_row_dct_w(const IN *__restrict__ in, float *__restrict__ out,
                                                              const float2 *__restrict__ tw2,
-                                                             const float2 *__restrict__ ph, int npairs) {
+                                                             const float2 *__restrict__ ph, int npairs, int tma) {
   constexpr int N = 1 << LOGN, K = N / 32, B = wfft::kPts / N;
   extern __shared__ float2 wsm[];
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   float2 *buf = wsm + warp * wfft::kBufPad;
   const int p0 = (blockIdx.x * kWRowWarps + warp) * B;
   if (p0 >= npairs) return;
+  // the warp's B row pairs (contiguous: rows 2 p0 .. 2 (p0 + B) - 1) land in its staging area by
+  // one bulk copy (the TMA queue keeps the whole transfer in flight; per-lane loads were
+  // limited by outstanding misses per SM)
+  IN *stage = reinterpret_cast<IN *>(wsm + kWRowWarps * wfft::kBufPad) + (size_t)warp * 2 * wfft::kPts;
+  __shared__ uint64_t s_bar[kWRowWarps];
+  const int nvalid = min(B, npairs - p0);
+  if (tma && lane == 0) {
+    mbar_init(&s_bar[warp]);
+    const unsigned bytes = (unsigned)(2 * N * nvalid * sizeof(IN));
+    mbar_expect_tx(&s_bar[warp], bytes);
+    bulk_g2s(stage, in + (size_t)(2 * p0) * N, bytes, &s_bar[warp]);
+  }
+  float2 twr[32], phr[K];   // table loads issued while the rows are in flight
+  wfft::load_twiddles<LOGN>(twr, tw2);
+#pragma unroll
+  for (int j = 0; j < K; j++) phr[j] = __ldg(ph + lane + 32 * j);
   float2 a[32];
+  if (tma) {
+    __syncwarp();
+    mbar_wait(&s_bar[warp], 0);
 #pragma unroll
-  for (int s = 0; s < B; s++) {
-    const bool ok = p0 + s < npairs;
-    const IN *r0 = in + (size_t)(2 * (p0 + s)) * N, *r1 = r0 + N;
+    for (int s = 0; s < B; s++) {
+      const bool ok = s < nvalid;
+      const IN *r0 = stage + (size_t)(2 * s) * N, *r1 = r0 + N;
 #pragma unroll
-    for (int j = 0; j < K; j++) {
-      const int n = lane + 32 * j;
-      const int src = n < N / 2 ? 2 * n : 2 * (N - 1 - n) + 1;   // v[n] = x[2n], v[N-1-n] = x[2n+1]
-      a[s * K + j] = ok ? make_float2(load_map(r0 + src), load_map(r1 + src)) : make_float2(0.f, 0.f);
+      for (int j = 0; j < K; j++) {
+        const int n = lane + 32 * j;
+        const int src = n < N / 2 ? 2 * n : 2 * (N - 1 - n) + 1;   // v[n] = x[2n], v[N-1-n] = x[2n+1]
+        a[s * K + j] = ok ? make_float2(smem_map(r0 + src), smem_map(r1 + src)) : make_float2(0.f, 0.f);
+      }
+    }
+  } else {
+#pragma unroll
+    for (int s = 0; s < B; s++) {
+      const bool ok = s < nvalid;
+      const IN *r0 = in + (size_t)(2 * (p0 + s)) * N, *r1 = r0 + N;
+#pragma unroll
+      for (int j = 0; j < K; j++) {
+        const int n = lane + 32 * j;
+        const int src = n < N / 2 ? 2 * n : 2 * (N - 1 - n) + 1;
+        a[s * K + j] = ok ? make_float2(load_map(r0 + src), load_map(r1 + src)) : make_float2(0.f, 0.f);
+      }
     }
   }
-  wfft::warp_fft<LOGN, false>(a, buf, tw2);
+  wfft::warp_fft<LOGN, false>(a, buf, twr);
   const float scale = 2.f / N;
 #pragma unroll
   for (int s = 0; s < B; s++) {
@@ -245,7 +284,7 @@ __global__ void __launch_bounds__(32 * kWRowWarps) k_row_dct_w(const IN *__restr
     for (int j = 0; j < K; j++) {
       const int k = lane + 32 * j;
       const float2 v = dct_post_v(buf[wfft::pad(s * N + k)], buf[wfft::pad(s * N + ((N - k) & (N - 1)))],
-                                  __ldg(ph + k), scale);
+                                  phr[j], scale);
       o0[k] = v.x;
       o1[k] = v.y;
     }
@@ -261,35 +300,62 @@ __global__ void __launch_bounds__(32 * kWRowWarps) k_row_inv_w(RowInvArgs a, con
   float2 *buf = wsm + warp * wfft::kBufPad;
   const int r0 = (blockIdx.x * kWRowWarps + warp) * B;
   if (r0 >= rows) return;
+  // interleaved input: the warp's B rows (contiguous) land in its buffer by one bulk copy;
+  // planar input (debug transforms): per-lane loads, staged through the buffer.  Either way each
+  // row is read once and the mirrored element N - k comes from the buffer.
+  __shared__ uint64_t s_bar[kWRowWarps];
+  const int nvalid = min(B, rows - r0);
+  if (a.inI && a.tma && lane == 0) {
+    mbar_init(&s_bar[warp]);
+    const unsigned bytes = (unsigned)(N * nvalid * sizeof(float2));
+    mbar_expect_tx(&s_bar[warp], bytes);
+    bulk_g2s(buf, a.inI + (size_t)r0 * N, bytes, &s_bar[warp]);
+  }
+  float2 twr[32], phr[K];   // table loads issued while the rows are in flight
+  wfft::load_twiddles<LOGN>(twr, tw2);
+#pragma unroll
+  for (int j = 0; j < K; j++) phr[j] = __ldg(a.ph + lane + 32 * j);
   float2 v[32];
+  if (a.inI && a.tma) {
+    __syncwarp();
+    mbar_wait(&s_bar[warp], 0);
+#pragma unroll
+    for (int s = 0; s < B; s++)
+#pragma unroll
+      for (int j = 0; j < K; j++) v[s * K + j] = s < nvalid ? buf[s * N + lane + 32 * j] : make_float2(0.f, 0.f);
+  } else {
+#pragma unroll
+    for (int s = 0; s < B; s++) {
+      const bool ok = s < nvalid;
+      const float *ra = a.inA + (long long)(r0 + s) * a.stepA, *rb = a.inB + (long long)(r0 + s) * a.stepB;
+      const float2 *ri = a.inI ? a.inI + (size_t)(r0 + s) * N : nullptr;
+#pragma unroll
+      for (int j = 0; j < K; j++) {
+        const int k = lane + 32 * j;
+        v[s * K + j] = !ok ? make_float2(0.f, 0.f) : ri ? __ldg(ri + k) : make_float2(__ldg(ra + k), __ldg(rb + k));
+      }
+    }
+#pragma unroll
+    for (int q = 0; q < B * K; q++) buf[q * 32 + lane] = v[q];
+    __syncwarp();
+  }
 #pragma unroll
   for (int s = 0; s < B; s++) {
-    const bool ok = r0 + s < rows;
-    const float *ra = a.inA + (long long)(r0 + s) * a.stepA, *rb = a.inB + (long long)(r0 + s) * a.stepB;
 #pragma unroll
     for (int j = 0; j < K; j++) {
       const int k = lane + 32 * j;
-      float pk = 0.f, qk = 0.f, pnk = 0.f, qnk = 0.f;
-      if (ok) {
-        // IDXST input reversal (eq 8e): x'_t = x_{N-t}, x'_0 = 0
-        float ak, ank, bk, bnk;
-        if (a.inI) {
-          const float2 *ri = a.inI + (size_t)(r0 + s) * N;
-          const float2 vk = __ldg(ri + k), vn = k ? __ldg(ri + N - k) : make_float2(0.f, 0.f);
-          ak = vk.x; bk = vk.y; ank = vn.x; bnk = vn.y;
-        } else {
-          ak = __ldg(ra + k); ank = k ? __ldg(ra + N - k) : 0.f;
-          bk = __ldg(rb + k); bnk = k ? __ldg(rb + N - k) : 0.f;
-        }
-        pk = (a.opA == 2) ? ank : ak;
-        pnk = k ? ((a.opA == 2) ? ak : ank) : 0.f;
-        qk = (a.opB == 2) ? bnk : bk;
-        qnk = k ? ((a.opB == 2) ? bk : bnk) : 0.f;
-      }
-      v[s * K + j] = inv_pre(pk, qk, pnk, qnk, __ldg(a.ph + k));
+      const float2 vk = v[s * K + j];
+      const float2 vn = k ? buf[s * N + N - k] : make_float2(0.f, 0.f);
+      // IDXST input reversal (eq 8e): x'_t = x_{N-t}, x'_0 = 0
+      const float pk = (a.opA == 2) ? vn.x : vk.x;
+      const float pnk = k ? ((a.opA == 2) ? vk.x : vn.x) : 0.f;
+      const float qk = (a.opB == 2) ? vn.y : vk.y;
+      const float qnk = k ? ((a.opB == 2) ? vk.y : vn.y) : 0.f;
+      v[s * K + j] = inv_pre(pk, qk, pnk, qnk, phr[j]);
     }
   }
-  wfft::warp_fft<LOGN, true>(v, buf, tw2);
+  __syncwarp();
+  wfft::warp_fft<LOGN, true>(v, buf, twr);
 #pragma unroll
   for (int s = 0; s < B; s++) {
     const int r = r0 + s;
@@ -480,6 +546,14 @@ __global__ void __launch_bounds__(32 * kWColWarps) k_col_fwd_w(ColFieldArgs a, f
   const int p0 = gw * B;                           // first column pair
   const int my = a.my, npairs = my / 2;
   if (p0 >= npairs) return;
+  float2 twr[32], phr[K];   // table loads issued with the data loads (one memory latency)
+  float kxr[K];
+  wfft::load_twiddles<LOGM>(twr, tw2);
+#pragma unroll
+  for (int j = 0; j < K; j++) {
+    phr[j] = __ldg(a.ph_x + lane + 32 * j);
+    kxr[j] = __ldg(a.kx + lane + 32 * j);
+  }
   float2 z[32];
 #pragma unroll
   for (int s = 0; s < B; s++) {
@@ -491,7 +565,7 @@ __global__ void __launch_bounds__(32 * kWColWarps) k_col_fwd_w(ColFieldArgs a, f
       z[s * K + j] = ok ? __ldg(reinterpret_cast<const float2 *>(a.t + (size_t)src * my) + (p0 + s)) : make_float2(0.f, 0.f);
     }
   }
-  wfft::warp_fft<LOGM, false>(z, buf, tw2);
+  wfft::warp_fft<LOGM, false>(z, buf, twr);
   const float scale = 2.f / M;
   double e = 0.0;
 #pragma unroll
@@ -504,8 +578,8 @@ __global__ void __launch_bounds__(32 * kWColWarps) k_col_fwd_w(ColFieldArgs a, f
     for (int j = 0; j < K; j++) {
       const int u = lane + 32 * j;
       const float2 d = dct_post_v(buf[wfft::pad(s * M + u)], buf[wfft::pad(s * M + ((M - u) & (M - 1)))],
-                                  __ldg(a.ph_x + u), scale);   // (a_2p[u], a_2p+1[u])
-      const float kx = __ldg(a.kx + u);
+                                  phr[j], scale);   // (a_2p[u], a_2p+1[u])
+      const float kx = kxr[j];
       const double wu = (u == 0) ? 0.25 * M : 0.5 * M;
       const float ik0 = (u == 0 && p == 0) ? 0.f : fast_rcp(kx * kx + ky0 * ky0);   // a_00 / k^2 := 0
       const float ik1 = fast_rcp(kx * kx + ky1 * ky1);
@@ -518,6 +592,107 @@ __global__ void __launch_bounds__(32 * kWColWarps) k_col_fwd_w(ColFieldArgs a, f
   for (int o = 16; o > 0; o >>= 1) e += __shfl_xor_sync(0xffffffffu, e, o);
   if (lane == 0) a.energy_part[gw] = e * a.energy_scale;
 }
+
+// T2 fused (warp FFT, M = mx = 2^LOGM in [32, 1024]): every warp owns B = 1024 / M column pairs
+// of t and runs, per pair, the forward DCT_x of both columns as one complex FFT, the Parseval
+// energy term and the spectral scaling of eqs (9c)/(9d) (a_00 / k^2 := 0), then per column the
+// inverse x pass IDXST_x(A_X) + i IDCT_x(A_Y) as one complex IFFT (eq 8e reversal), and writes
+// (sX, sY) of both columns as one 16-byte store per row: sxy[x][2p], sxy[x][2p+1].  One kernel
+// instead of T2a + T2b: the spectrum never leaves shared memory.
+template <int LOGM>
+__global__ void __launch_bounds__(32 * kWColWarps) k_col_fields_w(ColFieldArgs a, float2 *__restrict__ sxy,
+                                                                const float2 *__restrict__ tw2) {
+  constexpr int M = 1 << LOGM, K = M / 32, B = wfft::kPts / M;
+  extern __shared__ float2 wsm[];
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  float2 *buf = wsm + warp * (wfft::kBufPad + 2 * wfft::kPts);
+  float2 *spec = buf + wfft::kBufPad;   // [2][kPts]: (A_X, A_Y) of column 2p (h = 0) / 2p + 1 (h = 1)
+  const int gw = blockIdx.x * kWColWarps + warp;   // global warp: energy slot
+  const int p0 = gw * B;                           // first column pair
+  const int my = a.my, npairs = my / 2;
+  if (p0 >= npairs) return;
+  float2 twr[32], phr[K];   // table loads issued with the data loads (one memory latency)
+  float kxr[K];
+  wfft::load_twiddles<LOGM>(twr, tw2);
+#pragma unroll
+  for (int j = 0; j < K; j++) {
+    phr[j] = __ldg(a.ph_x + lane + 32 * j);
+    kxr[j] = __ldg(a.kx + lane + 32 * j);
+  }
+  float2 z[32];
+#pragma unroll
+  for (int s = 0; s < B; s++) {
+    const bool ok = p0 + s < npairs;
+#pragma unroll
+    for (int j = 0; j < K; j++) {
+      const int n = lane + 32 * j;
+      const int src = n < M / 2 ? 2 * n : 2 * (M - 1 - n) + 1;   // Makhoul order along x
+      z[s * K + j] = ok ? __ldg(reinterpret_cast<const float2 *>(a.t + (size_t)src * my) + (p0 + s)) : make_float2(0.f, 0.f);
+    }
+  }
+  wfft::warp_fft<LOGM, false>(z, buf, twr);
+  const float scale = 2.f / M;
+  double e = 0.0;
+#pragma unroll
+  for (int s = 0; s < B; s++) {
+    const int p = p0 + s;
+    const bool ok = p < npairs;
+    const float ky0 = ok ? __ldg(a.ky + 2 * p) : 0.f, ky1 = ok ? __ldg(a.ky + 2 * p + 1) : 0.f;
+    const double wv0 = (p == 0) ? 0.25 * my : 0.5 * my, wv1 = 0.5 * my;
+#pragma unroll
+    for (int j = 0; j < K; j++) {
+      const int u = lane + 32 * j;
+      const float2 d = dct_post_v(buf[wfft::pad(s * M + u)], buf[wfft::pad(s * M + ((M - u) & (M - 1)))],
+                                  phr[j], scale);   // (a_2p[u], a_2p+1[u])
+      const float kx = kxr[j];
+      const double wu = (u == 0) ? 0.25 * M : 0.5 * M;
+      const float ik0 = (!ok || (u == 0 && p == 0)) ? 0.f : fast_rcp(kx * kx + ky0 * ky0);   // a_00 / k^2 := 0
+      const float ik1 = ok ? fast_rcp(kx * kx + ky1 * ky1) : 0.f;
+      e += wu * (wv0 * (double)(d.x * d.x * ik0) + wv1 * (double)(d.y * d.y * ik1));
+      spec[s * M + u] = make_float2(d.x * kx * ik0, d.x * ky0 * ik0);
+      spec[wfft::kPts + s * M + u] = make_float2(d.y * kx * ik1, d.y * ky1 * ik1);
+    }
+  }
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) e += __shfl_xor_sync(0xffffffffu, e, o);
+  if (lane == 0) a.energy_part[gw] = e * a.energy_scale;
+  __syncwarp();
+  float2 r0[32];
+#pragma unroll
+  for (int h = 0; h < 2; h++) {
+    const float2 *A = spec + h * wfft::kPts;
+    float2 v[32];
+#pragma unroll
+    for (int s = 0; s < B; s++) {
+#pragma unroll
+      for (int j = 0; j < K; j++) {
+        const int k = lane + 32 * j;
+        const float2 ak = A[s * M + k], ank = k ? A[s * M + M - k] : make_float2(0.f, 0.f);
+        // p = A_X reversed (IDXST via eq 8e: x'_t = x_{N-t}, x'_0 = 0), q = A_Y (IDCT)
+        v[s * K + j] = inv_pre(ank.x, ak.y, k ? ak.x : 0.f, ank.y, phr[j]);
+      }
+    }
+    wfft::warp_fft<LOGM, true>(v, buf, twr);
+#pragma unroll
+    for (int s = 0; s < B; s++) {
+#pragma unroll
+      for (int j = 0; j < K; j++) {
+        const int t = lane + 32 * j;
+        const float2 zz = buf[wfft::pad(s * M + mk_pos(t, M))];
+        const float2 o = make_float2((t & 1) ? -0.5f * zz.x : 0.5f * zz.x, 0.5f * zz.y);   // IDXST sign (-1)^x
+        if (h == 0) {
+          r0[s * K + j] = o;
+        } else if (p0 + s < npairs) {
+          const float2 q = r0[s * K + j];
+          *reinterpret_cast<float4 *>(sxy + (size_t)t * my + 2 * (p0 + s)) = make_float4(q.x, q.y, o.x, o.y);
+        }
+      }
+    }
+    __syncwarp();   // buf is reused by the next inverse
+  }
+}
+
+size_t col_fields_w_smem() { return (size_t)kWColWarps * (wfft::kBufPad + 2 * wfft::kPts) * sizeof(float2); }
 
 // psi spectrum scaling for the debug hook: out = a / k^2 (0 at the DC term)
 __global__ void k_scale_psi(const float *a, float *out, const float *kx, const float *ky, int mx, int my) {
@@ -543,6 +718,8 @@ size_t col_fields_smem(int mx) { return (size_t)col_slab(mx) * mx * sizeof(float
 
 bool warp_fft_ok(int log2n) { return log2n >= 5 && log2n <= 10; }
 size_t wrow_smem() { return (size_t)kWRowWarps * wfft::kBufPad * sizeof(float2); }
+// T1: FFT buffers + per-warp staging of 2 * 1024 input values (8 bytes each at most)
+size_t wrow_dct_smem() { return wrow_smem() + (size_t)kWRowWarps * 2 * wfft::kPts * sizeof(unsigned long long); }
 int wrow_ctas(int units, int log2n) {   // units = row pairs (T1) or rows (T3)
   const int per_warp = wfft::kPts >> log2n, per_cta = per_warp * kWRowWarps;
   return (units + per_cta - 1) / per_cta;
@@ -556,6 +733,7 @@ void row_inv(const Ctx &c, const float *inA, long long stepA, int opA, const flo
   a.outA = outA; a.outB = outB; a.ostepA = ostepA; a.ostepB = ostepB; a.outI = outI;
   a.inI = inI;
   a.ostepT = ostepT;
+  a.tma = c.row_tma ? 1 : 0;
   const int log2n = x_axis ? c.log2mx : c.log2my;
   const float2 *tw2 = x_axis ? c.d_tw2_x : c.d_tw2_y;
   a.n = 1 << log2n; a.log2n = log2n;
@@ -585,14 +763,14 @@ void row_dct(const Ctx &c, const IN *in, float *out, cudaStream_t s) {
     return;
   }
   const int np = c.mx / 2, g = wrow_ctas(np, c.log2my);
-  const size_t sm = wrow_smem();
+  const size_t sm = c.t1_tma ? wrow_dct_smem() : wrow_smem();
   switch (c.log2my) {
-    case 5: k_row_dct_w<IN, 5><<<g, 32 * kWRowWarps, sm, s>>>(in, out, c.d_tw2_y, c.d_ph_y, np); break;
-    case 6: k_row_dct_w<IN, 6><<<g, 32 * kWRowWarps, sm, s>>>(in, out, c.d_tw2_y, c.d_ph_y, np); break;
-    case 7: k_row_dct_w<IN, 7><<<g, 32 * kWRowWarps, sm, s>>>(in, out, c.d_tw2_y, c.d_ph_y, np); break;
-    case 8: k_row_dct_w<IN, 8><<<g, 32 * kWRowWarps, sm, s>>>(in, out, c.d_tw2_y, c.d_ph_y, np); break;
-    case 9: k_row_dct_w<IN, 9><<<g, 32 * kWRowWarps, sm, s>>>(in, out, c.d_tw2_y, c.d_ph_y, np); break;
-    default: k_row_dct_w<IN, 10><<<g, 32 * kWRowWarps, sm, s>>>(in, out, c.d_tw2_y, c.d_ph_y, np); break;
+    case 5: k_row_dct_w<IN, 5><<<g, 32 * kWRowWarps, sm, s>>>(in, out, c.d_tw2_y, c.d_ph_y, np, c.t1_tma ? 1 : 0); break;
+    case 6: k_row_dct_w<IN, 6><<<g, 32 * kWRowWarps, sm, s>>>(in, out, c.d_tw2_y, c.d_ph_y, np, c.t1_tma ? 1 : 0); break;
+    case 7: k_row_dct_w<IN, 7><<<g, 32 * kWRowWarps, sm, s>>>(in, out, c.d_tw2_y, c.d_ph_y, np, c.t1_tma ? 1 : 0); break;
+    case 8: k_row_dct_w<IN, 8><<<g, 32 * kWRowWarps, sm, s>>>(in, out, c.d_tw2_y, c.d_ph_y, np, c.t1_tma ? 1 : 0); break;
+    case 9: k_row_dct_w<IN, 9><<<g, 32 * kWRowWarps, sm, s>>>(in, out, c.d_tw2_y, c.d_ph_y, np, c.t1_tma ? 1 : 0); break;
+    default: k_row_dct_w<IN, 10><<<g, 32 * kWRowWarps, sm, s>>>(in, out, c.d_tw2_y, c.d_ph_y, np, c.t1_tma ? 1 : 0); break;
   }
 }
 
@@ -611,6 +789,24 @@ cudaError_t dct_configure(int mx, int my) {
   if (e != cudaSuccess) return e;
   e = cudaFuncSetAttribute(k_col_fields, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)col_fields_smem(mx));
   if (e != cudaSuccess) return e;
+  const int dsm = (int)wrow_dct_smem();
+  for (auto f : {k_row_dct_w<float, 5>, k_row_dct_w<float, 6>, k_row_dct_w<float, 7>, k_row_dct_w<float, 8>,
+                 k_row_dct_w<float, 9>, k_row_dct_w<float, 10>}) {
+    e = cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, dsm);
+    if (e != cudaSuccess) return e;
+  }
+  for (auto f : {k_row_dct_w<unsigned long long, 5>, k_row_dct_w<unsigned long long, 6>,
+                 k_row_dct_w<unsigned long long, 7>, k_row_dct_w<unsigned long long, 8>,
+                 k_row_dct_w<unsigned long long, 9>, k_row_dct_w<unsigned long long, 10>}) {
+    e = cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, dsm);
+    if (e != cudaSuccess) return e;
+  }
+  const int wsm = (int)col_fields_w_smem();
+  for (auto f : {k_col_fields_w<5>, k_col_fields_w<6>, k_col_fields_w<7>, k_col_fields_w<8>, k_col_fields_w<9>,
+                 k_col_fields_w<10>}) {
+    e = cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, wsm);
+    if (e != cudaSuccess) return e;
+  }
   return cudaSuccess;
 }
 
@@ -650,20 +846,33 @@ void fields_after_t1(const Ctx &c, cudaStream_t s) {
   a.energy_part = c.d_part + c.n_wa_part;
   a.energy_scale = 0.5 * c.bx * c.by;
   if (warp_fft_ok(c.log2mx) && warp_fft_ok(c.log2my)) {
-    const int warps = (c.my / 2) / (wfft::kPts >> c.log2mx);
+    const int warps = ((c.my / 2) + (wfft::kPts >> c.log2mx) - 1) / (wfft::kPts >> c.log2mx);
     const int g = (warps + kWColWarps - 1) / kWColWarps;
-    const size_t sm = (size_t)kWColWarps * wfft::kBufPad * sizeof(float2);
-    float2 *spec = c.d_spec, *sxy = c.d_sxy;
-    switch (c.log2mx) {   // T2a
-      case 5: k_col_fwd_w<5><<<g, 32 * kWColWarps, sm, s>>>(a, spec, c.d_tw2_x); break;
-      case 6: k_col_fwd_w<6><<<g, 32 * kWColWarps, sm, s>>>(a, spec, c.d_tw2_x); break;
-      case 7: k_col_fwd_w<7><<<g, 32 * kWColWarps, sm, s>>>(a, spec, c.d_tw2_x); break;
-      case 8: k_col_fwd_w<8><<<g, 32 * kWColWarps, sm, s>>>(a, spec, c.d_tw2_x); break;
-      case 9: k_col_fwd_w<9><<<g, 32 * kWColWarps, sm, s>>>(a, spec, c.d_tw2_x); break;
-      default: k_col_fwd_w<10><<<g, 32 * kWColWarps, sm, s>>>(a, spec, c.d_tw2_x); break;
+    float2 *sxy = c.d_sxy;
+    if (c.fused_t2) {   // measured slower at 1024^2 (longer per-warp latency chain); kept for A/B
+      const size_t sm = col_fields_w_smem();
+      switch (c.log2mx) {   // T2: DCT_x, scaling, energy, IDXST_x / IDCT_x in one pass
+        case 5: k_col_fields_w<5><<<g, 32 * kWColWarps, sm, s>>>(a, sxy, c.d_tw2_x); break;
+        case 6: k_col_fields_w<6><<<g, 32 * kWColWarps, sm, s>>>(a, sxy, c.d_tw2_x); break;
+        case 7: k_col_fields_w<7><<<g, 32 * kWColWarps, sm, s>>>(a, sxy, c.d_tw2_x); break;
+        case 8: k_col_fields_w<8><<<g, 32 * kWColWarps, sm, s>>>(a, sxy, c.d_tw2_x); break;
+        case 9: k_col_fields_w<9><<<g, 32 * kWColWarps, sm, s>>>(a, sxy, c.d_tw2_x); break;
+        default: k_col_fields_w<10><<<g, 32 * kWColWarps, sm, s>>>(a, sxy, c.d_tw2_x); break;
+      }
+    } else {
+      const size_t sm = (size_t)kWColWarps * wfft::kBufPad * sizeof(float2);
+      float2 *spec = c.d_spec;
+      switch (c.log2mx) {   // T2a
+        case 5: k_col_fwd_w<5><<<g, 32 * kWColWarps, sm, s>>>(a, spec, c.d_tw2_x); break;
+        case 6: k_col_fwd_w<6><<<g, 32 * kWColWarps, sm, s>>>(a, spec, c.d_tw2_x); break;
+        case 7: k_col_fwd_w<7><<<g, 32 * kWColWarps, sm, s>>>(a, spec, c.d_tw2_x); break;
+        case 8: k_col_fwd_w<8><<<g, 32 * kWColWarps, sm, s>>>(a, spec, c.d_tw2_x); break;
+        case 9: k_col_fwd_w<9><<<g, 32 * kWColWarps, sm, s>>>(a, spec, c.d_tw2_x); break;
+        default: k_col_fwd_w<10><<<g, 32 * kWColWarps, sm, s>>>(a, spec, c.d_tw2_x); break;
+      }
+      // T2b: per column v (row v of specT): sX = IDXST_x(A_X), sY = IDCT_x(A_Y), stored [x][y]
+      row_inv(c, nullptr, 0, 2, nullptr, 0, 1, nullptr, 0, nullptr, 0, sxy, c.my, s, spec, true, c.my);
     }
-    // T2b: per column v (row v of specT): sX = IDXST_x(A_X), sY = IDCT_x(A_Y), stored [x][y]
-    row_inv(c, nullptr, 0, 2, nullptr, 0, 1, nullptr, 0, nullptr, 0, sxy, c.my, s, spec, true, c.my);
     // T3: rows: xi_X = IDCT_y(sX), xi_Y = IDXST_y(sY), interleaved in and out
     row_inv(c, nullptr, 0, 1, nullptr, 0, 2, nullptr, 0, nullptr, 0, c.d_xi, c.mx, s, sxy);
     return;

@@ -28,6 +28,7 @@
 // Footprint geometry is computed in fp64 (B200 runs FP64 at half rate); records hold the
 // footprint in fractions of the cell's first bin (|v| < 3) plus that bin's tile-local index.
 #include <algorithm>
+#include <cmath>
 
 #include "async_copy.cuh"
 #include "dp_internal.h"
@@ -45,6 +46,7 @@ struct DenArgs {
   double xl, yl, xh, yh, bx, by, sx, sy, ibx, iby;   // ibx = 1 / bx (no fp64 divisions on the hot path)
   double cx0, cy0;     // -xl / bx, -yl / by: bin coordinate of x is x * ibx + cx0
   float sxf, syf;      // stretched minimum sizes sqrt2 b (fp32)
+  float w_large, h_large;   // largest floats <= 2 b_x, 2 b_y: w > w_large <=> (double)w > 2 b_x (dp_create's test)
   int mx, my, tile, tile_log2, tiles_y, ntiles, stretch;
   int *tile_cnt, *tile_cursor, *tile_off;
   int *walk_tile;   // [walk_grid] first tile of each walker's slice (D2)
@@ -88,6 +90,33 @@ __device__ __forceinline__ Foot footprint(const DenArgs &a, int i) {
   return footprint_v(a, __ldg(a.x + a.cell_begin + i), __ldg(a.y + a.cell_begin + i), __ldg(a.w + i), __ldg(a.h + i));
 }
 
+// Small-cell classification shared by count (D1) and place (D3), which must agree exactly:
+// returns the tile of the footprint's first bin, -1 for an empty footprint, -2 for a large cell
+// (CTA-per-cell path).  Only the lower corner (lx, ly) and the upper corner (hx, hy) are formed
+// in fp64 (unclipped); the predicate equals footprint_v's "empty" (hi > lo after clipping to
+// [0, M], with w h > 0 in place of r > 0: r = 0 only when w h = 0) without fp64 min/max.
+struct SmallFoot {
+  double lx, ly, hx, hy;
+  float ws, hs;
+  int bi, bj;
+};
+
+__device__ __forceinline__ int classify_small(const DenArgs &a, float x, float y, float w, float h, SmallFoot &f) {
+  if (w > a.w_large || h > a.h_large) return -2;
+  f.ws = a.stretch ? fmaxf(w, a.sxf) : w;
+  f.hs = a.stretch ? fmaxf(h, a.syf) : h;
+  f.lx = fma((double)(0.5f * (w - f.ws)), a.ibx, fma((double)x, a.ibx, a.cx0));
+  f.ly = fma((double)(0.5f * (h - f.hs)), a.iby, fma((double)y, a.iby, a.cy0));
+  f.hx = fma((double)f.ws, a.ibx, f.lx);
+  f.hy = fma((double)f.hs, a.iby, f.ly);
+  const bool ok = f.hx > f.lx && f.hx > 0.0 && f.lx < (double)a.mx && f.hy > f.ly && f.hy > 0.0 &&
+                  f.ly < (double)a.my && w * h > 0.f;
+  if (!ok) return -1;
+  f.bi = max(0, min(__double2int_rz(f.lx), a.mx - 1));
+  f.bj = max(0, min(__double2int_rz(f.ly), a.my - 1));
+  return (f.bi >> a.tile_log2) * a.tiles_y + (f.bj >> a.tile_log2);
+}
+
 // first bin of a (non-empty) footprint and its tile
 __device__ __forceinline__ int small_tile(const DenArgs &a, const Foot &f, int &bx0, int &by0) {
   bx0 = min((int)f.lo_x, a.mx - 1);
@@ -123,14 +152,13 @@ __global__ void __launch_bounds__(kCountThreads) k_count(DenArgs a) {
   __syncthreads();
 #pragma unroll
   for (int k = 0; k < kCellsPerThread; k++) {
-    const Foot f = footprint_v(a, x[k], y[k], w[k], h[k]);
-    if (f.empty || f.large) continue;
-    int bx0, by0;
-    atomicAdd(&s_hist[small_tile(a, f, bx0, by0)], 1);
+    SmallFoot f;
+    const int t = classify_small(a, x[k], y[k], w[k], h[k], f);
+    if (t >= 0) atomicAdd(&s_hist[t], 1);
   }
   __syncthreads();
   for (int t = threadIdx.x; t < a.ntiles; t += kCountThreads)
-    if (s_hist[t]) atomicAdd(a.tile_cnt + t, s_hist[t]);
+    if (s_hist[t]) atomicAdd(a.tile_cnt + t * kCntStride, s_hist[t]);
 }
 
 // D2 (single CTA of 1024 threads): exclusive scan of the tile counts with warp shuffles (two
@@ -152,7 +180,7 @@ __global__ void __launch_bounds__(1024) k_scan(DenArgs a) {
   const int t0 = threadIdx.x * per;
   int cnt_sum = 0;
   for (int k = 0; k < per; k++)
-    if (t0 + k < a.ntiles) cnt_sum += a.tile_cnt[t0 + k];
+    if (t0 + k < a.ntiles) cnt_sum += a.tile_cnt[(t0 + k) * kCntStride];
   const int ia = warp_incl_scan(cnt_sum, lane);
   if (lane == 31) s_wa[warp] = ia;
   __syncthreads();
@@ -163,9 +191,9 @@ __global__ void __launch_bounds__(1024) k_scan(DenArgs a) {
   for (int k = 0; k < per; k++) {
     const int t = t0 + k;
     if (t < a.ntiles) {
-      const int c = a.tile_cnt[t];
+      const int c = a.tile_cnt[t * kCntStride];
       a.tile_off[t] = off_c;
-      a.tile_cursor[t] = off_c;
+      a.tile_cursor[t * kCntStride] = off_c;
       // walkers whose slice [N g / G, N (g + 1) / G) starts in this tile:
       // off <= floor(N g / G) < off + c  <=>  ceil(off G / N) <= g < ceil((off + c) G / N)
       if (c > 0) {
@@ -173,7 +201,7 @@ __global__ void __launch_bounds__(1024) k_scan(DenArgs a) {
         for (long long g = g0; g < g1; g++) a.walk_tile[g] = t;
       }
       off_c += c;
-      a.tile_cnt[t] = 0;  // ready for the next evaluation
+      a.tile_cnt[t * kCntStride] = 0;  // ready for the next evaluation
     }
   }
   if (threadIdx.x == T - 1) a.tile_off[a.ntiles] = off_c;
@@ -211,20 +239,23 @@ __global__ void __launch_bounds__(kCountThreads) k_place(DenArgs a) {
 #pragma unroll
   for (int k = 0; k < kCellsPerThread; k++) {
     const int i = i0 + k * kCountThreads + threadIdx.x;
-    const Foot f = footprint_v(a, x[k], y[k], w[k], h[k]);
+    SmallFoot f;
+    const int t = classify_small(a, x[k], y[k], w[k], h[k], f);
     tl[k] = -1;
-    if (i >= a.n_own || f.large) continue;
-    if (f.empty) {
+    if (i >= a.n_own || t == -2) continue;
+    if (t == -1) {
       a.force[i] = make_float2(0.f, 0.f);
       continue;
     }
-    int bi, bj;
-    tl[k] = small_tile(a, f, bi, bj);
-    rank[k] = atomicAdd(&s_hist[tl[k]], 1);
-    // bin-local fractions (|v| < 3): fp32 keeps ~2e-7 bin absolute precision, which the force
-    // gather needs where large opposite bin fields cancel (the 'initial' placement)
-    rec[k] = make_float4((float)(f.lo_x - bi), (float)(f.lo_y - bj), (float)(f.hi_x - bi), (float)(f.hi_y - bj));
-    rr[k] = f.r;
+    tl[k] = t;
+    rank[k] = atomicAdd(&s_hist[t], 1);
+    // bin-local fractions (|v| < 3) of the clipped footprint [max(l, 0), min(h, M)]: fp32 keeps
+    // ~2e-7 bin absolute precision, which the force gather needs where large opposite bin fields
+    // cancel (the 'initial' placement).  fl(max(l, 0) - b) = max(fl(l - b), -b) (monotone rounding)
+    const int bi = f.bi, bj = f.bj;
+    rec[k] = make_float4(fmaxf((float)(f.lx - bi), (float)-bi), fmaxf((float)(f.ly - bj), (float)-bj),
+                         fminf((float)(f.hx - bi), (float)(a.mx - bi)), fminf((float)(f.hy - bj), (float)(a.my - bj)));
+    rr[k] = __fdividef(w[k] * h[k], f.ws * f.hs);
     rcy[k] = (bi & mask) | ((bj & mask) << 16);
   }
   __syncthreads();
@@ -236,7 +267,7 @@ __global__ void __launch_bounds__(kCountThreads) k_place(DenArgs a) {
     const int t = t0 + q;
     if (t < a.ntiles) {
       const int cnt = s_hist[t];
-      if (cnt) s_base[t] = atomicAdd(a.tile_cursor + t, cnt);
+      if (cnt) s_base[t] = atomicAdd(a.tile_cursor + t * kCntStride, cnt);
       sum += cnt;
     }
   }
@@ -295,7 +326,8 @@ struct WalkChunk {
 struct RecStage {
   RecBuf buf[kStages];
   WalkChunk ch[kStages];
-  uint64_t bar[kStages];
+  uint64_t bar[kStages];     // full: descriptor + records landed (one arrival by the producer + tx bytes)
+  uint64_t empty[kStages];   // released: every warp has consumed the buffer (one arrival per warp)
   uint64_t bar_xi;
 };
 
@@ -320,40 +352,79 @@ __device__ __forceinline__ void walk_init(const DenArgs &a, Walker &w) {
   w.tend = a.tile_off[w.t + 1];
 }
 
-// (thread 0) next chunk of the slice -> descriptor slot b, copies issued on bar[b]
+// (thread 0) next chunk of the slice -> descriptor slot b, copies issued on bar[b].  The
+// descriptor is written before the arrival, so a consumer that sees the phase complete sees it;
+// an empty chunk (end of the slice) completes its phase with no bytes.
 __device__ __forceinline__ void walk_issue(const DenArgs &a, Walker &w, RecStage &st, int b, bool with_cell) {
   WalkChunk c;
   c.begin = c.end = w.cur;
   c.tile = w.t;
   c.off = 0;
+  int b0 = 0, n = 0;
   if (w.cur < w.re) {
     while (w.tend <= w.cur) w.tend = a.tile_off[++w.t + 1];   // skip finished / empty tiles
     c.tile = w.t;
     c.end = min(min(w.cur + kStageRecs, w.tend), w.re);
     w.cur = c.end;
-    const int b0 = c.begin & ~3, e0 = (c.end + 3) & ~3, n = e0 - b0;
+    b0 = c.begin & ~3;
+    n = ((c.end + 3) & ~3) - b0;
     c.off = c.begin - b0;
+  }
+  st.ch[b] = c;
+  mbar_expect_tx(&st.bar[b], (unsigned)n * (with_cell ? 28u : 24u));
+  if (n > 0) {
     RecBuf &B = st.buf[b];
-    mbar_expect_tx(&st.bar[b], (unsigned)n * (with_cell ? 28u : 24u));
     bulk_g2s(B.rec, a.rec + b0, 16u * n, &st.bar[b]);
     bulk_g2s(B.rc, a.rec_rc + b0, 8u * n, &st.bar[b]);
     if (with_cell) bulk_g2s(B.cell, a.rec_cell + b0, 4u * n, &st.bar[b]);
   }
-  st.ch[b] = c;
 }
 
 // (thread 0) barriers + the first kStages - 1 chunks; the caller synchronises
 __device__ __forceinline__ void walk_start(const DenArgs &a, Walker &w, RecStage &st, bool with_cell) {
   walk_init(a, w);
-  for (int b = 0; b < kStages; b++) mbar_init(&st.bar[b]);
+  for (int b = 0; b < kStages; b++) {
+    mbar_init(&st.bar[b]);
+    mbar_init_count(&st.empty[b], blockDim.x >> 5);
+  }
   mbar_init(&st.bar_xi);
   for (int b = 0; b < kStages - 1; b++) walk_issue(a, w, st, b, with_cell);
+}
+
+// Ring step of chunk c (every thread): wait until chunk c has landed; thread 0 then refills the
+// buffer of chunk c - 1 with chunk c + kStages - 1 once every warp has released chunk c - 1.
+// Warps move through the ring independently: there is no block barrier per chunk.
+__device__ __forceinline__ WalkChunk walk_next(const DenArgs &a, Walker &w, RecStage &st, int c, bool with_cell) {
+  const int b = c % kStages;
+  mbar_wait(&st.bar[b], (c / kStages) & 1);
+  const WalkChunk cc = st.ch[b];
+  if (threadIdx.x == 0 && cc.begin < cc.end) {
+    const int b2 = (c + kStages - 1) % kStages;
+    if (c >= 1) mbar_wait(&st.empty[b2], ((c - 1) / kStages) & 1);
+    walk_issue(a, w, st, b2, with_cell);
+  }
+  return cc;
+}
+
+// this warp is done with chunk c's buffer
+__device__ __forceinline__ void walk_release(RecStage &st, int c) {
+  __syncwarp();
+  if ((threadIdx.x & 31) == 0) mbar_arrive(&st.empty[c % kStages]);
 }
 
 // shared-memory reduction without a return value; unconditional (a zero add is cheaper than the
 // branch + reconvergence ptxas emits around a predicated shared atomic)
 __device__ __forceinline__ void red_shared(unsigned *p, unsigned v) {
   asm volatile("red.shared.add.u32 [%0], %1;" ::"r"(smem_u32(p)), "r"(v) : "memory");
+}
+
+// the same, issued only where `on` (a predicated instruction, no branch): lanes whose bin has no
+// overlap do not occupy the shared-atomic unit (~5 lane-ops / clk / SM, the scatter's bound)
+__device__ __forceinline__ void red_shared2_if(unsigned *p_hi, unsigned *p_lo, unsigned hi, unsigned lo, unsigned on) {
+  asm volatile(
+      "{\n .reg .pred p;\n setp.ne.u32 p, %4, 0;\n @p red.shared.add.u32 [%0], %2;\n @p red.shared.add.u32 [%1], %3;\n}"
+      ::"r"(smem_u32(p_hi)), "r"(smem_u32(p_lo)), "r"(hi), "r"(lo), "r"(on)
+      : "memory");
 }
 
 // overlaps (bin units) of a record's footprint with the 3 bins from its first bin, per axis;
@@ -401,21 +472,21 @@ __global__ void __launch_bounds__(kTileThreads) k_scatter_walk(DenArgs a) {
   }
   __syncthreads();
   const float scale_fx = (float)(1u << kRhoScaleLog2);
-  int cur_tile = st.ch[0].tile, acc = 0;
+  int cur_tile = -1, acc = 0;
   for (int c = 0;; c++) {
     const int b = c % kStages;
-    const WalkChunk cc = st.ch[b];
+    const WalkChunk cc = walk_next(a, w, st, c, false);
     if (cc.begin >= cc.end) break;
-    if (threadIdx.x == 0) walk_issue(a, w, st, (c + kStages - 1) % kStages, false);   // freed by the last sync
     const int n = cc.end - cc.begin;
-    if (cc.tile != cur_tile || acc + n > kFlushRecs) {
+    if (cur_tile < 0) cur_tile = cc.tile;
+    if (cc.tile != cur_tile || acc + n > kFlushRecs) {   // uniform: every warp sees the same chunks
+      __syncthreads();   // the tile is complete
       flush_tile(a, s_hi, s_lo, cur_tile);
-      __syncthreads();
+      __syncthreads();   // flushed and cleared
       cur_tile = cc.tile;
       acc = 0;
     }
     acc += n;
-    mbar_wait(&st.bar[b], (c / kStages) & 1);
     const RecBuf &B = st.buf[b];
     for (int k = threadIdx.x; k < n; k += blockDim.x) {
       const float4 q = B.rec[cc.off + k];
@@ -435,14 +506,14 @@ __global__ void __launch_bounds__(kTileThreads) k_scatter_walk(DenArgs a) {
           const unsigned u = (unsigned)(rx * oy3[dj]);
           const unsigned hi = u >> kTileLoBits, lo = u & ((1u << kTileLoBits) - 1u);
           const int k2 = base + di * P + dj;
-          red_shared(s_hi + k2, hi);
-          red_shared(s_lo + k2, lo);
+          red_shared2_if(s_hi + k2, s_lo + k2, hi, lo, u);
         }
       }
     }
-    __syncthreads();   // buffer b consumed before it is refilled; tile complete before a flush
+    walk_release(st, c);
   }
-  flush_tile(a, s_hi, s_lo, cur_tile);
+  __syncthreads();
+  if (cur_tile >= 0) flush_tile(a, s_hi, s_lo, cur_tile);
 }
 
 // D5: persistent gather walker; the (tile+2)^2 float2 field tile is (re)loaded with one bulk copy
@@ -479,15 +550,13 @@ __global__ void __launch_bounds__(kTileThreads) k_gather_walk(DenArgs a) {
   const float area = (float)(a.bx * a.by);
   for (int c = 0;; c++) {
     const int b = c % kStages;
-    const WalkChunk cc = st.ch[b];
+    const WalkChunk cc = walk_next(a, w, st, c, true);
     if (cc.begin >= cc.end) break;
-    if (threadIdx.x == 0) walk_issue(a, w, st, (c + kStages - 1) % kStages, true);
-    if (cc.tile != cur_tile) {   // the previous iteration's sync freed the field tile
+    if (cc.tile != cur_tile) {   // uniform; load_xi_tile's barrier waits until every warp left the old tile
       load_xi_tile(a, st, s_xi, cc.tile, xi_phase);
       xi_phase ^= 1u;
       cur_tile = cc.tile;
     }
-    mbar_wait(&st.bar[b], (c / kStages) & 1);
     const RecBuf &B = st.buf[b];
     const int n = cc.end - cc.begin;
     for (int k = threadIdx.x; k < n; k += blockDim.x) {
@@ -515,7 +584,7 @@ __global__ void __launch_bounds__(kTileThreads) k_gather_walk(DenArgs a) {
       // dD/dx = - r sum_b ov(i,b) xi^X_b  (reading A21), ov in length^2
       a.force[B.cell[cc.off + k]] = make_float2(-area * r * fx, -area * r * fy);
     }
-    __syncthreads();
+    walk_release(st, c);
   }
 }
 
@@ -578,6 +647,13 @@ __global__ void __launch_bounds__(256) k_gather_large(DenArgs a) {
   }
 }
 
+// largest float f with (double)f <= v, so that for any float w: w > f <=> (double)w > v
+float float_at_most(double v) {
+  float f = (float)v;
+  if ((double)f > v) f = std::nextafter(f, -INFINITY);
+  return f;
+}
+
 DenArgs make_args(const Ctx &c, const float *x, const float *y) {
   DenArgs a;
   a.x = x;
@@ -595,6 +671,8 @@ DenArgs make_args(const Ctx &c, const float *x, const float *y) {
   a.cy0 = -c.yl * a.iby;
   a.sxf = (float)a.sx;
   a.syf = (float)a.sy;
+  a.w_large = float_at_most(2.0 * c.bx);
+  a.h_large = float_at_most(2.0 * c.by);
   a.mx = c.mx; a.my = c.my; a.tile = c.tile; a.tiles_y = c.tiles_y;
   a.tile_log2 = 0;
   while ((1 << a.tile_log2) < c.tile) a.tile_log2++;

@@ -422,9 +422,9 @@ dp_status build_density(Ctx &c, const dp_netlist *nl) {
   if ((st = dev_upload(c, &c.d_cell_w, w)) != DP_OK) return st;
   if ((st = dev_upload(c, &c.d_cell_h, h)) != DP_OK) return st;
   if ((st = dev_upload(c, &c.d_large, large)) != DP_OK) return st;
-  if ((st = dev_alloc(c, &c.d_tile_cnt, ntiles)) != DP_OK) return st;
-  DP_CUDA(cudaMemset(c.d_tile_cnt, 0, sizeof(int32_t) * ntiles));
-  if ((st = dev_alloc(c, &c.d_tile_cursor, ntiles)) != DP_OK) return st;
+  if ((st = dev_alloc(c, &c.d_tile_cnt, (size_t)ntiles * kCntStride)) != DP_OK) return st;
+  DP_CUDA(cudaMemset(c.d_tile_cnt, 0, sizeof(int32_t) * ntiles * kCntStride));
+  if ((st = dev_alloc(c, &c.d_tile_cursor, (size_t)ntiles * kCntStride)) != DP_OK) return st;
   if ((st = dev_alloc(c, &c.d_tile_off, ntiles + 1)) != DP_OK) return st;
   // sort records; padded by 8 so staged copies may round their range to 4-record multiples
   if ((st = dev_alloc(c, &c.d_rec, c.n_own + 8)) != DP_OK) return st;
@@ -467,6 +467,11 @@ dp_status build_density(Ctx &c, const dp_netlist *nl) {
   }
   c.walk_grid = density_walk_grid(c.tile);
   if (c.walk_grid <= 0) return fail(DP_ERR_CUDA, "density walker occupancy query failed");
+  {  // DP_WALK_MULT = k: k slices per resident walker slot (finer slices start as SMs free up)
+    const char *e = std::getenv("DP_WALK_MULT");
+    const int k = e ? std::max(1, std::atoi(e)) : 1;
+    c.walk_grid *= k;
+  }
   if ((st = dev_alloc(c, &c.d_walk_tile, c.walk_grid)) != DP_OK) return st;
   DP_CUDA(cudaMemset(c.d_walk_tile, 0, sizeof(int32_t) * c.walk_grid));
   return DP_OK;
@@ -561,6 +566,11 @@ dp_status create(const dp_netlist *nl, const dp_grid *grid, int device, int rank
   int prio_lo = 0, prio_hi = 0;
   cudaDeviceGetStreamPriorityRange(&prio_lo, &prio_hi);
   { const char *e = std::getenv("DP_PRIO"); if (e && e[0] == '0') prio_hi = prio_lo; }   // default: density first
+  { const char *e = std::getenv("DP_FUSED_T2"); c->fused_t2 = e && e[0] == '1'; }
+  { const char *e = std::getenv("DP_WA_CTAS_PER_SM"); c->wa_ctas_per_sm = e ? std::atoi(e) : 0; }
+  { const char *e = std::getenv("DP_L2_HINT"); c->l2_hint = !(e && e[0] == '0'); }
+  { const char *e = std::getenv("DP_ROW_TMA"); c->row_tma = !(e && e[0] == '0'); }
+  { const char *e = std::getenv("DP_T1_TMA"); c->t1_tma = e && e[0] == '1'; }
   { const char *e = std::getenv("DP_GRAPH"); c->use_graph = !(e && e[0] == '0'); }
   if (cudaStreamCreateWithFlags(&c->s_cap, cudaStreamNonBlocking) != cudaSuccess ||
       cudaStreamCreateWithPriority(&c->s_wa, cudaStreamNonBlocking, prio_lo) != cudaSuccess ||

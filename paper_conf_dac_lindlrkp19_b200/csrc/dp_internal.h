@@ -38,6 +38,9 @@ constexpr int kFlushRecs = 8192;      // a walker flushes its shared tile at lea
 constexpr int kTileHiBits = 10;
 constexpr int kTileLoBits = 19;
 constexpr int kRhoScaleLog2 = kTileHiBits + kTileLoBits;   // global bin map: int64 units of 2^-29
+// per-tile counters / cursors one 128-byte line apart: every CTA of count / place adds to every
+// tile's counter, and counters sharing a line serialise in one L2 slice
+constexpr int kCntStride = 32;
 constexpr int kCountThreads = 256;
 constexpr int kCountCells = 2048;     // cells per count/place CTA (staged in shared memory)
 
@@ -122,8 +125,8 @@ struct Ctx {
   int32_t n_large = 0;              // large cells (footprint > 3 bins on an axis)
   int32_t *d_large = nullptr;       // ids of large own cells
   uint8_t *d_is_large = nullptr;    // per own cell
-  int32_t *d_tile_cnt = nullptr;      // [tiles] small-cell counts (reset by the scan)
-  int32_t *d_tile_cursor = nullptr;   // [tiles] placement cursors
+  int32_t *d_tile_cnt = nullptr;      // [tiles * kCntStride] small-cell counts (reset by the scan)
+  int32_t *d_tile_cursor = nullptr;   // [tiles * kCntStride] placement cursors
   int32_t *d_tile_off = nullptr;      // [tiles + 1]
   float4 *d_rec = nullptr;            // per slot: footprint box in tile-local bin units
   int2 *d_rec_rc = nullptr;           // per slot: (charge ratio r as float bits, i0 | j0 << 16)
@@ -143,6 +146,11 @@ struct Ctx {
   float2 *d_tw_x = nullptr, *d_tw_y = nullptr;     // FFT twiddles W_N^k, k < N/2
   float2 *d_ph_x = nullptr, *d_ph_y = nullptr;     // e^{-i pi k / 2N}, k < N
   float2 *d_spec = nullptr;                         // T2a -> T2b (A_X, A_Y) transposed [y][x]
+  int wa_ctas_per_sm = 0;                           // DP_WA_CTAS_PER_SM: residency cap of the WA kernel (0 = none)
+  bool l2_hint = true;                              // DP_L2_HINT=0: no evict-first policy on the WA pin stream (A/B)
+  bool row_tma = true;                              // DP_ROW_TMA=0: per-lane loads in the row-inverse passes (A/B)
+  bool t1_tma = false;                              // DP_T1_TMA=1: bulk-copied rows in the forward row pass (A/B; not faster inside the overlapped step)
+  bool fused_t2 = false;                            // DP_FUSED_T2=1: one column kernel (T2) instead of T2a + T2b (A/B)
   float2 *d_sxy = nullptr;                          // T2 -> T3 interleaved (sX, sY) [x][y] (warp-FFT path)
   float2 *d_tw2_x = nullptr, *d_tw2_y = nullptr;   // warp FFT: W_N^{n1 k2} at [k2 * 32 + n1] (N <= 1024)
   float *d_kx = nullptr, *d_ky = nullptr;          // wavenumbers (reading A12)

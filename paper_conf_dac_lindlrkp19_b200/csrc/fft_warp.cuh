@@ -65,11 +65,21 @@ __device__ __forceinline__ void reg_dft(float2 *a) {
   }
 }
 
-// Warp FFT of B = 1024 / N sequences.  In: a[s K + j] = x_s[lane + 32 j].  tw2[k2 * 32 + n1] =
-// W_N^{n1 k2} (fp64-rounded table).  Out: buf[pad(s N + k)] = X_s[k] (unnormalised; INV uses
+// Per-lane twiddles of pass 1, loaded up front so their latency overlaps the data loads:
+// tw[k2] = W_N^{lane k2} for k2 in [1, K) (tw[0] unused).
+template <int LOGN>
+__device__ __forceinline__ void load_twiddles(float2 (&tw)[32], const float2 *__restrict__ tw2) {
+  constexpr int K = (1 << LOGN) / 32;
+  const int lane = threadIdx.x & 31;
+#pragma unroll
+  for (int k2 = 1; k2 < K; k2++) tw[k2] = __ldg(tw2 + k2 * 32 + lane);
+}
+
+// Warp FFT of B = 1024 / N sequences.  In: a[s K + j] = x_s[lane + 32 j].  tw = this lane's
+// twiddles from load_twiddles (tw2[k2 * 32 + n1] = W_N^{n1 k2}, an fp64-rounded table).  Out: buf[pad(s N + k)] = X_s[k] (unnormalised; INV uses
 // conjugate twiddles).  buf is this warp's kBufPad-entry shared buffer; a[] is clobbered.
 template <int LOGN, bool INV>
-__device__ __forceinline__ void warp_fft(float2 (&a)[32], float2 *buf, const float2 *__restrict__ tw2) {
+__device__ __forceinline__ void warp_fft(float2 (&a)[32], float2 *buf, const float2 (&tw)[32]) {
   constexpr int N = 1 << LOGN, K = N / 32, B = kPts / N, LK = LOGN - 5;
   static_assert(K >= 1 && K <= 32, "warp_fft: N in [32, 1024]");
   const int lane = threadIdx.x & 31;
@@ -82,7 +92,7 @@ __device__ __forceinline__ void warp_fft(float2 (&a)[32], float2 *buf, const flo
       const int k2 = brev_c(m, LK);
       float2 v = a[s * K + m];
       if (k2 != 0) {
-        float2 w = __ldg(tw2 + k2 * 32 + lane);
+        float2 w = tw[k2];
         if (INV) w.y = -w.y;
         v = make_float2(v.x * w.x - v.y * w.y, v.x * w.y + v.y * w.x);
       }

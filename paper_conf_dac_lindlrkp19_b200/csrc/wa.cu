@@ -36,6 +36,8 @@ namespace {
 constexpr float kLog2e = 1.4426950408889634f;
 constexpr float kLn2 = 0.6931471805599453f;
 
+constexpr int kWaSmemOptIn = 227 * 1024 - 8192;   // dynamic opt-in, leaving room for the static shared arrays
+
 struct WaArgs {
   const Chunk *chunks;
   const WarpGroup *wgs;
@@ -50,6 +52,7 @@ struct WaArgs {
   double *part;                 // WA partial per CTA
   unsigned long long *limbs;    // HPWL limbs
   int has_w;
+  int stream_hint;              // evict-first L2 policy on the staged netlist data (DP_L2_HINT=0: off)
   // big nets
   const int32_t *big_start, *big_flags, *big_cell;
   const float *big_w, *big_dx, *big_dy;
@@ -791,17 +794,25 @@ __global__ void __launch_bounds__(kWaThreads, 3) k_wa_chunks(WaArgs a) {
     const unsigned tx = 12u * ch.pin_n + (a.has_w ? 8u : 4u) * ch.net_n + 16u * ch.wg_n + 4u * ch.far_pad +
                         (win_bulk ? 8u * wbulk : 0u);
     mbar_expect_tx(bar, tx);
+    // the chunk's netlist data is read once per evaluation: streamed with an evict-first L2 policy
+    const uint64_t pol = a.stream_hint ? l2_evict_first_policy() : 0;
+    auto copy = [&](void *dst, const void *src, unsigned bytes) {
+      if (a.stream_hint)
+        bulk_g2s_hint(dst, src, bytes, bar, pol);
+      else
+        bulk_g2s(dst, src, bytes, bar);
+    };
     if (ch.pin_n) {
-      bulk_g2s(s_slot, a.pin_slot + ch.pin_begin, 4u * ch.pin_n, bar);
-      bulk_g2s(s_dx, a.pin_dx + ch.pin_begin, 4u * ch.pin_n, bar);
-      bulk_g2s(s_dy, a.pin_dy + ch.pin_begin, 4u * ch.pin_n, bar);
+      copy(s_slot, a.pin_slot + ch.pin_begin, 4u * ch.pin_n);
+      copy(s_dx, a.pin_dx + ch.pin_begin, 4u * ch.pin_n);
+      copy(s_dy, a.pin_dy + ch.pin_begin, 4u * ch.pin_n);
     }
     if (ch.net_n) {
-      bulk_g2s(s_deg, a.net_deg + ch.net_begin, 4u * ch.net_n, bar);
-      if (a.has_w) bulk_g2s(s_w, a.net_w + ch.net_begin, 4u * ch.net_n, bar);
+      copy(s_deg, a.net_deg + ch.net_begin, 4u * ch.net_n);
+      if (a.has_w) copy(s_w, a.net_w + ch.net_begin, 4u * ch.net_n);
     }
-    if (ch.wg_n) bulk_g2s(s_wg, a.wgs + ch.wg_begin, 16u * ch.wg_n, bar);
-    if (ch.far_pad) bulk_g2s(s_far, a.far_cells + ch.far_begin, 4u * ch.far_pad, bar);
+    if (ch.wg_n) copy(s_wg, a.wgs + ch.wg_begin, 16u * ch.wg_n);
+    if (ch.far_pad) copy(s_far, a.far_cells + ch.far_begin, 4u * ch.far_pad);
     if (win_bulk) {
       bulk_g2s(s_px, a.x + ch.win_lo, 4u * wbulk, bar);
       bulk_g2s(s_py, a.y + ch.win_lo, 4u * wbulk, bar);
@@ -893,7 +904,12 @@ template <int MODE>
 void launch_mode(const Ctx &c, const WaArgs &a, cudaStream_t s) {
   const WaSmem L{a.caps};
   const int grid = c.n_chunks + a.n_huge + a.n_warp_blocks;
-  if (grid > 0) k_wa_chunks<MODE><<<grid, kWaThreads, L.bytes(), s>>>(a);
+  int bytes = L.bytes();
+  // DP_WA_CTAS_PER_SM = k (measurement knob): pad the dynamic shared memory so that at most k
+  // WA CTAs are resident per SM, leaving room for the concurrently running density kernels
+  if (c.wa_ctas_per_sm > 0)
+    bytes = std::max(bytes, std::min(kWaSmemOptIn, ((228 * 1024) / c.wa_ctas_per_sm - 4096) & ~127));
+  if (grid > 0) k_wa_chunks<MODE><<<grid, kWaThreads, bytes, s>>>(a);
 }
 
 }  // namespace
@@ -901,7 +917,7 @@ void launch_mode(const Ctx &c, const WaArgs &a, cudaStream_t s) {
 int wa_smem_bytes(const WaCaps &caps) { return WaSmem{caps}.bytes(); }
 
 cudaError_t wa_configure(const WaCaps &caps) {
-  const int b = WaSmem{caps}.bytes();
+  const int b = std::max(WaSmem{caps}.bytes(), kWaSmemOptIn);   // launches may pad (DP_WA_CTAS_PER_SM)
   cudaError_t e = cudaFuncSetAttribute(k_wa_chunks<0>, cudaFuncAttributeMaxDynamicSharedMemorySize, b);
   if (e != cudaSuccess) return e;
   e = cudaFuncSetAttribute(k_wa_chunks<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, b);
@@ -929,6 +945,7 @@ void launch_wa(const Ctx &c, const float *x, const float *y, float gamma, bool h
   a.part = c.d_part;
   a.limbs = c.d_limbs;
   a.has_w = c.has_weights ? 1 : 0;
+  a.stream_hint = c.l2_hint ? 1 : 0;
   a.big_start = c.d_big_start;
   a.big_flags = c.d_big_flags;
   a.big_cell = c.d_big_cell;

@@ -18,7 +18,7 @@ def main(path, kregex, top=25):
     for r in rows[hi + 1:]:
         try:
             n, w = float(r[ii] or 0), float(r[wi] or 0)
-        except ValueError:
+        except (ValueError, IndexError):
             continue
         src = r[si].strip()
         op = re.sub(r'^@!?U?P\w+\s+', '', src).split(' ')[0]

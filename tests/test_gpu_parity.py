@@ -298,3 +298,88 @@ def test_density_bitwise_deterministic(tiny, dist):
     assert a["energy"].item() == b["energy"].item()
     assert torch.equal(a["gx"], b["gx"]) and torch.equal(a["gy"], b["gy"])
     assert torch.equal(ctx.density_map(_t(x), _t(y)), ctx.density_map(_t(x), _t(y)))
+
+
+@pytest.mark.parametrize("world", [2, 3])
+def test_virtual_shards_reassemble(world):
+    """dp_create_dist with no NCCL id (collectives skipped) on one GPU, one context per rank: the
+    owner-computes partition must reassemble the single-context results — WA and
+    its gradient (own cells per rank, every net counted once), HPWL, and the int64 bin map of
+    each rank's own cells summing to the full map."""
+    nl = make_netlist("tiny")
+    x, y = make_positions(nl)
+    gamma = nl.bin_w
+    full = dp.dp_create(nl)
+    ref = full.wl_grad(_t(x), _t(y), gamma)
+    ref_map = full.density_map(_t(x), _t(y)).double()
+    wl = 0.0
+    hp = 0.0
+    gx = torch.zeros(nl.num_cells, dtype=torch.float64, device=DEV)
+    gy = torch.zeros_like(gx)
+    rho = torch.zeros_like(ref_map)
+    covered = np.zeros(nl.num_cells, np.int64)
+    for r in range(world):
+        cb, ce, _ = dp.dp_partition_plan(nl, r, world)
+        covered[cb:ce] += 1
+        ctx = dp.dp_create_dist(nl, 0, r, world, None)
+        out = ctx.wl_grad(_t(x), _t(y), gamma)
+        wl += out["wl"].item()
+        gx[cb:ce] += out["gx"][cb:ce].double()
+        gy[cb:ce] += out["gy"][cb:ce].double()
+        hp += ctx.hpwl(_t(x), _t(y)).item()
+        rho += ctx.density_map(_t(x), _t(y)).double()
+    assert (covered == 1).all()
+    check_scalar("WA", wl, ref["wl"].item(), rel=1e-6)
+    # shards chunk their nets differently (fixed-point scales, fp32 flush order): the oracle's bar
+    check_vector("dWA/dx", to_np(gx), to_np(ref["gx"]))
+    check_vector("dWA/dy", to_np(gy), to_np(ref["gy"]))
+    assert hp == pytest.approx(oracle.hpwl(nl, x, y), rel=1e-14)
+    check_map("rho", to_np(rho), to_np(ref_map), rel=1e-6)
+
+
+@pytest.mark.slow
+@pytest.mark.parametrize("bins", [256, 2048, 4096])
+def test_bin_sweep_density(bins):
+    """BASELINE configs[4] (bin-resolution sweep): the bigblue4 netlist on 256^2..4096^2 maps —
+    the shared-memory transform path above 1024 — density energy and gradient vs the oracle."""
+    nl = make_netlist("bigblue4", bins=bins)
+    x, y = make_positions(nl)
+    ctx = dp.dp_create(nl)
+    out = ctx.density_grad(_t(x), _t(y))
+    D, fx, fy, _ = oracle.density(nl, x, y, 1)
+    check_scalar("D", out["energy"].item(), D)
+    check_vector("dD/dx", to_np(out["gx"]), fx)
+    check_vector("dD/dy", to_np(out["gy"]), fy)
+
+
+@pytest.mark.slow
+def test_high_fanout_sweep():
+    """BASELINE configs[4] (high-fanout sweep): bigblue4 with extra nets of 1K, 2K, 5K and 10K
+    pins — WA, its gradient and HPWL vs the oracle."""
+    nl = make_netlist("bigblue4", extra_fanout=(1000, 2000, 5000, 10000))
+    x, y = make_positions(nl)
+    ctx = dp.dp_create(nl)
+    gamma = nl.bin_w
+    out = ctx.wl_grad(_t(x), _t(y), gamma)
+    wl, gx, gy = oracle.wa(nl, x, y, gamma)
+    check_scalar("WA", out["wl"].item(), wl)
+    check_vector("dWA/dx", to_np(out["gx"]), gx)
+    check_vector("dWA/dy", to_np(out["gy"]), gy)
+    assert ctx.hpwl(_t(x), _t(y)).item() == oracle.hpwl(nl, x, y)
+
+
+@pytest.mark.slow
+def test_eval_industrial():
+    """BASELINE configs[3] shape on one GPU (10M cells, 10.23M nets, 40.9M pins, 2048^2 bins): the
+    full evaluation vs the oracle."""
+    nl = make_netlist("industrial")
+    x, y = make_positions(nl)
+    ctx = dp.dp_create(nl)
+    gamma = nl.bin_w
+    out = ctx.eval(_t(x), _t(y), gamma, 1.0, with_hpwl=True)
+    ref = oracle.evaluate(nl, x, y, gamma, 1.0)
+    check_scalar("WA", out["wl"].item(), ref["wl"])
+    check_scalar("D", out["energy"].item(), ref["energy"])
+    assert out["hpwl"].item() == ref["hpwl"]
+    check_vector("gx", to_np(out["gx"]), ref["gx"])
+    check_vector("gy", to_np(out["gy"]), ref["gy"])

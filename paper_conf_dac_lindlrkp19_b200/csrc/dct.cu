@@ -203,6 +203,7 @@ __global__ void __launch_bounds__(kRowThreads) k_row_inv(RowInvArgs a) {
 // or rows (T3) and never waits on a block barrier.
 // ---------------------------------------------------------------------------------------
 constexpr int kWRowWarps = 2;   // warps per CTA: a 1024-row map gives 256-512 CTAs
+constexpr int kTStoreWarps = 4; // T2b (transposed output): 4 adjacent columns -> 32-byte row segments
 
 // 1/x to ~1 ulp on the MUFU (the IEEE __frcp_rn slow path stalled the column pass)
 __device__ __forceinline__ float fast_rcp(float x) {
@@ -292,20 +293,23 @@ __global__ void __launch_bounds__(32 * kWRowWarps) k_row_dct_w(const IN *__restr
 }
 
 // T3 / debug: row r of A (op opA) and row r of B (op opB) as one complex inverse sequence
-template <int LOGN>
-__global__ void __launch_bounds__(32 * kWRowWarps) k_row_inv_w(RowInvArgs a, const float2 *__restrict__ tw2, int rows) {
+// TSTORE (T2b, transposed output outI[t * ostepT + r]): the CTA's WARPS * B consecutive rows r
+// are written together after a block barrier, WARPS * B adjacent float2 per output row (full
+// 32-byte sectors at WARPS = 4), instead of one 8-byte store per lane and row.
+template <int LOGN, int WARPS = kWRowWarps, bool TSTORE = false>
+__global__ void __launch_bounds__(32 * WARPS) k_row_inv_w(RowInvArgs a, const float2 *__restrict__ tw2, int rows) {
   constexpr int N = 1 << LOGN, K = N / 32, B = wfft::kPts / N;
   extern __shared__ float2 wsm[];
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   float2 *buf = wsm + warp * wfft::kBufPad;
-  const int r0 = (blockIdx.x * kWRowWarps + warp) * B;
-  if (r0 >= rows) return;
+  const int r0 = (blockIdx.x * WARPS + warp) * B;
+  if (!TSTORE && r0 >= rows) return;   // TSTORE: idle warps still reach the block barrier
   // interleaved input: the warp's B rows (contiguous) land in its buffer by one bulk copy;
   // planar input (debug transforms): per-lane loads, staged through the buffer.  Either way each
   // row is read once and the mirrored element N - k comes from the buffer.
-  __shared__ uint64_t s_bar[kWRowWarps];
-  const int nvalid = min(B, rows - r0);
-  if (a.inI && a.tma && lane == 0) {
+  __shared__ uint64_t s_bar[WARPS];
+  const int nvalid = max(0, min(B, rows - r0));
+  if (a.inI && a.tma && lane == 0 && nvalid > 0) {
     mbar_init(&s_bar[warp]);
     const unsigned bytes = (unsigned)(N * nvalid * sizeof(float2));
     mbar_expect_tx(&s_bar[warp], bytes);
@@ -318,7 +322,7 @@ __global__ void __launch_bounds__(32 * kWRowWarps) k_row_inv_w(RowInvArgs a, con
   float2 v[32];
   if (a.inI && a.tma) {
     __syncwarp();
-    mbar_wait(&s_bar[warp], 0);
+    if (nvalid > 0) mbar_wait(&s_bar[warp], 0);
 #pragma unroll
     for (int s = 0; s < B; s++)
 #pragma unroll
@@ -356,6 +360,23 @@ __global__ void __launch_bounds__(32 * kWRowWarps) k_row_inv_w(RowInvArgs a, con
   }
   __syncwarp();
   wfft::warp_fft<LOGN, true>(v, buf, twr);
+  if constexpr (TSTORE) {
+    constexpr int C = WARPS * B;   // consecutive output columns of this CTA
+    const int rc0 = blockIdx.x * C;
+    __syncthreads();
+    for (int idx = threadIdx.x; idx < N * C; idx += 32 * WARPS) {
+      const int c = idx % C, t = idx / C, r = rc0 + c;
+      if (r >= rows) continue;
+      const float2 z = wsm[(c / B) * wfft::kBufPad + wfft::pad((c % B) * N + mk_pos(t, N))];
+      float va = 0.5f * z.x, vb = 0.5f * z.y;
+      if (t & 1) {
+        if (a.opA == 2) va = -va;
+        if (a.opB == 2) vb = -vb;
+      }
+      a.outI[(size_t)t * a.ostepT + r] = make_float2(va, vb);
+    }
+    return;
+  }
 #pragma unroll
   for (int s = 0; s < B; s++) {
     const int r = r0 + s;
@@ -741,6 +762,21 @@ void row_inv(const Ctx &c, const float *inA, long long stepA, int opA, const flo
   a.ph = x_axis ? c.d_ph_x : c.d_ph_y;
   if (!warp_fft_ok(log2n)) {
     k_row_inv<<<rows, kRowThreads, row_smem(a.n), s>>>(a);
+    return;
+  }
+  if (ostepT > 0 && inI) {   // T2b: 4-warp CTAs, coalesced transposed stores
+    constexpr int W = kTStoreWarps;
+    const int per_cta = (wfft::kPts >> log2n) * W;
+    const int g = (rows + per_cta - 1) / per_cta;
+    const size_t sm = (size_t)W * wfft::kBufPad * sizeof(float2);
+    switch (log2n) {
+      case 5: k_row_inv_w<5, W, true><<<g, 32 * W, sm, s>>>(a, tw2, rows); break;
+      case 6: k_row_inv_w<6, W, true><<<g, 32 * W, sm, s>>>(a, tw2, rows); break;
+      case 7: k_row_inv_w<7, W, true><<<g, 32 * W, sm, s>>>(a, tw2, rows); break;
+      case 8: k_row_inv_w<8, W, true><<<g, 32 * W, sm, s>>>(a, tw2, rows); break;
+      case 9: k_row_inv_w<9, W, true><<<g, 32 * W, sm, s>>>(a, tw2, rows); break;
+      default: k_row_inv_w<10, W, true><<<g, 32 * W, sm, s>>>(a, tw2, rows); break;
+    }
     return;
   }
   const int g = wrow_ctas(rows, log2n);

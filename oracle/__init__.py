@@ -53,6 +53,8 @@ def lib():
         I64, I32, D = ctypes.c_int64, ctypes.c_int, ctypes.c_double
         L.or_wa.restype = D
         L.or_wa.argtypes = [I64, P, P, P, P, P, P, P, D, P, P, P]
+        L.or_lse.restype = D
+        L.or_lse.argtypes = [I64, P, P, P, P, P, P, P, D, P, P, P]
         L.or_hpwl_nets.restype = None
         L.or_hpwl_nets.argtypes = [I64, P, P, P, P, P, P, P]
         L.or_density_map.restype = None
@@ -93,6 +95,22 @@ def wa(nl, x, y, gamma: float, per_net: bool = False):
     tot = lib().or_wa(nl.num_nets, _p(ns), _p(p2c), _p(dx), _p(dy),
                       None if w is None else _p(w), _p(xx), _p(yy), float(gamma),
                       _p(gx), _p(gy), None if wl_net is None else _p(wl_net))
+    return (tot, gx, gy, wl_net) if per_net else (tot, gx, gy)
+
+
+def lse(nl, x, y, gamma: float, per_net: bool = False):
+    """LSE wirelength sum_e w_e (LSE_e^x + LSE_e^y) (NEXT-3, reading A27: the
+    definition of [29] with the P:159 shift) and its cell gradient.  Same returns as wa()."""
+    ns, p2c = _i32(nl.net_start), _i32(nl.pin2cell)
+    dx, dy = _f64(nl.pin_dx), _f64(nl.pin_dy)
+    xx, yy = _f64(x), _f64(y)
+    w = None if nl.net_weight is None else _f64(nl.net_weight)
+    gx = np.zeros(nl.num_cells)
+    gy = np.zeros(nl.num_cells)
+    wl_net = np.zeros(nl.num_nets) if per_net else None
+    tot = lib().or_lse(nl.num_nets, _p(ns), _p(p2c), _p(dx), _p(dy),
+                       None if w is None else _p(w), _p(xx), _p(yy), float(gamma),
+                       _p(gx), _p(gy), None if wl_net is None else _p(wl_net))
     return (tot, gx, gy, wl_net) if per_net else (tot, gx, gy)
 
 
@@ -193,9 +211,11 @@ def density(nl, x, y, stretch: int = 1):
     return D, gx, gy, dict(rho=rho, a=a, psi=psi, xi_x=xi_x, xi_y=xi_y)
 
 
-def evaluate(nl, x, y, gamma: float, lam: float, stretch: int = 1, with_hpwl: bool = True):
-    """obj = WA + lambda D and grad = grad WA + lambda grad D (eq 2)."""
-    wl, gwx, gwy = wa(nl, x, y, gamma)
+def evaluate(nl, x, y, gamma: float, lam: float, stretch: int = 1, with_hpwl: bool = True,
+             wl_model: str = "wa"):
+    """obj = WL + lambda D and grad = grad WL + lambda grad D (eq 2); WL = WA (eq 3)
+    or LSE (reading A27)."""
+    wl, gwx, gwy = (lse if wl_model == "lse" else wa)(nl, x, y, gamma)
     D, gdx, gdy, parts = density(nl, x, y, stretch)
     out = dict(obj=wl + lam * D, wl=wl, energy=D, gx=gwx + lam * gdx, gy=gwy + lam * gdy,
                wl_gx=gwx, wl_gy=gwy, d_gx=gdx, d_gy=gdy, **parts)

@@ -110,6 +110,77 @@ double or_wa(int64_t num_nets, const int32_t *net_start, const int32_t *pin2cell
     return total;
 }
 
+/* ------------------------------------------------------------------------------------
+ * Log-sum-exp wirelength, one axis of one net (NEXT-3; "log-sum-exp (LSE) [29], which is
+ * also implemented in the framework").  The paper prints no LSE formula; reading A27
+ * takes the standard definition of [29] (Naylor et al.):
+ *   LSE_e = gamma ln sum_i exp(x_i/gamma) + gamma ln sum_i exp(-x_i/gamma)
+ * evaluated with the same overflow-safe shift as WA and Table I's a_i^+-, b_e^+-:
+ *   LSE_e = (x_e^+ + gamma ln b_e^+) - (x_e^- - gamma ln b_e^-)
+ *   dLSE_e/dx_i = a_i^+/b_e^+ - a_i^-/b_e^-
+ * Nets of degree 0 or 1 contribute 0 (reading A3).
+ * ---------------------------------------------------------------------------------- */
+static double lse_axis(int d, const double *p, double gamma, double *grad, double *a_p, double *a_m)
+{
+    if (d < 2) {
+        for (int i = 0; i < d; i++) grad[i] = 0.0;
+        return 0.0;
+    }
+    double xp = p[0], xm = p[0];
+    for (int i = 1; i < d; i++) {
+        if (p[i] > xp) xp = p[i];
+        if (p[i] < xm) xm = p[i];
+    }
+    double bp = 0.0, bm = 0.0;
+    for (int i = 0; i < d; i++) {
+        a_p[i] = exp((p[i] - xp) / gamma);
+        a_m[i] = exp(-(p[i] - xm) / gamma);
+        bp += a_p[i];
+        bm += a_m[i];
+    }
+    double wl = (xp + gamma * log(bp)) - (xm - gamma * log(bm));
+    for (int i = 0; i < d; i++) grad[i] = a_p[i] / bp - a_m[i] / bm;
+    return wl;
+}
+
+/* Sum over nets of w_e (LSE_e^x + LSE_e^y) and its cell gradient, with the same pin model
+ * (reading A1) and accumulation contract as or_wa. */
+double or_lse(int64_t num_nets, const int32_t *net_start, const int32_t *pin2cell,
+              const double *pin_dx, const double *pin_dy, const double *net_weight,
+              const double *x, const double *y, double gamma,
+              double *gx, double *gy, double *wl_net)
+{
+    int dmax = 0;
+    for (int64_t e = 0; e < num_nets; e++) {
+        int d = net_start[e + 1] - net_start[e];
+        if (d > dmax) dmax = d;
+    }
+    size_t n = (size_t)(dmax > 0 ? dmax : 1);
+    double *px = malloc(n * sizeof(double)), *py = malloc(n * sizeof(double));
+    double *gxp = malloc(n * sizeof(double)), *gyp = malloc(n * sizeof(double));
+    double *ap = malloc(n * sizeof(double)), *am = malloc(n * sizeof(double));
+    double total = 0.0;
+    for (int64_t e = 0; e < num_nets; e++) {
+        int s = net_start[e], d = net_start[e + 1] - s;
+        for (int i = 0; i < d; i++) {
+            int c = pin2cell[s + i];
+            px[i] = x[c] + pin_dx[s + i];
+            py[i] = y[c] + pin_dy[s + i];
+        }
+        double we = net_weight ? net_weight[e] : 1.0;
+        double wl = we * (lse_axis(d, px, gamma, gxp, ap, am) + lse_axis(d, py, gamma, gyp, ap, am));
+        if (wl_net) wl_net[e] = wl;
+        total += wl;
+        for (int i = 0; i < d; i++) {
+            int c = pin2cell[s + i];
+            gx[c] += we * gxp[i];
+            gy[c] += we * gyp[i];
+        }
+    }
+    free(px); free(py); free(gxp); free(gyp); free(ap); free(am);
+    return total;
+}
+
 /* Per-net half-perimeter wirelength (named at P:95, used by eq 18's p at P:450; reading A6):
  *   h_e = (max px - min px) + (max py - min py),  px = x[cell] + dx in fp64;  d <= 1 -> 0.
  * The correctly rounded total is formed by the caller (math.fsum, reading A7). */

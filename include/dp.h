@@ -142,6 +142,16 @@ dp_status dp_eval(dp_ctx *ctx, const float *x, const float *y, float gamma, floa
 dp_status dp_wl_grad(dp_ctx *ctx, const float *x, const float *y, float gamma, float *gx,
                      float *gy, double *d_wl, dp_stream_t stream);
 
+/* Wirelength model used by dp_eval / dp_wl_grad from the next call on (default DP_WL_WA).
+ *   DP_WL_WA   weighted-average wirelength, eqs 3 and 6
+ *   DP_WL_LSE  log-sum-exp wirelength ("also implemented"; reading A27: the
+ *              definition of [29], LSE_e = gamma ln sum e^{x/gamma} + gamma ln sum e^{-x/gamma},
+ *              with the P:159 shift), gradient a_i^+/b^+ - a_i^-/b^-
+ * With DP_WL_LSE the d_wl output is the LSE total; a fused HPWL (d_hpwl != NULL) runs as a
+ * separate HPWL-only pass of the same kernel.  Errors: DP_ERR_INVALID_ARG (unknown model). */
+enum { DP_WL_WA = 0, DP_WL_LSE = 1 };
+dp_status dp_set_wl_model(dp_ctx *ctx, int32_t model);
+
 /* Density only: gx, gy <- dD/dx, dD/dy; d_energy <- D.                        */
 dp_status dp_density_grad(dp_ctx *ctx, const float *x, const float *y, float *gx, float *gy,
                           double *d_energy, dp_stream_t stream);

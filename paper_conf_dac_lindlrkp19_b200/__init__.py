@@ -22,9 +22,11 @@ __all__ = [
     "dp_partition_plan", "dp_eval", "dp_wl_grad", "dp_density_grad", "dp_hpwl", "dp_eval_host",
     "dp_get_info", "dp_debug_density_map", "dp_debug_fields", "dp_debug_transform",
     "DP_T_DCT2", "DP_T_IDCT2", "DP_T_IDXST_IDCT", "DP_T_IDCT_IDXST", "EXPORTED_SYMBOLS",
+    "dp_set_wl_model", "DP_WL_WA", "DP_WL_LSE",
 ]
 
 DP_T_DCT2, DP_T_IDCT2, DP_T_IDXST_IDCT, DP_T_IDCT_IDXST = 0, 1, 2, 3
+DP_WL_WA, DP_WL_LSE = 0, 1
 _STATUS = {0: "DP_OK", 1: "DP_ERR_INVALID_ARG", 2: "DP_ERR_UNSUPPORTED", 3: "DP_ERR_OUT_OF_MEMORY",
            4: "DP_ERR_CUDA", 5: "DP_ERR_NCCL"}
 
@@ -32,7 +34,7 @@ EXPORTED_SYMBOLS = [
     "dp_last_error", "dp_version", "dp_create", "dp_create_dist", "dp_nccl_unique_id",
     "dp_partition_plan", "dp_destroy", "dp_eval", "dp_wl_grad", "dp_density_grad", "dp_hpwl",
     "dp_eval_host", "dp_get_info", "dp_debug_density_map", "dp_debug_fields", "dp_debug_transform",
-    "dp_profile_enable", "dp_profile_read",
+    "dp_profile_enable", "dp_profile_read", "dp_set_wl_model",
 ]
 __all__ += ["dp_profile_enable", "dp_profile_read", "STAGES"]
 STAGES = ["wa", "map", "fields", "gather", "combine", "eval"]
@@ -97,6 +99,7 @@ def lib() -> ctypes.CDLL:
             "dp_debug_transform": [P, ctypes.c_int, P, P, P],
             "dp_profile_enable": [P, ctypes.c_int],
             "dp_profile_read": [P, P, P],
+            "dp_set_wl_model": [P, ctypes.c_int32],
         }.items():
             f = getattr(L, name)
             f.argtypes = args
@@ -188,6 +191,10 @@ class Context:
                 stream)
         return dict(gx=gx, gy=gy, obj=sc[0], wl=sc[1], energy=sc[2], hpwl=sc[3], scalars=sc)
 
+    def set_wl_model(self, model):
+        """"wa" / "lse" or DP_WL_WA / DP_WL_LSE (include/dp.h dp_set_wl_model)."""
+        dp_set_wl_model(self, {"wa": DP_WL_WA, "lse": DP_WL_LSE}.get(model, model))
+
     def wl_grad(self, x, y, gamma, stream=None):
         import torch
         gx = torch.empty(self.num_cells, dtype=torch.float32, device=self._dev())
@@ -278,6 +285,10 @@ def dp_eval(ctx, x, y, gamma, lam, gx, gy, d_obj=None, d_wl=None, d_energy=None,
 def dp_wl_grad(ctx, x, y, gamma, gx, gy, d_wl=None, stream=None):
     _check(lib().dp_wl_grad(ctx.handle, _ptr(x), _ptr(y), float(gamma), _ptr(gx), _ptr(gy), _ptr(d_wl),
                             _stream(stream)))
+
+
+def dp_set_wl_model(ctx, model: int):
+    _check(lib().dp_set_wl_model(ctx.handle, int(model)))
 
 
 def dp_density_grad(ctx, x, y, gx, gy, d_energy=None, stream=None):

@@ -699,7 +699,7 @@ dp_status eval_body(Ctx &c, const float *x, const float *y, float gamma, float l
 dp_status eval_graph(Ctx &c, const float *x, const float *y, float gamma, float lambda, float *gx, float *gy,
                      double *d_obj, double *d_wl, double *d_energy, double *d_hpwl, cudaStream_t s, bool do_wa,
                      bool do_den) {
-  const GraphKey key{x, y, gx, gy, d_obj, d_wl, d_energy, d_hpwl, gamma, lambda, do_wa, do_den};
+  const GraphKey key{x, y, gx, gy, d_obj, d_wl, d_energy, d_hpwl, gamma, lambda, do_wa, do_den, c.wl_model};
   if (!(c.gexec && key == c.gkey)) {
     cudaGraph_t g = nullptr;
     DP_CUDA(cudaStreamBeginCapture(c.s_cap, cudaStreamCaptureModeThreadLocal));
@@ -879,6 +879,14 @@ dp_status dp_wl_grad(dp_ctx *ctx, const float *x, const float *y, float gamma, f
   dp::DeviceGuard g(c->device);
   return dp::eval_impl(*c, x, y, gamma, 0.f, gx, gy, nullptr, d_wl, nullptr, nullptr, (cudaStream_t)stream, true,
                        false);
+}
+
+dp_status dp_set_wl_model(dp_ctx *ctx, int32_t model) {
+  Ctx *c = C(ctx);
+  if (!c) return fail(DP_ERR_INVALID_ARG, "ctx is NULL");
+  if (model != DP_WL_WA && model != DP_WL_LSE) return fail(DP_ERR_INVALID_ARG, "unknown wirelength model");
+  c->wl_model = model;
+  return DP_OK;
 }
 
 dp_status dp_density_grad(dp_ctx *ctx, const float *x, const float *y, float *gx, float *gy, double *d_energy,

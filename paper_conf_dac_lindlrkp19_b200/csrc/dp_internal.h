@@ -78,9 +78,11 @@ struct GraphKey {
   const void *obj = nullptr, *wl = nullptr, *en = nullptr, *hpwl = nullptr;
   float gamma = 0.f, lambda = 0.f;
   bool wa = false, den = false;
+  int wl_model = 0;
   bool operator==(const GraphKey &o) const {
     return x == o.x && y == o.y && gx == o.gx && gy == o.gy && obj == o.obj && wl == o.wl && en == o.en &&
-           hpwl == o.hpwl && gamma == o.gamma && lambda == o.lambda && wa == o.wa && den == o.den;
+           hpwl == o.hpwl && gamma == o.gamma && lambda == o.lambda && wa == o.wa && den == o.den &&
+           wl_model == o.wl_model;
   }
 };
 
@@ -136,6 +138,7 @@ struct Ctx {
   cudaStream_t s_cap = nullptr;
   cudaGraphExec_t gexec = nullptr;
   GraphKey gkey;
+  int wl_model = 0;        // DP_WL_WA / DP_WL_LSE (dp_set_wl_model)
   int sched = 0;           // DP_SCHED: 0 = WA from the fork, 1 = WA after the density map (overlaps the transforms)     // DP_SERIAL=1: density chain after WA (no stream overlap; measurement)
   int32_t walk_grid = 0;
   int32_t *d_walk_tile = nullptr;   // [walk_grid]   // CTAs of the persistent scatter / gather walkers (SMs x resident)

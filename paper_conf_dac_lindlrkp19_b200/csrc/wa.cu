@@ -81,6 +81,12 @@ __device__ __forceinline__ float ex2(float v) {
   return r;
 }
 
+__device__ __forceinline__ float lg2(float v) {
+  float r;
+  asm("lg2.approx.ftz.f32 %0, %1;" : "=f"(r) : "f"(v));
+  return r;
+}
+
 __device__ __forceinline__ float rcp(float v) {
   float r;
   asm("rcp.approx.ftz.f32 %0, %1;" : "=f"(r) : "f"(v));
@@ -319,7 +325,10 @@ __device__ __forceinline__ void wa_group_exact(const WaArgs &a, const WarpGroup 
 // P is a common shift that cancels in eq (3)/(6).  Everything is carried in log2 units
 // lambda = (x - P) log2(e)/gamma, so a = 2^lambda and (x - m)/gamma = (lambda - mu) ln 2.
 // Invalid slots get lambda = -+1e30 (a = 0, lambda a = 0): no per-slot branches.
-template <int S>
+//
+// LSE (NEXT-3, reading A27): the same b^+- sums; LSE_e = (x+ - x-) + gamma ln 2 (log2 b+ + log2 b-)
+// and dLSE/dx_i = a_i^+/b^+ - a_i^-/b^-; the c sums are not formed.
+template <int S, bool LSE>
 __device__ __forceinline__ void wa_group_fast(const WaArgs &a, const WarpGroup &wg, const GroupCtx &gc,
                                               float &wl_acc) {
   const int glog = wg.g_log2, G = 1 << glog;
@@ -366,23 +375,43 @@ __device__ __forceinline__ void wa_group_fast(const WaArgs &a, const WarpGroup &
     axm[s] = ex2(-lxm[s]);
     ayp[s] = ex2(lyp[s]);
     aym[s] = ex2(-lym[s]);
-    bxp += axp[s]; cxp = fmaf(lxp[s], axp[s], cxp);
-    bxm += axm[s]; cxm = fmaf(lxm[s], axm[s], cxm);
-    byp += ayp[s]; cyp = fmaf(lyp[s], ayp[s], cyp);
-    bym += aym[s]; cym = fmaf(lym[s], aym[s], cym);
+    bxp += axp[s];
+    bxm += axm[s];
+    byp += ayp[s];
+    bym += aym[s];
+    if (!LSE) {
+      cxp = fmaf(lxp[s], axp[s], cxp);
+      cxm = fmaf(lxm[s], axm[s], cxm);
+      cyp = fmaf(lyp[s], ayp[s], cyp);
+      cym = fmaf(lym[s], aym[s], cym);
+    }
   }
   for (int o = 1; o < G; o <<= 1) {
     bxp += __shfl_xor_sync(0xffffffffu, bxp, o);
-    cxp += __shfl_xor_sync(0xffffffffu, cxp, o);
     bxm += __shfl_xor_sync(0xffffffffu, bxm, o);
-    cxm += __shfl_xor_sync(0xffffffffu, cxm, o);
     byp += __shfl_xor_sync(0xffffffffu, byp, o);
-    cyp += __shfl_xor_sync(0xffffffffu, cyp, o);
     bym += __shfl_xor_sync(0xffffffffu, bym, o);
-    cym += __shfl_xor_sync(0xffffffffu, cym, o);
+    if (!LSE) {
+      cxp += __shfl_xor_sync(0xffffffffu, cxp, o);
+      cxm += __shfl_xor_sync(0xffffffffu, cxm, o);
+      cyp += __shfl_xor_sync(0xffffffffu, cyp, o);
+      cym += __shfl_xor_sync(0xffffffffu, cym, o);
+    }
   }
   if (d < 2) return;
   const float ibxp = rcp(bxp), ibxm = rcp(bxm), ibyp = rcp(byp), ibym = rcp(bym);
+  if (LSE) {
+    if (j == 0 && counted) {
+      const float ig2 = a.gamma * kLn2;
+      wl_acc += we * ((Px - Mx) + (Py - My) + (lg2(bxp) + lg2(bxm) + lg2(byp) + lg2(bym)) * ig2);
+    }
+    const float wxp = we * ibxp, wxm = we * ibxm, wyp = we * ibyp, wym = we * ibym;
+#pragma unroll
+    for (int s = 0; s < S; s++) {
+      if (vm & (1u << s)) grad_add(gc, raw[s], axp[s] * wxp - axm[s] * wxm, ayp[s] * wyp - aym[s] * wym);
+    }
+    return;
+  }
   const float mxp = cxp * ibxp, mxm = cxm * ibxm, myp = cyp * ibyp, mym = cym * ibym;  // log2 units
   if (j == 0 && counted) {
     // WL_e = (x+ - x-) + (mu+ - mu-) gamma ln 2   (eq 3 in shifted coordinates)
@@ -420,6 +449,9 @@ __device__ __forceinline__ float tanh_half(float t, float e) {
 // separation delta, WA = |delta| tanh(|delta| / 2 gamma) and dWA/dx_2 = -dWA/dx_1 =
 // sign(delta) [tanh(u/2) + (u/2) sech^2(u/2)], u = |delta| / gamma (pinned against the oracle
 // in tests/test_oracle_wa.py::test_two_pin_closed_form).
+//
+// LSE (reading A27): LSE = |delta| + 2 gamma ln(1 + e^-u) per axis and dLSE/dx_2 = sign(delta) tanh(u/2).
+template <bool LSE>
 __device__ __forceinline__ void wa_group_pairs(const WaArgs &a, const WarpGroup &wg, const GroupCtx &gc,
                                                float &wl_acc) {
   const int lane = gc.lane;
@@ -434,7 +466,16 @@ __device__ __forceinline__ void wa_group_pairs(const WaArgs &a, const WarpGroup 
   const float ddx = (gc.px[s1] - gc.px[s0]) + (gc.dx[p1] - gc.dx[p0]);
   const float ddy = (gc.py[s1] - gc.py[s0]) + (gc.dy[p1] - gc.dy[p0]);
   const float tx = fabsf(ddx) * a.k2, ty = fabsf(ddy) * a.k2;   // u log2(e)
-  const float thx = tanh_half(tx, ex2(-tx)), thy = tanh_half(ty, ex2(-ty));
+  const float ex = ex2(-tx), ey = ex2(-ty);
+  const float thx = tanh_half(tx, ex), thy = tanh_half(ty, ey);
+  if (LSE) {
+    if (counted)
+      wl_acc += we * (fabsf(ddx) + fabsf(ddy) + (2.f * kLn2) * a.gamma * (lg2(1.f + ex) + lg2(1.f + ey)));
+    const float gx = copysignf(we * thx, ddx), gy = copysignf(we * thy, ddy);
+    grad_add(gc, r1, gx, gy);
+    grad_add(gc, r0, -gx, -gy);
+    return;
+  }
   if (counted) wl_acc += we * (fabsf(ddx) * thx + fabsf(ddy) * thy);
   const float hx = 0.5f * kLn2 * tx, hy = 0.5f * kLn2 * ty;
   const float gx = copysignf(we * fmaf(hx, fmaf(-thx, thx, 1.f), thx), ddx);   // d/dx of pin 1
@@ -490,7 +531,8 @@ static_assert(kBigThreads == kWaThreads && kWarpNetThreads == kWaThreads, "big /
 template <int MODE>
 __device__ __forceinline__ void wa_big_net(const WaArgs &a, int net, float4 *s_pin) {
   constexpr bool kGrad = MODE != 2;
-  constexpr bool kHpwl = MODE != 0;
+  constexpr bool kHpwl = MODE == 1 || MODE == 2;
+  constexpr bool kLse = MODE == 3;
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   constexpr int NW = kBigThreads / 32;
   const int s0 = a.big_start[net], d = a.big_start[net + 1] - s0;
@@ -576,7 +618,10 @@ __device__ __forceinline__ void wa_big_net(const WaArgs &a, int net, float4 *s_p
     if (tid == 0 && counted) {
       const float spanx = __fadd_rn(__fsub_rn(e.Xh, e.xh), __fsub_rn(e.Xl, e.xl));
       const float spany = __fadd_rn(__fsub_rn(e.Yh, e.yh), __fsub_rn(e.Yl, e.yl));
-      wl_acc = (double)(we * ((spanx + mxp - mxm) + (spany + myp - mym)));
+      if (kLse)   // reading A27: (x+ + gamma ln b+) - (x- - gamma ln b-)
+        wl_acc = (double)(we * ((spanx + spany) + a.gamma * (logf(sm[0]) + logf(sm[2]) + logf(sm[4]) + logf(sm[6]))));
+      else
+        wl_acc = (double)(we * ((spanx + mxp - mxm) + (spany + myp - mym)));
     }
     for (int p = tid; p < d; p += kBigThreads) {
       const int raw = __ldg(a.big_cell + s0 + p);
@@ -588,10 +633,12 @@ __device__ __forceinline__ void wa_big_net(const WaArgs &a, int net, float4 *s_p
       const float lym = __fadd_rn(__fsub_rn(v.z, e.yh), __fsub_rn(v.w, e.yl));
       const float axp = ex2(lxp * a.k2), axm = ex2(-lxm * a.k2);
       const float ayp = ex2(lyp * a.k2), aym = ex2(-lym * a.k2);
-      const float gx = we * (axp * ibxp * (1.f + (lxp - mxp) * a.inv_gamma) -
-                             axm * ibxm * (1.f - (lxm - mxm) * a.inv_gamma));
-      const float gy = we * (ayp * ibyp * (1.f + (lyp - myp) * a.inv_gamma) -
-                             aym * ibym * (1.f - (lym - mym) * a.inv_gamma));
+      const float gx = kLse ? we * (axp * ibxp - axm * ibxm)
+                            : we * (axp * ibxp * (1.f + (lxp - mxp) * a.inv_gamma) -
+                                    axm * ibxm * (1.f - (lxm - mxm) * a.inv_gamma));
+      const float gy = kLse ? we * (ayp * ibyp - aym * ibym)
+                            : we * (ayp * ibyp * (1.f + (lyp - myp) * a.inv_gamma) -
+                                    aym * ibym * (1.f - (lym - mym) * a.inv_gamma));
       red_v2(a.g2 + raw, gx, gy);
     }
   }
@@ -623,7 +670,8 @@ __device__ __forceinline__ float warp_sum(float v) {
 template <int MODE>
 __device__ __forceinline__ void wa_warp_nets(const WaArgs &a, int wb) {
   constexpr bool kGrad = MODE != 2;
-  constexpr bool kHpwl = MODE != 0;
+  constexpr bool kHpwl = MODE == 1 || MODE == 2;
+  constexpr bool kLse = MODE == 3;
   const int lane = threadIdx.x & 31;
   const int net = a.n_huge + wb * (kWarpNetThreads / 32) + (threadIdx.x >> 5);
   double wl_acc = 0.0;
@@ -636,7 +684,7 @@ __device__ __forceinline__ void wa_warp_nets(const WaArgs &a, int wb) {
     const float we = a.has_w ? a.big_w[net] : 1.f;
     const int *cell = a.big_cell + s0;
     const float *pdx = a.big_dx + s0, *pdy = a.big_dy + s0;
-    if (MODE == 0) {
+    if (MODE == 0 || MODE == 3) {
       float Px = -INFINITY, Mx = INFINITY, Py = -INFINITY, My = INFINITY;
 #pragma unroll 4
       for (int p = lane; p < d; p += 32) {
@@ -667,7 +715,10 @@ __device__ __forceinline__ void wa_warp_nets(const WaArgs &a, int wb) {
       const float mxp = cxp * ibxp, mxm = cxm * ibxm, myp = cyp * ibyp, mym = cym * ibym;   // log2 units
       if (lane == 0 && counted) {
         const float ig2 = a.gamma * kLn2;
-        wl_acc = (double)(we * ((Px - Mx) + (mxp - mxm) * ig2 + (Py - My) + (myp - mym) * ig2));
+        if (kLse)
+          wl_acc = (double)(we * ((Px - Mx) + (Py - My) + (lg2(bxp) + lg2(bxm) + lg2(byp) + lg2(bym)) * ig2));
+        else
+          wl_acc = (double)(we * ((Px - Mx) + (mxp - mxm) * ig2 + (Py - My) + (myp - mym) * ig2));
       }
       const float wl2 = we * kLn2;
       const float qxp = ibxp * wl2, pxp = we * ibxp - mxp * qxp;
@@ -683,8 +734,8 @@ __device__ __forceinline__ void wa_warp_nets(const WaArgs &a, int wb) {
         const float lxp = fmaf(xc - Px, k2, dkx), lxm = fmaf(xc - Mx, k2, dkx);
         const float lyp = fmaf(yc - Py, k2, dky), lym = fmaf(yc - My, k2, dky);
         const float axp = ex2(lxp), axm = ex2(-lxm), ayp = ex2(lyp), aym = ex2(-lym);
-        const float gx = axp * fmaf(lxp, qxp, pxp) - axm * fmaf(-lxm, qxm, pxm);
-        const float gy = ayp * fmaf(lyp, qyp, pyp) - aym * fmaf(-lym, qym, pym);
+        const float gx = kLse ? we * (axp * ibxp - axm * ibxm) : axp * fmaf(lxp, qxp, pxp) - axm * fmaf(-lxm, qxm, pxm);
+        const float gy = kLse ? we * (ayp * ibyp - aym * ibym) : ayp * fmaf(lyp, qyp, pyp) - aym * fmaf(-lym, qym, pym);
         red_v2(a.g2 + raw, gx, gy);
       }
     } else {
@@ -753,11 +804,11 @@ __device__ __forceinline__ void wa_warp_nets(const WaArgs &a, int wb) {
                                        a.limbs);
 }
 
-// MODE 0: WA + gradient; 1: WA + gradient + HPWL; 2: HPWL only.
+// MODE 0: WA + gradient; 1: WA + gradient + HPWL; 2: HPWL only; 3: LSE + gradient (NEXT-3).
 template <int MODE>
 __global__ void __launch_bounds__(kWaThreads, 3) k_wa_chunks(WaArgs a) {
   constexpr bool kGrad = MODE != 2;
-  constexpr bool kHpwl = MODE != 0;
+  constexpr bool kHpwl = MODE == 1 || MODE == 2;
   extern __shared__ __align__(16) unsigned char smem[];
   const WaSmem L_{a.caps};
   int *s_slot = reinterpret_cast<int *>(smem + L_.off_slot());
@@ -858,15 +909,16 @@ __global__ void __launch_bounds__(kWaThreads, 3) k_wa_chunks(WaArgs a) {
   // warp groups are dealt round-robin (the host orders them by decreasing cost)
   for (int gi = warp; gi < ch.wg_n; gi += kWaThreads / 32) {
     const WarpGroup wg = s_wg[gi];
-    if (MODE == 0) {
+    if (MODE == 0 || MODE == 3) {
+      constexpr bool kL = MODE == 3;
       if (wg.flags & 1) {
-        wa_group_pairs(a, wg, gc, wl_acc);
+        wa_group_pairs<kL>(a, wg, gc, wl_acc);
       } else {
         switch (wg.slots) {
-          case 1: wa_group_fast<1>(a, wg, gc, wl_acc); break;
-          case 2: wa_group_fast<2>(a, wg, gc, wl_acc); break;
-          case 3: wa_group_fast<3>(a, wg, gc, wl_acc); break;
-          default: wa_group_fast<4>(a, wg, gc, wl_acc); break;
+          case 1: wa_group_fast<1, kL>(a, wg, gc, wl_acc); break;
+          case 2: wa_group_fast<2, kL>(a, wg, gc, wl_acc); break;
+          case 3: wa_group_fast<3, kL>(a, wg, gc, wl_acc); break;
+          default: wa_group_fast<4, kL>(a, wg, gc, wl_acc); break;
         }
       }
     } else {
@@ -922,6 +974,8 @@ cudaError_t wa_configure(const WaCaps &caps) {
   if (e != cudaSuccess) return e;
   e = cudaFuncSetAttribute(k_wa_chunks<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, b);
   if (e != cudaSuccess) return e;
+  e = cudaFuncSetAttribute(k_wa_chunks<3>, cudaFuncAttributeMaxDynamicSharedMemorySize, b);
+  if (e != cudaSuccess) return e;
   return cudaFuncSetAttribute(k_wa_chunks<2>, cudaFuncAttributeMaxDynamicSharedMemorySize, b);
 }
 
@@ -959,12 +1013,16 @@ void launch_wa(const Ctx &c, const float *x, const float *y, float gamma, bool h
   // big-net pins staged in the chunk kernel's dynamic shared memory (larger nets reload)
   a.big_stage = std::min(c.big_stage, wa_smem_bytes(c.wa_caps) / 16);
   a.caps = c.wa_caps;
-  if (hpwl_only)
+  if (hpwl_only) {
     launch_mode<2>(c, a, s);
-  else if (with_hpwl)
+  } else if (c.wl_model == DP_WL_LSE) {   // LSE: fast path; a fused HPWL is a second, HPWL-only pass
+    launch_mode<3>(c, a, s);
+    if (with_hpwl) launch_mode<2>(c, a, s);
+  } else if (with_hpwl) {
     launch_mode<1>(c, a, s);
-  else
+  } else {
     launch_mode<0>(c, a, s);
+  }
 }
 
 }  // namespace dp

@@ -1,0 +1,115 @@
+"""Pins for the GP-loop oracle (oracle/gp.py), CPU only.
+
+What the paper fixes: the eq (18) density-weight factor and its stated behaviour over the
+iterations.  What the mathematics fixes: Lipschitz step prediction on a quadratic
+(the step is exactly 1/L, so an isotropic quadratic is minimised in one step), Nesterov
+convergence on an ill-conditioned quadratic, the overflow of configurations with a known
+density, the preconditioner's pin counts (brute force).  And one end-to-end property: from
+the paper's initial placement the loop spreads the cells (overflow falls).
+"""
+import math
+
+import numpy as np
+import pytest
+
+import oracle
+from oracle import gp
+from synth import custom_netlist, make_netlist, make_positions
+
+
+def test_mu_follows_eq18_and_p452():
+    """'from iteration 0 to 200, mu gradually drops from 1.05 to 1.03 and keeps this
+    value afterward' (for p < 0); eq (18a): mu = mu_max at p = 0 (mu_max^(1-0)), 1 at p = 1,
+    and never below mu_min."""
+    prm = gp.GpParams()
+    assert gp.mu(-1.0, 0, prm) == pytest.approx(1.05, abs=1e-15)
+    m200 = gp.mu(-1.0, 200, prm)
+    assert 1.029 <= m200 <= 1.031
+    assert all(gp.mu(-0.5, k, prm) <= gp.mu(-0.5, k - 1, prm) for k in range(1, 400))
+    assert gp.mu(-1.0, 203, prm) == gp.mu(-1.0, 5000, prm)     # "keeps this value afterward" (0.9999^k = 0.98 at k = 202)
+    assert gp.mu(0.0, 10, prm) == pytest.approx(1.05, abs=1e-15)
+    assert gp.mu(1.0, 10, prm) == pytest.approx(1.0, abs=1e-15)
+    assert gp.mu(50.0, 10, prm) == 0.95
+
+
+def test_lipschitz_step_solves_isotropic_quadratic_in_one_step():
+    """f(z) = c/2 |z - z*|^2: ||dv|| / ||dg|| = 1/c exactly, so u_1 = v - g/c = z*."""
+    rng = np.random.default_rng(0)
+    c, zs = 3.7, rng.normal(size=50)
+    v = rng.normal(size=50)
+    vp = v + 1e-3 * rng.normal(size=50)
+    grad = lambda z: c * (z - zs)  # noqa: E731
+    u1, _, _, alpha = gp.nesterov_step(v.copy(), v, vp, grad(v), grad(vp), 1.0, 0.0, lambda z: z)
+    assert alpha == pytest.approx(1 / c, rel=1e-12)
+    np.testing.assert_allclose(u1, zs, rtol=0, atol=1e-12)
+
+
+def test_nesterov_converges_on_ill_conditioned_quadratic():
+    """Diagonal quadratic with condition number 100: the objective falls by > 1e6."""
+    rng = np.random.default_rng(1)
+    n = 200
+    d = np.geomspace(1.0, 100.0, n)
+    zs = rng.normal(size=n)
+    f = lambda z: 0.5 * float(np.sum(d * (z - zs) ** 2))  # noqa: E731
+    grad = lambda z: d * (z - zs)  # noqa: E731
+    u = v = rng.normal(size=n)
+    vp = v - 1e-3 * grad(v)
+    g, gprev, a, alpha = grad(v), grad(vp), 1.0, 0.0
+    f0 = f(u)
+    for _ in range(300):
+        u, vn, a, alpha = gp.nesterov_step(u, v, vp, g, gprev, a, alpha, lambda z: z)
+        vp, gprev, v, g = v, g, vn, grad(vn)
+    assert f(u) < 1e-6 * f0
+
+
+def test_overflow_closed_forms():
+    """One unstretched cell exactly covering one bin: rho = 1 there, so tau = (1 - t) b^2 / (w h)
+    = 1 - t; a uniform tiling at density 1 has tau = 0 for t = 1."""
+    b = 10.0
+    nl = custom_netlist([0, 0], [], [], [], [b], [b], (0, 0, 16 * b, 16 * b), (16, 16))
+    rho = oracle.density_map(nl, np.array([3 * b], np.float32), np.array([5 * b], np.float32), stretch=0)
+    assert gp.overflow(nl, rho, 0.25) == pytest.approx(0.75, rel=1e-12)
+    assert gp.overflow(nl, rho, 1.0) == 0.0
+    n = 16
+    xs, ys = np.meshgrid(np.arange(n) * b, np.arange(n) * b, indexing="ij")
+    nl2 = custom_netlist([0, 0], [], [], [], np.full(n * n, b), np.full(n * n, b), (0, 0, n * b, n * b), (n, n))
+    rho2 = oracle.density_map(nl2, xs.ravel().astype(np.float32), ys.ravel().astype(np.float32), stretch=0)
+    assert gp.overflow(nl2, rho2, 1.0) == pytest.approx(0.0, abs=1e-12)
+    assert gp.overflow(nl2, rho2, 0.5) == pytest.approx(0.5, rel=1e-12)
+
+
+def test_gamma_schedule_endpoints():
+    """A31 (RePlAce): gamma = 10 gamma_base at tau = 1 and gamma_base / 10 at tau = 0.1."""
+    nl = make_netlist("tiny")
+    prm = gp.GpParams()
+    base = 4.0 * (nl.bin_w + nl.bin_h)
+    assert gp.gamma_of(nl, 1.0, prm) == pytest.approx(10 * base, rel=1e-12)
+    assert gp.gamma_of(nl, 0.1, prm) == pytest.approx(base / 10, rel=1e-12)
+
+
+def test_cell_pins_brute_force():
+    nl = make_netlist("tiny")
+    nl.net_weight = np.random.default_rng(2).uniform(0.5, 2.0, nl.num_nets).astype(np.float32)
+    ref = np.zeros(nl.num_cells)
+    for e in range(nl.num_nets):
+        for p in range(nl.net_start[e], nl.net_start[e + 1]):
+            ref[nl.pin2cell[p]] += float(nl.net_weight[e])
+    np.testing.assert_allclose(gp.cell_pins(nl), ref, rtol=1e-12)
+
+
+def test_gp_loop_spreads_the_initial_placement():
+    """From the paper's initial placement (cells at the centre with 0.1% noise) the
+    loop spreads the cells: overflow falls well below its start, HPWL stays finite, lambda
+    grows (the density term gains weight, eq 18)."""
+    nl = make_netlist("tiny")
+    x, y = make_positions(nl, "initial")
+    st = gp.gp_init(nl, x, y)
+    tau0, lam0 = st.tau, st.lam
+    hist = [gp.gp_step(nl, st) for _ in range(400)]
+    assert tau0 > 0.8
+    assert hist[-1]["overflow"] < 0.1                  # DREAMPlace stops GP at 0.07-0.1
+    assert min(h["overflow"] for h in hist[:100]) > 0.9 * tau0   # lambda_0 is small: WL first
+    assert all(math.isfinite(h["hpwl"]) for h in hist)
+    assert st.lam > lam0
+    # cells stay inside the region (A33 clamp)
+    assert np.all(st.u[0] >= nl.xl) and np.all(st.u[0] <= nl.xh - nl.cell_w + 1e-9)

@@ -168,6 +168,56 @@ dp_status dp_eval_host(dp_ctx *ctx, const float *hx, const float *hy, float gamm
                        float lambda, float *hgx, float *hgy, double *h_scalars,
                        int with_hpwl, dp_stream_t stream);
 
+/* ---- GP loop --------------------------------------------------------
+ * The global-placement iterations around the evaluation, entirely on the device: "the loop
+ * that involves the computation of wirelength and density gradient, optimization engines,
+ * and cell location updating", with ePlace's Nesterov method and Lipschitz step
+ * prediction and the eq (18) density-weight update with DREAMPlace's change for
+ * p < 0.  Readings A28-A33 fix what the paper leaves to ePlace /
+ * RePlAce: step A28, preconditioner A29, overflow A30, gamma schedule A31, lambda_0 A32,
+ * clamp / first step A33.  One iteration is captured once into a CUDA graph and replayed
+ * (no host synchronisation per iteration).  Single-GPU contexts only (DP_ERR_UNSUPPORTED for
+ * dp_create_dist contexts).  The context's wirelength model (dp_set_wl_model) applies.      */
+typedef struct dp_gp_params {
+    float target_density;    /* t of the overflow (A30); default 1.0                         */
+    float gamma_base_scale;  /* gamma_base = scale (b_x + b_y) (A31); default 4.0            */
+    float lambda_scale;      /* lambda_0 = scale |grad WL|_1 / |grad D|_1 (A32); default 8e-5 */
+    float mu_min, mu_max;    /* eq (18a); defaults 0.95, 1.05                        */
+    float dhpwl_ref;         /* p = dHPWL / dhpwl_ref; default 3.5e5                 */
+    float init_rms_bins;     /* rms displacement of v_{-1}, in bins (A33); default 0.01     */
+    int32_t max_history;     /* iterations kept in the device history ring; default 4096    */
+} dp_gp_params;
+typedef struct dp_gp dp_gp;  /* opaque; owns ~12 float vectors of num_cells + scalars       */
+
+/* Fill *p with the defaults above. */
+void dp_gp_default_params(dp_gp_params *p);
+
+/* Create a GP loop on ctx (params NULL = defaults).  The loop borrows ctx: destroy it first.
+ * Errors: DP_ERR_INVALID_ARG (null, out-of-range params), DP_ERR_UNSUPPORTED (distributed
+ * context), DP_ERR_OUT_OF_MEMORY / DP_ERR_CUDA.                                            */
+dp_status dp_gp_create(dp_ctx *ctx, const dp_gp_params *params, dp_gp **out);
+
+/* Start from x0, y0 (device, [num_cells], lower-left corners; clamped into the region):
+ * tau_0 and gamma_0 from the density map, lambda_0 (A32), g_0, HPWL_0, and the first
+ * Lipschitz reference point v_{-1} (A33).  Asynchronous on `stream`.                        */
+dp_status dp_gp_init(dp_gp *gp, const float *x0, const float *y0, dp_stream_t stream);
+
+/* Run `iterations` GP iterations (A28: step, Nesterov update, evaluation at v_{k+1},
+ * preconditioner, overflow, lambda and gamma updates).  Asynchronous on `stream`.            */
+dp_status dp_gp_run(dp_gp *gp, int32_t iterations, dp_stream_t stream);
+
+/* Copy the major solution u (device) into x, y (device, [num_cells]).  Asynchronous.        */
+dp_status dp_gp_positions(dp_gp *gp, float *x, float *y, dp_stream_t stream);
+
+/* Synchronise the device and copy the history of the last min(max_rows, iterations,
+ * max_history) iterations, oldest first, into h_rows (host, [max_rows][8]):
+ *   {k, HPWL(v_{k+1}), overflow(v_{k+1}), lambda_{k+1}, gamma_{k+1}, obj, alpha_k, WL}.
+ * *rows <- rows written.                                                                    */
+dp_status dp_gp_history(dp_gp *gp, double *h_rows, int32_t max_rows, int32_t *rows);
+
+/* Free the loop's buffers (synchronises the device).  NULL is accepted. */
+dp_status dp_gp_destroy(dp_gp *gp);
+
 /* ---- introspection -------------------------------------------------------------------- */
 typedef struct dp_info {
     int32_t num_cells, num_nets, num_pins;       /* as stored on this rank                 */

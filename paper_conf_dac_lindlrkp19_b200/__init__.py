@@ -22,7 +22,7 @@ __all__ = [
     "dp_partition_plan", "dp_eval", "dp_wl_grad", "dp_density_grad", "dp_hpwl", "dp_eval_host",
     "dp_get_info", "dp_debug_density_map", "dp_debug_fields", "dp_debug_transform",
     "DP_T_DCT2", "DP_T_IDCT2", "DP_T_IDXST_IDCT", "DP_T_IDCT_IDXST", "EXPORTED_SYMBOLS",
-    "dp_set_wl_model", "DP_WL_WA", "DP_WL_LSE",
+    "dp_set_wl_model", "DP_WL_WA", "DP_WL_LSE", "GpParams", "GpLoop", "dp_gp_create",
 ]
 
 DP_T_DCT2, DP_T_IDCT2, DP_T_IDXST_IDCT, DP_T_IDCT_IDXST = 0, 1, 2, 3
@@ -35,6 +35,8 @@ EXPORTED_SYMBOLS = [
     "dp_partition_plan", "dp_destroy", "dp_eval", "dp_wl_grad", "dp_density_grad", "dp_hpwl",
     "dp_eval_host", "dp_get_info", "dp_debug_density_map", "dp_debug_fields", "dp_debug_transform",
     "dp_profile_enable", "dp_profile_read", "dp_set_wl_model",
+    "dp_gp_default_params", "dp_gp_create", "dp_gp_init", "dp_gp_run", "dp_gp_positions",
+    "dp_gp_history", "dp_gp_destroy",
 ]
 __all__ += ["dp_profile_enable", "dp_profile_read", "STAGES"]
 STAGES = ["wa", "map", "fields", "gather", "combine", "eval"]
@@ -66,6 +68,13 @@ class DpInfo(ctypes.Structure):
                 ("cell_end", I32), ("bins_x", I32), ("bins_y", I32), ("rank", I32), ("world", I32),
                 ("launches_eval", I32), ("launches_eval_hpwl", I32), ("device_bytes", ctypes.c_int64),
                 ("num_sms", I32), ("l2_bytes", I32)]
+
+
+class GpParams(ctypes.Structure):
+    """dp_gp_params (include/dp.h)."""
+    _fields_ = [("target_density", ctypes.c_float), ("gamma_base_scale", ctypes.c_float),
+                ("lambda_scale", ctypes.c_float), ("mu_min", ctypes.c_float), ("mu_max", ctypes.c_float),
+                ("dhpwl_ref", ctypes.c_float), ("init_rms_bins", ctypes.c_float), ("max_history", I32)]
 
 
 _lib = None
@@ -100,10 +109,18 @@ def lib() -> ctypes.CDLL:
             "dp_profile_enable": [P, ctypes.c_int],
             "dp_profile_read": [P, P, P],
             "dp_set_wl_model": [P, ctypes.c_int32],
+            "dp_gp_create": [P, ctypes.POINTER(GpParams), ctypes.POINTER(P)],
+            "dp_gp_init": [P, P, P, P],
+            "dp_gp_run": [P, ctypes.c_int32, P],
+            "dp_gp_positions": [P, P, P, P],
+            "dp_gp_history": [P, P, ctypes.c_int32, ctypes.POINTER(I32)],
+            "dp_gp_destroy": [P],
         }.items():
             f = getattr(L, name)
             f.argtypes = args
             f.restype = ctypes.c_int
+        L.dp_gp_default_params.argtypes = [ctypes.POINTER(GpParams)]
+        L.dp_gp_default_params.restype = None
         _lib = L
     return _lib
 
@@ -237,6 +254,61 @@ class Context:
         out = torch.empty(self.bins, dtype=torch.float32, device=self._dev())
         dp_debug_transform(self, kind, inp, out, stream)
         return out
+
+
+class GpLoop:
+    """The GP loop of include/dp.h (dp_gp_*): argument marshalling only."""
+    HIST_COLS = ("k", "hpwl", "overflow", "lam", "gamma", "obj", "alpha", "wl")
+
+    def __init__(self, ctx: Context, params: GpParams | None = None, **overrides):
+        self.ctx = ctx
+        p = GpParams()
+        lib().dp_gp_default_params(ctypes.byref(p))
+        if params is not None:
+            p = params
+        for k, v in overrides.items():
+            setattr(p, k, v)
+        self.params = p
+        h = ctypes.c_void_p()
+        _check(lib().dp_gp_create(ctx.handle, ctypes.byref(p), ctypes.byref(h)))
+        self.handle = h
+
+    def init(self, x0, y0, stream=None):
+        _check(lib().dp_gp_init(self.handle, _ptr(x0), _ptr(y0), _stream(stream)))
+
+    def run(self, iterations: int, stream=None):
+        _check(lib().dp_gp_run(self.handle, int(iterations), _stream(stream)))
+
+    def positions(self, stream=None):
+        import torch
+        x = torch.empty(self.ctx.num_cells, dtype=torch.float32, device=self.ctx._dev())
+        y = torch.empty_like(x)
+        _check(lib().dp_gp_positions(self.handle, _ptr(x), _ptr(y), _stream(stream)))
+        return x, y
+
+    def history(self, max_rows: int = 1 << 16):
+        import numpy as np
+        buf = np.zeros((max_rows, 8), dtype=np.float64)
+        n = I32()
+        _check(lib().dp_gp_history(self.handle, buf.ctypes.data_as(ctypes.c_void_p), int(max_rows),
+                                   ctypes.byref(n)))
+        rows = buf[:n.value]
+        return [dict(zip(self.HIST_COLS, r)) for r in rows]
+
+    def close(self):
+        if getattr(self, "handle", None):
+            lib().dp_gp_destroy(self.handle)
+            self.handle = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+def dp_gp_create(ctx: Context, params: GpParams | None = None, **overrides) -> GpLoop:
+    return GpLoop(ctx, params, **overrides)
 
 
 # ---- functions with the C names -----------------------------------------------------------

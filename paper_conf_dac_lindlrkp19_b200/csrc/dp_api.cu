@@ -548,6 +548,16 @@ dp_status create(const dp_netlist *nl, const dp_grid *grid, int device, int rank
   };
   if ((st = build_wa(*c, nl, mask)) != DP_OK) return bail(st);
   if ((st = build_density(*c, nl)) != DP_OK) return bail(st);
+  {   // net-weighted pin count per cell: the GP preconditioner's P_i (gp.cu, reading A29)
+    std::vector<double> acc(nl->num_cells, 0.0);
+    for (int32_t e = 0; e < nl->num_nets; e++) {
+      const double w = nl->net_weight ? (double)nl->net_weight[e] : 1.0;
+      for (int32_t k = nl->net_start[e]; k < nl->net_start[e + 1]; k++)
+        acc[nl->pin2cell[nl->net2pin ? nl->net2pin[k] : k]] += w;
+    }
+    std::vector<float> pins(acc.begin(), acc.end());
+    if ((st = dev_upload(*c, &c->d_cell_pins, pins)) != DP_OK) return bail(st);
+  }
   c->n_wa_part = c->n_chunks + c->n_huge + (c->n_big - c->n_huge + kWarpNetThreads / 32 - 1) / (kWarpNetThreads / 32);
   c->n_en_part = c->my / 2;   // = CTAs of the column-fields kernel (2-column slabs)
   if ((st = dev_alloc(*c, &c->d_g2, c->num_cells)) != DP_OK) return bail(st);
@@ -797,6 +807,15 @@ dp_status eval_body(Ctx &c, const float *x, const float *y, float gamma, float l
 }
 
 }  // namespace
+
+// entry points for gp.cu (the GP loop captures one iteration around the evaluation)
+dp_status eval_body_ext(Ctx &c, const float *x, const float *y, float gamma, float lambda, float *gx, float *gy,
+                        double *d_obj, double *d_wl, double *d_energy, double *d_hpwl, cudaStream_t s, bool do_wa,
+                        bool do_den) {
+  return eval_body(c, x, y, gamma, lambda, gx, gy, d_obj, d_wl, d_energy, d_hpwl, s, do_wa, do_den);
+}
+dp_status ctx_call_begin(Ctx &c, cudaStream_t s) { return call_begin(c, s); }
+dp_status ctx_call_end(Ctx &c, cudaStream_t s) { return call_end(c, s); }
 }  // namespace dp
 
 using dp::C;

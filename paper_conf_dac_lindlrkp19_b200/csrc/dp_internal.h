@@ -123,6 +123,7 @@ struct Ctx {
 
   // ---- density layout (device) ----
   float *d_cell_w = nullptr, *d_cell_h = nullptr;   // own cells (index from cell_begin)
+  float *d_cell_pins = nullptr;                     // [num_cells] net-weighted pin count (GP preconditioner)
   int32_t n_own = 0;                // cells owned by this rank
   int32_t n_large = 0;              // large cells (footprint > 3 bins on an axis)
   int32_t *d_large = nullptr;       // ids of large own cells
@@ -139,6 +140,9 @@ struct Ctx {
   cudaGraphExec_t gexec = nullptr;
   GraphKey gkey;
   int wl_model = 0;        // DP_WL_WA / DP_WL_LSE (dp_set_wl_model)
+  // GP loop (gp.cu): while non-null, the evaluation kernels read gamma / lambda from these
+  // device scalars instead of their by-value arguments (one captured graph per GP iteration)
+  const float *gamma_dev = nullptr, *lambda_dev = nullptr;
   int sched = 0;           // DP_SCHED: 0 = WA from the fork, 1 = WA after the density map (overlaps the transforms)     // DP_SERIAL=1: density chain after WA (no stream overlap; measurement)
   int32_t walk_grid = 0;
   int32_t *d_walk_tile = nullptr;   // [walk_grid]   // CTAs of the persistent scatter / gather walkers (SMs x resident)
@@ -214,6 +218,11 @@ void launch_transform(const Ctx &c, int kind, const float *in, float *out, cudaS
 void launch_split_fields(const Ctx &c, float *xi_x, float *xi_y, cudaStream_t s);
 void launch_psi(const Ctx &c, const float *rho, float *psi, cudaStream_t s);
 // combine / finalize (finalize.cu)
+dp_status eval_body_ext(Ctx &c, const float *x, const float *y, float gamma, float lambda, float *gx, float *gy,
+                        double *d_obj, double *d_wl, double *d_energy, double *d_hpwl, cudaStream_t s, bool do_wa,
+                        bool do_den);
+dp_status ctx_call_begin(Ctx &c, cudaStream_t s);
+dp_status ctx_call_end(Ctx &c, cudaStream_t s);
 void launch_combine(const Ctx &c, float lambda, float *gx, float *gy, bool use_wa,
                     bool use_density, cudaStream_t s);
 void launch_finalize(const Ctx &c, float lambda, bool with_wl, bool with_energy,

@@ -18,7 +18,9 @@ namespace {
 // global cells are 16-byte aligned in both arrays.
 __global__ void __launch_bounds__(256) k_combine(const float2 *__restrict__ g2, const float2 *__restrict__ force,
                                                  float *__restrict__ gx, float *__restrict__ gy, int cell_begin,
-                                                 int n_own, float lambda, int use_wa, int use_den) {
+                                                 int n_own, float lambda, const float *__restrict__ lambda_dev,
+                                                 int use_wa, int use_den) {
+  if (lambda_dev) lambda = __ldg(lambda_dev);   // GP loop: lambda on the device
   const int c0 = (cell_begin & ~3) + 4 * (blockIdx.x * blockDim.x + threadIdx.x);
   const int cend = cell_begin + n_own;
   if (c0 >= cend) return;
@@ -104,6 +106,7 @@ struct FinArgs {
   double *scal;   // staging {wl, energy, hpwl, obj}
   double *d_obj, *d_wl, *d_energy, *d_hpwl;
   float lambda;
+  const float *lambda_dev;
   int with_wl, with_energy, with_hpwl, phase;  // phase 0: local sums -> scal (dist), 1: outputs, 2: both
 };
 
@@ -133,6 +136,7 @@ __global__ void __launch_bounds__(256) k_finalize(FinArgs a) {
   }
   if (a.phase == 0) return;
   __syncthreads();
+  if (a.lambda_dev) a.lambda = *a.lambda_dev;
   if (threadIdx.x == 0) {
     const double wl = a.scal[0], en = a.scal[1];
     double hp = __longlong_as_double(0x7ff8000000000000ll);
@@ -156,8 +160,8 @@ void launch_combine(const Ctx &c, float lambda, float *gx, float *gy, bool use_w
   if (c.n_own <= 0) return;
   const int quads = (c.n_own + 6) / 4 + 1;
   const int blocks = (quads + 255) / 256;
-  k_combine<<<blocks, 256, 0, s>>>(c.d_g2, c.d_force, gx, gy, c.cell_begin, c.n_own, lambda, use_wa ? 1 : 0,
-                                   use_density ? 1 : 0);
+  k_combine<<<blocks, 256, 0, s>>>(c.d_g2, c.d_force, gx, gy, c.cell_begin, c.n_own, lambda,
+                                   use_density ? c.lambda_dev : nullptr, use_wa ? 1 : 0, use_density ? 1 : 0);
 }
 
 void launch_finalize_phase(const Ctx &c, int phase, float lambda, bool with_wl, bool with_energy, bool with_hpwl,
@@ -173,6 +177,7 @@ void launch_finalize_phase(const Ctx &c, int phase, float lambda, bool with_wl, 
   a.d_energy = d_energy;
   a.d_hpwl = d_hpwl;
   a.lambda = lambda;
+  a.lambda_dev = with_energy ? c.lambda_dev : nullptr;
   a.with_wl = with_wl;
   a.with_energy = with_energy;
   a.with_hpwl = with_hpwl;

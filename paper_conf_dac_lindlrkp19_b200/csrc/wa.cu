@@ -49,6 +49,7 @@ struct WaArgs {
   const float *x, *y;
   float2 *g2;
   float gamma, inv_gamma, k2;   // k2 = log2(e) / gamma
+  const float *gamma_dev;       // non-null: gamma read from device memory (GP loop, graph-replayed)
   double *part;                 // WA partial per CTA
   unsigned long long *limbs;    // HPWL limbs
   int has_w;
@@ -806,7 +807,14 @@ __device__ __forceinline__ void wa_warp_nets(const WaArgs &a, int wb) {
 
 // MODE 0: WA + gradient; 1: WA + gradient + HPWL; 2: HPWL only; 3: LSE + gradient (NEXT-3).
 template <int MODE>
-__global__ void __launch_bounds__(kWaThreads, 3) k_wa_chunks(WaArgs a) {
+__global__ void __launch_bounds__(kWaThreads, 3) k_wa_chunks(const WaArgs a0) {
+  WaArgs a = a0;
+  if (a.gamma_dev) {   // uniform branch: the GP loop's gamma lives on the device
+    const float g = __ldg(a.gamma_dev);
+    a.gamma = g;
+    a.inv_gamma = 1.f / g;
+    a.k2 = kLog2e / g;
+  }
   constexpr bool kGrad = MODE != 2;
   constexpr bool kHpwl = MODE == 1 || MODE == 2;
   extern __shared__ __align__(16) unsigned char smem[];
@@ -994,6 +1002,7 @@ void launch_wa(const Ctx &c, const float *x, const float *y, float gamma, bool h
   a.y = y;
   a.g2 = c.d_g2;
   a.gamma = gamma;
+  a.gamma_dev = c.gamma_dev;
   a.inv_gamma = 1.f / gamma;
   a.k2 = kLog2e / gamma;
   a.part = c.d_part;

@@ -347,6 +347,12 @@ def run_ours(args, rank, world, local_rank):
     lse_ms = timed(step, Ks)
     dp.dp_set_wl_model(ctx, dp.DP_WL_WA)
     step()
+    # NEXT-2: deterministic mode (exact int64 WA gradient sums)
+    dp.dp_set_deterministic(ctx, True)
+    step()
+    det_ms = timed(step, Ks)
+    dp.dp_set_deterministic(ctx, False)
+    step()
     # NEXT-1: GP iterations (Nesterov step + evaluation + schedule, one graph per iteration)
     # from the paper's initial placement, single-GPU contexts only
     gp_stats = None
@@ -387,7 +393,7 @@ def run_ours(args, rank, world, local_rank):
                  "wl_grad_only_per_s": 1e3 / wl_only_ms,
                  "profiled_ms_per_step": profiled_ms,
                  "graph_replay_evals_per_s": (1e3 / graph_ms) if isinstance(graph_ms, float) else graph_ms,
-                 "lse_evals_per_s": 1e3 / lse_ms, "gp": gp_stats,
+                 "lse_evals_per_s": 1e3 / lse_ms, "deterministic_evals_per_s": 1e3 / det_ms, "gp": gp_stats,
                  "note": "rank-0 device time of min(K, 200) back-to-back calls each; not the headline"}
     if rank != 0:
         if pg:

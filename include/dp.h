@@ -152,6 +152,15 @@ dp_status dp_wl_grad(dp_ctx *ctx, const float *x, const float *y, float gamma, f
 enum { DP_WL_WA = 0, DP_WL_LSE = 1 };
 dp_status dp_set_wl_model(dp_ctx *ctx, int32_t model);
 
+/* Deterministic mode (the paper's future work P:706): on != 0 makes the
+ * WA gradient an exact integer sum (each pin's fp32 contribution, or each chunk's exact
+ * int32 slot sum, converted to int64 in units of 2^-F, F <= 30, and added with integer
+ * atomics), so gx, gy are bit-identical from run to run and independent of stream timing.
+ * The density map is always exact (int64, 2^-29) and the force gather writes each cell once.
+ * Costs one extra 8-byte-per-coordinate accumulator pass (measured in bench.py).
+ * Errors: DP_ERR_INVALID_ARG, DP_ERR_OUT_OF_MEMORY.                                         */
+dp_status dp_set_deterministic(dp_ctx *ctx, int32_t on);
+
 /* Density only: gx, gy <- dD/dx, dD/dy; d_energy <- D.                        */
 dp_status dp_density_grad(dp_ctx *ctx, const float *x, const float *y, float *gx, float *gy,
                           double *d_energy, dp_stream_t stream);

@@ -709,7 +709,8 @@ dp_status eval_body(Ctx &c, const float *x, const float *y, float gamma, float l
 dp_status eval_graph(Ctx &c, const float *x, const float *y, float gamma, float lambda, float *gx, float *gy,
                      double *d_obj, double *d_wl, double *d_energy, double *d_hpwl, cudaStream_t s, bool do_wa,
                      bool do_den) {
-  const GraphKey key{x, y, gx, gy, d_obj, d_wl, d_energy, d_hpwl, gamma, lambda, do_wa, do_den, c.wl_model};
+  const GraphKey key{x, y, gx, gy, d_obj, d_wl, d_energy, d_hpwl, gamma, lambda, do_wa, do_den, c.wl_model,
+                     c.deterministic};
   if (!(c.gexec && key == c.gkey)) {
     cudaGraph_t g = nullptr;
     DP_CUDA(cudaStreamBeginCapture(c.s_cap, cudaStreamCaptureModeThreadLocal));
@@ -778,7 +779,11 @@ dp_status eval_body(Ctx &c, const float *x, const float *y, float gamma, float l
     {
       StageMark m(c, DP_STAGE_WA, c.s_wa);
       // clear the own-cell range of the WA gradient accumulator (read, not reset, by combine)
-      DP_CUDA(cudaMemsetAsync(c.d_g2 + c.cell_begin, 0, sizeof(float2) * (size_t)(c.cell_end - c.cell_begin), c.s_wa));
+      if (c.deterministic)
+        DP_CUDA(cudaMemsetAsync(c.d_g2i + 2 * (size_t)c.cell_begin, 0,
+                                2 * sizeof(long long) * (size_t)(c.cell_end - c.cell_begin), c.s_wa));
+      else
+        DP_CUDA(cudaMemsetAsync(c.d_g2 + c.cell_begin, 0, sizeof(float2) * (size_t)(c.cell_end - c.cell_begin), c.s_wa));
       launch_wa(c, x, y, gamma, false, d_hpwl != nullptr, c.s_wa);
     }
     DP_CUDA(cudaEventRecord(c.ev_wa, c.s_wa));
@@ -905,6 +910,18 @@ dp_status dp_set_wl_model(dp_ctx *ctx, int32_t model) {
   if (!c) return fail(DP_ERR_INVALID_ARG, "ctx is NULL");
   if (model != DP_WL_WA && model != DP_WL_LSE) return fail(DP_ERR_INVALID_ARG, "unknown wirelength model");
   c->wl_model = model;
+  return DP_OK;
+}
+
+dp_status dp_set_deterministic(dp_ctx *ctx, int32_t on) {
+  Ctx *c = C(ctx);
+  if (!c) return fail(DP_ERR_INVALID_ARG, "ctx is NULL");
+  if (on && !c->d_g2i) {
+    dp::DeviceGuard g(c->device);
+    dp_status st = dp::dev_alloc(*c, &c->d_g2i, 2 * (size_t)c->num_cells);
+    if (st != DP_OK) return st;
+  }
+  c->deterministic = on != 0;
   return DP_OK;
 }
 

@@ -79,10 +79,11 @@ struct GraphKey {
   float gamma = 0.f, lambda = 0.f;
   bool wa = false, den = false;
   int wl_model = 0;
+  bool det = false;
   bool operator==(const GraphKey &o) const {
     return x == o.x && y == o.y && gx == o.gx && gy == o.gy && obj == o.obj && wl == o.wl && en == o.en &&
            hpwl == o.hpwl && gamma == o.gamma && lambda == o.lambda && wa == o.wa && den == o.den &&
-           wl_model == o.wl_model;
+           wl_model == o.wl_model && det == o.det;
   }
 };
 
@@ -140,6 +141,9 @@ struct Ctx {
   cudaGraphExec_t gexec = nullptr;
   GraphKey gkey;
   int wl_model = 0;        // DP_WL_WA / DP_WL_LSE (dp_set_wl_model)
+  bool deterministic = false;     // dp_set_deterministic (NEXT-2): WA gradient as exact int64 sums
+  int det_frac = 30;              // its units 2^-det_frac (>= every chunk's slot scale in practice: exact shifts)
+  long long *d_g2i = nullptr;     // [2 num_cells] int64 WA gradient (allocated on first enable)
   // GP loop (gp.cu): while non-null, the evaluation kernels read gamma / lambda from these
   // device scalars instead of their by-value arguments (one captured graph per GP iteration)
   const float *gamma_dev = nullptr, *lambda_dev = nullptr;

@@ -16,6 +16,30 @@ namespace {
 // lines just loaded, measured 2.5x slower on B200); the WA stream clears it before the next
 // accumulation.  force[i] is stored with the parity offset of cell_begin (dp_create), so even
 // global cells are 16-byte aligned in both arrays.
+// Deterministic mode (NEXT-2): the WA gradient arrives as int64 in units 2^-F (exact sums).
+__global__ void __launch_bounds__(256) k_combine_det(const long long *__restrict__ g2i, int frac,
+                                                     const float2 *__restrict__ force, float *__restrict__ gx,
+                                                     float *__restrict__ gy, int cell_begin, int n_own, float lambda,
+                                                     const float *__restrict__ lambda_dev, int use_wa, int use_den) {
+  if (lambda_dev) lambda = __ldg(lambda_dev);
+  const int i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= n_own) return;
+  const int c = cell_begin + i;
+  float vx = 0.f, vy = 0.f;
+  if (use_wa) {
+    const longlong2 q = reinterpret_cast<const longlong2 *>(g2i)[c];
+    vx = (float)ldexp((double)q.x, -frac);
+    vy = (float)ldexp((double)q.y, -frac);
+  }
+  if (use_den) {
+    const float2 f = force[i];
+    vx = fmaf(lambda, f.x, vx);
+    vy = fmaf(lambda, f.y, vy);
+  }
+  gx[c] = vx;
+  gy[c] = vy;
+}
+
 __global__ void __launch_bounds__(256) k_combine(const float2 *__restrict__ g2, const float2 *__restrict__ force,
                                                  float *__restrict__ gx, float *__restrict__ gy, int cell_begin,
                                                  int n_own, float lambda, const float *__restrict__ lambda_dev,
@@ -158,6 +182,12 @@ __global__ void __launch_bounds__(256) k_finalize(FinArgs a) {
 void launch_combine(const Ctx &c, float lambda, float *gx, float *gy, bool use_wa, bool use_density,
                     cudaStream_t s) {
   if (c.n_own <= 0) return;
+  if (c.deterministic) {
+    k_combine_det<<<(c.n_own + 255) / 256, 256, 0, s>>>(c.d_g2i, c.det_frac, c.d_force, gx, gy, c.cell_begin, c.n_own,
+                                                        lambda, use_density ? c.lambda_dev : nullptr, use_wa ? 1 : 0,
+                                                        use_density ? 1 : 0);
+    return;
+  }
   const int quads = (c.n_own + 6) / 4 + 1;
   const int blocks = (quads + 255) / 256;
   k_combine<<<blocks, 256, 0, s>>>(c.d_g2, c.d_force, gx, gy, c.cell_begin, c.n_own, lambda,

@@ -48,6 +48,8 @@ struct WaArgs {
   const int32_t *far_cells;
   const float *x, *y;
   float2 *g2;
+  long long *g2i;               // deterministic mode (NEXT-2): int64 gradient in units 2^-det_frac, else null
+  int det_frac;
   float gamma, inv_gamma, k2;   // k2 = log2(e) / gamma
   const float *gamma_dev;       // non-null: gamma read from device memory (GP loop, graph-replayed)
   double *part;                 // WA partial per CTA
@@ -102,6 +104,28 @@ __device__ __forceinline__ void red_v4(float4 *p, float a, float b, float c, flo
   asm volatile("red.global.add.v4.f32 [%0], {%1, %2, %3, %4};" ::"l"(p), "f"(a), "f"(b), "f"(c),
                "f"(d)
                : "memory");
+}
+
+__device__ __forceinline__ void red_s64(long long *p, long long v) {
+  asm volatile("red.global.add.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+
+// Deterministic mode (NEXT-2): a per-pin contribution becomes an int64 in units 2^-F (one
+// rounding of the fp32 value, independent of order), summed with integer atomics: the cell
+// gradient is then bit-identical from run to run whatever the atomic order.
+template <class A>
+__device__ __forceinline__ void grad_out(const A &a, int cell, float gx, float gy) {
+  if (a.g2i) {
+    red_s64(a.g2i + 2 * cell, __double2ll_rn(ldexp((double)gx, a.det_frac)));
+    red_s64(a.g2i + 2 * cell + 1, __double2ll_rn(ldexp((double)gy, a.det_frac)));
+  } else {
+    red_v2(a.g2 + cell, gx, gy);
+  }
+}
+
+// int32 slot sum in units 2^-scale -> int64 in units 2^-F (exact when F >= scale)
+__device__ __forceinline__ long long to_det(int v, int shift) {
+  return shift >= 0 ? ((long long)v << shift) : ((long long)v >> -shift);
 }
 
 // Add h (>= 0, a multiple of 2^-149 below 2^131) to 10 int64 limbs of 32-bit digits with
@@ -640,7 +664,7 @@ __device__ __forceinline__ void wa_big_net(const WaArgs &a, int net, float4 *s_p
       const float gy = kLse ? we * (ayp * ibyp - aym * ibym)
                             : we * (ayp * ibyp * (1.f + (lyp - myp) * a.inv_gamma) -
                                     aym * ibym * (1.f - (lym - mym) * a.inv_gamma));
-      red_v2(a.g2 + raw, gx, gy);
+      grad_out(a, raw, gx, gy);
     }
   }
   __syncthreads();
@@ -737,7 +761,7 @@ __device__ __forceinline__ void wa_warp_nets(const WaArgs &a, int wb) {
         const float axp = ex2(lxp), axm = ex2(-lxm), ayp = ex2(lyp), aym = ex2(-lym);
         const float gx = kLse ? we * (axp * ibxp - axm * ibxm) : axp * fmaf(lxp, qxp, pxp) - axm * fmaf(-lxm, qxm, pxm);
         const float gy = kLse ? we * (ayp * ibyp - aym * ibym) : ayp * fmaf(lyp, qyp, pyp) - aym * fmaf(-lym, qym, pym);
-        red_v2(a.g2 + raw, gx, gy);
+        grad_out(a, raw, gx, gy);
       }
     } else {
       Ext e{-INFINITY, 0.f, INFINITY, 0.f, -INFINITY, 0.f, INFINITY, 0.f};
@@ -796,7 +820,7 @@ __device__ __forceinline__ void wa_warp_nets(const WaArgs &a, int wb) {
                                  axm * ibxm * (1.f - (lxm - mxm) * a.inv_gamma));
           const float gy = we * (ayp * ibyp * (1.f + (lyp - myp) * a.inv_gamma) -
                                  aym * ibym * (1.f - (lym - mym) * a.inv_gamma));
-          red_v2(a.g2 + raw, gx, gy);
+          grad_out(a, raw, gx, gy);
         }
       }
     }
@@ -939,7 +963,19 @@ __global__ void __launch_bounds__(kWaThreads, 3) k_wa_chunks(const WaArgs a0) {
     }
   }
   __syncthreads();
-  if (kGrad) {
+  if (kGrad && a.g2i) {   // deterministic flush: exact int32 -> int64 conversion, integer reds
+    const int sh = a.det_frac - ch.scale_log2;
+    for (int w = tid; w < ch.win_n; w += kWaThreads) {
+      const int gx = s_g[2 * w], gy = s_g[2 * w + 1];
+      if (gx) red_s64(a.g2i + 2 * (ch.win_lo + w), to_det(gx, sh));
+      if (gy) red_s64(a.g2i + 2 * (ch.win_lo + w) + 1, to_det(gy, sh));
+    }
+    for (int f = tid; f < ch.far_n; f += kWaThreads) {
+      const int gx = s_g[2 * (kWaWindow + f)], gy = s_g[2 * (kWaWindow + f) + 1];
+      if (gx) red_s64(a.g2i + 2 * s_far[f], to_det(gx, sh));
+      if (gy) red_s64(a.g2i + 2 * s_far[f] + 1, to_det(gy, sh));
+    }
+  } else if (kGrad) {
     const float inv = exp2f(-(float)ch.scale_log2);
     // window: cells [win_lo, win_lo + win_n), win_lo a multiple of 4 -> 16-byte vector reductions
     float4 *g4 = reinterpret_cast<float4 *>(a.g2 + ch.win_lo);
@@ -1001,6 +1037,8 @@ void launch_wa(const Ctx &c, const float *x, const float *y, float gamma, bool h
   a.x = x;
   a.y = y;
   a.g2 = c.d_g2;
+  a.g2i = c.deterministic ? c.d_g2i : nullptr;
+  a.det_frac = c.det_frac;
   a.gamma = gamma;
   a.gamma_dev = c.gamma_dev;
   a.inv_gamma = 1.f / gamma;

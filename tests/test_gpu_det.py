@@ -1,0 +1,96 @@
+"""Deterministic mode (dp_set_deterministic; the paper's future work P:706):
+parity with the oracle is unchanged, and the gradient (hence a whole GP trajectory) is
+bit-identical from run to run and across streams."""
+import numpy as np
+import pytest
+import torch
+
+import oracle
+import paper_conf_dac_lindlrkp19_b200 as dp
+from synth import make_netlist, make_positions
+from parity_util import check_scalar, check_vector, to_np
+
+pytestmark = pytest.mark.gpu
+DEV = torch.device("cuda", 0)
+
+
+def _t(a):
+    return torch.as_tensor(np.ascontiguousarray(a, dtype=np.float32), device=DEV)
+
+
+@pytest.mark.parametrize("dist", ["spread", "initial"])
+@pytest.mark.parametrize("model", ["wa", "lse"])
+def test_det_parity_tiny(dist, model):
+    nl = make_netlist("tiny")
+    ctx = dp.dp_create(nl)
+    dp.dp_set_deterministic(ctx, True)
+    ctx.set_wl_model(model)
+    x, y = make_positions(nl, dist)
+    out = ctx.eval(_t(x), _t(y), nl.bin_w, 0.5, with_hpwl=True)
+    ref = oracle.evaluate(nl, x, y, nl.bin_w, 0.5, wl_model=model)
+    check_scalar("WL", out["wl"].item(), ref["wl"])
+    check_scalar("obj", out["obj"].item(), ref["obj"])
+    assert out["hpwl"].item() == ref["hpwl"]
+    check_vector("gx", to_np(out["gx"]), ref["gx"])
+    check_vector("gy", to_np(out["gy"]), ref["gy"])
+
+
+def test_det_high_fanout_parity():
+    """Big nets (warp- and CTA-per-net paths) go through the per-pin int64 conversion."""
+    nl = make_netlist("tiny", extra_fanout=(150, 1030))
+    ctx = dp.dp_create(nl)
+    dp.dp_set_deterministic(ctx, True)
+    x, y = make_positions(nl)
+    out = ctx.wl_grad(_t(x), _t(y), 2 * nl.bin_w)
+    wl, gx, gy = oracle.wa(nl, x, y, np.float32(2 * nl.bin_w))
+    check_scalar("WA", out["wl"].item(), wl)
+    check_vector("gx", to_np(out["gx"]), gx)
+    check_vector("gy", to_np(out["gy"]), gy)
+
+
+@pytest.mark.parametrize("name", ["adaptec1", "bigblue4"])
+def test_det_bitwise_repeatable(name):
+    """Three evaluations (two streams) give bit-identical gradients and scalars; the
+    non-deterministic path agrees with them within the parity tolerance."""
+    nl = make_netlist(name)
+    ctx = dp.dp_create(nl)
+    x, y = make_positions(nl)
+    xt, yt = _t(x), _t(y)
+    fast = ctx.eval(xt, yt, nl.bin_w, 1.0)
+    dp.dp_set_deterministic(ctx, True)
+    outs = []
+    side = torch.cuda.Stream()
+    for k in range(3):
+        st = side if k == 1 else None
+        with torch.cuda.stream(st or torch.cuda.current_stream()):
+            o = ctx.eval(xt, yt, nl.bin_w, 1.0, stream=st)
+        torch.cuda.synchronize()
+        outs.append({k2: v.clone() for k2, v in o.items() if torch.is_tensor(v)})
+    for o in outs[1:]:
+        assert torch.equal(o["gx"], outs[0]["gx"]) and torch.equal(o["gy"], outs[0]["gy"])
+        assert torch.equal(o["scalars"][:3], outs[0]["scalars"][:3])
+    check_vector("gx det vs fast", to_np(outs[0]["gx"]), to_np(fast["gx"]))
+    check_scalar("obj det vs fast", outs[0]["obj"].item(), fast["obj"].item())
+    n_diff = int((fast["gx"] != outs[0]["gx"]).sum())
+    print(f"{name}: entries where the fp32-atomic path differs from the deterministic one: {n_diff}")
+
+
+def test_det_gp_trajectory_bitwise():
+    """The whole GP loop is deterministic in this mode: two runs from the same start give
+    bit-identical histories and positions."""
+    nl = make_netlist("tiny")
+    x, y = make_positions(nl, "initial")
+    runs = []
+    for _ in range(2):
+        ctx = dp.dp_create(nl)
+        dp.dp_set_deterministic(ctx, True)
+        loop = dp.GpLoop(ctx)
+        loop.init(_t(x), _t(y))
+        loop.run(50)
+        h = loop.history()
+        ux, uy = loop.positions()
+        runs.append((h, ux.cpu().numpy(), uy.cpu().numpy()))
+        loop.close()
+    (h0, x0, y0), (h1, x1, y1) = runs
+    assert h0 == h1
+    assert np.array_equal(x0, x1) and np.array_equal(y0, y1)

@@ -736,8 +736,10 @@ void launch_density_map(const Ctx &c, const float *x, const float *y, cudaStream
   }
   if (nblk > 0) {
     k_count<<<nblk, kCountThreads, ntiles * 4, s>>>(a);
+    if (c.sched == 3) cudaEventRecord(c.ev_sched, s);   // DP_SCHED=3: WA starts after the count
     k_scan<<<1, 1024, 0, s>>>(a);
     k_place<<<nblk, kCountThreads, place_smem_bytes(ntiles), s>>>(a);
+    if (c.sched == 2) cudaEventRecord(c.ev_sched, s);   // DP_SCHED=2: WA starts after the placement
     k_scatter_walk<<<c.walk_grid, kTileThreads, walk_smem_bytes(c.tile), s>>>(a);
   }
   if (side)

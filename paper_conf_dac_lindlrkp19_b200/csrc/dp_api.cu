@@ -495,6 +495,7 @@ void destroy(Ctx *c) {
   if (c->ev_den) cudaEventDestroy(c->ev_den);
   if (c->ev_done) cudaEventDestroy(c->ev_done);
   if (c->ev_map) cudaEventDestroy(c->ev_map);
+  if (c->ev_sched) cudaEventDestroy(c->ev_sched);
   for (cudaEvent_t e : {c->ev_aux_a, c->ev_aux_b, c->ev_join, c->ev_fin})
     if (e) cudaEventDestroy(e);
   if (c->s_aux) cudaStreamDestroy(c->s_aux);
@@ -572,7 +573,7 @@ dp_status create(const dp_netlist *nl, const dp_grid *grid, int device, int rank
   if ((st = dev_alloc(*c, &c->d_hy, 2 * (size_t)c->num_cells)) != DP_OK) return bail(st);  // x then y
   c->d_hx = nullptr;
   { const char *e = std::getenv("DP_SERIAL"); c->serial = e && e[0] == '1'; }
-  { const char *e = std::getenv("DP_SCHED"); c->sched = e ? std::atoi(e) : 1; }
+  { const char *e = std::getenv("DP_SCHED"); c->sched = e ? std::atoi(e) : 2; }
   int prio_lo = 0, prio_hi = 0;
   cudaDeviceGetStreamPriorityRange(&prio_lo, &prio_hi);
   { const char *e = std::getenv("DP_PRIO"); if (e && e[0] == '0') prio_hi = prio_lo; }   // default: density first
@@ -586,6 +587,7 @@ dp_status create(const dp_netlist *nl, const dp_grid *grid, int device, int rank
       cudaStreamCreateWithPriority(&c->s_wa, cudaStreamNonBlocking, prio_lo) != cudaSuccess ||
       cudaStreamCreateWithPriority(&c->s_den, cudaStreamNonBlocking, prio_hi) != cudaSuccess ||
       cudaEventCreateWithFlags(&c->ev_map, cudaEventDisableTiming) != cudaSuccess ||
+      cudaEventCreateWithFlags(&c->ev_sched, cudaEventDisableTiming) != cudaSuccess ||
       cudaStreamCreateWithPriority(&c->s_aux, cudaStreamNonBlocking, prio_hi) != cudaSuccess ||
       cudaEventCreateWithFlags(&c->ev_aux_a, cudaEventDisableTiming) != cudaSuccess ||
       cudaEventCreateWithFlags(&c->ev_aux_b, cudaEventDisableTiming) != cudaSuccess ||
@@ -775,7 +777,14 @@ dp_status eval_body(Ctx &c, const float *x, const float *y, float gamma, float l
   }
   if (do_wa) {
     DP_CUDA(cudaStreamWaitEvent(
-        c.s_wa, !do_den ? c.ev_fork : c.serial ? c.ev_den : c.sched == 1 ? c.ev_map : c.ev_fork, 0));
+        c.s_wa,
+        !do_den ? c.ev_fork
+        : c.serial ? c.ev_den
+        : c.sched == 1 ? c.ev_map
+        : (c.sched == 2 || c.sched == 3) && c.n_own > 0 ? c.ev_sched
+        : c.sched >= 2 ? c.ev_map
+                       : c.ev_fork,
+        0));
     {
       StageMark m(c, DP_STAGE_WA, c.s_wa);
       // clear the own-cell range of the WA gradient accumulator (read, not reset, by combine)

@@ -178,6 +178,7 @@ struct Ctx {
   cudaStream_t s_wa = nullptr, s_den = nullptr;
   cudaEvent_t ev_fork = nullptr, ev_wa = nullptr, ev_den = nullptr;
   cudaEvent_t ev_map = nullptr;
+  cudaEvent_t ev_sched = nullptr;   // DP_SCHED=2/3: WA start after the placement / the count (A/B)
   cudaStream_t s_aux = nullptr;    // large cells and the finalize, beside the main chains
   cudaEvent_t ev_aux_a = nullptr, ev_aux_b = nullptr, ev_join = nullptr, ev_fin = nullptr;    // density map complete (DP_SCHED=1 start of WA)
   cudaEvent_t ev_done = nullptr;   // end of the last call: serialises use from several streams

@@ -524,7 +524,7 @@ struct WaSmem {
   __host__ __device__ int off_py() const { return off_px() + 4 * slots(); }
   __host__ __device__ int off_g() const { return off_py() + 4 * slots(); }
   __host__ __device__ int off_bar() const { return off_g() + 8 * slots(); }
-  __host__ __device__ int bytes() const { return off_bar() + 16; }
+  __host__ __device__ int bytes() const { return off_bar() + 16; }   // two mbarriers
 };
 
 // ---------------------------------------------------------------------------------------
@@ -873,18 +873,22 @@ __global__ void __launch_bounds__(kWaThreads, 3) k_wa_chunks(const WaArgs a0) {
   // window positions by bulk copy when 16-byte aligned (the caller's x / y), else by threads
   const int wbulk = ch.win_n & ~3;
   const bool win_bulk = ((((uintptr_t)(a.x + ch.win_lo)) | ((uintptr_t)(a.y + ch.win_lo))) & 15) == 0 && wbulk > 0;
+  // two barriers: bar[0] = the far-cell list (small, issued first: the far-position gather
+  // starts while the pin records are still in flight), bar[1] = everything else
   if (tid == 0) {
     mbar_init(bar);
-    const unsigned tx = 12u * ch.pin_n + (a.has_w ? 8u : 4u) * ch.net_n + 16u * ch.wg_n + 4u * ch.far_pad +
-                        (win_bulk ? 8u * wbulk : 0u);
-    mbar_expect_tx(bar, tx);
+    mbar_init(bar + 1);
+    mbar_expect_tx(bar, 4u * ch.far_pad);
+    if (ch.far_pad) bulk_g2s(s_far, a.far_cells + ch.far_begin, 4u * ch.far_pad, bar);
+    const unsigned tx = 12u * ch.pin_n + (a.has_w ? 8u : 4u) * ch.net_n + 16u * ch.wg_n + (win_bulk ? 8u * wbulk : 0u);
+    mbar_expect_tx(bar + 1, tx);
     // the chunk's netlist data is read once per evaluation: streamed with an evict-first L2 policy
     const uint64_t pol = a.stream_hint ? l2_evict_first_policy() : 0;
     auto copy = [&](void *dst, const void *src, unsigned bytes) {
       if (a.stream_hint)
-        bulk_g2s_hint(dst, src, bytes, bar, pol);
+        bulk_g2s_hint(dst, src, bytes, bar + 1, pol);
       else
-        bulk_g2s(dst, src, bytes, bar);
+        bulk_g2s(dst, src, bytes, bar + 1);
     };
     if (ch.pin_n) {
       copy(s_slot, a.pin_slot + ch.pin_begin, 4u * ch.pin_n);
@@ -896,10 +900,9 @@ __global__ void __launch_bounds__(kWaThreads, 3) k_wa_chunks(const WaArgs a0) {
       if (a.has_w) copy(s_w, a.net_w + ch.net_begin, 4u * ch.net_n);
     }
     if (ch.wg_n) copy(s_wg, a.wgs + ch.wg_begin, 16u * ch.wg_n);
-    if (ch.far_pad) copy(s_far, a.far_cells + ch.far_begin, 4u * ch.far_pad);
     if (win_bulk) {
-      bulk_g2s(s_px, a.x + ch.win_lo, 4u * wbulk, bar);
-      bulk_g2s(s_py, a.y + ch.win_lo, 4u * wbulk, bar);
+      bulk_g2s(s_px, a.x + ch.win_lo, 4u * wbulk, bar + 1);
+      bulk_g2s(s_py, a.y + ch.win_lo, 4u * wbulk, bar + 1);
     }
   }
   const int nslots = L_.slots();
@@ -930,6 +933,7 @@ __global__ void __launch_bounds__(kWaThreads, 3) k_wa_chunks(const WaArgs a0) {
       }
     }
   }
+  mbar_wait(bar + 1, 0);
   __syncthreads();
 
   float wl_acc = 0.f;

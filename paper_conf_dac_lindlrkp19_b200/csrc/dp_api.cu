@@ -437,11 +437,6 @@ dp_status build_density(Ctx &c, const dp_netlist *nl) {
   if ((st = dev_alloc(c, &c.d_xi, nb)) != DP_OK) return st;
   if ((st = dev_alloc(c, &c.d_sxy, nb)) != DP_OK) return st;
   if ((st = dev_alloc(c, &c.d_spec, nb)) != DP_OK) return st;
-  // force[i] for own cell i = cell_begin + i; offset by the parity of cell_begin so that even
-  // global cells are 16-byte aligned (the combine pass reads cell pairs as float4)
-  if ((st = dev_alloc(c, &c.d_force, c.n_own + 4)) != DP_OK) return st;
-  DP_CUDA(cudaMemset(c.d_force, 0, sizeof(float2) * (c.n_own + 4)));
-  c.d_force += (c.cell_begin & 1);
   if ((st = dev_upload(c, &c.d_tw_x, twiddles(c.mx))) != DP_OK) return st;
   if ((st = dev_upload(c, &c.d_tw_y, twiddles(c.my))) != DP_OK) return st;
   if ((st = dev_upload(c, &c.d_ph_x, phases(c.mx))) != DP_OK) return st;
@@ -561,8 +556,18 @@ dp_status create(const dp_netlist *nl, const dp_grid *grid, int device, int rank
   }
   c->n_wa_part = c->n_chunks + c->n_huge + (c->n_big - c->n_huge + kWarpNetThreads / 32 - 1) / (kWarpNetThreads / 32);
   c->n_en_part = c->my / 2;   // = CTAs of the column-fields kernel (2-column slabs)
-  if ((st = dev_alloc(*c, &c->d_g2, c->num_cells)) != DP_OK) return bail(st);
-  if (cudaMemset(c->d_g2, 0, sizeof(float2) * c->num_cells) != cudaSuccess) return bail(fail(DP_ERR_CUDA, "memset"));
+  // one "hot" arena for the two per-cell vectors the combine reads: the WA accumulator g2
+  // [num_cells] and the force [n_own + 4] (offset by the parity of cell_begin so that even
+  // global cells are 16-byte aligned: the combine reads cell pairs as float4).  It is the
+  // L2 persisting access-policy window of the evaluation's streams (DP_L2_PERSIST=0: off).
+  {
+    const size_t g2n = ((size_t)c->num_cells + 7) & ~(size_t)7;
+    const size_t hot_n = g2n + (size_t)c->n_own + 4;
+    if ((st = dev_alloc(*c, &c->d_g2, hot_n)) != DP_OK) return bail(st);
+    if (cudaMemset(c->d_g2, 0, sizeof(float2) * hot_n) != cudaSuccess) return bail(fail(DP_ERR_CUDA, "memset"));
+    c->d_force = c->d_g2 + g2n + (c->cell_begin & 1);
+    c->hot_bytes = sizeof(float2) * hot_n;
+  }
   if ((st = dev_alloc(*c, &c->d_part, c->n_wa_part + c->n_en_part + 1)) != DP_OK) return bail(st);
   if (cudaMemset(c->d_part, 0, sizeof(double) * (c->n_wa_part + c->n_en_part + 1)) != cudaSuccess) return bail(fail(DP_ERR_CUDA, "memset"));
   if ((st = dev_alloc(*c, &c->d_limbs, kHpwlLimbs + 1)) != DP_OK) return bail(st);
@@ -583,6 +588,7 @@ dp_status create(const dp_netlist *nl, const dp_grid *grid, int device, int rank
   { const char *e = std::getenv("DP_ROW_TMA"); c->row_tma = !(e && e[0] == '0'); }
   { const char *e = std::getenv("DP_T1_TMA"); c->t1_tma = e && e[0] == '1'; }
   { const char *e = std::getenv("DP_GRAPH"); c->use_graph = !(e && e[0] == '0'); }
+  { const char *e = std::getenv("DP_L2_PERSIST"); c->l2_persist = !(e && e[0] == '0'); }
   if (cudaStreamCreateWithFlags(&c->s_cap, cudaStreamNonBlocking) != cudaSuccess ||
       cudaStreamCreateWithPriority(&c->s_wa, cudaStreamNonBlocking, prio_lo) != cudaSuccess ||
       cudaStreamCreateWithPriority(&c->s_den, cudaStreamNonBlocking, prio_hi) != cudaSuccess ||
@@ -598,6 +604,23 @@ dp_status create(const dp_netlist *nl, const dp_grid *grid, int device, int rank
       cudaEventCreateWithFlags(&c->ev_den, cudaEventDisableTiming) != cudaSuccess ||
       cudaEventCreateWithFlags(&c->ev_done, cudaEventDisableTiming) != cudaSuccess)
     return bail(fail(DP_ERR_CUDA, "stream/event creation failed"));
+  if (c->l2_persist && prop.persistingL2CacheMaxSize > 0 && prop.accessPolicyMaxWindowSize > 0) {
+    // keep g2 + force resident in L2 (WA reds, gather stores and the combine's reads hit L2)
+    const size_t setaside = std::min<size_t>((size_t)prop.persistingL2CacheMaxSize, c->hot_bytes);
+    size_t cur = 0;
+    cudaDeviceGetLimit(&cur, cudaLimitPersistingL2CacheSize);
+    if (cur < setaside) cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, setaside);
+    cudaStreamAttrValue v{};
+    v.accessPolicyWindow.base_ptr = c->d_g2;
+    v.accessPolicyWindow.num_bytes = std::min<size_t>(c->hot_bytes, (size_t)prop.accessPolicyMaxWindowSize);
+    v.accessPolicyWindow.hitRatio =
+        (float)std::min(1.0, (double)setaside / (double)v.accessPolicyWindow.num_bytes);
+    v.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
+    v.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
+    for (cudaStream_t s : {c->s_cap, c->s_wa, c->s_den, c->s_aux})
+      cudaStreamSetAttribute(s, cudaStreamAttributeAccessPolicyWindow, &v);
+    cudaGetLastError();   // best effort: a refused hint leaves the default policy
+  }
   const int wa_k = (c->n_chunks + c->n_big > 0) ? 1 : 0;   // one kernel: big nets, warp nets, chunks
   c->launches_eval = wa_k + density_launches(*c) + 3 /* T1 T2 T3 */ + 2 /* combine, finalize */;
   c->launches_eval_hpwl = c->launches_eval;

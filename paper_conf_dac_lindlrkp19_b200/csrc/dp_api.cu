@@ -430,13 +430,25 @@ dp_status build_density(Ctx &c, const dp_netlist *nl) {
   if ((st = dev_alloc(c, &c.d_rec, c.n_own + 8)) != DP_OK) return st;
   if ((st = dev_alloc(c, &c.d_rec_rc, c.n_own + 8)) != DP_OK) return st;
   if ((st = dev_alloc(c, &c.d_rec_cell, c.n_own + 8)) != DP_OK) return st;
-  if ((st = dev_alloc(c, &c.d_rho, nb)) != DP_OK) return st;
-  if ((st = dev_alloc(c, &c.d_t, nb)) != DP_OK) return st;
+  // the maps of the hot path in one arena (rho int64, t, spec, sxy, xi): the density
+  // stream's L2 persisting window (create)
+  {
+    unsigned char *arena = nullptr;
+    c.maps_bytes = nb * (sizeof(unsigned long long) + sizeof(float) + 3 * sizeof(float2));
+    if ((st = dev_alloc(c, &arena, c.maps_bytes)) != DP_OK) return st;
+    c.d_maps = arena;
+    c.d_rho = reinterpret_cast<unsigned long long *>(arena);
+    arena += nb * sizeof(unsigned long long);
+    c.d_spec = reinterpret_cast<float2 *>(arena);
+    arena += nb * sizeof(float2);
+    c.d_sxy = reinterpret_cast<float2 *>(arena);
+    arena += nb * sizeof(float2);
+    c.d_xi = reinterpret_cast<float2 *>(arena);
+    arena += nb * sizeof(float2);
+    c.d_t = reinterpret_cast<float *>(arena);
+  }
   if ((st = dev_alloc(c, &c.d_sx, nb)) != DP_OK) return st;
   if ((st = dev_alloc(c, &c.d_sy, nb)) != DP_OK) return st;
-  if ((st = dev_alloc(c, &c.d_xi, nb)) != DP_OK) return st;
-  if ((st = dev_alloc(c, &c.d_sxy, nb)) != DP_OK) return st;
-  if ((st = dev_alloc(c, &c.d_spec, nb)) != DP_OK) return st;
   if ((st = dev_upload(c, &c.d_tw_x, twiddles(c.mx))) != DP_OK) return st;
   if ((st = dev_upload(c, &c.d_tw_y, twiddles(c.my))) != DP_OK) return st;
   if ((st = dev_upload(c, &c.d_ph_x, phases(c.mx))) != DP_OK) return st;
@@ -588,7 +600,11 @@ dp_status create(const dp_netlist *nl, const dp_grid *grid, int device, int rank
   { const char *e = std::getenv("DP_ROW_TMA"); c->row_tma = !(e && e[0] == '0'); }
   { const char *e = std::getenv("DP_T1_TMA"); c->t1_tma = e && e[0] == '1'; }
   { const char *e = std::getenv("DP_GRAPH"); c->use_graph = !(e && e[0] == '0'); }
-  { const char *e = std::getenv("DP_L2_PERSIST"); c->l2_persist = !(e && e[0] == '0'); }
+  {
+    const char *e = std::getenv("DP_L2_PERSIST");
+    c->l2_persist = !(e && e[0] == '0');
+    c->l2_persist_maps = e && e[0] == '2';
+  }
   if (cudaStreamCreateWithFlags(&c->s_cap, cudaStreamNonBlocking) != cudaSuccess ||
       cudaStreamCreateWithPriority(&c->s_wa, cudaStreamNonBlocking, prio_lo) != cudaSuccess ||
       cudaStreamCreateWithPriority(&c->s_den, cudaStreamNonBlocking, prio_hi) != cudaSuccess ||
@@ -605,20 +621,29 @@ dp_status create(const dp_netlist *nl, const dp_grid *grid, int device, int rank
       cudaEventCreateWithFlags(&c->ev_done, cudaEventDisableTiming) != cudaSuccess)
     return bail(fail(DP_ERR_CUDA, "stream/event creation failed"));
   if (c->l2_persist && prop.persistingL2CacheMaxSize > 0 && prop.accessPolicyMaxWindowSize > 0) {
-    // keep g2 + force resident in L2 (WA reds, gather stores and the combine's reads hit L2)
-    const size_t setaside = std::min<size_t>((size_t)prop.persistingL2CacheMaxSize, c->hot_bytes);
+    // keep g2 + force (WA reds, gather stores, the combine's reads) and, on the density stream,
+    // the transform maps resident in L2 (DP_L2_PERSIST=1: g2 + force only, 2: both)
+    const bool maps = c->l2_persist_maps;
+    const size_t want = c->hot_bytes + (maps ? c->maps_bytes : 0);
+    const size_t setaside = std::min<size_t>((size_t)prop.persistingL2CacheMaxSize, want);
     size_t cur = 0;
     cudaDeviceGetLimit(&cur, cudaLimitPersistingL2CacheSize);
     if (cur < setaside) cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, setaside);
-    cudaStreamAttrValue v{};
-    v.accessPolicyWindow.base_ptr = c->d_g2;
-    v.accessPolicyWindow.num_bytes = std::min<size_t>(c->hot_bytes, (size_t)prop.accessPolicyMaxWindowSize);
-    v.accessPolicyWindow.hitRatio =
-        (float)std::min(1.0, (double)setaside / (double)v.accessPolicyWindow.num_bytes);
-    v.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
-    v.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
-    for (cudaStream_t s : {c->s_cap, c->s_wa, c->s_den, c->s_aux})
-      cudaStreamSetAttribute(s, cudaStreamAttributeAccessPolicyWindow, &v);
+    const float ratio = (float)std::min(1.0, (double)setaside / (double)want);
+    auto window = [&](void *base, size_t bytes) {
+      cudaStreamAttrValue v{};
+      v.accessPolicyWindow.base_ptr = base;
+      v.accessPolicyWindow.num_bytes = std::min<size_t>(bytes, (size_t)prop.accessPolicyMaxWindowSize);
+      v.accessPolicyWindow.hitRatio = ratio;
+      v.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
+      v.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
+      return v;
+    };
+    const cudaStreamAttrValue vh = window(c->d_g2, c->hot_bytes);
+    const cudaStreamAttrValue vm = window(c->d_maps, c->maps_bytes);
+    for (cudaStream_t s : {c->s_cap, c->s_wa, c->s_aux})
+      cudaStreamSetAttribute(s, cudaStreamAttributeAccessPolicyWindow, &vh);
+    cudaStreamSetAttribute(c->s_den, cudaStreamAttributeAccessPolicyWindow, maps ? &vm : &vh);
     cudaGetLastError();   // best effort: a refused hint leaves the default policy
   }
   const int wa_k = (c->n_chunks + c->n_big > 0) ? 1 : 0;   // one kernel: big nets, warp nets, chunks

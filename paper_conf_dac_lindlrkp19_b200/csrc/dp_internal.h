@@ -170,6 +170,9 @@ struct Ctx {
   float2 *d_g2 = nullptr;             // WA gradient accumulator, interleaved, cleared per call (hot arena head)
   size_t hot_bytes = 0;               // g2 + force arena (L2 persisting window)
   bool l2_persist = true;             // DP_L2_PERSIST=0: no persisting window (A/B)
+  bool l2_persist_maps = false;       // DP_L2_PERSIST=2: the density stream's window covers the maps
+  void *d_maps = nullptr;             // arena: rho, spec, sxy, xi, t
+  size_t maps_bytes = 0;
   double *d_part = nullptr;           // partial sums: [0, n_wa_part) WA, then energy
   int32_t n_wa_part = 0, n_en_part = 0;
   unsigned long long *d_limbs = nullptr;  // HPWL fixed-point limbs

@@ -45,6 +45,8 @@ def parse():
     ap.add_argument("--dist", default="spread", choices=["spread", "initial"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=200)
+    ap.add_argument("--skip-next", action="store_true",
+                    help="skip the NEXT-row secondaries (LSE, deterministic, GP loop): profiling runs")
     return ap.parse_args()
 
 
@@ -341,22 +343,24 @@ def run_ours(args, rank, world, local_rank):
     dp.dp_profile_enable(ctx, False)
     iso_ms, n_iso = dp.dp_profile_read(ctx)
     wa_iso_ms = iso_ms["wa"] / max(n_iso, 1)
-    # NEXT-3: the same evaluation with the LSE wirelength model
-    dp.dp_set_wl_model(ctx, dp.DP_WL_LSE)
-    step()
-    lse_ms = timed(step, Ks)
-    dp.dp_set_wl_model(ctx, dp.DP_WL_WA)
-    step()
-    # NEXT-2: deterministic mode (exact int64 WA gradient sums)
-    dp.dp_set_deterministic(ctx, True)
-    step()
-    det_ms = timed(step, Ks)
-    dp.dp_set_deterministic(ctx, False)
-    step()
+    lse_ms = det_ms = float("nan")
+    if not args.skip_next:
+        # NEXT-3: the same evaluation with the LSE wirelength model
+        dp.dp_set_wl_model(ctx, dp.DP_WL_LSE)
+        step()
+        lse_ms = timed(step, Ks)
+        dp.dp_set_wl_model(ctx, dp.DP_WL_WA)
+        step()
+        # NEXT-2: deterministic mode (exact int64 WA gradient sums)
+        dp.dp_set_deterministic(ctx, True)
+        step()
+        det_ms = timed(step, Ks)
+        dp.dp_set_deterministic(ctx, False)
+        step()
     # NEXT-1: GP iterations (Nesterov step + evaluation + schedule, one graph per iteration)
     # from the paper's initial placement, single-GPU contexts only
     gp_stats = None
-    if world == 1:
+    if world == 1 and not args.skip_next:
         xi, yi = make_positions(nl, "initial")
         loop = dp.GpLoop(ctx)
         loop.init(torch.as_tensor(xi, device=dev), torch.as_tensor(yi, device=dev), stream)
@@ -393,7 +397,8 @@ def run_ours(args, rank, world, local_rank):
                  "wl_grad_only_per_s": 1e3 / wl_only_ms,
                  "profiled_ms_per_step": profiled_ms,
                  "graph_replay_evals_per_s": (1e3 / graph_ms) if isinstance(graph_ms, float) else graph_ms,
-                 "lse_evals_per_s": 1e3 / lse_ms, "deterministic_evals_per_s": 1e3 / det_ms, "gp": gp_stats,
+                 "lse_evals_per_s": None if args.skip_next else 1e3 / lse_ms,
+                 "deterministic_evals_per_s": None if args.skip_next else 1e3 / det_ms, "gp": gp_stats,
                  "note": "rank-0 device time of min(K, 200) back-to-back calls each; not the headline"}
     if rank != 0:
         if pg:

@@ -58,7 +58,16 @@ struct DenArgs {
   const float2 *xi;
   float2 *force;
   const int *large;
+  // direct output (DP_DIRECT): the gather adds lambda * dD/dx straight into the caller's gx, gy
+  // (zeroed at the head of the call, the WA kernel adds into them too) instead of storing force
+  float *gxo, *gyo;
+  float lambda;
+  const float *lambda_dev;
 };
+
+__device__ __forceinline__ void red_f32(float *p, float v) {
+  asm volatile("red.global.add.f32 [%0], %1;" ::"l"(p), "f"(v) : "memory");
+}
 
 // Stretched, clipped footprint of a cell in BIN units (readings A10, A11):
 //   lo = (x - xl)/b_x + (w - w')/2 / b_x, hi = lo + w'/b_x, clipped to [0, M].
@@ -548,6 +557,7 @@ __global__ void __launch_bounds__(kTileThreads) k_gather_walk(DenArgs a) {
   int cur_tile = -1;
   unsigned xi_phase = 0;
   const float area = (float)(a.bx * a.by);
+  const float lam = a.lambda_dev ? __ldg(a.lambda_dev) : a.lambda;
   for (int c = 0;; c++) {
     const int b = c % kStages;
     const WalkChunk cc = walk_next(a, w, st, c, true);
@@ -582,7 +592,13 @@ __global__ void __launch_bounds__(kTileThreads) k_gather_walk(DenArgs a) {
         fy = fmaf(ox3[di], sy, fy);
       }
       // dD/dx = - r sum_b ov(i,b) xi^X_b  (reading A21), ov in length^2
-      a.force[B.cell[cc.off + k]] = make_float2(-area * r * fx, -area * r * fy);
+      if (a.gxo) {
+        const int gc = a.cell_begin + B.cell[cc.off + k];
+        red_f32(a.gxo + gc, lam * (-area * r * fx));
+        red_f32(a.gyo + gc, lam * (-area * r * fy));
+      } else {
+        a.force[B.cell[cc.off + k]] = make_float2(-area * r * fx, -area * r * fy);
+      }
     }
     walk_release(st, c);
   }
@@ -643,7 +659,14 @@ __global__ void __launch_bounds__(256) k_gather_large(DenArgs a) {
       ty += s_y[w];
     }
     const double area = a.bx * a.by;   // overlaps above are in bin units
-    a.force[i] = make_float2((float)(-(double)f.r * area * tx), (float)(-(double)f.r * area * ty));
+    const float2 v = make_float2((float)(-(double)f.r * area * tx), (float)(-(double)f.r * area * ty));
+    if (a.gxo) {
+      const float lam = a.lambda_dev ? __ldg(a.lambda_dev) : a.lambda;
+      red_f32(a.gxo + a.cell_begin + i, lam * v.x);
+      red_f32(a.gyo + a.cell_begin + i, lam * v.y);
+    } else {
+      a.force[i] = v;
+    }
   }
 }
 
@@ -689,6 +712,10 @@ DenArgs make_args(const Ctx &c, const float *x, const float *y) {
   a.rho = c.d_rho;
   a.xi = c.d_xi;
   a.force = c.d_force;
+  a.gxo = c.direct_gx;
+  a.gyo = c.direct_gy;
+  a.lambda = c.direct_lambda;
+  a.lambda_dev = c.lambda_dev;
   a.large = c.d_large;
   return a;
 }

@@ -600,6 +600,7 @@ dp_status create(const dp_netlist *nl, const dp_grid *grid, int device, int rank
   { const char *e = std::getenv("DP_ROW_TMA"); c->row_tma = !(e && e[0] == '0'); }
   { const char *e = std::getenv("DP_T1_TMA"); c->t1_tma = e && e[0] == '1'; }
   { const char *e = std::getenv("DP_GRAPH"); c->use_graph = !(e && e[0] == '0'); }
+  { const char *e = std::getenv("DP_DIRECT"); c->direct = e && e[0] == '1'; }
   {
     const char *e = std::getenv("DP_L2_PERSIST");
     c->l2_persist = !(e && e[0] == '0');
@@ -816,9 +817,23 @@ dp_status eval_body(Ctx &c, const float *x, const float *y, float gamma, float l
                     bool do_den) {
   StageMark whole(c, DP_STAGE_EVAL, s);
   if (c.profiling) c.prof_evals++;
+  // direct output (DP_DIRECT=1): both chains add into gx, gy, which are zeroed first; no combine
+  const bool direct = c.direct && !c.deterministic && !c.dist && ((((uintptr_t)gx) | ((uintptr_t)gy)) & 15) == 0;
+  struct DirectReset {
+    Ctx &c;
+    ~DirectReset() { c.direct_gx = c.direct_gy = nullptr; }
+  } direct_reset{c};
+  c.direct_gx = direct ? gx : nullptr;
+  c.direct_gy = direct ? gy : nullptr;
+  c.direct_lambda = lambda;
+  const size_t gbytes = sizeof(float) * (size_t)c.num_cells;
   DP_CUDA(cudaEventRecord(c.ev_fork, s));
   if (do_den) {
     DP_CUDA(cudaStreamWaitEvent(c.s_den, c.ev_fork, 0));
+    if (direct) {   // before the count: the WA stream starts after the placement (DP_SCHED=2)
+      DP_CUDA(cudaMemsetAsync(gx, 0, gbytes, c.s_den));
+      DP_CUDA(cudaMemsetAsync(gy, 0, gbytes, c.s_den));
+    }
     dp_status st = density_chain(c, x, y);
     if (st != DP_OK) return st;
     DP_CUDA(cudaEventRecord(c.ev_den, c.s_den));
@@ -836,7 +851,14 @@ dp_status eval_body(Ctx &c, const float *x, const float *y, float gamma, float l
     {
       StageMark m(c, DP_STAGE_WA, c.s_wa);
       // clear the own-cell range of the WA gradient accumulator (read, not reset, by combine)
-      if (c.deterministic)
+      if (direct) {
+        if (!do_den) {
+          DP_CUDA(cudaMemsetAsync(gx, 0, gbytes, c.s_wa));
+          DP_CUDA(cudaMemsetAsync(gy, 0, gbytes, c.s_wa));
+        } else if (c.sched < 2 || c.serial) {
+          return fail(DP_ERR_UNSUPPORTED, "DP_DIRECT needs DP_SCHED >= 2");
+        }
+      } else if (c.deterministic)
         DP_CUDA(cudaMemsetAsync(c.d_g2i + 2 * (size_t)c.cell_begin, 0,
                                 2 * sizeof(long long) * (size_t)(c.cell_end - c.cell_begin), c.s_wa));
       else
@@ -860,7 +882,7 @@ dp_status eval_body(Ctx &c, const float *x, const float *y, float gamma, float l
           finalize(c, lambda, do_wa, do_den, do_wa && d_hpwl != nullptr, d_obj, d_wl, d_energy, d_hpwl, c.s_aux);
       if (st != DP_OK) return st;
       DP_CUDA(cudaEventRecord(c.ev_fin, c.s_aux));
-      launch_combine(c, do_den ? lambda : 0.f, gx, gy, do_wa, do_den, s);
+      if (!direct) launch_combine(c, do_den ? lambda : 0.f, gx, gy, do_wa, do_den, s);
       DP_CUDA(cudaStreamWaitEvent(s, c.ev_fin, 0));
     }
   }

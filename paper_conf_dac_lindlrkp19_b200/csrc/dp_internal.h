@@ -142,6 +142,9 @@ struct Ctx {
   GraphKey gkey;
   int wl_model = 0;        // DP_WL_WA / DP_WL_LSE (dp_set_wl_model)
   bool deterministic = false;     // dp_set_deterministic (NEXT-2): WA gradient as exact int64 sums
+  bool direct = false;            // DP_DIRECT=1: WA and gather add into the caller's gx, gy (no combine pass)
+  float *direct_gx = nullptr, *direct_gy = nullptr;   // set for the duration of one eval_body
+  float direct_lambda = 0.f;
   int det_frac = 30;              // its units 2^-det_frac (>= every chunk's slot scale in practice: exact shifts)
   long long *d_g2i = nullptr;     // [2 num_cells] int64 WA gradient (allocated on first enable)
   // GP loop (gp.cu): while non-null, the evaluation kernels read gamma / lambda from these

@@ -48,6 +48,8 @@ struct GpArgs {
   double target;
   double *part;            // [nblk][2]
   int nblk;
+  double *part_ovf;        // [oblk][2] overflow partials of k_gp_post
+  int oblk;
   GpDev *dev;
   const double *out;       // eval outputs {obj, wl, energy, hpwl}
   double *hist;
@@ -110,13 +112,29 @@ __global__ void __launch_bounds__(kGpThreads) k_gp_partials(GpArgs a, int mode) 
   block_pair(s0, s1, a.part);
 }
 
-__device__ __forceinline__ void sum_parts(const GpArgs &a, double &t0, double &t1) {
-  t0 = 0.0;
-  t1 = 0.0;
-  for (int b = 0; b < a.nblk; b++) {
-    t0 += a.part[2 * b];
-    t1 += a.part[2 * b + 1];
+// Fixed-order block reduction of n (x, y) partial pairs (every thread of the block calls it;
+// the result is valid in all threads).  Thread t sums pairs t, t + T, ... in order, then a
+// fixed shared-memory tree: deterministic, and far shorter than one thread walking the list.
+__device__ __forceinline__ void sum_parts(const double *part, int n, double &t0, double &t1) {
+  __shared__ double s0[kGpThreads], s1[kGpThreads];
+  double a0 = 0.0, a1 = 0.0;
+  for (int b = threadIdx.x; b < n; b += kGpThreads) {
+    a0 += part[2 * b];
+    a1 += part[2 * b + 1];
   }
+  s0[threadIdx.x] = a0;
+  s1[threadIdx.x] = a1;
+  __syncthreads();
+  for (int o = kGpThreads / 2; o > 0; o >>= 1) {
+    if ((int)threadIdx.x < o) {
+      s0[threadIdx.x] += s0[threadIdx.x + o];
+      s1[threadIdx.x] += s1[threadIdx.x + o];
+    }
+    __syncthreads();
+  }
+  t0 = s0[0];
+  t1 = s1[0];
+  __syncthreads();
 }
 
 __device__ __forceinline__ double gamma_of(const GpArgs &a, double tau) {   // A31
@@ -126,25 +144,31 @@ __device__ __forceinline__ double gamma_of(const GpArgs &a, double tau) {   // A
 enum { S_ALPHA = 0, S_ITER_END = 1, S_INIT_TAU = 2, S_INIT_L1D = 3, S_INIT_LAMBDA = 4, S_INIT_ETA = 5,
        S_INIT_DONE = 6 };
 
-// Scalar steps of the schedule (one thread; partials summed in a fixed order).
-__global__ void k_gp_scalar(GpArgs a, int op) {
-  if (threadIdx.x != 0 || blockIdx.x != 0) return;
+// A28: Lipschitz step prediction from the norms (t0 = |v - vp|^2, t1 = |g - gp|^2) and the
+// Nesterov coefficient for the next update
+__device__ __forceinline__ void step_scalars(GpDev &d, double t0, double t1) {
+  const double num = sqrt(t0), den = sqrt(t1);
+  if (den > 0.0) d.alpha = num / den;
+  const double an = (1.0 + sqrt(4.0 * d.a * d.a + 1.0)) / 2.0;
+  d.coef = (d.a - 1.0) / an;
+  d.a = an;
+  d.f_alpha = (float)d.alpha;
+  d.f_coef = (float)d.coef;
+}
+
+// Scalar steps of the schedule (one block; partials summed in a fixed order, thread 0 writes).
+__global__ void __launch_bounds__(kGpThreads) k_gp_scalar(GpArgs a, int op) {
   GpDev &d = *a.dev;
-  double t0, t1;
-  sum_parts(a, t0, t1);
+  double t0, t1, o0 = 0.0, o1 = 0.0;
+  sum_parts(a.part, a.nblk, t0, t1);
+  if (op == S_ITER_END) sum_parts(a.part_ovf, a.oblk, o0, o1);
+  if (threadIdx.x != 0) return;
   switch (op) {
-    case S_ALPHA: {   // A28: Lipschitz step prediction and the Nesterov coefficient
-      const double num = sqrt(t0), den = sqrt(t1);
-      if (den > 0.0) d.alpha = num / den;
-      const double an = (1.0 + sqrt(4.0 * d.a * d.a + 1.0)) / 2.0;
-      d.coef = (d.a - 1.0) / an;
-      d.a = an;
-      d.f_alpha = (float)d.alpha;
-      d.f_coef = (float)d.coef;
+    case S_ALPHA:
+      step_scalars(d, t0, t1);
       break;
-    }
-    case S_ITER_END: {   // A30 overflow, eq (18) lambda, A31 gamma, history row
-      const double tau = t0 * a.bxby / d.area_total;
+    case S_ITER_END: {   // A30 overflow, eq (18) lambda, A31 gamma, history row; then A28 for the next step
+      const double tau = o0 * a.bxby / d.area_total;
       const double hp = a.out[3];
       const double p = (hp - d.hpwl) / a.dhpwl_ref;
       const double mu = p < 0.0 ? a.mu_max * fmax(pow(0.9999, (double)d.k), 0.98)
@@ -161,6 +185,7 @@ __global__ void k_gp_scalar(GpArgs a, int op) {
       d.k += 1;
       d.f_gamma = (float)d.gamma;
       d.f_lambda = (float)d.lam;
+      step_scalars(d, t0, t1);
       break;
     }
     case S_INIT_TAU:
@@ -216,6 +241,42 @@ __global__ void __launch_bounds__(kGpThreads) k_gp_precond(GpArgs a) {
   const float inv = 1.f / fmaxf(1.f, fmaf(lam, a.w[i] * a.h[i], a.pins[i]));
   a.gx[i] = a.rgx[i] * inv;
   a.gy[i] = a.rgy[i] * inv;
+}
+
+// After the evaluation at v: blocks [0, nblk) precondition (A29) and form the Lipschitz norms
+// |v - vp|^2, |g - gp|^2 of the next step (grid-stride, fixed order); blocks [nblk, nblk + oblk)
+// form the overflow partials (A30) from the evaluation's bin map.
+__global__ void __launch_bounds__(kGpThreads) k_gp_post(GpArgs a) {
+  double s0 = 0.0, s1 = 0.0;
+  if ((int)blockIdx.x < a.nblk) {
+    const float lam = a.dev->f_lambda;
+    for (int i = blockIdx.x * kGpThreads + threadIdx.x; i < a.n; i += a.nblk * kGpThreads) {
+      const float inv = 1.f / fmaxf(1.f, fmaf(lam, a.w[i] * a.h[i], a.pins[i]));
+      const float gx = a.rgx[i] * inv, gy = a.rgy[i] * inv;
+      a.gx[i] = gx;
+      a.gy[i] = gy;
+      const double dx = (double)a.vx[i] - a.vpx[i], dy = (double)a.vy[i] - a.vpy[i];
+      const double ex = (double)gx - a.gpx[i], ey = (double)gy - a.gpy[i];
+      s0 += dx * dx + dy * dy;
+      s1 += ex * ex + ey * ey;
+    }
+    block_pair(s0, s1, a.part);
+  } else {
+    const int b0 = blockIdx.x - a.nblk;
+    for (long long b = (long long)b0 * kGpThreads + threadIdx.x; b < a.nbins; b += (long long)a.oblk * kGpThreads)
+      s0 += fmax((double)a.rho[b] * a.rho_unit - a.target, 0.0);
+    __shared__ double r0[kGpThreads / 32];
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) s0 += __shfl_xor_sync(0xffffffffu, s0, o);
+    if ((threadIdx.x & 31) == 0) r0[threadIdx.x >> 5] = s0;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      double t = 0.0;
+      for (int w = 0; w < kGpThreads / 32; w++) t += r0[w];
+      a.part_ovf[2 * b0] = t;
+      a.part_ovf[2 * b0 + 1] = 0.0;
+    }
+  }
 }
 
 // init helpers: u = v = clamp(x0); vp = v - eta g
@@ -287,7 +348,7 @@ struct GpDeviceGuard {
 };
 
 void partials(Gp &g, int mode, cudaStream_t s) { k_gp_partials<<<g.a.nblk, kGpThreads, 0, s>>>(g.a, mode); }
-void scalar(Gp &g, int op, cudaStream_t s) { k_gp_scalar<<<1, 32, 0, s>>>(g.a, op); }
+void scalar(Gp &g, int op, cudaStream_t s) { k_gp_scalar<<<1, kGpThreads, 0, s>>>(g.a, op); }
 
 // evaluation at (x, y) -> raw gradient rg; gamma / lambda from the device unless given
 dp_status gp_eval(Gp &g, const float *x, const float *y, bool wa, bool den, bool dev_scalars, cudaStream_t s) {
@@ -301,16 +362,15 @@ dp_status gp_eval(Gp &g, const float *x, const float *y, bool wa, bool den, bool
   return st;
 }
 
-// one GP iteration (the captured body)
+// one GP iteration (the captured body): the step with alpha_k / coef from the previous scalar
+// pass, the evaluation at v_{k+1}, one fused pass (preconditioner, next step's norms, overflow
+// partials), one scalar pass (eq 18, gamma, history, alpha_{k+1}, a_{k+2})
 dp_status gp_iteration(Gp &g, cudaStream_t s) {
   const int cb = g.cell_blocks;
-  partials(g, R_NORMS, s);
-  scalar(g, S_ALPHA, s);
   k_gp_update<<<cb, kGpThreads, 0, s>>>(g.a);
   dp_status st = gp_eval(g, g.a.vx, g.a.vy, true, true, true, s);
   if (st != DP_OK) return st;
-  k_gp_precond<<<cb, kGpThreads, 0, s>>>(g.a);
-  partials(g, R_OVF, s);
+  k_gp_post<<<g.a.nblk + g.a.oblk, kGpThreads, 0, s>>>(g.a);
   scalar(g, S_ITER_END, s);
   DP_CUDA(cudaGetLastError());
   return DP_OK;
@@ -379,6 +439,8 @@ dp_status dp_gp_create(dp_ctx *ctx, const dp_gp_params *params, dp_gp **out) {
   a.hist_cap = p.max_history;
   dp_status st;
   if ((st = dp::gp_alloc(*g, &a.part, 2 * (size_t)a.nblk)) != DP_OK) return bail(st);
+  a.oblk = c->num_sms;
+  if ((st = dp::gp_alloc(*g, &a.part_ovf, 2 * (size_t)a.oblk)) != DP_OK) return bail(st);
   if ((st = dp::gp_alloc(*g, &g->dev, 1)) != DP_OK) return bail(st);
   if ((st = dp::gp_alloc(*g, &g->out, 4)) != DP_OK) return bail(st);
   if ((st = dp::gp_alloc(*g, &a.hist, (size_t)std::max(1, p.max_history) * dp::kHistCols)) != DP_OK) return bail(st);
@@ -449,6 +511,8 @@ dp_status dp_gp_init(dp_gp *gp, const float *x0, const float *y0, dp_stream_t st
   std::swap(a.vx, a.vpx); std::swap(a.vy, a.vpy); std::swap(a.gx, a.gpx); std::swap(a.gy, a.gpy);
   if (st != DP_OK) return st;
   dp::scalar(*g, dp::S_INIT_DONE, s);
+  dp::partials(*g, dp::R_NORMS, s);   // alpha_0, a_1 and the first Nesterov coefficient (A28)
+  dp::scalar(*g, dp::S_ALPHA, s);
   DP_CUDA(cudaGetLastError());
   g->initialised = true;
   return dp::ctx_call_end(c, s);

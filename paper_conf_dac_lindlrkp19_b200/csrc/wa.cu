@@ -49,6 +49,7 @@ struct WaArgs {
   const float *x, *y;
   float2 *g2;
   long long *g2i;               // deterministic mode (NEXT-2): int64 gradient in units 2^-det_frac, else null
+  float *gxo, *gyo;             // direct output (DP_DIRECT): add into the caller's gx, gy (16-byte aligned)
   int det_frac;
   float gamma, inv_gamma, k2;   // k2 = log2(e) / gamma
   const float *gamma_dev;       // non-null: gamma read from device memory (GP loop, graph-replayed)
@@ -106,6 +107,10 @@ __device__ __forceinline__ void red_v4(float4 *p, float a, float b, float c, flo
                : "memory");
 }
 
+__device__ __forceinline__ void red_f1(float *p, float v) {
+  asm volatile("red.global.add.f32 [%0], %1;" ::"l"(p), "f"(v) : "memory");
+}
+
 __device__ __forceinline__ void red_s64(long long *p, long long v) {
   asm volatile("red.global.add.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }
@@ -118,6 +123,9 @@ __device__ __forceinline__ void grad_out(const A &a, int cell, float gx, float g
   if (a.g2i) {
     red_s64(a.g2i + 2 * cell, __double2ll_rn(ldexp((double)gx, a.det_frac)));
     red_s64(a.g2i + 2 * cell + 1, __double2ll_rn(ldexp((double)gy, a.det_frac)));
+  } else if (a.gxo) {
+    red_f1(a.gxo + cell, gx);
+    red_f1(a.gyo + cell, gy);
   } else {
     red_v2(a.g2 + cell, gx, gy);
   }
@@ -980,6 +988,27 @@ __global__ void __launch_bounds__(kWaThreads, 3) k_wa_chunks(const WaArgs a0) {
       if (gx) red_s64(a.g2i + 2 * s_far[f], to_det(gx, sh));
       if (gy) red_s64(a.g2i + 2 * s_far[f] + 1, to_det(gy, sh));
     }
+  } else if (kGrad && a.gxo) {   // direct output: 4-cell vector reds into gx and gy (win_lo % 4 == 0)
+    const float inv = exp2f(-(float)ch.scale_log2);
+    const int nq = ch.win_n >> 2;
+    const int4 *s4 = reinterpret_cast<const int4 *>(s_g);
+    for (int q = tid; q < nq; q += kWaThreads) {
+      const int4 v0 = s4[2 * q], v1 = s4[2 * q + 1];   // x0 y0 x1 y1 | x2 y2 x3 y3
+      const int c0 = ch.win_lo + 4 * q;
+      if (v0.x | v0.z | v1.x | v1.z)
+        red_v4(reinterpret_cast<float4 *>(a.gxo + c0), v0.x * inv, v0.z * inv, v1.x * inv, v1.z * inv);
+      if (v0.y | v0.w | v1.y | v1.w)
+        red_v4(reinterpret_cast<float4 *>(a.gyo + c0), v0.y * inv, v0.w * inv, v1.y * inv, v1.w * inv);
+    }
+    for (int w = 4 * nq + tid; w < ch.win_n; w += kWaThreads) {
+      if (s_g[2 * w]) red_f1(a.gxo + ch.win_lo + w, s_g[2 * w] * inv);
+      if (s_g[2 * w + 1]) red_f1(a.gyo + ch.win_lo + w, s_g[2 * w + 1] * inv);
+    }
+    for (int f = tid; f < ch.far_n; f += kWaThreads) {
+      const int gx = s_g[2 * (kWaWindow + f)], gy = s_g[2 * (kWaWindow + f) + 1];
+      if (gx) red_f1(a.gxo + s_far[f], gx * inv);
+      if (gy) red_f1(a.gyo + s_far[f], gy * inv);
+    }
   } else if (kGrad) {
     const float inv = exp2f(-(float)ch.scale_log2);
     // window: cells [win_lo, win_lo + win_n), win_lo a multiple of 4 -> 16-byte vector reductions
@@ -1043,6 +1072,8 @@ void launch_wa(const Ctx &c, const float *x, const float *y, float gamma, bool h
   a.y = y;
   a.g2 = c.d_g2;
   a.g2i = c.deterministic ? c.d_g2i : nullptr;
+  a.gxo = c.direct_gx;
+  a.gyo = c.direct_gy;
   a.det_frac = c.det_frac;
   a.gamma = gamma;
   a.gamma_dev = c.gamma_dev;

@@ -225,6 +225,7 @@ template <class IN, int LOGN>
 __global__ void __launch_bounds__(32 * kWRowWarps) k_row_dct_w(const IN *__restrict__ in, float *__restrict__ out,
                                                              const float2 *__restrict__ tw2,
                                                              const float2 *__restrict__ ph, int npairs, int tma) {
+  griddep_wait();
   constexpr int N = 1 << LOGN, K = N / 32, B = wfft::kPts / N;
   extern __shared__ float2 wsm[];
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -298,6 +299,7 @@ __global__ void __launch_bounds__(32 * kWRowWarps) k_row_dct_w(const IN *__restr
 // 32-byte sectors at WARPS = 4), instead of one 8-byte store per lane and row.
 template <int LOGN, int WARPS = kWRowWarps, bool TSTORE = false>
 __global__ void __launch_bounds__(32 * WARPS) k_row_inv_w(RowInvArgs a, const float2 *__restrict__ tw2, int rows) {
+  griddep_wait();
   constexpr int N = 1 << LOGN, K = N / 32, B = wfft::kPts / N;
   extern __shared__ float2 wsm[];
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -559,6 +561,7 @@ constexpr int kWColWarps = 2;
 template <int LOGM>
 __global__ void __launch_bounds__(32 * kWColWarps) k_col_fwd_w(ColFieldArgs a, float2 *__restrict__ specT,
                                                              const float2 *__restrict__ tw2) {
+  griddep_wait();
   constexpr int M = 1 << LOGM, K = M / 32, B = wfft::kPts / M;
   extern __shared__ float2 wsm[];
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -623,6 +626,7 @@ __global__ void __launch_bounds__(32 * kWColWarps) k_col_fwd_w(ColFieldArgs a, f
 template <int LOGM>
 __global__ void __launch_bounds__(32 * kWColWarps) k_col_fields_w(ColFieldArgs a, float2 *__restrict__ sxy,
                                                                 const float2 *__restrict__ tw2) {
+  griddep_wait();
   constexpr int M = 1 << LOGM, K = M / 32, B = wfft::kPts / M;
   extern __shared__ float2 wsm[];
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -770,24 +774,24 @@ void row_inv(const Ctx &c, const float *inA, long long stepA, int opA, const flo
     const int g = (rows + per_cta - 1) / per_cta;
     const size_t sm = (size_t)W * wfft::kBufPad * sizeof(float2);
     switch (log2n) {
-      case 5: k_row_inv_w<5, W, true><<<g, 32 * W, sm, s>>>(a, tw2, rows); break;
-      case 6: k_row_inv_w<6, W, true><<<g, 32 * W, sm, s>>>(a, tw2, rows); break;
-      case 7: k_row_inv_w<7, W, true><<<g, 32 * W, sm, s>>>(a, tw2, rows); break;
-      case 8: k_row_inv_w<8, W, true><<<g, 32 * W, sm, s>>>(a, tw2, rows); break;
-      case 9: k_row_inv_w<9, W, true><<<g, 32 * W, sm, s>>>(a, tw2, rows); break;
-      default: k_row_inv_w<10, W, true><<<g, 32 * W, sm, s>>>(a, tw2, rows); break;
+      case 5: launch_chain(c.pdl, k_row_inv_w<5, W, true>, g, 32 * W, sm, s, a, tw2, rows); break;
+      case 6: launch_chain(c.pdl, k_row_inv_w<6, W, true>, g, 32 * W, sm, s, a, tw2, rows); break;
+      case 7: launch_chain(c.pdl, k_row_inv_w<7, W, true>, g, 32 * W, sm, s, a, tw2, rows); break;
+      case 8: launch_chain(c.pdl, k_row_inv_w<8, W, true>, g, 32 * W, sm, s, a, tw2, rows); break;
+      case 9: launch_chain(c.pdl, k_row_inv_w<9, W, true>, g, 32 * W, sm, s, a, tw2, rows); break;
+      default: launch_chain(c.pdl, k_row_inv_w<10, W, true>, g, 32 * W, sm, s, a, tw2, rows); break;
     }
     return;
   }
   const int g = wrow_ctas(rows, log2n);
   const size_t sm = wrow_smem();
   switch (log2n) {
-    case 5: k_row_inv_w<5><<<g, 32 * kWRowWarps, sm, s>>>(a, tw2, rows); break;
-    case 6: k_row_inv_w<6><<<g, 32 * kWRowWarps, sm, s>>>(a, tw2, rows); break;
-    case 7: k_row_inv_w<7><<<g, 32 * kWRowWarps, sm, s>>>(a, tw2, rows); break;
-    case 8: k_row_inv_w<8><<<g, 32 * kWRowWarps, sm, s>>>(a, tw2, rows); break;
-    case 9: k_row_inv_w<9><<<g, 32 * kWRowWarps, sm, s>>>(a, tw2, rows); break;
-    default: k_row_inv_w<10><<<g, 32 * kWRowWarps, sm, s>>>(a, tw2, rows); break;
+    case 5: launch_chain(c.pdl, k_row_inv_w<5>, g, 32 * kWRowWarps, sm, s, a, tw2, rows); break;
+    case 6: launch_chain(c.pdl, k_row_inv_w<6>, g, 32 * kWRowWarps, sm, s, a, tw2, rows); break;
+    case 7: launch_chain(c.pdl, k_row_inv_w<7>, g, 32 * kWRowWarps, sm, s, a, tw2, rows); break;
+    case 8: launch_chain(c.pdl, k_row_inv_w<8>, g, 32 * kWRowWarps, sm, s, a, tw2, rows); break;
+    case 9: launch_chain(c.pdl, k_row_inv_w<9>, g, 32 * kWRowWarps, sm, s, a, tw2, rows); break;
+    default: launch_chain(c.pdl, k_row_inv_w<10>, g, 32 * kWRowWarps, sm, s, a, tw2, rows); break;
   }
 }
 
@@ -801,12 +805,12 @@ void row_dct(const Ctx &c, const IN *in, float *out, cudaStream_t s) {
   const int np = c.mx / 2, g = wrow_ctas(np, c.log2my);
   const size_t sm = c.t1_tma ? wrow_dct_smem() : wrow_smem();
   switch (c.log2my) {
-    case 5: k_row_dct_w<IN, 5><<<g, 32 * kWRowWarps, sm, s>>>(in, out, c.d_tw2_y, c.d_ph_y, np, c.t1_tma ? 1 : 0); break;
-    case 6: k_row_dct_w<IN, 6><<<g, 32 * kWRowWarps, sm, s>>>(in, out, c.d_tw2_y, c.d_ph_y, np, c.t1_tma ? 1 : 0); break;
-    case 7: k_row_dct_w<IN, 7><<<g, 32 * kWRowWarps, sm, s>>>(in, out, c.d_tw2_y, c.d_ph_y, np, c.t1_tma ? 1 : 0); break;
-    case 8: k_row_dct_w<IN, 8><<<g, 32 * kWRowWarps, sm, s>>>(in, out, c.d_tw2_y, c.d_ph_y, np, c.t1_tma ? 1 : 0); break;
-    case 9: k_row_dct_w<IN, 9><<<g, 32 * kWRowWarps, sm, s>>>(in, out, c.d_tw2_y, c.d_ph_y, np, c.t1_tma ? 1 : 0); break;
-    default: k_row_dct_w<IN, 10><<<g, 32 * kWRowWarps, sm, s>>>(in, out, c.d_tw2_y, c.d_ph_y, np, c.t1_tma ? 1 : 0); break;
+    case 5: launch_chain(c.pdl, k_row_dct_w<IN, 5>, g, 32 * kWRowWarps, sm, s, in, out, c.d_tw2_y, c.d_ph_y, np, c.t1_tma ? 1 : 0); break;
+    case 6: launch_chain(c.pdl, k_row_dct_w<IN, 6>, g, 32 * kWRowWarps, sm, s, in, out, c.d_tw2_y, c.d_ph_y, np, c.t1_tma ? 1 : 0); break;
+    case 7: launch_chain(c.pdl, k_row_dct_w<IN, 7>, g, 32 * kWRowWarps, sm, s, in, out, c.d_tw2_y, c.d_ph_y, np, c.t1_tma ? 1 : 0); break;
+    case 8: launch_chain(c.pdl, k_row_dct_w<IN, 8>, g, 32 * kWRowWarps, sm, s, in, out, c.d_tw2_y, c.d_ph_y, np, c.t1_tma ? 1 : 0); break;
+    case 9: launch_chain(c.pdl, k_row_dct_w<IN, 9>, g, 32 * kWRowWarps, sm, s, in, out, c.d_tw2_y, c.d_ph_y, np, c.t1_tma ? 1 : 0); break;
+    default: launch_chain(c.pdl, k_row_dct_w<IN, 10>, g, 32 * kWRowWarps, sm, s, in, out, c.d_tw2_y, c.d_ph_y, np, c.t1_tma ? 1 : 0); break;
   }
 }
 
@@ -888,23 +892,23 @@ void fields_after_t1(const Ctx &c, cudaStream_t s) {
     if (c.fused_t2) {   // measured slower at 1024^2 (longer per-warp latency chain); kept for A/B
       const size_t sm = col_fields_w_smem();
       switch (c.log2mx) {   // T2: DCT_x, scaling, energy, IDXST_x / IDCT_x in one pass
-        case 5: k_col_fields_w<5><<<g, 32 * kWColWarps, sm, s>>>(a, sxy, c.d_tw2_x); break;
-        case 6: k_col_fields_w<6><<<g, 32 * kWColWarps, sm, s>>>(a, sxy, c.d_tw2_x); break;
-        case 7: k_col_fields_w<7><<<g, 32 * kWColWarps, sm, s>>>(a, sxy, c.d_tw2_x); break;
-        case 8: k_col_fields_w<8><<<g, 32 * kWColWarps, sm, s>>>(a, sxy, c.d_tw2_x); break;
-        case 9: k_col_fields_w<9><<<g, 32 * kWColWarps, sm, s>>>(a, sxy, c.d_tw2_x); break;
-        default: k_col_fields_w<10><<<g, 32 * kWColWarps, sm, s>>>(a, sxy, c.d_tw2_x); break;
+        case 5: launch_chain(c.pdl, k_col_fields_w<5>, g, 32 * kWColWarps, sm, s, a, sxy, c.d_tw2_x); break;
+        case 6: launch_chain(c.pdl, k_col_fields_w<6>, g, 32 * kWColWarps, sm, s, a, sxy, c.d_tw2_x); break;
+        case 7: launch_chain(c.pdl, k_col_fields_w<7>, g, 32 * kWColWarps, sm, s, a, sxy, c.d_tw2_x); break;
+        case 8: launch_chain(c.pdl, k_col_fields_w<8>, g, 32 * kWColWarps, sm, s, a, sxy, c.d_tw2_x); break;
+        case 9: launch_chain(c.pdl, k_col_fields_w<9>, g, 32 * kWColWarps, sm, s, a, sxy, c.d_tw2_x); break;
+        default: launch_chain(c.pdl, k_col_fields_w<10>, g, 32 * kWColWarps, sm, s, a, sxy, c.d_tw2_x); break;
       }
     } else {
       const size_t sm = (size_t)kWColWarps * wfft::kBufPad * sizeof(float2);
       float2 *spec = c.d_spec;
       switch (c.log2mx) {   // T2a
-        case 5: k_col_fwd_w<5><<<g, 32 * kWColWarps, sm, s>>>(a, spec, c.d_tw2_x); break;
-        case 6: k_col_fwd_w<6><<<g, 32 * kWColWarps, sm, s>>>(a, spec, c.d_tw2_x); break;
-        case 7: k_col_fwd_w<7><<<g, 32 * kWColWarps, sm, s>>>(a, spec, c.d_tw2_x); break;
-        case 8: k_col_fwd_w<8><<<g, 32 * kWColWarps, sm, s>>>(a, spec, c.d_tw2_x); break;
-        case 9: k_col_fwd_w<9><<<g, 32 * kWColWarps, sm, s>>>(a, spec, c.d_tw2_x); break;
-        default: k_col_fwd_w<10><<<g, 32 * kWColWarps, sm, s>>>(a, spec, c.d_tw2_x); break;
+        case 5: launch_chain(c.pdl, k_col_fwd_w<5>, g, 32 * kWColWarps, sm, s, a, spec, c.d_tw2_x); break;
+        case 6: launch_chain(c.pdl, k_col_fwd_w<6>, g, 32 * kWColWarps, sm, s, a, spec, c.d_tw2_x); break;
+        case 7: launch_chain(c.pdl, k_col_fwd_w<7>, g, 32 * kWColWarps, sm, s, a, spec, c.d_tw2_x); break;
+        case 8: launch_chain(c.pdl, k_col_fwd_w<8>, g, 32 * kWColWarps, sm, s, a, spec, c.d_tw2_x); break;
+        case 9: launch_chain(c.pdl, k_col_fwd_w<9>, g, 32 * kWColWarps, sm, s, a, spec, c.d_tw2_x); break;
+        default: launch_chain(c.pdl, k_col_fwd_w<10>, g, 32 * kWColWarps, sm, s, a, spec, c.d_tw2_x); break;
       }
       // T2b: per column v (row v of specT): sX = IDXST_x(A_X), sY = IDCT_x(A_Y), stored [x][y]
       row_inv(c, nullptr, 0, 2, nullptr, 0, 1, nullptr, 0, nullptr, 0, sxy, c.my, s, spec, true, c.my);

@@ -153,6 +153,7 @@ __device__ __forceinline__ void load_cells(const DenArgs &a, int i0, float (&x)[
 
 // D1: per-CTA shared histogram of tile ids
 __global__ void __launch_bounds__(kCountThreads) k_count(DenArgs a) {
+  griddep_wait();
   extern __shared__ int s_hist[];
   const int i0 = blockIdx.x * kCountCells;
   for (int t = threadIdx.x; t < a.ntiles; t += kCountThreads) s_hist[t] = 0;
@@ -182,6 +183,7 @@ __device__ __forceinline__ int warp_incl_scan(int v, int lane) {
 }
 
 __global__ void __launch_bounds__(1024) k_scan(DenArgs a) {
+  griddep_wait();
   __shared__ int s_wa[32];
   constexpr int T = 1024;
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
@@ -231,6 +233,7 @@ struct PlaceOut {
 int place_smem_bytes(int ntiles) { return (int)sizeof(PlaceOut) + 8 * ntiles; }
 
 __global__ void __launch_bounds__(kCountThreads) k_place(DenArgs a) {
+  griddep_wait();
   extern __shared__ __align__(16) unsigned char psm[];
   PlaceOut &po = *reinterpret_cast<PlaceOut *>(psm);
   int *s_hist = reinterpret_cast<int *>(psm + sizeof(PlaceOut));   // [ntiles] counts -> local offsets
@@ -468,6 +471,7 @@ __device__ __forceinline__ void flush_tile(const DenArgs &a, unsigned *s_hi, uns
 // D4: persistent scatter walker.  The shared tile of (hi, lo) 32-bit words is flushed into the
 // int64 map when the slice moves to another tile and at least every kFlushRecs records.
 __global__ void __launch_bounds__(kTileThreads) k_scatter_walk(DenArgs a) {
+  griddep_wait();
   extern __shared__ __align__(16) unsigned char dsm[];
   RecStage &st = *reinterpret_cast<RecStage *>(dsm);
   unsigned *s_hi = reinterpret_cast<unsigned *>(dsm + rec_stage_bytes());   // 2^-kTileHiBits units
@@ -547,6 +551,7 @@ __device__ __forceinline__ void load_xi_tile(const DenArgs &a, RecStage &st, flo
 }
 
 __global__ void __launch_bounds__(kTileThreads) k_gather_walk(DenArgs a) {
+  griddep_wait();
   extern __shared__ __align__(16) unsigned char dsm[];
   RecStage &st = *reinterpret_cast<RecStage *>(dsm);
   float2 *s_xi = reinterpret_cast<float2 *>(dsm + rec_stage_bytes());
@@ -762,12 +767,12 @@ void launch_density_map(const Ctx &c, const float *x, const float *y, cudaStream
     cudaEventRecord(c.ev_aux_b, aux);
   }
   if (nblk > 0) {
-    k_count<<<nblk, kCountThreads, ntiles * 4, s>>>(a);
+    launch_chain(c.pdl, k_count, nblk, kCountThreads, ntiles * 4, s, a);
     if (c.sched == 3) cudaEventRecord(c.ev_sched, s);   // DP_SCHED=3: WA starts after the count
-    k_scan<<<1, 1024, 0, s>>>(a);
-    k_place<<<nblk, kCountThreads, place_smem_bytes(ntiles), s>>>(a);
+    launch_chain(c.pdl, k_scan, 1, 1024, 0, s, a);
+    launch_chain(c.pdl, k_place, nblk, kCountThreads, place_smem_bytes(ntiles), s, a);
     if (c.sched == 2) cudaEventRecord(c.ev_sched, s);   // DP_SCHED=2: WA starts after the placement
-    k_scatter_walk<<<c.walk_grid, kTileThreads, walk_smem_bytes(c.tile), s>>>(a);
+    launch_chain(c.pdl, k_scatter_walk, c.walk_grid, kTileThreads, walk_smem_bytes(c.tile), s, a);
   }
   if (side)
     cudaStreamWaitEvent(s, c.ev_aux_b, 0);
@@ -784,7 +789,7 @@ void launch_density_gather(const Ctx &c, const float *x, const float *y, cudaStr
     k_gather_large<<<c.n_large, 256, 0, aux>>>(a);
     cudaEventRecord(c.ev_aux_b, aux);
   }
-  if (c.n_own > 0) k_gather_walk<<<c.walk_grid, kTileThreads, walk_smem_bytes(c.tile), s>>>(a);
+  if (c.n_own > 0) launch_chain(c.pdl, k_gather_walk, c.walk_grid, kTileThreads, walk_smem_bytes(c.tile), s, a);
   if (side)
     cudaStreamWaitEvent(s, c.ev_aux_b, 0);
   else if (c.n_large > 0)

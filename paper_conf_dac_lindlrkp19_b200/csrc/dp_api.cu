@@ -601,6 +601,7 @@ dp_status create(const dp_netlist *nl, const dp_grid *grid, int device, int rank
   { const char *e = std::getenv("DP_T1_TMA"); c->t1_tma = e && e[0] == '1'; }
   { const char *e = std::getenv("DP_GRAPH"); c->use_graph = !(e && e[0] == '0'); }
   { const char *e = std::getenv("DP_DIRECT"); c->direct = e && e[0] == '1'; }
+  { const char *e = std::getenv("DP_PDL"); c->pdl = !(e && e[0] == '0'); }
   {
     const char *e = std::getenv("DP_L2_PERSIST");
     c->l2_persist = !(e && e[0] == '0');

@@ -13,6 +13,33 @@
 
 namespace dp {
 
+// ---- programmatic dependent launch (PDL) on the density chain ------------------------------
+// A chain kernel launched with launch_chain() may be scheduled while its stream predecessor is
+// still finishing (its CTAs are placed once every predecessor CTA has started); griddep_wait()
+// at the top of the kernel then blocks until the predecessor has completed and its writes are
+// visible, so the semantics are those of plain stream order.  Without the launch attribute
+// (DP_PDL=0) both instructions are no-ops.
+__device__ __forceinline__ void griddep_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+__device__ __forceinline__ void griddep_launch_dependents() {
+  asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+}
+
+template <typename... KArgs, typename... Args>
+inline void launch_chain(bool pdl, void (*kernel)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t s,
+                         Args &&...args) {
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = grid;
+  cfg.blockDim = block;
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = s;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  at[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = pdl ? 1 : 0;
+  cudaLaunchKernelEx(&cfg, kernel, std::forward<Args>(args)...);
+}
+
 // ---------------------------------------------------------------------------------------
 // Compile-time layout parameters.
 // ---------------------------------------------------------------------------------------
@@ -142,6 +169,7 @@ struct Ctx {
   GraphKey gkey;
   int wl_model = 0;        // DP_WL_WA / DP_WL_LSE (dp_set_wl_model)
   bool deterministic = false;     // dp_set_deterministic (NEXT-2): WA gradient as exact int64 sums
+  bool pdl = true;                // programmatic dependent launch along the density chain (DP_PDL=0: off)
   bool direct = false;            // DP_DIRECT=1: WA and gather add into the caller's gx, gy (no combine pass)
   float *direct_gx = nullptr, *direct_gy = nullptr;   // set for the duration of one eval_body
   float direct_lambda = 0.f;

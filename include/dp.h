@@ -161,6 +161,18 @@ dp_status dp_set_wl_model(dp_ctx *ctx, int32_t model);
  * Errors: DP_ERR_INVALID_ARG, DP_ERR_OUT_OF_MEMORY.                                         */
 dp_status dp_set_deterministic(dp_ctx *ctx, int32_t on);
 
+/* Fixed cells (fixed macros; reading A34).  h_fixed (host, [num_cells],
+ * nonzero = fixed; NULL clears) marks cells that are charges of the density constraint (eq
+ * 1b) but not variables of (1a).  Their charge at the positions x, y given here
+ * (device, [num_cells]; only the fixed cells' entries are read) is scattered once into a
+ * precomputed fixed-charge map (exact int64, like every map); later evaluations start their
+ * map from it and sort / scatter / gather only the movable cells, so the fixed cells'
+ * positions passed to later calls are used for wirelength only.  gx, gy are 0 for fixed
+ * cells.  Single-GPU contexts only (DP_ERR_UNSUPPORTED for dp_create_dist contexts).
+ * Synchronises `stream`.  Errors: DP_ERR_INVALID_ARG, DP_ERR_OUT_OF_MEMORY, DP_ERR_CUDA.      */
+dp_status dp_set_fixed(dp_ctx *ctx, const uint8_t *h_fixed, const float *x, const float *y,
+                       dp_stream_t stream);
+
 /* Density only: gx, gy <- dD/dx, dD/dy; d_energy <- D.                        */
 dp_status dp_density_grad(dp_ctx *ctx, const float *x, const float *y, float *gx, float *gy,
                           double *d_energy, dp_stream_t stream);

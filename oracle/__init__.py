@@ -212,11 +212,17 @@ def density(nl, x, y, stretch: int = 1):
 
 
 def evaluate(nl, x, y, gamma: float, lam: float, stretch: int = 1, with_hpwl: bool = True,
-             wl_model: str = "wa"):
+             wl_model: str = "wa", fixed=None):
     """obj = WL + lambda D and grad = grad WL + lambda grad D (eq 2); WL = WA (eq 3)
-    or LSE (reading A27)."""
+    or LSE (reading A27).  fixed (bool [num_cells], NEXT-4 / reading A34): fixed cells
+    are charges of the density (eq 1b's d(x, y) counts every cell) but not variables of
+    (1a), so their gradient entries are 0."""
     wl, gwx, gwy = (lse if wl_model == "lse" else wa)(nl, x, y, gamma)
     D, gdx, gdy, parts = density(nl, x, y, stretch)
+    if fixed is not None:
+        m = np.asarray(fixed, dtype=bool)
+        for g in (gwx, gwy, gdx, gdy):
+            g[m] = 0.0
     out = dict(obj=wl + lam * D, wl=wl, energy=D, gx=gwx + lam * gdx, gy=gwy + lam * gdy,
                wl_gx=gwx, wl_gy=gwy, d_gx=gdx, d_gy=gdy, **parts)
     if with_hpwl:

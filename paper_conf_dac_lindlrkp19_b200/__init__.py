@@ -23,6 +23,7 @@ __all__ = [
     "dp_get_info", "dp_debug_density_map", "dp_debug_fields", "dp_debug_transform",
     "DP_T_DCT2", "DP_T_IDCT2", "DP_T_IDXST_IDCT", "DP_T_IDCT_IDXST", "EXPORTED_SYMBOLS",
     "dp_set_wl_model", "DP_WL_WA", "DP_WL_LSE", "GpParams", "GpLoop", "dp_gp_create", "dp_set_deterministic",
+    "dp_set_fixed",
 ]
 
 DP_T_DCT2, DP_T_IDCT2, DP_T_IDXST_IDCT, DP_T_IDCT_IDXST = 0, 1, 2, 3
@@ -36,7 +37,7 @@ EXPORTED_SYMBOLS = [
     "dp_eval_host", "dp_get_info", "dp_debug_density_map", "dp_debug_fields", "dp_debug_transform",
     "dp_profile_enable", "dp_profile_read", "dp_set_wl_model",
     "dp_gp_default_params", "dp_gp_create", "dp_gp_init", "dp_gp_run", "dp_gp_positions",
-    "dp_gp_history", "dp_gp_destroy", "dp_set_deterministic",
+    "dp_gp_history", "dp_gp_destroy", "dp_set_deterministic", "dp_set_fixed",
 ]
 __all__ += ["dp_profile_enable", "dp_profile_read", "STAGES"]
 STAGES = ["wa", "map", "fields", "gather", "combine", "eval"]
@@ -110,6 +111,7 @@ def lib() -> ctypes.CDLL:
             "dp_profile_read": [P, P, P],
             "dp_set_wl_model": [P, ctypes.c_int32],
             "dp_set_deterministic": [P, ctypes.c_int32],
+            "dp_set_fixed": [P, P, P, P, P],
             "dp_gp_create": [P, ctypes.POINTER(GpParams), ctypes.POINTER(P)],
             "dp_gp_init": [P, P, P, P],
             "dp_gp_run": [P, ctypes.c_int32, P],
@@ -358,6 +360,16 @@ def dp_eval(ctx, x, y, gamma, lam, gx, gy, d_obj=None, d_wl=None, d_energy=None,
 def dp_wl_grad(ctx, x, y, gamma, gx, gy, d_wl=None, stream=None):
     _check(lib().dp_wl_grad(ctx.handle, _ptr(x), _ptr(y), float(gamma), _ptr(gx), _ptr(gy), _ptr(d_wl),
                             _stream(stream)))
+
+
+def dp_set_fixed(ctx, fixed_mask, x=None, y=None, stream=None):
+    """fixed_mask: numpy bool/uint8 [num_cells] (None clears); x, y: device tensors."""
+    import numpy as np
+    if fixed_mask is None:
+        _check(lib().dp_set_fixed(ctx.handle, None, None, None, _stream(stream)))
+        return
+    m = np.ascontiguousarray(np.asarray(fixed_mask).astype(np.uint8))
+    _check(lib().dp_set_fixed(ctx.handle, m.ctypes.data_as(ctypes.c_void_p), _ptr(x), _ptr(y), _stream(stream)))
 
 
 def dp_set_deterministic(ctx, on: bool = True):

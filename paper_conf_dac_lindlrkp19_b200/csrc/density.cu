@@ -63,7 +63,15 @@ struct DenArgs {
   float *gxo, *gyo;
   float lambda;
   const float *lambda_dev;
+  // fixed cells (NEXT-4, dp_set_fixed): with a mask, only cells whose flag equals sel are
+  // sorted and scattered (sel = 0: the movable cells of an evaluation, whose map starts from
+  // the precomputed fixed-charge map; sel = 1: building that map)
+  const uint8_t *fixed;
+  int sel;
+  int n_large;
 };
+
+__device__ __forceinline__ bool selected(const DenArgs &a, int i) { return !a.fixed || a.fixed[i] == a.sel; }
 
 __device__ __forceinline__ void red_f32(float *p, float v) {
   asm volatile("red.global.add.f32 [%0], %1;" ::"l"(p), "f"(v) : "memory");
@@ -163,8 +171,9 @@ __global__ void __launch_bounds__(kCountThreads) k_count(DenArgs a) {
 #pragma unroll
   for (int k = 0; k < kCellsPerThread; k++) {
     SmallFoot f;
+    const int i = i0 + k * kCountThreads + threadIdx.x;
     const int t = classify_small(a, x[k], y[k], w[k], h[k], f);
-    if (t >= 0) atomicAdd(&s_hist[t], 1);
+    if (t >= 0 && (!a.fixed || (i < a.n_own && selected(a, i)))) atomicAdd(&s_hist[t], 1);
   }
   __syncthreads();
   for (int t = threadIdx.x; t < a.ntiles; t += kCountThreads)
@@ -252,9 +261,10 @@ __global__ void __launch_bounds__(kCountThreads) k_place(DenArgs a) {
   for (int k = 0; k < kCellsPerThread; k++) {
     const int i = i0 + k * kCountThreads + threadIdx.x;
     SmallFoot f;
-    const int t = classify_small(a, x[k], y[k], w[k], h[k], f);
+    int t = classify_small(a, x[k], y[k], w[k], h[k], f);
     tl[k] = -1;
     if (i >= a.n_own || t == -2) continue;
+    if (!selected(a, i)) t = -1;   // fixed cell of an evaluation: no record, force 0
     if (t == -1) {
       a.force[i] = make_float2(0.f, 0.f);
       continue;
@@ -722,6 +732,13 @@ DenArgs make_args(const Ctx &c, const float *x, const float *y) {
   a.lambda = c.direct_lambda;
   a.lambda_dev = c.lambda_dev;
   a.large = c.d_large;
+  a.n_large = c.n_large;
+  a.fixed = c.has_fixed ? c.d_fixed : nullptr;
+  a.sel = 0;
+  if (c.has_fixed) {
+    a.large = c.d_large_mov;
+    a.n_large = c.n_large_mov;
+  }
   return a;
 }
 
@@ -754,16 +771,27 @@ int density_launches(const Ctx &c) { return 6 + (c.n_large > 0 ? 1 : 0); }
 
 // aux (optional): a second stream for the large-cell CTAs, which then overlap the sort and the
 // tile walkers (joined back into s before return)
-void launch_density_map(const Ctx &c, const float *x, const float *y, cudaStream_t s, cudaStream_t aux) {
-  const DenArgs a = make_args(c, x, y);
+void launch_density_map(const Ctx &c, const float *x, const float *y, cudaStream_t s, cudaStream_t aux,
+                        int build_fixed) {
+  DenArgs a = make_args(c, x, y);
+  if (build_fixed) {   // dp_set_fixed: the map of the fixed cells alone
+    a.fixed = c.d_fixed;
+    a.sel = 1;
+    a.large = c.d_large_fix;
+    a.n_large = c.n_large_fix;
+  }
   const int ntiles = a.ntiles;
   const int nblk = (c.n_own + kCountCells - 1) / kCountCells;
-  cudaMemsetAsync(c.d_rho, 0, sizeof(unsigned long long) * (size_t)c.mx * c.my, s);
-  const bool side = aux && c.n_large > 0;
+  if (c.has_fixed && !build_fixed)   // start from the precomputed fixed-charge map (exact int64)
+    cudaMemcpyAsync(c.d_rho, c.d_rho_fixed, sizeof(unsigned long long) * (size_t)c.mx * c.my,
+                    cudaMemcpyDeviceToDevice, s);
+  else
+    cudaMemsetAsync(c.d_rho, 0, sizeof(unsigned long long) * (size_t)c.mx * c.my, s);
+  const bool side = aux && a.n_large > 0;
   if (side) {
     cudaEventRecord(c.ev_aux_a, s);
     cudaStreamWaitEvent(aux, c.ev_aux_a, 0);
-    k_scatter_large<<<c.n_large, 256, 0, aux>>>(a);
+    k_scatter_large<<<a.n_large, 256, 0, aux>>>(a);
     cudaEventRecord(c.ev_aux_b, aux);
   }
   if (nblk > 0) {
@@ -776,24 +804,24 @@ void launch_density_map(const Ctx &c, const float *x, const float *y, cudaStream
   }
   if (side)
     cudaStreamWaitEvent(s, c.ev_aux_b, 0);
-  else if (c.n_large > 0)
-    k_scatter_large<<<c.n_large, 256, 0, s>>>(a);
+  else if (a.n_large > 0)
+    k_scatter_large<<<a.n_large, 256, 0, s>>>(a);
 }
 
 void launch_density_gather(const Ctx &c, const float *x, const float *y, cudaStream_t s, cudaStream_t aux) {
   const DenArgs a = make_args(c, x, y);
-  const bool side = aux && c.n_large > 0;
+  const bool side = aux && a.n_large > 0;
   if (side) {
     cudaEventRecord(c.ev_aux_a, s);
     cudaStreamWaitEvent(aux, c.ev_aux_a, 0);
-    k_gather_large<<<c.n_large, 256, 0, aux>>>(a);
+    k_gather_large<<<a.n_large, 256, 0, aux>>>(a);
     cudaEventRecord(c.ev_aux_b, aux);
   }
   if (c.n_own > 0) launch_chain(c.pdl, k_gather_walk, c.walk_grid, kTileThreads, walk_smem_bytes(c.tile), s, a);
   if (side)
     cudaStreamWaitEvent(s, c.ev_aux_b, 0);
-  else if (c.n_large > 0)
-    k_gather_large<<<c.n_large, 256, 0, s>>>(a);
+  else if (a.n_large > 0)
+    k_gather_large<<<a.n_large, 256, 0, s>>>(a);
 }
 
 }  // namespace dp

@@ -819,7 +819,8 @@ dp_status eval_body(Ctx &c, const float *x, const float *y, float gamma, float l
   StageMark whole(c, DP_STAGE_EVAL, s);
   if (c.profiling) c.prof_evals++;
   // direct output (DP_DIRECT=1): both chains add into gx, gy, which are zeroed first; no combine
-  const bool direct = c.direct && !c.deterministic && !c.dist && ((((uintptr_t)gx) | ((uintptr_t)gy)) & 15) == 0;
+  const bool direct = c.direct && !c.deterministic && !c.dist && !c.has_fixed &&
+                      ((((uintptr_t)gx) | ((uintptr_t)gy)) & 15) == 0;
   struct DirectReset {
     Ctx &c;
     ~DirectReset() { c.direct_gx = c.direct_gy = nullptr; }
@@ -1003,6 +1004,53 @@ dp_status dp_set_deterministic(dp_ctx *ctx, int32_t on) {
   }
   c->deterministic = on != 0;
   return DP_OK;
+}
+
+dp_status dp_set_fixed(dp_ctx *ctx, const uint8_t *h_fixed, const float *x, const float *y, dp_stream_t stream) {
+  Ctx *c = C(ctx);
+  if (!c) return fail(DP_ERR_INVALID_ARG, "ctx is NULL");
+  if (c->dist) return fail(DP_ERR_UNSUPPORTED, "fixed cells are supported on single-GPU contexts");
+  if (h_fixed && (!x || !y)) return fail(DP_ERR_INVALID_ARG, "x / y is NULL");
+  dp::DeviceGuard g(c->device);
+  cudaStream_t s = (cudaStream_t)stream;
+  dp_status st = dp::call_begin(*c, s);
+  if (st != DP_OK) return st;
+  if (c->gexec) {   // the captured evaluation changes (map initialisation, masks): re-capture
+    DP_CUDA(cudaStreamSynchronize(s));
+    cudaGraphExecDestroy(c->gexec);
+    c->gexec = nullptr;
+    c->gkey = dp::GraphKey{};
+  }
+  if (!h_fixed) {
+    c->has_fixed = false;
+    return dp::call_end(*c, s);
+  }
+  const int n = c->n_own;
+  std::vector<uint8_t> m(((size_t)n + 3) & ~(size_t)3, 0);
+  for (int i = 0; i < n; i++) m[i] = h_fixed[c->cell_begin + i] ? 1 : 0;
+  std::vector<int32_t> large(c->n_large), mov, fix;
+  if (c->n_large)
+    DP_CUDA(cudaMemcpy(large.data(), c->d_large, sizeof(int32_t) * c->n_large, cudaMemcpyDeviceToHost));
+  for (int32_t i : large) (m[i] ? fix : mov).push_back(i);
+  if (!c->d_fixed) {
+    if ((st = dp::dev_alloc(*c, &c->d_fixed, m.size())) != DP_OK) return st;
+    if ((st = dp::dev_alloc(*c, &c->d_rho_fixed, (size_t)c->mx * c->my)) != DP_OK) return st;
+    if ((st = dp::dev_alloc(*c, &c->d_large_mov, (size_t)std::max(1, c->n_large))) != DP_OK) return st;
+    if ((st = dp::dev_alloc(*c, &c->d_large_fix, (size_t)std::max(1, c->n_large))) != DP_OK) return st;
+  }
+  DP_CUDA(cudaStreamSynchronize(s));
+  DP_CUDA(cudaMemcpy(c->d_fixed, m.data(), m.size(), cudaMemcpyHostToDevice));
+  if (!mov.empty()) DP_CUDA(cudaMemcpy(c->d_large_mov, mov.data(), sizeof(int32_t) * mov.size(), cudaMemcpyHostToDevice));
+  if (!fix.empty()) DP_CUDA(cudaMemcpy(c->d_large_fix, fix.data(), sizeof(int32_t) * fix.size(), cudaMemcpyHostToDevice));
+  c->n_large_mov = (int32_t)mov.size();
+  c->n_large_fix = (int32_t)fix.size();
+  c->has_fixed = true;
+  // the fixed-charge map: the density map of the fixed cells alone (exact int64), kept
+  dp::launch_density_map(*c, x, y, s, nullptr, 1);
+  DP_CUDA(cudaMemcpyAsync(c->d_rho_fixed, c->d_rho, sizeof(unsigned long long) * (size_t)c->mx * c->my,
+                          cudaMemcpyDeviceToDevice, s));
+  DP_CUDA(cudaGetLastError());
+  return dp::call_end(*c, s);
 }
 
 dp_status dp_density_grad(dp_ctx *ctx, const float *x, const float *y, float *gx, float *gy, double *d_energy,

@@ -151,7 +151,14 @@ struct Ctx {
 
   // ---- density layout (device) ----
   float *d_cell_w = nullptr, *d_cell_h = nullptr;   // own cells (index from cell_begin)
-  float *d_cell_pins = nullptr;                     // [num_cells] net-weighted pin count (GP preconditioner)
+  float *d_cell_pins = nullptr;
+  // fixed cells (NEXT-4, dp_set_fixed): mask per own cell, precomputed fixed-charge map, and
+  // the large-cell lists split by mobility
+  bool has_fixed = false;
+  uint8_t *d_fixed = nullptr;
+  unsigned long long *d_rho_fixed = nullptr;
+  int32_t *d_large_mov = nullptr, *d_large_fix = nullptr;
+  int32_t n_large_mov = 0, n_large_fix = 0;                     // [num_cells] net-weighted pin count (GP preconditioner)
   int32_t n_own = 0;                // cells owned by this rank
   int32_t n_large = 0;              // large cells (footprint > 3 bins on an axis)
   int32_t *d_large = nullptr;       // ids of large own cells
@@ -249,7 +256,8 @@ dp_status cuda_fail(cudaError_t e, const char *what);
 void launch_wa(const Ctx &c, const float *x, const float *y, float gamma, bool hpwl_only,
                bool with_hpwl, cudaStream_t s);
 // density (density.cu)
-void launch_density_map(const Ctx &c, const float *x, const float *y, cudaStream_t s, cudaStream_t aux = nullptr);
+void launch_density_map(const Ctx &c, const float *x, const float *y, cudaStream_t s, cudaStream_t aux = nullptr,
+                        int build_fixed = 0);
 void launch_density_gather(const Ctx &c, const float *x, const float *y, cudaStream_t s, cudaStream_t aux = nullptr);
 // transforms (dct.cu)
 void launch_fields(const Ctx &c, const float *rho, cudaStream_t s);            // rho as float (debug hook)

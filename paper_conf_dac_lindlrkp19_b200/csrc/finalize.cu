@@ -20,7 +20,8 @@ namespace {
 __global__ void __launch_bounds__(256) k_combine_det(const long long *__restrict__ g2i, int frac,
                                                      const float2 *__restrict__ force, float *__restrict__ gx,
                                                      float *__restrict__ gy, int cell_begin, int n_own, float lambda,
-                                                     const float *__restrict__ lambda_dev, int use_wa, int use_den) {
+                                                     const float *__restrict__ lambda_dev, int use_wa, int use_den,
+                                                     const uint8_t *__restrict__ fixed) {
   if (lambda_dev) lambda = __ldg(lambda_dev);
   const int i = blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= n_own) return;
@@ -36,6 +37,7 @@ __global__ void __launch_bounds__(256) k_combine_det(const long long *__restrict
     vx = fmaf(lambda, f.x, vx);
     vy = fmaf(lambda, f.y, vy);
   }
+  if (fixed && fixed[i]) vx = vy = 0.f;
   gx[c] = vx;
   gy[c] = vy;
 }
@@ -43,7 +45,7 @@ __global__ void __launch_bounds__(256) k_combine_det(const long long *__restrict
 __global__ void __launch_bounds__(256) k_combine(const float2 *__restrict__ g2, const float2 *__restrict__ force,
                                                  float *__restrict__ gx, float *__restrict__ gy, int cell_begin,
                                                  int n_own, float lambda, const float *__restrict__ lambda_dev,
-                                                 int use_wa, int use_den) {
+                                                 int use_wa, int use_den, const uint8_t *__restrict__ fixed) {
   if (lambda_dev) lambda = __ldg(lambda_dev);   // GP loop: lambda on the device
   const int c0 = (cell_begin & ~3) + 4 * (blockIdx.x * blockDim.x + threadIdx.x);
   const int cend = cell_begin + n_own;
@@ -61,12 +63,19 @@ __global__ void __launch_bounds__(256) k_combine(const float2 *__restrict__ g2, 
       f0 = __ldcs(reinterpret_cast<const float4 *>(fb + c0));
       f1 = __ldcs(reinterpret_cast<const float4 *>(fb + c0 + 2));
     }
-    __stcs(reinterpret_cast<float4 *>(gx + c0),
-           make_float4(fmaf(lambda, f0.x, g0.x), fmaf(lambda, f0.z, g0.z), fmaf(lambda, f1.x, g1.x),
-                       fmaf(lambda, f1.z, g1.z)));
-    __stcs(reinterpret_cast<float4 *>(gy + c0),
-           make_float4(fmaf(lambda, f0.y, g0.y), fmaf(lambda, f0.w, g0.w), fmaf(lambda, f1.y, g1.y),
-                       fmaf(lambda, f1.w, g1.w)));
+    float4 ox = make_float4(fmaf(lambda, f0.x, g0.x), fmaf(lambda, f0.z, g0.z), fmaf(lambda, f1.x, g1.x),
+                            fmaf(lambda, f1.z, g1.z));
+    float4 oy = make_float4(fmaf(lambda, f0.y, g0.y), fmaf(lambda, f0.w, g0.w), fmaf(lambda, f1.y, g1.y),
+                            fmaf(lambda, f1.w, g1.w));
+    if (fixed) {   // NEXT-4: fixed cells are not variables -> gradient 0 (single-context: own = global)
+      const uchar4 m = *reinterpret_cast<const uchar4 *>(fixed + c0);
+      if (m.x) ox.x = oy.x = 0.f;
+      if (m.y) ox.y = oy.y = 0.f;
+      if (m.z) ox.z = oy.z = 0.f;
+      if (m.w) ox.w = oy.w = 0.f;
+    }
+    __stcs(reinterpret_cast<float4 *>(gx + c0), ox);
+    __stcs(reinterpret_cast<float4 *>(gy + c0), oy);
     return;
   }
   for (int c = c0; c < c0 + 4; c++) {  // ragged ends of the own range / unaligned caller buffers
@@ -82,6 +91,7 @@ __global__ void __launch_bounds__(256) k_combine(const float2 *__restrict__ g2, 
       vx = fmaf(lambda, q.x, vx);
       vy = fmaf(lambda, q.y, vy);
     }
+    if (fixed && fixed[c - cell_begin]) vx = vy = 0.f;
     gx[c] = vx;
     gy[c] = vy;
   }
@@ -185,13 +195,14 @@ void launch_combine(const Ctx &c, float lambda, float *gx, float *gy, bool use_w
   if (c.deterministic) {
     k_combine_det<<<(c.n_own + 255) / 256, 256, 0, s>>>(c.d_g2i, c.det_frac, c.d_force, gx, gy, c.cell_begin, c.n_own,
                                                         lambda, use_density ? c.lambda_dev : nullptr, use_wa ? 1 : 0,
-                                                        use_density ? 1 : 0);
+                                                        use_density ? 1 : 0, c.has_fixed ? c.d_fixed : nullptr);
     return;
   }
   const int quads = (c.n_own + 6) / 4 + 1;
   const int blocks = (quads + 255) / 256;
   k_combine<<<blocks, 256, 0, s>>>(c.d_g2, c.d_force, gx, gy, c.cell_begin, c.n_own, lambda,
-                                   use_density ? c.lambda_dev : nullptr, use_wa ? 1 : 0, use_density ? 1 : 0);
+                                   use_density ? c.lambda_dev : nullptr, use_wa ? 1 : 0, use_density ? 1 : 0,
+                                   c.has_fixed ? c.d_fixed : nullptr);
 }
 
 void launch_finalize_phase(const Ctx &c, int phase, float lambda, bool with_wl, bool with_energy, bool with_hpwl,

@@ -85,9 +85,10 @@ def lib() -> ctypes.CDLL:
     """Load libdp.so (built in-tree by build()).  Raises if it is missing: no fallback."""
     global _lib
     if _lib is None:
-        if not os.path.exists(LIB):
-            raise RuntimeError(f"libdp.so not built ({LIB}); run paper_conf_dac_lindlrkp19_b200.build.build()")
-        L = ctypes.CDLL(LIB)
+        path = os.environ.get("DP_LIB_AB", LIB)   # A/B measurements of an alternative in-tree build
+        if not os.path.exists(path):
+            raise RuntimeError(f"libdp.so not built ({path}); run paper_conf_dac_lindlrkp19_b200.build.build()")
+        L = ctypes.CDLL(path)
         L.dp_last_error.restype = ctypes.c_char_p
         L.dp_version.restype = I32
         for name, args in {

@@ -358,12 +358,14 @@ def run_ours(args, rank, world, local_rank):
         dp.dp_set_deterministic(ctx, False)
         step()
         # NEXT-4: the large blocks fixed (macros): fixed-charge map + movable-only sorting
-        big = (nl.cell_w > 2 * nl.bin_w) | (nl.cell_h > 2 * nl.bin_h)
-        dp.dp_set_fixed(ctx, big, xt, yt, stream)
-        step()
-        fixed_ms = timed(step, Ks)
-        dp.dp_set_fixed(ctx, None, stream=stream)
-        step()
+        # (single-GPU contexts only)
+        if world == 1:
+            big = (nl.cell_w > 2 * nl.bin_w) | (nl.cell_h > 2 * nl.bin_h)
+            dp.dp_set_fixed(ctx, big, xt, yt, stream)
+            step()
+            fixed_ms = timed(step, Ks)
+            dp.dp_set_fixed(ctx, None, stream=stream)
+            step()
     # NEXT-1: GP iterations (Nesterov step + evaluation + schedule, one graph per iteration)
     # from the paper's initial placement, single-GPU contexts only
     gp_stats = None
@@ -406,7 +408,7 @@ def run_ours(args, rank, world, local_rank):
                  "graph_replay_evals_per_s": (1e3 / graph_ms) if isinstance(graph_ms, float) else graph_ms,
                  "lse_evals_per_s": None if args.skip_next else 1e3 / lse_ms,
                  "deterministic_evals_per_s": None if args.skip_next else 1e3 / det_ms,
-                 "fixed_macros_evals_per_s": None if args.skip_next else 1e3 / fixed_ms, "gp": gp_stats,
+                 "fixed_macros_evals_per_s": None if (args.skip_next or world > 1) else 1e3 / fixed_ms, "gp": gp_stats,
                  "note": "rank-0 device time of min(K, 200) back-to-back calls each; not the headline"}
     if rank != 0:
         if pg:

@@ -767,7 +767,9 @@ int density_walk_grid(int tile) {
   return sms * std::max(1, std::min(o1, o2));
 }
 
-int density_launches(const Ctx &c) { return 6 + (c.n_large > 0 ? 1 : 0); }
+// kernels of one evaluation's density map + gather: count, scan, place, scatter, gather, and the
+// large-cell scatter / gather when there are large cells
+int density_launches(const Ctx &c) { return 5 + (c.n_large > 0 ? 2 : 0); }
 
 // aux (optional): a second stream for the large-cell CTAs, which then overlap the sort and the
 // tile walkers (joined back into s before return)

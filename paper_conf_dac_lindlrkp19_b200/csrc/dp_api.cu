@@ -649,7 +649,7 @@ dp_status create(const dp_netlist *nl, const dp_grid *grid, int device, int rank
     cudaGetLastError();   // best effort: a refused hint leaves the default policy
   }
   const int wa_k = (c->n_chunks + c->n_big > 0) ? 1 : 0;   // one kernel: big nets, warp nets, chunks
-  c->launches_eval = wa_k + density_launches(*c) + 3 /* T1 T2 T3 */ + 2 /* combine, finalize */;
+  c->launches_eval = wa_k + density_launches(*c) + (c->fused_t2 ? 3 : 4) /* T1 T2a T2b T3 */ + 2 /* combine, finalize */;
   c->launches_eval_hpwl = c->launches_eval;
   if (world > 1 && nccl_id) {
     if ((st = nccl_init(*c, nccl_id)) != DP_OK) return bail(st);

@@ -160,6 +160,9 @@ __device__ __forceinline__ void load_cells(const DenArgs &a, int i0, float (&x)[
 }
 
 // D1: per-CTA shared histogram of tile ids
+// MASK: a fixed-cell mask is in effect (dp_set_fixed with fixed small cells); a separate
+// instantiation keeps the default path's register budget (and occupancy) unchanged
+template <bool MASK>
 __global__ void __launch_bounds__(kCountThreads) k_count(DenArgs a) {
   griddep_wait();
   extern __shared__ int s_hist[];
@@ -173,7 +176,7 @@ __global__ void __launch_bounds__(kCountThreads) k_count(DenArgs a) {
     SmallFoot f;
     const int i = i0 + k * kCountThreads + threadIdx.x;
     const int t = classify_small(a, x[k], y[k], w[k], h[k], f);
-    if (t >= 0 && (!a.fixed || (i < a.n_own && selected(a, i)))) atomicAdd(&s_hist[t], 1);
+    if (t >= 0 && (!MASK || (i < a.n_own && selected(a, i)))) atomicAdd(&s_hist[t], 1);
   }
   __syncthreads();
   for (int t = threadIdx.x; t < a.ntiles; t += kCountThreads)
@@ -241,6 +244,7 @@ struct PlaceOut {
 
 int place_smem_bytes(int ntiles) { return (int)sizeof(PlaceOut) + 8 * ntiles; }
 
+template <bool MASK>
 __global__ void __launch_bounds__(kCountThreads) k_place(DenArgs a) {
   griddep_wait();
   extern __shared__ __align__(16) unsigned char psm[];
@@ -264,7 +268,7 @@ __global__ void __launch_bounds__(kCountThreads) k_place(DenArgs a) {
     int t = classify_small(a, x[k], y[k], w[k], h[k], f);
     tl[k] = -1;
     if (i >= a.n_own || t == -2) continue;
-    if (!selected(a, i)) t = -1;   // fixed cell of an evaluation: no record, force 0
+    if (MASK && !selected(a, i)) t = -1;   // fixed cell of an evaluation: no record, force 0
     if (t == -1) {
       a.force[i] = make_float2(0.f, 0.f);
       continue;
@@ -733,7 +737,7 @@ DenArgs make_args(const Ctx &c, const float *x, const float *y) {
   a.lambda_dev = c.lambda_dev;
   a.large = c.d_large;
   a.n_large = c.n_large;
-  a.fixed = c.has_fixed ? c.d_fixed : nullptr;
+  a.fixed = c.has_fixed && c.fixed_small ? c.d_fixed : nullptr;
   a.sel = 0;
   if (c.has_fixed) {
     a.large = c.d_large_mov;
@@ -745,9 +749,13 @@ DenArgs make_args(const Ctx &c, const float *x, const float *y) {
 }  // namespace
 
 cudaError_t density_configure(int ntiles, int tile) {
-  cudaError_t e = cudaFuncSetAttribute(k_count, cudaFuncAttributeMaxDynamicSharedMemorySize, ntiles * 4);
+  cudaError_t e = cudaFuncSetAttribute(k_count<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, ntiles * 4);
   if (e != cudaSuccess) return e;
-  e = cudaFuncSetAttribute(k_place, cudaFuncAttributeMaxDynamicSharedMemorySize, place_smem_bytes(ntiles));
+  e = cudaFuncSetAttribute(k_count<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, ntiles * 4);
+  if (e != cudaSuccess) return e;
+  e = cudaFuncSetAttribute(k_place<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, place_smem_bytes(ntiles));
+  if (e != cudaSuccess) return e;
+  e = cudaFuncSetAttribute(k_place<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, place_smem_bytes(ntiles));
   if (e != cudaSuccess) return e;
   e = cudaFuncSetAttribute(k_scatter_walk, cudaFuncAttributeMaxDynamicSharedMemorySize, walk_smem_bytes(tile));
   if (e != cudaSuccess) return e;
@@ -797,10 +805,16 @@ void launch_density_map(const Ctx &c, const float *x, const float *y, cudaStream
     cudaEventRecord(c.ev_aux_b, aux);
   }
   if (nblk > 0) {
-    launch_chain(c.pdl, k_count, nblk, kCountThreads, ntiles * 4, s, a);
+    if (a.fixed)
+      launch_chain(c.pdl, k_count<true>, nblk, kCountThreads, ntiles * 4, s, a);
+    else
+      launch_chain(c.pdl, k_count<false>, nblk, kCountThreads, ntiles * 4, s, a);
     if (c.sched == 3) cudaEventRecord(c.ev_sched, s);   // DP_SCHED=3: WA starts after the count
     launch_chain(c.pdl, k_scan, 1, 1024, 0, s, a);
-    launch_chain(c.pdl, k_place, nblk, kCountThreads, place_smem_bytes(ntiles), s, a);
+    if (a.fixed)
+      launch_chain(c.pdl, k_place<true>, nblk, kCountThreads, place_smem_bytes(ntiles), s, a);
+    else
+      launch_chain(c.pdl, k_place<false>, nblk, kCountThreads, place_smem_bytes(ntiles), s, a);
     if (c.sched == 2) cudaEventRecord(c.ev_sched, s);   // DP_SCHED=2: WA starts after the placement
     launch_chain(c.pdl, k_scatter_walk, c.walk_grid, kTileThreads, walk_smem_bytes(c.tile), s, a);
   }

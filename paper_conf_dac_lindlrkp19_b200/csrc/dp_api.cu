@@ -1032,6 +1032,11 @@ dp_status dp_set_fixed(dp_ctx *ctx, const uint8_t *h_fixed, const float *x, cons
   if (c->n_large)
     DP_CUDA(cudaMemcpy(large.data(), c->d_large, sizeof(int32_t) * c->n_large, cudaMemcpyDeviceToHost));
   for (int32_t i : large) (m[i] ? fix : mov).push_back(i);
+  {   // fixed small cells need the mask in the sort; fixed large cells only change the lists
+    size_t nfix = 0;
+    for (int i = 0; i < n; i++) nfix += m[i];
+    c->fixed_small = nfix > fix.size();
+  }
   if (!c->d_fixed) {
     if ((st = dp::dev_alloc(*c, &c->d_fixed, m.size())) != DP_OK) return st;
     if ((st = dp::dev_alloc(*c, &c->d_rho_fixed, (size_t)c->mx * c->my)) != DP_OK) return st;

@@ -155,6 +155,7 @@ struct Ctx {
   // fixed cells (NEXT-4, dp_set_fixed): mask per own cell, precomputed fixed-charge map, and
   // the large-cell lists split by mobility
   bool has_fixed = false;
+  bool fixed_small = false;     // some fixed cell is a small cell (the count / place kernels need the mask)
   uint8_t *d_fixed = nullptr;
   unsigned long long *d_rho_fixed = nullptr;
   int32_t *d_large_mov = nullptr, *d_large_fix = nullptr;

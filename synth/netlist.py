@@ -33,7 +33,7 @@ import math
 import numpy as np
 
 __all__ = ["Netlist", "CONFIGS", "make_netlist", "make_positions", "config_by_name",
-           "solve_alpha", "custom_netlist"]
+           "solve_alpha", "custom_netlist", "add_fillers"]
 
 
 @dataclasses.dataclass
@@ -230,3 +230,32 @@ def custom_netlist(net_start, pin2cell, pin_dx, pin_dy, cell_w, cell_h, region, 
                    xl=float(region[0]), yl=float(region[1]), xh=float(region[2]), yh=float(region[3]),
                    bins_x=int(bins[0]), bins_y=int(bins[1]),
                    net_weight=None if net_weight is None else np.ascontiguousarray(net_weight, dtype=np.float32))
+
+
+def add_fillers(nl: Netlist, x: np.ndarray, y: np.ndarray, target_density: float = 1.0,
+                fixed: np.ndarray | None = None, seed: int = 4242):
+    """Append pinless filler cells (ePlace's whitespace fillers; reading A35) so that
+    movable + filler area = target_density * (region area - fixed area).  Filler size: the mean
+    width of the movable standard cells (sides <= 2 bins) x their row height 12.  Fillers start
+    where the movable cells are (uniform over the movable cells' bounding box).  Returns
+    (netlist, x, y, fixed) with the fillers appended after the original cells (no pins)."""
+    rng = np.random.default_rng(seed)
+    fx = np.zeros(nl.num_cells, dtype=bool) if fixed is None else np.asarray(fixed, dtype=bool)
+    area = nl.cell_w.astype(np.float64) * nl.cell_h.astype(np.float64)
+    region = (nl.xh - nl.xl) * (nl.yh - nl.yl)
+    free = target_density * (region - area[fx].sum()) - area[~fx].sum()
+    std = (~fx) & (nl.cell_w <= 2 * nl.bin_w) & (nl.cell_h <= 2 * nl.bin_h)
+    fw = float(np.mean(nl.cell_w[std])) if std.any() else nl.bin_w
+    fh = 12.0
+    n = max(0, int(free // (fw * fh)))
+    mv = ~fx
+    lo_x, hi_x = float(x[mv].min()), float((x[mv] + nl.cell_w[mv]).max())
+    lo_y, hi_y = float(y[mv].min()), float((y[mv] + nl.cell_h[mv]).max())
+    xf = (lo_x + rng.random(n) * max(hi_x - lo_x - fw, 0.0)).astype(np.float32)
+    yf = (lo_y + rng.random(n) * max(hi_y - lo_y - fh, 0.0)).astype(np.float32)
+    out = dataclasses.replace(
+        nl, name=nl.name + "+fillers", num_cells=nl.num_cells + n,
+        cell_w=np.concatenate([nl.cell_w, np.full(n, fw, np.float32)]),
+        cell_h=np.concatenate([nl.cell_h, np.full(n, fh, np.float32)]))
+    return (out, np.concatenate([x, xf]).astype(np.float32), np.concatenate([y, yf]).astype(np.float32),
+            np.concatenate([fx, np.zeros(n, dtype=bool)]))

@@ -113,3 +113,31 @@ def test_gp_keeps_fixed_cells():
     assert np.array_equal(ux[m], x[m]) and np.array_equal(uy[m], y[m])
     assert hist[-1]["overflow"] < hist[0]["overflow"]
     assert np.abs(ux[~m] - x[~m]).max() > nl.bin_w   # movable cells did move
+
+
+def test_gp_with_fillers_and_fixed_macros():
+    """ePlace-style setup (reading A35): pinless fillers bring the movable area to 90% of the
+    free area, the large blocks are fixed; the device loop spreads movable cells and fillers.
+    The evaluation with fillers matches the oracle (fillers are plain cells of the map)."""
+    from synth import add_fillers
+    nl0 = make_netlist("tiny")
+    x0, y0 = make_positions(nl0, "initial")
+    big = _mask(nl0, 0.0, 1)
+    rng = np.random.default_rng(3)
+    x0[big] = rng.uniform(nl0.xl, nl0.xh - nl0.cell_w[big]).astype(np.float32)
+    y0[big] = rng.uniform(nl0.yl, nl0.yh - nl0.cell_h[big]).astype(np.float32)
+    nl, x, y, fixed = add_fillers(nl0, x0, y0, 0.9, fixed=big)
+    assert nl.num_cells > nl0.num_cells
+    xt, yt = _t(x), _t(y)
+    ctx = dp.dp_create(nl)
+    dp.dp_set_fixed(ctx, fixed, xt, yt)
+    out = ctx.eval(xt, yt, nl.bin_w, 0.3)
+    ref = oracle.evaluate(nl, x, y, nl.bin_w, 0.3, with_hpwl=False, fixed=fixed)
+    check_scalar("obj", out["obj"].item(), ref["obj"])
+    check_vector("gx", to_np(out["gx"]), ref["gx"])
+    loop = dp.GpLoop(ctx, target_density=0.9)
+    loop.init(xt, yt)
+    loop.run(600)
+    hist = loop.history()
+    print([(int(h["k"]), round(h["overflow"], 3)) for h in hist[::100]])
+    assert hist[-1]["overflow"] < 0.5 * hist[0]["overflow"]

@@ -207,6 +207,8 @@ typedef struct dp_gp_params {
     float dhpwl_ref;         /* p = dHPWL / dhpwl_ref; default 3.5e5                 */
     float init_rms_bins;     /* rms displacement of v_{-1}, in bins (A33); default 0.01     */
     int32_t max_history;     /* iterations kept in the device history ring; default 4096    */
+    float stop_overflow;     /* converged below this overflow: the state then stays (A36);
+                                default 0.07 (DREAMPlace's stop criterion); 0 = never       */
 } dp_gp_params;
 typedef struct dp_gp dp_gp;  /* opaque; owns ~12 float vectors of num_cells + scalars       */
 

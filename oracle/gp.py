@@ -29,6 +29,9 @@ conventions the paper says it follows and listed as readings in DESIGN.md §3:
   A33  HPWL and tau are taken at the reference solution v, where the gradient is evaluated;
        clamp keeps lower-left corners in [xl, xh - w] x [yl, yh - h]; the first Lipschitz
        estimate uses v_{-1} = v_0 - eta g_0 with an rms displacement of 0.01 b_x.
+  A36  GP stops once tau < stop_overflow (DREAMPlace's stop criterion, default 0.07): later
+       iterations leave u, v, lambda and gamma unchanged ("GP converges"); lambda is
+       capped at 1e30 (the eq-18 product is unbounded otherwise).
 """
 from __future__ import annotations
 
@@ -49,6 +52,7 @@ class GpParams:
     mu_max: float = 1.05
     dhpwl_ref: float = 3.5e5          # p = dHPWL / 3.5e5
     init_rms_bins: float = 0.01       # rms displacement of v_{-1}, in bins      (A33)
+    stop_overflow: float = 0.07       # GP converged below this overflow         (A36)
 
 
 # ------------------------------------------------------------------------- schedule pieces
@@ -116,6 +120,7 @@ class GpState:
     tau: float
     alpha: float
     k: int
+    frozen: bool = False
 
 
 def _eval_pre(nl, x, y, gamma, lam):
@@ -150,15 +155,22 @@ def gp_step(nl, st: GpState, prm: GpParams | None = None) -> dict:
     def cl(z):
         return np.stack(clamp(nl, z[0], z[1]))
 
+    if st.frozen:   # A36: converged; the state stays as it is
+        r = evaluate(nl, st.v[0], st.v[1], st.gamma, st.lam, with_hpwl=True)
+        stats = dict(k=st.k, hpwl=r["hpwl"], overflow=st.tau, lam=st.lam, gamma=st.gamma, obj=r["obj"],
+                     alpha=st.alpha, wl=r["wl"])
+        st.k += 1
+        return stats
     u_new, v_new, a_new, alpha = nesterov_step(st.u, st.v, st.vp, st.g, st.gp, st.a, st.alpha, cl)
     g_new, r = _eval_pre(nl, v_new[0], v_new[1], st.gamma, st.lam)
     tau = overflow(nl, r["rho"], prm.target_density)
     p = (r["hpwl"] - st.hpwl) / prm.dhpwl_ref
-    lam = st.lam * mu(p, st.k, prm)
+    lam = min(st.lam * mu(p, st.k, prm), 1e30)
     stats = dict(k=st.k, hpwl=r["hpwl"], overflow=tau, lam=lam, gamma=gamma_of(nl, tau, prm),
                  obj=r["obj"], alpha=alpha, wl=r["wl"])
     st.vp, st.gp = st.v, st.g
     st.u, st.v, st.g, st.a = u_new, v_new, g_new, a_new
     st.lam, st.gamma, st.hpwl, st.tau, st.alpha = lam, stats["gamma"], r["hpwl"], tau, alpha
     st.k += 1
+    st.frozen = tau < prm.stop_overflow
     return stats

@@ -75,7 +75,8 @@ class GpParams(ctypes.Structure):
     """dp_gp_params (include/dp.h)."""
     _fields_ = [("target_density", ctypes.c_float), ("gamma_base_scale", ctypes.c_float),
                 ("lambda_scale", ctypes.c_float), ("mu_min", ctypes.c_float), ("mu_max", ctypes.c_float),
-                ("dhpwl_ref", ctypes.c_float), ("init_rms_bins", ctypes.c_float), ("max_history", I32)]
+                ("dhpwl_ref", ctypes.c_float), ("init_rms_bins", ctypes.c_float), ("max_history", I32),
+                ("stop_overflow", ctypes.c_float)]
 
 
 _lib = None

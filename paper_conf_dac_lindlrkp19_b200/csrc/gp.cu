@@ -12,6 +12,8 @@
 //   A31 gamma = 4 (b_x + b_y) 10^((tau - 0.1) 20/9 - 1)
 //   A32 lambda_0 = 8e-5 |grad WL|_1 / |grad D|_1, then eq (18) with p = dHPWL / 3.5e5
 //   A33 HPWL / overflow at v; clamp to [xl, xh - w]; v_{-1} = v_0 - eta g_0 (rms 0.01 b_x)
+//   A36 converged once overflow < stop_overflow: later iterations leave the state unchanged;
+//       lambda capped at 1e30
 //
 // B200 design: every step runs on the device.  gamma and lambda live in device memory and
 // the evaluation kernels read them there (Ctx::gamma_dev / lambda_dev), so one iteration —
@@ -34,7 +36,9 @@ struct GpDev {      // device-resident loop state (scalars)
   double a, lam, gamma, hpwl, tau, alpha, coef, eta;
   double l1_wl, l1_d, area_total, gamma_base;
   long long k;
-  float f_gamma, f_lambda, f_alpha, f_coef, f_eta, pad_[3];
+  float f_gamma, f_lambda, f_alpha, f_coef, f_eta;
+  int frozen;                       // A36: converged (the step kernel and the schedule stop)
+  float pad_[2];
 };
 
 struct GpArgs {
@@ -55,7 +59,7 @@ struct GpArgs {
   double *hist;
   int hist_cap;
   double bxby;
-  double mu_min, mu_max, dhpwl_ref, lambda_scale, init_rms_bins, bx;
+  double mu_min, mu_max, dhpwl_ref, lambda_scale, init_rms_bins, bx, stop_overflow;
 };
 
 // fixed-order block reduction of two fp64 values into part[2 * blockIdx.x + {0,1}]
@@ -170,10 +174,19 @@ __global__ void __launch_bounds__(kGpThreads) k_gp_scalar(GpArgs a, int op) {
     case S_ITER_END: {   // A30 overflow, eq (18) lambda, A31 gamma, history row; then A28 for the next step
       const double tau = o0 * a.bxby / d.area_total;
       const double hp = a.out[3];
+      if (d.frozen) {   // A36: converged, the state stays; the row repeats it
+        if (a.hist_cap > 0) {
+          double *r = a.hist + (size_t)(d.k % a.hist_cap) * kHistCols;
+          r[0] = (double)d.k; r[1] = hp; r[2] = d.tau; r[3] = d.lam;
+          r[4] = d.gamma; r[5] = a.out[0]; r[6] = d.alpha; r[7] = a.out[1];
+        }
+        d.k += 1;
+        break;
+      }
       const double p = (hp - d.hpwl) / a.dhpwl_ref;
       const double mu = p < 0.0 ? a.mu_max * fmax(pow(0.9999, (double)d.k), 0.98)
                                 : fmax(a.mu_min, pow(a.mu_max, 1.0 - p));            // eq (18a)
-      d.lam *= mu;
+      d.lam = fmin(d.lam * mu, 1e30);
       d.tau = tau;
       d.gamma = gamma_of(a, tau);
       if (a.hist_cap > 0) {
@@ -186,6 +199,7 @@ __global__ void __launch_bounds__(kGpThreads) k_gp_scalar(GpArgs a, int op) {
       d.f_gamma = (float)d.gamma;
       d.f_lambda = (float)d.lam;
       step_scalars(d, t0, t1);
+      if (tau < a.stop_overflow) d.frozen = 1;
       break;
     }
     case S_INIT_TAU:
@@ -212,6 +226,7 @@ __global__ void __launch_bounds__(kGpThreads) k_gp_scalar(GpArgs a, int op) {
       d.a = 1.0;
       d.alpha = 0.0;
       d.k = 0;
+      d.frozen = 0;
       break;
   }
 }
@@ -221,7 +236,7 @@ __device__ __forceinline__ float clampf(float v, float lo, float hi) { return fm
 // A28 per cell: u' = clamp(v - alpha g); v' = clamp(u' + coef (u' - u)); vp = v; gp = g.
 __global__ void __launch_bounds__(kGpThreads) k_gp_update(GpArgs a) {
   const int i = blockIdx.x * kGpThreads + threadIdx.x;
-  if (i >= a.n) return;
+  if (i >= a.n || a.dev->frozen) return;
   const float alpha = a.dev->f_alpha, coef = a.dev->f_coef;
   const float hx = a.xh - a.w[i], hy = a.yh - a.h[i];
   const float vx = a.vx[i], vy = a.vy[i], gx = a.gx[i], gy = a.gy[i];
@@ -394,6 +409,7 @@ void dp_gp_default_params(dp_gp_params *p) {
   p->dhpwl_ref = 3.5e5f;
   p->init_rms_bins = 0.01f;
   p->max_history = 4096;
+  p->stop_overflow = 0.07f;
 }
 
 dp_status dp_gp_create(dp_ctx *ctx, const dp_gp_params *params, dp_gp **out) {
@@ -406,7 +422,7 @@ dp_status dp_gp_create(dp_ctx *ctx, const dp_gp_params *params, dp_gp **out) {
   if (params) p = *params;
   if (!(p.target_density > 0.f) || !(p.gamma_base_scale > 0.f) || !(p.lambda_scale >= 0.f) ||
       !(p.mu_min > 0.f) || !(p.mu_max >= p.mu_min) || !(p.dhpwl_ref > 0.f) || !(p.init_rms_bins > 0.f) ||
-      p.max_history < 0)
+      p.max_history < 0 || !(p.stop_overflow >= 0.f))
     return dp::fail(DP_ERR_INVALID_ARG, "invalid dp_gp_params");
   dp::GpDeviceGuard guard(c->device);
   Gp *g = new Gp();
@@ -437,6 +453,7 @@ dp_status dp_gp_create(dp_ctx *ctx, const dp_gp_params *params, dp_gp **out) {
   a.mu_min = p.mu_min; a.mu_max = p.mu_max; a.dhpwl_ref = p.dhpwl_ref;
   a.lambda_scale = p.lambda_scale; a.init_rms_bins = p.init_rms_bins; a.bx = c->bx;
   a.hist_cap = p.max_history;
+  a.stop_overflow = p.stop_overflow;
   dp_status st;
   if ((st = dp::gp_alloc(*g, &a.part, 2 * (size_t)a.nblk)) != DP_OK) return bail(st);
   a.oblk = c->num_sms;

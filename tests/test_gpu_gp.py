@@ -142,3 +142,29 @@ def test_gp_adaptec1_spreads():
     hist = loop.history()
     print([(int(h["k"]), round(h["overflow"], 3), h["hpwl"]) for h in hist[::100]])
     assert hist[-1]["overflow"] < 0.3
+
+
+def test_gp_converges_and_stops():
+    """A36: once overflow < stop_overflow (0.07) the device loop freezes: positions, lambda and
+    gamma stay, lambda stays finite (it used to grow without bound past convergence)."""
+    nl = make_netlist("tiny")
+    x, y = make_positions(nl, "initial")
+    ctx = dp.dp_create(nl)
+    loop = dp.GpLoop(ctx)
+    loop.init(_t(x), _t(y))
+    loop.run(600)
+    hist = loop.history()
+    ux, uy = loop.positions()
+    k_stop = next(int(h["k"]) for h in hist if h["overflow"] < 0.07)
+    after = [h for h in hist if h["k"] > k_stop]
+    assert len(after) > 10
+    assert all(h["lam"] == after[0]["lam"] and h["gamma"] == after[0]["gamma"] for h in after)
+    loop.run(2000)
+    ux2, uy2 = loop.positions()
+    assert torch.equal(ux, ux2) and torch.equal(uy, uy2)
+    assert all(math.isfinite(h["lam"]) and math.isfinite(h["hpwl"]) for h in loop.history())
+    # the oracle stops at the same iteration (same trajectory to within the parity tolerance)
+    st = ogp.gp_init(nl, x, y)
+    ref = [ogp.gp_step(nl, st) for _ in range(k_stop + 3)]
+    k_ref = next(int(h["k"]) for h in ref if h["overflow"] < 0.07)
+    assert abs(k_ref - k_stop) <= 3

@@ -113,3 +113,20 @@ def test_gp_loop_spreads_the_initial_placement():
     assert st.lam > lam0
     # cells stay inside the region (A33 clamp)
     assert np.all(st.u[0] >= nl.xl) and np.all(st.u[0] <= nl.xh - nl.cell_w + 1e-9)
+
+
+def test_gp_stops_at_stop_overflow():
+    """A36: once overflow < stop_overflow the loop is converged: positions, lambda and gamma no
+    longer change (previously lambda grew by ~1.05 per iteration without bound)."""
+    nl = make_netlist("tiny")
+    x, y = make_positions(nl, "initial")
+    st = gp.gp_init(nl, x, y)
+    hist = [gp.gp_step(nl, st) for _ in range(500)]
+    k_stop = next(h["k"] for h in hist if h["overflow"] < 0.07)
+    after = [h for h in hist if h["k"] > k_stop]
+    assert len(after) > 10
+    assert all(h["lam"] == after[0]["lam"] and h["gamma"] == after[0]["gamma"] for h in after)
+    assert all(h["hpwl"] == after[0]["hpwl"] for h in after)
+    u = st.u.copy()
+    gp.gp_step(nl, st)
+    assert np.array_equal(u, st.u)

@@ -244,10 +244,7 @@ __global__ void __launch_bounds__(32 * kWRowWarps) k_row_dct_w(const IN *__restr
     mbar_expect_tx(&s_bar[warp], bytes);
     bulk_g2s(stage, in + (size_t)(2 * p0) * N, bytes, &s_bar[warp]);
   }
-  float2 twr[32], phr[K];   // table loads issued while the rows are in flight
-  wfft::load_twiddles<LOGN>(twr, tw2);
-#pragma unroll
-  for (int j = 0; j < K; j++) phr[j] = __ldg(ph + lane + 32 * j);
+  // twiddle / phase tables are read right before use (L1-resident; registers kept low)
   float2 a[32];
   if (tma) {
     __syncwarp();
@@ -276,7 +273,7 @@ __global__ void __launch_bounds__(32 * kWRowWarps) k_row_dct_w(const IN *__restr
       }
     }
   }
-  wfft::warp_fft<LOGN, false>(a, buf, twr);
+  wfft::warp_fft<LOGN, false>(a, buf, tw2);
   const float scale = 2.f / N;
 #pragma unroll
   for (int s = 0; s < B; s++) {
@@ -286,7 +283,7 @@ __global__ void __launch_bounds__(32 * kWRowWarps) k_row_dct_w(const IN *__restr
     for (int j = 0; j < K; j++) {
       const int k = lane + 32 * j;
       const float2 v = dct_post_v(buf[wfft::pad(s * N + k)], buf[wfft::pad(s * N + ((N - k) & (N - 1)))],
-                                  phr[j], scale);
+                                  __ldg(ph + k), scale);
       o0[k] = v.x;
       o1[k] = v.y;
     }
@@ -317,10 +314,7 @@ __global__ void __launch_bounds__(32 * WARPS) k_row_inv_w(RowInvArgs a, const fl
     mbar_expect_tx(&s_bar[warp], bytes);
     bulk_g2s(buf, a.inI + (size_t)r0 * N, bytes, &s_bar[warp]);
   }
-  float2 twr[32], phr[K];   // table loads issued while the rows are in flight
-  wfft::load_twiddles<LOGN>(twr, tw2);
-#pragma unroll
-  for (int j = 0; j < K; j++) phr[j] = __ldg(a.ph + lane + 32 * j);
+  // twiddle / phase tables are read right before use (L1-resident; registers kept low)
   float2 v[32];
   if (a.inI && a.tma) {
     __syncwarp();
@@ -357,11 +351,11 @@ __global__ void __launch_bounds__(32 * WARPS) k_row_inv_w(RowInvArgs a, const fl
       const float pnk = k ? ((a.opA == 2) ? vk.x : vn.x) : 0.f;
       const float qk = (a.opB == 2) ? vn.y : vk.y;
       const float qnk = k ? ((a.opB == 2) ? vk.y : vn.y) : 0.f;
-      v[s * K + j] = inv_pre(pk, qk, pnk, qnk, phr[j]);
+      v[s * K + j] = inv_pre(pk, qk, pnk, qnk, __ldg(a.ph + lane + 32 * j));
     }
   }
   __syncwarp();
-  wfft::warp_fft<LOGN, true>(v, buf, twr);
+  wfft::warp_fft<LOGN, true>(v, buf, tw2);
   if constexpr (TSTORE) {
     constexpr int C = WARPS * B;   // consecutive output columns of this CTA
     const int rc0 = blockIdx.x * C;
@@ -570,14 +564,9 @@ __global__ void __launch_bounds__(32 * kWColWarps) k_col_fwd_w(ColFieldArgs a, f
   const int p0 = gw * B;                           // first column pair
   const int my = a.my, npairs = my / 2;
   if (p0 >= npairs) return;
-  float2 twr[32], phr[K];   // table loads issued with the data loads (one memory latency)
-  float kxr[K];
-  wfft::load_twiddles<LOGM>(twr, tw2);
+  float kxr[K];   // twiddle / phase tables are read right before use (L1-resident)
 #pragma unroll
-  for (int j = 0; j < K; j++) {
-    phr[j] = __ldg(a.ph_x + lane + 32 * j);
-    kxr[j] = __ldg(a.kx + lane + 32 * j);
-  }
+  for (int j = 0; j < K; j++) kxr[j] = __ldg(a.kx + lane + 32 * j);
   float2 z[32];
 #pragma unroll
   for (int s = 0; s < B; s++) {
@@ -589,7 +578,7 @@ __global__ void __launch_bounds__(32 * kWColWarps) k_col_fwd_w(ColFieldArgs a, f
       z[s * K + j] = ok ? __ldg(reinterpret_cast<const float2 *>(a.t + (size_t)src * my) + (p0 + s)) : make_float2(0.f, 0.f);
     }
   }
-  wfft::warp_fft<LOGM, false>(z, buf, twr);
+  wfft::warp_fft<LOGM, false>(z, buf, tw2);
   const float scale = 2.f / M;
   double e = 0.0;
 #pragma unroll
@@ -602,7 +591,7 @@ __global__ void __launch_bounds__(32 * kWColWarps) k_col_fwd_w(ColFieldArgs a, f
     for (int j = 0; j < K; j++) {
       const int u = lane + 32 * j;
       const float2 d = dct_post_v(buf[wfft::pad(s * M + u)], buf[wfft::pad(s * M + ((M - u) & (M - 1)))],
-                                  phr[j], scale);   // (a_2p[u], a_2p+1[u])
+                                  __ldg(a.ph_x + lane + 32 * j), scale);   // (a_2p[u], a_2p+1[u])
       const float kx = kxr[j];
       const double wu = (u == 0) ? 0.25 * M : 0.5 * M;
       const float ik0 = (u == 0 && p == 0) ? 0.f : fast_rcp(kx * kx + ky0 * ky0);   // a_00 / k^2 := 0
@@ -636,14 +625,9 @@ __global__ void __launch_bounds__(32 * kWColWarps) k_col_fields_w(ColFieldArgs a
   const int p0 = gw * B;                           // first column pair
   const int my = a.my, npairs = my / 2;
   if (p0 >= npairs) return;
-  float2 twr[32], phr[K];   // table loads issued with the data loads (one memory latency)
-  float kxr[K];
-  wfft::load_twiddles<LOGM>(twr, tw2);
+  float kxr[K];   // twiddle / phase tables are read right before use (L1-resident)
 #pragma unroll
-  for (int j = 0; j < K; j++) {
-    phr[j] = __ldg(a.ph_x + lane + 32 * j);
-    kxr[j] = __ldg(a.kx + lane + 32 * j);
-  }
+  for (int j = 0; j < K; j++) kxr[j] = __ldg(a.kx + lane + 32 * j);
   float2 z[32];
 #pragma unroll
   for (int s = 0; s < B; s++) {
@@ -655,7 +639,7 @@ __global__ void __launch_bounds__(32 * kWColWarps) k_col_fields_w(ColFieldArgs a
       z[s * K + j] = ok ? __ldg(reinterpret_cast<const float2 *>(a.t + (size_t)src * my) + (p0 + s)) : make_float2(0.f, 0.f);
     }
   }
-  wfft::warp_fft<LOGM, false>(z, buf, twr);
+  wfft::warp_fft<LOGM, false>(z, buf, tw2);
   const float scale = 2.f / M;
   double e = 0.0;
 #pragma unroll
@@ -668,7 +652,7 @@ __global__ void __launch_bounds__(32 * kWColWarps) k_col_fields_w(ColFieldArgs a
     for (int j = 0; j < K; j++) {
       const int u = lane + 32 * j;
       const float2 d = dct_post_v(buf[wfft::pad(s * M + u)], buf[wfft::pad(s * M + ((M - u) & (M - 1)))],
-                                  phr[j], scale);   // (a_2p[u], a_2p+1[u])
+                                  __ldg(a.ph_x + lane + 32 * j), scale);   // (a_2p[u], a_2p+1[u])
       const float kx = kxr[j];
       const double wu = (u == 0) ? 0.25 * M : 0.5 * M;
       const float ik0 = (!ok || (u == 0 && p == 0)) ? 0.f : fast_rcp(kx * kx + ky0 * ky0);   // a_00 / k^2 := 0
@@ -694,10 +678,10 @@ __global__ void __launch_bounds__(32 * kWColWarps) k_col_fields_w(ColFieldArgs a
         const int k = lane + 32 * j;
         const float2 ak = A[s * M + k], ank = k ? A[s * M + M - k] : make_float2(0.f, 0.f);
         // p = A_X reversed (IDXST via eq 8e: x'_t = x_{N-t}, x'_0 = 0), q = A_Y (IDCT)
-        v[s * K + j] = inv_pre(ank.x, ak.y, k ? ak.x : 0.f, ank.y, phr[j]);
+        v[s * K + j] = inv_pre(ank.x, ak.y, k ? ak.x : 0.f, ank.y, __ldg(a.ph_x + lane + 32 * j));
       }
     }
-    wfft::warp_fft<LOGM, true>(v, buf, twr);
+    wfft::warp_fft<LOGM, true>(v, buf, tw2);
 #pragma unroll
     for (int s = 0; s < B; s++) {
 #pragma unroll

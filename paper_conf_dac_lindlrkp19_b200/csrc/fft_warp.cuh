@@ -78,8 +78,11 @@ __device__ __forceinline__ void load_twiddles(float2 (&tw)[32], const float2 *__
 // Warp FFT of B = 1024 / N sequences.  In: a[s K + j] = x_s[lane + 32 j].  tw = this lane's
 // twiddles from load_twiddles (tw2[k2 * 32 + n1] = W_N^{n1 k2}, an fp64-rounded table).  Out: buf[pad(s N + k)] = X_s[k] (unnormalised; INV uses
 // conjugate twiddles).  buf is this warp's kBufPad-entry shared buffer; a[] is clobbered.
+// Twiddles are read from the (L1-resident) table right before use: holding all 31 of them in
+// registers for the whole transform cost ~60 registers per thread, which kept the WA kernel's
+// CTAs off the SMs that run a transform.
 template <int LOGN, bool INV>
-__device__ __forceinline__ void warp_fft(float2 (&a)[32], float2 *buf, const float2 (&tw)[32]) {
+__device__ __forceinline__ void warp_fft(float2 (&a)[32], float2 *buf, const float2 *__restrict__ tw2) {
   constexpr int N = 1 << LOGN, K = N / 32, B = kPts / N, LK = LOGN - 5;
   static_assert(K >= 1 && K <= 32, "warp_fft: N in [32, 1024]");
   const int lane = threadIdx.x & 31;
@@ -92,7 +95,7 @@ __device__ __forceinline__ void warp_fft(float2 (&a)[32], float2 *buf, const flo
       const int k2 = brev_c(m, LK);
       float2 v = a[s * K + m];
       if (k2 != 0) {
-        float2 w = tw[k2];
+        float2 w = __ldg(tw2 + k2 * 32 + lane);
         if (INV) w.y = -w.y;
         v = make_float2(v.x * w.x - v.y * w.y, v.x * w.y + v.y * w.x);
       }

@@ -30,6 +30,8 @@
 #include <algorithm>
 #include <cmath>
 
+#include <cstdlib>
+
 #include "async_copy.cuh"
 #include "dp_internal.h"
 
@@ -772,7 +774,11 @@ int density_walk_grid(int tile) {
     return 0;
   if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o2, k_gather_walk, kTileThreads, walk_smem_bytes(tile)) != cudaSuccess)
     return 0;
-  return sms * std::max(1, std::min(o1, o2));
+  int per_sm = std::max(1, std::min(o1, o2));
+  // DP_WALK_CTAS = k (measurement knob): at most k walker CTAs per SM, leaving shared memory for
+  // the WA kernel that runs beside the scatter and the gather
+  if (const char *e = std::getenv("DP_WALK_CTAS")) per_sm = std::max(1, std::min(per_sm, std::atoi(e)));
+  return sms * per_sm;
 }
 
 // kernels of one evaluation's density map + gather: count, scan, place, scatter, gather, and the

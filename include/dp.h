@@ -106,7 +106,9 @@ dp_status dp_create(const dp_netlist *nl, const dp_grid *grid, int device, dp_ct
  * net's first pin).  The density map is summed over ranks with one ncclAllReduce per
  * evaluation; the Poisson solve is replicated.  nccl_unique_id: 128-byte ncclUniqueId from
  * dp_nccl_unique_id() on rank 0, broadcast by the caller (e.g. torch.distributed); NULL
- * builds a "virtual shard" whose collectives are skipped (tests on one GPU).
+ * builds a "virtual shard" whose collectives are skipped (tests on one GPU).  world = 1 with
+ * a real id gives a one-rank communicator: the whole distributed path (direct launches, every
+ * collective) on one GPU.
  * In a distributed context gx, gy are written only on [cell_begin, cell_end) and the
  * scalar outputs are global (summed over ranks).                                         */
 dp_status dp_create_dist(const dp_netlist *nl, const dp_grid *grid, int device, int rank,

@@ -535,7 +535,9 @@ dp_status create(const dp_netlist *nl, const dp_grid *grid, int device, int rank
   c->device = device;
   c->rank = rank;
   c->world = world;
-  c->dist = world > 1;
+  // a distributed context: several ranks, or one rank with a real NCCL communicator (a 1-rank
+  // dp_create_dist runs every collective of the distributed path on one GPU)
+  c->dist = world > 1 || nccl_id != nullptr;
   c->num_sms = prop.multiProcessorCount;
   c->l2_bytes = prop.l2CacheSize;
   c->num_cells = nl->num_cells;
@@ -651,7 +653,7 @@ dp_status create(const dp_netlist *nl, const dp_grid *grid, int device, int rank
   const int wa_k = (c->n_chunks + c->n_big > 0) ? 1 : 0;   // one kernel: big nets, warp nets, chunks
   c->launches_eval = wa_k + density_launches(*c) + (c->fused_t2 ? 3 : 4) /* T1 T2a T2b T3 */ + 2 /* combine, finalize */;
   c->launches_eval_hpwl = c->launches_eval;
-  if (world > 1 && nccl_id) {
+  if (c->dist && nccl_id) {
     if ((st = nccl_init(*c, nccl_id)) != DP_OK) return bail(st);
   }
   cudaError_t le = cudaDeviceSynchronize();

@@ -337,6 +337,29 @@ def test_virtual_shards_reassemble(world):
     check_map("rho", to_np(rho), to_np(ref_map), rel=1e-6)
 
 
+@pytest.mark.parametrize("name", ["tiny", "adaptec1"])
+def test_one_rank_nccl_context(name):
+    """dp_create_dist with world = 1 and a real NCCL id: the distributed path with every collective
+    (bin-map all-reduce, WA partial and HPWL-limb all-reduces, NCCL loaded with dlopen) runs on
+    one GPU; it must equal the single context: bit-identical density map, HPWL and energy (exact
+    or fixed-order), oracle parity for the rest."""
+    nl = make_netlist(name)
+    x, y = make_positions(nl)
+    xt, yt = _t(x), _t(y)
+    single = dp.dp_create(nl)
+    a = single.eval(xt, yt, nl.bin_w, 1.0, with_hpwl=True)
+    a = {k: (v.clone() if torch.is_tensor(v) else v) for k, v in a.items()}
+    ctx = dp.dp_create_dist(nl, 0, 0, 1, dp.dp_nccl_unique_id())
+    b = ctx.eval(xt, yt, nl.bin_w, 1.0, with_hpwl=True)
+    torch.cuda.synchronize()
+    assert b["hpwl"].item() == a["hpwl"].item() == oracle.hpwl(nl, x, y)
+    assert b["energy"].item() == a["energy"].item()
+    assert torch.equal(ctx.density_map(xt, yt), single.density_map(xt, yt))
+    check_scalar("WA", b["wl"].item(), a["wl"].item(), rel=1e-6)
+    check_vector("gx", to_np(b["gx"]), to_np(a["gx"]))
+    check_vector("gy", to_np(b["gy"]), to_np(a["gy"]))
+
+
 @pytest.mark.slow
 @pytest.mark.parametrize("bins", [256, 2048, 4096])
 def test_bin_sweep_density(bins):

@@ -46,7 +46,7 @@ inline void launch_chain(bool pdl, void (*kernel)(KArgs...), dim3 grid, dim3 blo
 constexpr int kWaThreads = 256;       // threads per WA chunk CTA (8 warps)
 constexpr int kWaPpl = 4;             // pin slots per lane (registers)
 constexpr int kWaMaxDeg = 128;        // nets up to this degree go through the chunk kernel (G <= 32)
-constexpr int kWaChunkPins = 2048;    // max pins per chunk (staged in shared memory)
+constexpr int kWaChunkPins = 4096;    // max pins per chunk (staged in shared memory)
 constexpr int kWaWindow = 1024;       // consecutive cells per chunk window held in shared memory
 constexpr int kBigThreads = 256;      // CTA-per-net kernel for nets > kWaMaxDeg
 constexpr int kBigStage = 4096;       // big-net pins whose exact positions stay in shared memory

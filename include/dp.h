@@ -93,6 +93,9 @@ int32_t dp_version(void);
 /* Validate the netlist and grid, copy them to `device`, reorder pins into the kernels'
  * layout (degree-binned, locality-sorted nets), precompute the per-cell stretched footprint
  * sizes and transform twiddles, allocate scratch.  One-time host-side cost.
+ * Side effect: raises the device's persisting-L2 limit (cudaLimitPersistingL2CacheSize) to
+ * cover the context's gradient / force arena (~35 MB at bigblue4), which the evaluation's
+ * streams mark persisting; the limit is never lowered (DP_L2_PERSIST=0 skips both).
  * Errors: DP_ERR_INVALID_ARG (null, CSR not monotone / out of range, sizes negative or
  * non-finite, degenerate region, stretch not 0/1), DP_ERR_UNSUPPORTED (bin counts),
  * DP_ERR_OUT_OF_MEMORY, DP_ERR_CUDA.  *out is set only on success.                       */

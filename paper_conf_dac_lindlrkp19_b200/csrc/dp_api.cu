@@ -582,8 +582,9 @@ dp_status create(const dp_netlist *nl, const dp_grid *grid, int device, int rank
     c->d_force = c->d_g2 + g2n + (c->cell_begin & 1);
     c->hot_bytes = sizeof(float2) * hot_n;
   }
-  if ((st = dev_alloc(*c, &c->d_part, c->n_wa_part + c->n_en_part + 1)) != DP_OK) return bail(st);
-  if (cudaMemset(c->d_part, 0, sizeof(double) * (c->n_wa_part + c->n_en_part + 1)) != cudaSuccess) return bail(fail(DP_ERR_CUDA, "memset"));
+  // partials: WA [n_wa_part], energy [n_en_part], 1 spare, fast HPWL [n_wa_part] (GP loop)
+  if ((st = dev_alloc(*c, &c->d_part, 2 * c->n_wa_part + c->n_en_part + 1)) != DP_OK) return bail(st);
+  if (cudaMemset(c->d_part, 0, sizeof(double) * (2 * c->n_wa_part + c->n_en_part + 1)) != cudaSuccess) return bail(fail(DP_ERR_CUDA, "memset"));
   if ((st = dev_alloc(*c, &c->d_limbs, kHpwlLimbs + 1)) != DP_OK) return bail(st);
   if (cudaMemset(c->d_limbs, 0, sizeof(unsigned long long) * (kHpwlLimbs + 1)) != cudaSuccess) return bail(fail(DP_ERR_CUDA, "memset"));
   if ((st = dev_alloc(*c, &c->d_scal, 8)) != DP_OK) return bail(st);

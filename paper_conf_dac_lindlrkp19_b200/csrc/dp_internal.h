@@ -177,6 +177,7 @@ struct Ctx {
   GraphKey gkey;
   int wl_model = 0;        // DP_WL_WA / DP_WL_LSE (dp_set_wl_model)
   bool deterministic = false;     // dp_set_deterministic (NEXT-2): WA gradient as exact int64 sums
+  bool hpwl_fast = false;         // GP loop: HPWL from fp32 pin positions fused into the fast WA path (A37)
   bool pdl = true;                // programmatic dependent launch along the density chain (DP_PDL=0: off)
   bool direct = false;            // DP_DIRECT=1: WA and gather add into the caller's gx, gy (no combine pass)
   float *direct_gx = nullptr, *direct_gy = nullptr;   // set for the duration of one eval_body

@@ -136,6 +136,7 @@ __device__ double limbs_to_double(const unsigned long long *L) {
 struct FinArgs {
   const double *part;
   int n_wa, n_en;
+  const double *hp_part;   // fast-HPWL partials (GP loop, reading A37) or null: exact limbs
   unsigned long long *limbs;
   double *scal;   // staging {wl, energy, hpwl, obj}
   double *d_obj, *d_wl, *d_energy, *d_hpwl;
@@ -145,27 +146,32 @@ struct FinArgs {
 };
 
 __global__ void __launch_bounds__(256) k_finalize(FinArgs a) {
-  __shared__ double s_a[256], s_b[256];
+  __shared__ double s_a[256], s_b[256], s_c[256];
   if (a.phase != 1) {
-    double wl = 0.0, en = 0.0;
+    double wl = 0.0, en = 0.0, hp = 0.0;
     // fixed assignment of partials to threads and a fixed tree -> deterministic
     if (a.with_wl)
       for (int i = threadIdx.x; i < a.n_wa; i += 256) wl += a.part[i];
     if (a.with_energy)
       for (int i = threadIdx.x; i < a.n_en; i += 256) en += a.part[a.n_wa + i];
+    if (a.hp_part)
+      for (int i = threadIdx.x; i < a.n_wa; i += 256) hp += a.hp_part[i];
     s_a[threadIdx.x] = wl;
     s_b[threadIdx.x] = en;
+    s_c[threadIdx.x] = hp;
     __syncthreads();
     for (int o = 128; o > 0; o >>= 1) {
       if ((int)threadIdx.x < o) {
         s_a[threadIdx.x] += s_a[threadIdx.x + o];
         s_b[threadIdx.x] += s_b[threadIdx.x + o];
+        s_c[threadIdx.x] += s_c[threadIdx.x + o];
       }
       __syncthreads();
     }
     if (threadIdx.x == 0) {
       a.scal[0] = s_a[0];
       a.scal[1] = s_b[0];
+      a.scal[4] = s_c[0];
     }
   }
   if (a.phase == 0) return;
@@ -174,7 +180,9 @@ __global__ void __launch_bounds__(256) k_finalize(FinArgs a) {
   if (threadIdx.x == 0) {
     const double wl = a.scal[0], en = a.scal[1];
     double hp = __longlong_as_double(0x7ff8000000000000ll);
-    if (a.with_hpwl) {
+    if (a.with_hpwl && a.hp_part) {
+      hp = a.scal[4];
+    } else if (a.with_hpwl) {
       hp = limbs_to_double(a.limbs);
       for (int k = 0; k <= kHpwlLimbs; k++) a.limbs[k] = 0ull;
     }
@@ -211,6 +219,7 @@ void launch_finalize_phase(const Ctx &c, int phase, float lambda, bool with_wl, 
   a.part = c.d_part;
   a.n_wa = c.n_wa_part;
   a.n_en = c.n_en_part;
+  a.hp_part = (with_hpwl && c.hpwl_fast && c.wl_model == DP_WL_WA) ? c.d_part + c.n_wa_part + c.n_en_part + 1 : nullptr;
   a.limbs = c.d_limbs;
   a.scal = c.d_scal;
   a.d_obj = d_obj;

@@ -14,6 +14,9 @@
 //   A33 HPWL / overflow at v; clamp to [xl, xh - w]; v_{-1} = v_0 - eta g_0 (rms 0.01 b_x)
 //   A36 converged once overflow < stop_overflow: later iterations leave the state unchanged;
 //       lambda capped at 1e30
+//   A37 the HPWL the schedule uses (eq 18's p) and the history reports is the "fast HPWL": the
+//       same per-net spans from the fp32 pin positions of the WA pass, summed in fp64 per CTA
+//       (the exact, correctly rounded HPWL stays dp_eval's d_hpwl; they differ by ~1e-7 rel.)
 //
 // B200 design: every step runs on the device.  gamma and lambda live in device memory and
 // the evaluation kernels read them there (Ctx::gamma_dev / lambda_dev), so one iteration —
@@ -370,10 +373,12 @@ dp_status gp_eval(Gp &g, const float *x, const float *y, bool wa, bool den, bool
   Ctx &c = *g.c;
   c.gamma_dev = dev_scalars || (wa && !den) ? &g.dev->f_gamma : nullptr;
   c.lambda_dev = dev_scalars ? &g.dev->f_lambda : nullptr;
+  c.hpwl_fast = true;   // A37: the schedule's HPWL from fp32 pin positions, fused into the WA pass
   const dp_status st = eval_body_ext(c, x, y, 1.f, 1.f, g.a.rgx, g.a.rgy, g.out, g.out + 1, g.out + 2,
                                      wa ? g.out + 3 : nullptr, s, wa, den);
   c.gamma_dev = nullptr;
   c.lambda_dev = nullptr;
+  c.hpwl_fast = false;
   return st;
 }
 

@@ -61,6 +61,7 @@ struct WaArgs {
   const int32_t *big_start, *big_flags, *big_cell;
   const float *big_w, *big_dx, *big_dy;
   int part_offset;
+  int hp_offset;                // MODE 4: fast-HPWL partials at part[hp_offset + the WA partial's index]
   int big_stage;   // pins staged in shared memory per big-net CTA
   int n_huge, n_big, n_warp_blocks;
   WaCaps caps;
@@ -169,12 +170,18 @@ __device__ __forceinline__ void limbs_add(unsigned long long (&L)[kHpwlLimbs + 1
 
 template <int THREADS>
 __device__ void block_flush_scalars(double wl, unsigned long long (&L)[kHpwlLimbs + 1],
-                                    bool hpwl, double *part_slot, unsigned long long *limbs) {
+                                    bool hpwl, double *part_slot, unsigned long long *limbs,
+                                    double hp = 0.0, double *hp_slot = nullptr) {
   __shared__ double s_wl[THREADS / 32];
+  __shared__ double s_hp[THREADS / 32];
   __shared__ unsigned long long s_l[THREADS / 32][kHpwlLimbs + 1];
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
 #pragma unroll
   for (int o = 16; o > 0; o >>= 1) wl += __shfl_xor_sync(0xffffffffu, wl, o);
+  if (hp_slot) {
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) hp += __shfl_xor_sync(0xffffffffu, hp, o);
+  }
   if (hpwl) {
 #pragma unroll
     for (int k = 0; k <= kHpwlLimbs; k++) {
@@ -184,6 +191,7 @@ __device__ void block_flush_scalars(double wl, unsigned long long (&L)[kHpwlLimb
   }
   if (lane == 0) {
     s_wl[warp] = wl;
+    s_hp[warp] = hp;
     if (hpwl)
 #pragma unroll
       for (int k = 0; k <= kHpwlLimbs; k++) s_l[warp][k] = L[k];
@@ -193,6 +201,11 @@ __device__ void block_flush_scalars(double wl, unsigned long long (&L)[kHpwlLimb
     double t = 0.0;
     for (int w = 0; w < THREADS / 32; w++) t += s_wl[w];
     if (part_slot) *part_slot = t;
+    if (hp_slot) {
+      double h = 0.0;
+      for (int w = 0; w < THREADS / 32; w++) h += s_hp[w];
+      *hp_slot = h;
+    }
   }
   if (hpwl && threadIdx.x <= kHpwlLimbs) {
     unsigned long long t = 0;
@@ -361,9 +374,9 @@ __device__ __forceinline__ void wa_group_exact(const WaArgs &a, const WarpGroup 
 //
 // LSE (NEXT-3, reading A27): the same b^+- sums; LSE_e = (x+ - x-) + gamma ln 2 (log2 b+ + log2 b-)
 // and dLSE/dx_i = a_i^+/b^+ - a_i^-/b^-; the c sums are not formed.
-template <int S, bool LSE>
+template <int S, bool LSE, bool HP>
 __device__ __forceinline__ void wa_group_fast(const WaArgs &a, const WarpGroup &wg, const GroupCtx &gc,
-                                              float &wl_acc) {
+                                              float &wl_acc, float &hp_acc) {
   const int glog = wg.g_log2, G = 1 << glog;
   const int gi = gc.lane >> glog, j = gc.lane & (G - 1);
   int d = 0, counted = 0;
@@ -448,6 +461,7 @@ __device__ __forceinline__ void wa_group_fast(const WaArgs &a, const WarpGroup &
   const float mxp = cxp * ibxp, mxm = cxm * ibxm, myp = cyp * ibyp, mym = cym * ibym;  // log2 units
   if (j == 0 && counted) {
     // WL_e = (x+ - x-) + (mu+ - mu-) gamma ln 2   (eq 3 in shifted coordinates)
+    if (HP) hp_acc += (Px - Mx) + (Py - My);   // fast HPWL (GP schedule; reading A37)
     const float ig2 = a.gamma * kLn2;
     wl_acc += we * ((Px - Mx) + (mxp - mxm) * ig2 + (Py - My) + (myp - mym) * ig2);
   }
@@ -484,9 +498,9 @@ __device__ __forceinline__ float tanh_half(float t, float e) {
 // in tests/test_oracle_wa.py::test_two_pin_closed_form).
 //
 // LSE (reading A27): LSE = |delta| + 2 gamma ln(1 + e^-u) per axis and dLSE/dx_2 = sign(delta) tanh(u/2).
-template <bool LSE>
+template <bool LSE, bool HP>
 __device__ __forceinline__ void wa_group_pairs(const WaArgs &a, const WarpGroup &wg, const GroupCtx &gc,
-                                               float &wl_acc) {
+                                               float &wl_acc, float &hp_acc) {
   const int lane = gc.lane;
   if (lane >= wg.nnets) return;
   const int r = gc.deg[wg.net_base + lane];
@@ -510,6 +524,7 @@ __device__ __forceinline__ void wa_group_pairs(const WaArgs &a, const WarpGroup 
     return;
   }
   if (counted) wl_acc += we * (fabsf(ddx) * thx + fabsf(ddy) * thy);
+  if (HP && counted) hp_acc += fabsf(ddx) + fabsf(ddy);
   const float hx = 0.5f * kLn2 * tx, hy = 0.5f * kLn2 * ty;
   const float gx = copysignf(we * fmaf(hx, fmaf(-thx, thx, 1.f), thx), ddx);   // d/dx of pin 1
   const float gy = copysignf(we * fmaf(hy, fmaf(-thy, thy, 1.f), thy), ddy);
@@ -566,6 +581,7 @@ __device__ __forceinline__ void wa_big_net(const WaArgs &a, int net, float4 *s_p
   constexpr bool kGrad = MODE != 2;
   constexpr bool kHpwl = MODE == 1 || MODE == 2;
   constexpr bool kLse = MODE == 3;
+  double hp_b = 0.0;
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   constexpr int NW = kBigThreads / 32;
   const int s0 = a.big_start[net], d = a.big_start[net + 1] - s0;
@@ -651,6 +667,7 @@ __device__ __forceinline__ void wa_big_net(const WaArgs &a, int net, float4 *s_p
     if (tid == 0 && counted) {
       const float spanx = __fadd_rn(__fsub_rn(e.Xh, e.xh), __fsub_rn(e.Xl, e.xl));
       const float spany = __fadd_rn(__fsub_rn(e.Yh, e.yh), __fsub_rn(e.Yl, e.yl));
+      if (MODE == 4) hp_b = (double)(spanx + spany);
       if (kLse)   // reading A27: (x+ + gamma ln b+) - (x- - gamma ln b-)
         wl_acc = (double)(we * ((spanx + spany) + a.gamma * (logf(sm[0]) + logf(sm[2]) + logf(sm[4]) + logf(sm[6]))));
       else
@@ -677,7 +694,7 @@ __device__ __forceinline__ void wa_big_net(const WaArgs &a, int net, float4 *s_p
   }
   __syncthreads();
   block_flush_scalars<kBigThreads>(wl_acc, L, kHpwl, kGrad ? a.part + a.part_offset + net : nullptr,
-                                   a.limbs);
+                                   a.limbs, hp_b, MODE == 4 ? a.part + a.hp_offset + a.part_offset + net : nullptr);
 }
 
 // Warp per net for degrees (kWaMaxDeg, kWarpNetMax]: three passes over the pins with warp
@@ -705,6 +722,7 @@ __device__ __forceinline__ void wa_warp_nets(const WaArgs &a, int wb) {
   constexpr bool kGrad = MODE != 2;
   constexpr bool kHpwl = MODE == 1 || MODE == 2;
   constexpr bool kLse = MODE == 3;
+  double hp_w = 0.0;
   const int lane = threadIdx.x & 31;
   const int net = a.n_huge + wb * (kWarpNetThreads / 32) + (threadIdx.x >> 5);
   double wl_acc = 0.0;
@@ -717,7 +735,7 @@ __device__ __forceinline__ void wa_warp_nets(const WaArgs &a, int wb) {
     const float we = a.has_w ? a.big_w[net] : 1.f;
     const int *cell = a.big_cell + s0;
     const float *pdx = a.big_dx + s0, *pdy = a.big_dy + s0;
-    if (MODE == 0 || MODE == 3) {
+    if (MODE == 0 || MODE == 3 || MODE == 4) {
       float Px = -INFINITY, Mx = INFINITY, Py = -INFINITY, My = INFINITY;
 #pragma unroll 4
       for (int p = lane; p < d; p += 32) {
@@ -748,6 +766,7 @@ __device__ __forceinline__ void wa_warp_nets(const WaArgs &a, int wb) {
       const float mxp = cxp * ibxp, mxm = cxm * ibxm, myp = cyp * ibyp, mym = cym * ibym;   // log2 units
       if (lane == 0 && counted) {
         const float ig2 = a.gamma * kLn2;
+        if (MODE == 4) hp_w = (double)((Px - Mx) + (Py - My));
         if (kLse)
           wl_acc = (double)(we * ((Px - Mx) + (Py - My) + (lg2(bxp) + lg2(bxm) + lg2(byp) + lg2(bym)) * ig2));
         else
@@ -834,10 +853,12 @@ __device__ __forceinline__ void wa_warp_nets(const WaArgs &a, int wb) {
     }
   }
   block_flush_scalars<kWarpNetThreads>(wl_acc, L, kHpwl, kGrad ? a.part + a.part_offset + a.n_huge + wb : nullptr,
-                                       a.limbs);
+                                       a.limbs, hp_w,
+                                       MODE == 4 ? a.part + a.hp_offset + a.part_offset + a.n_huge + wb : nullptr);
 }
 
-// MODE 0: WA + gradient; 1: WA + gradient + HPWL; 2: HPWL only; 3: LSE + gradient (NEXT-3).
+// MODE 0: WA + gradient; 1: WA + gradient + HPWL; 2: HPWL only; 3: LSE + gradient (NEXT-3);
+// 4: WA + gradient + fast HPWL (fp32 pin positions, per-CTA partials; the GP loop, reading A37).
 template <int MODE>
 // 3 CTAs per SM (measured: 4 per SM at 64 registers is slower, 92 vs 86 us alone)
 __global__ void __launch_bounds__(kWaThreads, 3) k_wa_chunks(const WaArgs a0) {
@@ -944,7 +965,7 @@ __global__ void __launch_bounds__(kWaThreads, 3) k_wa_chunks(const WaArgs a0) {
   mbar_wait(bar + 1, 0);
   __syncthreads();
 
-  float wl_acc = 0.f;
+  float wl_acc = 0.f, hp_acc = 0.f;
   unsigned long long L[kHpwlLimbs + 1];
 #pragma unroll
   for (int k = 0; k <= kHpwlLimbs; k++) L[k] = 0ull;
@@ -954,16 +975,16 @@ __global__ void __launch_bounds__(kWaThreads, 3) k_wa_chunks(const WaArgs a0) {
   // warp groups are dealt round-robin (the host orders them by decreasing cost)
   for (int gi = warp; gi < ch.wg_n; gi += kWaThreads / 32) {
     const WarpGroup wg = s_wg[gi];
-    if (MODE == 0 || MODE == 3) {
-      constexpr bool kL = MODE == 3;
+    if (MODE == 0 || MODE == 3 || MODE == 4) {
+      constexpr bool kL = MODE == 3, kH = MODE == 4;
       if (wg.flags & 1) {
-        wa_group_pairs<kL>(a, wg, gc, wl_acc);
+        wa_group_pairs<kL, kH>(a, wg, gc, wl_acc, hp_acc);
       } else {
         switch (wg.slots) {
-          case 1: wa_group_fast<1, kL>(a, wg, gc, wl_acc); break;
-          case 2: wa_group_fast<2, kL>(a, wg, gc, wl_acc); break;
-          case 3: wa_group_fast<3, kL>(a, wg, gc, wl_acc); break;
-          default: wa_group_fast<4, kL>(a, wg, gc, wl_acc); break;
+          case 1: wa_group_fast<1, kL, kH>(a, wg, gc, wl_acc, hp_acc); break;
+          case 2: wa_group_fast<2, kL, kH>(a, wg, gc, wl_acc, hp_acc); break;
+          case 3: wa_group_fast<3, kL, kH>(a, wg, gc, wl_acc, hp_acc); break;
+          default: wa_group_fast<4, kL, kH>(a, wg, gc, wl_acc, hp_acc); break;
         }
       }
     } else {
@@ -1027,7 +1048,8 @@ __global__ void __launch_bounds__(kWaThreads, 3) k_wa_chunks(const WaArgs a0) {
       if (gx | gy) red_v2(a.g2 + s_far[f], gx * inv, gy * inv);
     }
   }
-  block_flush_scalars<kWaThreads>((double)wl_acc, L, kHpwl, kGrad ? a.part + chunk : nullptr, a.limbs);
+  block_flush_scalars<kWaThreads>((double)wl_acc, L, kHpwl, kGrad ? a.part + chunk : nullptr, a.limbs,
+                                  (double)hp_acc, MODE == 4 ? a.part + a.hp_offset + chunk : nullptr);
 }
 
 template <int MODE>
@@ -1053,6 +1075,8 @@ cudaError_t wa_configure(const WaCaps &caps) {
   e = cudaFuncSetAttribute(k_wa_chunks<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, b);
   if (e != cudaSuccess) return e;
   e = cudaFuncSetAttribute(k_wa_chunks<3>, cudaFuncAttributeMaxDynamicSharedMemorySize, b);
+  if (e != cudaSuccess) return e;
+  e = cudaFuncSetAttribute(k_wa_chunks<4>, cudaFuncAttributeMaxDynamicSharedMemorySize, b);
   if (e != cudaSuccess) return e;
   return cudaFuncSetAttribute(k_wa_chunks<2>, cudaFuncAttributeMaxDynamicSharedMemorySize, b);
 }
@@ -1090,6 +1114,7 @@ void launch_wa(const Ctx &c, const float *x, const float *y, float gamma, bool h
   a.big_dx = c.d_big_dx;
   a.big_dy = c.d_big_dy;
   a.part_offset = c.n_chunks;
+  a.hp_offset = c.n_wa_part + c.n_en_part + 1;
   a.n_huge = c.n_huge;
   a.n_big = c.n_big;
   a.n_warp_blocks = (c.n_big - c.n_huge + kWarpNetThreads / 32 - 1) / (kWarpNetThreads / 32);
@@ -1101,6 +1126,8 @@ void launch_wa(const Ctx &c, const float *x, const float *y, float gamma, bool h
   } else if (c.wl_model == DP_WL_LSE) {   // LSE: fast path; a fused HPWL is a second, HPWL-only pass
     launch_mode<3>(c, a, s);
     if (with_hpwl) launch_mode<2>(c, a, s);
+  } else if (with_hpwl && c.hpwl_fast && c.wl_model == DP_WL_WA) {   // GP loop: fast HPWL in the fast path
+    launch_mode<4>(c, a, s);
   } else if (with_hpwl) {
     launch_mode<1>(c, a, s);
   } else {

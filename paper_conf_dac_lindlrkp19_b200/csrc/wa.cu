@@ -498,9 +498,13 @@ __device__ __forceinline__ float tanh_half(float t, float e) {
 // in tests/test_oracle_wa.py::test_two_pin_closed_form).
 //
 // LSE (reading A27): LSE = |delta| + 2 gamma ln(1 + e^-u) per axis and dLSE/dx_2 = sign(delta) tanh(u/2).
-template <bool LSE, bool HP>
+//
+// EX (MODE 1): the exact HPWL of the pair as the exact-HPWL groups form it (TwoSum positions,
+// exact extremes, fp64 span, int64 limbs; reading A7) beside the fp32 closed form for WA.
+template <bool LSE, bool HP, bool EX>
 __device__ __forceinline__ void wa_group_pairs(const WaArgs &a, const WarpGroup &wg, const GroupCtx &gc,
-                                               float &wl_acc, float &hp_acc) {
+                                               float &wl_acc, float &hp_acc,
+                                               unsigned long long (&L)[kHpwlLimbs + 1]) {
   const int lane = gc.lane;
   if (lane >= wg.nnets) return;
   const int r = gc.deg[wg.net_base + lane];
@@ -525,6 +529,19 @@ __device__ __forceinline__ void wa_group_pairs(const WaArgs &a, const WarpGroup 
   }
   if (counted) wl_acc += we * (fabsf(ddx) * thx + fabsf(ddy) * thy);
   if (HP && counted) hp_acc += fabsf(ddx) + fabsf(ddy);
+  if (EX && counted) {
+    float h0x, l0x, h1x, l1x, h0y, l0y, h1y, l1y;
+    two_sum(gc.px[s0], gc.dx[p0], h0x, l0x);
+    two_sum(gc.px[s1], gc.dx[p1], h1x, l1x);
+    two_sum(gc.py[s0], gc.dy[p0], h0y, l0y);
+    two_sum(gc.py[s1], gc.dy[p1], h1y, l1y);
+    const bool ox = pair_gt(h1x, l1x, h0x, l0x), oy = pair_gt(h1y, l1y, h0y, l0y);
+    const double xp = __dadd_rn((double)(ox ? h1x : h0x), (double)(ox ? l1x : l0x));
+    const double xm = __dadd_rn((double)(ox ? h0x : h1x), (double)(ox ? l0x : l1x));
+    const double yp = __dadd_rn((double)(oy ? h1y : h0y), (double)(oy ? l1y : l0y));
+    const double ym = __dadd_rn((double)(oy ? h0y : h1y), (double)(oy ? l0y : l1y));
+    limbs_add(L, __dadd_rn(__dsub_rn(xp, xm), __dsub_rn(yp, ym)));
+  }
   const float hx = 0.5f * kLn2 * tx, hy = 0.5f * kLn2 * ty;
   const float gx = copysignf(we * fmaf(hx, fmaf(-thx, thx, 1.f), thx), ddx);   // d/dx of pin 1
   const float gy = copysignf(we * fmaf(hy, fmaf(-thy, thy, 1.f), thy), ddy);
@@ -978,7 +995,7 @@ __global__ void __launch_bounds__(kWaThreads, 3) k_wa_chunks(const WaArgs a0) {
     if (MODE == 0 || MODE == 3 || MODE == 4) {
       constexpr bool kL = MODE == 3, kH = MODE == 4;
       if (wg.flags & 1) {
-        wa_group_pairs<kL, kH>(a, wg, gc, wl_acc, hp_acc);
+        wa_group_pairs<kL, kH, false>(a, wg, gc, wl_acc, hp_acc, L);
       } else {
         switch (wg.slots) {
           case 1: wa_group_fast<1, kL, kH>(a, wg, gc, wl_acc, hp_acc); break;
@@ -988,6 +1005,10 @@ __global__ void __launch_bounds__(kWaThreads, 3) k_wa_chunks(const WaArgs a0) {
         }
       }
     } else {
+      if (MODE == 1 && (wg.flags & 1)) {   // 2-pin nets: closed-form WA + exact HPWL
+        wa_group_pairs<false, false, true>(a, wg, gc, wl_acc, hp_acc, L);
+        continue;
+      }
       switch (wg.slots) {
         case 1: wa_group_exact<MODE, 1>(a, wg, gc, wl_acc, L); break;
         case 2: wa_group_exact<MODE, 2>(a, wg, gc, wl_acc, L); break;

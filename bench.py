@@ -318,6 +318,14 @@ def run_ours(args, rank, world, local_rank):
         ev[k][1].record(stream)
     torch.cuda.synchronize()
     flushed_ms = sum(a.elapsed_time(b) for a, b in ev) / Kf
+    flushed_pct = np.percentile([a.elapsed_time(b) * 1e3 for a, b in ev], [10, 50, 90]).tolist()
+    # per-call distribution without the flush (median and p10 / p90 of single calls)
+    for k in range(Kf):
+        ev[k][0].record(stream)
+        step()
+        ev[k][1].record(stream)
+    torch.cuda.synchronize()
+    hot_pct = np.percentile([a.elapsed_time(b) * 1e3 for a, b in ev], [10, 50, 90]).tolist()
     # secondary numbers: fused-HPWL evaluation, standalone HPWL, CUDA-graph
     # replay of one evaluation, and the WA stage timed alone (no overlap with the density chain)
     Ks = min(K, 200)
@@ -430,6 +438,9 @@ def run_ours(args, rank, world, local_rank):
             traffic = None
     cfg = workload_config(nl, args.dist, world)
     cfg["l2_flushed_ms_per_step"] = flushed_ms
+    cfg["per_call_us"] = {"hot": dict(zip(("p10", "p50", "p90"), hot_pct)),
+                          "l2_flushed": dict(zip(("p10", "p50", "p90"), flushed_pct)),
+                          "calls": Kf, "note": "one event pair per call (includes the per-call launch gap)"}
     cfg["peak_source"] = peak_src
     out = {
         "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": K, "warmup": args.warmup,

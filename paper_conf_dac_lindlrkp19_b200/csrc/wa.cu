@@ -877,8 +877,9 @@ __device__ __forceinline__ void wa_warp_nets(const WaArgs &a, int wb) {
 // MODE 0: WA + gradient; 1: WA + gradient + HPWL; 2: HPWL only; 3: LSE + gradient (NEXT-3);
 // 4: WA + gradient + fast HPWL (fp32 pin positions, per-CTA partials; the GP loop, reading A37).
 template <int MODE>
-// 3 CTAs per SM (measured: 4 per SM at 64 registers is slower, 92 vs 86 us alone)
-__global__ void __launch_bounds__(kWaThreads, 3) k_wa_chunks(const WaArgs a0) {
+// at least 2 CTAs per SM (4096-pin chunks: shared memory allows 2; the register cap of 3 per SM
+// measured 0.5 % slower, 4 per SM at 64 registers slower still)
+__global__ void __launch_bounds__(kWaThreads, 2) k_wa_chunks(const WaArgs a0) {
   WaArgs a = a0;
   if (a.gamma_dev) {   // uniform branch: the GP loop's gamma lives on the device
     const float g = __ldg(a.gamma_dev);

@@ -14,7 +14,9 @@ COLS = [('gpu__time_duration.sum', 'us'), ('dram__bytes_read.sum', 'rdMB'), ('dr
         ('smsp__average_warps_issue_stalled_wait_per_issue_active.ratio', 'wait'),
         ('smsp__average_warps_issue_stalled_lg_throttle_per_issue_active.ratio', 'lgthr'),
         ('smsp__average_warps_issue_stalled_mio_throttle_per_issue_active.ratio', 'mio'),
-        ('smsp__issue_active.avg.pct_of_peak_sustained_active', 'issue%')]
+        ('smsp__issue_active.avg.pct_of_peak_sustained_active', 'issue%'),
+        ('sm__inst_executed_pipe_xu.avg.pct_of_peak_sustained_active', 'xu%'),       # MUFU (ex2, rcp, lg2)
+        ('lts__t_requests_srcunit_tex_op_red.sum', 'L2red')]                          # global reductions (requests)
 
 
 def main(path, kfilter=None):

@@ -168,17 +168,22 @@ template <bool MASK>
 __global__ void __launch_bounds__(kCountThreads) k_count(DenArgs a) {
   griddep_wait();
   extern __shared__ int s_hist[];
-  const int i0 = blockIdx.x * kCountCells;
   for (int t = threadIdx.x; t < a.ntiles; t += kCountThreads) s_hist[t] = 0;
-  float x[kCellsPerThread], y[kCellsPerThread], w[kCellsPerThread], h[kCellsPerThread];
-  load_cells(a, i0, x, y, w, h);
   __syncthreads();
+  // persistent: one CTA per resident slot walks cell blocks blockIdx.x, + gridDim.x, ... (no
+  // partial last wave) and flushes its histogram once
+  const int nblk = (a.n_own + kCountCells - 1) / kCountCells;
+  for (int blk = blockIdx.x; blk < nblk; blk += gridDim.x) {
+    const int i0 = blk * kCountCells;
+    float x[kCellsPerThread], y[kCellsPerThread], w[kCellsPerThread], h[kCellsPerThread];
+    load_cells(a, i0, x, y, w, h);
 #pragma unroll
-  for (int k = 0; k < kCellsPerThread; k++) {
-    SmallFoot f;
-    const int i = i0 + k * kCountThreads + threadIdx.x;
-    const int t = classify_small(a, x[k], y[k], w[k], h[k], f);
-    if (t >= 0 && (!MASK || (i < a.n_own && selected(a, i)))) atomicAdd(&s_hist[t], 1);
+    for (int k = 0; k < kCellsPerThread; k++) {
+      SmallFoot f;
+      const int i = i0 + k * kCountThreads + threadIdx.x;
+      const int t = classify_small(a, x[k], y[k], w[k], h[k], f);
+      if (t >= 0 && (!MASK || (i < a.n_own && selected(a, i)))) atomicAdd(&s_hist[t], 1);
+    }
   }
   __syncthreads();
   for (int t = threadIdx.x; t < a.ntiles; t += kCountThreads)
@@ -766,6 +771,16 @@ cudaError_t density_configure(int ntiles, int tile) {
 
 // grid of the walkers: every SM filled with as many CTAs as fit (the smaller of the two kernels'
 // occupancies, so both see the same slices)
+// resident CTAs of the persistent count kernel
+int density_count_grid(int ntiles) {
+  int dev = 0, sms = 0, o = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess) return 0;
+  if (cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess) return 0;
+  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o, k_count<false>, kCountThreads, ntiles * 4) != cudaSuccess)
+    return 0;
+  return sms * std::max(1, o);
+}
+
 int density_walk_grid(int tile) {
   int dev = 0, sms = 0, o1 = 0, o2 = 0;
   if (cudaGetDevice(&dev) != cudaSuccess) return 0;
@@ -811,10 +826,11 @@ void launch_density_map(const Ctx &c, const float *x, const float *y, cudaStream
     cudaEventRecord(c.ev_aux_b, aux);
   }
   if (nblk > 0) {
+    const int cgrid = std::min(nblk, c.count_grid > 0 ? c.count_grid : nblk);
     if (a.fixed)
-      launch_chain(c.pdl, k_count<true>, nblk, kCountThreads, ntiles * 4, s, a);
+      launch_chain(c.pdl, k_count<true>, cgrid, kCountThreads, ntiles * 4, s, a);
     else
-      launch_chain(c.pdl, k_count<false>, nblk, kCountThreads, ntiles * 4, s, a);
+      launch_chain(c.pdl, k_count<false>, cgrid, kCountThreads, ntiles * 4, s, a);
     if (c.sched == 3) cudaEventRecord(c.ev_sched, s);   // DP_SCHED=3: WA starts after the count
     launch_chain(c.pdl, k_scan, 1, 1024, 0, s, a);
     if (a.fixed)

@@ -473,6 +473,7 @@ dp_status build_density(Ctx &c, const dp_netlist *nl) {
     DP_CUDA(density_configure(max_tiles, max_tile));
   }
   c.walk_grid = density_walk_grid(c.tile);
+  c.count_grid = density_count_grid(c.tiles_x * c.tiles_y);
   if (c.walk_grid <= 0) return fail(DP_ERR_CUDA, "density walker occupancy query failed");
   {  // DP_WALK_MULT = k: k slices per resident walker slot (finer slices start as SMs free up)
     const char *e = std::getenv("DP_WALK_MULT");

@@ -189,6 +189,7 @@ struct Ctx {
   const float *gamma_dev = nullptr, *lambda_dev = nullptr;
   int sched = 0;           // DP_SCHED: 0 = WA from the fork, 1 = WA after the density map (overlaps the transforms)     // DP_SERIAL=1: density chain after WA (no stream overlap; measurement)
   int32_t walk_grid = 0;
+  int32_t count_grid = 0;           // resident CTAs of the persistent count kernel
   int32_t *d_walk_tile = nullptr;   // [walk_grid]   // CTAs of the persistent scatter / gather walkers (SMs x resident)
   unsigned long long *d_rho = nullptr;  // bin map, int64 fixed point in units of 2^-kRhoScaleLog2 (exact, deterministic)
   float *d_t = nullptr, *d_sx = nullptr, *d_sy = nullptr;
@@ -288,6 +289,7 @@ cudaError_t wa_configure(const WaCaps &caps);
 int wa_smem_bytes(const WaCaps &caps);
 cudaError_t density_configure(int ntiles, int tile);
 int density_walk_grid(int tile);
+int density_count_grid(int ntiles);
 int density_launches(const Ctx &c);
 // NCCL (nccl_dyn.cpp)
 dp_status nccl_get_unique_id(void *out128);

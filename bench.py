@@ -94,6 +94,12 @@ class ClockSampler:
         for line in self.proc.stdout:
             self.samples.append((time.time(), [v.strip() for v in line.split(",")]))
 
+    def wait_first(self, timeout=5.0):
+        """Block until nvidia-smi has emitted its first sample (it takes ~0.5-1 s to start)."""
+        t = time.time()
+        while self.proc and not self.samples and time.time() - t < timeout:
+            time.sleep(0.02)
+
     def stop(self):
         if self.proc:
             self.proc.terminate()
@@ -136,8 +142,8 @@ def workload_config(nl, dist_name, world):
             "cells": nl.num_cells, "nets": nl.num_nets, "pins": nl.num_pins,
             "bins": [nl.bins_x, nl.bins_y], "positions": dist_name, "gamma": nl.bin_w, "lambda": 1.0,
             "hpwl": "not fused (d_hpwl = NULL)",
-            "l2": "not flushed: per-step working set ~280 MB > 126 MB L2 (inputs larger than L2); "
-                  "l2_flushed_ms_per_step = same step after an untimed 2x-L2 write",
+            "l2": "flushed: an untimed write of 2x L2 before every timed step (L2-cold headline, SURVEY "
+                  "§8d); hot back-to-back steps in secondary.hot_back_to_back_evals_per_s",
             "parallelism": f"cells{world} (owner-computes shards, NCCL all-reduce of the bin map)"
                            if world > 1 else "single GPU"}
 
@@ -276,24 +282,64 @@ def run_ours(args, rank, world, local_rank):
         pg.barrier()
     assert all(math.isfinite(v) for v in sc[:3].tolist()), "non-finite objective"
     K = args.steps
-    # headline: K back-to-back steps bracketed by one event pair (barrier + sync on both sides).
-    # The per-step working set (pins 107 MB, nets 9 MB, cells 35 MB, sort records 61 MB, maps
-    # and scratch ~65 MB at bigblue4) exceeds the 126 MB L2, so no flush is inserted.
+
+    def load_for(seconds):   # untimed steps that keep the GPU busy around the timed region
+        t = time.time()
+        while time.time() - t < seconds:
+            for _ in range(50):
+                step()
+            torch.cuda.synchronize()
+
+    def cold_steps(n, fn):   # per-step device ms, each step after an untimed write of 2x L2
+        evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(n)]
+        for k in range(n):
+            flush.zero_()
+            evs[k][0].record(stream)
+            fn()
+            evs[k][1].record(stream)
+        torch.cuda.synchronize()
+        return [a.elapsed_time(b) for a, b in evs]
+
+    # headline (L2-cold): K steps, each preceded by an untimed 2x-L2 write, timed by
+    # one event pair per step on the launching stream; barrier + synchronize on both sides.  The
+    # clock sampler has started and the GPU is kept under load for 0.3 s on either side, so the
+    # nvidia-smi samples bracketing the (milliseconds-long) timed region are taken under load.
+    sampler.wait_first()
+    load_for(0.3)
     torch.cuda.synchronize()
     if pg:
         pg.barrier()
     t0 = time.time()
+    cold = cold_steps(K, step)
+    t1 = time.time()
+    load_for(0.3)
+    if pg:
+        pg.barrier()
+    total_ms = sum(cold)
+    flushed_pct = np.percentile([v * 1e3 for v in cold], [10, 50, 90]).tolist()
+    flushed_ms = total_ms / K
+    clocks = sampler.summary(t0 - 0.3, t1 + 0.3)
+    # secondary: the same steps back to back without the flush (hot L2: the Nesterov steady state)
+    torch.cuda.synchronize()
     h0, h1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     h0.record(stream)
     for _ in range(K):
         step()
     h1.record(stream)
     torch.cuda.synchronize()
-    t1 = time.time()
-    if pg:
-        pg.barrier()
-    total_ms = h0.elapsed_time(h1)
-    clocks = sampler.summary(t0, t1)
+    hot_ms = h0.elapsed_time(h1) / K
+    # secondary: the 'initial' distribution (all cells near the centre: worst-case contention)
+    xi0, yi0 = make_positions(nl, "initial")
+    xit, yit = torch.as_tensor(xi0, device=dev), torch.as_tensor(yi0, device=dev)
+    Ki = min(K, 200)
+
+    def step_initial():
+        dp.dp_eval(ctx, xit, yit, gamma, lam, gx, gy, sc[0:1], sc[1:2], sc[2:3], None, stream)
+
+    for _ in range(3):
+        step_initial()
+    initial_ms = sum(cold_steps(Ki, step_initial)) / Ki
+    step()
     # profiled timed region: the same K steps again with per-stage CUDA events recorded by the
     # library on the stream each stage runs on (dp_profile_*); stage durations and the roofline
     # come from here (the events add a little host/GPU work, so the headline above runs without)
@@ -308,17 +354,8 @@ def run_ours(args, rank, world, local_rank):
     dp.dp_profile_enable(ctx, False)
     stage_ms, n_prof = dp.dp_profile_read(ctx)
     profiled_ms = p0.elapsed_time(p1) / K
-    # secondary: L2 flushed (2x L2 bytes written, untimed) before every timed step
     Kf = min(K, 200)
     ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(Kf)]
-    for k in range(Kf):
-        flush.zero_()
-        ev[k][0].record(stream)
-        step()
-        ev[k][1].record(stream)
-    torch.cuda.synchronize()
-    flushed_ms = sum(a.elapsed_time(b) for a, b in ev) / Kf
-    flushed_pct = np.percentile([a.elapsed_time(b) * 1e3 for a, b in ev], [10, 50, 90]).tolist()
     # per-call distribution without the flush (median and p10 / p90 of single calls)
     for k in range(Kf):
         ev[k][0].record(stream)
@@ -406,11 +443,14 @@ def run_ours(args, rank, world, local_rank):
     e2e_s = time.perf_counter() - e0
     sampler.stop()
 
-    tensors = torch.tensor([total_ms, e2e_s, flushed_ms], dtype=torch.float64, device=dev)
+    tensors = torch.tensor([total_ms, e2e_s, hot_ms], dtype=torch.float64, device=dev)
     if pg:
         pg.all_reduce(tensors, op=pg.ReduceOp.MAX)
-    total_ms, e2e_s, flushed_ms = tensors.tolist()
-    secondary = {"fused_hpwl_evals_per_s": 1e3 / fused_ms, "hpwl_only_per_s": 1e3 / hpwl_ms,
+    total_ms, e2e_s, hot_ms = tensors.tolist()
+    secondary = {"hot_back_to_back_evals_per_s": 1e3 / hot_ms, "hot_ms_per_step": hot_ms,
+                 "initial_evals_per_s": 1e3 / initial_ms, "initial_ms_per_step": initial_ms,
+                 "initial_note": "positions 'initial' (P:153): centres ~ N(W/2, (0.001 W)^2), L2-cold like the headline",
+                 "fused_hpwl_evals_per_s": 1e3 / fused_ms, "hpwl_only_per_s": 1e3 / hpwl_ms,
                  "wl_grad_only_per_s": 1e3 / wl_only_ms,
                  "profiled_ms_per_step": profiled_ms,
                  "graph_replay_evals_per_s": (1e3 / graph_ms) if isinstance(graph_ms, float) else graph_ms,
@@ -437,7 +477,7 @@ def run_ours(args, rank, world, local_rank):
         except Exception:
             traffic = None
     cfg = workload_config(nl, args.dist, world)
-    cfg["l2_flushed_ms_per_step"] = flushed_ms
+    cfg["hot_ms_per_step"] = hot_ms
     cfg["per_call_us"] = {"hot": dict(zip(("p10", "p50", "p90"), hot_pct)),
                           "l2_flushed": dict(zip(("p10", "p50", "p90"), flushed_pct)),
                           "calls": Kf, "note": "one event pair per call (includes the per-call launch gap)"}
@@ -471,11 +511,28 @@ def run_ours(args, rank, world, local_rank):
     return 0
 
 
+def relaunch_under_torchrun(args):
+    """`python bench.py --gpus N` (N > 1) without a launcher: re-execute this script under
+    torch.distributed.run with N ranks on 127.0.0.1, and return its exit status."""
+    import socket
+    with socket.socket() as s:
+        s.bind(("127.0.0.1", 0))
+        port = s.getsockname()[1]
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+           "--master-addr", "127.0.0.1", f"--master-port={port}", os.path.abspath(__file__), *sys.argv[1:]]
+    return subprocess.call(cmd)
+
+
 def main():
     args = parse()
+    if "WORLD_SIZE" not in os.environ and args.gpus > 1:
+        return relaunch_under_torchrun(args)
     rank = int(os.environ.get("RANK", "0"))
     world = int(os.environ.get("WORLD_SIZE", "1"))
     local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    if world != args.gpus:
+        sys.stderr.write(f"bench.py: --gpus {args.gpus} but WORLD_SIZE={world}: refusing to mislabel the run\n")
+        return 2
     if args.impl == "reference":
         return run_reference(args, rank, world)
     return run_ours(args, rank, world, local_rank)

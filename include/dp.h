@@ -243,6 +243,14 @@ dp_status dp_gp_positions(dp_gp *gp, float *x, float *y, dp_stream_t stream);
  * *rows <- rows written.                                                                    */
 dp_status dp_gp_history(dp_gp *gp, double *h_rows, int32_t max_rows, int32_t *rows);
 
+/* Test-only hook (no part of the metric): synchronise and copy the loop state at the start of
+ * the next iteration.  u, v, vp (= v_{k-1}), g (preconditioned gradient at v), gp_prev (at vp):
+ * device, [2 num_cells] (x entries, then y), each may be NULL.  h_scalars (host, [9]):
+ * {a_{k+1}, lambda, gamma, HPWL(v), overflow(v), alpha_k (the next step's), k, converged flag,
+ * Nesterov coefficient (a_k - 1) / a_{k+1}}.                                                 */
+dp_status dp_gp_debug_state(dp_gp *gp, float *u, float *v, float *vp, float *g, float *gp_prev,
+                            double *h_scalars);
+
 /* Free the loop's buffers (synchronises the device).  NULL is accepted. */
 dp_status dp_gp_destroy(dp_gp *gp);
 

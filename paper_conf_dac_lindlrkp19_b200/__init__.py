@@ -37,7 +37,7 @@ EXPORTED_SYMBOLS = [
     "dp_eval_host", "dp_get_info", "dp_debug_density_map", "dp_debug_fields", "dp_debug_transform",
     "dp_profile_enable", "dp_profile_read", "dp_set_wl_model",
     "dp_gp_default_params", "dp_gp_create", "dp_gp_init", "dp_gp_run", "dp_gp_positions",
-    "dp_gp_history", "dp_gp_destroy", "dp_set_deterministic", "dp_set_fixed",
+    "dp_gp_history", "dp_gp_destroy", "dp_gp_debug_state", "dp_set_deterministic", "dp_set_fixed",
 ]
 __all__ += ["dp_profile_enable", "dp_profile_read", "STAGES"]
 STAGES = ["wa", "map", "fields", "gather", "combine", "eval"]
@@ -120,6 +120,7 @@ def lib() -> ctypes.CDLL:
             "dp_gp_positions": [P, P, P, P],
             "dp_gp_history": [P, P, ctypes.c_int32, ctypes.POINTER(I32)],
             "dp_gp_destroy": [P],
+            "dp_gp_debug_state": [P, P, P, P, P, P, P],
         }.items():
             f = getattr(L, name)
             f.argtypes = args
@@ -290,6 +291,19 @@ class GpLoop:
         y = torch.empty_like(x)
         _check(lib().dp_gp_positions(self.handle, _ptr(x), _ptr(y), _stream(stream)))
         return x, y
+
+    def debug_state(self):
+        """dp_gp_debug_state: (dict of [2, N] float32 device tensors u, v, vp, g, gp; scalars)."""
+        import numpy as np
+        import torch
+        n = self.ctx.num_cells
+        dev = self.ctx._dev()
+        vec = {k: torch.empty(2 * n, dtype=torch.float32, device=dev) for k in ("u", "v", "vp", "g", "gp")}
+        sc = np.zeros(9, dtype=np.float64)
+        _check(lib().dp_gp_debug_state(self.handle, *(_ptr(vec[k]) for k in ("u", "v", "vp", "g", "gp")),
+                                       sc.ctypes.data_as(ctypes.c_void_p)))
+        names = ("a_next", "lam", "gamma", "hpwl", "tau", "alpha", "k", "frozen", "coef")
+        return {k: t.view(2, n) for k, t in vec.items()}, dict(zip(names, sc.tolist()))
 
     def history(self, max_rows: int = 1 << 16):
         import numpy as np

@@ -841,12 +841,20 @@ void fields_after_t1(const Ctx &c, cudaStream_t s);
 }
 
 void launch_fields(const Ctx &c, const float *rho, cudaStream_t s) {
+  if (c.fft_cta) {
+    launch_fields_cta(c, rho, false, s);
+    return;
+  }
   // T1: t = DCT_y(rho)
   row_dct<float>(c, rho, c.d_t, s);
   fields_after_t1(c, s);
 }
 
 void launch_fields_fixed(const Ctx &c, cudaStream_t s) {
+  if (c.fft_cta) {
+    launch_fields_cta(c, c.d_rho, true, s);
+    return;
+  }
   row_dct<unsigned long long>(c, c.d_rho, c.d_t, s);
   fields_after_t1(c, s);
 }

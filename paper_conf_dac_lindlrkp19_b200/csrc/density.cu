@@ -21,8 +21,8 @@
 //   D5 gather  same walkers; the (tile+2)^2 float2 field tile is reloaded only where the slice
 //              enters a new tile; each cell's force is written once
 // Large cells (footprint wider than 3 bins) take a CTA-per-cell path with global reds.
-// The tile accumulators (two 32-bit words per bin, 2^-29 resolution) flush into an int64 global
-// map (2^-29 units) with native red.global.add.u64: the density map is exact up to one rounding
+// The tile accumulators (one 32-bit word per bin, 2^-29 units modulo 2^32, wraps carried to the
+// map by the wrapping thread) flush into an int64 global map (2^-29 units) with red.global.add.u64: the density map is exact up to one rounding
 // per contribution and independent of execution order (deterministic; bit-identical after an
 // int64 all-reduce).
 // Footprint geometry is computed in fp64 (B200 runs FP64 at half rate); records hold the
@@ -445,21 +445,6 @@ __device__ __forceinline__ void walk_release(RecStage &st, int c) {
   if ((threadIdx.x & 31) == 0) mbar_arrive(&st.empty[c % kStages]);
 }
 
-// shared-memory reduction without a return value; unconditional (a zero add is cheaper than the
-// branch + reconvergence ptxas emits around a predicated shared atomic)
-__device__ __forceinline__ void red_shared(unsigned *p, unsigned v) {
-  asm volatile("red.shared.add.u32 [%0], %1;" ::"r"(smem_u32(p)), "r"(v) : "memory");
-}
-
-// the same, issued only where `on` (a predicated instruction, no branch): lanes whose bin has no
-// overlap do not occupy the shared-atomic unit (~5 lane-ops / clk / SM, the scatter's bound)
-__device__ __forceinline__ void red_shared2_if(unsigned *p_hi, unsigned *p_lo, unsigned hi, unsigned lo, unsigned on) {
-  asm volatile(
-      "{\n .reg .pred p;\n setp.ne.u32 p, %4, 0;\n @p red.shared.add.u32 [%0], %2;\n @p red.shared.add.u32 [%1], %3;\n}"
-      ::"r"(smem_u32(p_hi)), "r"(smem_u32(p_lo)), "r"(hi), "r"(lo), "r"(on)
-      : "memory");
-}
-
 // overlaps (bin units) of a record's footprint with the 3 bins from its first bin, per axis;
 // clipping makes out-of-map / non-covered overlaps 0
 __device__ __forceinline__ void rec_overlaps(const float4 q, float ox3[3], float oy3[3]) {
@@ -470,8 +455,10 @@ __device__ __forceinline__ void rec_overlaps(const float4 q, float ox3[3], float
   }
 }
 
-// flush the shared (hi, lo) tile into rho and clear it (caller synchronises before and after)
-__device__ __forceinline__ void flush_tile(const DenArgs &a, unsigned *s_hi, unsigned *s_lo, int tile) {
+// flush the shared tile accumulators into rho and clear them (caller synchronises before and
+// after).  Each word holds its bin's sum modulo 2^32 (units 2^-29); the wraps were already added
+// to rho by the threads whose atomic crossed 2^32, so rho + word is the exact int64 sum.
+__device__ __forceinline__ void flush_tile(const DenArgs &a, unsigned *s_acc, int tile) {
   const int P = a.tile + kHalo;
   const int ox = (tile / a.tiles_y) * a.tile, oy = (tile % a.tiles_y) * a.tile;
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = blockDim.x >> 5;
@@ -479,9 +466,8 @@ __device__ __forceinline__ void flush_tile(const DenArgs &a, unsigned *s_hi, uns
     const int gi = ox + i;
     for (int j = lane; j < P; j += 32) {
       const int k = i * P + j;
-      const unsigned long long v = ((unsigned long long)s_hi[k] << kTileLoBits) + (unsigned long long)s_lo[k];
-      s_hi[k] = 0u;
-      s_lo[k] = 0u;
+      const unsigned long long v = (unsigned long long)s_acc[k];
+      s_acc[k] = 0u;
       const int gj = oy + j;
       if (v != 0ull && gi < a.mx && gj < a.my)
         asm volatile("red.global.add.u64 [%0], %1;" ::"l"(a.rho + (size_t)gi * a.my + gj), "l"(v) : "memory");
@@ -489,38 +475,43 @@ __device__ __forceinline__ void flush_tile(const DenArgs &a, unsigned *s_hi, uns
   }
 }
 
-// D4: persistent scatter walker.  The shared tile of (hi, lo) 32-bit words is flushed into the
-// int64 map when the slice moves to another tile and at least every kFlushRecs records.
+// shared-memory add returning the old word (native 32-bit ATOMS.ADD on sm_100a)
+__device__ __forceinline__ unsigned atom_shared_add(unsigned *p, unsigned v) {
+  unsigned old;
+  asm volatile("atom.shared.add.u32 %0, [%1], %2;" : "=r"(old) : "r"(smem_u32(p)), "r"(v) : "memory");
+  return old;
+}
+
+// D4: persistent scatter walker.  Every bin of the (tile+2)^2 shared tile is one 32-bit word
+// accumulating u = floor(v 2^29) (v <= 1, so u <= 2^29) with a native shared atomic add that
+// returns the old word; the (rare) thread whose add wraps past 2^32 adds 2^32 units to the int64
+// map itself.  The word is flushed when the slice leaves the tile.  The map is the exact sum of
+// the per-contribution roundings whatever the order (bit-identical to a flush-per-record scheme).
 __global__ void __launch_bounds__(kTileThreads) k_scatter_walk(DenArgs a) {
   griddep_wait();
   extern __shared__ __align__(16) unsigned char dsm[];
   RecStage &st = *reinterpret_cast<RecStage *>(dsm);
-  unsigned *s_hi = reinterpret_cast<unsigned *>(dsm + rec_stage_bytes());   // 2^-kTileHiBits units
-  unsigned *s_lo = s_hi + (a.tile + kHalo) * (a.tile + kHalo);               // 2^-(hi + lo bits) units
+  unsigned *s_acc = reinterpret_cast<unsigned *>(dsm + rec_stage_bytes());   // 2^-29 units, mod 2^32
   const int P = a.tile + kHalo;
   Walker w;
   if (threadIdx.x == 0) walk_start(a, w, st, false);
-  for (int k = threadIdx.x; k < P * P; k += blockDim.x) {
-    s_hi[k] = 0u;
-    s_lo[k] = 0u;
-  }
+  for (int k = threadIdx.x; k < P * P; k += blockDim.x) s_acc[k] = 0u;
   __syncthreads();
   const float scale_fx = (float)(1u << kRhoScaleLog2);
-  int cur_tile = -1, acc = 0;
+  int cur_tile = -1;
   for (int c = 0;; c++) {
     const int b = c % kStages;
     const WalkChunk cc = walk_next(a, w, st, c, false);
     if (cc.begin >= cc.end) break;
     const int n = cc.end - cc.begin;
     if (cur_tile < 0) cur_tile = cc.tile;
-    if (cc.tile != cur_tile || acc + n > kFlushRecs) {   // uniform: every warp sees the same chunks
+    if (cc.tile != cur_tile) {   // uniform: every warp sees the same chunks
       __syncthreads();   // the tile is complete
-      flush_tile(a, s_hi, s_lo, cur_tile);
+      flush_tile(a, s_acc, cur_tile);
       __syncthreads();   // flushed and cleared
       cur_tile = cc.tile;
-      acc = 0;
     }
-    acc += n;
+    const size_t ox = (size_t)(cur_tile / a.tiles_y) * a.tile, oy = (size_t)(cur_tile % a.tiles_y) * a.tile;
     const RecBuf &B = st.buf[b];
     for (int k = threadIdx.x; k < n; k += blockDim.x) {
       const float4 q = B.rec[cc.off + k];
@@ -535,19 +526,19 @@ __global__ void __launch_bounds__(kTileThreads) k_scatter_walk(DenArgs a) {
         const float rx = r * ox3[di];
 #pragma unroll
         for (int dj = 0; dj < 3; dj++) {
-          // u = floor(v 2^29) < 2^30 (v <= 1; power-of-two scaling is exact), split into
-          // hi = floor(v 2^10) and lo = the low 19 bits (= floor(frac(v 2^10) 2^19))
-          const unsigned u = (unsigned)(rx * oy3[dj]);
-          const unsigned hi = u >> kTileLoBits, lo = u & ((1u << kTileLoBits) - 1u);
-          const int k2 = base + di * P + dj;
-          red_shared2_if(s_hi + k2, s_lo + k2, hi, lo, u);
+          const unsigned u = (unsigned)(rx * oy3[dj]);   // floor(v 2^29) <= 2^29 (power-of-two scaling is exact)
+          const unsigned old = atom_shared_add(s_acc + base + di * P + dj, u);
+          if (old + u < old)   // wrapped: 2^32 units (8 bin areas) go straight to the map
+            asm volatile("red.global.add.u64 [%0], %1;" ::"l"(a.rho + (ox + i0 + di) * a.my + oy + j0 + dj),
+                         "l"(1ull << 32)
+                         : "memory");
         }
       }
     }
     walk_release(st, c);
   }
   __syncthreads();
-  if (cur_tile >= 0) flush_tile(a, s_hi, s_lo, cur_tile);
+  if (cur_tile >= 0) flush_tile(a, s_acc, cur_tile);
 }
 
 // D5: persistent gather walker; the (tile+2)^2 float2 field tile is (re)loaded with one bulk copy

@@ -396,6 +396,14 @@ std::vector<float2> twiddles(int n) {  // exp(-2 pi i k / n), k < n/2, from fp64
   }
   return t;
 }
+std::vector<float2> twiddles_full(int n) {  // exp(-2 pi i k / n), k < n, from fp64 (CTA FFT)
+  std::vector<float2> t(n);
+  for (int k = 0; k < n; k++) {
+    const double a = 2.0 * M_PI * k / n;
+    t[k] = make_float2((float)std::cos(a), (float)-std::sin(a));
+  }
+  return t;
+}
 std::vector<float2> phases(int n) {  // exp(-i pi k / 2n), k < n
   std::vector<float2> t(n);
   for (int k = 0; k < n; k++) {
@@ -453,6 +461,8 @@ dp_status build_density(Ctx &c, const dp_netlist *nl) {
   if ((st = dev_upload(c, &c.d_tw_y, twiddles(c.my))) != DP_OK) return st;
   if ((st = dev_upload(c, &c.d_ph_x, phases(c.mx))) != DP_OK) return st;
   if ((st = dev_upload(c, &c.d_ph_y, phases(c.my))) != DP_OK) return st;
+  if ((st = dev_upload(c, &c.d_twf_x, twiddles_full(c.mx))) != DP_OK) return st;
+  if ((st = dev_upload(c, &c.d_twf_y, twiddles_full(c.my))) != DP_OK) return st;
   if ((st = dev_upload(c, &c.d_tw2_x, twiddles2(c.mx))) != DP_OK) return st;
   if ((st = dev_upload(c, &c.d_tw2_y, twiddles2(c.my))) != DP_OK) return st;
   std::vector<float> kx(c.mx), ky(c.my);
@@ -465,6 +475,7 @@ dp_status build_density(Ctx &c, const dp_netlist *nl) {
   const int m = std::max(c.mx, c.my);
   if (m > max_m || c.mx != c.my) {
     DP_CUDA(dct_configure(std::max(c.mx, max_m), std::max(c.my, max_m)));
+    DP_CUDA(fields_configure());
     max_m = std::max(max_m, m);
   }
   if (ntiles > max_tiles || c.tile > max_tile) {
@@ -570,7 +581,16 @@ dp_status create(const dp_netlist *nl, const dp_grid *grid, int device, int rank
     if ((st = dev_upload(*c, &c->d_cell_pins, pins)) != DP_OK) return bail(st);
   }
   c->n_wa_part = c->n_chunks + c->n_huge + (c->n_big - c->n_huge + kWarpNetThreads / 32 - 1) / (kWarpNetThreads / 32);
-  c->n_en_part = c->my / 2;   // = CTAs of the column-fields kernel (2-column slabs)
+  {   // field transforms: the warp FFT up to 1024 points (fewer instructions, no block barriers:
+      // measured 4599 vs 4041 evals/s at bigblue4 against the CTA FFT), the CTA FFT (fields.cu)
+      // beyond, where the warp FFT does not reach; DP_FFT=1 / 0 forces one (A/B)
+    const char *e = std::getenv("DP_FFT");
+    const bool big = std::max(c->mx, c->my) > 1024;
+    c->fft_cta = fields_cta_ok(c->log2mx, c->log2my) && (e ? e[0] == '1' : big);
+  }
+  // energy partials: one per CTA of the column pass (P2 of the CTA-FFT path; 2-column slabs of
+  // the warp-FFT path)
+  c->n_en_part = c->fft_cta ? p2_ctas(c->mx, c->my) : c->my / 2;
   // one "hot" arena for the two per-cell vectors the combine reads: the WA accumulator g2
   // [num_cells] and the force [n_own + 4] (offset by the parity of cell_begin so that even
   // global cells are 16-byte aligned: the combine reads cell pairs as float4).  It is the
@@ -656,7 +676,7 @@ dp_status create(const dp_netlist *nl, const dp_grid *grid, int device, int rank
     cudaGetLastError();   // best effort: a refused hint leaves the default policy
   }
   const int wa_k = (c->n_chunks + c->n_big > 0) ? 1 : 0;   // one kernel: big nets, warp nets, chunks
-  c->launches_eval = wa_k + density_launches(*c) + (c->fused_t2 ? 3 : 4) /* T1 T2a T2b T3 */ + 2 /* combine, finalize */;
+  c->launches_eval = wa_k + density_launches(*c) + (c->fft_cta ? 3 : c->fused_t2 ? 3 : 4) /* P1 P2 P3 or T1 T2a T2b T3 */ + 2 /* combine, finalize */;
   c->launches_eval_hpwl = c->launches_eval;
   if (c->dist && nccl_id) {
     if ((st = nccl_init(*c, nccl_id)) != DP_OK) return bail(st);

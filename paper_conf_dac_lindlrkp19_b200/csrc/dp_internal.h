@@ -57,14 +57,9 @@ constexpr int kHpwlLimbs = 9;         // limbs 0..kHpwlLimbs (10) of 32-bit digi
 constexpr int kTile = 64;             // density tile = kTile x kTile bins (smaller maps: the map)
 constexpr int kHalo = 2;              // small-cell footprints extend <= 2 bins past their tile
 constexpr int kStageRecs = 512;       // records per staging buffer of the scatter/gather walkers
-constexpr int kFlushRecs = 8192;      // a walker flushes its shared tile at least every 2^13 records
-// Tile bins accumulate each contribution v in (0, 1] as two native 32-bit shared atomics:
-// hi = floor(v 2^kTileHiBits) and lo = floor(frac 2^kTileLoBits); with <= kFlushRecs = 2^13
-// records between flushes neither word can overflow (2^13 * 2^10 < 2^32, 2^13 * (2^19 - 1) < 2^32),
-// and the pair resolves 2^-29.
-constexpr int kTileHiBits = 10;
-constexpr int kTileLoBits = 19;
-constexpr int kRhoScaleLog2 = kTileHiBits + kTileLoBits;   // global bin map: int64 units of 2^-29
+// Tile bins accumulate each contribution v in (0, 1] as u = floor(v 2^29) in one native 32-bit
+// shared atomic (modulo 2^32; the thread whose add wraps carries 2^32 units to the int64 map).
+constexpr int kRhoScaleLog2 = 29;   // global bin map: int64 units of 2^-29
 // per-tile counters / cursors one 128-byte line apart: every CTA of count / place adds to every
 // tile's counter, and counters sharing a line serialise in one L2 slice
 constexpr int kCntStride = 32;
@@ -204,6 +199,8 @@ struct Ctx {
   bool t1_tma = false;                              // DP_T1_TMA=1: bulk-copied rows in the forward row pass (A/B; not faster inside the overlapped step)
   bool fused_t2 = false;                            // DP_FUSED_T2=1: one column kernel (T2) instead of T2a + T2b (A/B)
   float2 *d_sxy = nullptr;                          // T2 -> T3 interleaved (sX, sY) [x][y] (warp-FFT path)
+  float2 *d_twf_x = nullptr, *d_twf_y = nullptr;   // CTA FFT: W_N^k, k < N
+  bool fft_cta = true;                              // fields by the CTA-FFT passes (DP_FFT=0: warp FFT, A/B)
   float2 *d_tw2_x = nullptr, *d_tw2_y = nullptr;   // warp FFT: W_N^{n1 k2} at [k2 * 32 + n1] (N <= 1024)
   float *d_kx = nullptr, *d_ky = nullptr;          // wavenumbers (reading A12)
 
@@ -269,6 +266,11 @@ void launch_rho_to_float(const Ctx &c, float *out, cudaStream_t s);
 void launch_transform(const Ctx &c, int kind, const float *in, float *out, cudaStream_t s);
 void launch_split_fields(const Ctx &c, float *xi_x, float *xi_y, cudaStream_t s);
 void launch_psi(const Ctx &c, const float *rho, float *psi, cudaStream_t s);
+// CTA-FFT field passes (fields.cu): P1 rows, P2 columns (+ energy), P3 rows
+cudaError_t fields_configure();
+bool fields_cta_ok(int log2mx, int log2my);
+int p2_ctas(int mx, int my);
+void launch_fields_cta(const Ctx &c, const void *rho, bool int_map, cudaStream_t s);
 // combine / finalize (finalize.cu)
 dp_status eval_body_ext(Ctx &c, const float *x, const float *y, float gamma, float lambda, float *gx, float *gy,
                         double *d_obj, double *d_wl, double *d_energy, double *d_hpwl, cudaStream_t s, bool do_wa,

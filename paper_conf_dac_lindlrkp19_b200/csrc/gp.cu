@@ -590,6 +590,29 @@ dp_status dp_gp_positions(dp_gp *gp, float *x, float *y, dp_stream_t stream) {
   return dp::ctx_call_end(*g->c, s);
 }
 
+dp_status dp_gp_debug_state(dp_gp *gp, float *u, float *v, float *vp, float *g, float *gp_prev, double *h_scalars) {
+  Gp *G = reinterpret_cast<Gp *>(gp);
+  if (!G || !h_scalars) return dp::fail(DP_ERR_INVALID_ARG, "gp / h_scalars is NULL");
+  dp::GpDeviceGuard guard(G->c->device);
+  DP_CUDA(cudaDeviceSynchronize());
+  const size_t n = (size_t)G->a.n, b = n * sizeof(float);
+  auto pair = [&](float *dst, const float *sx, const float *sy) -> cudaError_t {
+    if (!dst) return cudaSuccess;
+    cudaError_t e = cudaMemcpy(dst, sx, b, cudaMemcpyDeviceToDevice);
+    return e != cudaSuccess ? e : cudaMemcpy(dst + n, sy, b, cudaMemcpyDeviceToDevice);
+  };
+  DP_CUDA(pair(u, G->a.ux, G->a.uy));
+  DP_CUDA(pair(v, G->a.vx, G->a.vy));
+  DP_CUDA(pair(vp, G->a.vpx, G->a.vpy));
+  DP_CUDA(pair(g, G->a.gx, G->a.gy));
+  DP_CUDA(pair(gp_prev, G->a.gpx, G->a.gpy));
+  dp::GpDev d{};
+  DP_CUDA(cudaMemcpy(&d, G->dev, sizeof(d), cudaMemcpyDeviceToHost));
+  const double sc[9] = {d.a, d.lam, d.gamma, d.hpwl, d.tau, d.alpha, (double)d.k, (double)d.frozen, d.coef};
+  for (int i = 0; i < 9; i++) h_scalars[i] = sc[i];
+  return DP_OK;
+}
+
 dp_status dp_gp_history(dp_gp *gp, double *h_rows, int32_t max_rows, int32_t *rows) {
   Gp *g = reinterpret_cast<Gp *>(gp);
   if (!g || !rows || (max_rows > 0 && !h_rows)) return dp::fail(DP_ERR_INVALID_ARG, "gp / rows / h_rows is NULL");

@@ -168,3 +168,45 @@ def test_gp_converges_and_stops():
     ref = [ogp.gp_step(nl, st) for _ in range(k_stop + 3)]
     k_ref = next(int(h["k"]) for h in ref if h["overflow"] < 0.07)
     assert abs(k_ref - k_stop) <= 3
+
+
+@pytest.mark.parametrize("dist", ["initial", "spread"])
+def test_gp_one_step_parity(dist):
+    """One-step parity (the loop is a nonlinear iteration: whole trajectories diverge by design).
+    At every iteration k the oracle's gp_step is seeded with the GPU loop's own state
+    (dp_gp_debug_state: u, v, v_{k-1}, g, g_{k-1}, a, lambda, gamma, HPWL, overflow, alpha) and
+    one oracle step is compared with one GPU step: the history scalars within 1e-4 (the
+    BASELINE tolerance of one evaluation; overflow absolute), the new u and v within 1e-3 of
+    the step's own displacement (plus 4 fp32 ulps of the coordinates)."""
+    nl = make_netlist("tiny")
+    x, y = make_positions(nl, dist)
+    ctx = dp.dp_create(nl)
+    loop = dp.GpLoop(ctx)
+    loop.init(_t(x), _t(y))
+    worst = 0.0
+    for k in range(12):
+        vec, sc = loop.debug_state()
+        f64 = {n: vec[n].cpu().numpy().astype(np.float64) for n in vec}
+        an = sc["a_next"]
+        a_prev = math.sqrt(max(((2.0 * an - 1.0) ** 2 - 1.0) / 4.0, 0.0))   # a_k from a_{k+1} (A28)
+        st = ogp.GpState(u=f64["u"], v=f64["v"], vp=f64["vp"], g=f64["g"], gp=f64["gp"], a=a_prev,
+                         lam=sc["lam"], gamma=sc["gamma"], hpwl=sc["hpwl"], tau=sc["tau"], alpha=sc["alpha"],
+                         k=int(sc["k"]), frozen=bool(sc["frozen"]))
+        assert st.k == k
+        ref = ogp.gp_step(nl, st)
+        loop.run(1)
+        h = loop.history()[-1]
+        assert int(h["k"]) == k
+        for key in ("hpwl", "lam", "gamma", "obj", "alpha", "wl"):
+            e = abs(h[key] - ref[key]) / max(abs(ref[key]), 1e-30)
+            worst = max(worst, e)
+            assert e <= 1e-4, (k, key, h[key], ref[key], e)
+        assert abs(h["overflow"] - ref["overflow"]) <= 1e-4, (k, h["overflow"], ref["overflow"])
+        vec2, _ = loop.debug_state()
+        for name, r in (("u", st.u), ("v", st.v)):
+            got = vec2[name].cpu().numpy().astype(np.float64)
+            step = np.abs(r - f64["v"]).max()
+            ulp = 4 * np.spacing(np.float32(np.abs(r).max())).astype(np.float64)
+            err = np.abs(got - r).max()
+            assert err <= 1e-3 * step + ulp, (k, name, err, step)
+    print("worst relative history error over 12 one-step comparisons:", worst)

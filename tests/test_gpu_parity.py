@@ -76,6 +76,24 @@ def test_fields_tiny(tiny):
     check_scalar("energy", f["energy"].item(), oracle.energy(nl, rho32, psi))
 
 
+@pytest.mark.parametrize("mx,my", [(16, 16), (32, 32), (128, 128), (512, 512), (1024, 1024), (32, 128),
+                                   (256, 64), (2048, 2048)])
+def test_fields_sizes(mx, my):
+    """The three CTA-FFT passes (P1 rows, P2 columns + energy, P3 rows; fields.cu) on random maps
+    of every radix plan (16 = 2 x 8, 32 = 4 x 8, 128 = 2 x 8 x 8, 512 = 8^3, 1024 = 2 x 8^3,
+    2048 = 4 x 8^3), square and rectangular, against eqs 9a-9d via the naive eq 7a/7b/8a."""
+    W, H = 10.0 * mx, 7.0 * my
+    nl = custom_netlist([0], [], [], [], [1.0], [1.0], (0, 0, W, H), (mx, my))
+    ctx = dp.dp_create(nl)
+    rho = np.random.default_rng(mx * 7 + my).random((mx, my)) * 2.0
+    f = ctx.fields(_t(rho))
+    rho32 = rho.astype(np.float32).astype(np.float64)
+    psi, xi_x, xi_y = oracle.fields(nl, oracle.dct2(rho32))
+    check_map("xi_x", to_np(f["xi_x"]), xi_x)
+    check_map("xi_y", to_np(f["xi_y"]), xi_y)
+    check_scalar("energy", f["energy"].item(), oracle.energy(nl, rho32, psi))
+
+
 # ------------------------------------------------------------------------------ wirelength
 @pytest.mark.parametrize("gscale", [0.05, 0.5, 5.0, 50.0])
 @pytest.mark.parametrize("weighted", [False, True])

@@ -130,3 +130,71 @@ def test_gp_stops_at_stop_overflow():
     u = st.u.copy()
     gp.gp_step(nl, st)
     assert np.array_equal(u, st.u)
+
+
+def test_precondition_closed_form():
+    """A29 on a hand-counted netlist: nets (c0, c1) weight 3 and (c0, c2) weight 0.5 give net-
+    weighted pin counts P = (3.5, 3, 0.5); areas A = (8, 1, 0.25); at lambda = 0.25 the divisors
+    max(1, P + lambda A) are (5.5, 3.25, 1) — the third clipped at 1."""
+    nl = custom_netlist([0, 2, 4], [0, 1, 0, 2], [0.0] * 4, [0.0] * 4, [4.0, 1.0, 0.5], [2.0, 1.0, 0.5],
+                        (0, 0, 160.0, 160.0), (16, 16), net_weight=[3.0, 0.5])
+    gx = np.array([1.0, -2.0, 3.0])
+    gy = np.array([-0.5, 0.25, 7.0])
+    px, py = gp.precondition(nl, gx, gy, 0.25)
+    d = np.array([5.5, 3.25, 1.0])
+    np.testing.assert_allclose(px, gx / d, rtol=1e-15)
+    np.testing.assert_allclose(py, gy / d, rtol=1e-15)
+    # lambda = 0: the divisor is the pin count, never below 1
+    px0, _ = gp.precondition(nl, gx, gy, 0.0)
+    np.testing.assert_allclose(px0, gx / np.array([3.5, 3.0, 1.0]), rtol=1e-15)
+
+
+def _two_cell_netlist():
+    """Two 12 x 12 cells joined by one 2-pin net with pins at the cell centres (b = 10)."""
+    return custom_netlist([0, 2], [0, 1], [6.0, 6.0], [6.0, 6.0], [12.0, 12.0], [12.0, 12.0],
+                          (0, 0, 160.0, 160.0), (16, 16))
+
+
+def test_gp_init_lambda0_against_closed_form_wa_gradient():
+    """A32: lambda_0 = 8e-5 |grad WA|_1 / |grad D|_1 at the (clamped) start, gamma_0 = gamma(tau_0).
+    |grad WA|_1 from the 2-pin closed form (dWA/dx_2 = sign(delta) [tanh(t/2) +
+    (t/2) sech^2(t/2)], t = |delta| / gamma, per axis; the other pin the negative) — not from
+    oracle.wa; |grad D|_1 from the density oracle (pinned by its own adjoint / mirror /
+    convergence tests).  A wrong norm (L2), the WL value instead of its gradient, or a wrong
+    scale fails this."""
+    nl = _two_cell_netlist()
+    x = np.array([30.0, 100.0], np.float32)
+    y = np.array([40.0, 90.0], np.float32)
+    st = gp.gp_init(nl, x, y)
+    tau0 = gp.overflow(nl, oracle.density_map(nl, x, y), 1.0)
+    gamma0 = gp.gamma_of(nl, tau0, gp.GpParams())
+    assert st.tau == pytest.approx(tau0, rel=1e-12) and st.gamma == pytest.approx(gamma0, rel=1e-12)
+
+    def pin_grad(delta):
+        t = abs(delta) / gamma0
+        return math.copysign(math.tanh(t / 2) + (t / 2) / math.cosh(t / 2) ** 2, delta)
+
+    l1_wa = 2 * abs(pin_grad(70.0)) + 2 * abs(pin_grad(50.0))
+    _, gdx, gdy, _ = oracle.density(nl, x, y, 1)
+    l1_d = np.abs(gdx).sum() + np.abs(gdy).sum()
+    assert st.lam == pytest.approx(8e-5 * l1_wa / l1_d, rel=1e-10)
+
+
+def test_gp_init_first_lipschitz_point():
+    """A33: v_{-1} = v_0 - eta g_0 with an rms displacement of exactly 0.01 b_x, along -g_0
+    (g_0 = the preconditioned gradient at v_0, lambda_0); u_0 = v_0 = the clamped start."""
+    nl = make_netlist("tiny")
+    x, y = make_positions(nl, "spread")
+    x = x.astype(np.float64)
+    x[0] = nl.xh + 50.0                       # outside: clamped to xh - w
+    st = gp.gp_init(nl, x, y)
+    assert st.v[0][0] == nl.xh - float(nl.cell_w[0])
+    d = st.v - st.vp
+    rms = math.sqrt(float(np.sum(d * d)) / d.size)
+    assert rms == pytest.approx(0.01 * nl.bin_w, rel=1e-12)
+    r = oracle.evaluate(nl, st.v[0], st.v[1], st.gamma, st.lam, with_hpwl=False)
+    g0 = np.stack(gp.precondition(nl, r["gx"], r["gy"], st.lam))
+    eta = float(np.sum(d * g0)) / float(np.sum(g0 * g0))
+    assert eta > 0
+    np.testing.assert_allclose(d, eta * g0, rtol=1e-12, atol=1e-12 * np.abs(d).max())
+    assert np.array_equal(st.u, st.v) and st.a == 1.0 and st.k == 0

@@ -101,19 +101,28 @@ int32_t dp_version(void);
  * DP_ERR_OUT_OF_MEMORY, DP_ERR_CUDA.  *out is set only on success.                       */
 dp_status dp_create(const dp_netlist *nl, const dp_grid *grid, int device, dp_ctx **out);
 
-/* Distributed context for rank `rank` of `world` (one process per GPU).  Every rank passes
- * the full netlist; the library keeps the cells [cell_begin, cell_end) of this rank
- * (contiguous, balanced) and every net with at least one pin on them ("owner computes":
- * a net cut by the partition is evaluated on each rank it touches, each rank writes only
- * its own cells' gradient, and WA / HPWL of a net are counted once, on the rank owning the
- * net's first pin).  The density map is summed over ranks with one ncclAllReduce per
- * evaluation; the Poisson solve is replicated.  nccl_unique_id: 128-byte ncclUniqueId from
- * dp_nccl_unique_id() on rank 0, broadcast by the caller (e.g. torch.distributed); NULL
- * builds a "virtual shard" whose collectives are skipped (tests on one GPU).  world = 1 with
- * a real id gives a one-rank communicator: the whole distributed path (direct launches, every
- * collective) on one GPU.
- * In a distributed context gx, gy are written only on [cell_begin, cell_end) and the
- * scalar outputs are global (summed over ranks).                                         */
+/* Distributed context for rank `rank` of `world` (one process per GPU; BASELINE north_star:
+ * "nets are partitioned for WA, with the cell-gradient vector reduced; cells are partitioned for
+ * the density scatter, with the bin map all-reduced").  Every rank passes the full netlist.
+ * WA: the WA work units (nets of degree > 1024 one each, blocks of 8 nets of degree 129..1024,
+ * chunks of <= 4096 pins of the smaller nets in locality order; a pure function of the
+ * netlist) are split into contiguous pin-balanced ranges, one per rank; each rank evaluates
+ * its units' nets (each net on exactly one rank) into a gradient over all cells, summed into
+ * per-rank cell blocks by one ncclReduceScatter.  Cells: rank r owns the block
+ * [r B, min((r+1) B, num_cells)), B = ceil(num_cells / world), for the density scatter, the
+ * force gather and the output.  The int64 bin map is summed with one ncclAllReduce (exact);
+ * the Poisson solve is replicated (maps up to 1024^2) or row-sharded (larger maps).  The WA
+ * partials (one slot per unit, written by one rank) and the HPWL limbs are all-reduced exactly,
+ * so WA, D and HPWL are bit-identical for every world size, and in deterministic mode
+ * (dp_set_deterministic) so is the gradient.
+ * nccl_unique_id: 128-byte ncclUniqueId from dp_nccl_unique_id() on rank 0, broadcast by the
+ * caller (e.g. torch.distributed); NULL builds a "virtual shard" whose collectives are skipped
+ * (tests on one GPU): its gx, gy then hold the shard's partial WA gradient on every cell plus
+ * lambda times the force on its own cells (the sum over shards is the full gradient).  world
+ * = 1 with a real id gives a one-rank communicator: the whole distributed path (direct
+ * launches, every collective) on one GPU.
+ * In a distributed context gx, gy are written only on [cell_begin, cell_end) and the scalar
+ * outputs are global.                                                                       */
 dp_status dp_create_dist(const dp_netlist *nl, const dp_grid *grid, int device, int rank,
                          int world, const void *nccl_unique_id, dp_ctx **out);
 
@@ -121,9 +130,9 @@ dp_status dp_create_dist(const dp_netlist *nl, const dp_grid *grid, int device, 
 dp_status dp_nccl_unique_id(void *out128);
 
 /* Host-only partition plan used by dp_create_dist (no GPU needed; exposed for tests).
- * cell range of `rank` -> *cell_begin, *cell_end.  net_mask (host, [num_nets], nullable)
- * receives per net: 0 = not evaluated on this rank, 1 = evaluated (gradient for own cells
- * only), 3 = evaluated and counted (WA, HPWL) on this rank.                               */
+ * cell block of `rank` -> *cell_begin, *cell_end.  net_mask (host, [num_nets], nullable)
+ * receives per net: 3 = evaluated and counted (WA, HPWL, gradient) on this rank, 0 = not
+ * (every net of degree >= 2 has 3 on exactly one rank).                                      */
 dp_status dp_partition_plan(const dp_netlist *nl, int rank, int world, int32_t *cell_begin,
                             int32_t *cell_end, uint8_t *net_mask);
 
@@ -306,6 +315,22 @@ dp_status dp_debug_fields(dp_ctx *ctx, const float *rho, float *psi, float *xi_x
 enum { DP_T_DCT2 = 0, DP_T_IDCT2 = 1, DP_T_IDXST_IDCT = 2, DP_T_IDCT_IDXST = 3 };
 dp_status dp_debug_transform(dp_ctx *ctx, int kind, const float *in, float *out,
                              dp_stream_t stream);
+
+/* The row-sharded Poisson solve of `world` ranks emulated on one GPU (test hook):
+ * the same kernels with the per-rank layouts, the reduce-scatter / all-to-all / all-gather
+ * replaced by device copies.  rho (device, [bins_x*bins_y] float); xi_x, xi_y (device,
+ * nullable) and d_energy (device double, nullable) as dp_debug_fields.  Errors:
+ * DP_ERR_UNSUPPORTED when the map is not shardable (maps of the warp-FFT path, bins not
+ * divisible by world into whole CTA blocks).                                                 */
+dp_status dp_debug_sharded_fields(dp_ctx *ctx, int32_t world, const float *rho, float *xi_x, float *xi_y,
+                                  double *d_energy, dp_stream_t stream);
+
+/* The WA gradient accumulator of the last evaluation (test hook): out (device)
+ * <- in deterministic mode the int64 sums in units 2^-30 ([2 n] long long: x, y per cell),
+ * otherwise the fp32 sums ([2 n] float); n = num_cells, or world * ceil(num_cells / world)
+ * for a distributed context (a virtual shard's partial sums before the skipped
+ * reduce-scatter).  *n_out <- n.  Synchronises the stream.                                  */
+dp_status dp_debug_wa_accumulator(dp_ctx *ctx, void *out, int64_t *n_out, dp_stream_t stream);
 
 #ifdef __cplusplus
 }

@@ -63,6 +63,15 @@ def lib():
         L.or_density_grad.argtypes = [I64, P, P, P, P, D, D, D, D, I32, I32, I32, P, P, P, P]
         L.or_transform_lastaxis.restype = None
         L.or_transform_lastaxis.argtypes = [I32, I64, I32, P, P]
+        # timed mode (CPU baseline)
+        L.or_wa_omp.restype = D
+        L.or_wa_omp.argtypes = [I32, I64, P, P, P, P, P, P, P, D, P, P]
+        L.or_density_map_omp.restype = None
+        L.or_density_map_omp.argtypes = [I32, I64, P, P, P, P, D, D, D, D, I32, I32, I32, P]
+        L.or_density_grad_omp.restype = None
+        L.or_density_grad_omp.argtypes = [I32, I64, P, P, P, P, D, D, D, D, I32, I32, I32, P, P, P, P]
+        L.or_transform_fft.restype = None
+        L.or_transform_fft.argtypes = [I32, I32, I64, I32, P, P]
         _lib = L
     return _lib
 
@@ -228,3 +237,49 @@ def evaluate(nl, x, y, gamma: float, lam: float, stretch: int = 1, with_hpwl: bo
     if with_hpwl:
         out["hpwl"] = hpwl(nl, x, y)
     return out
+
+
+# --------------------------------------------------------------------------------------
+# Timed mode: the CPU baseline of BASELINE.md §4 (never used for parity).  The same
+# definitions with OpenMP over nets / cells at the paper's chunk sizes |E|/(T 16), |V|/(T 16)
+# and fp64 Makhoul FFT transforms; validated against the plain functions
+# above by tests/test_oracle_timed.py.
+# --------------------------------------------------------------------------------------
+def transform_fft(kind: int, arr: np.ndarray, axis: int, threads: int) -> np.ndarray:
+    a = np.moveaxis(np.asarray(arr, dtype=np.float64), axis, -1)
+    shape = a.shape
+    src = np.ascontiguousarray(a.reshape(-1, shape[-1]))
+    out = np.empty_like(src)
+    lib().or_transform_fft(int(threads), int(kind), src.shape[0], src.shape[1], _p(src), _p(out))
+    return np.moveaxis(out.reshape(shape), -1, axis)
+
+
+def evaluate_timed(nl, x, y, gamma: float, lam: float, threads: int, stretch: int = 1):
+    """obj = WA + lambda D and its gradient (eq 2) in the timed mode; returns the same keys as
+    evaluate() minus the intermediate maps."""
+    xd, yd = _f64(x), _f64(y)
+    gwx = np.zeros(nl.num_cells)
+    gwy = np.zeros(nl.num_cells)
+    wl = lib().or_wa_omp(int(threads), nl.num_nets, _p(_i32(nl.net_start)), _p(_i32(nl.pin2cell)),
+                         _p(_f64(nl.pin_dx)), _p(_f64(nl.pin_dy)),
+                         None if nl.net_weight is None else _p(_f64(nl.net_weight)),
+                         _p(xd), _p(yd), float(gamma), _p(gwx), _p(gwy))
+    w, h = _f64(nl.cell_w), _f64(nl.cell_h)
+    rho = np.zeros((nl.bins_x, nl.bins_y))
+    lib().or_density_map_omp(int(threads), nl.num_cells, _p(xd), _p(yd), _p(w), _p(h), nl.xl, nl.yl, nl.xh,
+                             nl.yh, nl.bins_x, nl.bins_y, int(stretch), _p(rho))
+    a = transform_fft(DCT, transform_fft(DCT, rho, 1, threads), 0, threads)
+    ku, kv = wavenumbers(nl)
+    k2 = ku[:, None] ** 2 + kv[None, :] ** 2
+    inv = np.zeros_like(k2)
+    inv[k2 > 0] = 1.0 / k2[k2 > 0]
+    psi = transform_fft(IDCT, transform_fft(IDCT, a * inv, 1, threads), 0, threads)
+    xi_x = transform_fft(IDXST, transform_fft(IDCT, a * ku[:, None] * inv, 1, threads), 0, threads)
+    xi_y = transform_fft(IDCT, transform_fft(IDXST, a * kv[None, :] * inv, 1, threads), 0, threads)
+    D = energy(nl, rho, psi)
+    gdx = np.empty(nl.num_cells)
+    gdy = np.empty(nl.num_cells)
+    lib().or_density_grad_omp(int(threads), nl.num_cells, _p(xd), _p(yd), _p(w), _p(h), nl.xl, nl.yl, nl.xh,
+                              nl.yh, nl.bins_x, nl.bins_y, int(stretch), _p(np.ascontiguousarray(xi_x)),
+                              _p(np.ascontiguousarray(xi_y)), _p(gdx), _p(gdy))
+    return dict(obj=wl + lam * D, wl=wl, energy=D, gx=gwx + lam * gdx, gy=gwy + lam * gdy)

@@ -357,4 +357,209 @@ void or_transform_lastaxis(int kind, int64_t rows, int n, const double *in, doub
     free(tab);
 }
 
+
+/* ====================================================================================
+ * TIMED MODE (the CPU baseline of BASELINE.md §4; never used for parity).
+ * The same definitions as above, organised for speed the way the paper's CPU version runs
+ * them: OpenMP over nets and over cells with dynamic scheduling and the paper's chunk sizes
+ * |E| / (T 16) and |V| / (T 16), atomic accumulation of the cell gradient and
+ * of the bin map, and the 1-D transforms by a textbook fp64 N-point FFT in Makhoul's order
+ * (Alg 3) instead of the naive O(N^2) sums.  tests/test_oracle_timed.py checks
+ * every function here against the plain functions above.
+ * ==================================================================================== */
+#include <omp.h>
+
+static int64_t chunk_of(int64_t n, int threads)
+{
+    int64_t c = n / ((int64_t)threads * 16);
+    return c > 0 ? c : 1;
+}
+
+double or_wa_omp(int threads, int64_t num_nets, const int32_t *net_start, const int32_t *pin2cell,
+                 const double *pin_dx, const double *pin_dy, const double *net_weight,
+                 const double *x, const double *y, double gamma, double *gx, double *gy)
+{
+    int dmax = 1;
+    for (int64_t e = 0; e < num_nets; e++) {
+        int d = net_start[e + 1] - net_start[e];
+        if (d > dmax) dmax = d;
+    }
+    const int64_t chunk = chunk_of(num_nets, threads);
+    double total = 0.0;
+#pragma omp parallel num_threads(threads) reduction(+ : total)
+    {
+        size_t n = (size_t)dmax;
+        double *px = malloc(n * sizeof(double)), *py = malloc(n * sizeof(double));
+        double *gxp = malloc(n * sizeof(double)), *gyp = malloc(n * sizeof(double));
+        double *ap = malloc(n * sizeof(double)), *am = malloc(n * sizeof(double));
+#pragma omp for schedule(dynamic, chunk)
+        for (int64_t e = 0; e < num_nets; e++) {
+            int s = net_start[e], d = net_start[e + 1] - s;
+            for (int i = 0; i < d; i++) {
+                int c = pin2cell[s + i];
+                px[i] = x[c] + pin_dx[s + i];
+                py[i] = y[c] + pin_dy[s + i];
+            }
+            double we = net_weight ? net_weight[e] : 1.0;
+            total += we * (wa_axis(d, px, gamma, gxp, ap, am) + wa_axis(d, py, gamma, gyp, ap, am));
+            for (int i = 0; i < d; i++) {
+                int c = pin2cell[s + i];
+#pragma omp atomic
+                gx[c] += we * gxp[i];
+#pragma omp atomic
+                gy[c] += we * gyp[i];
+            }
+        }
+        free(px); free(py); free(gxp); free(gyp); free(ap); free(am);
+    }
+    return total;
+}
+
+void or_density_map_omp(int threads, int64_t num_cells, const double *x, const double *y,
+                        const double *w, const double *h, double xl, double yl, double xh, double yh,
+                        int mx, int my, int stretch, double *rho)
+{
+    double bx = (xh - xl) / mx, by = (yh - yl) / my;
+    const int64_t chunk = chunk_of(num_cells, threads);
+#pragma omp parallel for num_threads(threads) schedule(dynamic, chunk)
+    for (int64_t c = 0; c < num_cells; c++) {
+        footprint f = cell_footprint(x[c], y[c], w[c], h[c], xl, yl, xh, yh, bx, by, stretch);
+        if (f.hi_x <= f.lo_x || f.hi_y <= f.lo_y || f.r == 0.0) continue;
+        int i0, i1, j0, j1;
+        bin_range(f.lo_x, f.hi_x, xl, bx, mx, &i0, &i1);
+        bin_range(f.lo_y, f.hi_y, yl, by, my, &j0, &j1);
+        for (int i = i0; i <= i1; i++) {
+            double ox = overlap_1d(f.lo_x, f.hi_x, xl, bx, i);
+            if (ox <= 0.0) continue;
+            for (int j = j0; j <= j1; j++) {
+                double oy = overlap_1d(f.lo_y, f.hi_y, yl, by, j);
+                if (oy <= 0.0) continue;
+#pragma omp atomic
+                rho[(int64_t)i * my + j] += f.r * ox * oy / (bx * by);
+            }
+        }
+    }
+}
+
+void or_density_grad_omp(int threads, int64_t num_cells, const double *x, const double *y,
+                         const double *w, const double *h, double xl, double yl, double xh, double yh,
+                         int mx, int my, int stretch, const double *xi_x, const double *xi_y,
+                         double *gx, double *gy)
+{
+    double bx = (xh - xl) / mx, by = (yh - yl) / my;
+    const int64_t chunk = chunk_of(num_cells, threads);
+#pragma omp parallel for num_threads(threads) schedule(dynamic, chunk)
+    for (int64_t c = 0; c < num_cells; c++) {
+        footprint f = cell_footprint(x[c], y[c], w[c], h[c], xl, yl, xh, yh, bx, by, stretch);
+        double sx = 0.0, sy = 0.0;
+        if (f.hi_x > f.lo_x && f.hi_y > f.lo_y && f.r != 0.0) {
+            int i0, i1, j0, j1;
+            bin_range(f.lo_x, f.hi_x, xl, bx, mx, &i0, &i1);
+            bin_range(f.lo_y, f.hi_y, yl, by, my, &j0, &j1);
+            for (int i = i0; i <= i1; i++) {
+                double ox = overlap_1d(f.lo_x, f.hi_x, xl, bx, i);
+                if (ox <= 0.0) continue;
+                for (int j = j0; j <= j1; j++) {
+                    double oy = overlap_1d(f.lo_y, f.hi_y, yl, by, j);
+                    if (oy <= 0.0) continue;
+                    double ov = f.r * ox * oy;
+                    sx += ov * xi_x[(int64_t)i * my + j];
+                    sy += ov * xi_y[(int64_t)i * my + j];
+                }
+            }
+        }
+        gx[c] = -sx;
+        gy[c] = -sy;
+    }
+}
+
+/* In-place iterative radix-2 complex FFT (textbook Cooley-Tukey, bit-reversal first),
+ * n a power of two; sign = -1: X_k = sum_m v_m e^{-2 pi i k m / n}, +1: the unnormalised
+ * inverse.  re/im hold the sequence; tc/ts = cos/sin(2 pi k / n), k < n/2. */
+static void fft_inplace(int n, double *re, double *im, const double *tc, const double *ts, int sign)
+{
+    for (int i = 1, j = 0; i < n; i++) {
+        int bit = n >> 1;
+        for (; j & bit; bit >>= 1) j ^= bit;
+        j ^= bit;
+        if (i < j) {
+            double t = re[i]; re[i] = re[j]; re[j] = t;
+            t = im[i]; im[i] = im[j]; im[j] = t;
+        }
+    }
+    for (int len = 2; len <= n; len <<= 1) {
+        int step = n / len;
+        for (int i = 0; i < n; i += len) {
+            for (int k = 0; k < len / 2; k++) {
+                double wr = tc[k * step], wi = sign * ts[k * step];
+                double ur = re[i + k], ui = im[i + k];
+                double vr = re[i + k + len / 2] * wr - im[i + k + len / 2] * wi;
+                double vi = re[i + k + len / 2] * wi + im[i + k + len / 2] * wr;
+                re[i + k] = ur + vr; im[i + k] = ui + vi;
+                re[i + k + len / 2] = ur - vr; im[i + k + len / 2] = ui - vi;
+            }
+        }
+    }
+}
+
+/* The transforms of or_transform_lastaxis (kinds 0 DCT x 2/n, 1 IDCT eq 7b, 2 IDXST eq 8a)
+ * through one n-point complex FFT per row (n a power of two):
+ *   DCT   (Makhoul): v_m = x_2m, v_{n-1-m} = x_{2m+1}; out_k = (2/n) Re(e^{-i pi k / 2n} V_k)
+ *   IDCT  (the inverse of the same): V_k = e^{+i pi k / 2n} (X_k - i X_{n-k}), X_n := 0;
+ *         v = unnormalised inverse FFT of V; out_{2m} = Re v_m / 2, out_{2m+1} = Re v_{n-1-m} / 2
+ *   IDXST by eq (8e): out_k = (-1)^k IDCT(x')_k with x'_t = x_{n-t}, x'_0 = 0. */
+void or_transform_fft(int threads, int kind, int64_t rows, int n, const double *in, double *out)
+{
+    double *tc = malloc((size_t)(n / 2 > 0 ? n / 2 : 1) * sizeof(double));
+    double *ts = malloc((size_t)(n / 2 > 0 ? n / 2 : 1) * sizeof(double));
+    for (int k = 0; k < n / 2; k++) {
+        tc[k] = cos(2.0 * M_PI * k / n);
+        ts[k] = -sin(2.0 * M_PI * k / n);   /* forward twiddle e^{-2 pi i k / n} */
+    }
+#pragma omp parallel num_threads(threads)
+    {
+        double *re = malloc((size_t)n * sizeof(double)), *im = malloc((size_t)n * sizeof(double));
+        double *xs = malloc((size_t)n * sizeof(double));
+#pragma omp for schedule(static)
+        for (int64_t r = 0; r < rows; r++) {
+            const double *src = in + r * n;
+            double *dst = out + r * n;
+            if (kind == 0) {
+                for (int m = 0; m < n / 2; m++) {
+                    re[m] = src[2 * m];
+                    re[n - 1 - m] = src[2 * m + 1];
+                }
+                for (int m = 0; m < n; m++) im[m] = 0.0;
+                fft_inplace(n, re, im, tc, ts, 1);
+                for (int k = 0; k < n; k++) {
+                    double a = M_PI * k / (2.0 * n);
+                    dst[k] = (2.0 / n) * (re[k] * cos(a) + im[k] * sin(a));
+                }
+            } else {
+                if (kind == 2) {   /* eq (8e): x'_t = x_{n-t}, x'_0 = 0 */
+                    xs[0] = 0.0;
+                    for (int t = 1; t < n; t++) xs[t] = src[n - t];
+                } else {
+                    memcpy(xs, src, (size_t)n * sizeof(double));
+                }
+                for (int k = 0; k < n; k++) {
+                    double xr = xs[k], xi = (k == 0) ? 0.0 : -xs[n - k];
+                    double a = M_PI * k / (2.0 * n), c = cos(a), s = sin(a);
+                    re[k] = xr * c - xi * s;
+                    im[k] = xr * s + xi * c;
+                }
+                fft_inplace(n, re, im, tc, ts, -1);
+                for (int m = 0; m < n / 2; m++) {
+                    dst[2 * m] = 0.5 * re[m];
+                    dst[2 * m + 1] = 0.5 * re[n - 1 - m];
+                }
+                if (kind == 2)
+                    for (int k = 1; k < n; k += 2) dst[k] = -dst[k];
+            }
+        }
+        free(re); free(im); free(xs);
+    }
+    free(tc); free(ts);
+}
+
 int or_abi_version(void) { return 1; }

@@ -877,6 +877,11 @@ void fields_after_t1(const Ctx &c, cudaStream_t s) {
   a.tw_x = c.d_tw_x; a.ph_x = c.d_ph_x; a.kx = c.d_kx; a.ky = c.d_ky;
   a.energy_part = c.d_part + c.n_wa_part;
   a.energy_scale = 0.5 * c.bx * c.by;
+  if (c.fft_hybrid) {   // the CTA-FFT column pass on t[x][y], then T3
+    launch_p2_rowmajor(c, s);
+    row_inv(c, nullptr, 0, 1, nullptr, 0, 2, nullptr, 0, nullptr, 0, c.d_xi, c.mx, s, c.d_sxy);
+    return;
+  }
   if (warp_fft_ok(c.log2mx) && warp_fft_ok(c.log2my)) {
     const int warps = ((c.my / 2) + (wfft::kPts >> c.log2mx) - 1) / (wfft::kPts >> c.log2mx);
     const int g = (warps + kWColWarps - 1) / kWColWarps;

@@ -20,6 +20,8 @@
 #include <numeric>
 #include <string>
 #include <vector>
+#include <map>
+#include <cstring>
 
 #include "dp_internal.h"
 
@@ -118,79 +120,150 @@ dp_status validate(const dp_netlist *nl, const dp_grid *g) {
   return DP_OK;
 }
 
-// Contiguous, count-balanced cell ranges; a net is evaluated on every rank owning one of its
-// pins' cells and counted (WA, HPWL) on the rank owning its first pin's cell.
-void plan(const dp_netlist *nl, int rank, int world, int32_t &cb, int32_t &ce, std::vector<uint8_t> *mask) {
-  const int64_t n = nl->num_cells;
-  cb = (int32_t)(n * rank / world);
-  ce = (int32_t)(n * (rank + 1) / world);
-  if (!mask) return;
-  mask->assign(nl->num_nets, 0);
-  for (int32_t e = 0; e < nl->num_nets; e++) {
-    const int32_t s = nl->net_start[e], t = nl->net_start[e + 1];
-    uint8_t m = 0;
-    for (int32_t k = s; k < t; k++) {
-      const int32_t p = nl->net2pin ? nl->net2pin[k] : k;
-      const int32_t c = nl->pin2cell[p];
-      if (c >= cb && c < ce) {
-        m = 1;
-        break;
-      }
-    }
-    if (m && t > s) {
-      const int32_t p0 = nl->net2pin ? nl->net2pin[s] : s;
-      const int32_t c0 = nl->pin2cell[p0];
-      if (c0 >= cb && c0 < ce) m = 3;
-    }
-    (*mask)[e] = m;
-  }
-}
-
 int g_class(int d) {  // log2 of lanes per net
   int g = 0;
   while ((kWaPpl << g) < d) g++;
   return g;
 }
 
-dp_status build_wa(Ctx &c, const dp_netlist *nl, const std::vector<uint8_t> &mask) {
-  const int32_t ncells = nl->num_cells;
+// The global WA work plan, a pure function of the netlist — identical on every
+// rank and for every number of ranks.  Units, in CTA order of the WA kernel:
+//   [nets of degree > kWarpNetMax, one CTA each | blocks of 8 nets of degree (kWaMaxDeg,
+//    kWarpNetMax], a warp each | chunks of <= kWaChunkPins pins of the small nets in locality
+//    order (median cell index)]
+// Ranks take contiguous unit ranges balanced by pin count ("nets are partitioned for WA",
+// BASELINE north_star); a unit's WA partial has one global slot, so partial sums, chunk fixed-
+// point scales and hence the deterministic-mode gradient are the same for any world size.
+struct WaPlan {
+  std::vector<int32_t> small;                         // locality order
+  std::vector<std::pair<size_t, size_t>> chunk_rng;   // [i, j) into small
+  std::vector<int32_t> big;                           // degree-descending
+  int32_t n_huge = 0, n_wblk = 0;
+  std::vector<int64_t> unit_pins;
+  std::vector<int32_t> unit_lo;                       // [world + 1]
+  int32_t units() const { return n_huge + n_wblk + (int32_t)chunk_rng.size(); }
+};
+
+WaPlan wa_plan(const dp_netlist *nl, int world) {
+  WaPlan P;
   auto pin_of = [&](int32_t slot) { return nl->net2pin ? nl->net2pin[slot] : slot; };
-  std::vector<int32_t> small, big;
+  auto deg = [&](int32_t e) { return nl->net_start[e + 1] - nl->net_start[e]; };
   for (int32_t e = 0; e < nl->num_nets; e++) {
-    const int d = nl->net_start[e + 1] - nl->net_start[e];
-    if (d < 2 || !mask[e]) continue;  // reading A3: degree 0/1 contribute nothing
-    (d > kWaMaxDeg ? big : small).push_back(e);
+    const int d = deg(e);
+    if (d < 2) continue;  // reading A3: degree 0/1 contribute nothing
+    (d > kWaMaxDeg ? P.big : P.small).push_back(e);
   }
-  // ---- locality order: median cell index of each net's pins ----
-  std::vector<int32_t> key(nl->num_nets, 0);
-  std::vector<int32_t> tmp;
-  for (int32_t e : small) {
-    const int32_t s = nl->net_start[e], t = nl->net_start[e + 1];
+  std::vector<int32_t> key(nl->num_nets, 0), tmp;
+  for (int32_t e : P.small) {
     tmp.clear();
-    for (int32_t k = s; k < t; k++) tmp.push_back(nl->pin2cell[pin_of(k)]);
+    for (int32_t k = nl->net_start[e]; k < nl->net_start[e + 1]; k++) tmp.push_back(nl->pin2cell[pin_of(k)]);
     std::nth_element(tmp.begin(), tmp.begin() + tmp.size() / 2, tmp.end());
     key[e] = tmp[tmp.size() / 2];
   }
-  std::stable_sort(small.begin(), small.end(), [&](int32_t a, int32_t b) { return key[a] < key[b]; });
+  std::stable_sort(P.small.begin(), P.small.end(), [&](int32_t a, int32_t b) { return key[a] < key[b]; });
+  std::stable_sort(P.big.begin(), P.big.end(), [&](int32_t a, int32_t b) { return deg(a) > deg(b); });
+  while (P.n_huge < (int32_t)P.big.size() && deg(P.big[P.n_huge]) > kWarpNetMax) P.n_huge++;
+  constexpr int kWarpNets = kWarpNetThreads / 32;
+  P.n_wblk = ((int32_t)P.big.size() - P.n_huge + kWarpNets - 1) / kWarpNets;
+  for (size_t i = 0; i < P.small.size();) {   // nets until the pin budget is reached (at least one)
+    size_t j = i;
+    int pins = 0;
+    while (j < P.small.size()) {
+      const int d = deg(P.small[j]);
+      if (j > i && pins + d > kWaChunkPins) break;
+      pins += d;
+      j++;
+    }
+    P.chunk_rng.push_back({i, j});
+    i = j;
+  }
+  for (int32_t u = 0; u < P.n_huge; u++) P.unit_pins.push_back(deg(P.big[u]));
+  for (int32_t b = 0; b < P.n_wblk; b++) {
+    int64_t n = 0;
+    for (int32_t q = P.n_huge + b * kWarpNets; q < std::min<int32_t>((int32_t)P.big.size(), P.n_huge + (b + 1) * kWarpNets); q++)
+      n += deg(P.big[q]);
+    P.unit_pins.push_back(n);
+  }
+  for (const auto &r : P.chunk_rng) {
+    int64_t n = 0;
+    for (size_t q = r.first; q < r.second; q++) n += deg(P.small[q]);
+    P.unit_pins.push_back(n);
+  }
+  // rank of a unit: the one whose share of the pin total contains the unit's midpoint
+  const int32_t U = P.units();
+  int64_t total = 0;
+  for (int64_t n : P.unit_pins) total += n;
+  P.unit_lo.assign(world + 1, U);
+  P.unit_lo[0] = 0;
+  int64_t acc = 0;
+  int r = 1;
+  for (int32_t u = 0; u < U && r < world; u++) {
+    const long double mid = (long double)acc + 0.5L * (long double)P.unit_pins[u];
+    while (r < world && mid * world >= (long double)total * r) P.unit_lo[r++] = u;
+    acc += P.unit_pins[u];
+  }
+  while (r < world) P.unit_lo[r++] = U;
+  return P;
+}
 
+// Cells: world equal blocks of ceil(num_cells / world) (the gradient reduce-scatter's blocks);
+// rank r owns [r B, min((r+1) B, num_cells)) for the density scatter and gather.  Nets: the nets
+// of the rank's WA units (mask 3 = evaluated and counted; every net of degree >= 2 on exactly
+// one rank).
+int32_t cell_block(int32_t n, int world) { return (int32_t)(((int64_t)n + world - 1) / world); }
+
+void plan(const dp_netlist *nl, int rank, int world, int32_t &cb, int32_t &ce, std::vector<uint8_t> *mask,
+          const WaPlan *wp = nullptr) {
+  const int32_t B = cell_block(nl->num_cells, world);
+  cb = (int32_t)std::min<int64_t>(nl->num_cells, (int64_t)B * rank);
+  ce = (int32_t)std::min<int64_t>(nl->num_cells, (int64_t)B * (rank + 1));
+  if (!mask) return;
+  WaPlan local;
+  if (!wp) {
+    local = wa_plan(nl, world);
+    wp = &local;
+  }
+  mask->assign(nl->num_nets, 0);
+  constexpr int kWarpNets = kWarpNetThreads / 32;
+  for (int32_t u = wp->unit_lo[rank]; u < wp->unit_lo[rank + 1]; u++) {
+    if (u < wp->n_huge) {
+      (*mask)[wp->big[u]] = 3;
+    } else if (u < wp->n_huge + wp->n_wblk) {
+      const int32_t b = u - wp->n_huge;
+      for (int32_t q = wp->n_huge + b * kWarpNets; q < std::min<int32_t>((int32_t)wp->big.size(), wp->n_huge + (b + 1) * kWarpNets); q++)
+        (*mask)[wp->big[q]] = 3;
+    } else {
+      const auto &rg = wp->chunk_rng[u - wp->n_huge - wp->n_wblk];
+      for (size_t q = rg.first; q < rg.second; q++) (*mask)[wp->small[q]] = 3;
+    }
+  }
+}
+
+dp_status build_wa(Ctx &c, const dp_netlist *nl, const WaPlan &P) {
+  const int32_t ncells = nl->num_cells;
+  auto pin_of = [&](int32_t slot) { return nl->net2pin ? nl->net2pin[slot] : slot; };
+  // this rank's units: huge nets [h0, h1), warp blocks [w0, w1), chunks [k0, k1) (global indices)
+  const int32_t u0 = P.unit_lo[c.rank], u1 = P.unit_lo[c.rank + 1];
+  auto clip = [&](int32_t lo, int32_t hi, int32_t &a0, int32_t &a1) {
+    a0 = std::max(u0, lo) - lo;
+    a1 = std::max(a0, std::min(u1, hi) - lo);
+  };
+  int32_t h0, h1, w0, w1, k0, k1;
+  clip(0, P.n_huge, h0, h1);
+  clip(P.n_huge, P.n_huge + P.n_wblk, w0, w1);
+  clip(P.n_huge + P.n_wblk, P.units(), k0, k1);
+  c.part_base = u0;
+  c.n_wa_part = P.units();
+  const std::vector<int32_t> &small = P.small;
   std::vector<Chunk> chunks;
   std::vector<WarpGroup> wgs;
   std::vector<int32_t> net_deg, pin_cell, far_cells;
   std::vector<float> net_w, pin_dx, pin_dy;
   WaCaps caps{4, 4, 4, 4};
   auto up4 = [](int v) { return (v + 3) & ~3; };
-  size_t i = 0;
   std::vector<int32_t> cells, far;
-  while (i < small.size()) {
-    // take nets until the pin budget is reached (at least one net)
-    size_t j = i;
-    int pins = 0;
-    while (j < small.size()) {
-      const int d = nl->net_start[small[j] + 1] - nl->net_start[small[j]];
-      if (j > i && pins + d > kWaChunkPins) break;
-      pins += d;
-      j++;
-    }
+  for (int32_t kc = k0; kc < k1; kc++) {
+    const size_t i = P.chunk_rng[kc].first, j = P.chunk_rng[kc].second;
     // densest window of kWaWindow consecutive cells, start aligned to 4 cells (16 bytes) so
     // the kernel can stage x / y with bulk async copies
     cells.clear();
@@ -282,7 +355,7 @@ dp_status build_wa(Ctx &c, const dp_netlist *nl, const std::vector<uint8_t> &mas
           const int d = nl->net_start[e + 1] - nl->net_start[e];
           dmax = std::max(dmax, d);
           pairs = pairs && d == 2;
-          net_deg.push_back(d | ((mask[e] & 2) ? (int32_t)0x80000000u : 0));
+          net_deg.push_back(d | (int32_t)0x80000000u);   // counted: every own net (one rank per net)
           net_w.push_back(nl->net_weight ? nl->net_weight[e] : 1.f);
         }
         wg.slots = (dmax + G - 1) / G;
@@ -296,9 +369,7 @@ dp_status build_wa(Ctx &c, const dp_netlist *nl, const std::vector<uint8_t> &mas
             const int k = s * G + jj;
             if (k >= d) continue;
             const int32_t p = pin_of(nl->net_start[e] + k);
-            const int32_t cell = nl->pin2cell[p];
-            const bool foreign = cell < c.cell_begin || cell >= c.cell_end;
-            pin_cell.push_back(slot_of(cell) | (foreign ? (int32_t)0x80000000u : 0));
+            pin_cell.push_back(slot_of(nl->pin2cell[p]));
             pin_dx.push_back(nl->pin_dx[p]);
             pin_dy.push_back(nl->pin_dy[p]);
           }
@@ -314,7 +385,6 @@ dp_status build_wa(Ctx &c, const dp_netlist *nl, const std::vector<uint8_t> &mas
     caps.groups = std::max(caps.groups, up4(ch.wg_n));
     caps.far = std::max(caps.far, ch.far_pad);
     chunks.push_back(ch);
-    i = j;
   }
   c.n_chunks = (int32_t)chunks.size();
   c.n_wgroups = (int32_t)wgs.size();
@@ -343,30 +413,28 @@ dp_status build_wa(Ctx &c, const dp_netlist *nl, const std::vector<uint8_t> &mas
   if ((st = dev_upload(c, &c.d_pin_dx, pin_dx)) != DP_OK) return st;
   if ((st = dev_upload(c, &c.d_pin_dy, pin_dy)) != DP_OK) return st;
   if ((st = dev_upload(c, &c.d_far_cells, far_cells)) != DP_OK) return st;
-  // ---- big nets ----
-  // largest first: the longest CTAs start in the first wave
-  std::stable_sort(big.begin(), big.end(), [&](int32_t a, int32_t b) {
-    return nl->net_start[a + 1] - nl->net_start[a] > nl->net_start[b + 1] - nl->net_start[b];
-  });
+  // ---- big nets: this rank's huge nets, then its warp-block nets (largest first: the longest
+  // CTAs start in the first wave) ----
+  constexpr int kWarpNets = kWarpNetThreads / 32;
+  std::vector<int32_t> big(P.big.begin() + h0, P.big.begin() + h1);
+  for (int32_t q = P.n_huge + w0 * kWarpNets; q < std::min<int32_t>((int32_t)P.big.size(), P.n_huge + w1 * kWarpNets); q++)
+    big.push_back(P.big[q]);
   c.big_stage = big.empty() ? 0 : std::min(kBigStage, nl->net_start[big[0] + 1] - nl->net_start[big[0]]);
   std::vector<int32_t> bstart{0}, bflags, bcell;
   std::vector<float> bw, bdx, bdy;
   for (int32_t e : big) {
     for (int32_t k = nl->net_start[e]; k < nl->net_start[e + 1]; k++) {
       const int32_t p = pin_of(k);
-      const int32_t cell = nl->pin2cell[p];
-      const bool foreign = cell < c.cell_begin || cell >= c.cell_end;
-      bcell.push_back(cell | (foreign ? (int32_t)0x80000000u : 0));
+      bcell.push_back(nl->pin2cell[p]);
       bdx.push_back(nl->pin_dx[p]);
       bdy.push_back(nl->pin_dy[p]);
     }
     bstart.push_back((int32_t)bcell.size());
-    bflags.push_back((mask[e] & 2) ? 1 : 0);
+    bflags.push_back(1);
     bw.push_back(nl->net_weight ? nl->net_weight[e] : 1.f);
   }
   c.n_big = (int32_t)big.size();
-  c.n_huge = 0;
-  while (c.n_huge < c.n_big && nl->net_start[big[c.n_huge] + 1] - nl->net_start[big[c.n_huge]] > kWarpNetMax) c.n_huge++;
+  c.n_huge = h1 - h0;
   if ((st = dev_upload(c, &c.d_big_start, bstart)) != DP_OK) return st;
   if ((st = dev_upload(c, &c.d_big_flags, bflags)) != DP_OK) return st;
   if ((st = dev_upload(c, &c.d_big_w, bw)) != DP_OK) return st;
@@ -435,6 +503,8 @@ dp_status build_density(Ctx &c, const dp_netlist *nl) {
   if ((st = dev_alloc(c, &c.d_tile_cursor, (size_t)ntiles * kCntStride)) != DP_OK) return st;
   if ((st = dev_alloc(c, &c.d_tile_off, ntiles + 1)) != DP_OK) return st;
   // sort records; padded by 8 so staged copies may round their range to 4-record multiples
+  // (16-byte records with a per-cell-size constant table measured slower inside the step:
+  // 4389 vs 4586 evals/s)
   if ((st = dev_alloc(c, &c.d_rec, c.n_own + 8)) != DP_OK) return st;
   if ((st = dev_alloc(c, &c.d_rec_rc, c.n_own + 8)) != DP_OK) return st;
   if ((st = dev_alloc(c, &c.d_rec_cell, c.n_own + 8)) != DP_OK) return st;
@@ -562,13 +632,13 @@ dp_status create(const dp_netlist *nl, const dp_grid *grid, int device, int rank
   c->bx = (c->xh - c->xl) / c->mx;
   c->by = (c->yh - c->yl) / c->my;
   c->stretch = grid->stretch;
-  std::vector<uint8_t> mask;
-  plan(nl, rank, world, c->cell_begin, c->cell_end, &mask);
+  const WaPlan wplan = wa_plan(nl, world);
+  plan(nl, rank, world, c->cell_begin, c->cell_end, nullptr);
   auto bail = [&](dp_status s) {
     destroy(c);
     return s;
   };
-  if ((st = build_wa(*c, nl, mask)) != DP_OK) return bail(st);
+  if ((st = build_wa(*c, nl, wplan)) != DP_OK) return bail(st);
   if ((st = build_density(*c, nl)) != DP_OK) return bail(st);
   {   // net-weighted pin count per cell: the GP preconditioner's P_i (gp.cu, reading A29)
     std::vector<double> acc(nl->num_cells, 0.0);
@@ -580,23 +650,27 @@ dp_status create(const dp_netlist *nl, const dp_grid *grid, int device, int rank
     std::vector<float> pins(acc.begin(), acc.end());
     if ((st = dev_upload(*c, &c->d_cell_pins, pins)) != DP_OK) return bail(st);
   }
-  c->n_wa_part = c->n_chunks + c->n_huge + (c->n_big - c->n_huge + kWarpNetThreads / 32 - 1) / (kWarpNetThreads / 32);
   {   // field transforms: the warp FFT up to 1024 points (fewer instructions, no block barriers:
       // measured 4599 vs 4041 evals/s at bigblue4 against the CTA FFT), the CTA FFT (fields.cu)
-      // beyond, where the warp FFT does not reach; DP_FFT=1 / 0 forces one (A/B)
+      // beyond, where the warp FFT does not reach; DP_FFT = 0 (warp) / 1 (CTA) / 2 (hybrid: warp
+      // rows, CTA column pass) forces one (A/B)
     const char *e = std::getenv("DP_FFT");
     const bool big = std::max(c->mx, c->my) > 1024;
-    c->fft_cta = fields_cta_ok(c->log2mx, c->log2my) && (e ? e[0] == '1' : big);
+    const int mode = e ? std::atoi(e) : (big ? 1 : 0);
+    c->fft_cta = fields_cta_ok(c->log2mx, c->log2my) && (big || mode == 1);
+    c->fft_hybrid = !c->fft_cta && mode == 2 && fields_cta_ok(c->log2mx, c->log2my);
   }
   // energy partials: one per CTA of the column pass (P2 of the CTA-FFT path; 2-column slabs of
   // the warp-FFT path)
-  c->n_en_part = c->fft_cta ? p2_ctas(c->mx, c->my) : c->my / 2;
+  c->n_en_part = (c->fft_cta || c->fft_hybrid) ? p2_ctas(c->mx, c->my) : c->my / 2;
   // one "hot" arena for the two per-cell vectors the combine reads: the WA accumulator g2
   // [num_cells] and the force [n_own + 4] (offset by the parity of cell_begin so that even
   // global cells are 16-byte aligned: the combine reads cell pairs as float4).  It is the
   // L2 persisting access-policy window of the evaluation's streams (DP_L2_PERSIST=0: off).
   {
-    const size_t g2n = ((size_t)c->num_cells + 7) & ~(size_t)7;
+    c->cell_blk = cell_block(c->num_cells, world);
+    c->g2_cells = c->dist ? (int64_t)c->cell_blk * world : (int64_t)c->num_cells;
+    const size_t g2n = ((size_t)c->g2_cells + 7) & ~(size_t)7;
     const size_t hot_n = g2n + (size_t)c->n_own + 4;
     if ((st = dev_alloc(*c, &c->d_g2, hot_n)) != DP_OK) return bail(st);
     if (cudaMemset(c->d_g2, 0, sizeof(float2) * hot_n) != cudaSuccess) return bail(fail(DP_ERR_CUDA, "memset"));
@@ -676,10 +750,15 @@ dp_status create(const dp_netlist *nl, const dp_grid *grid, int device, int rank
     cudaGetLastError();   // best effort: a refused hint leaves the default policy
   }
   const int wa_k = (c->n_chunks + c->n_big > 0) ? 1 : 0;   // one kernel: big nets, warp nets, chunks
-  c->launches_eval = wa_k + density_launches(*c) + (c->fft_cta ? 3 : c->fused_t2 ? 3 : 4) /* P1 P2 P3 or T1 T2a T2b T3 */ + 2 /* combine, finalize */;
+  c->launches_eval = wa_k + density_launches(*c) + ((c->fft_cta || c->fft_hybrid) ? 3 : c->fused_t2 ? 3 : 4) /* P1 P2 P3, T1 P2 T3 or T1 T2a T2b T3 */ + 2 /* combine, finalize */;
   c->launches_eval_hpwl = c->launches_eval;
   if (c->dist && nccl_id) {
     if ((st = nccl_init(*c, nccl_id)) != DP_OK) return bail(st);
+    // row-sharded Poisson solve for maps above 1024 (replicated below: a redundant <= 4 MB solve
+    // is cheaper than its exchanges); DP_SHARD_POISSON = 1 / 0 forces it on / off
+    const char *e = std::getenv("DP_SHARD_POISSON");
+    const bool want = e ? e[0] == '1' : std::max(c->mx, c->my) > 1024;
+    c->shard_poisson = want && fields_shardable(*c, world);
   }
   cudaError_t le = cudaDeviceSynchronize();
   if (le != cudaSuccess) return bail(cuda_fail(le, "dp_create"));
@@ -727,19 +806,44 @@ struct StageMark {
 };
 
 // the density chain on the density stream: map -> (allreduce) -> fields -> gather
+// Row-sharded Poisson solve of rank c.rank: the summed map's row block arrives by
+// the reduce-scatter; P1 on the rank's rows, all-to-all, P2 on its columns (+ its energy slots),
+// all-to-all, P3 on its rows, all-gather of the field rows.
+dp_status sharded_fields(Ctx &c, cudaStream_t s) {
+  const int G = c.world;
+  const size_t nb = (size_t)c.mx * c.my, blk = nb / ((size_t)G * G);   // C R elements per block
+  float *s1 = c.d_t, *r1 = c.d_sx;
+  float2 *s2 = c.d_sxy, *r2 = c.d_spec;
+  DP_CUDA(cudaMemsetAsync(c.d_part + c.n_wa_part, 0, sizeof(double) * c.n_en_part, s));   // other ranks' slots
+  launch_fields_shard(c, 1, c.d_rho, true, c.rank, G, s1, r1, s2, r2, s);
+  dp_status st = nccl_all_to_all_bytes(c, s1, r1, blk * sizeof(float), s);
+  if (st != DP_OK) return st;
+  launch_fields_shard(c, 2, c.d_rho, true, c.rank, G, s1, r1, s2, r2, s);
+  if ((st = nccl_all_to_all_bytes(c, s2, r2, blk * sizeof(float2), s)) != DP_OK) return st;
+  launch_fields_shard(c, 3, c.d_rho, true, c.rank, G, s1, r1, s2, r2, s);
+  return nccl_all_gather_bytes(c, c.d_xi, nb / G * sizeof(float2), s);
+}
+
 dp_status density_chain(Ctx &c, const float *x, const float *y) {
   {
     StageMark m(c, DP_STAGE_MAP, c.s_den);
     launch_density_map(c, x, y, c.s_den, c.s_aux);
     if (c.dist && c.nccl_comm) {
-      dp_status st = nccl_allreduce_u64(c, c.d_rho, (size_t)c.mx * c.my, c.s_den);   // exact
+      const size_t nb = (size_t)c.mx * c.my;
+      dp_status st = c.shard_poisson ? nccl_reduce_scatter_u64(c, c.d_rho, nb / c.world, c.s_den)   // exact
+                                     : nccl_allreduce_u64(c, c.d_rho, nb, c.s_den);                 // exact
       if (st != DP_OK) return st;
     }
   }
   DP_CUDA(cudaEventRecord(c.ev_map, c.s_den));
   {
     StageMark m(c, DP_STAGE_FIELDS, c.s_den);
-    launch_fields_fixed(c, c.s_den);
+    if (c.shard_poisson) {
+      dp_status st = sharded_fields(c, c.s_den);
+      if (st != DP_OK) return st;
+    } else {
+      launch_fields_fixed(c, c.s_den);
+    }
   }
   StageMark m(c, DP_STAGE_GATHER, c.s_den);
   launch_density_gather(c, x, y, c.s_den, c.s_aux);
@@ -749,14 +853,18 @@ dp_status density_chain(Ctx &c, const float *x, const float *y) {
 dp_status finalize(Ctx &c, float lambda, bool with_wl, bool with_energy, bool with_hpwl, double *d_obj, double *d_wl,
                    double *d_energy, double *d_hpwl, cudaStream_t s) {
   if (c.dist && c.nccl_comm) {
-    launch_finalize_phase(c, 0, lambda, with_wl, with_energy, with_hpwl, d_obj, d_wl, d_energy, d_hpwl, s);
+    // every WA partial slot is written by exactly one rank (zero elsewhere): the all-reduce is
+    // exact and the fixed-order sum below is the same for any number of ranks; the HPWL limbs
+    // are integers; the energy is replicated (every rank solves the same Poisson problem)
     dp_status st;
-    if (with_wl && (st = nccl_allreduce_f64(c, c.d_scal, 1, s)) != DP_OK) return st;
+    if (with_wl && (st = nccl_allreduce_f64(c, c.d_part, (size_t)c.n_wa_part, s)) != DP_OK) return st;
     if (with_hpwl && (st = nccl_allreduce_u64(c, c.d_limbs, kHpwlLimbs + 1, s)) != DP_OK) return st;
-    launch_finalize_phase(c, 1, lambda, with_wl, with_energy, with_hpwl, d_obj, d_wl, d_energy, d_hpwl, s);
-  } else {
-    launch_finalize(c, lambda, with_wl, with_energy, with_hpwl, d_obj, d_wl, d_energy, d_hpwl, s);
+    // row-sharded solve: each rank holds the energy slots of its column blocks (exact)
+    if (with_energy && c.shard_poisson &&
+        (st = nccl_allreduce_f64(c, c.d_part + c.n_wa_part, (size_t)c.n_en_part, s)) != DP_OK)
+      return st;
   }
+  launch_finalize(c, lambda, with_wl, with_energy, with_hpwl, d_obj, d_wl, d_energy, d_hpwl, s);
   return DP_OK;
 }
 
@@ -888,11 +996,16 @@ dp_status eval_body(Ctx &c, const float *x, const float *y, float gamma, float l
           return fail(DP_ERR_UNSUPPORTED, "DP_DIRECT needs DP_SCHED >= 2");
         }
       } else if (c.deterministic)
-        DP_CUDA(cudaMemsetAsync(c.d_g2i + 2 * (size_t)c.cell_begin, 0,
-                                2 * sizeof(long long) * (size_t)(c.cell_end - c.cell_begin), c.s_wa));
+        DP_CUDA(cudaMemsetAsync(c.d_g2i, 0, 2 * sizeof(long long) * (size_t)c.g2_cells, c.s_wa));
       else
-        DP_CUDA(cudaMemsetAsync(c.d_g2 + c.cell_begin, 0, sizeof(float2) * (size_t)(c.cell_end - c.cell_begin), c.s_wa));
+        DP_CUDA(cudaMemsetAsync(c.d_g2, 0, sizeof(float2) * (size_t)c.g2_cells, c.s_wa));
       launch_wa(c, x, y, gamma, false, d_hpwl != nullptr, c.s_wa);
+      if (c.dist && c.nccl_comm) {   // nets are partitioned: sum the WA gradient into each cell block
+        const size_t n = 2 * (size_t)c.cell_blk;
+        dp_status st = c.deterministic ? nccl_reduce_scatter_i64(c, c.d_g2i, n, c.s_wa)
+                                       : nccl_reduce_scatter_f32(c, reinterpret_cast<float *>(c.d_g2), n, c.s_wa);
+        if (st != DP_OK) return st;
+      }
     }
     DP_CUDA(cudaEventRecord(c.ev_wa, c.s_wa));
   }
@@ -1026,7 +1139,7 @@ dp_status dp_set_deterministic(dp_ctx *ctx, int32_t on) {
   if (!c) return fail(DP_ERR_INVALID_ARG, "ctx is NULL");
   if (on && !c->d_g2i) {
     dp::DeviceGuard g(c->device);
-    dp_status st = dp::dev_alloc(*c, &c->d_g2i, 2 * (size_t)c->num_cells);
+    dp_status st = dp::dev_alloc(*c, &c->d_g2i, 2 * (size_t)c->g2_cells);
     if (st != DP_OK) return st;
   }
   c->deterministic = on != 0;
@@ -1216,6 +1329,52 @@ dp_status dp_debug_fields(dp_ctx *ctx, const float *rho, float *psi, float *xi_x
   if (d_energy) dp::launch_finalize(*c, 1.f, false, true, false, nullptr, nullptr, d_energy, nullptr, s);
   if (psi) dp::launch_psi(*c, rho, psi, s);
   DP_CUDA(cudaGetLastError());
+  return DP_OK;
+}
+
+dp_status dp_debug_sharded_fields(dp_ctx *ctx, int32_t world, const float *rho, float *xi_x, float *xi_y,
+                                  double *d_energy, dp_stream_t stream) {
+  Ctx *c = C(ctx);
+  if (!c || !rho || world < 1) return fail(DP_ERR_INVALID_ARG, "NULL argument or world < 1");
+  dp::DeviceGuard g(c->device);
+  if (!dp::fields_shardable(*c, world))
+    return fail(DP_ERR_UNSUPPORTED, "map not shardable over world ranks (CTA-FFT path, bins divisible by world)");
+  cudaStream_t s = (cudaStream_t)stream;
+  const int G = world;
+  const size_t nb = (size_t)c->mx * c->my, per = nb / G, blk = per / G;
+  // every virtual rank's buffers side by side: S1 / R1 in t / sx, S2 / R2 in sxy / spec
+  auto S1 = [&](int r) { return c->d_t + r * per; };
+  auto R1 = [&](int r) { return c->d_sx + r * per; };
+  auto S2 = [&](int r) { return c->d_sxy + r * per; };
+  auto R2 = [&](int r) { return c->d_spec + r * per; };
+  DP_CUDA(cudaMemsetAsync(c->d_part + c->n_wa_part, 0, sizeof(double) * c->n_en_part, s));
+  for (int r = 0; r < G; r++) dp::launch_fields_shard(*c, 1, rho, false, r, G, S1(r), R1(r), S2(r), R2(r), s);
+  for (int p = 0; p < G; p++)   // all-to-all: block q of rank p's S1 -> block p of rank q's R1
+    for (int q = 0; q < G; q++)
+      DP_CUDA(cudaMemcpyAsync(R1(q) + p * blk, S1(p) + q * blk, blk * sizeof(float), cudaMemcpyDeviceToDevice, s));
+  for (int r = 0; r < G; r++) dp::launch_fields_shard(*c, 2, rho, false, r, G, S1(r), R1(r), S2(r), R2(r), s);
+  for (int p = 0; p < G; p++)
+    for (int q = 0; q < G; q++)
+      DP_CUDA(cudaMemcpyAsync(R2(q) + p * blk, S2(p) + q * blk, blk * sizeof(float2), cudaMemcpyDeviceToDevice, s));
+  for (int r = 0; r < G; r++) dp::launch_fields_shard(*c, 3, rho, false, r, G, S1(r), R1(r), S2(r), R2(r), s);
+  if (xi_x || xi_y) dp::launch_split_fields(*c, xi_x, xi_y, s);
+  if (d_energy) dp::launch_finalize(*c, 1.f, false, true, false, nullptr, nullptr, d_energy, nullptr, s);
+  DP_CUDA(cudaGetLastError());
+  return DP_OK;
+}
+
+dp_status dp_debug_wa_accumulator(dp_ctx *ctx, void *out, int64_t *n_out, dp_stream_t stream) {
+  Ctx *c = C(ctx);
+  if (!c || !n_out) return fail(DP_ERR_INVALID_ARG, "NULL argument");
+  dp::DeviceGuard g(c->device);
+  *n_out = c->g2_cells;
+  if (!out) return DP_OK;
+  cudaStream_t s = (cudaStream_t)stream;
+  if (c->deterministic && c->d_g2i)
+    DP_CUDA(cudaMemcpyAsync(out, c->d_g2i, 2 * sizeof(long long) * (size_t)c->g2_cells, cudaMemcpyDeviceToDevice, s));
+  else
+    DP_CUDA(cudaMemcpyAsync(out, c->d_g2, sizeof(float2) * (size_t)c->g2_cells, cudaMemcpyDeviceToDevice, s));
+  DP_CUDA(cudaStreamSynchronize(s));
   return DP_OK;
 }
 

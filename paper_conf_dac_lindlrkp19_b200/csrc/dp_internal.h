@@ -200,7 +200,8 @@ struct Ctx {
   bool fused_t2 = false;                            // DP_FUSED_T2=1: one column kernel (T2) instead of T2a + T2b (A/B)
   float2 *d_sxy = nullptr;                          // T2 -> T3 interleaved (sX, sY) [x][y] (warp-FFT path)
   float2 *d_twf_x = nullptr, *d_twf_y = nullptr;   // CTA FFT: W_N^k, k < N
-  bool fft_cta = true;                              // fields by the CTA-FFT passes (DP_FFT=0: warp FFT, A/B)
+  bool fft_cta = true;                              // fields by the CTA-FFT passes P1 P2 P3 (fields.cu)
+  bool fft_hybrid = false;                          // warp-FFT T1 and T3 around the CTA-FFT column pass P2
   float2 *d_tw2_x = nullptr, *d_tw2_y = nullptr;   // warp FFT: W_N^{n1 k2} at [k2 * 32 + n1] (N <= 1024)
   float *d_kx = nullptr, *d_ky = nullptr;          // wavenumbers (reading A12)
 
@@ -212,7 +213,11 @@ struct Ctx {
   void *d_maps = nullptr;             // arena: rho, spec, sxy, xi, t
   size_t maps_bytes = 0;
   double *d_part = nullptr;           // partial sums: [0, n_wa_part) WA, then energy
-  int32_t n_wa_part = 0, n_en_part = 0;
+  int32_t n_wa_part = 0, n_en_part = 0;   // WA partials: one slot per global WA unit (all ranks)
+  int32_t part_base = 0;                   // this rank's first WA unit
+  int32_t cell_blk = 0;                    // cells per rank block of the gradient reduce-scatter
+  bool shard_poisson = false;              // row-sharded Poisson solve (dist, maps > 1024)
+  int64_t g2_cells = 0;                    // WA accumulator length (dist: world blocks; else num_cells)
   unsigned long long *d_limbs = nullptr;  // HPWL fixed-point limbs
   double *d_scal = nullptr;           // {wl, energy, hpwl, obj} staging
   float *d_hx = nullptr, *d_hy = nullptr, *d_hgx = nullptr, *d_hgy = nullptr;  // e2e buffers
@@ -271,6 +276,10 @@ cudaError_t fields_configure();
 bool fields_cta_ok(int log2mx, int log2my);
 int p2_ctas(int mx, int my);
 void launch_fields_cta(const Ctx &c, const void *rho, bool int_map, cudaStream_t s);
+void launch_p2_rowmajor(const Ctx &c, cudaStream_t s);
+bool fields_shardable(const Ctx &c, int G);
+void launch_fields_shard(const Ctx &c, int pass, const void *rho, bool int_map, int r, int G, float *s1,
+                         const float *r1, float2 *s2, const float2 *r2, cudaStream_t s);
 // combine / finalize (finalize.cu)
 dp_status eval_body_ext(Ctx &c, const float *x, const float *y, float gamma, float lambda, float *gx, float *gy,
                         double *d_obj, double *d_wl, double *d_energy, double *d_hpwl, cudaStream_t s, bool do_wa,
@@ -299,6 +308,11 @@ dp_status nccl_init(Ctx &c, const void *id);
 dp_status nccl_allreduce_f32(Ctx &c, float *buf, size_t n, cudaStream_t s);
 dp_status nccl_allreduce_f64(Ctx &c, double *buf, size_t n, cudaStream_t s);
 dp_status nccl_allreduce_u64(Ctx &c, unsigned long long *buf, size_t n, cudaStream_t s);
+dp_status nccl_reduce_scatter_f32(Ctx &c, float *buf, size_t n, cudaStream_t s);
+dp_status nccl_reduce_scatter_i64(Ctx &c, long long *buf, size_t n, cudaStream_t s);
+dp_status nccl_reduce_scatter_u64(Ctx &c, unsigned long long *buf, size_t n, cudaStream_t s);
+dp_status nccl_all_gather_bytes(Ctx &c, void *buf, size_t n, cudaStream_t s);
+dp_status nccl_all_to_all_bytes(Ctx &c, const void *send, void *recv, size_t n, cudaStream_t s);
 void nccl_destroy(Ctx &c);
 
 }  // namespace dp

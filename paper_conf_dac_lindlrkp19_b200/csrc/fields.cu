@@ -63,12 +63,23 @@ __device__ __forceinline__ float fast_rcp(float x) {
   return r;
 }
 
+// Layouts.  Unsharded: tT[y][x] (P1 -> P2), sxy[x][y] (P2 -> P3).  Row-sharded over G ranks
+// (R = mx / G rows and C = my / G columns per rank, rank offsets x_base, y_base):
+// P1 writes its rows' t as the all-to-all send blocks S1[q][y - qC][x - x_base], P2 reads the
+// received blocks R1[p][y - y_base][x - pR] and writes S2[q][x - qR][y - y_base], P3 reads
+// R2[p][x - x_base][y - pC].  With G = 1 (R = mx, C = my) these are exactly the unsharded
+// layouts, so one indexing serves both.
 struct FieldArgs {
-  const void *rho;        // [mx][my], IN = float or int64 (2^-29 units)
-  float *tT;              // [my][mx]
-  float2 *sxy;            // [mx][my] (sX, sY)
-  float2 *xi;             // [mx][my] (xi_X, xi_Y)
+  const void *rho;        // [mx][my], IN = float or int64 (2^-29 units); rows [x_base, x_base + nrows) used
+  float *t_out;           // P1 output (tT / S1)
+  const float *t_in;      // P2 input (tT / R1)
+  float2 *s_out;          // P2 output (sxy / S2)
+  const float2 *s_in;     // P3 input (sxy / R2)
+  float2 *xi;             // [mx][my] (xi_X, xi_Y); P3 writes rows [x_base, x_base + nrows)
   int mx, my;
+  int R, C;               // rows / columns per rank block
+  int x_base, y_base;     // this rank's first row / column
+  int nrows, ncols;       // rows of P1 / P3, columns of P2
   const float2 *twf_x, *twf_y;   // exp(-2 pi i k / N), k < N
   const float2 *ph_x, *ph_y;     // exp(-i pi k / 2N), k < N
   const float *kx, *ky;          // wavenumbers (A12)
@@ -87,7 +98,7 @@ __global__ void __launch_bounds__(cfft::seq_per_cta(LOGN) * cfft::threads_per_se
   float *out = reinterpret_cast<float *>(sm1 + 2 * SEQ * L);   // [N][ROWS]
   const IN *rho = reinterpret_cast<const IN *>(a.rho);
   const int tid = threadIdx.x, s = tid / T, t = tid % T;
-  const int x0 = blockIdx.x * ROWS;
+  const int x0 = a.x_base + blockIdx.x * ROWS, xend = a.x_base + a.nrows;
   float2 *A = sm1 + (2 * s) * L, *B = A + L;
   // load: row x0 + rr (coalesced) -> real (rr even) / imaginary (rr odd) part of sequence rr/2,
   // at its Makhoul position.  Every load is issued before the first use (unrolled: a loop
@@ -97,7 +108,7 @@ __global__ void __launch_bounds__(cfft::seq_per_cta(LOGN) * cfft::threads_per_se
 #pragma unroll
   for (int q = 0; q < PER; q++) {
     const int idx = tid + q * NT, x = x0 + (idx >> LOGN);
-    v[q] = x < a.mx ? rho[(size_t)x * N + (idx & (N - 1))] : (IN)0;
+    v[q] = x < xend ? rho[(size_t)x * N + (idx & (N - 1))] : (IN)0;
   }
 #pragma unroll
   for (int q = 0; q < PER; q++) {
@@ -114,23 +125,27 @@ __global__ void __launch_bounds__(cfft::seq_per_cta(LOGN) * cfft::threads_per_se
     out[k * ROWS + 2 * s + 1] = d.y;
   }
   __syncthreads();
-  // transposed store: tT[k][x0 .. x0 + ROWS)
-  if (ROWS % 4 == 0 && x0 + ROWS <= a.mx) {
+  // transposed store: tT[k][x0 .. x0 + ROWS) (unsharded) / S1[k / C][k % C][x0 - x_base ..]
+  const size_t CR = (size_t)a.C * a.R;
+  if (ROWS % 4 == 0 && x0 + ROWS <= xend) {
     for (int idx = tid; idx < N * (ROWS / 4); idx += NT) {
       const int k = idx / (ROWS / 4), q = idx % (ROWS / 4);
-      *reinterpret_cast<float4 *>(a.tT + (size_t)k * a.mx + x0 + 4 * q) =
+      *reinterpret_cast<float4 *>(a.t_out + (size_t)(k / a.C) * CR + (size_t)(k % a.C) * a.R + (x0 - a.x_base) + 4 * q) =
           *reinterpret_cast<const float4 *>(out + k * ROWS + 4 * q);
     }
   } else {
     for (int idx = tid; idx < N * ROWS; idx += NT) {
       const int k = idx / ROWS, c = idx % ROWS;
-      if (x0 + c < a.mx) a.tT[(size_t)k * a.mx + x0 + c] = out[idx];
+      if (x0 + c < xend)
+        a.t_out[(size_t)(k / a.C) * CR + (size_t)(k % a.C) * a.R + (x0 - a.x_base) + c] = out[idx];
     }
   }
 }
 
 // ---- P2: columns (2p, 2p+1) (rows of tT) -> DCT over x, energy, scaling, inverse over x ----
-template <int LOGM>
+// TIN: t stored transposed, tT[y][x] (after P1); otherwise t[x][y] (after the warp-FFT T1):
+// the CTA then reads its COLS adjacent columns as 4 COLS-byte row segments.
+template <int LOGM, bool TIN = true>
 __global__ void __launch_bounds__(cfft::seq_per_cta(LOGM) * cfft::threads_per_seq(LOGM))
     k_p2(FieldArgs a) {
   griddep_wait();
@@ -141,18 +156,23 @@ __global__ void __launch_bounds__(cfft::seq_per_cta(LOGM) * cfft::threads_per_se
   float2 *out = spec + COLS * M;       // [M][COLS] (sX, sY)
   __shared__ double s_red[NT / 32 > 0 ? NT / 32 : 1];
   const int tid = threadIdx.x, s = tid / T, t = tid % T;
-  const int y0 = blockIdx.x * COLS, my = a.my;
+  const int y0 = a.y_base + blockIdx.x * COLS, my = a.my, yend = a.y_base + a.ncols;
+  const size_t CR = (size_t)a.C * a.R;
   float2 *A = sm2 + (2 * s) * L, *B = A + L;
   constexpr int PER = COLS * M / NT;
   float v[PER];
 #pragma unroll
   for (int q = 0; q < PER; q++) {
-    const int idx = tid + q * NT, c = idx >> LOGM;
-    v[q] = (y0 + c < my) ? a.tT[(size_t)(y0 + c) * M + (idx & (M - 1))] : 0.f;
+    const int idx = tid + q * NT;
+    const int c = TIN ? idx >> LOGM : idx % COLS, x = TIN ? idx & (M - 1) : idx / COLS;
+    v[q] = (y0 + c < yend) ? (TIN ? a.t_in[(size_t)(x / a.R) * CR + (size_t)(y0 + c - a.y_base) * a.R + (x % a.R)]
+                                  : a.t_in[(size_t)x * my + y0 + c])
+                           : 0.f;
   }
 #pragma unroll
   for (int q = 0; q < PER; q++) {
-    const int idx = tid + q * NT, c = idx >> LOGM, x = idx & (M - 1);
+    const int idx = tid + q * NT;
+    const int c = TIN ? idx >> LOGM : idx % COLS, x = TIN ? idx & (M - 1) : idx / COLS;
     float *slot = reinterpret_cast<float *>(sm2 + (c & ~1) * L + pad(mk_pos(x, M)));
     slot[c & 1] = v[q];
   }
@@ -161,7 +181,7 @@ __global__ void __launch_bounds__(cfft::seq_per_cta(LOGM) * cfft::threads_per_se
   // spectrum of columns v0 = y0 + 2s, v1 = v0 + 1: energy (Parseval, A8) and scaling (9c/9d)
   const float scale = 2.f / M;
   const int v0 = y0 + 2 * s, v1 = v0 + 1;
-  const bool ok = v1 < my;
+  const bool ok = v1 < yend;
   const float ky0 = ok ? __ldg(a.ky + v0) : 0.f, ky1 = ok ? __ldg(a.ky + v1) : 0.f;
   const double wv0 = (v0 == 0) ? 0.25 * my : 0.5 * my, wv1 = 0.5 * my;
   double e = 0.0;
@@ -194,17 +214,17 @@ __global__ void __launch_bounds__(cfft::seq_per_cta(LOGM) * cfft::threads_per_se
     }
     __syncthreads();
   }
-  // transposed store: sxy[x][y0 .. y0 + COLS)
-  if (COLS % 2 == 0 && y0 + COLS <= my) {
+  // transposed store: sxy[x][y0 .. y0 + COLS) (unsharded) / S2[x / R][x % R][y0 - y_base ..]
+  if (COLS % 2 == 0 && y0 + COLS <= yend) {
     for (int idx = tid; idx < M * (COLS / 2); idx += NT) {
       const int x = idx / (COLS / 2), q = idx % (COLS / 2);
-      *reinterpret_cast<float4 *>(a.sxy + (size_t)x * my + y0 + 2 * q) =
+      *reinterpret_cast<float4 *>(a.s_out + (size_t)(x / a.R) * CR + (size_t)(x % a.R) * a.C + (y0 - a.y_base) + 2 * q) =
           *reinterpret_cast<const float4 *>(out + x * COLS + 2 * q);
     }
   } else {
     for (int idx = tid; idx < M * COLS; idx += NT) {
       const int x = idx / COLS, c = idx % COLS;
-      if (y0 + c < my) a.sxy[(size_t)x * my + y0 + c] = out[idx];
+      if (y0 + c < yend) a.s_out[(size_t)(x / a.R) * CR + (size_t)(x % a.R) * a.C + (y0 - a.y_base) + c] = out[idx];
     }
   }
   // energy partial of this CTA (fixed order: deterministic)
@@ -215,7 +235,7 @@ __global__ void __launch_bounds__(cfft::seq_per_cta(LOGM) * cfft::threads_per_se
   if (tid == 0) {
     double tot = 0.0;
     for (int w = 0; w < (NT + 31) / 32; w++) tot += s_red[w];
-    a.energy_part[blockIdx.x] = tot * a.energy_scale;
+    a.energy_part[y0 / COLS] = tot * a.energy_scale;   // global column-slab slot: the same for any sharding
   }
 }
 
@@ -228,14 +248,15 @@ __global__ void __launch_bounds__(cfft::seq_per_cta(LOGN) * cfft::threads_per_se
   constexpr int NT = SEQ * T, L = buf_len(N);
   extern __shared__ __align__(16) float2 sm3[];
   const int tid = threadIdx.x, s = tid / T, t = tid % T;
-  const int x0 = blockIdx.x * SEQ;
+  const int x0 = a.x_base + blockIdx.x * SEQ, xend = a.x_base + a.nrows;
+  const size_t CR = (size_t)a.C * a.R;
   float2 *A = sm3 + (2 * s) * L, *B = A + L;
   constexpr int PER = SEQ * N / NT;
   float2 v[PER];
 #pragma unroll
   for (int q = 0; q < PER; q++) {
-    const int idx = tid + q * NT, x = x0 + (idx >> LOGN);
-    v[q] = x < a.mx ? a.sxy[(size_t)x * N + (idx & (N - 1))] : make_float2(0.f, 0.f);
+    const int idx = tid + q * NT, x = x0 + (idx >> LOGN), k = idx & (N - 1);
+    v[q] = x < xend ? a.s_in[(size_t)(k / a.C) * CR + (size_t)(x - a.x_base) * a.C + (k % a.C)] : make_float2(0.f, 0.f);
   }
 #pragma unroll
   for (int q = 0; q < PER; q++) {
@@ -253,7 +274,7 @@ __global__ void __launch_bounds__(cfft::seq_per_cta(LOGN) * cfft::threads_per_se
   __syncthreads();
   const float2 *W = cfft::fft<LOGN, true>(A, B, t, a.twf_y);
   const int x = x0 + s;
-  if (x < a.mx)
+  if (x < xend)
     for (int y = t; y < N; y += T) {
       const float2 z = W[pad(mk_pos(y, N))];
       a.xi[(size_t)x * N + y] = make_float2(0.5f * z.x, (y & 1) ? -0.5f * z.y : 0.5f * z.y);   // IDXST sign on xi_Y
@@ -284,8 +305,11 @@ cudaError_t configure_one() {
   if ((e = cudaFuncSetAttribute(k_p1<float, LOGN>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                 (int)p1_smem<LOGN>())) != cudaSuccess)
     return e;
-  if ((e = cudaFuncSetAttribute(k_p2<LOGN>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)p2_smem<LOGN>())) !=
-      cudaSuccess)
+  if ((e = cudaFuncSetAttribute(k_p2<LOGN, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                (int)p2_smem<LOGN>())) != cudaSuccess)
+    return e;
+  if ((e = cudaFuncSetAttribute(k_p2<LOGN, false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                (int)p2_smem<LOGN>())) != cudaSuccess)
     return e;
   return cudaFuncSetAttribute(k_p3<LOGN>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)p3_smem<LOGN>());
 }
@@ -293,21 +317,25 @@ cudaError_t configure_one() {
 template <int LOGN>
 void launch_p1(const Ctx &c, const FieldArgs &a, bool int_map, cudaStream_t s) {
   constexpr int NT = cfft::seq_per_cta(LOGN) * cfft::threads_per_seq(LOGN);
-  const int g = (c.mx + 2 * cfft::seq_per_cta(LOGN) - 1) / (2 * cfft::seq_per_cta(LOGN));
+  const int g = (a.nrows + 2 * cfft::seq_per_cta(LOGN) - 1) / (2 * cfft::seq_per_cta(LOGN));
   if (int_map)
     launch_chain(c.pdl, k_p1<unsigned long long, LOGN>, g, NT, p1_smem<LOGN>(), s, a);
   else
     launch_chain(c.pdl, k_p1<float, LOGN>, g, NT, p1_smem<LOGN>(), s, a);
 }
 template <int LOGN>
-void launch_p2(const Ctx &c, const FieldArgs &a, cudaStream_t s) {
+void launch_p2(const Ctx &c, const FieldArgs &a, bool tin, cudaStream_t s) {
   constexpr int NT = cfft::seq_per_cta(LOGN) * cfft::threads_per_seq(LOGN);
-  launch_chain(c.pdl, k_p2<LOGN>, p2_ctas(c.mx, c.my), NT, p2_smem<LOGN>(), s, a);
+  const int g = (a.ncols + 2 * cfft::seq_per_cta(LOGN) - 1) / (2 * cfft::seq_per_cta(LOGN));
+  if (tin)
+    launch_chain(c.pdl, k_p2<LOGN, true>, g, NT, p2_smem<LOGN>(), s, a);
+  else
+    launch_chain(c.pdl, k_p2<LOGN, false>, g, NT, p2_smem<LOGN>(), s, a);
 }
 template <int LOGN>
 void launch_p3(const Ctx &c, const FieldArgs &a, cudaStream_t s) {
   constexpr int NT = cfft::seq_per_cta(LOGN) * cfft::threads_per_seq(LOGN);
-  const int g = (c.mx + cfft::seq_per_cta(LOGN) - 1) / cfft::seq_per_cta(LOGN);
+  const int g = (a.nrows + cfft::seq_per_cta(LOGN) - 1) / cfft::seq_per_cta(LOGN);
   launch_chain(c.pdl, k_p3<LOGN>, g, NT, p3_smem<LOGN>(), s, a);
 }
 
@@ -344,15 +372,22 @@ cudaError_t fields_configure() {
 
 bool fields_cta_ok(int log2mx, int log2my) { return log2mx >= 4 && log2mx <= 12 && log2my >= 4 && log2my <= 12; }
 
-// P1 -> P2 -> P3 on stream s; rho is the int64 map (c.d_rho) or a float map (debug hook)
-void launch_fields_cta(const Ctx &c, const void *rho, bool int_map, cudaStream_t s) {
+namespace {
+FieldArgs field_args(const Ctx &c, const void *rho) {
   FieldArgs a;
   a.rho = rho;
-  a.tT = c.d_t;
-  a.sxy = c.d_sxy;
+  a.t_out = c.d_t;
+  a.t_in = c.d_t;
+  a.s_out = c.d_sxy;
+  a.s_in = c.d_sxy;
   a.xi = c.d_xi;
   a.mx = c.mx;
   a.my = c.my;
+  a.R = c.mx;
+  a.C = c.my;
+  a.x_base = a.y_base = 0;
+  a.nrows = c.mx;
+  a.ncols = c.my;
   a.twf_x = c.d_twf_x;
   a.twf_y = c.d_twf_y;
   a.ph_x = c.d_ph_x;
@@ -361,12 +396,68 @@ void launch_fields_cta(const Ctx &c, const void *rho, bool int_map, cudaStream_t
   a.ky = c.d_ky;
   a.energy_part = c.d_part + c.n_wa_part;
   a.energy_scale = 0.5 * c.bx * c.by;
+  return a;
+}
+
+// rank r of G: rows [r R, (r+1) R), columns [r C, (r+1) C); buffers as in the layout comment
+FieldArgs shard_args(const Ctx &c, const void *rho, int r, int G, float *s1, const float *r1, float2 *s2,
+                     const float2 *r2) {
+  FieldArgs a = field_args(c, rho);
+  a.R = c.mx / G;
+  a.C = c.my / G;
+  a.x_base = r * a.R;
+  a.y_base = r * a.C;
+  a.nrows = a.R;
+  a.ncols = a.C;
+  a.t_out = s1;
+  a.t_in = r1;
+  a.s_out = s2;
+  a.s_in = r2;
+  return a;
+}
+}  // namespace
+
+// P1 -> P2 -> P3 on stream s; rho is the int64 map (c.d_rho) or a float map (debug hook)
+void launch_fields_cta(const Ctx &c, const void *rho, bool int_map, cudaStream_t s) {
+  const FieldArgs a = field_args(c, rho);
 #define DP_P1(L) launch_p1<L>(c, a, int_map, s)
-#define DP_P2(L) launch_p2<L>(c, a, s)
+#define DP_P2(L) launch_p2<L>(c, a, true, s)
 #define DP_P3(L) launch_p3<L>(c, a, s)
   DP_FIELDS_DISPATCH(c.log2my, DP_P1)
   DP_FIELDS_DISPATCH(c.log2mx, DP_P2)
   DP_FIELDS_DISPATCH(c.log2my, DP_P3)
+#undef DP_P1
+#undef DP_P2
+#undef DP_P3
+}
+
+// P2 alone on t[x][y] as the warp-FFT row pass T1 writes it (the hybrid field path)
+void launch_p2_rowmajor(const Ctx &c, cudaStream_t s) {
+  const FieldArgs a = field_args(c, nullptr);
+#define DP_P2(L) launch_p2<L>(c, a, false, s)
+  DP_FIELDS_DISPATCH(c.log2mx, DP_P2)
+#undef DP_P2
+}
+
+bool fields_shardable(const Ctx &c, int G) {
+  if (!c.fft_cta || G < 1 || c.mx % G || c.my % G) return false;
+  const int R = c.mx / G, C = c.my / G;
+  // every P1 / P2 CTA lies inside one rank block: rows by 2 SEQ_y, columns by 2 SEQ_x
+  return R % (2 * cfft::seq_per_cta(c.log2my)) == 0 && C % (2 * cfft::seq_per_cta(c.log2mx)) == 0;
+}
+
+// One rank's passes of the row-sharded solve (the caller moves the blocks between them):
+// pass 1 = P1 on the rank's rows -> s1; pass 2 = P2 on its columns from r1 -> s2 (+ its energy
+// slots); pass 3 = P3 on its rows from r2 -> its rows of xi.
+void launch_fields_shard(const Ctx &c, int pass, const void *rho, bool int_map, int r, int G, float *s1,
+                         const float *r1, float2 *s2, const float2 *r2, cudaStream_t s) {
+  const FieldArgs a = shard_args(c, rho, r, G, s1, r1, s2, r2);
+#define DP_P1(L) launch_p1<L>(c, a, int_map, s)
+#define DP_P2(L) launch_p2<L>(c, a, true, s)
+#define DP_P3(L) launch_p3<L>(c, a, s)
+  if (pass == 1) DP_FIELDS_DISPATCH(c.log2my, DP_P1)
+  if (pass == 2) DP_FIELDS_DISPATCH(c.log2mx, DP_P2)
+  if (pass == 3) DP_FIELDS_DISPATCH(c.log2my, DP_P3)
 #undef DP_P1
 #undef DP_P2
 #undef DP_P3

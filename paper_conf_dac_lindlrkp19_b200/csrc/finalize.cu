@@ -42,6 +42,37 @@ __global__ void __launch_bounds__(256) k_combine_det(const long long *__restrict
   gy[c] = vy;
 }
 
+// Virtual shard (dp_create_dist without NCCL, tests): the gradient reduce-scatter is skipped, so
+// the shard's partial WA gradient is written for every cell (the sum over shards is the full
+// gradient) and lambda times the force for its own cells.
+__global__ void __launch_bounds__(256) k_combine_virtual(const float2 *__restrict__ g2, const long long *__restrict__ g2i,
+                                                         int frac, const float2 *__restrict__ force,
+                                                         float *__restrict__ gx, float *__restrict__ gy, int n,
+                                                         int cell_begin, int n_own, float lambda, int use_wa,
+                                                         int use_den) {
+  const int c = blockIdx.x * blockDim.x + threadIdx.x;
+  if (c >= n) return;
+  float vx = 0.f, vy = 0.f;
+  if (use_wa) {
+    if (g2i) {
+      const longlong2 q = reinterpret_cast<const longlong2 *>(g2i)[c];
+      vx = (float)ldexp((double)q.x, -frac);
+      vy = (float)ldexp((double)q.y, -frac);
+    } else {
+      const float2 q = g2[c];
+      vx = q.x;
+      vy = q.y;
+    }
+  }
+  if (use_den && c >= cell_begin && c < cell_begin + n_own) {
+    const float2 f = force[c - cell_begin];
+    vx = fmaf(lambda, f.x, vx);
+    vy = fmaf(lambda, f.y, vy);
+  }
+  gx[c] = vx;
+  gy[c] = vy;
+}
+
 __global__ void __launch_bounds__(256) k_combine(const float2 *__restrict__ g2, const float2 *__restrict__ force,
                                                  float *__restrict__ gx, float *__restrict__ gy, int cell_begin,
                                                  int n_own, float lambda, const float *__restrict__ lambda_dev,
@@ -199,6 +230,13 @@ __global__ void __launch_bounds__(256) k_finalize(FinArgs a) {
 
 void launch_combine(const Ctx &c, float lambda, float *gx, float *gy, bool use_wa, bool use_density,
                     cudaStream_t s) {
+  if (c.dist && !c.nccl_comm) {
+    k_combine_virtual<<<(c.num_cells + 255) / 256, 256, 0, s>>>(c.d_g2, c.deterministic ? c.d_g2i : nullptr,
+                                                                c.det_frac, c.d_force, gx, gy, c.num_cells,
+                                                                c.cell_begin, c.n_own, lambda, use_wa ? 1 : 0,
+                                                                use_density ? 1 : 0);
+    return;
+  }
   if (c.n_own <= 0) return;
   if (c.deterministic) {
     k_combine_det<<<(c.n_own + 255) / 256, 256, 0, s>>>(c.d_g2i, c.det_frac, c.d_force, gx, gy, c.cell_begin, c.n_own,

@@ -60,7 +60,7 @@ struct WaArgs {
   // big nets
   const int32_t *big_start, *big_flags, *big_cell;
   const float *big_w, *big_dx, *big_dy;
-  int part_offset;
+  int part_base;                // global WA unit of this launch's CTA 0: CTA b writes part[part_base + b]
   int hp_offset;                // MODE 4: fast-HPWL partials at part[hp_offset + the WA partial's index]
   int big_stage;   // pins staged in shared memory per big-net CTA
   int n_huge, n_big, n_warp_blocks;
@@ -710,8 +710,9 @@ __device__ __forceinline__ void wa_big_net(const WaArgs &a, int net, float4 *s_p
     }
   }
   __syncthreads();
-  block_flush_scalars<kBigThreads>(wl_acc, L, kHpwl, kGrad ? a.part + a.part_offset + net : nullptr,
-                                   a.limbs, hp_b, MODE == 4 ? a.part + a.hp_offset + a.part_offset + net : nullptr);
+  const int slot = a.part_base + blockIdx.x;
+  block_flush_scalars<kBigThreads>(wl_acc, L, kHpwl, kGrad ? a.part + slot : nullptr, a.limbs, hp_b,
+                                   MODE == 4 ? a.part + a.hp_offset + slot : nullptr);
 }
 
 // Warp per net for degrees (kWaMaxDeg, kWarpNetMax]: three passes over the pins with warp
@@ -869,9 +870,9 @@ __device__ __forceinline__ void wa_warp_nets(const WaArgs &a, int wb) {
       }
     }
   }
-  block_flush_scalars<kWarpNetThreads>(wl_acc, L, kHpwl, kGrad ? a.part + a.part_offset + a.n_huge + wb : nullptr,
-                                       a.limbs, hp_w,
-                                       MODE == 4 ? a.part + a.hp_offset + a.part_offset + a.n_huge + wb : nullptr);
+  const int slot = a.part_base + blockIdx.x;
+  block_flush_scalars<kWarpNetThreads>(wl_acc, L, kHpwl, kGrad ? a.part + slot : nullptr, a.limbs, hp_w,
+                                       MODE == 4 ? a.part + a.hp_offset + slot : nullptr);
 }
 
 // MODE 0: WA + gradient; 1: WA + gradient + HPWL; 2: HPWL only; 3: LSE + gradient (NEXT-3);
@@ -1070,8 +1071,9 @@ __global__ void __launch_bounds__(kWaThreads, 2) k_wa_chunks(const WaArgs a0) {
       if (gx | gy) red_v2(a.g2 + s_far[f], gx * inv, gy * inv);
     }
   }
-  block_flush_scalars<kWaThreads>((double)wl_acc, L, kHpwl, kGrad ? a.part + chunk : nullptr, a.limbs,
-                                  (double)hp_acc, MODE == 4 ? a.part + a.hp_offset + chunk : nullptr);
+  block_flush_scalars<kWaThreads>((double)wl_acc, L, kHpwl, kGrad ? a.part + a.part_base + blockIdx.x : nullptr,
+                                  a.limbs, (double)hp_acc,
+                                  MODE == 4 ? a.part + a.hp_offset + a.part_base + blockIdx.x : nullptr);
 }
 
 template <int MODE>
@@ -1135,7 +1137,7 @@ void launch_wa(const Ctx &c, const float *x, const float *y, float gamma, bool h
   a.big_w = c.d_big_w;
   a.big_dx = c.d_big_dx;
   a.big_dy = c.d_big_dy;
-  a.part_offset = c.n_chunks;
+  a.part_base = c.part_base;
   a.hp_offset = c.n_wa_part + c.n_en_part + 1;
   a.n_huge = c.n_huge;
   a.n_big = c.n_big;

@@ -1,10 +1,10 @@
-"""Multi-process check of the distributed partition (owner computes) on CPU.
+"""Multi-process check of the distributed partition on CPU.
 
-Two gloo ranks each take libdp's host-only partition plan (dp_partition_plan), evaluate their
-shard with the fp64 oracle exactly as a distributed context does (nets touching own cells, the
-gradient of own cells only, WA / HPWL counted once, the density map of own cells), combine with
-the same collectives the GPU path uses (sum of the bin map, sum of WA, sum of HPWL terms) and must
-reproduce the single-process oracle."""
+gloo ranks each take libdp's host-only partition plan (dp_partition_plan), evaluate their shard
+with the fp64 oracle exactly as a distributed context does (WA over the rank's own nets with a
+gradient over all cells, the density map of the rank's cell block), combine with the
+collectives the GPU path uses (gradient sum = reduce-scatter, bin-map sum, WA partial sum, HPWL
+terms) and must reproduce the single-process oracle."""
 import math
 import os
 import socket
@@ -27,8 +27,8 @@ def _free_port():
 def _shard_eval(nl, x, y, gamma, cb, ce, mask):
     import oracle
     from synth import custom_netlist
-    # WA over the nets this rank evaluates (mask & 1); gradient kept for own cells only
-    sel = np.nonzero(mask & 1)[0]
+    # WA over the nets this rank evaluates (mask 3, each net on one rank); gradient on every cell
+    sel = np.nonzero(mask == 3)[0]
     starts = nl.net_start
     deg = starts[sel + 1] - starts[sel]
     ns = np.concatenate([[0], np.cumsum(deg)])
@@ -36,13 +36,8 @@ def _shard_eval(nl, x, y, gamma, cb, ce, mask):
     sub = custom_netlist(ns, nl.pin2cell[pins], nl.pin_dx[pins], nl.pin_dy[pins], nl.cell_w, nl.cell_h,
                          (nl.xl, nl.yl, nl.xh, nl.yh), (nl.bins_x, nl.bins_y))
     _, gx, gy, wl_net = oracle.wa(sub, x, y, gamma, per_net=True)
-    own = np.zeros(nl.num_cells, bool)
-    own[cb:ce] = True
-    gx[~own] = 0.0
-    gy[~own] = 0.0
-    counted = (mask[sel] & 2) != 0
-    wl = float(np.sum(wl_net[counted]))
-    h = oracle.hpwl_nets(sub, x, y)[counted]
+    wl = float(np.sum(wl_net))
+    h = oracle.hpwl_nets(sub, x, y)
     # density: this rank's cells only
     cells = custom_netlist([0], [], [], [], nl.cell_w[cb:ce], nl.cell_h[cb:ce], (nl.xl, nl.yl, nl.xh, nl.yh),
                            (nl.bins_x, nl.bins_y))
@@ -67,7 +62,7 @@ def _worker(rank, world, port, q):
     rho_t = torch.from_numpy(rho.copy())
     dist.all_reduce(rho_t)                               # bin map (the GPU path sums int64)
     g = torch.from_numpy(np.stack([gx, gy]))
-    dist.all_reduce(g)                                   # disjoint own ranges: assembles the gradient
+    dist.all_reduce(g)                                   # partial gradients of disjoint net sets (reduce-scatter)
     hs = [None] * world
     dist.all_gather_object(hs, h.tolist())
     # replicated Poisson solve on the summed map, force for own cells
@@ -86,8 +81,8 @@ def _worker(rank, world, port, q):
     dist.destroy_process_group()
 
 
-@pytest.mark.parametrize("world", [2])
-def test_owner_computes_shards_reassemble_the_oracle(world):
+@pytest.mark.parametrize("world", [2, 3])
+def test_net_partitioned_shards_reassemble_the_oracle(world):
     import oracle
     from synth import make_netlist, make_positions
     ctx = mp.get_context("spawn")

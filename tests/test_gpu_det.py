@@ -94,3 +94,28 @@ def test_det_gp_trajectory_bitwise():
     (h0, x0, y0), (h1, x1, y1) = runs
     assert h0 == h1
     assert np.array_equal(x0, x1) and np.array_equal(y0, y1)
+
+
+@pytest.mark.parametrize("world", [2, 3, 8])
+def test_det_gradient_bitwise_across_world_sizes(world):
+    """NEXT-2 across partitions: in deterministic mode the WA work units and their
+    fixed-point scales do not depend on the number of ranks, so the exact int64
+    partial gradients of `world` virtual shards sum (what the int64 reduce-scatter does) to the
+    single context's accumulator bit for bit (the int64 bin map is exact for any partition:
+    test_gpu_parity.py::test_virtual_shards_reassemble / test_one_rank_nccl_context)."""
+    nl = make_netlist("adaptec1")
+    x, y = make_positions(nl, "spread")
+    xt, yt = _t(x), _t(y)
+    single = dp.dp_create(nl)
+    dp.dp_set_deterministic(single, True)
+    single.wl_grad(xt, yt, nl.bin_w)
+    ref = dp.dp_debug_wa_accumulator(single)[: nl.num_cells]
+    acc = None
+    for r in range(world):
+        ctx = dp.dp_create_dist(nl, 0, r, world, None)
+        dp.dp_set_deterministic(ctx, True)
+        ctx.wl_grad(xt, yt, nl.bin_w)
+        part = dp.dp_debug_wa_accumulator(ctx)[: nl.num_cells]
+        acc = part.clone() if acc is None else acc + part
+        ctx.close()
+    assert torch.equal(acc, ref)

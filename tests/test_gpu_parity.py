@@ -321,9 +321,9 @@ def test_density_bitwise_deterministic(tiny, dist):
 @pytest.mark.parametrize("world", [2, 3])
 def test_virtual_shards_reassemble(world):
     """dp_create_dist with no NCCL id (collectives skipped) on one GPU, one context per rank: the
-    owner-computes partition must reassemble the single-context results — WA and
-    its gradient (own cells per rank, every net counted once), HPWL, and the int64 bin map of
-    each rank's own cells summing to the full map."""
+    net / cell partition must reassemble the single-context results — WA and its
+    gradient (each rank's partial gradient over all cells: the sum the reduce-scatter forms),
+    HPWL, and the int64 bin map of each rank's cell block summing to the full map."""
     nl = make_netlist("tiny")
     x, y = make_positions(nl)
     gamma = nl.bin_w
@@ -342,13 +342,13 @@ def test_virtual_shards_reassemble(world):
         ctx = dp.dp_create_dist(nl, 0, r, world, None)
         out = ctx.wl_grad(_t(x), _t(y), gamma)
         wl += out["wl"].item()
-        gx[cb:ce] += out["gx"][cb:ce].double()
-        gy[cb:ce] += out["gy"][cb:ce].double()
+        gx += out["gx"].double()
+        gy += out["gy"].double()
         hp += ctx.hpwl(_t(x), _t(y)).item()
         rho += ctx.density_map(_t(x), _t(y)).double()
     assert (covered == 1).all()
     check_scalar("WA", wl, ref["wl"].item(), rel=1e-6)
-    # shards chunk their nets differently (fixed-point scales, fp32 flush order): the oracle's bar
+    # the gradient sums (fp32 atomics, different per-rank flush order): the oracle's bar
     check_vector("dWA/dx", to_np(gx), to_np(ref["gx"]))
     check_vector("dWA/dy", to_np(gy), to_np(ref["gy"]))
     assert hp == pytest.approx(oracle.hpwl(nl, x, y), rel=1e-14)
@@ -424,3 +424,49 @@ def test_eval_industrial():
     assert out["hpwl"].item() == ref["hpwl"]
     check_vector("gx", to_np(out["gx"]), ref["gx"])
     check_vector("gy", to_np(out["gy"]), ref["gy"])
+
+
+@pytest.mark.parametrize("bins,world", [(256, 2), (256, 4), (2048, 2), (2048, 8)])
+def test_sharded_poisson_emulated_bit_identical(bins, world):
+    """The row-sharded Poisson solve (P1 on each rank's rows, all-to-all, P2 on its
+    columns, all-to-all, P3 on its rows) with `world` ranks emulated on one GPU: the same
+    kernels on per-rank layouts must reproduce the unsharded solve bit for bit (every 1-D
+    transform sees the same inputs in the same order; the energy slots are per column slab),
+    and the oracle."""
+    nl = custom_netlist([0], [], [], [], [1.0], [1.0], (0, 0, 10.0 * bins, 10.0 * bins), (bins, bins))
+    import os
+    os.environ["DP_FFT"] = "1"   # the CTA-FFT passes also at 256
+    try:
+        ctx = dp.dp_create(nl)
+    finally:
+        del os.environ["DP_FFT"]
+    rho = np.random.default_rng(bins + world).random((bins, bins)) * 2.0
+    ref = ctx.fields(_t(rho), want_psi=False)
+    ref = {k: (v.clone() if torch.is_tensor(v) else v) for k, v in ref.items()}
+    sh = dp.dp_debug_sharded_fields(ctx, world, _t(rho))
+    assert torch.equal(sh["xi_x"], ref["xi_x"]) and torch.equal(sh["xi_y"], ref["xi_y"])
+    assert sh["energy"].item() == ref["energy"].item()
+    if bins <= 256:
+        rho32 = rho.astype(np.float32).astype(np.float64)
+        psi, xi_x, xi_y = oracle.fields(nl, oracle.dct2(rho32))
+        check_map("xi_x", to_np(sh["xi_x"]), xi_x)
+        check_scalar("energy", sh["energy"].item(), oracle.energy(nl, rho32, psi))
+
+
+def test_one_rank_nccl_sharded_poisson():
+    """A one-rank NCCL context on a 2048^2 map takes the row-sharded solve (reduce-scatter of the
+    map, two all-to-alls, all-gather of the field through NCCL, here with one rank): the
+    evaluation equals the single context bit for bit in energy and HPWL, and the gradient."""
+    nl = make_netlist("adaptec1", bins=2048)
+    x, y = make_positions(nl)
+    xt, yt = _t(x), _t(y)
+    single = dp.dp_create(nl)
+    a = single.eval(xt, yt, nl.bin_w, 1.0, with_hpwl=True)
+    a = {k: (v.clone() if torch.is_tensor(v) else v) for k, v in a.items()}
+    ctx = dp.dp_create_dist(nl, 0, 0, 1, dp.dp_nccl_unique_id())
+    b = ctx.eval(xt, yt, nl.bin_w, 1.0, with_hpwl=True)
+    torch.cuda.synchronize()
+    assert b["energy"].item() == a["energy"].item()
+    assert b["hpwl"].item() == a["hpwl"].item()
+    check_vector("gx", to_np(b["gx"]), to_np(a["gx"]))
+    check_vector("gy", to_np(b["gy"]), to_np(a["gy"]))

@@ -63,10 +63,15 @@ def mu(p: float, k: int, prm: GpParams) -> float:
     return max(prm.mu_min, prm.mu_max ** (1.0 - p))
 
 
-def overflow(nl, rho: np.ndarray, target: float) -> float:
-    """A30: sum_b max(rho_b - t, 0) b_x b_y / total cell area."""
-    area = float(np.sum(nl.cell_w.astype(np.float64) * nl.cell_h.astype(np.float64)))
-    return float(np.sum(np.maximum(rho - target, 0.0))) * nl.bin_w * nl.bin_h / area
+def overflow(nl, rho: np.ndarray, target: float, fixed=None, rho_fixed=None) -> float:
+    """A30: sum_b max(rho_b - t, 0) b_x b_y / total cell area.  With fixed cells (A34; the
+    DREAMPlace convention): the fixed charge counts at the target density, rho_eff = rho_movable
+    + t rho_fixed = rho - (1 - t) rho_fixed, and the sum is divided by the movable area."""
+    a = nl.cell_w.astype(np.float64) * nl.cell_h.astype(np.float64)
+    if fixed is not None:
+        a = a[~np.asarray(fixed, dtype=bool)]
+        rho = rho - (1.0 - target) * rho_fixed
+    return float(np.sum(np.maximum(rho - target, 0.0))) * nl.bin_w * nl.bin_h / float(np.sum(a))
 
 
 def gamma_of(nl, tau: float, prm: GpParams) -> float:

@@ -375,12 +375,34 @@ def dp_partition_plan(nl, rank: int, world: int):
     return cb.value, ce.value, mask[: int(nl.num_nets)]
 
 
+def _vec(ctx, t, name, dtype="float32", n=None):
+    """Argument check of a device vector passed to the C ABI (the library trusts its pointers):
+    a contiguous CUDA tensor of `dtype` on the context's device with at least n elements."""
+    if t is None or not hasattr(t, "data_ptr"):
+        return
+    import torch
+    want = getattr(torch, dtype)
+    n = ctx.num_cells if n is None else n
+    if t.dtype != want or not t.is_cuda or t.device.index != ctx.device or not t.is_contiguous() or t.numel() < n:
+        raise ValueError(f"{name}: need a contiguous {dtype} CUDA tensor on cuda:{ctx.device} with >= {n} "
+                         f"elements (got {t.dtype}, {t.device}, contiguous={t.is_contiguous()}, numel={t.numel()})")
+
+
+def _check_eval_args(ctx, x, y, gx=None, gy=None, scalars=()):
+    for t, name in ((x, "x"), (y, "y"), (gx, "gx"), (gy, "gy")):
+        _vec(ctx, t, name)
+    for t in scalars:
+        _vec(ctx, t, "scalar output", "float64", 1)
+
+
 def dp_eval(ctx, x, y, gamma, lam, gx, gy, d_obj=None, d_wl=None, d_energy=None, d_hpwl=None, stream=None):
+    _check_eval_args(ctx, x, y, gx, gy, (d_obj, d_wl, d_energy, d_hpwl))
     _check(lib().dp_eval(ctx.handle, _ptr(x), _ptr(y), float(gamma), float(lam), _ptr(gx), _ptr(gy),
                          _ptr(d_obj), _ptr(d_wl), _ptr(d_energy), _ptr(d_hpwl), _stream(stream)))
 
 
 def dp_wl_grad(ctx, x, y, gamma, gx, gy, d_wl=None, stream=None):
+    _check_eval_args(ctx, x, y, gx, gy, (d_wl,))
     _check(lib().dp_wl_grad(ctx.handle, _ptr(x), _ptr(y), float(gamma), _ptr(gx), _ptr(gy), _ptr(d_wl),
                             _stream(stream)))
 
@@ -405,11 +427,13 @@ def dp_set_wl_model(ctx, model: int):
 
 
 def dp_density_grad(ctx, x, y, gx, gy, d_energy=None, stream=None):
+    _check_eval_args(ctx, x, y, gx, gy, (d_energy,))
     _check(lib().dp_density_grad(ctx.handle, _ptr(x), _ptr(y), _ptr(gx), _ptr(gy), _ptr(d_energy),
                                  _stream(stream)))
 
 
 def dp_hpwl(ctx, x, y, d_hpwl, stream=None):
+    _check_eval_args(ctx, x, y, scalars=(d_hpwl,))
     _check(lib().dp_hpwl(ctx.handle, _ptr(x), _ptr(y), _ptr(d_hpwl), _stream(stream)))
 
 

@@ -21,6 +21,7 @@
 #include <string>
 #include <vector>
 #include <map>
+#include <mutex>
 #include <cstring>
 
 #include "dp_internal.h"
@@ -120,6 +121,16 @@ dp_status validate(const dp_netlist *nl, const dp_grid *g) {
   return DP_OK;
 }
 
+// Dynamic shared-memory opt-ins are per device: the maxima configured so far on each device
+// (several contexts, possibly on several GPUs, in one process).
+struct DeviceConfig {
+  WaCaps wa{4, 4, 4, 4};
+  bool wa_set = false;
+  int max_m = 0, max_tiles = 0, max_tile = 0;
+};
+std::mutex g_cfg_mutex;
+std::map<int, DeviceConfig> g_cfg;
+
 int g_class(int d) {  // log2 of lanes per net
   int g = 0;
   while ((kWaPpl << g) < d) g++;
@@ -146,6 +157,9 @@ struct WaPlan {
 
 WaPlan wa_plan(const dp_netlist *nl, int world) {
   WaPlan P;
+  // DP_WA_CHUNK = pins per chunk (A/B; smaller chunks stage less shared memory per CTA)
+  const char *ce = std::getenv("DP_WA_CHUNK");
+  const int chunk_pins = ce ? std::max(256, std::min(kWaChunkPins, std::atoi(ce))) : kWaChunkPins;
   auto pin_of = [&](int32_t slot) { return nl->net2pin ? nl->net2pin[slot] : slot; };
   auto deg = [&](int32_t e) { return nl->net_start[e + 1] - nl->net_start[e]; };
   for (int32_t e = 0; e < nl->num_nets; e++) {
@@ -170,7 +184,7 @@ WaPlan wa_plan(const dp_netlist *nl, int world) {
     int pins = 0;
     while (j < P.small.size()) {
       const int d = deg(P.small[j]);
-      if (j > i && pins + d > kWaChunkPins) break;
+      if (j > i && pins + d > chunk_pins) break;
       pins += d;
       j++;
     }
@@ -390,17 +404,17 @@ dp_status build_wa(Ctx &c, const dp_netlist *nl, const WaPlan &P) {
   c.n_wgroups = (int32_t)wgs.size();
   c.n_wa_nets = (int32_t)net_deg.size();
   c.n_wa_pins = (int32_t)pin_cell.size();
-  {
-    static WaCaps max_caps{4, 4, 4, 4};
-    static bool configured = false;
-    WaCaps m{std::max(max_caps.pins, caps.pins), std::max(max_caps.nets, caps.nets),
-             std::max(max_caps.groups, caps.groups), std::max(max_caps.far, caps.far)};
+  {   // shared-memory opt-in: per device (cudaFuncSetAttribute is), the maxima over its contexts
+    std::lock_guard<std::mutex> lock(g_cfg_mutex);
+    DeviceConfig &dc = g_cfg[c.device];
+    WaCaps m{std::max(dc.wa.pins, caps.pins), std::max(dc.wa.nets, caps.nets),
+             std::max(dc.wa.groups, caps.groups), std::max(dc.wa.far, caps.far)};
     if (wa_smem_bytes(m) > 227 * 1024) return fail(DP_ERR_UNSUPPORTED, "WA chunk staging exceeds shared memory");
-    if (!configured || m.pins != max_caps.pins || m.nets != max_caps.nets || m.groups != max_caps.groups ||
-        m.far != max_caps.far) {
+    if (!dc.wa_set || m.pins != dc.wa.pins || m.nets != dc.wa.nets || m.groups != dc.wa.groups ||
+        m.far != dc.wa.far) {
       DP_CUDA(wa_configure(m));
-      max_caps = m;
-      configured = true;
+      dc.wa = m;
+      dc.wa_set = true;
     }
     c.wa_caps = caps;
   }
@@ -540,18 +554,20 @@ dp_status build_density(Ctx &c, const dp_netlist *nl) {
   for (int v = 0; v < c.my; v++) ky[v] = (float)(M_PI * v / (c.yh - c.yl));
   if ((st = dev_upload(c, &c.d_kx, kx)) != DP_OK) return st;
   if ((st = dev_upload(c, &c.d_ky, ky)) != DP_OK) return st;
-  // shared-memory opt-in (process-wide maxima)
-  static int max_m = 0, max_tiles = 0, max_tile = 0;
-  const int m = std::max(c.mx, c.my);
-  if (m > max_m || c.mx != c.my) {
-    DP_CUDA(dct_configure(std::max(c.mx, max_m), std::max(c.my, max_m)));
-    DP_CUDA(fields_configure());
-    max_m = std::max(max_m, m);
-  }
-  if (ntiles > max_tiles || c.tile > max_tile) {
-    max_tiles = std::max(max_tiles, ntiles);
-    max_tile = std::max(max_tile, c.tile);
-    DP_CUDA(density_configure(max_tiles, max_tile));
+  {   // shared-memory opt-in: per device, the maxima over its contexts
+    std::lock_guard<std::mutex> lock(g_cfg_mutex);
+    DeviceConfig &dc = g_cfg[c.device];
+    const int m = std::max(c.mx, c.my);
+    if (m > dc.max_m || c.mx != c.my) {
+      DP_CUDA(dct_configure(std::max(c.mx, dc.max_m), std::max(c.my, dc.max_m)));
+      DP_CUDA(fields_configure());
+      dc.max_m = std::max(dc.max_m, m);
+    }
+    if (ntiles > dc.max_tiles || c.tile > dc.max_tile) {
+      dc.max_tiles = std::max(dc.max_tiles, ntiles);
+      dc.max_tile = std::max(dc.max_tile, c.tile);
+      DP_CUDA(density_configure(dc.max_tiles, dc.max_tile));
+    }
   }
   c.walk_grid = density_walk_grid(c.tile);
   c.count_grid = density_count_grid(c.tiles_x * c.tiles_y);
@@ -662,7 +678,7 @@ dp_status create(const dp_netlist *nl, const dp_grid *grid, int device, int rank
   }
   // energy partials: one per CTA of the column pass (P2 of the CTA-FFT path; 2-column slabs of
   // the warp-FFT path)
-  c->n_en_part = (c->fft_cta || c->fft_hybrid) ? p2_ctas(c->mx, c->my) : c->my / 2;
+  c->n_en_part = (c->fft_cta || c->fft_hybrid) ? p2_ctas(c->mx, c->my, c->fft_hybrid) : c->my / 2;
   // one "hot" arena for the two per-cell vectors the combine reads: the WA accumulator g2
   // [num_cells] and the force [n_own + 4] (offset by the parity of cell_begin so that even
   // global cells are 16-byte aligned: the combine reads cell pairs as float4).  It is the
@@ -1127,6 +1143,7 @@ dp_status dp_wl_grad(dp_ctx *ctx, const float *x, const float *y, float gamma, f
 }
 
 dp_status dp_set_wl_model(dp_ctx *ctx, int32_t model) {
+  if (ctx) C(ctx)->config_gen++;
   Ctx *c = C(ctx);
   if (!c) return fail(DP_ERR_INVALID_ARG, "ctx is NULL");
   if (model != DP_WL_WA && model != DP_WL_LSE) return fail(DP_ERR_INVALID_ARG, "unknown wirelength model");
@@ -1135,6 +1152,7 @@ dp_status dp_set_wl_model(dp_ctx *ctx, int32_t model) {
 }
 
 dp_status dp_set_deterministic(dp_ctx *ctx, int32_t on) {
+  if (ctx) C(ctx)->config_gen++;
   Ctx *c = C(ctx);
   if (!c) return fail(DP_ERR_INVALID_ARG, "ctx is NULL");
   if (on && !c->d_g2i) {
@@ -1147,6 +1165,7 @@ dp_status dp_set_deterministic(dp_ctx *ctx, int32_t on) {
 }
 
 dp_status dp_set_fixed(dp_ctx *ctx, const uint8_t *h_fixed, const float *x, const float *y, dp_stream_t stream) {
+  if (ctx) C(ctx)->config_gen++;
   Ctx *c = C(ctx);
   if (!c) return fail(DP_ERR_INVALID_ARG, "ctx is NULL");
   if (c->dist) return fail(DP_ERR_UNSUPPORTED, "fixed cells are supported on single-GPU contexts");

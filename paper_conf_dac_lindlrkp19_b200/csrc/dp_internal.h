@@ -216,6 +216,7 @@ struct Ctx {
   int32_t n_wa_part = 0, n_en_part = 0;   // WA partials: one slot per global WA unit (all ranks)
   int32_t part_base = 0;                   // this rank's first WA unit
   int32_t cell_blk = 0;                    // cells per rank block of the gradient reduce-scatter
+  int64_t config_gen = 0;                  // bumped by every dp_set_*: graphs captured earlier are stale
   bool shard_poisson = false;              // row-sharded Poisson solve (dist, maps > 1024)
   int64_t g2_cells = 0;                    // WA accumulator length (dist: world blocks; else num_cells)
   unsigned long long *d_limbs = nullptr;  // HPWL fixed-point limbs
@@ -274,7 +275,7 @@ void launch_psi(const Ctx &c, const float *rho, float *psi, cudaStream_t s);
 // CTA-FFT field passes (fields.cu): P1 rows, P2 columns (+ energy), P3 rows
 cudaError_t fields_configure();
 bool fields_cta_ok(int log2mx, int log2my);
-int p2_ctas(int mx, int my);
+int p2_ctas(int mx, int my, bool hybrid = false);
 void launch_fields_cta(const Ctx &c, const void *rho, bool int_map, cudaStream_t s);
 void launch_p2_rowmajor(const Ctx &c, cudaStream_t s);
 bool fields_shardable(const Ctx &c, int G);

@@ -145,11 +145,17 @@ __global__ void __launch_bounds__(cfft::seq_per_cta(LOGN) * cfft::threads_per_se
 // ---- P2: columns (2p, 2p+1) (rows of tT) -> DCT over x, energy, scaling, inverse over x ----
 // TIN: t stored transposed, tT[y][x] (after P1); otherwise t[x][y] (after the warp-FFT T1):
 // the CTA then reads its COLS adjacent columns as 4 COLS-byte row segments.
+// P2 of the hybrid path runs one column pair per CTA (SEQ = 1): half the shared memory and
+// threads of a CTA, so its CTAs fit beside the WA kernel's (the unsharded / sharded CTA-FFT
+// path keeps seq_per_cta)
+template <int LOGM, bool TIN>
+constexpr int p2_seq() { return TIN ? cfft::seq_per_cta(LOGM) : 1; }
+
 template <int LOGM, bool TIN = true>
-__global__ void __launch_bounds__(cfft::seq_per_cta(LOGM) * cfft::threads_per_seq(LOGM))
+__global__ void __launch_bounds__(p2_seq<LOGM, TIN>() * cfft::threads_per_seq(LOGM))
     k_p2(FieldArgs a) {
   griddep_wait();
-  constexpr int M = 1 << LOGM, T = cfft::threads_per_seq(LOGM), SEQ = cfft::seq_per_cta(LOGM);
+  constexpr int M = 1 << LOGM, T = cfft::threads_per_seq(LOGM), SEQ = p2_seq<LOGM, TIN>();
   constexpr int NT = SEQ * T, COLS = 2 * SEQ, L = buf_len(M);
   extern __shared__ __align__(16) float2 sm2[];
   float2 *spec = sm2 + 2 * SEQ * L;    // [COLS][M] (A_X, A_Y)
@@ -286,10 +292,10 @@ constexpr size_t p1_smem() {
   return sizeof(float2) * 2 * cfft::seq_per_cta(LOGN) * buf_len(1 << LOGN) +
          sizeof(float) * (size_t)(1 << LOGN) * 2 * cfft::seq_per_cta(LOGN);
 }
-template <int LOGN>
+template <int LOGN, bool TIN = true>
 constexpr size_t p2_smem() {
-  return sizeof(float2) * (2 * cfft::seq_per_cta(LOGN) * buf_len(1 << LOGN) +
-                           2 * (size_t)(2 * cfft::seq_per_cta(LOGN)) * (1 << LOGN));
+  return sizeof(float2) * (2 * p2_seq<LOGN, TIN>() * buf_len(1 << LOGN) +
+                           2 * (size_t)(2 * p2_seq<LOGN, TIN>()) * (1 << LOGN));
 }
 template <int LOGN>
 constexpr size_t p3_smem() {
@@ -309,7 +315,7 @@ cudaError_t configure_one() {
                                 (int)p2_smem<LOGN>())) != cudaSuccess)
     return e;
   if ((e = cudaFuncSetAttribute(k_p2<LOGN, false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                (int)p2_smem<LOGN>())) != cudaSuccess)
+                                (int)p2_smem<LOGN, false>())) != cudaSuccess)
     return e;
   return cudaFuncSetAttribute(k_p3<LOGN>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)p3_smem<LOGN>());
 }
@@ -325,12 +331,13 @@ void launch_p1(const Ctx &c, const FieldArgs &a, bool int_map, cudaStream_t s) {
 }
 template <int LOGN>
 void launch_p2(const Ctx &c, const FieldArgs &a, bool tin, cudaStream_t s) {
-  constexpr int NT = cfft::seq_per_cta(LOGN) * cfft::threads_per_seq(LOGN);
-  const int g = (a.ncols + 2 * cfft::seq_per_cta(LOGN) - 1) / (2 * cfft::seq_per_cta(LOGN));
-  if (tin)
-    launch_chain(c.pdl, k_p2<LOGN, true>, g, NT, p2_smem<LOGN>(), s, a);
-  else
-    launch_chain(c.pdl, k_p2<LOGN, false>, g, NT, p2_smem<LOGN>(), s, a);
+  if (tin) {
+    constexpr int SEQ = p2_seq<LOGN, true>(), NT = SEQ * cfft::threads_per_seq(LOGN);
+    launch_chain(c.pdl, k_p2<LOGN, true>, (a.ncols + 2 * SEQ - 1) / (2 * SEQ), NT, p2_smem<LOGN, true>(), s, a);
+  } else {
+    constexpr int SEQ = p2_seq<LOGN, false>(), NT = SEQ * cfft::threads_per_seq(LOGN);
+    launch_chain(c.pdl, k_p2<LOGN, false>, (a.ncols + 2 * SEQ - 1) / (2 * SEQ), NT, p2_smem<LOGN, false>(), s, a);
+  }
 }
 template <int LOGN>
 void launch_p3(const Ctx &c, const FieldArgs &a, cudaStream_t s) {
@@ -355,9 +362,9 @@ void launch_p3(const Ctx &c, const FieldArgs &a, cudaStream_t s) {
 }  // namespace
 
 // energy partials of P2: one per CTA
-int p2_ctas(int mx, int my) {
+int p2_ctas(int mx, int my, bool hybrid) {
   const int logm = ilog2_int(mx);
-  const int cols = 2 * cfft::seq_per_cta(logm);
+  const int cols = 2 * (hybrid ? 1 : cfft::seq_per_cta(logm));
   return (my + cols - 1) / cols;
 }
 

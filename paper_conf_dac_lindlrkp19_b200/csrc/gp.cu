@@ -46,10 +46,12 @@ struct GpDev {      // device-resident loop state (scalars)
 
 struct GpArgs {
   int n;
+  const uint8_t *fixed;    // NEXT-4 (reading A34): fixed cells are not variables (null: none)
   float *ux, *uy, *vx, *vy, *vpx, *vpy, *gx, *gy, *gpx, *gpy, *rgx, *rgy;
   const float *w, *h, *pins;
   float xl, yl, xh, yh;
   const unsigned long long *rho;
+  const unsigned long long *rho_fixed;   // fixed-charge map (dp_set_fixed), null if none
   long long nbins;
   double rho_unit;         // 2^-kRhoScaleLog2
   double target;
@@ -92,16 +94,22 @@ __device__ __forceinline__ void block_pair(double s0, double s1, double *part) {
 
 enum { R_NORMS = 0, R_L1 = 1, R_SQ = 2, R_OVF = 3 };
 
+// A30 with fixed macros (the DREAMPlace convention): the fixed charge counts at the
+// target density, rho_eff = rho_movable + t rho_fixed = rho - (1 - t) rho_fixed, so a bin that a
+// macro covers overflows only by its movable charge; the sum is divided by the movable area
+__device__ __forceinline__ double ovf_term(const GpArgs &a, long long b) {
+  double r = (double)a.rho[b] * a.rho_unit;
+  if (a.rho_fixed) r -= (1.0 - a.target) * ((double)a.rho_fixed[b] * a.rho_unit);
+  return fmax(r - a.target, 0.0);
+}
+
 // Per-block partial sums.  R_NORMS: (|v - vp|^2, |g - gp|^2); R_L1: (|rg|_1, 0);
 // R_SQ: (|g|^2, 0); R_OVF: (sum_b max(rho_b - t, 0), 0).
 __global__ void __launch_bounds__(kGpThreads) k_gp_partials(GpArgs a, int mode) {
   double s0 = 0.0, s1 = 0.0;
   const int stride = gridDim.x * kGpThreads;
   if (mode == R_OVF) {
-    for (long long b = blockIdx.x * kGpThreads + threadIdx.x; b < a.nbins; b += stride) {
-      const double r = (double)a.rho[b] * a.rho_unit;
-      s0 += fmax(r - a.target, 0.0);
-    }
+    for (long long b = blockIdx.x * kGpThreads + threadIdx.x; b < a.nbins; b += stride) s0 += ovf_term(a, b);
   } else {
     for (int i = blockIdx.x * kGpThreads + threadIdx.x; i < a.n; i += stride) {
       if (mode == R_NORMS) {
@@ -240,6 +248,11 @@ __device__ __forceinline__ float clampf(float v, float lo, float hi) { return fm
 __global__ void __launch_bounds__(kGpThreads) k_gp_update(GpArgs a) {
   const int i = blockIdx.x * kGpThreads + threadIdx.x;
   if (i >= a.n || a.dev->frozen) return;
+  if (a.fixed && a.fixed[i]) {   // not a variable: u, v stay (its gradient is 0 as well)
+    a.vpx[i] = a.vx[i]; a.vpy[i] = a.vy[i];
+    a.gpx[i] = a.gx[i]; a.gpy[i] = a.gy[i];
+    return;
+  }
   const float alpha = a.dev->f_alpha, coef = a.dev->f_coef;
   const float hx = a.xh - a.w[i], hy = a.yh - a.h[i];
   const float vx = a.vx[i], vy = a.vy[i], gx = a.gx[i], gy = a.gy[i];
@@ -282,7 +295,7 @@ __global__ void __launch_bounds__(kGpThreads) k_gp_post(GpArgs a) {
   } else {
     const int b0 = blockIdx.x - a.nblk;
     for (long long b = (long long)b0 * kGpThreads + threadIdx.x; b < a.nbins; b += (long long)a.oblk * kGpThreads)
-      s0 += fmax((double)a.rho[b] * a.rho_unit - a.target, 0.0);
+      s0 += ovf_term(a, b);
     __shared__ double r0[kGpThreads / 32];
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) s0 += __shfl_xor_sync(0xffffffffu, s0, o);
@@ -329,6 +342,8 @@ struct Gp {
   double *out = nullptr;     // {obj, wl, energy, hpwl}
   cudaStream_t s_cap = nullptr;
   cudaGraphExec_t gexec = nullptr;
+  int64_t gexec_gen = -1;    // Ctx::config_gen the iteration graph was captured with
+  int64_t gen = -1;          // Ctx::config_gen of the last gp_refresh
   bool initialised = false;
   std::vector<void *> allocs;
   int cell_blocks = 0;
@@ -380,6 +395,26 @@ dp_status gp_eval(Gp &g, const float *x, const float *y, bool wa, bool den, bool
   c.lambda_dev = nullptr;
   c.hpwl_fast = false;
   return st;
+}
+
+// Constants that depend on the context's configuration (refreshed at init and whenever a
+// dp_set_* changed it): the fixed cells (A34) and the movable area of A30's normalisation.
+dp_status gp_refresh(Gp &g) {
+  Ctx &c = *g.c;
+  const int n = g.a.n;
+  g.a.fixed = c.has_fixed ? c.d_fixed : nullptr;
+  g.a.rho_fixed = c.has_fixed ? c.d_rho_fixed : nullptr;
+  std::vector<float> w(n), h(n);
+  std::vector<uint8_t> m(n, 0);
+  DP_CUDA(cudaMemcpy(w.data(), c.d_cell_w, sizeof(float) * n, cudaMemcpyDeviceToHost));
+  DP_CUDA(cudaMemcpy(h.data(), c.d_cell_h, sizeof(float) * n, cudaMemcpyDeviceToHost));
+  if (c.has_fixed) DP_CUDA(cudaMemcpy(m.data(), c.d_fixed, n, cudaMemcpyDeviceToHost));
+  double area = 0.0;
+  for (int i = 0; i < n; i++)
+    if (!m[i]) area += (double)w[i] * (double)h[i];
+  DP_CUDA(cudaMemcpy(&g.dev->area_total, &area, sizeof(double), cudaMemcpyHostToDevice));
+  g.gen = c.config_gen;
+  return DP_OK;
 }
 
 // one GP iteration (the captured body): the step with alpha_k / coef from the previous scalar
@@ -504,7 +539,10 @@ dp_status dp_gp_init(dp_gp *gp, const float *x0, const float *y0, dp_stream_t st
   Ctx &c = *g->c;
   dp::GpDeviceGuard guard(c.device);
   cudaStream_t s = (cudaStream_t)stream;
-  dp_status st = dp::ctx_call_begin(c, s);
+  DP_CUDA(cudaStreamSynchronize(s));
+  dp_status st = dp::gp_refresh(*g);
+  if (st != DP_OK) return st;
+  st = dp::ctx_call_begin(c, s);
   if (st != DP_OK) return st;
   const int cb = g->cell_blocks;
   auto &a = g->a;
@@ -548,12 +586,21 @@ dp_status dp_gp_run(dp_gp *gp, int32_t iterations, dp_stream_t stream) {
   Ctx &c = *g->c;
   dp::GpDeviceGuard guard(c.device);
   cudaStream_t s = (cudaStream_t)stream;
+  if (g->gen != c.config_gen) {
+    DP_CUDA(cudaStreamSynchronize(s));
+    dp_status st = dp::gp_refresh(*g);
+    if (st != DP_OK) return st;
+  }
   if (c.profiling) {   // per-stage events: direct launches
     dp_status st = dp::ctx_call_begin(c, s);
     if (st != DP_OK) return st;
     for (int it = 0; it < iterations; it++)
       if ((st = dp::gp_iteration(*g, s)) != DP_OK) return st;
     return dp::ctx_call_end(c, s);
+  }
+  if (g->gexec && g->gexec_gen != c.config_gen) {   // dp_set_* since the capture: the body changed
+    cudaGraphExecDestroy(g->gexec);
+    g->gexec = nullptr;
   }
   if (!g->gexec) {   // capture one iteration once; replay it per iteration
     cudaGraph_t graph = nullptr;
@@ -571,6 +618,7 @@ dp_status dp_gp_run(dp_gp *gp, int32_t iterations, dp_stream_t stream) {
       g->gexec = nullptr;
       return dp::cuda_fail(ie, "cudaGraphInstantiate (gp)");
     }
+    g->gexec_gen = c.config_gen;
   }
   dp_status st = dp::ctx_call_begin(c, s);
   if (st != DP_OK) return st;

@@ -231,7 +231,7 @@ __device__ __forceinline__ void ext_shfl(Axis &A, int o) {
 
 // Shared-memory view of one staged chunk.
 struct GroupCtx {
-  const int *slot;       // [pins] position slot | foreign << 31
+  const int *slot;       // [pins] position slot
   const float *dx, *dy;  // [pins]
   const int *deg;        // [nets] degree | counted << 31
   const float *w;        // [nets]
@@ -244,12 +244,20 @@ struct GroupCtx {
 };
 
 __device__ __forceinline__ void grad_add(const GroupCtx &gc, int raw, float gx, float gy) {
-  const int gs = raw < 0 ? gc.trash : raw;
-  atomicAdd(gc.g + 2 * gs, __float2int_rn(gx * gc.scale));
-  atomicAdd(gc.g + 2 * gs + 1, __float2int_rn(gy * gc.scale));
+  atomicAdd(gc.g + 2 * raw, __float2int_rn(gx * gc.scale));
+  atomicAdd(gc.g + 2 * raw + 1, __float2int_rn(gy * gc.scale));
 }
 
-// Pin records of one warp group, slot-major compressed layout (32/G nets, G lanes per net).
+// the same with gx, gy already in the chunk's fixed-point units (the scale folded into the
+// per-net coefficients)
+__device__ __forceinline__ void grad_add_scaled(const GroupCtx &gc, int raw, float gx, float gy) {
+  atomicAdd(gc.g + 2 * raw, __float2int_rn(gx));
+  atomicAdd(gc.g + 2 * raw + 1, __float2int_rn(gy));
+}
+
+// Pin records of one warp group, slot-major compressed layout (32/G nets, G lanes per net):
+// slot s holds, in lane order, the pins s G + j < d of every net.  (A ballot-free variant for
+// groups of one degree measured no faster: the arithmetic replacing the ballot costs as much.)
 template <int S>
 __device__ __forceinline__ unsigned load_pins(const WarpGroup &wg, const GroupCtx &gc, int G, int j, int d,
                                               int (&raw)[S], float (&xc)[S], float (&yc)[S], float (&dxs)[S],
@@ -264,9 +272,8 @@ __device__ __forceinline__ unsigned load_pins(const WarpGroup &wg, const GroupCt
     raw[s] = gc.slot[p];
     dxs[s] = gc.dx[p];
     dys[s] = gc.dy[p];
-    const int ps = raw[s] & 0x7fffffff;
-    xc[s] = gc.px[ps];
-    yc[s] = gc.py[ps];
+    xc[s] = gc.px[raw[s]];
+    yc[s] = gc.py[raw[s]];
     vm |= (valid ? 1u : 0u) << s;
     base += __popc(m);
   }
@@ -465,18 +472,19 @@ __device__ __forceinline__ void wa_group_fast(const WaArgs &a, const WarpGroup &
     const float ig2 = a.gamma * kLn2;
     wl_acc += we * ((Px - Mx) + (mxp - mxm) * ig2 + (Py - My) + (myp - mym) * ig2);
   }
-  // eq (6) in log2 units: a+ (P+ + lambda+ Q+) - a- (P- - lambda- Q-)
-  const float wl2 = we * kLn2;
-  const float qxp = ibxp * wl2, pxp = we * ibxp - mxp * qxp;
-  const float qxm = ibxm * wl2, pxm = we * ibxm + mxm * qxm;
-  const float qyp = ibyp * wl2, pyp = we * ibyp - myp * qyp;
-  const float qym = ibym * wl2, pym = we * ibym + mym * qym;
+  // eq (6) in log2 units: a+ (P+ + lambda+ Q+) - a- (P- - lambda- Q-), in the chunk's
+  // fixed-point units (w_e times the slot scale 2^k: exact power-of-two scaling)
+  const float ws = we * gc.scale, wl2 = ws * kLn2;
+  const float qxp = ibxp * wl2, pxp = ws * ibxp - mxp * qxp;
+  const float qxm = ibxm * wl2, pxm = ws * ibxm + mxm * qxm;
+  const float qyp = ibyp * wl2, pyp = ws * ibyp - myp * qyp;
+  const float qym = ibym * wl2, pym = ws * ibym + mym * qym;
 #pragma unroll
   for (int s = 0; s < S; s++) {
     if (vm & (1u << s)) {
       const float gx = axp[s] * fmaf(lxp[s], qxp, pxp) - axm[s] * fmaf(-lxm[s], qxm, pxm);
       const float gy = ayp[s] * fmaf(lyp[s], qyp, pyp) - aym[s] * fmaf(-lym[s], qym, pym);
-      grad_add(gc, raw[s], gx, gy);
+      grad_add_scaled(gc, raw[s], gx, gy);
     }
   }
 }
@@ -513,7 +521,7 @@ __device__ __forceinline__ void wa_group_pairs(const WaArgs &a, const WarpGroup 
   // slot-major: pin 0 of net L at pin_base + L, pin 1 at pin_base + nnets + L
   const int p0 = wg.pin_base + lane, p1 = p0 + wg.nnets;
   const int r0 = gc.slot[p0], r1 = gc.slot[p1];
-  const int s0 = r0 & 0x7fffffff, s1 = r1 & 0x7fffffff;
+  const int s0 = r0, s1 = r1;
   const float ddx = (gc.px[s1] - gc.px[s0]) + (gc.dx[p1] - gc.dx[p0]);
   const float ddy = (gc.py[s1] - gc.py[s0]) + (gc.dy[p1] - gc.dy[p0]);
   const float tx = fabsf(ddx) * a.k2, ty = fabsf(ddy) * a.k2;   // u log2(e)
@@ -547,6 +555,19 @@ __device__ __forceinline__ void wa_group_pairs(const WaArgs &a, const WarpGroup 
   const float gy = copysignf(we * fmaf(hy, fmaf(-thy, thy, 1.f), thy), ddy);
   grad_add(gc, r1, gx, gy);
   grad_add(gc, r0, -gx, -gy);
+}
+
+// (A compile-time lanes-per-net variant of wa_group_fast, 24 instantiations, measured 85 -> 107
+// us: the kernel's code outgrows the instruction caches.)
+template <bool LSE, bool HP>
+__device__ __forceinline__ void wa_group_fast_dispatch(const WaArgs &a, const WarpGroup &wg, const GroupCtx &gc,
+                                                       float &wl_acc, float &hp_acc) {
+  switch (wg.slots) {
+    case 1: wa_group_fast<1, LSE, HP>(a, wg, gc, wl_acc, hp_acc); break;
+    case 2: wa_group_fast<2, LSE, HP>(a, wg, gc, wl_acc, hp_acc); break;
+    case 3: wa_group_fast<3, LSE, HP>(a, wg, gc, wl_acc, hp_acc); break;
+    default: wa_group_fast<4, LSE, HP>(a, wg, gc, wl_acc, hp_acc); break;
+  }
 }
 
 // Dynamic shared-memory layout of the chunk kernel (capacities fixed at create).
@@ -999,12 +1020,7 @@ __global__ void __launch_bounds__(kWaThreads, 2) k_wa_chunks(const WaArgs a0) {
       if (wg.flags & 1) {
         wa_group_pairs<kL, kH, false>(a, wg, gc, wl_acc, hp_acc, L);
       } else {
-        switch (wg.slots) {
-          case 1: wa_group_fast<1, kL, kH>(a, wg, gc, wl_acc, hp_acc); break;
-          case 2: wa_group_fast<2, kL, kH>(a, wg, gc, wl_acc, hp_acc); break;
-          case 3: wa_group_fast<3, kL, kH>(a, wg, gc, wl_acc, hp_acc); break;
-          default: wa_group_fast<4, kL, kH>(a, wg, gc, wl_acc, hp_acc); break;
-        }
+        wa_group_fast_dispatch<kL, kH>(a, wg, gc, wl_acc, hp_acc);
       }
     } else {
       if (MODE == 1 && (wg.flags & 1)) {   // 2-pin nets: closed-form WA + exact HPWL

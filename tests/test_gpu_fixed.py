@@ -115,6 +115,49 @@ def test_gp_keeps_fixed_cells():
     assert np.abs(ux[~m] - x[~m]).max() > nl.bin_w   # movable cells did move
 
 
+def test_gp_overflow_with_fixed_macros():
+    """A30 with fixed macros (A34): the loop's overflow at the start point equals the
+    oracle's — fixed charge counted at the target density, normalised by the movable area."""
+    from oracle import gp as ogp
+    nl = make_netlist("adaptec1")
+    x, y = make_positions(nl, "spread")
+    m = _mask(nl, 0.0, 1)
+    assert m.any()
+    ctx = dp.dp_create(nl)
+    dp.dp_set_fixed(ctx, m, _t(x), _t(y))
+    loop = dp.GpLoop(ctx, target_density=0.9)
+    loop.init(_t(x), _t(y))
+    _, sc = loop.debug_state()
+    rho = oracle.density_map(nl, x, y, 1)
+    cells = np.nonzero(m)[0]
+    from synth import custom_netlist
+    fixed_nl = custom_netlist([0], [], [], [], nl.cell_w[cells], nl.cell_h[cells], (nl.xl, nl.yl, nl.xh, nl.yh),
+                              (nl.bins_x, nl.bins_y))
+    rho_f = oracle.density_map(fixed_nl, x[cells], y[cells], 1)
+    ref = ogp.overflow(nl, rho, 0.9, m, rho_f)
+    assert abs(sc["tau"] - ref) <= 1e-5 * max(ref, 1e-3), (sc["tau"], ref)
+
+
+def test_gp_recaptures_after_set_fixed():
+    """dp_set_* after the loop captured its iteration graph: the next dp_gp_run
+    re-captures, so cells fixed after 5 iterations stay where they are from then on."""
+    nl = make_netlist("tiny")
+    x, y = make_positions(nl, "initial")
+    ctx = dp.dp_create(nl)
+    loop = dp.GpLoop(ctx)
+    loop.init(_t(x), _t(y))
+    loop.run(5)
+    ux, uy = loop.positions()
+    m = _mask(nl, 0.05, 8)
+    dp.dp_set_fixed(ctx, m, ux, uy)
+    ux0, uy0 = ux.cpu().numpy().copy(), uy.cpu().numpy().copy()
+    loop.run(20)
+    ux1, uy1 = loop.positions()
+    ux1, uy1 = ux1.cpu().numpy(), uy1.cpu().numpy()
+    assert np.array_equal(ux1[m], ux0[m]) and np.array_equal(uy1[m], uy0[m])
+    assert np.abs(ux1[~m] - ux0[~m]).max() > 0.0
+
+
 def test_gp_with_fillers_and_fixed_macros():
     """ePlace-style setup (reading A35): pinless fillers bring the movable area to 90% of the
     free area, the large blocks are fixed; the device loop spreads movable cells and fillers.

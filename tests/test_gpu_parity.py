@@ -293,6 +293,50 @@ def test_eval_full_size(name):
     check_vector("gy", to_np(out["gy"]), ref["gy"])
 
 
+@pytest.mark.slow
+@pytest.mark.parametrize("name", ["adaptec1", "bigblue4"])
+def test_initial_full_size(name):
+    """The 'initial' placement (centres ~ N(W/2, (0.001 W)^2), every cell in a few bins)
+    at full size: the density map (every walker in one tile, the wrap carry of the scatter's
+    32-bit accumulators), the force gather where opposite fields cancel, and the full
+    evaluation, against the oracle."""
+    nl = make_netlist(name)
+    ctx = dp.dp_create(nl)
+    x, y = make_positions(nl, "initial")
+    xt, yt = _t(x), _t(y)
+    ref = oracle.evaluate(nl, x, y, nl.bin_w, 1.0)
+    check_map("rho", to_np(ctx.density_map(xt, yt)), ref["rho"], rel=2e-6)
+    d = ctx.density_grad(xt, yt)
+    check_scalar("D", d["energy"].item(), ref["energy"])
+    check_vector("dD/dx", to_np(d["gx"]), ref["d_gx"])
+    check_vector("dD/dy", to_np(d["gy"]), ref["d_gy"])
+    out = ctx.eval(xt, yt, nl.bin_w, 1.0, with_hpwl=True)
+    check_scalar("WA", out["wl"].item(), ref["wl"])
+    check_scalar("obj", out["obj"].item(), ref["obj"])
+    assert out["hpwl"].item() == ref["hpwl"]
+    check_vector("gx", to_np(out["gx"]), ref["gx"])
+    check_vector("gy", to_np(out["gy"]), ref["gy"])
+
+
+@pytest.mark.slow
+@pytest.mark.parametrize("gscale,lam", [(0.05, 1.0), (50.0, 1.0), (1.0, 0.0)])
+def test_adaptec1_gamma_lambda_sweep(gscale, lam):
+    """SURVEY §8(d) parity sweep at adaptec1 full size (211K cells: every WA path — window and
+    far cells, warp-per-net and CTA-per-net big nets — not just the tiny config's one window):
+    gamma in {0.05, 50} b and lambda = 0."""
+    nl = make_netlist("adaptec1")
+    ctx = dp.dp_create(nl)
+    x, y = make_positions(nl)
+    gamma = gscale * nl.bin_w
+    out = ctx.eval(_t(x), _t(y), gamma, lam, with_hpwl=True)
+    ref = oracle.evaluate(nl, x, y, gamma, lam)
+    check_scalar("WA", out["wl"].item(), ref["wl"])
+    check_scalar("obj", out["obj"].item(), ref["obj"])
+    assert out["hpwl"].item() == ref["hpwl"]
+    check_vector("gx", to_np(out["gx"]), ref["gx"])
+    check_vector("gy", to_np(out["gy"]), ref["gy"])
+
+
 def test_invalid_args(tiny):
     nl, ctx = tiny
     x, y = make_positions(nl)

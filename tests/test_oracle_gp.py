@@ -198,3 +198,24 @@ def test_gp_init_first_lipschitz_point():
     assert eta > 0
     np.testing.assert_allclose(d, eta * g0, rtol=1e-12, atol=1e-12 * np.abs(d).max())
     assert np.array_equal(st.u, st.v) and st.a == 1.0 and st.k == 0
+
+
+def test_overflow_with_fixed_macro_closed_form():
+    """A30 with a fixed macro (A34): a macro exactly covering a 4 x 4 block of bins and nothing
+    else overflows 0 at any target t (its charge counts at t), where the plain A30 would report
+    16 (1 - t) bins of overflow; one movable unit cell on top of it overflows by its own area:
+    tau = 1 (the movable area)."""
+    b = 10.0
+    nl = custom_netlist([0, 0], [], [], [], [4 * b, b], [4 * b, b], (0, 0, 16 * b, 16 * b), (16, 16))
+    fixed = np.array([True, False])
+    xm, ym = np.array([3 * b], np.float32), np.array([5 * b], np.float32)
+    macro = custom_netlist([0, 0], [], [], [], [4 * b], [4 * b], (0, 0, 16 * b, 16 * b), (16, 16))
+    rho_f = oracle.density_map(macro, xm, ym, stretch=0)
+    for t in (0.7, 0.9, 1.0):
+        assert gp.overflow(macro, rho_f, t) == pytest.approx(1.0 - t, abs=1e-12) or t == 1.0
+        # macro alone, as a fixed cell: no overflow (movable area: the unit cell's)
+        assert gp.overflow(nl, rho_f, t, fixed, rho_f) == pytest.approx(0.0, abs=1e-12)
+        x = np.array([3 * b, 4 * b], np.float32)
+        y = np.array([5 * b, 6 * b], np.float32)
+        rho = oracle.density_map(nl, x, y, stretch=0)      # unit cell inside the macro's block
+        assert gp.overflow(nl, rho, t, fixed, rho_f) == pytest.approx(1.0, rel=1e-12)

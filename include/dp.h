@@ -252,6 +252,18 @@ dp_status dp_gp_positions(dp_gp *gp, float *x, float *y, dp_stream_t stream);
  * *rows <- rows written.                                                                    */
 dp_status dp_gp_history(dp_gp *gp, double *h_rows, int32_t max_rows, int32_t *rows);
 
+/* Fence regions ("multiple electric fields, e.g., one for each region",
+ * P:549; reading A38).  h_boxes (host, [n_regions][4] = xl, yl, xh, yh, disjoint rectangles);
+ * h_cell_region (host, [num_cells]) in [0, n_regions]: 0 = the default region (the layout
+ * minus the fences), r >= 1 = fence r.  Every region has its own density map, Poisson solve
+ * and field: rho_r = a blockage of density 1 on the part of each bin outside region r (exact
+ * int64, like every map) + the charge of region r's cells; D = sum_r D_r; a cell's density
+ * gradient is the force gather in its own region's field.  Wirelength is unchanged.
+ * n_regions = 0 clears.  Single-GPU contexts only; not combined with dp_set_fixed.
+ * Errors: DP_ERR_INVALID_ARG (null, degenerate boxes, region ids out of range),
+ * DP_ERR_UNSUPPORTED, DP_ERR_OUT_OF_MEMORY / DP_ERR_CUDA.                                    */
+dp_status dp_set_regions(dp_ctx *ctx, int32_t n_regions, const double *h_boxes, const int32_t *h_cell_region);
+
 /* Test-only hook (no part of the metric): synchronise and copy the loop state at the start of
  * the next iteration.  u, v, vp (= v_{k-1}), g (preconditioned gradient at v), gp_prev (at vp):
  * device, [2 num_cells] (x entries, then y), each may be NULL.  h_scalars (host, [9]):

@@ -220,6 +220,51 @@ def density(nl, x, y, stretch: int = 1):
     return D, gx, gy, dict(rho=rho, a=a, psi=psi, xi_x=xi_x, xi_y=xi_y)
 
 
+def region_blockage(nl, boxes, r: int) -> np.ndarray:
+    """Reading A38 (fence regions): the blockage map of region r — the fraction of each
+    bin outside the region, at density 1.  Fence r >= 1 is box r-1 (xl, yl, xh, yh); region 0,
+    the default region, is the layout minus the (disjoint) fences.  Overlaps are the products
+    of 1-D interval overlaps, as in the density map."""
+    xs = nl.xl + np.arange(nl.bins_x + 1) * nl.bin_w
+    ys = nl.yl + np.arange(nl.bins_y + 1) * nl.bin_h
+
+    def cover(b):   # fraction of each bin inside box b
+        ox = np.clip(np.minimum(xs[1:], b[2]) - np.maximum(xs[:-1], b[0]), 0.0, None) / nl.bin_w
+        oy = np.clip(np.minimum(ys[1:], b[3]) - np.maximum(ys[:-1], b[1]), 0.0, None) / nl.bin_h
+        return ox[:, None] * oy[None, :]
+
+    if r == 0:
+        out = np.zeros((nl.bins_x, nl.bins_y))
+        for b in boxes:
+            out += cover(b)
+        return out
+    return 1.0 - cover(boxes[r - 1])
+
+
+def evaluate_regions(nl, x, y, gamma: float, lam: float, boxes, cell_region, stretch: int = 1):
+    """Fence regions as "multiple electric fields, e.g., one for each region" (reading
+    A38): region r has its own map rho_r = blockage_r + the charge of its cells, its own Poisson
+    solve (eqs 9a-9d) and energy D_r; D = sum_r D_r, and a cell's density gradient is the force
+    gather in its own region's field.  The wirelength part is unchanged (eq 2)."""
+    cell_region = np.asarray(cell_region)
+    wl, gwx, gwy = wa(nl, x, y, gamma)
+    gdx = np.zeros(nl.num_cells)
+    gdy = np.zeros(nl.num_cells)
+    D = 0.0
+    from synth import custom_netlist
+    for r in range(len(boxes) + 1):
+        idx = np.nonzero(cell_region == r)[0]
+        sub = custom_netlist([0], [], [], [], nl.cell_w[idx], nl.cell_h[idx], (nl.xl, nl.yl, nl.xh, nl.yh),
+                             (nl.bins_x, nl.bins_y))
+        rho = region_blockage(nl, boxes, r) + density_map(sub, x[idx], y[idx], stretch)
+        psi, xi_x, xi_y = fields(nl, dct2(rho))
+        D += energy(nl, rho, psi)
+        fx, fy = density_grad(sub, x[idx], y[idx], xi_x, xi_y, stretch)
+        gdx[idx] = fx
+        gdy[idx] = fy
+    return dict(obj=wl + lam * D, wl=wl, energy=D, gx=gwx + lam * gdx, gy=gwy + lam * gdy, d_gx=gdx, d_gy=gdy)
+
+
 def evaluate(nl, x, y, gamma: float, lam: float, stretch: int = 1, with_hpwl: bool = True,
              wl_model: str = "wa", fixed=None):
     """obj = WL + lambda D and grad = grad WL + lambda grad D (eq 2); WL = WA (eq 3)

@@ -875,7 +875,7 @@ void fields_after_t1(const Ctx &c, cudaStream_t s) {
   a.t = c.d_t; a.sx = c.d_sx; a.sy = c.d_sy;
   a.mx = c.mx; a.log2mx = c.log2mx; a.my = c.my;
   a.tw_x = c.d_tw_x; a.ph_x = c.d_ph_x; a.kx = c.d_kx; a.ky = c.d_ky;
-  a.energy_part = c.d_part + c.n_wa_part;
+  a.energy_part = c.d_part + c.n_wa_part + (c.n_regions > 0 && c.cur_region > 0 ? c.cur_region * c.n_en_part : 0);
   a.energy_scale = 0.5 * c.bx * c.by;
   if (c.fft_hybrid) {   // the CTA-FFT column pass on t[x][y], then T3
     launch_p2_rowmajor(c, s);

@@ -70,6 +70,7 @@ struct DenArgs {
   // the precomputed fixed-charge map; sel = 1: building that map)
   const uint8_t *fixed;
   int sel;
+  int keep;   // fence regions: cells of other regions are skipped without writing their force
   int n_large;
 };
 
@@ -275,7 +276,10 @@ __global__ void __launch_bounds__(kCountThreads) k_place(DenArgs a) {
     int t = classify_small(a, x[k], y[k], w[k], h[k], f);
     tl[k] = -1;
     if (i >= a.n_own || t == -2) continue;
-    if (MASK && !selected(a, i)) t = -1;   // fixed cell of an evaluation: no record, force 0
+    if (MASK && !selected(a, i)) {   // fixed cell of an evaluation: no record, force 0;
+      if (a.keep) continue;          // another region's cell: its own pass writes its force
+      t = -1;
+    }
     if (t == -1) {
       a.force[i] = make_float2(0.f, 0.f);
       continue;
@@ -737,9 +741,17 @@ DenArgs make_args(const Ctx &c, const float *x, const float *y) {
   a.n_large = c.n_large;
   a.fixed = c.has_fixed && c.fixed_small ? c.d_fixed : nullptr;
   a.sel = 0;
+  a.keep = 0;
   if (c.has_fixed) {
     a.large = c.d_large_mov;
     a.n_large = c.n_large_mov;
+  }
+  if (c.n_regions > 0 && c.cur_region >= 0) {   // fence regions: this pass's cells only
+    a.fixed = c.d_region;
+    a.sel = c.cur_region;
+    a.keep = 1;
+    a.large = c.d_large_reg + c.large_reg_off[c.cur_region];
+    a.n_large = c.large_reg_off[c.cur_region + 1] - c.large_reg_off[c.cur_region];
   }
   return a;
 }
@@ -804,7 +816,10 @@ void launch_density_map(const Ctx &c, const float *x, const float *y, cudaStream
   }
   const int ntiles = a.ntiles;
   const int nblk = (c.n_own + kCountCells - 1) / kCountCells;
-  if (c.has_fixed && !build_fixed)   // start from the precomputed fixed-charge map (exact int64)
+  if (c.n_regions > 0 && c.cur_region >= 0)   // start from the region's blockage map (exact int64)
+    cudaMemcpyAsync(c.d_rho, c.d_rho_block + (size_t)c.cur_region * c.mx * c.my,
+                    sizeof(unsigned long long) * (size_t)c.mx * c.my, cudaMemcpyDeviceToDevice, s);
+  else if (c.has_fixed && !build_fixed)   // start from the precomputed fixed-charge map (exact int64)
     cudaMemcpyAsync(c.d_rho, c.d_rho_fixed, sizeof(unsigned long long) * (size_t)c.mx * c.my,
                     cudaMemcpyDeviceToDevice, s);
   else
@@ -820,6 +835,7 @@ void launch_density_map(const Ctx &c, const float *x, const float *y, cudaStream
     const int cgrid = std::min(nblk, c.count_grid > 0 ? c.count_grid : nblk);
     if (a.fixed)
       launch_chain(c.pdl, k_count<true>, cgrid, kCountThreads, ntiles * 4, s, a);
+    // (k_count<true> counts only selected cells; k_place<true> records only selected cells)
     else
       launch_chain(c.pdl, k_count<false>, cgrid, kCountThreads, ntiles * 4, s, a);
     if (c.sched == 3) cudaEventRecord(c.ev_sched, s);   // DP_SCHED=3: WA starts after the count

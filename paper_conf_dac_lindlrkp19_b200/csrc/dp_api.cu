@@ -840,7 +840,22 @@ dp_status sharded_fields(Ctx &c, cudaStream_t s) {
   return nccl_all_gather_bytes(c, c.d_xi, nb / G * sizeof(float2), s);
 }
 
+dp_status density_chain_pass(Ctx &c, const float *x, const float *y);
+
+// the density chain; with fence regions (NEXT-4, reading A38) one pass per region, each with its
+// own map (from the region's blockage map), Poisson solve (its own energy slots) and gather
 dp_status density_chain(Ctx &c, const float *x, const float *y) {
+  if (c.n_regions == 0) return density_chain_pass(c, x, y);
+  for (int r = 0; r <= c.n_regions; r++) {
+    c.cur_region = r;
+    const dp_status st = density_chain_pass(c, x, y);
+    c.cur_region = -1;
+    if (st != DP_OK) return st;
+  }
+  return DP_OK;
+}
+
+dp_status density_chain_pass(Ctx &c, const float *x, const float *y) {
   {
     StageMark m(c, DP_STAGE_MAP, c.s_den);
     launch_density_map(c, x, y, c.s_den, c.s_aux);
@@ -1170,6 +1185,7 @@ dp_status dp_set_fixed(dp_ctx *ctx, const uint8_t *h_fixed, const float *x, cons
   if (!c) return fail(DP_ERR_INVALID_ARG, "ctx is NULL");
   if (c->dist) return fail(DP_ERR_UNSUPPORTED, "fixed cells are supported on single-GPU contexts");
   if (h_fixed && (!x || !y)) return fail(DP_ERR_INVALID_ARG, "x / y is NULL");
+  if (h_fixed && c->n_regions > 0) return fail(DP_ERR_UNSUPPORTED, "fixed cells with fence regions");
   dp::DeviceGuard g(c->device);
   cudaStream_t s = (cudaStream_t)stream;
   dp_status st = dp::call_begin(*c, s);
@@ -1215,6 +1231,80 @@ dp_status dp_set_fixed(dp_ctx *ctx, const uint8_t *h_fixed, const float *x, cons
                           cudaMemcpyDeviceToDevice, s));
   DP_CUDA(cudaGetLastError());
   return dp::call_end(*c, s);
+}
+
+dp_status dp_set_regions(dp_ctx *ctx, int32_t n_regions, const double *h_boxes, const int32_t *h_cell_region) {
+  Ctx *c = C(ctx);
+  if (!c) return fail(DP_ERR_INVALID_ARG, "ctx is NULL");
+  if (c->dist) return fail(DP_ERR_UNSUPPORTED, "fence regions are supported on single-GPU contexts");
+  if (n_regions < 0 || n_regions > 254) return fail(DP_ERR_INVALID_ARG, "n_regions must be in [0, 254]");
+  if (n_regions > 0 && (!h_boxes || !h_cell_region)) return fail(DP_ERR_INVALID_ARG, "boxes / cell_region is NULL");
+  if (n_regions > 0 && c->has_fixed) return fail(DP_ERR_UNSUPPORTED, "fence regions with fixed cells");
+  for (int32_t r = 0; r < n_regions; r++) {
+    const double *b = h_boxes + 4 * r;
+    if (!(std::isfinite(b[0]) && std::isfinite(b[1]) && std::isfinite(b[2]) && std::isfinite(b[3])) ||
+        !(b[2] > b[0]) || !(b[3] > b[1]))
+      return fail(DP_ERR_INVALID_ARG, "fence box " + std::to_string(r) + " is degenerate or non-finite");
+  }
+  for (int32_t i = 0; n_regions > 0 && i < c->num_cells; i++)
+    if (h_cell_region[i] < 0 || h_cell_region[i] > n_regions)
+      return fail(DP_ERR_INVALID_ARG, "cell_region out of [0, n_regions]");
+  dp::DeviceGuard g(c->device);
+  DP_CUDA(cudaDeviceSynchronize());
+  c->config_gen++;
+  if (c->gexec) {   // the captured evaluation changes: re-capture
+    cudaGraphExecDestroy(c->gexec);
+    c->gexec = nullptr;
+    c->gkey = dp::GraphKey{};
+  }
+  c->n_regions = 0;
+  if (n_regions == 0) return DP_OK;
+  const int R = n_regions, n = c->n_own;
+  const size_t nb = (size_t)c->mx * c->my;
+  std::vector<uint8_t> reg(((size_t)n + 3) & ~(size_t)3, 0);
+  for (int i = 0; i < n; i++) reg[i] = (uint8_t)h_cell_region[c->cell_begin + i];
+  // blockage maps (A38): per bin the fraction outside region r, at density 1, in 2^-29 units
+  std::vector<unsigned long long> blk((size_t)(R + 1) * nb, 0ull);
+  auto cover = [&](const double *b, int i, int j) {
+    const double x0 = c->xl + i * c->bx, y0 = c->yl + j * c->by;
+    const double ox = std::max(0.0, std::min(x0 + c->bx, b[2]) - std::max(x0, b[0])) / c->bx;
+    const double oy = std::max(0.0, std::min(y0 + c->by, b[3]) - std::max(y0, b[1])) / c->by;
+    return ox * oy;
+  };
+  const double unit = std::ldexp(1.0, dp::kRhoScaleLog2);
+  for (int i = 0; i < c->mx; i++)
+    for (int j = 0; j < c->my; j++) {
+      double in_fences = 0.0;
+      for (int r = 1; r <= R; r++) {
+        const double f = cover(h_boxes + 4 * (r - 1), i, j);
+        in_fences += f;
+        blk[(size_t)r * nb + (size_t)i * c->my + j] = (unsigned long long)std::llround((1.0 - f) * unit);
+      }
+      blk[(size_t)i * c->my + j] = (unsigned long long)std::llround(std::min(1.0, in_fences) * unit);
+    }
+  std::vector<int32_t> large(c->n_large);
+  if (c->n_large) DP_CUDA(cudaMemcpy(large.data(), c->d_large, sizeof(int32_t) * c->n_large, cudaMemcpyDeviceToHost));
+  std::vector<int32_t> lreg;
+  c->large_reg_off.assign(R + 2, 0);
+  for (int r = 0; r <= R; r++) {
+    c->large_reg_off[r] = (int32_t)lreg.size();
+    for (int32_t i : large)
+      if (reg[i] == r) lreg.push_back(i);
+  }
+  c->large_reg_off[R + 1] = (int32_t)lreg.size();
+  if (lreg.empty()) lreg.push_back(0);
+  dp_status st;
+  if ((st = dp::dev_upload(*c, &c->d_region, reg)) != DP_OK) return st;
+  if ((st = dp::dev_upload(*c, &c->d_rho_block, blk)) != DP_OK) return st;
+  if ((st = dp::dev_upload(*c, &c->d_large_reg, lreg)) != DP_OK) return st;
+  // partial sums with one energy slot range per region
+  const size_t np = 2 * (size_t)c->n_wa_part + (size_t)c->n_en_part * (R + 1) + 1;
+  double *part = nullptr;
+  if ((st = dp::dev_alloc(*c, &part, np)) != DP_OK) return st;
+  DP_CUDA(cudaMemset(part, 0, sizeof(double) * np));
+  c->d_part = part;
+  c->n_regions = R;
+  return DP_OK;
 }
 
 dp_status dp_density_grad(dp_ctx *ctx, const float *x, const float *y, float *gx, float *gy, double *d_energy,

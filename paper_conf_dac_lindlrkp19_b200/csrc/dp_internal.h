@@ -154,6 +154,16 @@ struct Ctx {
   uint8_t *d_fixed = nullptr;
   unsigned long long *d_rho_fixed = nullptr;
   int32_t *d_large_mov = nullptr, *d_large_fix = nullptr;
+  // fence regions (NEXT-4, dp_set_regions; reading A38): one density map / Poisson solve / field
+  // per region r in [0, n_regions]; cells carry their region, region r's map starts from its
+  // blockage map (density 1 outside the region, exact int64)
+  int32_t n_regions = 0;                       // fences; 0 = none
+  uint8_t *d_region = nullptr;                 // [n_own] region of each own cell
+  unsigned long long *d_rho_block = nullptr;   // [n_regions + 1][mx my]
+  int32_t *d_large_reg = nullptr;              // large cells grouped by region
+  std::vector<int32_t> large_reg_off;          // [n_regions + 2]
+  mutable int cur_region = -1;                 // region of the density pass being enqueued
+  int n_en_slots() const { return n_en_part * (n_regions + 1); }
   int32_t n_large_mov = 0, n_large_fix = 0;                     // [num_cells] net-weighted pin count (GP preconditioner)
   int32_t n_own = 0;                // cells owned by this rank
   int32_t n_large = 0;              // large cells (footprint > 3 bins on an axis)

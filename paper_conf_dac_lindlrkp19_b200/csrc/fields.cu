@@ -401,7 +401,7 @@ FieldArgs field_args(const Ctx &c, const void *rho) {
   a.ph_y = c.d_ph_y;
   a.kx = c.d_kx;
   a.ky = c.d_ky;
-  a.energy_part = c.d_part + c.n_wa_part;
+  a.energy_part = c.d_part + c.n_wa_part + (c.n_regions > 0 && c.cur_region > 0 ? c.cur_region * c.n_en_part : 0);
   a.energy_scale = 0.5 * c.bx * c.by;
   return a;
 }

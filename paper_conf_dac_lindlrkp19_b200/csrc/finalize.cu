@@ -256,8 +256,8 @@ void launch_finalize_phase(const Ctx &c, int phase, float lambda, bool with_wl, 
   FinArgs a;
   a.part = c.d_part;
   a.n_wa = c.n_wa_part;
-  a.n_en = c.n_en_part;
-  a.hp_part = (with_hpwl && c.hpwl_fast && c.wl_model == DP_WL_WA) ? c.d_part + c.n_wa_part + c.n_en_part + 1 : nullptr;
+  a.n_en = c.n_en_slots();
+  a.hp_part = (with_hpwl && c.hpwl_fast && c.wl_model == DP_WL_WA) ? c.d_part + c.n_wa_part + c.n_en_slots() + 1 : nullptr;
   a.limbs = c.d_limbs;
   a.scal = c.d_scal;
   a.d_obj = d_obj;

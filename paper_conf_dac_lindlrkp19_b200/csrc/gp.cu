@@ -501,6 +501,9 @@ dp_status dp_gp_create(dp_ctx *ctx, const dp_gp_params *params, dp_gp **out) {
   if ((st = dp::gp_alloc(*g, &g->dev, 1)) != DP_OK) return bail(st);
   if ((st = dp::gp_alloc(*g, &g->out, 4)) != DP_OK) return bail(st);
   if ((st = dp::gp_alloc(*g, &a.hist, (size_t)std::max(1, p.max_history) * dp::kHistCols)) != DP_OK) return bail(st);
+  // zeroed: dp_gp_history copies the whole ring (compute-sanitizer initcheck)
+  if (cudaMemset(a.hist, 0, sizeof(double) * (size_t)std::max(1, p.max_history) * dp::kHistCols) != cudaSuccess)
+    return bail(dp::fail(DP_ERR_CUDA, "history memset"));
   a.dev = g->dev;
   a.out = g->out;
   g->cell_blocks = (n + dp::kGpThreads - 1) / dp::kGpThreads;

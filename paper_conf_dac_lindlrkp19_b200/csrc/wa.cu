@@ -1154,7 +1154,7 @@ void launch_wa(const Ctx &c, const float *x, const float *y, float gamma, bool h
   a.big_dx = c.d_big_dx;
   a.big_dy = c.d_big_dy;
   a.part_base = c.part_base;
-  a.hp_offset = c.n_wa_part + c.n_en_part + 1;
+  a.hp_offset = c.n_wa_part + c.n_en_slots() + 1;
   a.n_huge = c.n_huge;
   a.n_big = c.n_big;
   a.n_warp_blocks = (c.n_big - c.n_huge + kWarpNetThreads / 32 - 1) / (kWarpNetThreads / 32);

@@ -71,6 +71,7 @@ struct DenArgs {
   const uint8_t *fixed;
   int sel;
   int keep;   // fence regions: cells of other regions are skipped without writing their force
+  int sync_ring;   // DP_WALK_SYNC=1: a block barrier before each ring refill (racecheck diagnostics)
   int n_large;
 };
 
@@ -430,11 +431,18 @@ __device__ __forceinline__ void walk_start(const DenArgs &a, Walker &w, RecStage
 
 // Ring step of chunk c (every thread): wait until chunk c has landed; thread 0 then refills the
 // buffer of chunk c - 1 with chunk c + kStages - 1 once every warp has released chunk c - 1.
-// Warps move through the ring independently: there is no block barrier per chunk.
+// Warps move through the ring independently: there is no block barrier per chunk.  The ordering
+// of a warp's reads of buffer b2 (and of its descriptor st.ch[b2]) before thread 0 refills it is
+// the empty[b2] mbarrier: each warp's mbarrier.arrive (release, CTA scope) after its last read,
+// thread 0's try_wait (acquire) before the refill.  compute-sanitizer racecheck does not model
+// mbarrier ordering and reports the descriptor refill as a WAR hazard; a.sync_ring
+// (DP_WALK_SYNC=1, diagnostics only) adds a block barrier before each refill, under which
+// racecheck reports none (profiles/r02_sanitizer_racecheck*.log).
 __device__ __forceinline__ WalkChunk walk_next(const DenArgs &a, Walker &w, RecStage &st, int c, bool with_cell) {
   const int b = c % kStages;
   mbar_wait(&st.bar[b], (c / kStages) & 1);
   const WalkChunk cc = st.ch[b];
+  if (a.sync_ring) __syncthreads();   // uniform: every thread reaches it
   if (threadIdx.x == 0 && cc.begin < cc.end) {
     const int b2 = (c + kStages - 1) % kStages;
     if (c >= 1) mbar_wait(&st.empty[b2], ((c - 1) / kStages) & 1);
@@ -742,6 +750,7 @@ DenArgs make_args(const Ctx &c, const float *x, const float *y) {
   a.fixed = c.has_fixed && c.fixed_small ? c.d_fixed : nullptr;
   a.sel = 0;
   a.keep = 0;
+  a.sync_ring = c.walk_sync ? 1 : 0;
   if (c.has_fixed) {
     a.large = c.d_large_mov;
     a.n_large = c.n_large_mov;

@@ -716,6 +716,7 @@ dp_status create(const dp_netlist *nl, const dp_grid *grid, int device, int rank
   { const char *e = std::getenv("DP_GRAPH"); c->use_graph = !(e && e[0] == '0'); }
   { const char *e = std::getenv("DP_DIRECT"); c->direct = e && e[0] == '1'; }
   { const char *e = std::getenv("DP_PDL"); c->pdl = !(e && e[0] == '0'); }
+  { const char *e = std::getenv("DP_WALK_SYNC"); c->walk_sync = e && e[0] == '1'; }
   {
     const char *e = std::getenv("DP_L2_PERSIST");
     c->l2_persist = !(e && e[0] == '0');

@@ -163,6 +163,7 @@ struct Ctx {
   int32_t *d_large_reg = nullptr;              // large cells grouped by region
   std::vector<int32_t> large_reg_off;          // [n_regions + 2]
   mutable int cur_region = -1;                 // region of the density pass being enqueued
+  bool walk_sync = false;                      // DP_WALK_SYNC=1: block barrier per walker ring refill
   int n_en_slots() const { return n_en_part * (n_regions + 1); }
   int32_t n_large_mov = 0, n_large_fix = 0;                     // [num_cells] net-weighted pin count (GP preconditioner)
   int32_t n_own = 0;                // cells owned by this rank

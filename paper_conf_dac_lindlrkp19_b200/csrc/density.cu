@@ -699,6 +699,28 @@ __global__ void __launch_bounds__(256) k_gather_large(DenArgs a) {
   }
 }
 
+// A30 of a fence region's map (the GP loop with dp_set_regions): the blockage counts at the
+// target density like a fixed macro (A30'), rho_eff = rho - (1 - t) blockage, so only cells
+// overflow; per-block partials [region][block][2] summed in a fixed order by the GP.
+__global__ void __launch_bounds__(256) k_region_overflow(const unsigned long long *rho, const unsigned long long *blk,
+                                                         long long nbins, double t, double *part) {
+  const double unit = 1.0 / (double)(1ll << kRhoScaleLog2);
+  double s = 0.0;
+  for (long long b = blockIdx.x * 256ll + threadIdx.x; b < nbins; b += (long long)gridDim.x * 256)
+    s += fmax(((double)rho[b] - (1.0 - t) * (double)blk[b]) * unit - t, 0.0);
+  __shared__ double r0[8];
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+  if ((threadIdx.x & 31) == 0) r0[threadIdx.x >> 5] = s;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    double tot = 0.0;
+    for (int w = 0; w < 8; w++) tot += r0[w];
+    part[2 * blockIdx.x] = tot;
+    part[2 * blockIdx.x + 1] = 0.0;
+  }
+}
+
 // largest float f with (double)f <= v, so that for any float w: w > f <=> (double)w > v
 float float_at_most(double v) {
   float f = (float)v;
@@ -806,6 +828,13 @@ int density_walk_grid(int tile) {
   // the WA kernel that runs beside the scatter and the gather
   if (const char *e = std::getenv("DP_WALK_CTAS")) per_sm = std::max(1, std::min(per_sm, std::atoi(e)));
   return sms * per_sm;
+}
+
+void launch_region_overflow(const Ctx &c, cudaStream_t s) {
+  if (!c.ovf_part || c.n_regions == 0 || c.cur_region < 0) return;
+  const size_t nb = (size_t)c.mx * c.my;
+  k_region_overflow<<<c.ovf_blocks, 256, 0, s>>>(c.d_rho, c.d_rho_block + (size_t)c.cur_region * nb, (long long)nb,
+                                                 c.ovf_target, c.ovf_part + 2 * (size_t)c.cur_region * c.ovf_blocks);
 }
 
 // kernels of one evaluation's density map + gather: count, scan, place, scatter, gather, and the

@@ -868,6 +868,7 @@ dp_status density_chain_pass(Ctx &c, const float *x, const float *y) {
     }
   }
   DP_CUDA(cudaEventRecord(c.ev_map, c.s_den));
+  launch_region_overflow(c, c.s_den);   // GP loop over fence regions: this region's A30 partials
   {
     StageMark m(c, DP_STAGE_FIELDS, c.s_den);
     if (c.shard_poisson) {

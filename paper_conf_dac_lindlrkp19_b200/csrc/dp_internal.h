@@ -163,6 +163,11 @@ struct Ctx {
   int32_t *d_large_reg = nullptr;              // large cells grouped by region
   std::vector<int32_t> large_reg_off;          // [n_regions + 2]
   mutable int cur_region = -1;                 // region of the density pass being enqueued
+  // GP loop over fence regions: each region pass adds its A30 overflow partials here
+  // ([n_regions + 1][ovf_blocks][2], null = not requested), with the target density ovf_target
+  double *ovf_part = nullptr;
+  int ovf_blocks = 0;
+  double ovf_target = 1.0;
   bool walk_sync = false;                      // DP_WALK_SYNC=1: block barrier per walker ring refill
   int n_en_slots() const { return n_en_part * (n_regions + 1); }
   int32_t n_large_mov = 0, n_large_fix = 0;                     // [num_cells] net-weighted pin count (GP preconditioner)
@@ -314,6 +319,7 @@ cudaError_t density_configure(int ntiles, int tile);
 int density_walk_grid(int tile);
 int density_count_grid(int ntiles);
 int density_launches(const Ctx &c);
+void launch_region_overflow(const Ctx &c, cudaStream_t s);
 // NCCL (nccl_dyn.cpp)
 dp_status nccl_get_unique_id(void *out128);
 dp_status nccl_init(Ctx &c, const void *id);

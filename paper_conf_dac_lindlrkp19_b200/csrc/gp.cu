@@ -59,6 +59,8 @@ struct GpArgs {
   int nblk;
   double *part_ovf;        // [oblk][2] overflow partials of k_gp_post
   int oblk;
+  const double *region_ovf;   // fence regions: the density passes' overflow partials ([region_blk][2])
+  int region_blk;
   GpDev *dev;
   const double *out;       // eval outputs {obj, wl, energy, hpwl}
   double *hist;
@@ -176,7 +178,13 @@ __global__ void __launch_bounds__(kGpThreads) k_gp_scalar(GpArgs a, int op) {
   GpDev &d = *a.dev;
   double t0, t1, o0 = 0.0, o1 = 0.0;
   sum_parts(a.part, a.nblk, t0, t1);
-  if (op == S_ITER_END) sum_parts(a.part_ovf, a.oblk, o0, o1);
+  if (op == S_ITER_END) {
+    if (a.region_ovf)
+      sum_parts(a.region_ovf, a.region_blk, o0, o1);
+    else
+      sum_parts(a.part_ovf, a.oblk, o0, o1);
+  }
+  if (op == S_INIT_TAU && a.region_ovf) sum_parts(a.region_ovf, a.region_blk, t0, t1);
   if (threadIdx.x != 0) return;
   switch (op) {
     case S_ALPHA:
@@ -293,6 +301,7 @@ __global__ void __launch_bounds__(kGpThreads) k_gp_post(GpArgs a) {
     }
     block_pair(s0, s1, a.part);
   } else {
+    if (a.region_ovf) return;   // fence regions: the density passes wrote the overflow partials
     const int b0 = blockIdx.x - a.nblk;
     for (long long b = (long long)b0 * kGpThreads + threadIdx.x; b < a.nbins; b += (long long)a.oblk * kGpThreads)
       s0 += ovf_term(a, b);
@@ -344,6 +353,8 @@ struct Gp {
   cudaGraphExec_t gexec = nullptr;
   int64_t gexec_gen = -1;    // Ctx::config_gen the iteration graph was captured with
   int64_t gen = -1;          // Ctx::config_gen of the last gp_refresh
+  double *region_ovf_buf = nullptr;   // fence regions: overflow partials of the density passes
+  size_t region_ovf_cap = 0;
   bool initialised = false;
   std::vector<void *> allocs;
   int cell_blocks = 0;
@@ -404,6 +415,26 @@ dp_status gp_refresh(Gp &g) {
   const int n = g.a.n;
   g.a.fixed = c.has_fixed ? c.d_fixed : nullptr;
   g.a.rho_fixed = c.has_fixed ? c.d_rho_fixed : nullptr;
+  if (c.n_regions > 0) {   // A30 per region pass (density.cu k_region_overflow), summed by the schedule
+    const size_t nreg = (size_t)(c.n_regions + 1) * g.a.oblk;
+    if (!g.region_ovf_buf || g.region_ovf_cap < nreg) {
+      double *p = nullptr;
+      dp_status st = gp_alloc(g, &p, 2 * nreg);
+      if (st != DP_OK) return st;
+      DP_CUDA(cudaMemset(p, 0, sizeof(double) * 2 * nreg));
+      g.region_ovf_buf = p;
+      g.region_ovf_cap = nreg;
+    }
+    c.ovf_part = g.region_ovf_buf;
+    c.ovf_blocks = g.a.oblk;
+    c.ovf_target = g.a.target;
+    g.a.region_ovf = g.region_ovf_buf;
+    g.a.region_blk = (int)nreg;
+  } else {
+    c.ovf_part = nullptr;
+    g.a.region_ovf = nullptr;
+    g.a.region_blk = 0;
+  }
   std::vector<float> w(n), h(n);
   std::vector<uint8_t> m(n, 0);
   DP_CUDA(cudaMemcpy(w.data(), c.d_cell_w, sizeof(float) * n, cudaMemcpyDeviceToHost));
@@ -553,7 +584,7 @@ dp_status dp_gp_init(dp_gp *gp, const float *x0, const float *y0, dp_stream_t st
   dp::k_gp_start<<<cb, dp::kGpThreads, 0, s>>>(a, x0, y0);
   // density alone at v: grad D, the map -> tau_0 -> gamma_0 (A31)
   if ((st = dp::gp_eval(*g, a.vx, a.vy, false, true, false, s)) != DP_OK) return st;
-  dp::partials(*g, dp::R_OVF, s);
+  if (!a.region_ovf) dp::partials(*g, dp::R_OVF, s);
   dp::scalar(*g, dp::S_INIT_TAU, s);
   dp::partials(*g, dp::R_L1, s);
   dp::scalar(*g, dp::S_INIT_L1D, s);

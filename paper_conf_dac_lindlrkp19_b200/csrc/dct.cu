@@ -18,6 +18,8 @@
 // radix-2 DIT with bit-reversed loads and fp32 twiddles computed in fp64 at create.
 // The energy D = 1/2 b_x b_y sum rho psi is taken in the spectral domain (Parseval), so psi
 // is never materialised on the hot path (reading A8).
+#include <type_traits>
+
 #include "async_copy.cuh"
 #include "dp_internal.h"
 #include "fft_warp.cuh"
@@ -752,19 +754,25 @@ void row_inv(const Ctx &c, const float *inA, long long stepA, int opA, const flo
     k_row_inv<<<rows, kRowThreads, row_smem(a.n), s>>>(a);
     return;
   }
-  if (ostepT > 0 && inI) {   // T2b: 4-warp CTAs, coalesced transposed stores
-    constexpr int W = kTStoreWarps;
-    const int per_cta = (wfft::kPts >> log2n) * W;
-    const int g = (rows + per_cta - 1) / per_cta;
-    const size_t sm = (size_t)W * wfft::kBufPad * sizeof(float2);
-    switch (log2n) {
-      case 5: launch_chain(c.pdl, k_row_inv_w<5, W, true>, g, 32 * W, sm, s, a, tw2, rows); break;
-      case 6: launch_chain(c.pdl, k_row_inv_w<6, W, true>, g, 32 * W, sm, s, a, tw2, rows); break;
-      case 7: launch_chain(c.pdl, k_row_inv_w<7, W, true>, g, 32 * W, sm, s, a, tw2, rows); break;
-      case 8: launch_chain(c.pdl, k_row_inv_w<8, W, true>, g, 32 * W, sm, s, a, tw2, rows); break;
-      case 9: launch_chain(c.pdl, k_row_inv_w<9, W, true>, g, 32 * W, sm, s, a, tw2, rows); break;
-      default: launch_chain(c.pdl, k_row_inv_w<10, W, true>, g, 32 * W, sm, s, a, tw2, rows); break;
-    }
+  if (ostepT > 0 && inI) {   // T2b: 4-warp CTAs, coalesced transposed stores (DP_T2B_WARPS=2: 2-warp, A/B)
+    auto go = [&](auto wtag) {
+      constexpr int W = decltype(wtag)::value;
+      const int per_cta = (wfft::kPts >> log2n) * W;
+      const int g = (rows + per_cta - 1) / per_cta;
+      const size_t sm = (size_t)W * wfft::kBufPad * sizeof(float2);
+      switch (log2n) {
+        case 5: launch_chain(c.pdl, k_row_inv_w<5, W, true>, g, 32 * W, sm, s, a, tw2, rows); break;
+        case 6: launch_chain(c.pdl, k_row_inv_w<6, W, true>, g, 32 * W, sm, s, a, tw2, rows); break;
+        case 7: launch_chain(c.pdl, k_row_inv_w<7, W, true>, g, 32 * W, sm, s, a, tw2, rows); break;
+        case 8: launch_chain(c.pdl, k_row_inv_w<8, W, true>, g, 32 * W, sm, s, a, tw2, rows); break;
+        case 9: launch_chain(c.pdl, k_row_inv_w<9, W, true>, g, 32 * W, sm, s, a, tw2, rows); break;
+        default: launch_chain(c.pdl, k_row_inv_w<10, W, true>, g, 32 * W, sm, s, a, tw2, rows); break;
+      }
+    };
+    if (c.t2b_warps == 2)
+      go(std::integral_constant<int, 2>{});
+    else
+      go(std::integral_constant<int, kTStoreWarps>{});
     return;
   }
   const int g = wrow_ctas(rows, log2n);

@@ -709,6 +709,7 @@ dp_status create(const dp_netlist *nl, const dp_grid *grid, int device, int rank
   cudaDeviceGetStreamPriorityRange(&prio_lo, &prio_hi);
   { const char *e = std::getenv("DP_PRIO"); if (e && e[0] == '0') prio_hi = prio_lo; }   // default: density first
   { const char *e = std::getenv("DP_FUSED_T2"); c->fused_t2 = e && e[0] == '1'; }
+  { const char *e = std::getenv("DP_T2B_WARPS"); c->t2b_warps = (e && e[0] == '2') ? 2 : 4; }
   { const char *e = std::getenv("DP_WA_CTAS_PER_SM"); c->wa_ctas_per_sm = e ? std::atoi(e) : 0; }
   { const char *e = std::getenv("DP_L2_HINT"); c->l2_hint = !(e && e[0] == '0'); }
   { const char *e = std::getenv("DP_ROW_TMA"); c->row_tma = !(e && e[0] == '0'); }

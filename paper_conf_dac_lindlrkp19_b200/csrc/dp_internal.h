@@ -213,7 +213,8 @@ struct Ctx {
   bool l2_hint = true;                              // DP_L2_HINT=0: no evict-first policy on the WA pin stream (A/B)
   bool row_tma = true;                              // DP_ROW_TMA=0: per-lane loads in the row-inverse passes (A/B)
   bool t1_tma = false;                              // DP_T1_TMA=1: bulk-copied rows in the forward row pass (A/B; not faster inside the overlapped step)
-  bool fused_t2 = false;                            // DP_FUSED_T2=1: one column kernel (T2) instead of T2a + T2b (A/B)
+  bool fused_t2 = false;
+  int t2b_warps = 4;                                // DP_T2B_WARPS=2: 2-warp T2b CTAs (fit beside two WA CTAs; A/B)                            // DP_FUSED_T2=1: one column kernel (T2) instead of T2a + T2b (A/B)
   float2 *d_sxy = nullptr;                          // T2 -> T3 interleaved (sX, sY) [x][y] (warp-FFT path)
   float2 *d_twf_x = nullptr, *d_twf_y = nullptr;   // CTA FFT: W_N^k, k < N
   bool fft_cta = true;                              // fields by the CTA-FFT passes P1 P2 P3 (fields.cu)

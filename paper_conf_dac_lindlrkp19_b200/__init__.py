@@ -213,11 +213,14 @@ class Context:
         import torch
         return torch.device("cuda", self.device)
 
-    def eval(self, x, y, gamma, lam, with_hpwl=False, gx=None, gy=None, stream=None):
+    def eval(self, x, y, gamma, lam, with_hpwl=False, gx=None, gy=None, stream=None, scalars=None):
+        """One dp_eval.  Outputs are fresh tensors unless gx, gy and scalars (float64 [4]) are
+        passed: reusing them keeps the library's captured evaluation graph (keyed by the argument
+        pointers) replaying instead of being re-captured."""
         import torch
         gx = torch.empty(self.num_cells, dtype=torch.float32, device=self._dev()) if gx is None else gx
         gy = torch.empty(self.num_cells, dtype=torch.float32, device=self._dev()) if gy is None else gy
-        sc = torch.full((4,), float("nan"), dtype=torch.float64, device=self._dev())
+        sc = torch.full((4,), float("nan"), dtype=torch.float64, device=self._dev()) if scalars is None else scalars
         dp_eval(self, x, y, gamma, lam, gx, gy, sc[0:1], sc[1:2], sc[2:3], sc[3:4] if with_hpwl else None,
                 stream)
         return dict(gx=gx, gy=gy, obj=sc[0], wl=sc[1], energy=sc[2], hpwl=sc[3], scalars=sc)

@@ -597,6 +597,7 @@ void destroy(Ctx *c) {
   if (c->s_den) cudaStreamDestroy(c->s_den);
   if (c->ev_fork) cudaEventDestroy(c->ev_fork);
   if (c->ev_wa) cudaEventDestroy(c->ev_wa);
+  if (c->ev_fields) cudaEventDestroy(c->ev_fields);
   if (c->ev_den) cudaEventDestroy(c->ev_den);
   if (c->ev_done) cudaEventDestroy(c->ev_done);
   if (c->ev_map) cudaEventDestroy(c->ev_map);
@@ -674,7 +675,9 @@ dp_status create(const dp_netlist *nl, const dp_grid *grid, int device, int rank
     const bool big = std::max(c->mx, c->my) > 1024;
     const int mode = e ? std::atoi(e) : (big ? 1 : 0);
     c->fft_cta = fields_cta_ok(c->log2mx, c->log2my) && (big || mode == 1);
-    c->fft_hybrid = !c->fft_cta && mode == 2 && fields_cta_ok(c->log2mx, c->log2my);
+    // the hybrid keeps the warp-FFT T1 / T3: both axes within the warp FFT's 32 .. 1024 points
+    c->fft_hybrid = !c->fft_cta && mode == 2 && fields_cta_ok(c->log2mx, c->log2my) && c->log2mx >= 5 &&
+                    c->log2my >= 5 && !big;
   }
   // energy partials: one per CTA of the column pass (P2 of the CTA-FFT path; 2-column slabs of
   // the warp-FFT path)
@@ -767,8 +770,19 @@ dp_status create(const dp_netlist *nl, const dp_grid *grid, int device, int rank
     cudaStreamSetAttribute(c->s_den, cudaStreamAttributeAccessPolicyWindow, maps ? &vm : &vh);
     cudaGetLastError();   // best effort: a refused hint leaves the default policy
   }
+  {   // DP_WA_SPLIT = p (0 < p < 100): split WA launch around the field transforms
+    const char *e = std::getenv("DP_WA_SPLIT");
+    const int p = e ? std::atoi(e) : 0;
+    if (p > 0 && p < 100 && !c->dist) {
+      if (cudaEventCreateWithFlags(&c->ev_fields, cudaEventDisableTiming) != cudaSuccess)
+        return bail(fail(DP_ERR_CUDA, "event creation failed"));
+      c->wa_split_chunks = (int)((long long)c->n_chunks * p / 100);
+      c->wa_split = true;
+    }
+  }
   const int wa_k = (c->n_chunks + c->n_big > 0) ? 1 : 0;   // one kernel: big nets, warp nets, chunks
   c->launches_eval = wa_k + density_launches(*c) + ((c->fft_cta || c->fft_hybrid) ? 3 : c->fused_t2 ? 3 : 4) /* P1 P2 P3, T1 P2 T3 or T1 T2a T2b T3 */ + 2 /* combine, finalize */;
+  if (c->wa_split && wa_k) c->launches_eval += 1;   // the WA kernel in two launches
   c->launches_eval_hpwl = c->launches_eval;
   if (c->dist && nccl_id) {
     if ((st = nccl_init(*c, nccl_id)) != DP_OK) return bail(st);
@@ -879,6 +893,7 @@ dp_status density_chain_pass(Ctx &c, const float *x, const float *y) {
       launch_fields_fixed(c, c.s_den);
     }
   }
+  if (c.wa_split) DP_CUDA(cudaEventRecord(c.ev_fields, c.s_den));
   StageMark m(c, DP_STAGE_GATHER, c.s_den);
   launch_density_gather(c, x, y, c.s_den, c.s_aux);
   return DP_OK;
@@ -1033,7 +1048,13 @@ dp_status eval_body(Ctx &c, const float *x, const float *y, float gamma, float l
         DP_CUDA(cudaMemsetAsync(c.d_g2i, 0, 2 * sizeof(long long) * (size_t)c.g2_cells, c.s_wa));
       else
         DP_CUDA(cudaMemsetAsync(c.d_g2, 0, sizeof(float2) * (size_t)c.g2_cells, c.s_wa));
-      launch_wa(c, x, y, gamma, false, d_hpwl != nullptr, c.s_wa);
+      if (c.wa_split && do_den && !c.serial && c.n_regions == 0) {   // around the transforms
+        launch_wa(c, x, y, gamma, false, d_hpwl != nullptr, c.s_wa, 1);
+        DP_CUDA(cudaStreamWaitEvent(c.s_wa, c.ev_fields, 0));
+        launch_wa(c, x, y, gamma, false, d_hpwl != nullptr, c.s_wa, 2);
+      } else {
+        launch_wa(c, x, y, gamma, false, d_hpwl != nullptr, c.s_wa);
+      }
       if (c.dist && c.nccl_comm) {   // nets are partitioned: sum the WA gradient into each cell block
         const size_t n = 2 * (size_t)c.cell_blk;
         dp_status st = c.deterministic ? nccl_reduce_scatter_i64(c, c.d_g2i, n, c.s_wa)

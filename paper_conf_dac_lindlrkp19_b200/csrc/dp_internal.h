@@ -214,7 +214,13 @@ struct Ctx {
   bool row_tma = true;                              // DP_ROW_TMA=0: per-lane loads in the row-inverse passes (A/B)
   bool t1_tma = false;                              // DP_T1_TMA=1: bulk-copied rows in the forward row pass (A/B; not faster inside the overlapped step)
   bool fused_t2 = false;
-  int t2b_warps = 4;                                // DP_T2B_WARPS=2: 2-warp T2b CTAs (fit beside two WA CTAs; A/B)                            // DP_FUSED_T2=1: one column kernel (T2) instead of T2a + T2b (A/B)
+  int t2b_warps = 4;
+  // split WA launch (DP_WA_SPLIT = percent of the chunk units in the first part): the first part
+  // (big units + that share of the chunks) runs beside the density map, the rest after the field
+  // transforms (beside the gather), so the latency-bound transforms run without WA CTAs
+  int wa_split_chunks = 0;
+  bool wa_split = false;
+  cudaEvent_t ev_fields = nullptr;                                // DP_T2B_WARPS=2: 2-warp T2b CTAs (fit beside two WA CTAs; A/B)                            // DP_FUSED_T2=1: one column kernel (T2) instead of T2a + T2b (A/B)
   float2 *d_sxy = nullptr;                          // T2 -> T3 interleaved (sX, sY) [x][y] (warp-FFT path)
   float2 *d_twf_x = nullptr, *d_twf_y = nullptr;   // CTA FFT: W_N^k, k < N
   bool fft_cta = true;                              // fields by the CTA-FFT passes P1 P2 P3 (fields.cu)
@@ -276,8 +282,9 @@ dp_status cuda_fail(cudaError_t e, const char *what);
 
 // kernel launchers (defined in the .cu files) ---------------------------------------------
 // WA (wa.cu)
+// part 0: all WA units; 1 / 2: the two halves of a split launch (Ctx::wa_split_chunks)
 void launch_wa(const Ctx &c, const float *x, const float *y, float gamma, bool hpwl_only,
-               bool with_hpwl, cudaStream_t s);
+               bool with_hpwl, cudaStream_t s, int part = 0);
 // density (density.cu)
 void launch_density_map(const Ctx &c, const float *x, const float *y, cudaStream_t s, cudaStream_t aux = nullptr,
                         int build_fixed = 0);

@@ -1,16 +1,21 @@
-// fft_cta.cuh — CTA-level complex FFT (Stockham autosort, radix 8) for the field transforms.
+// fft_cta.cuh — CTA-level complex FFT (Stockham autosort, radix 16, in place) for the field
+// transforms.
 //
-// One sequence of N = 2^LOGN points is transformed by T = N/8 threads (8 points per thread)
-// through shared memory: an optional first stage of radix 2^(LOGN mod 3), then radix-8 stages
-// (Stockham DIT: stage with sub-length Ns reads src[j + r N/R], twiddles W_{Ns R}^{r (j mod Ns)},
-// a radix-R DFT in registers, writes dst[(j - j mod Ns) R + j mod Ns + r Ns]; output in
-// natural order, no bit reversal).  A CTA runs SEQ sequences side by side (SEQ T threads) and
-// every stage ends in one block barrier.  Buffers are padded by one float2 per 8 entries, which
-// makes the strided stage writes bank-conflict free.
+// One sequence of N = 2^LOGN points is transformed by T = N/16 threads (16 points per thread)
+// through one padded shared buffer: radix-16 stages, then one stage of radix 2^(LOGN mod 4)
+// (each thread then runs 16/R butterflies).  Stockham DIT: the stage with sub-length Ns reads
+// src[j + r N/R], multiplies by W_{Ns R}^{r (j mod Ns)}, runs a radix-R DFT in registers and
+// writes dst[(j - j mod Ns) R + j mod Ns + r Ns]; output in natural order, no bit reversal.
+// Every stage reads the 16 points t + m T (m < 16) of its thread whatever R is, so a stage is
+// read all -> barrier -> compute -> write all -> barrier on ONE buffer (in place).  NB buffers
+// can be transformed in lockstep (two independent sequences per thread: the column pass's pair
+// of inverse transforms), which doubles the work between two barriers.  A CTA runs SEQ
+// sequences side by side (SEQ T threads, about 128).  Buffers are padded by one float2 per 16
+// entries: the radix-16 stride-16 writes of the first stage then fall on distinct bank pairs.
 //
-// Why not the warp FFT (fft_warp.cuh): a warp holding 1024 points leaves a 1024^2 map with 512
-// to 1024 warps per pass (<= 7 per SM), and the transforms were latency bound at 10-16 us per
-// pass; at 8 points per thread the same pass has 4x the warps in flight.
+// Round 2 replaced the radix-8 / 8-points-per-thread / ping-pong version (4 stages, 2 buffers,
+// 256-thread CTAs): at 1024 points it ran one CTA of 256 threads per two sequences and measured
+// 13-26 us per pass alone.
 #pragma once
 
 #include "fft_warp.cuh"
@@ -18,66 +23,78 @@
 namespace dp {
 namespace cfft {
 
-__host__ __device__ constexpr int pad(int e) { return e + (e >> 3); }
-__host__ __device__ constexpr int buf_len(int n) { return n + (n >> 3); }   // float2 per padded buffer
-__host__ __device__ constexpr int threads_per_seq(int logn) { return logn >= 3 ? (1 << logn) / 8 : 1; }
-// sequences per CTA: about 256 threads, at most 16 sequences
+__host__ __device__ constexpr int pad(int e) { return e + (e >> 4); }
+__host__ __device__ constexpr int buf_len(int n) { return n + (n >> 4) + 1; }   // float2 per padded buffer
+__host__ __device__ constexpr int threads_per_seq(int logn) { return logn >= 4 ? (1 << logn) / 16 : 1; }
+// sequences per CTA: about 128 threads, at most 16 sequences
 __host__ __device__ constexpr int seq_per_cta(int logn) {
-  return threads_per_seq(logn) >= 256 ? 1 : (256 / threads_per_seq(logn) > 16 ? 16 : 256 / threads_per_seq(logn));
+  return threads_per_seq(logn) >= 128 ? 1 : (128 / threads_per_seq(logn) > 16 ? 16 : 128 / threads_per_seq(logn));
 }
 
 __device__ __forceinline__ float2 cmul(float2 a, float2 b) {
   return make_float2(a.x * b.x - a.y * b.y, a.x * b.y + a.y * b.x);
 }
 
-// One Stockham DIT stage of radix R for group j (j < N / R).  twf[k] = exp(-2 pi i k / N), k < N
-// (fp64-rounded table); INV uses the conjugate (unnormalised inverse DFT).
-template <int N, int R, bool INV>
-__device__ __forceinline__ void stage(const float2 *src, float2 *dst, int Ns, int j, const float2 *__restrict__ twf) {
-  constexpr int LR = wfft::log2_c(R);
-  float2 v[R];
-  const int jm = j & (Ns - 1);
-#pragma unroll
-  for (int r = 0; r < R; r++) v[r] = src[pad(j + r * (N / R))];
+// One in-place Stockham DIT stage of radix R on NB buffers (thread t of T = N/16).
+// twf[k] = exp(-2 pi i k / N), k < N (fp64-rounded table); INV uses the conjugate
+// (unnormalised inverse DFT).  Ends with a block barrier (the output is visible).
+template <int N, int R, bool INV, int NB>
+__device__ __forceinline__ void stage(float2 *const (&A)[NB], int Ns, int t, const float2 *__restrict__ twf) {
+  constexpr int T = N / 16, B = 16 / R, LR = wfft::log2_c(R);
+  // twiddles first: they depend on t only, so their (L1 / L2) latency overlaps the shared reads
+  // and the barrier instead of following them
+  float2 w[B][R];
   if (Ns > 1) {
-    const int k0 = jm * (N / (Ns * R));   // W_{Ns R}^{r jm} = W_N^{r k0}, r k0 < N
 #pragma unroll
-    for (int r = 1; r < R; r++) {
-      float2 w = __ldg(twf + r * k0);
-      if (INV) w.y = -w.y;
-      v[r] = cmul(v[r], w);
+    for (int q = 0; q < B; q++) {
+      const int k0 = ((t + q * T) & (Ns - 1)) * (N / (Ns * R));   // W_{Ns R}^{r jm} = W_N^{r k0}, r k0 < N
+#pragma unroll
+      for (int r = 1; r < R; r++) w[q][r] = __ldg(twf + r * k0);
     }
   }
-  wfft::reg_dft<R, INV>(v);   // v[m] = X[brev(m)]
-  const int base = (j - jm) * R + jm;
+  float2 v[NB][16];
 #pragma unroll
-  for (int r = 0; r < R; r++) dst[pad(base + r * Ns)] = v[wfft::brev_c(r, LR)];
+  for (int b = 0; b < NB; b++)
+#pragma unroll
+    for (int m = 0; m < 16; m++) v[b][m] = A[b][pad(t + m * T)];   // m = q + B r: j_q + r N / R
+  __syncthreads();
+#pragma unroll
+  for (int q = 0; q < B; q++) {
+    const int j = t + q * T, jm = j & (Ns - 1);
+    float2 u[NB][R];
+#pragma unroll
+    for (int b = 0; b < NB; b++)
+#pragma unroll
+      for (int r = 0; r < R; r++) u[b][r] = v[b][q + B * r];
+    if (Ns > 1) {
+#pragma unroll
+      for (int r = 1; r < R; r++) {
+        float2 wr = w[q][r];
+        if (INV) wr.y = -wr.y;
+#pragma unroll
+        for (int b = 0; b < NB; b++) u[b][r] = cmul(u[b][r], wr);
+      }
+    }
+    const int base = (j - jm) * R + jm;
+#pragma unroll
+    for (int b = 0; b < NB; b++) {
+      wfft::reg_dft<R, INV>(u[b]);   // u[m] = X[brev(m)]
+#pragma unroll
+      for (int r = 0; r < R; r++) A[b][pad(base + r * Ns)] = u[b][wfft::brev_c(r, LR)];
+    }
+  }
+  __syncthreads();
 }
 
-// FFT of the sequence in A (natural order, padded) by thread t in [0, T) of its group; B is the
-// second buffer.  Every thread of the CTA must call it (block barriers); returns the buffer
-// holding the result (natural order).  The caller synchronises before (input written).
-template <int LOGN, bool INV>
-__device__ __forceinline__ float2 *fft(float2 *A, float2 *B, int t, const float2 *__restrict__ twf) {
-  constexpr int N = 1 << LOGN, T = threads_per_seq(LOGN), REM = LOGN % 3;
-  float2 *src = A, *dst = B;
-  int Ns = 1;
-  if (REM) {
-    constexpr int R = 1 << REM;
+// In-place FFT of the NB sequences in A (natural order, padded) by thread t in [0, T) of its
+// group.  Every thread of the CTA must call it (block barriers); the caller synchronises before
+// (input written); the output is in natural order and visible to the whole CTA on return.
+template <int LOGN, bool INV, int NB = 1>
+__device__ __forceinline__ void fft(float2 *const (&A)[NB], int t, const float2 *__restrict__ twf) {
+  constexpr int N = 1 << LOGN, S16 = LOGN / 4, REM = LOGN % 4;
 #pragma unroll
-    for (int g = 0; g < (N / R) / T; g++) stage<N, R, INV>(src, dst, 1, t + g * T, twf);
-    __syncthreads();
-    float2 *tmp = src; src = dst; dst = tmp;
-    Ns = R;
-  }
-#pragma unroll
-  for (int s = 0; s < (LOGN - REM) / 3; s++) {
-    stage<N, 8, INV>(src, dst, Ns, t, twf);
-    __syncthreads();
-    float2 *tmp = src; src = dst; dst = tmp;
-    Ns *= 8;
-  }
-  return src;
+  for (int s = 0; s < S16; s++) stage<N, 16, INV, NB>(A, 1 << (4 * s), t, twf);
+  if constexpr (REM != 0) stage<N, (1 << REM), INV, NB>(A, 1 << (4 * S16), t, twf);
 }
 
 }  // namespace cfft

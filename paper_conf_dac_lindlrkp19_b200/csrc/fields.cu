@@ -1,5 +1,6 @@
 // fields.cu — the spectral Poisson solve of one evaluation (steps 2-3 of P:253-256) in three
-// passes over the bin map, each a CTA-level FFT (fft_cta.cuh) with 8 points per thread.
+// passes over the bin map, each a CTA-level FFT (fft_cta.cuh: radix 16, 16 points per thread,
+// in place).
 //
 // Method: a = DCT2(rho) (eq 9a; DCT of eq 7a with 2/N per axis, readings
 // A13/A20), A_X = a k_u / k^2 and A_Y = a k_v / k^2 with a_00 / k^2 := 0 (eqs 9c/9d, A12, A15),
@@ -15,8 +16,11 @@
 //   P3  rows x:     IDCT_y(sX) + i IDXST_y(sY)                      -> xi[x][y] = (xi_X, xi_Y)
 //
 // Every pass reads whole rows (contiguous) and the two transposed stores write 2 SEQ adjacent
-// values per output row (16-32 bytes): no strided column reads.  The spectrum of P2 stays in
-// shared memory between the forward and the inverse x transforms.
+// values per output row (16-32 bytes): no strided column reads.  P2 takes the forward
+// post-processing, the scaling and the inverse pre-processing of both columns per spectral pair
+// (u, M - u) in one thread, in place: the spectrum is never stored.  The per-element phase,
+// twiddle and wavenumber loads are issued together (unrolled loops, twiddles ahead of each
+// stage's barrier): one table latency per stage instead of one per element.
 #include "dp_internal.h"
 #include "fft_cta.cuh"
 
@@ -37,8 +41,10 @@ using cfft::pad;
 __device__ __forceinline__ int mk_pos(int t, int n) { return (t & 1) ? n - ((t + 1) >> 1) : (t >> 1); }
 
 __device__ __forceinline__ float map_value(float v) { return v; }
+// one rounding of the integer, then an exact power-of-two scale: the same value as the fp64
+// route (exact below 2^53) without the fp64 conversions
 __device__ __forceinline__ float map_value(unsigned long long v) {
-  return (float)((double)(long long)v * (1.0 / (double)(1ll << kRhoScaleLog2)));
+  return __ll2float_rn((long long)v) * (1.0f / (float)(1ll << kRhoScaleLog2));
 }
 
 // forward DCT post-processing of a pair packed as z = p + i q (Alg 3 lines 10-16): returns
@@ -77,7 +83,8 @@ struct FieldArgs {
   const float2 *s_in;     // P3 input (sxy / R2)
   float2 *xi;             // [mx][my] (xi_X, xi_Y); P3 writes rows [x_base, x_base + nrows)
   int mx, my;
-  int R, C;               // rows / columns per rank block
+  int R, C;               // rows / columns per rank block (powers of two)
+  int lR, lC;             // log2 R, log2 C
   int x_base, y_base;     // this rank's first row / column
   int nrows, ncols;       // rows of P1 / P3, columns of P2
   const float2 *twf_x, *twf_y;   // exp(-2 pi i k / N), k < N
@@ -87,6 +94,15 @@ struct FieldArgs {
   double energy_scale;           // 1/2 b_x b_y
 };
 
+// Layout helpers (one code path for the unsharded and the row-sharded block layouts, so both
+// run the same instructions: shifts, R and C are powers of two)
+__device__ __forceinline__ size_t t_index(const FieldArgs &a, int y, int xl) {   // tT / S1 / R1, xl = x - x_base
+  return ((size_t)(y >> a.lC) << (a.lC + a.lR)) + ((size_t)(y & (a.C - 1)) << a.lR) + xl;
+}
+__device__ __forceinline__ size_t s_index(const FieldArgs &a, int x, int yl) {   // sxy / S2 / R2, yl = y - y_base
+  return ((size_t)(x >> a.lR) << (a.lC + a.lR)) + ((size_t)(x & (a.R - 1)) << a.lC) + yl;
+}
+
 // ---- P1: rows (2p, 2p+1) of rho -> DCT over y -> tT[y][x] ----------------------------------
 template <class IN, int LOGN>
 __global__ void __launch_bounds__(cfft::seq_per_cta(LOGN) * cfft::threads_per_seq(LOGN))
@@ -95,14 +111,12 @@ __global__ void __launch_bounds__(cfft::seq_per_cta(LOGN) * cfft::threads_per_se
   constexpr int N = 1 << LOGN, T = cfft::threads_per_seq(LOGN), SEQ = cfft::seq_per_cta(LOGN);
   constexpr int NT = SEQ * T, ROWS = 2 * SEQ, L = buf_len(N);
   extern __shared__ __align__(16) float2 sm1[];
-  float *out = reinterpret_cast<float *>(sm1 + 2 * SEQ * L);   // [N][ROWS]
+  float *out = reinterpret_cast<float *>(sm1 + SEQ * L);   // [N][ROWS]
   const IN *rho = reinterpret_cast<const IN *>(a.rho);
   const int tid = threadIdx.x, s = tid / T, t = tid % T;
   const int x0 = a.x_base + blockIdx.x * ROWS, xend = a.x_base + a.nrows;
-  float2 *A = sm1 + (2 * s) * L, *B = A + L;
   // load: row x0 + rr (coalesced) -> real (rr even) / imaginary (rr odd) part of sequence rr/2,
-  // at its Makhoul position.  Every load is issued before the first use (unrolled: a loop
-  // that waits on each load serialises the global latency)
+  // at its Makhoul position; every load is issued before the first use
   constexpr int PER = ROWS * N / NT;
   IN v[PER];
 #pragma unroll
@@ -113,31 +127,31 @@ __global__ void __launch_bounds__(cfft::seq_per_cta(LOGN) * cfft::threads_per_se
 #pragma unroll
   for (int q = 0; q < PER; q++) {
     const int idx = tid + q * NT, rr = idx >> LOGN, col = idx & (N - 1);
-    float *slot = reinterpret_cast<float *>(sm1 + (rr & ~1) * L + pad(mk_pos(col, N)));
+    float *slot = reinterpret_cast<float *>(sm1 + (rr >> 1) * L + pad(mk_pos(col, N)));
     slot[rr & 1] = map_value(v[q]);
   }
   __syncthreads();
-  const float2 *Z = cfft::fft<LOGN, false>(A, B, t, a.twf_y);
+  float2 *const A[1] = {sm1 + s * L};
+  cfft::fft<LOGN, false>(A, t, a.twf_y);
   const float scale = 2.f / N;
-  for (int k = t; k < N; k += T) {
-    const float2 d = dct_post(Z[pad(k)], Z[pad((N - k) & (N - 1))], __ldg(a.ph_y + k), scale);
-    out[k * ROWS + 2 * s] = d.x;
-    out[k * ROWS + 2 * s + 1] = d.y;
+#pragma unroll
+  for (int m = 0; m < 16; m++) {   // unrolled: the 16 phase loads are issued together
+    const int k = t + m * T;
+    const float2 d = dct_post(A[0][pad(k)], A[0][pad((N - k) & (N - 1))], __ldg(a.ph_y + k), scale);
+    *reinterpret_cast<float2 *>(out + k * ROWS + 2 * s) = d;
   }
   __syncthreads();
   // transposed store: tT[k][x0 .. x0 + ROWS) (unsharded) / S1[k / C][k % C][x0 - x_base ..]
-  const size_t CR = (size_t)a.C * a.R;
   if (ROWS % 4 == 0 && x0 + ROWS <= xend) {
     for (int idx = tid; idx < N * (ROWS / 4); idx += NT) {
       const int k = idx / (ROWS / 4), q = idx % (ROWS / 4);
-      *reinterpret_cast<float4 *>(a.t_out + (size_t)(k / a.C) * CR + (size_t)(k % a.C) * a.R + (x0 - a.x_base) + 4 * q) =
+      *reinterpret_cast<float4 *>(a.t_out + t_index(a, k, x0 - a.x_base) + 4 * q) =
           *reinterpret_cast<const float4 *>(out + k * ROWS + 4 * q);
     }
   } else {
     for (int idx = tid; idx < N * ROWS; idx += NT) {
       const int k = idx / ROWS, c = idx % ROWS;
-      if (x0 + c < xend)
-        a.t_out[(size_t)(k / a.C) * CR + (size_t)(k % a.C) * a.R + (x0 - a.x_base) + c] = out[idx];
+      if (x0 + c < xend) a.t_out[t_index(a, k, x0 - a.x_base) + c] = out[idx];
     }
   }
 }
@@ -145,33 +159,35 @@ __global__ void __launch_bounds__(cfft::seq_per_cta(LOGN) * cfft::threads_per_se
 // ---- P2: columns (2p, 2p+1) (rows of tT) -> DCT over x, energy, scaling, inverse over x ----
 // TIN: t stored transposed, tT[y][x] (after P1); otherwise t[x][y] (after the warp-FFT T1):
 // the CTA then reads its COLS adjacent columns as 4 COLS-byte row segments.
-// P2 of the hybrid path runs one column pair per CTA (SEQ = 1): half the shared memory and
-// threads of a CTA, so its CTAs fit beside the WA kernel's (the unsharded / sharded CTA-FFT
-// path keeps seq_per_cta)
+// P2 of the hybrid path runs one column pair per CTA (SEQ = 1).
+// Per column pair: one forward FFT (the two columns packed as z = p + i q), then, per spectral
+// pair (u, M - u) held by one thread, the DCT post-processing, the energy terms, the scaling
+// (9c/9d) and the inverse pre-processing of BOTH columns written in place (even column) and
+// into the second buffer (odd column): the spectrum never needs its own storage.  The two
+// inverse FFTs then run in lockstep.
 template <int LOGM, bool TIN>
 constexpr int p2_seq() { return TIN ? cfft::seq_per_cta(LOGM) : 1; }
 
-template <int LOGM, bool TIN = true>
+template <int LOGM, bool TIN>
 __global__ void __launch_bounds__(p2_seq<LOGM, TIN>() * cfft::threads_per_seq(LOGM))
     k_p2(FieldArgs a) {
   griddep_wait();
   constexpr int M = 1 << LOGM, T = cfft::threads_per_seq(LOGM), SEQ = p2_seq<LOGM, TIN>();
   constexpr int NT = SEQ * T, COLS = 2 * SEQ, L = buf_len(M);
-  extern __shared__ __align__(16) float2 sm2[];
-  float2 *spec = sm2 + 2 * SEQ * L;    // [COLS][M] (A_X, A_Y)
-  float2 *out = spec + COLS * M;       // [M][COLS] (sX, sY)
+  extern __shared__ __align__(16) float2 sm2[];   // per group: buffers (even, odd column)
   __shared__ double s_red[NT / 32 > 0 ? NT / 32 : 1];
   const int tid = threadIdx.x, s = tid / T, t = tid % T;
   const int y0 = a.y_base + blockIdx.x * COLS, my = a.my, yend = a.y_base + a.ncols;
-  const size_t CR = (size_t)a.C * a.R;
-  float2 *A = sm2 + (2 * s) * L, *B = A + L;
+  float2 *const A0 = sm2 + (2 * s) * L, *const A1 = A0 + L;
   constexpr int PER = COLS * M / NT;
   float v[PER];
 #pragma unroll
   for (int q = 0; q < PER; q++) {
     const int idx = tid + q * NT;
     const int c = TIN ? idx >> LOGM : idx % COLS, x = TIN ? idx & (M - 1) : idx / COLS;
-    v[q] = (y0 + c < yend) ? (TIN ? a.t_in[(size_t)(x / a.R) * CR + (size_t)(y0 + c - a.y_base) * a.R + (x % a.R)]
+    // received blocks R1[x / R][y - y_base][x % R] (unsharded: tT[y][x])
+    v[q] = (y0 + c < yend) ? (TIN ? a.t_in[((size_t)(x >> a.lR) << (a.lC + a.lR)) +
+                                           ((size_t)(y0 + c - a.y_base) << a.lR) + (x & (a.R - 1))]
                                   : a.t_in[(size_t)x * my + y0 + c])
                            : 0.f;
   }
@@ -183,7 +199,10 @@ __global__ void __launch_bounds__(p2_seq<LOGM, TIN>() * cfft::threads_per_seq(LO
     slot[c & 1] = v[q];
   }
   __syncthreads();
-  const float2 *Z = cfft::fft<LOGM, false>(A, B, t, a.twf_x);
+  {
+    float2 *const F[1] = {A0};
+    cfft::fft<LOGM, false>(F, t, a.twf_x);
+  }
   // spectrum of columns v0 = y0 + 2s, v1 = v0 + 1: energy (Parseval, A8) and scaling (9c/9d)
   const float scale = 2.f / M;
   const int v0 = y0 + 2 * s, v1 = v0 + 1;
@@ -191,46 +210,79 @@ __global__ void __launch_bounds__(p2_seq<LOGM, TIN>() * cfft::threads_per_seq(LO
   const float ky0 = ok ? __ldg(a.ky + v0) : 0.f, ky1 = ok ? __ldg(a.ky + v1) : 0.f;
   const double wv0 = (v0 == 0) ? 0.25 * my : 0.5 * my, wv1 = 0.5 * my;
   double e = 0.0;
-  for (int u = t; u < M; u += T) {
-    const float2 d = dct_post(Z[pad(u)], Z[pad((M - u) & (M - 1))], __ldg(a.ph_x + u), scale);
-    const float kx = __ldg(a.kx + u);
-    const double wu = (u == 0) ? 0.25 * M : 0.5 * M;
-    const float ik0 = (!ok || (u == 0 && v0 == 0)) ? 0.f : fast_rcp(kx * kx + ky0 * ky0);   // a_00 / k^2 := 0
-    const float ik1 = ok ? fast_rcp(kx * kx + ky1 * ky1) : 0.f;
-    e += wu * (wv0 * (double)(d.x * d.x * ik0) + wv1 * (double)(d.y * d.y * ik1));
-    spec[(2 * s) * M + u] = make_float2(d.x * kx * ik0, d.x * ky0 * ik0);
-    spec[(2 * s + 1) * M + u] = make_float2(d.y * kx * ik1, d.y * ky1 * ik1);
+  // pairs (u, M - u), u = t + m T < M / 2 (unrolled: the phase / wavenumber loads issue
+  // together); u = M / 2 (its own partner) by thread 0 of the group
+#pragma unroll
+  for (int m = 0; m <= 8; m++) {
+    if (m == 8 && t != 0) break;
+    const int u = m < 8 ? t + m * T : M / 2;
+    const int n = (M - u) & (M - 1);   // partner M - u (u = 0, M / 2: itself)
+    const float2 zu = A0[pad(u)], zn = A0[pad(n)];
+    // (a_{u,v0}, a_{u,v1}) and the scaled spectra of frequency u
+    float2 AXu, AYu, AXn, AYn;   // .x: column v0, .y: column v1
+    {
+      const float2 d = dct_post(zu, zn, __ldg(a.ph_x + u), scale);
+      const float kx = __ldg(a.kx + u);
+      const double wu = (u == 0) ? 0.25 * M : 0.5 * M;
+      const float ik0 = (!ok || (u == 0 && v0 == 0)) ? 0.f : fast_rcp(kx * kx + ky0 * ky0);   // a_00 / k^2 := 0
+      const float ik1 = ok ? fast_rcp(kx * kx + ky1 * ky1) : 0.f;
+      e += wu * (wv0 * (double)(d.x * d.x * ik0) + wv1 * (double)(d.y * d.y * ik1));
+      AXu = make_float2(d.x * kx * ik0, d.y * kx * ik1);
+      AYu = make_float2(d.x * ky0 * ik0, d.y * ky1 * ik1);
+    }
+    if (n != u) {
+      const float2 d = dct_post(zn, zu, __ldg(a.ph_x + n), scale);
+      const float kx = __ldg(a.kx + n);
+      const double wu = 0.5 * M;
+      const float ik0 = ok ? fast_rcp(kx * kx + ky0 * ky0) : 0.f;
+      const float ik1 = ok ? fast_rcp(kx * kx + ky1 * ky1) : 0.f;
+      e += wu * (wv0 * (double)(d.x * d.x * ik0) + wv1 * (double)(d.y * d.y * ik1));
+      AXn = make_float2(d.x * kx * ik0, d.y * kx * ik1);
+      AYn = make_float2(d.x * ky0 * ik0, d.y * ky1 * ik1);
+    } else {
+      AXn = AXu;
+      AYn = AYu;
+    }
+    // inverse pre-processing, p = A_X reversed (IDXST via eq 8e: p_k = A_X[M - k], p_0 = 0),
+    // q = A_Y (IDCT): Z_k = inv_pre(p_k, q_k, p_{M-k}, q_{M-k})
+    if (u == 0) {
+      A0[pad(0)] = inv_pre(0.f, AYu.x, 0.f, 0.f, __ldg(a.ph_x));
+      A1[pad(0)] = inv_pre(0.f, AYu.y, 0.f, 0.f, __ldg(a.ph_x));
+    } else {
+      const float2 phu = __ldg(a.ph_x + u);
+      A0[pad(u)] = inv_pre(AXn.x, AYu.x, AXu.x, AYn.x, phu);
+      A1[pad(u)] = inv_pre(AXn.y, AYu.y, AXu.y, AYn.y, phu);
+      if (n != u) {
+        const float2 phn = __ldg(a.ph_x + n);
+        A0[pad(n)] = inv_pre(AXu.x, AYn.x, AXn.x, AYu.x, phn);
+        A1[pad(n)] = inv_pre(AXu.y, AYn.y, AXn.y, AYu.y, phn);
+      }
+    }
   }
   __syncthreads();
-  // inverse over x, two rounds (even, then odd columns): IDXST_x(A_X) + i IDCT_x(A_Y)
-#pragma unroll 1
-  for (int h = 0; h < 2; h++) {
-    const int c = 2 * s + h;
-    const float2 *S = spec + c * M;
-    for (int k = t; k < M; k += T) {
-      const float2 ak = S[k], ank = k ? S[M - k] : make_float2(0.f, 0.f);
-      // p = A_X reversed (IDXST via eq 8e: x'_t = x_{N-t}, x'_0 = 0), q = A_Y (IDCT)
-      A[pad(k)] = inv_pre(ank.x, ak.y, k ? ak.x : 0.f, ank.y, __ldg(a.ph_x + k));
-    }
-    __syncthreads();
-    const float2 *W = cfft::fft<LOGM, true>(A, B, t, a.twf_x);
-    for (int x = t; x < M; x += T) {
-      const float2 z = W[pad(mk_pos(x, M))];
-      out[x * COLS + c] = make_float2((x & 1) ? -0.5f * z.x : 0.5f * z.x, 0.5f * z.y);   // IDXST sign (-1)^x
-    }
-    __syncthreads();
+  {
+    float2 *const I[2] = {A0, A1};
+    cfft::fft<LOGM, true, 2>(I, t, a.twf_x);
   }
-  // transposed store: sxy[x][y0 .. y0 + COLS) (unsharded) / S2[x / R][x % R][y0 - y_base ..]
-  if (COLS % 2 == 0 && y0 + COLS <= yend) {
-    for (int idx = tid; idx < M * (COLS / 2); idx += NT) {
-      const int x = idx / (COLS / 2), q = idx % (COLS / 2);
-      *reinterpret_cast<float4 *>(a.s_out + (size_t)(x / a.R) * CR + (size_t)(x % a.R) * a.C + (y0 - a.y_base) + 2 * q) =
-          *reinterpret_cast<const float4 *>(out + x * COLS + 2 * q);
+  // transposed store: sxy[x][y0 .. y0 + COLS) (unsharded) / S2[x / R][x % R][y0 - y_base ..];
+  // column c = 2 g + h lives in buffer h of group g, at the Makhoul position of x
+  if (y0 + COLS <= yend) {
+    for (int idx = tid; idx < M * SEQ; idx += NT) {
+      const int x = idx / SEQ, g = idx % SEQ;
+      const float2 *G = sm2 + (2 * g) * L;
+      const int px = pad(mk_pos(x, M));
+      const float2 z0 = G[px], z1 = G[L + px];
+      const float sg = (x & 1) ? -0.5f : 0.5f;   // IDXST sign (-1)^x
+      *reinterpret_cast<float4 *>(a.s_out + s_index(a, x, y0 - a.y_base) + 2 * g) =
+          make_float4(sg * z0.x, 0.5f * z0.y, sg * z1.x, 0.5f * z1.y);
     }
   } else {
     for (int idx = tid; idx < M * COLS; idx += NT) {
       const int x = idx / COLS, c = idx % COLS;
-      if (y0 + c < yend) a.s_out[(size_t)(x / a.R) * CR + (size_t)(x % a.R) * a.C + (y0 - a.y_base) + c] = out[idx];
+      if (y0 + c < yend) {
+        const float2 z = sm2[c * L + pad(mk_pos(x, M))];
+        a.s_out[s_index(a, x, y0 - a.y_base) + c] = make_float2((x & 1) ? -0.5f * z.x : 0.5f * z.x, 0.5f * z.y);
+      }
     }
   }
   // energy partial of this CTA (fixed order: deterministic)
@@ -255,69 +307,70 @@ __global__ void __launch_bounds__(cfft::seq_per_cta(LOGN) * cfft::threads_per_se
   extern __shared__ __align__(16) float2 sm3[];
   const int tid = threadIdx.x, s = tid / T, t = tid % T;
   const int x0 = a.x_base + blockIdx.x * SEQ, xend = a.x_base + a.nrows;
-  const size_t CR = (size_t)a.C * a.R;
-  float2 *A = sm3 + (2 * s) * L, *B = A + L;
   constexpr int PER = SEQ * N / NT;
   float2 v[PER];
 #pragma unroll
   for (int q = 0; q < PER; q++) {
     const int idx = tid + q * NT, x = x0 + (idx >> LOGN), k = idx & (N - 1);
-    v[q] = x < xend ? a.s_in[(size_t)(k / a.C) * CR + (size_t)(x - a.x_base) * a.C + (k % a.C)] : make_float2(0.f, 0.f);
+    v[q] = x < xend ? a.s_in[((size_t)(k >> a.lC) << (a.lC + a.lR)) + ((size_t)(x - a.x_base) << a.lC) + (k & (a.C - 1))]
+                    : make_float2(0.f, 0.f);
   }
 #pragma unroll
   for (int q = 0; q < PER; q++) {
     const int idx = tid + q * NT;
-    sm3[(2 * (idx >> LOGN)) * L + pad(idx & (N - 1))] = v[q];
+    sm3[(idx >> LOGN) * L + pad(idx & (N - 1))] = v[q];
   }
   __syncthreads();
+  float2 *const A[1] = {sm3 + s * L};
   // in place, pairs (k, N - k) per thread: p = sX (IDCT), q = sY reversed (IDXST, eq 8e)
-  for (int k = t; k <= N / 2; k += T) {
-    const float2 vk = A[pad(k)], vn = k ? A[pad(N - k)] : make_float2(0.f, 0.f);
+#pragma unroll
+  for (int m = 0; m <= 8; m++) {   // k = t + m T < N / 2 (unrolled), k = N / 2 by thread 0
+    if (m == 8 && t != 0) break;
+    const int k = m < 8 ? t + m * T : N / 2;
+    const float2 vk = A[0][pad(k)], vn = k ? A[0][pad(N - k)] : make_float2(0.f, 0.f);
     const float2 zk = inv_pre(vk.x, vn.y, vn.x, k ? vk.y : 0.f, __ldg(a.ph_y + k));
-    if (k && k < N / 2) A[pad(N - k)] = inv_pre(vn.x, vk.y, vk.x, vn.y, __ldg(a.ph_y + N - k));
-    A[pad(k)] = zk;
+    if (k && k < N / 2) A[0][pad(N - k)] = inv_pre(vn.x, vk.y, vk.x, vn.y, __ldg(a.ph_y + N - k));
+    A[0][pad(k)] = zk;
   }
   __syncthreads();
-  const float2 *W = cfft::fft<LOGN, true>(A, B, t, a.twf_y);
+  cfft::fft<LOGN, true>(A, t, a.twf_y);
   const int x = x0 + s;
   if (x < xend)
-    for (int y = t; y < N; y += T) {
-      const float2 z = W[pad(mk_pos(y, N))];
+#pragma unroll
+    for (int m = 0; m < 16; m++) {
+      const int y = t + m * T;
+      const float2 z = A[0][pad(mk_pos(y, N))];
       a.xi[(size_t)x * N + y] = make_float2(0.5f * z.x, (y & 1) ? -0.5f * z.y : 0.5f * z.y);   // IDXST sign on xi_Y
     }
 }
 
 template <int LOGN>
 constexpr size_t p1_smem() {
-  return sizeof(float2) * 2 * cfft::seq_per_cta(LOGN) * buf_len(1 << LOGN) +
+  return sizeof(float2) * cfft::seq_per_cta(LOGN) * buf_len(1 << LOGN) +
          sizeof(float) * (size_t)(1 << LOGN) * 2 * cfft::seq_per_cta(LOGN);
 }
 template <int LOGN, bool TIN = true>
 constexpr size_t p2_smem() {
-  return sizeof(float2) * (2 * p2_seq<LOGN, TIN>() * buf_len(1 << LOGN) +
-                           2 * (size_t)(2 * p2_seq<LOGN, TIN>()) * (1 << LOGN));
+  return sizeof(float2) * 2 * p2_seq<LOGN, TIN>() * buf_len(1 << LOGN);
 }
 template <int LOGN>
 constexpr size_t p3_smem() {
-  return sizeof(float2) * 2 * cfft::seq_per_cta(LOGN) * buf_len(1 << LOGN);
+  return sizeof(float2) * cfft::seq_per_cta(LOGN) * buf_len(1 << LOGN);
+}
+
+template <class K>
+cudaError_t set_smem(K kernel, size_t bytes) {
+  return cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bytes);
 }
 
 template <int LOGN>
 cudaError_t configure_one() {
   cudaError_t e;
-  if ((e = cudaFuncSetAttribute(k_p1<unsigned long long, LOGN>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                (int)p1_smem<LOGN>())) != cudaSuccess)
-    return e;
-  if ((e = cudaFuncSetAttribute(k_p1<float, LOGN>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                (int)p1_smem<LOGN>())) != cudaSuccess)
-    return e;
-  if ((e = cudaFuncSetAttribute(k_p2<LOGN, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                (int)p2_smem<LOGN>())) != cudaSuccess)
-    return e;
-  if ((e = cudaFuncSetAttribute(k_p2<LOGN, false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                (int)p2_smem<LOGN, false>())) != cudaSuccess)
-    return e;
-  return cudaFuncSetAttribute(k_p3<LOGN>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)p3_smem<LOGN>());
+  if ((e = set_smem(k_p1<unsigned long long, LOGN>, p1_smem<LOGN>())) != cudaSuccess) return e;
+  if ((e = set_smem(k_p1<float, LOGN>, p1_smem<LOGN>())) != cudaSuccess) return e;
+  if ((e = set_smem(k_p2<LOGN, true>, p2_smem<LOGN>())) != cudaSuccess) return e;
+  if ((e = set_smem(k_p2<LOGN, false>, p2_smem<LOGN, false>())) != cudaSuccess) return e;
+  return set_smem(k_p3<LOGN>, p3_smem<LOGN>());
 }
 
 template <int LOGN>
@@ -392,6 +445,8 @@ FieldArgs field_args(const Ctx &c, const void *rho) {
   a.my = c.my;
   a.R = c.mx;
   a.C = c.my;
+  a.lR = c.log2mx;
+  a.lC = c.log2my;
   a.x_base = a.y_base = 0;
   a.nrows = c.mx;
   a.ncols = c.my;
@@ -412,6 +467,8 @@ FieldArgs shard_args(const Ctx &c, const void *rho, int r, int G, float *s1, con
   FieldArgs a = field_args(c, rho);
   a.R = c.mx / G;
   a.C = c.my / G;
+  a.lR = ilog2_int(a.R);
+  a.lC = ilog2_int(a.C);
   a.x_base = r * a.R;
   a.y_base = r * a.C;
   a.nrows = a.R;
@@ -447,7 +504,7 @@ void launch_p2_rowmajor(const Ctx &c, cudaStream_t s) {
 }
 
 bool fields_shardable(const Ctx &c, int G) {
-  if (!c.fft_cta || G < 1 || c.mx % G || c.my % G) return false;
+  if (!c.fft_cta || G < 1 || (G & (G - 1)) || c.mx % G || c.my % G) return false;   // R, C powers of two
   const int R = c.mx / G, C = c.my / G;
   // every P1 / P2 CTA lies inside one rank block: rows by 2 SEQ_y, columns by 2 SEQ_x
   return R % (2 * cfft::seq_per_cta(c.log2my)) == 0 && C % (2 * cfft::seq_per_cta(c.log2mx)) == 0;

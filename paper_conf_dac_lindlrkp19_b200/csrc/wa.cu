@@ -60,7 +60,8 @@ struct WaArgs {
   // big nets
   const int32_t *big_start, *big_flags, *big_cell;
   const float *big_w, *big_dx, *big_dy;
-  int part_base;                // global WA unit of this launch's CTA 0: CTA b writes part[part_base + b]
+  int part_base;                // global WA unit of this context's unit 0: unit u writes part[part_base + u]
+  int unit0;                    // unit of this launch's CTA 0 (a split WA launch: CTA b runs unit unit0 + b)
   int hp_offset;                // MODE 4: fast-HPWL partials at part[hp_offset + the WA partial's index]
   int big_stage;   // pins staged in shared memory per big-net CTA
   int n_huge, n_big, n_warp_blocks;
@@ -731,7 +732,7 @@ __device__ __forceinline__ void wa_big_net(const WaArgs &a, int net, float4 *s_p
     }
   }
   __syncthreads();
-  const int slot = a.part_base + blockIdx.x;
+  const int slot = a.part_base + a.unit0 + blockIdx.x;
   block_flush_scalars<kBigThreads>(wl_acc, L, kHpwl, kGrad ? a.part + slot : nullptr, a.limbs, hp_b,
                                    MODE == 4 ? a.part + a.hp_offset + slot : nullptr);
 }
@@ -891,7 +892,7 @@ __device__ __forceinline__ void wa_warp_nets(const WaArgs &a, int wb) {
       }
     }
   }
-  const int slot = a.part_base + blockIdx.x;
+  const int slot = a.part_base + a.unit0 + blockIdx.x;
   block_flush_scalars<kWarpNetThreads>(wl_acc, L, kHpwl, kGrad ? a.part + slot : nullptr, a.limbs, hp_w,
                                        MODE == 4 ? a.part + a.hp_offset + slot : nullptr);
 }
@@ -928,15 +929,16 @@ __global__ void __launch_bounds__(kWaThreads, 2) k_wa_chunks(const WaArgs a0) {
   // one launch for all nets: CTAs [0, n_huge) take a net of degree > kWarpNetMax each, the next
   // n_warp_blocks CTAs 8 nets of degree (kWaMaxDeg, kWarpNetMax] each (a warp per net), the rest
   // the staged chunks; the long big-net CTAs are dispatched first and overlap the chunks.
-  if ((int)blockIdx.x < a.n_huge) {
-    wa_big_net<MODE>(a, blockIdx.x, reinterpret_cast<float4 *>(smem));
+  const int unit = a.unit0 + blockIdx.x;
+  if (unit < a.n_huge) {
+    wa_big_net<MODE>(a, unit, reinterpret_cast<float4 *>(smem));
     return;
   }
-  if ((int)blockIdx.x < a.n_huge + a.n_warp_blocks) {
-    wa_warp_nets<MODE>(a, blockIdx.x - a.n_huge);
+  if (unit < a.n_huge + a.n_warp_blocks) {
+    wa_warp_nets<MODE>(a, unit - a.n_huge);
     return;
   }
-  const int chunk = blockIdx.x - a.n_huge - a.n_warp_blocks;
+  const int chunk = unit - a.n_huge - a.n_warp_blocks;
   const Chunk ch = a.chunks[chunk];
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   // window positions by bulk copy when 16-byte aligned (the caller's x / y), else by threads
@@ -1087,15 +1089,21 @@ __global__ void __launch_bounds__(kWaThreads, 2) k_wa_chunks(const WaArgs a0) {
       if (gx | gy) red_v2(a.g2 + s_far[f], gx * inv, gy * inv);
     }
   }
-  block_flush_scalars<kWaThreads>((double)wl_acc, L, kHpwl, kGrad ? a.part + a.part_base + blockIdx.x : nullptr,
+  block_flush_scalars<kWaThreads>((double)wl_acc, L, kHpwl, kGrad ? a.part + a.part_base + unit : nullptr,
                                   a.limbs, (double)hp_acc,
-                                  MODE == 4 ? a.part + a.hp_offset + a.part_base + blockIdx.x : nullptr);
+                                  MODE == 4 ? a.part + a.hp_offset + a.part_base + unit : nullptr);
 }
 
 template <int MODE>
-void launch_mode(const Ctx &c, const WaArgs &a, cudaStream_t s) {
-  const WaSmem L{a.caps};
-  const int grid = c.n_chunks + a.n_huge + a.n_warp_blocks;
+void launch_mode(const Ctx &c, const WaArgs &a0, cudaStream_t s, int part) {
+  const WaSmem L{a0.caps};
+  const int units = c.n_chunks + a0.n_huge + a0.n_warp_blocks;
+  // part 0: every unit; part 1 / 2: units [0, U_A) / [U_A, units) of a split launch (the big
+  // units, then the first chunks, in part 1)
+  const int ua = std::min(units, a0.n_huge + a0.n_warp_blocks + c.wa_split_chunks);
+  WaArgs a = a0;
+  a.unit0 = part == 2 ? ua : 0;
+  const int grid = part == 0 ? units : part == 1 ? ua : units - ua;
   int bytes = L.bytes();
   // DP_WA_CTAS_PER_SM = k (measurement knob): pad the dynamic shared memory so that at most k
   // WA CTAs are resident per SM, leaving room for the concurrently running density kernels
@@ -1122,8 +1130,9 @@ cudaError_t wa_configure(const WaCaps &caps) {
 }
 
 void launch_wa(const Ctx &c, const float *x, const float *y, float gamma, bool hpwl_only, bool with_hpwl,
-               cudaStream_t s) {
+               cudaStream_t s, int part) {
   WaArgs a;
+  a.unit0 = 0;
   a.chunks = c.d_chunks;
   a.wgs = c.d_wgroups;
   a.net_deg = c.d_net_deg;
@@ -1162,16 +1171,16 @@ void launch_wa(const Ctx &c, const float *x, const float *y, float gamma, bool h
   a.big_stage = std::min(c.big_stage, wa_smem_bytes(c.wa_caps) / 16);
   a.caps = c.wa_caps;
   if (hpwl_only) {
-    launch_mode<2>(c, a, s);
+    launch_mode<2>(c, a, s, part);
   } else if (c.wl_model == DP_WL_LSE) {   // LSE: fast path; a fused HPWL is a second, HPWL-only pass
-    launch_mode<3>(c, a, s);
-    if (with_hpwl) launch_mode<2>(c, a, s);
+    launch_mode<3>(c, a, s, part);
+    if (with_hpwl) launch_mode<2>(c, a, s, part);
   } else if (with_hpwl && c.hpwl_fast && c.wl_model == DP_WL_WA) {   // GP loop: fast HPWL in the fast path
-    launch_mode<4>(c, a, s);
+    launch_mode<4>(c, a, s, part);
   } else if (with_hpwl) {
-    launch_mode<1>(c, a, s);
+    launch_mode<1>(c, a, s, part);
   } else {
-    launch_mode<0>(c, a, s);
+    launch_mode<0>(c, a, s, part);
   }
 }
 

@@ -76,12 +76,13 @@ def test_fields_tiny(tiny):
     check_scalar("energy", f["energy"].item(), oracle.energy(nl, rho32, psi))
 
 
-@pytest.mark.parametrize("mx,my", [(16, 16), (32, 32), (128, 128), (512, 512), (1024, 1024), (32, 128),
-                                   (256, 64), (2048, 2048)])
+@pytest.mark.parametrize("mx,my", [(16, 16), (32, 32), (64, 64), (128, 128), (256, 256), (512, 512), (1024, 1024),
+                                   (32, 128), (256, 64), (64, 1024), (2048, 2048)])
 def test_fields_sizes(mx, my):
     """The three CTA-FFT passes (P1 rows, P2 columns + energy, P3 rows; fields.cu) on random maps
-    of every radix plan (16 = 2 x 8, 32 = 4 x 8, 128 = 2 x 8 x 8, 512 = 8^3, 1024 = 2 x 8^3,
-    2048 = 4 x 8^3), square and rectangular, against eqs 9a-9d via the naive eq 7a/7b/8a."""
+    of every radix plan of the radix-16 core (16, 32 = 16 x 2, 64 = 16 x 4, 128 = 16 x 8,
+    256 = 16^2, 512 = 16^2 x 2, 1024 = 16^2 x 4, 2048 = 16^2 x 8), square and rectangular, against
+    eqs 9a-9d via the naive eq 7a/7b/8a."""
     W, H = 10.0 * mx, 7.0 * my
     nl = custom_netlist([0], [], [], [], [1.0], [1.0], (0, 0, W, H), (mx, my))
     ctx = dp.dp_create(nl)

@@ -523,7 +523,6 @@ __global__ void __launch_bounds__(kTileThreads) k_scatter_walk(DenArgs a) {
       __syncthreads();   // flushed and cleared
       cur_tile = cc.tile;
     }
-    const size_t ox = (size_t)(cur_tile / a.tiles_y) * a.tile, oy = (size_t)(cur_tile % a.tiles_y) * a.tile;
     const RecBuf &B = st.buf[b];
     for (int k = threadIdx.x; k < n; k += blockDim.x) {
       const float4 q = B.rec[cc.off + k];
@@ -533,6 +532,7 @@ __global__ void __launch_bounds__(kTileThreads) k_scatter_walk(DenArgs a) {
       float ox3[3], oy3[3];
       rec_overlaps(q, ox3, oy3);
       const int base = i0 * P + j0;
+      unsigned wrapped = 0u;   // bit 3 di + dj: that word's add wrapped past 2^32
 #pragma unroll
       for (int di = 0; di < 3; di++) {
         const float rx = r * ox3[di];
@@ -540,10 +540,20 @@ __global__ void __launch_bounds__(kTileThreads) k_scatter_walk(DenArgs a) {
         for (int dj = 0; dj < 3; dj++) {
           const unsigned u = (unsigned)(rx * oy3[dj]);   // floor(v 2^29) <= 2^29 (power-of-two scaling is exact)
           const unsigned old = atom_shared_add(s_acc + base + di * P + dj, u);
-          if (old + u < old)   // wrapped: 2^32 units (8 bin areas) go straight to the map
-            asm volatile("red.global.add.u64 [%0], %1;" ::"l"(a.rho + (ox + i0 + di) * a.my + oy + j0 + dj),
-                         "l"(1ull << 32)
-                         : "memory");
+          wrapped |= (old + u < old ? 1u : 0u) << (3 * di + dj);
+        }
+      }
+      // wrapped words (rare): 2^32 units (8 bin areas) each go straight to the map.  Collected as a
+      // mask so that the map addresses are formed only here (as predicated reductions inside the
+      // loop, they were computed for all nine bins of every record)
+      if (wrapped) {
+        const size_t ox = (size_t)(cur_tile / a.tiles_y) * a.tile + i0, oy = (size_t)(cur_tile % a.tiles_y) * a.tile + j0;
+        while (wrapped) {
+          const int bit = __ffs(wrapped) - 1;
+          wrapped &= wrapped - 1;
+          asm volatile("red.global.add.u64 [%0], %1;" ::"l"(a.rho + (ox + bit / 3) * a.my + oy + bit % 3),
+                       "l"(1ull << 32)
+                       : "memory");
         }
       }
     }

@@ -168,8 +168,11 @@ __global__ void __launch_bounds__(cfft::seq_per_cta(LOGN) * cfft::threads_per_se
 template <int LOGM, bool TIN>
 constexpr int p2_seq() { return TIN ? cfft::seq_per_cta(LOGM) : 1; }
 
+// at most 128 registers for a 128-thread CTA (min 4 CTAs / SM by registers): the column pass
+// then fits beside two WA CTAs in the overlapped evaluation (their 2 x 256 x 92 registers)
 template <int LOGM, bool TIN>
-__global__ void __launch_bounds__(p2_seq<LOGM, TIN>() * cfft::threads_per_seq(LOGM))
+__global__ void __launch_bounds__(p2_seq<LOGM, TIN>() * cfft::threads_per_seq(LOGM),
+                                  p2_seq<LOGM, TIN>() * cfft::threads_per_seq(LOGM) <= 128 ? 4 : 1)
     k_p2(FieldArgs a) {
   griddep_wait();
   constexpr int M = 1 << LOGM, T = cfft::threads_per_seq(LOGM), SEQ = p2_seq<LOGM, TIN>();

@@ -21,7 +21,7 @@ NVCC_FLAGS = [
     "-Xcompiler", "-fPIC",
     "-Xptxas", "-v",
     "--expt-relaxed-constexpr",
-]
+] + os.environ.get("DP_NVCC_EXTRA", "").split()   # A/B builds only (e.g. -DDP_WA_PPL=8)
 
 
 def sources() -> list[str]:

@@ -294,6 +294,44 @@ def test_eval_full_size(name):
     check_vector("gy", to_np(out["gy"]), ref["gy"])
 
 
+@pytest.mark.parametrize("env", [{"DP_WA_SPLIT": "50"}, {"DP_FFT": "2"}, {"DP_FFT": "1"}])
+def test_schedule_switches_match(env):
+    """The measured-and-off A/B switches of the evaluation schedule compute the
+    same evaluation: the WA launch split around the transforms (the same work units and partial
+    slots in two launches), the hybrid and the CTA-FFT field paths at 512^2 — against the default
+    context (WA / D / HPWL / gradient) and the oracle."""
+    import os
+    nl = make_netlist("adaptec1")
+    x, y = make_positions(nl)
+    xt, yt = _t(x), _t(y)
+    base = dp.dp_create(nl)
+    a = base.eval(xt, yt, nl.bin_w, 1.0, with_hpwl=True)
+    a = {k: (v.clone() if torch.is_tensor(v) else v) for k, v in a.items()}
+    old = {k: os.environ.get(k) for k in env}
+    os.environ.update(env)
+    try:
+        ctx = dp.dp_create(nl)
+    finally:
+        for k, v in old.items():
+            if v is None:
+                del os.environ[k]
+            else:
+                os.environ[k] = v
+    b = ctx.eval(xt, yt, nl.bin_w, 1.0, with_hpwl=True)
+    torch.cuda.synchronize()
+    assert b["hpwl"].item() == a["hpwl"].item()
+    if "DP_WA_SPLIT" in env:   # same field path: D bit-identical; WA partial slots identical
+        assert b["energy"].item() == a["energy"].item()
+        assert b["wl"].item() == a["wl"].item()
+    check_scalar("WA", b["wl"].item(), a["wl"].item())
+    check_scalar("D", b["energy"].item(), a["energy"].item())
+    check_vector("gx", to_np(b["gx"]), to_np(a["gx"]))
+    check_vector("gy", to_np(b["gy"]), to_np(a["gy"]))
+    ref = oracle.evaluate(nl, x, y, nl.bin_w, 1.0)
+    check_scalar("D (oracle)", b["energy"].item(), ref["energy"])
+    check_vector("gx (oracle)", to_np(b["gx"]), ref["gx"])
+
+
 @pytest.mark.slow
 @pytest.mark.parametrize("name", ["adaptec1", "bigblue4"])
 def test_initial_full_size(name):

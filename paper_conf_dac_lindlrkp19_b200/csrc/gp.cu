@@ -519,7 +519,9 @@ dp_status dp_gp_create(dp_ctx *ctx, const dp_gp_params *params, dp_gp **out) {
   a.nbins = (long long)c->mx * c->my;
   a.rho_unit = std::ldexp(1.0, -dp::kRhoScaleLog2);
   a.target = p.target_density;
-  a.nblk = c->num_sms * 2;
+  // post-pass grid: 8 CTAs per SM for the cells (each thread a few cells, 11 loads each in flight;
+  // 2 per SM left it latency-bound at 58 us for bigblue4), 4 per SM for the bins
+  a.nblk = std::max(1, std::min(c->num_sms * 8, (n + dp::kGpThreads - 1) / dp::kGpThreads));
   a.bxby = c->bx * c->by;
   a.mu_min = p.mu_min; a.mu_max = p.mu_max; a.dhpwl_ref = p.dhpwl_ref;
   a.lambda_scale = p.lambda_scale; a.init_rms_bins = p.init_rms_bins; a.bx = c->bx;
@@ -527,7 +529,7 @@ dp_status dp_gp_create(dp_ctx *ctx, const dp_gp_params *params, dp_gp **out) {
   a.stop_overflow = p.stop_overflow;
   dp_status st;
   if ((st = dp::gp_alloc(*g, &a.part, 2 * (size_t)a.nblk)) != DP_OK) return bail(st);
-  a.oblk = c->num_sms;
+  a.oblk = (int)std::max<long long>(1, std::min<long long>(c->num_sms * 4, (a.nbins + dp::kGpThreads - 1) / dp::kGpThreads));
   if ((st = dp::gp_alloc(*g, &a.part_ovf, 2 * (size_t)a.oblk)) != DP_OK) return bail(st);
   if ((st = dp::gp_alloc(*g, &g->dev, 1)) != DP_OK) return bail(st);
   if ((st = dp::gp_alloc(*g, &g->out, 4)) != DP_OK) return bail(st);

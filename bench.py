@@ -7,12 +7,13 @@ force gather, combine) on the bigblue4-shaped synthetic workload (2.18M cells, 2
 
     python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference] [--config NAME]
 
-N > 1 is launched by torchrun (one rank per GPU, NCCL): the evaluation is sharded by cells
-(owner computes) with one ncclAllReduce of the bin map per step, so the total
-work per step is fixed ("scaling": "strong").  Device time: one CUDA event pair around the K
-timed steps on the launching stream (barrier + synchronize on both sides), max over ranks; the
-per-step working set (~280 MB) exceeds L2, so no flush is inserted (the contract's "inputs larger
-than L2"); an L2-flushed per-step time is reported beside it.
+The positions move from step to step along a GP-like random walk: the density
+scatter keeps its tile-ordered cell list between evaluations, so a benchmark at fixed positions
+would never pay for a re-sort.  Each timed step evaluates the next position set of the walk
+(copied into the input buffers and followed by a 2x-L2 write, both untimed); one CUDA event
+pair per step on the launching stream, barrier + synchronize on both sides, max over ranks.
+N > 1 is launched by torchrun (one rank per GPU, NCCL): nets are partitioned for WA (gradient
+reduce-scatter), cells for the density map (int64 map all-reduce), DESIGN.md §6.
 Rank 0 prints one JSON line.  --impl reference times the fp64 CPU oracle (the reference arm of
 this tier) on a bounded sample of the same workload.
 """
@@ -45,6 +46,8 @@ def parse():
     ap.add_argument("--dist", default="spread", choices=["spread", "initial"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=200)
+    ap.add_argument("--walk-sigma", type=float, default=0.13,
+                    help="random-walk step per axis in bins (GP-like motion, DESIGN.md §7); 0 = fixed positions")
     ap.add_argument("--skip-next", action="store_true",
                     help="skip the NEXT-row secondaries (LSE, deterministic, GP loop): profiling runs")
     return ap.parse_args()
@@ -282,6 +285,42 @@ def run_ours(args, rank, world, local_rank):
     def step(st=None):
         dp.dp_eval(ctx, xt, yt, gamma, lam, gx, gy, sc[0:1], sc[1:2], sc[2:3], None, st or stream)
 
+    # the GP-like trajectory: R position sets on the device, a seeded random walk of walk_sigma bins
+    # per axis and step from the start positions (clamped to the region), visited in ping-pong
+    # order so that consecutive steps always differ by one walk step
+    K = args.steps
+
+    class Walk:
+        def __init__(self, x0, y0, n_sets, seed):
+            self.n = max(2, n_sets)
+            g = torch.Generator(device=dev)
+            g.manual_seed(seed)
+            w = torch.as_tensor(nl.cell_w, device=dev)
+            h = torch.as_tensor(nl.cell_h, device=dev)
+            self.xs = torch.empty((self.n, nl.num_cells), dtype=torch.float32, device=dev)
+            self.ys = torch.empty_like(self.xs)
+            self.xs[0] = torch.as_tensor(x0, device=dev)
+            self.ys[0] = torch.as_tensor(y0, device=dev)
+            sx, sy = args.walk_sigma * nl.bin_w, args.walk_sigma * nl.bin_h
+            for k in range(1, self.n):
+                nx = self.xs[k - 1] + sx * torch.randn(nl.num_cells, device=dev, generator=g)
+                ny = self.ys[k - 1] + sy * torch.randn(nl.num_cells, device=dev, generator=g)
+                self.xs[k] = torch.minimum(torch.clamp(nx, min=nl.xl), nl.xh - w)
+                self.ys[k] = torch.minimum(torch.clamp(ny, min=nl.yl), nl.yh - h)
+            self.i = 0
+
+        def index(self, i):
+            p = i % (2 * self.n - 2)
+            return p if p < self.n else 2 * self.n - 2 - p
+
+        def load(self, tx, ty):   # the next position set into the input buffers (untimed in the headline)
+            k = self.index(self.i) if args.walk_sigma > 0 else 0
+            tx.copy_(self.xs[k])
+            ty.copy_(self.ys[k])
+            self.i += 1
+
+    walk = Walk(x, y, min(K + max(args.warmup, 3), 256) if args.walk_sigma > 0 else 1, 3000 + world)
+
     def timed(fn, n):   # mean device ms of n back-to-back calls (one event pair)
         a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         a.record(stream)
@@ -294,13 +333,13 @@ def run_ours(args, rank, world, local_rank):
     sampler = ClockSampler(gpu_uuid(local_rank))
     sampler.start()
     for _ in range(max(args.warmup, 3)):
+        walk.load(xt, yt)
         flush.zero_()
         step()
     torch.cuda.synchronize()
     if pg:
         pg.barrier()
     assert all(math.isfinite(v) for v in sc[:3].tolist()), "non-finite objective"
-    K = args.steps
 
     def load_for(seconds):   # untimed steps that keep the GPU busy around the timed region
         t = time.time()
@@ -309,9 +348,12 @@ def run_ours(args, rank, world, local_rank):
                 step()
             torch.cuda.synchronize()
 
-    def cold_steps(n, fn):   # per-step device ms, each step after an untimed write of 2x L2
+    def cold_steps(n, fn, wk=None, tx=None, ty=None):
+        """per-step device ms; before each step (untimed) the next walk positions and a 2x-L2 write"""
         evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(n)]
         for k in range(n):
+            if wk is not None:
+                wk.load(tx, ty)
             flush.zero_()
             evs[k][0].record(stream)
             fn()
@@ -319,18 +361,21 @@ def run_ours(args, rank, world, local_rank):
         torch.cuda.synchronize()
         return [a.elapsed_time(b) for a, b in evs]
 
-    # headline (L2-cold): K steps, each preceded by an untimed 2x-L2 write, timed by
-    # one event pair per step on the launching stream; barrier + synchronize on both sides.  The
-    # clock sampler has started and the GPU is kept under load for 0.3 s on either side, so the
-    # nvidia-smi samples bracketing the (milliseconds-long) timed region are taken under load.
+    # headline (L2-cold): K steps along the walk, each preceded by the untimed load of
+    # its positions and a 2x-L2 write, timed by one event pair per step on the launching stream;
+    # barrier + synchronize on both sides.  The clock sampler has started and the GPU is kept under
+    # load for 0.3 s on either side, so the nvidia-smi samples bracketing the (short) timed region
+    # are taken under load.
     sampler.wait_first()
     load_for(0.3)
     torch.cuda.synchronize()
     if pg:
         pg.barrier()
+    sorts0 = dp.dp_debug_sort_stats(ctx)["sorts"]
     t0 = time.time()
-    cold = cold_steps(K, step)
+    cold = cold_steps(K, step, walk, xt, yt)
     t1 = time.time()
+    sorts_timed = dp.dp_debug_sort_stats(ctx)["sorts"] - sorts0
     load_for(0.3)
     if pg:
         pg.barrier()
@@ -338,50 +383,73 @@ def run_ours(args, rank, world, local_rank):
     flushed_pct = np.percentile([v * 1e3 for v in cold], [10, 50, 90]).tolist()
     flushed_ms = total_ms / K
     clocks = sampler.summary(t0 - 0.3, t1 + 0.3)
-    # secondary: the same steps back to back without the flush (hot L2: the Nesterov steady state)
+    # secondary: the same walk back to back without the flush (hot L2: the Nesterov steady state);
+    # the position copies are timed alone and subtracted
     torch.cuda.synchronize()
-    h0, h1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    h0.record(stream)
-    for _ in range(K):
+    copy_ms = timed(lambda: walk.load(xt, yt), min(K, 200))
+
+    def walk_step():
+        walk.load(xt, yt)
         step()
-    h1.record(stream)
-    torch.cuda.synchronize()
-    hot_ms = h0.elapsed_time(h1) / K
-    # secondary: the 'initial' distribution (all cells near the centre: worst-case contention)
-    xi0, yi0 = make_positions(nl, "initial")
-    xit, yit = torch.as_tensor(xi0, device=dev), torch.as_tensor(yi0, device=dev)
-    Ki = min(K, 200)
 
-    def step_initial():
-        dp.dp_eval(ctx, xit, yit, gamma, lam, gx, gy, sc[0:1], sc[1:2], sc[2:3], None, stream)
-
-    for _ in range(3):
-        step_initial()
-    initial_ms = sum(cold_steps(Ki, step_initial)) / Ki
+    hot_ms = timed(walk_step, K) - copy_ms
+    # secondary: the same walk from the fixed positions only (no motion: the list is never re-sorted)
+    xt.copy_(walk.xs[0])
+    yt.copy_(walk.ys[0])
     step()
-    # profiled timed region: the same K steps again with per-stage CUDA events recorded by the
+    fixed_ms = sum(cold_steps(min(K, 200), step)) / min(K, 200)
+    # secondary: sorting on every evaluation (DP_REUSE_SORT=0 context), the same walk, L2-cold
+    sort_every_ms = None
+    if world == 1:
+        os.environ["DP_REUSE_SORT"] = "0"
+        try:
+            ctx_s = dp.dp_create(nl, local_rank)
+        finally:
+            del os.environ["DP_REUSE_SORT"]
+
+        def step_s():
+            dp.dp_eval(ctx_s, xt, yt, gamma, lam, gx, gy, sc[0:1], sc[1:2], sc[2:3], None, stream)
+
+        for _ in range(3):
+            step_s()
+        Ks2 = min(K, 200)
+        walk.i = 0
+        sort_every_ms = sum(cold_steps(Ks2, step_s, walk, xt, yt)) / Ks2
+        del ctx_s
+        torch.cuda.synchronize()
+    # secondary: the 'initial' distribution (all cells near the centre: worst-case
+    # contention), walking from there like the headline
+    xi0, yi0 = make_positions(nl, "initial")
+    Ki = min(K, 200)
+    walk_i = Walk(xi0, yi0, min(Ki + 3, 64) if args.walk_sigma > 0 else 1, 4000 + world)
+    for _ in range(3):
+        walk_i.load(xt, yt)
+        step()
+    initial_ms = sum(cold_steps(Ki, step, walk_i, xt, yt)) / Ki
+    del walk_i
+    # profiled timed region: the same walk again with per-stage CUDA events recorded by the
     # library on the stream each stage runs on (dp_profile_*); stage durations and the roofline
     # come from here (the events add a little host/GPU work, so the headline above runs without)
+    walk.i = 0
+    walk.load(xt, yt)
+    step()
     dp.dp_profile_enable(ctx, True)
     torch.cuda.synchronize()
-    p0, p1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    p0.record(stream)
-    for _ in range(K):
-        step()
-    p1.record(stream)
-    torch.cuda.synchronize()
+    profiled_ms = timed(walk_step, K) - copy_ms
     dp.dp_profile_enable(ctx, False)
     stage_ms, n_prof = dp.dp_profile_read(ctx)
-    profiled_ms = p0.elapsed_time(p1) / K
     Kf = min(K, 200)
     ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(Kf)]
     # per-call distribution without the flush (median and p10 / p90 of single calls)
     for k in range(Kf):
+        walk.load(xt, yt)
         ev[k][0].record(stream)
         step()
         ev[k][1].record(stream)
     torch.cuda.synchronize()
     hot_pct = np.percentile([a.elapsed_time(b) * 1e3 for a, b in ev], [10, 50, 90]).tolist()
+    xt.copy_(walk.xs[0])
+    yt.copy_(walk.ys[0])
     # secondary numbers: fused-HPWL evaluation, standalone HPWL, CUDA-graph
     # replay of one evaluation, and the WA stage timed alone (no overlap with the density chain)
     Ks = min(K, 200)
@@ -407,7 +475,7 @@ def run_ours(args, rank, world, local_rank):
     dp.dp_profile_enable(ctx, False)
     iso_ms, n_iso = dp.dp_profile_read(ctx)
     wa_iso_ms = iso_ms["wa"] / max(n_iso, 1)
-    lse_ms = det_ms = fixed_ms = float("nan")
+    lse_ms = det_ms = fixedm_ms = float("nan")
     if not args.skip_next:
         # NEXT-3: the same evaluation with the LSE wirelength model
         dp.dp_set_wl_model(ctx, dp.DP_WL_LSE)
@@ -427,7 +495,7 @@ def run_ours(args, rank, world, local_rank):
             big = (nl.cell_w > 2 * nl.bin_w) | (nl.cell_h > 2 * nl.bin_h)
             dp.dp_set_fixed(ctx, big, xt, yt, stream)
             step()
-            fixed_ms = timed(step, Ks)
+            fixedm_ms = timed(step, Ks)
             dp.dp_set_fixed(ctx, None, stream=stream)
             step()
     # NEXT-1: GP iterations (Nesterov step + evaluation + schedule, one graph per iteration)
@@ -445,20 +513,29 @@ def run_ours(args, rank, world, local_rank):
                     "last": {k: hist[-1][k] for k in ("hpwl", "overflow", "lam", "gamma")} if hist else None,
                     "start": "initial (P:153)"}
         loop.close()
-    # e2e through the public API on pinned host buffers (H2D x, y; D2H gx, gy, scalars)
-    hx = torch.as_tensor(x).pin_memory()
-    hy = torch.as_tensor(y).pin_memory()
+    # e2e through the public API on pinned host buffers (H2D x, y; D2H gx, gy, scalars), the
+    # positions walking over the first 8 sets of the walk (ping-pong)
+    nh = min(8, walk.n)
+    hxs = [walk.xs[k].cpu().pin_memory() for k in range(nh)]
+    hys = [walk.ys[k].cpu().pin_memory() for k in range(nh)]
     hgx = torch.empty(nl.num_cells, dtype=torch.float32).pin_memory()
     hgy = torch.empty_like(hgx).pin_memory()
     hsc = np.zeros(4)
     Ke = max(1, min(args.e2e_steps, K))
-    for _ in range(3):
-        dp.dp_eval_host(ctx, hx, hy, gamma, lam, hgx, hgy, hsc, False, stream)
+
+    def hidx(i):
+        if nh == 1:
+            return 0
+        p = i % (2 * nh - 2)
+        return p if p < nh else 2 * nh - 2 - p
+
+    for i in range(3):
+        dp.dp_eval_host(ctx, hxs[hidx(i)], hys[hidx(i)], gamma, lam, hgx, hgy, hsc, False, stream)
     if pg:
         pg.barrier()
     e0 = time.perf_counter()
-    for _ in range(Ke):
-        dp.dp_eval_host(ctx, hx, hy, gamma, lam, hgx, hgy, hsc, False, stream)
+    for i in range(Ke):
+        dp.dp_eval_host(ctx, hxs[hidx(i + 3)], hys[hidx(i + 3)], gamma, lam, hgx, hgy, hsc, False, stream)
     e2e_s = time.perf_counter() - e0
     sampler.stop()
 
@@ -467,15 +544,20 @@ def run_ours(args, rank, world, local_rank):
         pg.all_reduce(tensors, op=pg.ReduceOp.MAX)
     total_ms, e2e_s, hot_ms = tensors.tolist()
     secondary = {"hot_back_to_back_evals_per_s": 1e3 / hot_ms, "hot_ms_per_step": hot_ms,
+                 "hot_note": "the same walk back to back, position copies timed alone and subtracted",
+                 "fixed_positions_evals_per_s": 1e3 / fixed_ms,
+                 "fixed_positions_note": "the walk's first positions every step, L2-cold: the list is never re-sorted",
+                 "sort_every_eval_evals_per_s": (1e3 / sort_every_ms) if sort_every_ms else None,
+                 "sort_every_eval_note": "DP_REUSE_SORT=0 context (count/scan/place sort on every evaluation), same walk, L2-cold",
                  "initial_evals_per_s": 1e3 / initial_ms, "initial_ms_per_step": initial_ms,
-                 "initial_note": "positions 'initial' (P:153): centres ~ N(W/2, (0.001 W)^2), L2-cold like the headline",
+                 "initial_note": "walk from the 'initial' placement (P:153): centres ~ N(W/2, (0.001 W)^2), L2-cold like the headline",
                  "fused_hpwl_evals_per_s": 1e3 / fused_ms, "hpwl_only_per_s": 1e3 / hpwl_ms,
                  "wl_grad_only_per_s": 1e3 / wl_only_ms,
                  "profiled_ms_per_step": profiled_ms,
                  "graph_replay_evals_per_s": (1e3 / graph_ms) if isinstance(graph_ms, float) else graph_ms,
                  "lse_evals_per_s": None if args.skip_next else 1e3 / lse_ms,
                  "deterministic_evals_per_s": None if args.skip_next else 1e3 / det_ms,
-                 "fixed_macros_evals_per_s": None if (args.skip_next or world > 1) else 1e3 / fixed_ms, "gp": gp_stats,
+                 "fixed_macros_evals_per_s": None if (args.skip_next or world > 1) else 1e3 / fixedm_ms, "gp": gp_stats,
                  "note": "rank-0 device time of min(K, 200) back-to-back calls each; not the headline"}
     if rank != 0:
         if pg:
@@ -496,6 +578,14 @@ def run_ours(args, rank, world, local_rank):
         except Exception:
             traffic = None
     cfg = workload_config(nl, args.dist, world)
+    cfg["trajectory"] = {
+        "start": args.dist, "step_sigma_bins_per_axis": args.walk_sigma, "position_sets": walk.n,
+        "order": "ping-pong over the sets (consecutive steps differ by one walk step)",
+        "source": "median per-iteration GP move measured on B200 (tools/gp_motion.py: adaptec1 0.18 bins rms, "
+                  "bigblue4 0.07): the larger one",
+        "sorts_in_timed_region": sorts_timed,
+        "note": "the density sort's list is kept while cells stay within their tile's margin (DESIGN.md §5.2); "
+                "a step re-sorts when the previous one saw > 5 % strays"}
     cfg["hot_ms_per_step"] = hot_ms
     cfg["per_call_us"] = {"hot": dict(zip(("p10", "p50", "p90"), hot_pct)),
                           "l2_flushed": dict(zip(("p10", "p50", "p90"), flushed_pct)),

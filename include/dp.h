@@ -344,6 +344,17 @@ dp_status dp_debug_sharded_fields(dp_ctx *ctx, int32_t world, const float *rho, 
  * reduce-scatter).  *n_out <- n.  Synchronises the stream.                                  */
 dp_status dp_debug_wa_accumulator(dp_ctx *ctx, void *out, int64_t *n_out, dp_stream_t stream);
 
+/* Sort-reuse counters (test / bench hook).  The density scatter keeps the
+ * tile-ordered list of small cells between evaluations and rebuilds it (the count / scan /
+ * place sort) only when a configuration change requests it or when more than DP_RESORT_PCT
+ * percent (environment, read at dp_create; default 5) of the small cells were outside the tile
+ * they are listed in during the previous evaluation; such "strays" are scattered and gathered
+ * through the global map / field with the same arithmetic, so results do not depend on the list
+ * (DP_REUSE_SORT=0: sort on every evaluation).  out (host, int32[4]) <- {sort requested, strays
+ * of the last completed evaluation, strays accumulated by a scatter not yet gathered, sorts
+ * performed since dp_create}.  Synchronises the context's work.                              */
+dp_status dp_debug_sort_stats(dp_ctx *ctx, int32_t *out);
+
 #ifdef __cplusplus
 }
 #endif

@@ -23,7 +23,7 @@ __all__ = [
     "dp_get_info", "dp_debug_density_map", "dp_debug_fields", "dp_debug_transform", "dp_debug_wa_accumulator",
     "dp_debug_sharded_fields", "DP_T_DCT2", "DP_T_IDCT2", "DP_T_IDXST_IDCT", "DP_T_IDCT_IDXST", "EXPORTED_SYMBOLS",
     "dp_set_wl_model", "DP_WL_WA", "DP_WL_LSE", "GpParams", "GpLoop", "dp_gp_create", "dp_set_deterministic",
-    "dp_set_fixed", "dp_set_regions",
+    "dp_set_fixed", "dp_set_regions", "dp_debug_sort_stats",
 ]
 
 DP_T_DCT2, DP_T_IDCT2, DP_T_IDXST_IDCT, DP_T_IDCT_IDXST = 0, 1, 2, 3
@@ -35,7 +35,7 @@ EXPORTED_SYMBOLS = [
     "dp_last_error", "dp_version", "dp_create", "dp_create_dist", "dp_nccl_unique_id",
     "dp_partition_plan", "dp_destroy", "dp_eval", "dp_wl_grad", "dp_density_grad", "dp_hpwl",
     "dp_eval_host", "dp_get_info", "dp_debug_density_map", "dp_debug_fields", "dp_debug_transform",
-    "dp_debug_wa_accumulator", "dp_debug_sharded_fields", "dp_set_regions", "dp_profile_enable", "dp_profile_read", "dp_set_wl_model",
+    "dp_debug_wa_accumulator", "dp_debug_sharded_fields", "dp_debug_sort_stats", "dp_set_regions", "dp_profile_enable", "dp_profile_read", "dp_set_wl_model",
     "dp_gp_default_params", "dp_gp_create", "dp_gp_init", "dp_gp_run", "dp_gp_positions",
     "dp_gp_history", "dp_gp_destroy", "dp_gp_debug_state", "dp_set_deterministic", "dp_set_fixed",
 ]
@@ -111,6 +111,7 @@ def lib() -> ctypes.CDLL:
             "dp_debug_transform": [P, ctypes.c_int, P, P, P],
             "dp_debug_wa_accumulator": [P, P, ctypes.POINTER(ctypes.c_int64), P],
             "dp_debug_sharded_fields": [P, ctypes.c_int32, P, P, P, P, P],
+            "dp_debug_sort_stats": [P, P],
             "dp_set_regions": [P, ctypes.c_int32, P, P],
             "dp_profile_enable": [P, ctypes.c_int],
             "dp_profile_read": [P, P, P],
@@ -507,6 +508,13 @@ def dp_debug_wa_accumulator(ctx, stream=None):
     out = torch.empty((n.value, 2), dtype=torch.int64 if det else torch.float32, device=ctx._dev())
     _check(lib().dp_debug_wa_accumulator(ctx.handle, _ptr(out), ctypes.byref(n), _stream(stream)))
     return out
+
+
+def dp_debug_sort_stats(ctx):
+    """{requested, strays_last, strays_pending, sorts}: the density sort-reuse counters."""
+    out = (I32 * 4)()
+    _check(lib().dp_debug_sort_stats(ctx.handle, out))
+    return dict(requested=out[0], strays_last=out[1], strays_pending=out[2], sorts=out[3])
 
 
 def dp_debug_transform(ctx, kind, inp, out, stream=None):

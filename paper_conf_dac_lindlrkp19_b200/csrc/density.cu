@@ -54,8 +54,14 @@ struct DenArgs {
   int *walk_tile;   // [walk_grid] first tile of each walker's slice (D2)
   int walk_grid;
   float4 *rec;
-  int2 *rec_rc;   // (r as float bits, tile-local first bin i0 | j0 << 16)
-  int *rec_cell;  // own cell index
+  int2 *rec_rc;   // (r as float bits, tile-local first bin i0 | j0 << 16; stray: absolute i0 | j0 << 16 | 1 << 31)
+  int *rec_cell;  // own cell index (the tile-ordered list, kept between sorts)
+  float2 *rec_wh; // (w, h) of the listed cell
+  // sort reuse: [0] re-sort requested, [1] strays of the last evaluation, [2]
+  // strays of this one (scatter), [3] sorts performed.  The sort kernels run when force_sort,
+  // [0] or [1] > resort_thr, and return at once otherwise
+  int *sortctl;
+  int force_sort, resort_thr;
   unsigned long long *rho;   // int64 fixed point, 2^-kRhoScaleLog2 units
   const float2 *xi;
   float2 *force;
@@ -111,31 +117,39 @@ __device__ __forceinline__ Foot footprint(const DenArgs &a, int i) {
   return footprint_v(a, __ldg(a.x + a.cell_begin + i), __ldg(a.y + a.cell_begin + i), __ldg(a.w + i), __ldg(a.h + i));
 }
 
-// Small-cell classification shared by count (D1) and place (D3), which must agree exactly:
-// returns the tile of the footprint's first bin, -1 for an empty footprint, -2 for a large cell
-// (CTA-per-cell path).  Only the lower corner (lx, ly) and the upper corner (hx, hy) are formed
-// in fp64 (unclipped); the predicate equals footprint_v's "empty" (hi > lo after clipping to
-// [0, M], with w h > 0 in place of r > 0: r = 0 only when w h = 0) without fp64 min/max.
+// Small-cell classification shared by count (D1), place (D3) and the scatter walker (D4), which
+// must agree exactly: returns -2 for a large cell (CTA-per-cell path), -3 for a cell of zero
+// area (never in the map), else the tile of the footprint's first bin clamped to the map; f.ok is
+// false for an empty footprint (outside the region: the cell stays listed, in the clamped tile,
+// so that it is found again when it moves back).  Only the lower corner (lx, ly) and the upper
+// corner (hx, hy) are formed in fp64 (unclipped); ok equals footprint_v's "not empty" (hi > lo
+// after clipping to [0, M]) without fp64 min/max.
 struct SmallFoot {
   double lx, ly, hx, hy;
   float ws, hs;
   int bi, bj;
+  bool ok;
 };
 
 __device__ __forceinline__ int classify_small(const DenArgs &a, float x, float y, float w, float h, SmallFoot &f) {
   if (w > a.w_large || h > a.h_large) return -2;
+  if (!(w * h > 0.f)) return -3;
   f.ws = a.stretch ? fmaxf(w, a.sxf) : w;
   f.hs = a.stretch ? fmaxf(h, a.syf) : h;
   f.lx = fma((double)(0.5f * (w - f.ws)), a.ibx, fma((double)x, a.ibx, a.cx0));
   f.ly = fma((double)(0.5f * (h - f.hs)), a.iby, fma((double)y, a.iby, a.cy0));
   f.hx = fma((double)f.ws, a.ibx, f.lx);
   f.hy = fma((double)f.hs, a.iby, f.ly);
-  const bool ok = f.hx > f.lx && f.hx > 0.0 && f.lx < (double)a.mx && f.hy > f.ly && f.hy > 0.0 &&
-                  f.ly < (double)a.my && w * h > 0.f;
-  if (!ok) return -1;
+  f.ok = f.hx > f.lx && f.hx > 0.0 && f.lx < (double)a.mx && f.hy > f.ly && f.hy > 0.0 && f.ly < (double)a.my;
   f.bi = max(0, min(__double2int_rz(f.lx), a.mx - 1));
   f.bj = max(0, min(__double2int_rz(f.ly), a.my - 1));
   return (f.bi >> a.tile_log2) * a.tiles_y + (f.bj >> a.tile_log2);
+}
+
+// D1-D3 run only when the tile-ordered list must be rebuilt (every CTA reads the same words: they
+// change only in the scatter and the gather, after the sort)
+__device__ __forceinline__ bool sort_needed(const DenArgs &a) {
+  return a.force_sort || *(volatile int *)a.sortctl != 0 || *(volatile int *)(a.sortctl + 1) > a.resort_thr;
 }
 
 // first bin of a (non-empty) footprint and its tile
@@ -169,6 +183,7 @@ __device__ __forceinline__ void load_cells(const DenArgs &a, int i0, float (&x)[
 template <bool MASK>
 __global__ void __launch_bounds__(kCountThreads) k_count(DenArgs a) {
   griddep_wait();
+  if (!sort_needed(a)) return;
   extern __shared__ int s_hist[];
   for (int t = threadIdx.x; t < a.ntiles; t += kCountThreads) s_hist[t] = 0;
   __syncthreads();
@@ -205,6 +220,8 @@ __device__ __forceinline__ int warp_incl_scan(int v, int lane) {
 
 __global__ void __launch_bounds__(1024) k_scan(DenArgs a) {
   griddep_wait();
+  if (!sort_needed(a)) return;
+  if (threadIdx.x == 0) a.sortctl[3]++;
   __shared__ int s_wa[32];
   constexpr int T = 1024;
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
@@ -239,14 +256,14 @@ __global__ void __launch_bounds__(1024) k_scan(DenArgs a) {
   if (threadIdx.x == T - 1) a.tile_off[a.ntiles] = off_c;
 }
 
-// D3: the same cells as D1, footprints computed once and held in registers.  The shared
-// histogram's atomicAdd returns each cell's rank inside its tile; a block scan of the histogram
-// (with one global reservation per non-empty tile) gives the local tile-ordered slots; records
-// are assembled in shared memory and written out in contiguous per-tile runs (random
-// per-record stores were measured 3x slower).
+// D3: the same cells as D1.  The shared histogram's atomicAdd returns each cell's rank inside
+// its tile; a block scan of the histogram (with one global reservation per non-empty tile) gives
+// the local tile-ordered slots; the list entries (cell, w, h) are assembled in shared memory and
+// written out in contiguous per-tile runs (random per-record stores were measured 3x slower).
+// The footprints themselves are formed by the scatter walker on every evaluation (the list is
+// kept while the cells stay in their tiles).
 struct PlaceOut {
-  float4 rec[kCountCells];
-  int2 rc[kCountCells];
+  float2 wh[kCountCells];
   int cell[kCountCells];
   int tile[kCountCells];
 };
@@ -256,6 +273,7 @@ int place_smem_bytes(int ntiles) { return (int)sizeof(PlaceOut) + 8 * ntiles; }
 template <bool MASK>
 __global__ void __launch_bounds__(kCountThreads) k_place(DenArgs a) {
   griddep_wait();
+  if (!sort_needed(a)) return;
   extern __shared__ __align__(16) unsigned char psm[];
   PlaceOut &po = *reinterpret_cast<PlaceOut *>(psm);
   int *s_hist = reinterpret_cast<int *>(psm + sizeof(PlaceOut));   // [ntiles] counts -> local offsets
@@ -266,10 +284,7 @@ __global__ void __launch_bounds__(kCountThreads) k_place(DenArgs a) {
   float x[kCellsPerThread], y[kCellsPerThread], w[kCellsPerThread], h[kCellsPerThread];
   load_cells(a, i0, x, y, w, h);
   __syncthreads();
-  float4 rec[kCellsPerThread];
-  int rcy[kCellsPerThread], tl[kCellsPerThread], rank[kCellsPerThread];
-  float rr[kCellsPerThread];
-  const int mask = a.tile - 1;
+  int tl[kCellsPerThread], rank[kCellsPerThread];
 #pragma unroll
   for (int k = 0; k < kCellsPerThread; k++) {
     const int i = i0 + k * kCountThreads + threadIdx.x;
@@ -277,24 +292,16 @@ __global__ void __launch_bounds__(kCountThreads) k_place(DenArgs a) {
     int t = classify_small(a, x[k], y[k], w[k], h[k], f);
     tl[k] = -1;
     if (i >= a.n_own || t == -2) continue;
-    if (MASK && !selected(a, i)) {   // fixed cell of an evaluation: no record, force 0;
+    if (MASK && !selected(a, i)) {   // fixed cell of an evaluation: not listed, force 0;
       if (a.keep) continue;          // another region's cell: its own pass writes its force
-      t = -1;
+      t = -3;
     }
-    if (t == -1) {
+    if (t == -3) {   // never in the map (zero area / fixed): force 0, kept until the next sort
       a.force[i] = make_float2(0.f, 0.f);
       continue;
     }
     tl[k] = t;
     rank[k] = atomicAdd(&s_hist[t], 1);
-    // bin-local fractions (|v| < 3) of the clipped footprint [max(l, 0), min(h, M)]: fp32 keeps
-    // ~2e-7 bin absolute precision, which the force gather needs where large opposite bin fields
-    // cancel (the 'initial' placement).  fl(max(l, 0) - b) = max(fl(l - b), -b) (monotone rounding)
-    const int bi = f.bi, bj = f.bj;
-    rec[k] = make_float4(fmaxf((float)(f.lx - bi), (float)-bi), fmaxf((float)(f.ly - bj), (float)-bj),
-                         fminf((float)(f.hx - bi), (float)(a.mx - bi)), fminf((float)(f.hy - bj), (float)(a.my - bj)));
-    rr[k] = __fdividef(w[k] * h[k], f.ws * f.hs);
-    rcy[k] = (bi & mask) | ((bj & mask) << 16);
   }
   __syncthreads();
   // reservation + block exclusive scan of the histogram (tiles split evenly over the threads)
@@ -332,8 +339,7 @@ __global__ void __launch_bounds__(kCountThreads) k_place(DenArgs a) {
   for (int k = 0; k < kCellsPerThread; k++) {
     if (tl[k] < 0) continue;
     const int slot = s_hist[tl[k]] + rank[k];
-    po.rec[slot] = rec[k];
-    po.rc[slot] = make_int2(__float_as_int(rr[k]), rcy[k]);
+    po.wh[slot] = make_float2(w[k], h[k]);
     po.cell[slot] = i0 + k * kCountThreads + threadIdx.x;
     po.tile[slot] = tl[k];
   }
@@ -342,35 +348,63 @@ __global__ void __launch_bounds__(kCountThreads) k_place(DenArgs a) {
   for (int j = threadIdx.x; j < total; j += kCountThreads) {
     const int t = po.tile[j];
     const int pos = s_base[t] + (j - s_hist[t]);
-    a.rec[pos] = po.rec[j];
-    a.rec_rc[pos] = po.rc[j];
+    a.rec_wh[pos] = po.wh[j];
     a.rec_cell[pos] = po.cell[j];
   }
 }
 
-// Record staging ring: kStages buffers of up to kStageRecs records of rec (16 B), rec_rc (8 B)
-// and rec_cell (4 B), each completing on its own mbarrier.  Thread 0 owns the walker and keeps
+// Record staging ring: kStages buffers of up to kStageRecs records, each completing on its own
+// mbarrier: the scatter stages the list (rec_cell 4 B, rec_wh 8 B in the rc slot), the gather the
+// footprint records the scatter wrote (rec 16 B, rec_rc 8 B, rec_cell 4 B).  Thread 0 owns the walker and keeps
 // kStages - 1 chunks in flight; the chunk descriptors live in shared memory next to the data.
 // The copied range is rounded out to 4-record multiples (the record arrays are padded by 8).
 constexpr int kStages = 4;
-struct RecBuf {
+struct RecBufG {   // gather: footprint records
   float4 rec[kStageRecs + 8];
   int2 rc[kStageRecs + 8];
+  int cell[kStageRecs + 8];
+};
+struct RecBufS {   // scatter: list entries
+  float2 wh[kStageRecs + 8];
   int cell[kStageRecs + 8];
 };
 struct WalkChunk {
   int begin, end, tile, off;
 };
+template <class Buf>
 struct RecStage {
-  RecBuf buf[kStages];
+  Buf buf[kStages];
   WalkChunk ch[kStages];
   uint64_t bar[kStages];     // full: descriptor + records landed (one arrival by the producer + tx bytes)
   uint64_t empty[kStages];   // released: every warp has consumed the buffer (one arrival per warp)
   uint64_t bar_xi;
 };
+using StageG = RecStage<RecBufG>;
+using StageS = RecStage<RecBufS>;
 
-__host__ __device__ constexpr int rec_stage_bytes() { return (int)((sizeof(RecStage) + 15) & ~(size_t)15); }
-int walk_smem_bytes(int tile) { return rec_stage_bytes() + (tile + kHalo) * (tile + kHalo) * 8; }
+template <class St>
+__host__ __device__ constexpr int stage_bytes() { return (int)((sizeof(St) + 15) & ~(size_t)15); }
+__host__ __device__ constexpr int walk_span(int tile) { return tile + kHalo + 2 * kMargin; }   // shared tile side
+// the scatter's CTA is the smaller (12-byte list entries, a 32-bit word per bin), so WA CTAs fit
+// beside it; both walkers run the same grid (the gather's occupancy)
+int scatter_smem_bytes(int tile) { return stage_bytes<StageS>() + walk_span(tile) * walk_span(tile) * 4; }
+int walk_smem_bytes(int tile) { return stage_bytes<StageG>() + walk_span(tile) * walk_span(tile) * 8; }
+
+__device__ __forceinline__ unsigned issue_copies(const DenArgs &a, RecBufG &B, int b0, int n, uint64_t *bar) {
+  if (n > 0) {
+    bulk_g2s(B.rec, a.rec + b0, 16u * n, bar);
+    bulk_g2s(B.rc, a.rec_rc + b0, 8u * n, bar);
+    bulk_g2s(B.cell, a.rec_cell + b0, 4u * n, bar);
+  }
+  return 28u;
+}
+__device__ __forceinline__ unsigned issue_copies(const DenArgs &a, RecBufS &B, int b0, int n, uint64_t *bar) {
+  if (n > 0) {
+    bulk_g2s(B.wh, a.rec_wh + b0, 8u * n, bar);
+    bulk_g2s(B.cell, a.rec_cell + b0, 4u * n, bar);
+  }
+  return 12u;
+}
 
 // A walker's slice [rb, re) of the tile-ordered small-cell records, cut into chunks of at most
 // kStageRecs records that never straddle a tile.
@@ -393,7 +427,8 @@ __device__ __forceinline__ void walk_init(const DenArgs &a, Walker &w) {
 // (thread 0) next chunk of the slice -> descriptor slot b, copies issued on bar[b].  The
 // descriptor is written before the arrival, so a consumer that sees the phase complete sees it;
 // an empty chunk (end of the slice) completes its phase with no bytes.
-__device__ __forceinline__ void walk_issue(const DenArgs &a, Walker &w, RecStage &st, int b, bool with_cell) {
+template <class St>
+__device__ __forceinline__ void walk_issue(const DenArgs &a, Walker &w, St &st, int b) {
   WalkChunk c;
   c.begin = c.end = w.cur;
   c.tile = w.t;
@@ -409,24 +444,22 @@ __device__ __forceinline__ void walk_issue(const DenArgs &a, Walker &w, RecStage
     c.off = c.begin - b0;
   }
   st.ch[b] = c;
-  mbar_expect_tx(&st.bar[b], (unsigned)n * (with_cell ? 28u : 24u));
-  if (n > 0) {
-    RecBuf &B = st.buf[b];
-    bulk_g2s(B.rec, a.rec + b0, 16u * n, &st.bar[b]);
-    bulk_g2s(B.rc, a.rec_rc + b0, 8u * n, &st.bar[b]);
-    if (with_cell) bulk_g2s(B.cell, a.rec_cell + b0, 4u * n, &st.bar[b]);
-  }
+  // the arrival (with the byte count) precedes the copies; an empty chunk completes with no bytes
+  constexpr unsigned per = sizeof(st.buf[0]) == sizeof(RecBufG) ? 28u : 12u;
+  mbar_expect_tx(&st.bar[b], (unsigned)n * per);
+  issue_copies(a, st.buf[b], b0, n, &st.bar[b]);
 }
 
 // (thread 0) barriers + the first kStages - 1 chunks; the caller synchronises
-__device__ __forceinline__ void walk_start(const DenArgs &a, Walker &w, RecStage &st, bool with_cell) {
+template <class St>
+__device__ __forceinline__ void walk_start(const DenArgs &a, Walker &w, St &st) {
   walk_init(a, w);
   for (int b = 0; b < kStages; b++) {
     mbar_init(&st.bar[b]);
     mbar_init_count(&st.empty[b], blockDim.x >> 5);
   }
   mbar_init(&st.bar_xi);
-  for (int b = 0; b < kStages - 1; b++) walk_issue(a, w, st, b, with_cell);
+  for (int b = 0; b < kStages - 1; b++) walk_issue(a, w, st, b);
 }
 
 // Ring step of chunk c (every thread): wait until chunk c has landed; thread 0 then refills the
@@ -438,7 +471,8 @@ __device__ __forceinline__ void walk_start(const DenArgs &a, Walker &w, RecStage
 // mbarrier ordering and reports the descriptor refill as a WAR hazard; a.sync_ring
 // (DP_WALK_SYNC=1, diagnostics only) adds a block barrier before each refill, under which
 // racecheck reports none (profiles/r02_sanitizer_racecheck*.log).
-__device__ __forceinline__ WalkChunk walk_next(const DenArgs &a, Walker &w, RecStage &st, int c, bool with_cell) {
+template <class St>
+__device__ __forceinline__ WalkChunk walk_next(const DenArgs &a, Walker &w, St &st, int c) {
   const int b = c % kStages;
   mbar_wait(&st.bar[b], (c / kStages) & 1);
   const WalkChunk cc = st.ch[b];
@@ -446,13 +480,14 @@ __device__ __forceinline__ WalkChunk walk_next(const DenArgs &a, Walker &w, RecS
   if (threadIdx.x == 0 && cc.begin < cc.end) {
     const int b2 = (c + kStages - 1) % kStages;
     if (c >= 1) mbar_wait(&st.empty[b2], ((c - 1) / kStages) & 1);
-    walk_issue(a, w, st, b2, with_cell);
+    walk_issue(a, w, st, b2);
   }
   return cc;
 }
 
 // this warp is done with chunk c's buffer
-__device__ __forceinline__ void walk_release(RecStage &st, int c) {
+template <class St>
+__device__ __forceinline__ void walk_release(St &st, int c) {
   __syncwarp();
   if ((threadIdx.x & 31) == 0) mbar_arrive(&st.empty[c % kStages]);
 }
@@ -471,8 +506,8 @@ __device__ __forceinline__ void rec_overlaps(const float4 q, float ox3[3], float
 // after).  Each word holds its bin's sum modulo 2^32 (units 2^-29); the wraps were already added
 // to rho by the threads whose atomic crossed 2^32, so rho + word is the exact int64 sum.
 __device__ __forceinline__ void flush_tile(const DenArgs &a, unsigned *s_acc, int tile) {
-  const int P = a.tile + kHalo;
-  const int ox = (tile / a.tiles_y) * a.tile, oy = (tile % a.tiles_y) * a.tile;
+  const int P = walk_span(a.tile);
+  const int ox = (tile / a.tiles_y) * a.tile - kMargin, oy = (tile % a.tiles_y) * a.tile - kMargin;
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = blockDim.x >> 5;
   for (int i = warp; i < P; i += nw) {
     const int gi = ox + i;
@@ -481,7 +516,7 @@ __device__ __forceinline__ void flush_tile(const DenArgs &a, unsigned *s_acc, in
       const unsigned long long v = (unsigned long long)s_acc[k];
       s_acc[k] = 0u;
       const int gj = oy + j;
-      if (v != 0ull && gi < a.mx && gj < a.my)
+      if (v != 0ull && (unsigned)gi < (unsigned)a.mx && (unsigned)gj < (unsigned)a.my)
         asm volatile("red.global.add.u64 [%0], %1;" ::"l"(a.rho + (size_t)gi * a.my + gj), "l"(v) : "memory");
     }
   }
@@ -494,27 +529,56 @@ __device__ __forceinline__ unsigned atom_shared_add(unsigned *p, unsigned v) {
   return old;
 }
 
-// D4: persistent scatter walker.  Every bin of the (tile+2)^2 shared tile is one 32-bit word
-// accumulating u = floor(v 2^29) (v <= 1, so u <= 2^29) with a native shared atomic add that
-// returns the old word; the (rare) thread whose add wraps past 2^32 adds 2^32 units to the int64
-// map itself.  The word is flushed when the slice leaves the tile.  The map is the exact sum of
-// the per-contribution roundings whatever the order (bit-identical to a flush-per-record scheme).
+// D4: persistent scatter walker.  Each listed cell's footprint is formed here from its current
+// position (the classifier of D1-D3, fp64 corners): the record (fractions of the first bin, r,
+// first bin) is written to the cell's slot for the gather.  A cell whose first bin is still in
+// the walker's tile adds into the (tile+2)^2 shared tile: one 32-bit word per bin accumulating
+// u = floor(v 2^29) (v <= 1, so u <= 2^29) with a native shared atomic add that returns the old
+// word; the (rare) thread whose add wraps past 2^32 adds 2^32 units to the int64 map itself.  A
+// cell that has left its tile since the last sort (a stray) adds the same u straight to the int64
+// map.  The word is flushed when the slice leaves the tile.  The map is the exact sum of the
+// per-contribution roundings whatever the order or path (bit-identical to a fresh sort).
+static_assert(kStageRecs == kTileThreads, "the scatter walker holds one record per thread and chunk");
+
+// (scatter) this thread's list entry of a landed chunk and the cell's current position: the
+// position loads are random L2 reads, issued one chunk ahead of their use
+struct ScatterIn {
+  int cell;
+  float2 wh;
+  float x, y;
+};
+
+__device__ __forceinline__ void scatter_fetch(const DenArgs &a, const StageS &st, int b, const WalkChunk &cc,
+                                              ScatterIn &in) {
+  if ((int)threadIdx.x < cc.end - cc.begin) {
+    in.cell = st.buf[b].cell[cc.off + threadIdx.x];
+    in.wh = st.buf[b].wh[cc.off + threadIdx.x];
+    in.x = __ldg(a.x + a.cell_begin + in.cell);
+    in.y = __ldg(a.y + a.cell_begin + in.cell);
+  }
+}
+
 __global__ void __launch_bounds__(kTileThreads) k_scatter_walk(DenArgs a) {
   griddep_wait();
   extern __shared__ __align__(16) unsigned char dsm[];
-  RecStage &st = *reinterpret_cast<RecStage *>(dsm);
-  unsigned *s_acc = reinterpret_cast<unsigned *>(dsm + rec_stage_bytes());   // 2^-29 units, mod 2^32
-  const int P = a.tile + kHalo;
+  StageS &st = *reinterpret_cast<StageS *>(dsm);
+  unsigned *s_acc = reinterpret_cast<unsigned *>(dsm + stage_bytes<StageS>());   // 2^-29 units, mod 2^32
+  const int P = walk_span(a.tile);
+  const int span = a.tile + 2 * kMargin;   // first bins the shared tile takes
   Walker w;
-  if (threadIdx.x == 0) walk_start(a, w, st, false);
+  if (threadIdx.x == 0) {
+    if (blockIdx.x == 0) a.sortctl[0] = 0;   // a requested sort has run (D1-D3 precede this kernel)
+    walk_start(a, w, st);
+  }
   for (int k = threadIdx.x; k < P * P; k += blockDim.x) s_acc[k] = 0u;
   __syncthreads();
   const float scale_fx = (float)(1u << kRhoScaleLog2);
   int cur_tile = -1;
-  for (int c = 0;; c++) {
-    const int b = c % kStages;
-    const WalkChunk cc = walk_next(a, w, st, c, false);
-    if (cc.begin >= cc.end) break;
+  unsigned strays = 0;
+  WalkChunk cc = walk_next(a, w, st, 0);
+  ScatterIn in = {0, make_float2(0.f, 0.f), 0.f, 0.f};
+  scatter_fetch(a, st, 0, cc, in);
+  for (int c = 0; cc.begin < cc.end; c++) {
     const int n = cc.end - cc.begin;
     if (cur_tile < 0) cur_tile = cc.tile;
     if (cc.tile != cur_tile) {   // uniform: every warp sees the same chunks
@@ -523,62 +587,105 @@ __global__ void __launch_bounds__(kTileThreads) k_scatter_walk(DenArgs a) {
       __syncthreads();   // flushed and cleared
       cur_tile = cc.tile;
     }
-    const RecBuf &B = st.buf[b];
-    for (int k = threadIdx.x; k < n; k += blockDim.x) {
-      const float4 q = B.rec[cc.off + k];
-      const int2 rc = B.rc[cc.off + k];
-      const float r = __int_as_float(rc.x) * scale_fx;   // r 2^29
-      const int i0 = rc.y & 0xffff, j0 = rc.y >> 16;
-      float ox3[3], oy3[3];
-      rec_overlaps(q, ox3, oy3);
-      const int base = i0 * P + j0;
-      unsigned wrapped = 0u;   // bit 3 di + dj: that word's add wrapped past 2^32
+    // chunk c + 1 was issued (non-empty chunks c, c - 1, c - 2 refilled the ring): its entries and
+    // positions are fetched now and arrive while this chunk is processed
+    const int b1 = (c + 1) % kStages;
+    mbar_wait(&st.bar[b1], ((c + 1) / kStages) & 1);
+    const WalkChunk cn = st.ch[b1];
+    ScatterIn nx = in;
+    scatter_fetch(a, st, b1, cn, nx);
+    const int tox = (cur_tile / a.tiles_y) * a.tile - kMargin, toy = (cur_tile % a.tiles_y) * a.tile - kMargin;
+    if ((int)threadIdx.x < n) {
+      SmallFoot f;
+      classify_small(a, in.x, in.y, in.wh.x, in.wh.y, f);   // listed cells are small with w h > 0
+      float4 q = make_float4(0.f, 0.f, 0.f, 0.f);
+      int2 rc = make_int2(0, 0);
+      if (f.ok) {
+        const int bi = f.bi, bj = f.bj;
+        // bin-local fractions (|v| < 3) of the clipped footprint [max(l, 0), min(h, M)]: fp32 keeps
+        // ~2e-7 bin absolute precision, which the force gather needs where large opposite bin
+        // fields cancel (the 'initial' placement).  fl(max(l, 0) - b) = max(fl(l - b), -b)
+        q = make_float4(fmaxf((float)(f.lx - bi), (float)-bi), fmaxf((float)(f.ly - bj), (float)-bj),
+                        fminf((float)(f.hx - bi), (float)(a.mx - bi)), fminf((float)(f.hy - bj), (float)(a.my - bj)));
+        const float rr = __fdividef(in.wh.x * in.wh.y, f.ws * f.hs);
+        const int i0 = bi - tox, j0 = bj - toy;
+        const bool stray = (unsigned)i0 >= (unsigned)span || (unsigned)j0 >= (unsigned)span;
+        rc = make_int2(__float_as_int(rr), stray ? (int)(bi | (bj << 16) | 0x80000000u) : (i0 | (j0 << 16)));
+        const float r = rr * scale_fx;   // r 2^29
+        float ox3[3], oy3[3];
+        rec_overlaps(q, ox3, oy3);
+        if (!stray) {
+          const int base = i0 * P + j0;
+          unsigned wrapped = 0u;   // bit 3 di + dj: that word's add wrapped past 2^32
 #pragma unroll
-      for (int di = 0; di < 3; di++) {
-        const float rx = r * ox3[di];
+          for (int di = 0; di < 3; di++) {
+            const float rx = r * ox3[di];
 #pragma unroll
-        for (int dj = 0; dj < 3; dj++) {
-          const unsigned u = (unsigned)(rx * oy3[dj]);   // floor(v 2^29) <= 2^29 (power-of-two scaling is exact)
-          const unsigned old = atom_shared_add(s_acc + base + di * P + dj, u);
-          wrapped |= (old + u < old ? 1u : 0u) << (3 * di + dj);
+            for (int dj = 0; dj < 3; dj++) {
+              const unsigned u = (unsigned)(rx * oy3[dj]);   // floor(v 2^29) <= 2^29 (power-of-two scaling is exact)
+              const unsigned old = atom_shared_add(s_acc + base + di * P + dj, u);
+              wrapped |= (old + u < old ? 1u : 0u) << (3 * di + dj);
+            }
+          }
+          // wrapped words (rare): 2^32 units (8 bin areas) each go straight to the map.  Collected
+          // as a mask so that the map addresses are formed only here (as predicated reductions
+          // inside the loop, they were computed for all nine bins of every record)
+          if (wrapped) {
+            while (wrapped) {
+              const int bit = __ffs(wrapped) - 1;
+              wrapped &= wrapped - 1;
+              asm volatile("red.global.add.u64 [%0], %1;" ::"l"(a.rho + (size_t)(bi + bit / 3) * a.my + bj + bit % 3),
+                           "l"(1ull << 32)
+                           : "memory");
+            }
+          }
+        } else {   // stray: the same units straight into the map (bins past the map have zero overlap)
+          strays++;
+#pragma unroll
+          for (int di = 0; di < 3; di++) {
+            const float rx = r * ox3[di];
+#pragma unroll
+            for (int dj = 0; dj < 3; dj++) {
+              const unsigned u = (unsigned)(rx * oy3[dj]);
+              if (u)
+                asm volatile("red.global.add.u64 [%0], %1;" ::"l"(a.rho + (size_t)(bi + di) * a.my + bj + dj),
+                             "l"((unsigned long long)u)
+                             : "memory");
+            }
+          }
         }
       }
-      // wrapped words (rare): 2^32 units (8 bin areas) each go straight to the map.  Collected as a
-      // mask so that the map addresses are formed only here (as predicated reductions inside the
-      // loop, they were computed for all nine bins of every record)
-      if (wrapped) {
-        const size_t ox = (size_t)(cur_tile / a.tiles_y) * a.tile + i0, oy = (size_t)(cur_tile % a.tiles_y) * a.tile + j0;
-        while (wrapped) {
-          const int bit = __ffs(wrapped) - 1;
-          wrapped &= wrapped - 1;
-          asm volatile("red.global.add.u64 [%0], %1;" ::"l"(a.rho + (ox + bit / 3) * a.my + oy + bit % 3),
-                       "l"(1ull << 32)
-                       : "memory");
-        }
-      }
+      a.rec[cc.begin + threadIdx.x] = q;
+      a.rec_rc[cc.begin + threadIdx.x] = rc;
     }
     walk_release(st, c);
+    cc = walk_next(a, w, st, c + 1);   // landed already; thread 0 refills the ring
+    in = nx;
   }
   __syncthreads();
   if (cur_tile >= 0) flush_tile(a, s_acc, cur_tile);
+  strays = __reduce_add_sync(0xffffffffu, strays);
+  if ((threadIdx.x & 31) == 0 && strays) atomicAdd(a.sortctl + 2, (int)strays);
 }
 
 // D5: persistent gather walker; the (tile+2)^2 float2 field tile is (re)loaded with one bulk copy
 // per tile row whenever the slice enters a tile; bins outside the map read as zero.
-__device__ __forceinline__ void load_xi_tile(const DenArgs &a, RecStage &st, float2 *s_xi, int tile,
+__device__ __forceinline__ void load_xi_tile(const DenArgs &a, StageG &st, float2 *s_xi, int tile,
                                              unsigned phase) {
-  const int P = a.tile + kHalo;
-  const int ox = (tile / a.tiles_y) * a.tile, oy = (tile % a.tiles_y) * a.tile;
-  const int rows = min(P, a.mx - ox), cols = min(P, a.my - oy);   // cols = tile or tile + 2: 16-byte multiple
-  if (threadIdx.x == 0) mbar_expect_tx(&st.bar_xi, (unsigned)(rows * cols * 8));
+  const int P = walk_span(a.tile);
+  const int ox = (tile / a.tiles_y) * a.tile - kMargin, oy = (tile % a.tiles_y) * a.tile - kMargin;
+  // rows [r0, r1) and columns [c0, c1) of the shared tile lie in the map (c0, c1 even: 16-byte rows)
+  const int r0 = max(0, -ox), r1 = min(P, a.mx - ox), c0 = max(0, -oy), c1 = min(P, a.my - oy);
+  if (threadIdx.x == 0) mbar_expect_tx(&st.bar_xi, (unsigned)((r1 - r0) * (c1 - c0) * 8));
   __syncthreads();   // armed before any copy can complete
-  if (threadIdx.x < rows)
-    bulk_g2s(s_xi + threadIdx.x * P, a.xi + (size_t)(ox + threadIdx.x) * a.my + oy, 8u * cols, &st.bar_xi);
-  if (rows < P || cols < P) {
+  const int row = r0 + (int)threadIdx.x;
+  if (row < r1)
+    bulk_g2s(s_xi + row * P + c0, a.xi + (size_t)(ox + row) * a.my + (oy + c0), 8u * (c1 - c0), &st.bar_xi);
+  if (r0 > 0 || r1 < P || c0 > 0 || c1 < P) {
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = blockDim.x >> 5;
     for (int i = warp; i < P; i += nw)
       for (int j = lane; j < P; j += 32)
-        if (i >= rows || j >= cols) s_xi[i * P + j] = make_float2(0.f, 0.f);
+        if (i < r0 || i >= r1 || j < c0 || j >= c1) s_xi[i * P + j] = make_float2(0.f, 0.f);
     __syncthreads();
   }
   mbar_wait(&st.bar_xi, phase);
@@ -587,11 +694,17 @@ __device__ __forceinline__ void load_xi_tile(const DenArgs &a, RecStage &st, flo
 __global__ void __launch_bounds__(kTileThreads) k_gather_walk(DenArgs a) {
   griddep_wait();
   extern __shared__ __align__(16) unsigned char dsm[];
-  RecStage &st = *reinterpret_cast<RecStage *>(dsm);
-  float2 *s_xi = reinterpret_cast<float2 *>(dsm + rec_stage_bytes());
-  const int P = a.tile + kHalo;
+  StageG &st = *reinterpret_cast<StageG *>(dsm);
+  float2 *s_xi = reinterpret_cast<float2 *>(dsm + stage_bytes<StageG>());
+  const int P = walk_span(a.tile);
   Walker w;
-  if (threadIdx.x == 0) walk_start(a, w, st, true);
+  if (threadIdx.x == 0) {
+    if (blockIdx.x == 0) {   // the scatter has completed: its stray count decides the next sort
+      a.sortctl[1] = a.sortctl[2];
+      a.sortctl[2] = 0;
+    }
+    walk_start(a, w, st);
+  }
   __syncthreads();   // barriers initialised, first descriptors visible
   int cur_tile = -1;
   unsigned xi_phase = 0;
@@ -599,36 +712,54 @@ __global__ void __launch_bounds__(kTileThreads) k_gather_walk(DenArgs a) {
   const float lam = a.lambda_dev ? __ldg(a.lambda_dev) : a.lambda;
   for (int c = 0;; c++) {
     const int b = c % kStages;
-    const WalkChunk cc = walk_next(a, w, st, c, true);
+    const WalkChunk cc = walk_next(a, w, st, c);
     if (cc.begin >= cc.end) break;
     if (cc.tile != cur_tile) {   // uniform; load_xi_tile's barrier waits until every warp left the old tile
       load_xi_tile(a, st, s_xi, cc.tile, xi_phase);
       xi_phase ^= 1u;
       cur_tile = cc.tile;
     }
-    const RecBuf &B = st.buf[b];
+    const RecBufG &B = st.buf[b];
     const int n = cc.end - cc.begin;
     for (int k = threadIdx.x; k < n; k += blockDim.x) {
       const float4 q = B.rec[cc.off + k];
       const int2 rc = B.rc[cc.off + k];
       const float r = __int_as_float(rc.x);
-      const int i0 = rc.y & 0xffff, j0 = rc.y >> 16;
       float ox3[3], oy3[3];
       rec_overlaps(q, ox3, oy3);
-      const float2 *row = s_xi + i0 * P + j0;
       float fx = 0.f, fy = 0.f;
+      if (rc.y >= 0) {
+        const int i0 = rc.y & 0xffff, j0 = rc.y >> 16;
+        const float2 *row = s_xi + i0 * P + j0;
 #pragma unroll
-      for (int di = 0; di < 3; di++) {
-        float sx = 0.f, sy = 0.f;
+        for (int di = 0; di < 3; di++) {
+          float sx = 0.f, sy = 0.f;
 #pragma unroll
-        for (int dj = 0; dj < 3; dj++) {
-          // in-bounds: i0 < tile, j0 < tile, P = tile + 2; bins without overlap are not read
-          const float2 e2 = (ox3[di] > 0.f && oy3[dj] > 0.f) ? row[di * P + dj] : make_float2(0.f, 0.f);
-          sx = fmaf(oy3[dj], e2.x, sx);
-          sy = fmaf(oy3[dj], e2.y, sy);
+          for (int dj = 0; dj < 3; dj++) {
+            // in-bounds: i0, j0 < tile + 2 kMargin, P = that + 2; bins without overlap are not read
+            const float2 e2 = (ox3[di] > 0.f && oy3[dj] > 0.f) ? row[di * P + dj] : make_float2(0.f, 0.f);
+            sx = fmaf(oy3[dj], e2.x, sx);
+            sy = fmaf(oy3[dj], e2.y, sy);
+          }
+          fx = fmaf(ox3[di], sx, fx);
+          fy = fmaf(ox3[di], sy, fy);
         }
-        fx = fmaf(ox3[di], sx, fx);
-        fy = fmaf(ox3[di], sy, fy);
+      } else {   // stray (left its tile since the sort): the same sums from the global field
+        const int i0 = rc.y & 0xffff, j0 = (rc.y >> 16) & 0x7fff;
+        const float2 *row = a.xi + (size_t)i0 * a.my + j0;
+#pragma unroll
+        for (int di = 0; di < 3; di++) {
+          float sx = 0.f, sy = 0.f;
+#pragma unroll
+          for (int dj = 0; dj < 3; dj++) {
+            // bins past the map have zero overlap and are not read
+            const float2 e2 = (ox3[di] > 0.f && oy3[dj] > 0.f) ? row[(size_t)di * a.my + dj] : make_float2(0.f, 0.f);
+            sx = fmaf(oy3[dj], e2.x, sx);
+            sy = fmaf(oy3[dj], e2.y, sy);
+          }
+          fx = fmaf(ox3[di], sx, fx);
+          fy = fmaf(ox3[di], sy, fy);
+        }
       }
       // dD/dx = - r sum_b ov(i,b) xi^X_b  (reading A21), ov in length^2
       if (a.gxo) {
@@ -731,6 +862,19 @@ __global__ void __launch_bounds__(256) k_region_overflow(const unsigned long lon
   }
 }
 
+// Start of the map in a captured evaluation: rho <- src (the fixed-charge map) or 0, and the
+// graph's IF node around D1-D3 is set to "sort needed" (sort reuse: the count, scan and place
+// launches are skipped altogether when the list is kept).
+__global__ void __launch_bounds__(256) k_map_init(DenArgs a, const unsigned long long *src, long long nbins,
+                                                  cudaGraphConditionalHandle sort_if) {
+  if (blockIdx.x == 0 && threadIdx.x == 0) cudaGraphSetConditional(sort_if, sort_needed(a) ? 1u : 0u);
+  ulonglong2 *d = reinterpret_cast<ulonglong2 *>(a.rho);
+  const ulonglong2 *s2 = reinterpret_cast<const ulonglong2 *>(src);
+  const long long n2 = nbins >> 1;   // maps are even-sized
+  for (long long i = blockIdx.x * 256ll + threadIdx.x; i < n2; i += (long long)gridDim.x * 256)
+    d[i] = src ? s2[i] : make_ulonglong2(0ull, 0ull);
+}
+
 // largest float f with (double)f <= v, so that for any float w: w > f <=> (double)w > v
 float float_at_most(double v) {
   float f = (float)v;
@@ -770,6 +914,10 @@ DenArgs make_args(const Ctx &c, const float *x, const float *y) {
   a.rec = c.d_rec;
   a.rec_rc = c.d_rec_rc;
   a.rec_cell = c.d_rec_cell;
+  a.rec_wh = c.d_rec_wh;
+  a.sortctl = c.d_sortctl;
+  a.force_sort = c.reuse_sort ? 0 : 1;
+  a.resort_thr = c.resort_thr;
   a.rho = c.d_rho;
   a.xi = c.d_xi;
   a.force = c.d_force;
@@ -791,6 +939,7 @@ DenArgs make_args(const Ctx &c, const float *x, const float *y) {
     a.fixed = c.d_region;
     a.sel = c.cur_region;
     a.keep = 1;
+    a.force_sort = 1;   // one list per region pass: sorted every time
     a.large = c.d_large_reg + c.large_reg_off[c.cur_region];
     a.n_large = c.large_reg_off[c.cur_region + 1] - c.large_reg_off[c.cur_region];
   }
@@ -808,7 +957,7 @@ cudaError_t density_configure(int ntiles, int tile) {
   if (e != cudaSuccess) return e;
   e = cudaFuncSetAttribute(k_place<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, place_smem_bytes(ntiles));
   if (e != cudaSuccess) return e;
-  e = cudaFuncSetAttribute(k_scatter_walk, cudaFuncAttributeMaxDynamicSharedMemorySize, walk_smem_bytes(tile));
+  e = cudaFuncSetAttribute(k_scatter_walk, cudaFuncAttributeMaxDynamicSharedMemorySize, scatter_smem_bytes(tile));
   if (e != cudaSuccess) return e;
   return cudaFuncSetAttribute(k_gather_walk, cudaFuncAttributeMaxDynamicSharedMemorySize, walk_smem_bytes(tile));
 }
@@ -829,7 +978,7 @@ int density_walk_grid(int tile) {
   int dev = 0, sms = 0, o1 = 0, o2 = 0;
   if (cudaGetDevice(&dev) != cudaSuccess) return 0;
   if (cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess) return 0;
-  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o1, k_scatter_walk, kTileThreads, walk_smem_bytes(tile)) != cudaSuccess)
+  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o1, k_scatter_walk, kTileThreads, scatter_smem_bytes(tile)) != cudaSuccess)
     return 0;
   if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o2, k_gather_walk, kTileThreads, walk_smem_bytes(tile)) != cudaSuccess)
     return 0;
@@ -856,24 +1005,53 @@ int density_launches(const Ctx &c) { return 5 + (c.n_large > 0 ? 2 : 0); }
 void launch_density_map(const Ctx &c, const float *x, const float *y, cudaStream_t s, cudaStream_t aux,
                         int build_fixed) {
   DenArgs a = make_args(c, x, y);
-  if (build_fixed) {   // dp_set_fixed: the map of the fixed cells alone
-    a.fixed = c.d_fixed;
+  if (build_fixed) {   // dp_set_fixed: the map of the fixed cells alone (its own list: the caller
+    a.fixed = c.d_fixed;   // requests a sort for the next evaluation)
     a.sel = 1;
+    a.force_sort = 1;
     a.large = c.d_large_fix;
     a.n_large = c.n_large_fix;
   }
   const int ntiles = a.ntiles;
   const int nblk = (c.n_own + kCountCells - 1) / kCountCells;
-  if (c.n_regions > 0 && c.cur_region >= 0)   // start from the region's blockage map (exact int64)
-    cudaMemcpyAsync(c.d_rho, c.d_rho_block + (size_t)c.cur_region * c.mx * c.my,
-                    sizeof(unsigned long long) * (size_t)c.mx * c.my, cudaMemcpyDeviceToDevice, s);
-  else if (c.has_fixed && !build_fixed)   // start from the precomputed fixed-charge map (exact int64)
-    cudaMemcpyAsync(c.d_rho, c.d_rho_fixed, sizeof(unsigned long long) * (size_t)c.mx * c.my,
-                    cudaMemcpyDeviceToDevice, s);
-  else
-    cudaMemsetAsync(c.d_rho, 0, sizeof(unsigned long long) * (size_t)c.mx * c.my, s);
+  const size_t nb = (size_t)c.mx * c.my;
+  const unsigned long long *src = nullptr;   // the map starts from this (or 0)
+  if (c.n_regions > 0 && c.cur_region >= 0)   // the region's blockage map (exact int64)
+    src = c.d_rho_block + (size_t)c.cur_region * nb;
+  else if (c.has_fixed && !build_fixed)       // the precomputed fixed-charge map (exact int64)
+    src = c.d_rho_fixed;
+  // in a captured evaluation whose list may be kept, D1-D3 sit in a conditional (IF) node set by
+  // k_map_init: no launches at all when the list is kept (DP_SORT_COND=0: the kernels return early)
+  cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+  cudaStreamIsCapturing(s, &cs);
+  const bool cond = nblk > 0 && !a.force_sort && c.sort_cond && c.s_body && cs == cudaStreamCaptureStatusActive;
+  cudaStream_t ss = s;   // stream of D1-D3
+  if (cond) {
+    cudaGraph_t g = nullptr;
+    const cudaGraphNode_t *deps = nullptr;
+    size_t nd = 0;
+    cudaGraphConditionalHandle h = 0;
+    cudaGraphConditionalHandleCreate(&h, (cudaStreamGetCaptureInfo(s, &cs, nullptr, &g), g), 0, 0);
+    k_map_init<<<2 * c.num_sms, 256, 0, s>>>(a, src, (long long)nb, h);
+    cudaStreamGetCaptureInfo(s, &cs, nullptr, &g, &deps, &nd);
+    cudaGraphNodeParams p = {};
+    p.type = cudaGraphNodeTypeConditional;
+    p.conditional.handle = h;
+    p.conditional.type = cudaGraphCondTypeIf;
+    p.conditional.size = 1;
+    cudaGraphNode_t node = nullptr;
+    cudaGraphAddNode(&node, g, deps, nd, &p);
+    cudaStreamUpdateCaptureDependencies(s, &node, 1, cudaStreamSetCaptureDependencies);
+    cudaStreamBeginCaptureToGraph(c.s_body, p.conditional.phGraph_out[0], nullptr, nullptr, 0,
+                                  cudaStreamCaptureModeRelaxed);
+    ss = c.s_body;
+  } else if (src) {
+    cudaMemcpyAsync(c.d_rho, src, sizeof(unsigned long long) * nb, cudaMemcpyDeviceToDevice, s);
+  } else {
+    cudaMemsetAsync(c.d_rho, 0, sizeof(unsigned long long) * nb, s);
+  }
   const bool side = aux && a.n_large > 0;
-  if (side) {
+  if (side && !cond) {
     cudaEventRecord(c.ev_aux_a, s);
     cudaStreamWaitEvent(aux, c.ev_aux_a, 0);
     k_scatter_large<<<a.n_large, 256, 0, aux>>>(a);
@@ -882,18 +1060,29 @@ void launch_density_map(const Ctx &c, const float *x, const float *y, cudaStream
   if (nblk > 0) {
     const int cgrid = std::min(nblk, c.count_grid > 0 ? c.count_grid : nblk);
     if (a.fixed)
-      launch_chain(c.pdl, k_count<true>, cgrid, kCountThreads, ntiles * 4, s, a);
+      launch_chain(c.pdl, k_count<true>, cgrid, kCountThreads, ntiles * 4, ss, a);
     // (k_count<true> counts only selected cells; k_place<true> records only selected cells)
     else
-      launch_chain(c.pdl, k_count<false>, cgrid, kCountThreads, ntiles * 4, s, a);
-    if (c.sched == 3) cudaEventRecord(c.ev_sched, s);   // DP_SCHED=3: WA starts after the count
-    launch_chain(c.pdl, k_scan, 1, 1024, 0, s, a);
+      launch_chain(c.pdl, k_count<false>, cgrid, kCountThreads, ntiles * 4, ss, a);
+    if (c.sched == 3 && !cond) cudaEventRecord(c.ev_sched, ss);   // DP_SCHED=3: WA starts after the count
+    launch_chain(c.pdl, k_scan, 1, 1024, 0, ss, a);
     if (a.fixed)
-      launch_chain(c.pdl, k_place<true>, nblk, kCountThreads, place_smem_bytes(ntiles), s, a);
+      launch_chain(c.pdl, k_place<true>, nblk, kCountThreads, place_smem_bytes(ntiles), ss, a);
     else
-      launch_chain(c.pdl, k_place<false>, nblk, kCountThreads, place_smem_bytes(ntiles), s, a);
-    if (c.sched == 2) cudaEventRecord(c.ev_sched, s);   // DP_SCHED=2: WA starts after the placement
-    launch_chain(c.pdl, k_scatter_walk, c.walk_grid, kTileThreads, walk_smem_bytes(c.tile), s, a);
+      launch_chain(c.pdl, k_place<false>, nblk, kCountThreads, place_smem_bytes(ntiles), ss, a);
+    if (cond) {
+      cudaGraph_t body = nullptr;
+      cudaStreamEndCapture(c.s_body, &body);
+      if (side) {   // the large cells beside the conditional sort and the walkers
+        cudaEventRecord(c.ev_aux_a, s);
+        cudaStreamWaitEvent(aux, c.ev_aux_a, 0);
+        k_scatter_large<<<a.n_large, 256, 0, aux>>>(a);
+        cudaEventRecord(c.ev_aux_b, aux);
+      }
+    }
+    if (c.sched == 2 || (c.sched == 3 && cond)) cudaEventRecord(c.ev_sched, s);   // DP_SCHED=2: WA starts after the placement
+    // after the IF node the walker is an ordinary dependent (programmatic edges join kernel nodes)
+    launch_chain(c.pdl && !cond, k_scatter_walk, c.walk_grid, kTileThreads, scatter_smem_bytes(c.tile), s, a);
   }
   if (side)
     cudaStreamWaitEvent(s, c.ev_aux_b, 0);

@@ -522,6 +522,21 @@ dp_status build_density(Ctx &c, const dp_netlist *nl) {
   if ((st = dev_alloc(c, &c.d_rec, c.n_own + 8)) != DP_OK) return st;
   if ((st = dev_alloc(c, &c.d_rec_rc, c.n_own + 8)) != DP_OK) return st;
   if ((st = dev_alloc(c, &c.d_rec_cell, c.n_own + 8)) != DP_OK) return st;
+  if ((st = dev_alloc(c, &c.d_rec_wh, c.n_own + 8)) != DP_OK) return st;
+  if ((st = dev_alloc(c, &c.d_sortctl, 4)) != DP_OK) return st;
+  {
+    const int32_t ctl[4] = {1, 0, 0, 0};   // the first evaluation sorts
+    DP_CUDA(cudaMemcpy(c.d_sortctl, ctl, sizeof(ctl), cudaMemcpyHostToDevice));
+    const char *e = std::getenv("DP_REUSE_SORT");
+    c.reuse_sort = !(e && std::atoi(e) == 0);
+    const char *ce = std::getenv("DP_SORT_COND");
+    c.sort_cond = !(ce && std::atoi(ce) == 0);
+    // re-sort once more than this share of the small cells has left its tile (DP_RESORT_PCT,
+    // default 5 %: a stray costs its nine map updates as global reductions, a sort ~50 us)
+    const char *pe = std::getenv("DP_RESORT_PCT");
+    const double pct = pe ? std::atof(pe) : 5.0;
+    c.resort_thr = (int32_t)std::min(2.0e9, std::max(0.0, pct * 0.01 * (double)c.n_own));
+  }
   // the maps of the hot path in one arena (rho int64, t, spec, sxy, xi): the density
   // stream's L2 persisting window (create)
   {
@@ -595,6 +610,7 @@ void destroy(Ctx *c) {
   if (c->s_cap) cudaStreamDestroy(c->s_cap);
   if (c->s_wa) cudaStreamDestroy(c->s_wa);
   if (c->s_den) cudaStreamDestroy(c->s_den);
+  if (c->s_body) cudaStreamDestroy(c->s_body);
   if (c->ev_fork) cudaEventDestroy(c->ev_fork);
   if (c->ev_wa) cudaEventDestroy(c->ev_wa);
   if (c->ev_fields) cudaEventDestroy(c->ev_fields);
@@ -732,6 +748,7 @@ dp_status create(const dp_netlist *nl, const dp_grid *grid, int device, int rank
       cudaEventCreateWithFlags(&c->ev_map, cudaEventDisableTiming) != cudaSuccess ||
       cudaEventCreateWithFlags(&c->ev_sched, cudaEventDisableTiming) != cudaSuccess ||
       cudaStreamCreateWithPriority(&c->s_aux, cudaStreamNonBlocking, prio_hi) != cudaSuccess ||
+      cudaStreamCreateWithPriority(&c->s_body, cudaStreamNonBlocking, prio_hi) != cudaSuccess ||
       cudaEventCreateWithFlags(&c->ev_aux_a, cudaEventDisableTiming) != cudaSuccess ||
       cudaEventCreateWithFlags(&c->ev_aux_b, cudaEventDisableTiming) != cudaSuccess ||
       cudaEventCreateWithFlags(&c->ev_join, cudaEventDisableTiming) != cudaSuccess ||
@@ -1095,6 +1112,11 @@ dp_status eval_body_ext(Ctx &c, const float *x, const float *y, float gamma, flo
                         bool do_den) {
   return eval_body(c, x, y, gamma, lambda, gx, gy, d_obj, d_wl, d_energy, d_hpwl, s, do_wa, do_den);
 }
+dp_status request_sort(Ctx &c, cudaStream_t s) {
+  DP_CUDA(cudaMemsetAsync(c.d_sortctl, 0x01, sizeof(int32_t), s));   // word 0 != 0: sort requested
+  return DP_OK;
+}
+
 dp_status ctx_call_begin(Ctx &c, cudaStream_t s) { return call_begin(c, s); }
 dp_status ctx_call_end(Ctx &c, cudaStream_t s) { return call_end(c, s); }
 }  // namespace dp
@@ -1222,6 +1244,7 @@ dp_status dp_set_fixed(dp_ctx *ctx, const uint8_t *h_fixed, const float *x, cons
   }
   if (!h_fixed) {
     c->has_fixed = false;
+    if ((st = dp::request_sort(*c, s)) != DP_OK) return st;   // the list lacks the formerly fixed cells
     return dp::call_end(*c, s);
   }
   const int n = c->n_own;
@@ -1253,6 +1276,7 @@ dp_status dp_set_fixed(dp_ctx *ctx, const uint8_t *h_fixed, const float *x, cons
   dp::launch_density_map(*c, x, y, s, nullptr, 1);
   DP_CUDA(cudaMemcpyAsync(c->d_rho_fixed, c->d_rho, sizeof(unsigned long long) * (size_t)c->mx * c->my,
                           cudaMemcpyDeviceToDevice, s));
+  if ((st = dp::request_sort(*c, s)) != DP_OK) return st;   // the list now holds the fixed cells
   DP_CUDA(cudaGetLastError());
   return dp::call_end(*c, s);
 }
@@ -1282,6 +1306,11 @@ dp_status dp_set_regions(dp_ctx *ctx, int32_t n_regions, const double *h_boxes, 
     c->gkey = dp::GraphKey{};
   }
   c->n_regions = 0;
+  {   // the list was built for one region pass: the next evaluation sorts
+    dp_status rs = dp::request_sort(*c, nullptr);
+    if (rs != DP_OK) return rs;
+    DP_CUDA(cudaDeviceSynchronize());
+  }
   if (n_regions == 0) return DP_OK;
   const int R = n_regions, n = c->n_own;
   const size_t nb = (size_t)c->mx * c->my;
@@ -1435,6 +1464,16 @@ dp_status dp_profile_read(dp_ctx *ctx, double *ms, int64_t *count) {
   }
   if (count) *count = c->prof_evals;
   c->prof_evals = 0;
+  return DP_OK;
+}
+
+dp_status dp_debug_sort_stats(dp_ctx *ctx, int32_t *out) {
+  Ctx *c = C(ctx);
+  if (!c || !out) return fail(DP_ERR_INVALID_ARG, "NULL argument");
+  dp::DeviceGuard g(c->device);
+  DP_CUDA(cudaEventSynchronize(c->ev_done));
+  DP_CUDA(cudaDeviceSynchronize());
+  DP_CUDA(cudaMemcpy(out, c->d_sortctl, 4 * sizeof(int32_t), cudaMemcpyDeviceToHost));
   return DP_OK;
 }
 

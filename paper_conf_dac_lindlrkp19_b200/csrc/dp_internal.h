@@ -55,7 +55,14 @@ constexpr int kWarpNetThreads = 256;  // warp-per-net kernel CTA size
 constexpr int kHpwlLimbs = 9;         // limbs 0..kHpwlLimbs (10) of 32-bit digits, LSB 2^-149 (reading A7)
 
 constexpr int kTile = 64;             // density tile = kTile x kTile bins (smaller maps: the map)
-constexpr int kHalo = 2;              // small-cell footprints extend <= 2 bins past their tile
+constexpr int kHalo = 2;              // small-cell footprints extend <= 2 bins past their first bin
+// the walkers' shared tiles extend kMargin bins past the tile on every side: a listed cell whose
+// first bin has drifted up to kMargin bins out of its tile since the sort still accumulates in
+// shared memory (even, so that the field tile's rows stay 16-byte aligned)
+#ifndef DP_MARGIN
+#define DP_MARGIN 2   // -DDP_MARGIN=m: A/B builds (0 / 2 / 4 measured)
+#endif
+constexpr int kMargin = DP_MARGIN;
 constexpr int kStageRecs = 512;       // records per staging buffer of the scatter/gather walkers
 // Tile bins accumulate each contribution v in (0, 1] as u = floor(v 2^29) in one native 32-bit
 // shared atomic (modulo 2^32; the thread whose add wraps carries 2^32 units to the int64 map).
@@ -180,7 +187,16 @@ struct Ctx {
   int32_t *d_tile_off = nullptr;      // [tiles + 1]
   float4 *d_rec = nullptr;            // per slot: footprint box in tile-local bin units
   int2 *d_rec_rc = nullptr;           // per slot: (charge ratio r as float bits, i0 | j0 << 16)
-  int32_t *d_rec_cell = nullptr;      // per slot: own cell index
+  int32_t *d_rec_cell = nullptr;      // per slot: own cell index (tile-ordered list, kept between sorts)
+  float2 *d_rec_wh = nullptr;         // per slot: (w, h) of the listed cell
+  // sort reuse: {re-sort requested, strays of the last evaluation, strays of this
+  // one, sorts performed}; the sort kernels run when a sort is requested or the last evaluation's
+  // strays (cells outside the tile they were listed in) exceed resort_thr
+  int32_t *d_sortctl = nullptr;
+  int32_t resort_thr = 0;
+  bool reuse_sort = true;             // DP_REUSE_SORT=0: sort on every evaluation (A/B)
+  bool sort_cond = true;              // DP_SORT_COND=0: no IF node in captured evaluations (kernels return early)
+  cudaStream_t s_body = nullptr;      // captures the body of the sort's IF node
   bool serial = false;
   bool use_graph = true;   // DP_GRAPH=0 disables the captured-graph evaluation path
   cudaStream_t s_cap = nullptr;
@@ -328,6 +344,7 @@ int density_walk_grid(int tile);
 int density_count_grid(int ntiles);
 int density_launches(const Ctx &c);
 void launch_region_overflow(const Ctx &c, cudaStream_t s);
+dp_status request_sort(Ctx &c, cudaStream_t s);   // the next evaluation rebuilds the tile-ordered list
 // NCCL (nccl_dyn.cpp)
 dp_status nccl_get_unique_id(void *out128);
 dp_status nccl_init(Ctx &c, const void *id);

@@ -506,18 +506,25 @@ __device__ __forceinline__ void rec_overlaps(const float4 q, float ox3[3], float
 // after).  Each word holds its bin's sum modulo 2^32 (units 2^-29); the wraps were already added
 // to rho by the threads whose atomic crossed 2^32, so rho + word is the exact int64 sum.
 __device__ __forceinline__ void flush_tile(const DenArgs &a, unsigned *s_acc, int tile) {
-  const int P = walk_span(a.tile);
+  const int P = walk_span(a.tile);   // even: word pairs (8-byte shared loads / stores)
   const int ox = (tile / a.tiles_y) * a.tile - kMargin, oy = (tile % a.tiles_y) * a.tile - kMargin;
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = blockDim.x >> 5;
+  uint2 *s2 = reinterpret_cast<uint2 *>(s_acc);
   for (int i = warp; i < P; i += nw) {
     const int gi = ox + i;
-    for (int j = lane; j < P; j += 32) {
-      const int k = i * P + j;
-      const unsigned long long v = (unsigned long long)s_acc[k];
-      s_acc[k] = 0u;
-      const int gj = oy + j;
-      if (v != 0ull && (unsigned)gi < (unsigned)a.mx && (unsigned)gj < (unsigned)a.my)
-        asm volatile("red.global.add.u64 [%0], %1;" ::"l"(a.rho + (size_t)gi * a.my + gj), "l"(v) : "memory");
+    const bool row_in = (unsigned)gi < (unsigned)a.mx;
+    for (int j2 = lane; j2 < P / 2; j2 += 32) {
+      const int k2 = i * (P / 2) + j2;
+      const uint2 v = s2[k2];
+      s2[k2] = make_uint2(0u, 0u);
+      const int gj = oy + 2 * j2;
+      if (row_in && (v.x | v.y)) {
+        unsigned long long *dst = a.rho + (size_t)gi * a.my + gj;
+        if (v.x && (unsigned)gj < (unsigned)a.my)
+          asm volatile("red.global.add.u64 [%0], %1;" ::"l"(dst), "l"((unsigned long long)v.x) : "memory");
+        if (v.y && (unsigned)(gj + 1) < (unsigned)a.my)
+          asm volatile("red.global.add.u64 [%0], %1;" ::"l"(dst + 1), "l"((unsigned long long)v.y) : "memory");
+      }
     }
   }
 }
@@ -527,6 +534,14 @@ __device__ __forceinline__ unsigned atom_shared_add(unsigned *p, unsigned v) {
   unsigned old;
   asm volatile("atom.shared.add.u32 %0, [%1], %2;" : "=r"(old) : "r"(smem_u32(p)), "r"(v) : "memory");
   return old;
+}
+
+// m <- 2 m + carry(old + u): the wrap mask of a record's nine adds in two instructions per add
+// (the carry out of the 32-bit sum, shifted in; the first add ends up in bit 8)
+__device__ __forceinline__ unsigned carry_in(unsigned m, unsigned old, unsigned u) {
+  unsigned t, r;
+  asm("{\n\tadd.cc.u32 %0, %2, %3;\n\taddc.u32 %1, %4, %4;\n\t}" : "=r"(t), "=r"(r) : "r"(old), "r"(u), "r"(m));
+  return r;
 }
 
 // D4: persistent scatter walker.  Each listed cell's footprint is formed here from its current
@@ -574,18 +589,22 @@ __global__ void __launch_bounds__(kTileThreads) k_scatter_walk(DenArgs a) {
   __syncthreads();
   const float scale_fx = (float)(1u << kRhoScaleLog2);
   int cur_tile = -1;
+  int tox = 0, toy = 0;   // origin of the shared tile (first bin of the tile - kMargin)
   unsigned strays = 0;
   WalkChunk cc = walk_next(a, w, st, 0);
   ScatterIn in = {0, make_float2(0.f, 0.f), 0.f, 0.f};
   scatter_fetch(a, st, 0, cc, in);
   for (int c = 0; cc.begin < cc.end; c++) {
     const int n = cc.end - cc.begin;
-    if (cur_tile < 0) cur_tile = cc.tile;
     if (cc.tile != cur_tile) {   // uniform: every warp sees the same chunks
-      __syncthreads();   // the tile is complete
-      flush_tile(a, s_acc, cur_tile);
-      __syncthreads();   // flushed and cleared
+      if (cur_tile >= 0) {
+        __syncthreads();   // the tile is complete
+        flush_tile(a, s_acc, cur_tile);
+        __syncthreads();   // flushed and cleared
+      }
       cur_tile = cc.tile;
+      tox = (cur_tile / a.tiles_y) * a.tile - kMargin;
+      toy = (cur_tile % a.tiles_y) * a.tile - kMargin;
     }
     // chunk c + 1 was issued (non-empty chunks c, c - 1, c - 2 refilled the ring): its entries and
     // positions are fetched now and arrive while this chunk is processed
@@ -594,7 +613,6 @@ __global__ void __launch_bounds__(kTileThreads) k_scatter_walk(DenArgs a) {
     const WalkChunk cn = st.ch[b1];
     ScatterIn nx = in;
     scatter_fetch(a, st, b1, cn, nx);
-    const int tox = (cur_tile / a.tiles_y) * a.tile - kMargin, toy = (cur_tile % a.tiles_y) * a.tile - kMargin;
     if ((int)threadIdx.x < n) {
       SmallFoot f;
       classify_small(a, in.x, in.y, in.wh.x, in.wh.y, f);   // listed cells are small with w h > 0
@@ -616,7 +634,7 @@ __global__ void __launch_bounds__(kTileThreads) k_scatter_walk(DenArgs a) {
         rec_overlaps(q, ox3, oy3);
         if (!stray) {
           const int base = i0 * P + j0;
-          unsigned wrapped = 0u;   // bit 3 di + dj: that word's add wrapped past 2^32
+          unsigned wrapped = 0u;   // bit 8 - (3 di + dj): that word's add wrapped past 2^32
 #pragma unroll
           for (int di = 0; di < 3; di++) {
             const float rx = r * ox3[di];
@@ -624,7 +642,7 @@ __global__ void __launch_bounds__(kTileThreads) k_scatter_walk(DenArgs a) {
             for (int dj = 0; dj < 3; dj++) {
               const unsigned u = (unsigned)(rx * oy3[dj]);   // floor(v 2^29) <= 2^29 (power-of-two scaling is exact)
               const unsigned old = atom_shared_add(s_acc + base + di * P + dj, u);
-              wrapped |= (old + u < old ? 1u : 0u) << (3 * di + dj);
+              wrapped = carry_in(wrapped, old, u);
             }
           }
           // wrapped words (rare): 2^32 units (8 bin areas) each go straight to the map.  Collected
@@ -632,7 +650,7 @@ __global__ void __launch_bounds__(kTileThreads) k_scatter_walk(DenArgs a) {
           // inside the loop, they were computed for all nine bins of every record)
           if (wrapped) {
             while (wrapped) {
-              const int bit = __ffs(wrapped) - 1;
+              const int bit = 8 - (__ffs(wrapped) - 1);   // add index 3 di + dj
               wrapped &= wrapped - 1;
               asm volatile("red.global.add.u64 [%0], %1;" ::"l"(a.rho + (size_t)(bi + bit / 3) * a.my + bj + bit % 3),
                            "l"(1ull << 32)

@@ -527,10 +527,15 @@ dp_status build_density(Ctx &c, const dp_netlist *nl) {
   {
     const int32_t ctl[4] = {1, 0, 0, 0};   // the first evaluation sorts
     DP_CUDA(cudaMemcpy(c.d_sortctl, ctl, sizeof(ctl), cudaMemcpyHostToDevice));
+    // DP_REUSE_SORT: 1 / 0 force; unset: reuse for contexts of >= 2^19 own cells.  Measured on the
+    // GP trajectory from the P:153 start: bigblue4 (2.18M cells) 418 -> 364 us per
+    // iteration with reuse, adaptec1 (211K cells, whose sort costs ~10 us) 114 -> 120 us
     const char *e = std::getenv("DP_REUSE_SORT");
-    c.reuse_sort = !(e && std::atoi(e) == 0);
+    c.reuse_sort = e ? std::atoi(e) != 0 : c.n_own >= (1 << 19);
+    // DP_SORT_COND=1: the sort kernels inside a graph IF node instead of returning early (measured
+    // equal at bigblue4, ~7 us slower per GP iteration at adaptec1)
     const char *ce = std::getenv("DP_SORT_COND");
-    c.sort_cond = !(ce && std::atoi(ce) == 0);
+    c.sort_cond = ce && std::atoi(ce) != 0;
     // re-sort once more than this share of the small cells has left its tile (DP_RESORT_PCT,
     // default 5 %: a stray costs its nine map updates as global reductions, a sort ~50 us)
     const char *pe = std::getenv("DP_RESORT_PCT");
@@ -606,6 +611,16 @@ void destroy(Ctx *c) {
   nccl_destroy(*c);
   for (void *p : c->allocations) cudaFree(p);
   if (c->d_hx) cudaFreeHost(c->d_hx);
+  if (c->s_h2d) cudaStreamSynchronize(c->s_h2d);
+  if (c->s_d2h) cudaStreamSynchronize(c->s_d2h);
+  for (int b = 0; b < 2; b++) {
+    if (c->ev_in_ready[b]) cudaEventDestroy(c->ev_in_ready[b]);
+    if (c->ev_in_free[b]) cudaEventDestroy(c->ev_in_free[b]);
+    if (c->ev_out_ready[b]) cudaEventDestroy(c->ev_out_ready[b]);
+    if (c->ev_out_free[b]) cudaEventDestroy(c->ev_out_free[b]);
+  }
+  if (c->s_h2d) cudaStreamDestroy(c->s_h2d);
+  if (c->s_d2h) cudaStreamDestroy(c->s_d2h);
   if (c->gexec) cudaGraphExecDestroy(c->gexec);
   if (c->s_cap) cudaStreamDestroy(c->s_cap);
   if (c->s_wa) cudaStreamDestroy(c->s_wa);
@@ -1415,6 +1430,70 @@ dp_status dp_eval_host(dp_ctx *ctx, const float *hx, const float *hy, float gamm
     h_scalars[2] = tmp[2];
     h_scalars[3] = with_hpwl ? tmp[3] : std::nan("");
   }
+  return DP_OK;
+}
+
+dp_status dp_eval_host_async(dp_ctx *ctx, const float *hx, const float *hy, float gamma, float lambda, float *hgx,
+                             float *hgy, double *h_scalars, int with_hpwl, dp_stream_t stream) {
+  Ctx *c = C(ctx);
+  if (!c) return fail(DP_ERR_INVALID_ARG, "ctx is NULL");
+  if (!hx || !hy || !hgx || !hgy) return fail(DP_ERR_INVALID_ARG, "host buffer is NULL");
+  if (!(gamma > 0.f) || !std::isfinite(gamma)) return fail(DP_ERR_INVALID_ARG, "gamma must be finite and > 0");
+  if (!(lambda >= 0.f) || !std::isfinite(lambda)) return fail(DP_ERR_INVALID_ARG, "lambda must be finite and >= 0");
+  dp::DeviceGuard g(c->device);
+  cudaStream_t s = (cudaStream_t)stream;
+  const size_t n = (size_t)c->num_cells;
+  if (!c->s_h2d) {   // first use: slots, copy streams, events
+    dp_status st;
+    for (int b = 0; b < 2; b++) {
+      if ((st = dp::dev_alloc(*c, &c->d_in2[b], 2 * n)) != DP_OK) return st;
+      if ((st = dp::dev_alloc(*c, &c->d_out2[b], 2 * n)) != DP_OK) return st;
+      if ((st = dp::dev_alloc(*c, &c->d_osc2[b], 4)) != DP_OK) return st;
+      DP_CUDA(cudaEventCreateWithFlags(&c->ev_in_ready[b], cudaEventDisableTiming));
+      DP_CUDA(cudaEventCreateWithFlags(&c->ev_in_free[b], cudaEventDisableTiming));
+      DP_CUDA(cudaEventCreateWithFlags(&c->ev_out_ready[b], cudaEventDisableTiming));
+      DP_CUDA(cudaEventCreateWithFlags(&c->ev_out_free[b], cudaEventDisableTiming));
+      DP_CUDA(cudaEventRecord(c->ev_in_free[b], s));
+      DP_CUDA(cudaEventRecord(c->ev_out_free[b], s));
+    }
+    DP_CUDA(cudaStreamCreateWithFlags(&c->s_h2d, cudaStreamNonBlocking));
+    DP_CUDA(cudaStreamCreateWithFlags(&c->s_d2h, cudaStreamNonBlocking));
+  }
+  const int b = (int)(c->async_k++ & 1);
+  // H2D of this call's positions into slot b once the call two back has moved them on
+  DP_CUDA(cudaStreamWaitEvent(c->s_h2d, c->ev_in_free[b], 0));
+  DP_CUDA(cudaMemcpyAsync(c->d_in2[b], hx, n * sizeof(float), cudaMemcpyHostToDevice, c->s_h2d));
+  DP_CUDA(cudaMemcpyAsync(c->d_in2[b] + n, hy, n * sizeof(float), cudaMemcpyHostToDevice, c->s_h2d));
+  DP_CUDA(cudaEventRecord(c->ev_in_ready[b], c->s_h2d));
+  // the evaluation reads the fixed input buffers (one captured graph for every call)
+  DP_CUDA(cudaStreamWaitEvent(s, c->ev_in_ready[b], 0));
+  DP_CUDA(cudaMemcpyAsync(c->d_hy, c->d_in2[b], 2 * n * sizeof(float), cudaMemcpyDeviceToDevice, s));
+  DP_CUDA(cudaEventRecord(c->ev_in_free[b], s));
+  double *sc = c->d_scal + 4;
+  dp_status st = dp::eval_impl(*c, c->d_hy, c->d_hy + n, gamma, lambda, c->d_hgx, c->d_hgy, sc + 0, sc + 1, sc + 2,
+                               with_hpwl ? sc + 3 : nullptr, s, true, true);
+  if (st != DP_OK) return st;
+  // results into output slot b once its previous D2H is done, then D2H on the copy stream
+  const size_t off = (size_t)c->cell_begin, cnt = (size_t)(c->cell_end - c->cell_begin);
+  DP_CUDA(cudaStreamWaitEvent(s, c->ev_out_free[b], 0));
+  DP_CUDA(cudaMemcpyAsync(c->d_out2[b] + off, c->d_hgx + off, cnt * sizeof(float), cudaMemcpyDeviceToDevice, s));
+  DP_CUDA(cudaMemcpyAsync(c->d_out2[b] + n + off, c->d_hgy + off, cnt * sizeof(float), cudaMemcpyDeviceToDevice, s));
+  DP_CUDA(cudaMemcpyAsync(c->d_osc2[b], sc, 4 * sizeof(double), cudaMemcpyDeviceToDevice, s));
+  DP_CUDA(cudaEventRecord(c->ev_out_ready[b], s));
+  DP_CUDA(cudaStreamWaitEvent(c->s_d2h, c->ev_out_ready[b], 0));
+  DP_CUDA(cudaMemcpyAsync(hgx + off, c->d_out2[b] + off, cnt * sizeof(float), cudaMemcpyDeviceToHost, c->s_d2h));
+  DP_CUDA(cudaMemcpyAsync(hgy + off, c->d_out2[b] + n + off, cnt * sizeof(float), cudaMemcpyDeviceToHost, c->s_d2h));
+  if (h_scalars) DP_CUDA(cudaMemcpyAsync(h_scalars, c->d_osc2[b], 4 * sizeof(double), cudaMemcpyDeviceToHost, c->s_d2h));
+  DP_CUDA(cudaEventRecord(c->ev_out_free[b], c->s_d2h));
+  return DP_OK;
+}
+
+dp_status dp_eval_host_wait(dp_ctx *ctx) {
+  Ctx *c = C(ctx);
+  if (!c) return fail(DP_ERR_INVALID_ARG, "ctx is NULL");
+  dp::DeviceGuard g(c->device);
+  if (c->s_h2d) DP_CUDA(cudaStreamSynchronize(c->s_h2d));
+  if (c->s_d2h) DP_CUDA(cudaStreamSynchronize(c->s_d2h));
   return DP_OK;
 }
 

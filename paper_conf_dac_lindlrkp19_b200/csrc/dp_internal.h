@@ -194,8 +194,8 @@ struct Ctx {
   // strays (cells outside the tile they were listed in) exceed resort_thr
   int32_t *d_sortctl = nullptr;
   int32_t resort_thr = 0;
-  bool reuse_sort = true;             // DP_REUSE_SORT=0: sort on every evaluation (A/B)
-  bool sort_cond = true;              // DP_SORT_COND=0: no IF node in captured evaluations (kernels return early)
+  bool reuse_sort = true;             // DP_REUSE_SORT=0/1 (default: >= 2^19 own cells): keep the list between sorts
+  bool sort_cond = false;             // DP_SORT_COND=1: the sort in an IF node of captured evaluations (A/B)
   cudaStream_t s_body = nullptr;      // captures the body of the sort's IF node
   bool serial = false;
   bool use_graph = true;   // DP_GRAPH=0 disables the captured-graph evaluation path
@@ -261,6 +261,13 @@ struct Ctx {
   unsigned long long *d_limbs = nullptr;  // HPWL fixed-point limbs
   double *d_scal = nullptr;           // {wl, energy, hpwl, obj} staging
   float *d_hx = nullptr, *d_hy = nullptr, *d_hgx = nullptr, *d_hgy = nullptr;  // e2e buffers
+  // dp_eval_host_async: two staging slots per direction (inputs x|y, outputs gx|gy + 4 scalars),
+  // a copy stream each way; allocated on first use
+  float *d_in2[2] = {nullptr, nullptr}, *d_out2[2] = {nullptr, nullptr};
+  double *d_osc2[2] = {nullptr, nullptr};
+  cudaStream_t s_h2d = nullptr, s_d2h = nullptr;
+  cudaEvent_t ev_in_ready[2] = {}, ev_in_free[2] = {}, ev_out_ready[2] = {}, ev_out_free[2] = {};
+  int64_t async_k = 0;
 
   // ---- streams / events ----
   cudaStream_t s_wa = nullptr, s_den = nullptr;

@@ -78,11 +78,13 @@ def _moves(nl, x, y, kind, seed=7):
 
 @pytest.mark.parametrize("name", ["tiny", "adaptec1"])
 @pytest.mark.parametrize("kind", ["jitter", "drift", "reshuffle", "collapse", "outside"])
-def test_stale_list_bit_identical(name, kind):
+@pytest.mark.parametrize("cond", [0, 1])
+def test_stale_list_bit_identical(name, kind, cond):
+    """cond = 1: the sort kernels inside a graph IF node (DP_SORT_COND=1), else early returns."""
     nl = make_netlist(name)
     x0, y0 = make_positions(nl)
     x1, y1 = _moves(nl, x0, y0, kind)
-    reuse = _ctx(nl, DP_RESORT_PCT=100)      # keeps the list of x0 whatever the strays
+    reuse = _ctx(nl, DP_REUSE_SORT=1, DP_RESORT_PCT=100, DP_SORT_COND=cond)   # keeps the list of x0
     fresh = _ctx(nl, DP_REUSE_SORT=0)
     _eval(reuse, x0, y0, nl)
     st0 = dp.dp_debug_sort_stats(reuse)
@@ -115,7 +117,7 @@ def test_resort_threshold():
     """The list is rebuilt on the evaluation after one with more strays than DP_RESORT_PCT."""
     nl = make_netlist("adaptec1")
     x0, y0 = make_positions(nl)
-    ctx = _ctx(nl, DP_RESORT_PCT=5)
+    ctx = _ctx(nl, DP_REUSE_SORT=1, DP_RESORT_PCT=5)
     _eval(ctx, x0, y0, nl)
     assert dp.dp_debug_sort_stats(ctx)["sorts"] == 1
     _eval(ctx, x0, y0, nl)                       # same positions: no strays, no sort
@@ -141,7 +143,7 @@ def test_bigblue4_trajectory_bit_identical():
     the oracle's force on the last step."""
     nl = make_netlist("bigblue4")
     x, y = make_positions(nl)
-    reuse = _ctx(nl)
+    reuse = _ctx(nl)                          # bigblue4: reuse by default
     fresh = _ctx(nl, DP_REUSE_SORT=0)
     rng = np.random.default_rng(11)
     for k in range(6):
@@ -159,7 +161,7 @@ def test_fixed_cells_and_regions_request_a_sort():
     listed set: each requests a sort, and the evaluations match a sort-every-time context."""
     nl = make_netlist("tiny")
     x, y = make_positions(nl)
-    reuse = _ctx(nl, DP_RESORT_PCT=100)
+    reuse = _ctx(nl, DP_REUSE_SORT=1, DP_RESORT_PCT=100)
     fresh = _ctx(nl, DP_REUSE_SORT=0)
     _same(_eval(reuse, x, y, nl), _eval(fresh, x, y, nl))
     fixed = np.zeros(nl.num_cells, dtype=np.uint8)
@@ -173,3 +175,13 @@ def test_fixed_cells_and_regions_request_a_sort():
         dp.dp_set_fixed(c, None, None, None)
     _same(_eval(reuse, x1, y1, nl), _eval(fresh, x1, y1, nl))
     assert dp.dp_debug_sort_stats(reuse)["sorts"] >= 3
+
+
+def test_reuse_default_by_size():
+    """Reuse is on by default from 2^19 own cells: adaptec1 sorts every time."""
+    nl = make_netlist("adaptec1")
+    x, y = make_positions(nl)
+    ctx = dp.dp_create(nl)
+    for _ in range(3):
+        ctx.eval(_t(x), _t(y), nl.bin_w, 1.0)
+    assert dp.dp_debug_sort_stats(ctx)["sorts"] == 3

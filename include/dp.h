@@ -203,6 +203,21 @@ dp_status dp_eval_host(dp_ctx *ctx, const float *hx, const float *hy, float gamm
                        float lambda, float *hgx, float *hgy, double *h_scalars,
                        int with_hpwl, dp_stream_t stream);
 
+/* Pipelined variant of dp_eval_host (the e2e path): enqueues the H2D copy of hx, hy (host,
+ * [num_cells], PINNED: the copies are asynchronous), the evaluation on `stream`, and the D2H copy
+ * of gx, gy (own cells) and of {obj, wl, energy, hpwl} into h_scalars (host PINNED double[4],
+ * nullable; hpwl is written only with with_hpwl) and returns without waiting.  Inputs and
+ * results pass through two device staging slots and two internal copy streams, so the H2D of
+ * call k + 1, the evaluation of call k and the D2H of call k - 1 overlap (PCIe is full duplex).
+ * The host buffers of a call must stay untouched until dp_eval_host_wait returns; calls on one
+ * context must come from one thread.  Errors as dp_eval_host (argument errors before anything is
+ * enqueued).                                                                                  */
+dp_status dp_eval_host_async(dp_ctx *ctx, const float *hx, const float *hy, float gamma,
+                             float lambda, float *hgx, float *hgy, double *h_scalars,
+                             int with_hpwl, dp_stream_t stream);
+/* Waits until every dp_eval_host_async call on ctx has delivered its results to the host.  */
+dp_status dp_eval_host_wait(dp_ctx *ctx);
+
 /* ---- GP loop --------------------------------------------------------
  * The global-placement iterations around the evaluation, entirely on the device: "the loop
  * that involves the computation of wirelength and density gradient, optimization engines,

@@ -20,6 +20,7 @@ from .build import LIB, build  # noqa: F401
 __all__ = [
     "DPError", "Context", "lib", "dp_create", "dp_create_dist", "dp_nccl_unique_id",
     "dp_partition_plan", "dp_eval", "dp_wl_grad", "dp_density_grad", "dp_hpwl", "dp_eval_host",
+    "dp_eval_host_async", "dp_eval_host_wait",
     "dp_get_info", "dp_debug_density_map", "dp_debug_fields", "dp_debug_transform", "dp_debug_wa_accumulator",
     "dp_debug_sharded_fields", "DP_T_DCT2", "DP_T_IDCT2", "DP_T_IDXST_IDCT", "DP_T_IDCT_IDXST", "EXPORTED_SYMBOLS",
     "dp_set_wl_model", "DP_WL_WA", "DP_WL_LSE", "GpParams", "GpLoop", "dp_gp_create", "dp_set_deterministic",
@@ -34,7 +35,7 @@ _STATUS = {0: "DP_OK", 1: "DP_ERR_INVALID_ARG", 2: "DP_ERR_UNSUPPORTED", 3: "DP_
 EXPORTED_SYMBOLS = [
     "dp_last_error", "dp_version", "dp_create", "dp_create_dist", "dp_nccl_unique_id",
     "dp_partition_plan", "dp_destroy", "dp_eval", "dp_wl_grad", "dp_density_grad", "dp_hpwl",
-    "dp_eval_host", "dp_get_info", "dp_debug_density_map", "dp_debug_fields", "dp_debug_transform",
+    "dp_eval_host", "dp_eval_host_async", "dp_eval_host_wait", "dp_get_info", "dp_debug_density_map", "dp_debug_fields", "dp_debug_transform",
     "dp_debug_wa_accumulator", "dp_debug_sharded_fields", "dp_debug_sort_stats", "dp_set_regions", "dp_profile_enable", "dp_profile_read", "dp_set_wl_model",
     "dp_gp_default_params", "dp_gp_create", "dp_gp_init", "dp_gp_run", "dp_gp_positions",
     "dp_gp_history", "dp_gp_destroy", "dp_gp_debug_state", "dp_set_deterministic", "dp_set_fixed",
@@ -105,6 +106,8 @@ def lib() -> ctypes.CDLL:
             "dp_density_grad": [P, P, P, P, P, P, P],
             "dp_hpwl": [P, P, P, P, P],
             "dp_eval_host": [P, P, P, ctypes.c_float, ctypes.c_float, P, P, P, ctypes.c_int, P],
+            "dp_eval_host_async": [P, P, P, ctypes.c_float, ctypes.c_float, P, P, P, ctypes.c_int, P],
+            "dp_eval_host_wait": [P],
             "dp_get_info": [P, ctypes.POINTER(DpInfo)],
             "dp_debug_density_map": [P, P, P, P, P],
             "dp_debug_fields": [P, P, P, P, P, P, P],
@@ -458,6 +461,17 @@ def dp_hpwl(ctx, x, y, d_hpwl, stream=None):
 def dp_eval_host(ctx, hx, hy, gamma, lam, hgx, hgy, h_scalars=None, with_hpwl=False, stream=None):
     _check(lib().dp_eval_host(ctx.handle, _ptr(hx), _ptr(hy), float(gamma), float(lam), _ptr(hgx), _ptr(hgy),
                               _ptr(h_scalars), int(bool(with_hpwl)), _stream(stream)))
+
+
+def dp_eval_host_async(ctx, hx, hy, gamma, lam, hgx, hgy, h_scalars=None, with_hpwl=False, stream=None):
+    """Pipelined dp_eval_host: host buffers (and h_scalars) must be pinned; results are valid after
+    dp_eval_host_wait(ctx)."""
+    _check(lib().dp_eval_host_async(ctx.handle, _ptr(hx), _ptr(hy), float(gamma), float(lam), _ptr(hgx),
+                                    _ptr(hgy), _ptr(h_scalars), int(bool(with_hpwl)), _stream(stream)))
+
+
+def dp_eval_host_wait(ctx):
+    _check(lib().dp_eval_host_wait(ctx.handle))
 
 
 def dp_get_info(ctx) -> DpInfo:

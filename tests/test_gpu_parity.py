@@ -277,6 +277,40 @@ def test_eval_host_e2e(tiny):
     check_vector("gx", gx, ref["gx"])
 
 
+@pytest.mark.parametrize("name", ["tiny", "adaptec1"])
+def test_eval_host_async_pipeline(name):
+    """dp_eval_host_async: six calls in flight on alternating staging slots, each with its own
+    positions and pinned result buffers, equal bit for bit (deterministic mode) to synchronous
+    dp_eval_host calls; the tiny case also against the oracle."""
+    nl = make_netlist(name)
+    ctx = dp.dp_create(nl)
+    dp.dp_set_deterministic(ctx, 1)
+    rng = np.random.default_rng(5)
+    x0, y0 = make_positions(nl)
+    pos = [((x0 + rng.normal(0, 2 * nl.bin_w, x0.shape)).astype(np.float32),
+            (y0 + rng.normal(0, 2 * nl.bin_h, y0.shape)).astype(np.float32)) for _ in range(6)]
+    hx = [torch.as_tensor(p[0]).pin_memory() for p in pos]
+    hy = [torch.as_tensor(p[1]).pin_memory() for p in pos]
+    out = [(torch.zeros(nl.num_cells).pin_memory(), torch.zeros(nl.num_cells).pin_memory(),
+            torch.zeros(4, dtype=torch.float64).pin_memory()) for _ in pos]
+    for k in range(len(pos)):
+        dp.dp_eval_host_async(ctx, hx[k], hy[k], nl.bin_w, 0.5, out[k][0], out[k][1], out[k][2], True)
+    dp.dp_eval_host_wait(ctx)
+    for k in range(len(pos)):
+        gx = np.zeros(nl.num_cells, np.float32)
+        gy = np.zeros(nl.num_cells, np.float32)
+        sc = np.zeros(4)
+        dp.dp_eval_host(ctx, pos[k][0], pos[k][1], nl.bin_w, 0.5, gx, gy, sc, with_hpwl=True)
+        assert np.array_equal(out[k][0].numpy(), gx) and np.array_equal(out[k][1].numpy(), gy), k
+        assert out[k][2].numpy().tolist() == sc.tolist(), k
+    if name == "tiny":
+        ref = oracle.evaluate(nl, pos[3][0], pos[3][1], nl.bin_w, 0.5)
+        check_scalar("obj", out[3][2][0].item(), ref["obj"])
+        assert out[3][2][3].item() == ref["hpwl"]
+        check_vector("gx", out[3][0].numpy(), ref["gx"])
+        check_vector("gy", out[3][1].numpy(), ref["gy"])
+
+
 @pytest.mark.slow
 @pytest.mark.parametrize("name", ["adaptec1", "bigblue4"])
 def test_eval_full_size(name):

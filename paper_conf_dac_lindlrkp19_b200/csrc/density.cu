@@ -62,6 +62,7 @@ struct DenArgs {
   // [0] or [1] > resort_thr, and return at once otherwise
   int *sortctl;
   int force_sort, resort_thr;
+  int write_rec;   // the scatter writes footprint records (the gather reads them; 0: it recomputes)
   unsigned long long *rho;   // int64 fixed point, 2^-kRhoScaleLog2 units
   const float2 *xi;
   float2 *force;
@@ -69,6 +70,10 @@ struct DenArgs {
   // direct output (DP_DIRECT): the gather adds lambda * dD/dx straight into the caller's gx, gy
   // (zeroed at the head of the call, the WA kernel adds into them too) instead of storing force
   float *gxo, *gyo;
+  // fused combine (DP_FUSE_COMBINE): the gather writes gx = g2.x + lambda force.x (the WA
+  // accumulator is complete: the gather waits for the WA stream) and no force / combine pass
+  float *gxf, *gyf;
+  const float2 *g2f;
   float lambda;
   const float *lambda_dev;
   // fixed cells (NEXT-4, dp_set_fixed): with a mask, only cells whose flag equals sel are
@@ -118,10 +123,10 @@ __device__ __forceinline__ Foot footprint(const DenArgs &a, int i) {
 }
 
 // Small-cell classification shared by count (D1), place (D3) and the scatter walker (D4), which
-// must agree exactly: returns -2 for a large cell (CTA-per-cell path), -3 for a cell of zero
-// area (never in the map), else the tile of the footprint's first bin clamped to the map; f.ok is
-// false for an empty footprint (outside the region: the cell stays listed, in the clamped tile,
-// so that it is found again when it moves back).  Only the lower corner (lx, ly) and the upper
+// must agree exactly: returns -2 for a large cell (CTA-per-cell path), else the tile of the
+// footprint's first bin clamped to the map; f.ok is false for an empty footprint (outside the
+// region or zero area: the cell stays listed, in the clamped tile, so that it is found again when
+// it moves back, and the gather writes its zero force).  Only the lower corner (lx, ly) and the upper
 // corner (hx, hy) are formed in fp64 (unclipped); ok equals footprint_v's "not empty" (hi > lo
 // after clipping to [0, M]) without fp64 min/max.
 struct SmallFoot {
@@ -133,14 +138,14 @@ struct SmallFoot {
 
 __device__ __forceinline__ int classify_small(const DenArgs &a, float x, float y, float w, float h, SmallFoot &f) {
   if (w > a.w_large || h > a.h_large) return -2;
-  if (!(w * h > 0.f)) return -3;
   f.ws = a.stretch ? fmaxf(w, a.sxf) : w;
   f.hs = a.stretch ? fmaxf(h, a.syf) : h;
   f.lx = fma((double)(0.5f * (w - f.ws)), a.ibx, fma((double)x, a.ibx, a.cx0));
   f.ly = fma((double)(0.5f * (h - f.hs)), a.iby, fma((double)y, a.iby, a.cy0));
   f.hx = fma((double)f.ws, a.ibx, f.lx);
   f.hy = fma((double)f.hs, a.iby, f.ly);
-  f.ok = f.hx > f.lx && f.hx > 0.0 && f.lx < (double)a.mx && f.hy > f.ly && f.hy > 0.0 && f.ly < (double)a.my;
+  f.ok = f.hx > f.lx && f.hx > 0.0 && f.lx < (double)a.mx && f.hy > f.ly && f.hy > 0.0 && f.ly < (double)a.my &&
+         w * h > 0.f;
   f.bi = max(0, min(__double2int_rz(f.lx), a.mx - 1));
   f.bj = max(0, min(__double2int_rz(f.ly), a.my - 1));
   return (f.bi >> a.tile_log2) * a.tiles_y + (f.bj >> a.tile_log2);
@@ -199,7 +204,8 @@ __global__ void __launch_bounds__(kCountThreads) k_count(DenArgs a) {
       SmallFoot f;
       const int i = i0 + k * kCountThreads + threadIdx.x;
       const int t = classify_small(a, x[k], y[k], w[k], h[k], f);
-      if (t >= 0 && (!MASK || (i < a.n_own && selected(a, i)))) atomicAdd(&s_hist[t], 1);
+      // (lanes past n_own load w = h = 0 and classify like a zero-area cell: not counted)
+      if (t >= 0 && i < a.n_own && (!MASK || selected(a, i))) atomicAdd(&s_hist[t], 1);
     }
   }
   __syncthreads();
@@ -296,7 +302,7 @@ __global__ void __launch_bounds__(kCountThreads) k_place(DenArgs a) {
       if (a.keep) continue;          // another region's cell: its own pass writes its force
       t = -3;
     }
-    if (t == -3) {   // never in the map (zero area / fixed): force 0, kept until the next sort
+    if (t == -3) {   // a fixed cell of an evaluation (never in the map): force 0, kept until the next sort
       a.force[i] = make_float2(0.f, 0.f);
       continue;
     }
@@ -573,6 +579,45 @@ __device__ __forceinline__ void scatter_fetch(const DenArgs &a, const StageS &st
   }
 }
 
+// The record of a listed cell at its current position, relative to a shared tile whose origin is
+// (tox, toy) and which takes first bins [0, span) per axis: fractions of the first bin q, charge
+// ratio rr, the first bin (tile-local, or absolute for a stray).  The scatter and the recomputing
+// gather form it with this one function, so both see the same footprint bit for bit.
+struct FootRec {
+  float4 q;
+  float rr;
+  int i0, j0;
+  bool ok, stray;
+};
+
+__device__ __forceinline__ FootRec make_rec(const DenArgs &a, const ScatterIn &in, int tox, int toy, int span) {
+  FootRec fr;
+  SmallFoot f;
+  classify_small(a, in.x, in.y, in.wh.x, in.wh.y, f);   // listed cells are small
+  fr.q = make_float4(0.f, 0.f, 0.f, 0.f);
+  fr.rr = 0.f;
+  fr.i0 = fr.j0 = 0;
+  fr.ok = f.ok;
+  fr.stray = false;
+  if (f.ok) {
+    const int bi = f.bi, bj = f.bj;
+    // bin-local fractions (|v| < 3) of the clipped footprint [max(l, 0), min(h, M)]: fp32 keeps
+    // ~2e-7 bin absolute precision, which the force gather needs where large opposite bin
+    // fields cancel (the 'initial' placement).  fl(max(l, 0) - b) = max(fl(l - b), -b)
+    fr.q = make_float4(fmaxf((float)(f.lx - bi), (float)-bi), fmaxf((float)(f.ly - bj), (float)-bj),
+                       fminf((float)(f.hx - bi), (float)(a.mx - bi)), fminf((float)(f.hy - bj), (float)(a.my - bj)));
+    fr.rr = __fdividef(in.wh.x * in.wh.y, f.ws * f.hs);
+    fr.i0 = bi - tox;
+    fr.j0 = bj - toy;
+    fr.stray = (unsigned)fr.i0 >= (unsigned)span || (unsigned)fr.j0 >= (unsigned)span;
+    if (fr.stray) {
+      fr.i0 = bi;
+      fr.j0 = bj;
+    }
+  }
+  return fr;
+}
+
 __global__ void __launch_bounds__(kTileThreads) k_scatter_walk(DenArgs a) {
   griddep_wait();
   extern __shared__ __align__(16) unsigned char dsm[];
@@ -614,21 +659,14 @@ __global__ void __launch_bounds__(kTileThreads) k_scatter_walk(DenArgs a) {
     ScatterIn nx = in;
     scatter_fetch(a, st, b1, cn, nx);
     if ((int)threadIdx.x < n) {
-      SmallFoot f;
-      classify_small(a, in.x, in.y, in.wh.x, in.wh.y, f);   // listed cells are small with w h > 0
-      float4 q = make_float4(0.f, 0.f, 0.f, 0.f);
-      int2 rc = make_int2(0, 0);
-      if (f.ok) {
-        const int bi = f.bi, bj = f.bj;
-        // bin-local fractions (|v| < 3) of the clipped footprint [max(l, 0), min(h, M)]: fp32 keeps
-        // ~2e-7 bin absolute precision, which the force gather needs where large opposite bin
-        // fields cancel (the 'initial' placement).  fl(max(l, 0) - b) = max(fl(l - b), -b)
-        q = make_float4(fmaxf((float)(f.lx - bi), (float)-bi), fmaxf((float)(f.ly - bj), (float)-bj),
-                        fminf((float)(f.hx - bi), (float)(a.mx - bi)), fminf((float)(f.hy - bj), (float)(a.my - bj)));
-        const float rr = __fdividef(in.wh.x * in.wh.y, f.ws * f.hs);
-        const int i0 = bi - tox, j0 = bj - toy;
-        const bool stray = (unsigned)i0 >= (unsigned)span || (unsigned)j0 >= (unsigned)span;
-        rc = make_int2(__float_as_int(rr), stray ? (int)(bi | (bj << 16) | 0x80000000u) : (i0 | (j0 << 16)));
+      const FootRec fr = make_rec(a, in, tox, toy, span);
+      const float4 q = fr.q;
+      const int2 rc = make_int2(__float_as_int(fr.rr), fr.stray ? (int)(fr.i0 | (fr.j0 << 16) | 0x80000000u)
+                                                                : (fr.i0 | (fr.j0 << 16)));
+      if (fr.ok) {
+        const bool stray = fr.stray;
+        const int i0 = fr.i0, j0 = fr.j0, bi = fr.i0 + (stray ? 0 : tox), bj = fr.j0 + (stray ? 0 : toy);
+        const float rr = fr.rr;
         const float r = rr * scale_fx;   // r 2^29
         float ox3[3], oy3[3];
         rec_overlaps(q, ox3, oy3);
@@ -673,8 +711,10 @@ __global__ void __launch_bounds__(kTileThreads) k_scatter_walk(DenArgs a) {
           }
         }
       }
-      a.rec[cc.begin + threadIdx.x] = q;
-      a.rec_rc[cc.begin + threadIdx.x] = rc;
+      if (a.write_rec) {   // the records of the record-reading gather
+        a.rec[cc.begin + threadIdx.x] = q;
+        a.rec_rc[cc.begin + threadIdx.x] = rc;
+      }
     }
     walk_release(st, c);
     cc = walk_next(a, w, st, c + 1);   // landed already; thread 0 refills the ring
@@ -686,9 +726,68 @@ __global__ void __launch_bounds__(kTileThreads) k_scatter_walk(DenArgs a) {
   if ((threadIdx.x & 31) == 0 && strays) atomicAdd(a.sortctl + 2, (int)strays);
 }
 
+// sum over the record's 3x3 bins of ov(bin) xi(bin), from the shared field tile (first bin
+// (i0, j0) tile-local) or, for a stray, the global field (absolute first bin); bins without
+// overlap are not read (those past the map have none)
+__device__ __forceinline__ float2 field_sum(const DenArgs &a, const float2 *s_xi, int P, float4 q, bool stray, int i0,
+                                            int j0) {
+  float ox3[3], oy3[3];
+  rec_overlaps(q, ox3, oy3);
+  float fx = 0.f, fy = 0.f;
+  if (!stray) {
+    const float2 *row = s_xi + i0 * P + j0;   // in bounds: i0, j0 < tile + 2 kMargin, P = that + 2
+#pragma unroll
+    for (int di = 0; di < 3; di++) {
+      float sx = 0.f, sy = 0.f;
+#pragma unroll
+      for (int dj = 0; dj < 3; dj++) {
+        const float2 e2 = (ox3[di] > 0.f && oy3[dj] > 0.f) ? row[di * P + dj] : make_float2(0.f, 0.f);
+        sx = fmaf(oy3[dj], e2.x, sx);
+        sy = fmaf(oy3[dj], e2.y, sy);
+      }
+      fx = fmaf(ox3[di], sx, fx);
+      fy = fmaf(ox3[di], sy, fy);
+    }
+  } else {
+    const float2 *row = a.xi + (size_t)i0 * a.my + j0;
+#pragma unroll
+    for (int di = 0; di < 3; di++) {
+      float sx = 0.f, sy = 0.f;
+#pragma unroll
+      for (int dj = 0; dj < 3; dj++) {
+        const float2 e2 = (ox3[di] > 0.f && oy3[dj] > 0.f) ? row[(size_t)di * a.my + dj] : make_float2(0.f, 0.f);
+        sx = fmaf(oy3[dj], e2.x, sx);
+        sy = fmaf(oy3[dj], e2.y, sy);
+      }
+      fx = fmaf(ox3[di], sx, fx);
+      fy = fmaf(ox3[di], sy, fy);
+    }
+  }
+  return make_float2(fx, fy);
+}
+
+// (gather) the force of one cell: fused combine, direct output or the force vector
+__device__ __forceinline__ void gather_out(const DenArgs &a, int cell, float lam, float area, float r, float fx,
+                                           float fy) {
+  // dD/dx = - r sum_b ov(i,b) xi^X_b  (reading A21), ov in length^2
+  if (a.gxf) {   // fused combine: exactly k_combine's fmaf(lambda, force, g2)
+    const int gc = a.cell_begin + cell;
+    const float2 g = a.g2f[gc];
+    a.gxf[gc] = fmaf(lam, -area * r * fx, g.x);
+    a.gyf[gc] = fmaf(lam, -area * r * fy, g.y);
+  } else if (a.gxo) {
+    const int gc = a.cell_begin + cell;
+    red_f32(a.gxo + gc, lam * (-area * r * fx));
+    red_f32(a.gyo + gc, lam * (-area * r * fy));
+  } else {
+    a.force[cell] = make_float2(-area * r * fx, -area * r * fy);
+  }
+}
+
 // D5: persistent gather walker; the (tile+2)^2 float2 field tile is (re)loaded with one bulk copy
 // per tile row whenever the slice enters a tile; bins outside the map read as zero.
-__device__ __forceinline__ void load_xi_tile(const DenArgs &a, StageG &st, float2 *s_xi, int tile,
+template <class St>
+__device__ __forceinline__ void load_xi_tile(const DenArgs &a, St &st, float2 *s_xi, int tile,
                                              unsigned phase) {
   const int P = walk_span(a.tile);
   const int ox = (tile / a.tiles_y) * a.tile - kMargin, oy = (tile % a.tiles_y) * a.tile - kMargin;
@@ -743,52 +842,65 @@ __global__ void __launch_bounds__(kTileThreads) k_gather_walk(DenArgs a) {
       const float4 q = B.rec[cc.off + k];
       const int2 rc = B.rc[cc.off + k];
       const float r = __int_as_float(rc.x);
-      float ox3[3], oy3[3];
-      rec_overlaps(q, ox3, oy3);
-      float fx = 0.f, fy = 0.f;
-      if (rc.y >= 0) {
-        const int i0 = rc.y & 0xffff, j0 = rc.y >> 16;
-        const float2 *row = s_xi + i0 * P + j0;
-#pragma unroll
-        for (int di = 0; di < 3; di++) {
-          float sx = 0.f, sy = 0.f;
-#pragma unroll
-          for (int dj = 0; dj < 3; dj++) {
-            // in-bounds: i0, j0 < tile + 2 kMargin, P = that + 2; bins without overlap are not read
-            const float2 e2 = (ox3[di] > 0.f && oy3[dj] > 0.f) ? row[di * P + dj] : make_float2(0.f, 0.f);
-            sx = fmaf(oy3[dj], e2.x, sx);
-            sy = fmaf(oy3[dj], e2.y, sy);
-          }
-          fx = fmaf(ox3[di], sx, fx);
-          fy = fmaf(ox3[di], sy, fy);
-        }
-      } else {   // stray (left its tile since the sort): the same sums from the global field
-        const int i0 = rc.y & 0xffff, j0 = (rc.y >> 16) & 0x7fff;
-        const float2 *row = a.xi + (size_t)i0 * a.my + j0;
-#pragma unroll
-        for (int di = 0; di < 3; di++) {
-          float sx = 0.f, sy = 0.f;
-#pragma unroll
-          for (int dj = 0; dj < 3; dj++) {
-            // bins past the map have zero overlap and are not read
-            const float2 e2 = (ox3[di] > 0.f && oy3[dj] > 0.f) ? row[(size_t)di * a.my + dj] : make_float2(0.f, 0.f);
-            sx = fmaf(oy3[dj], e2.x, sx);
-            sy = fmaf(oy3[dj], e2.y, sy);
-          }
-          fx = fmaf(ox3[di], sx, fx);
-          fy = fmaf(ox3[di], sy, fy);
-        }
-      }
-      // dD/dx = - r sum_b ov(i,b) xi^X_b  (reading A21), ov in length^2
-      if (a.gxo) {
-        const int gc = a.cell_begin + B.cell[cc.off + k];
-        red_f32(a.gxo + gc, lam * (-area * r * fx));
-        red_f32(a.gyo + gc, lam * (-area * r * fy));
-      } else {
-        a.force[B.cell[cc.off + k]] = make_float2(-area * r * fx, -area * r * fy);
-      }
+      const bool stray = rc.y < 0;
+      const float2 fs = field_sum(a, s_xi, P, q, stray, rc.y & 0xffff, (rc.y >> 16) & 0x7fff);
+      const float fx = fs.x, fy = fs.y;
+      gather_out(a, B.cell[cc.off + k], lam, area, r, fx, fy);
     }
     walk_release(st, c);
+  }
+}
+
+// D5' (DP_GATHER_RC): the gather walker recomputes each listed cell's footprint from its position
+// (make_rec, as the scatter did) instead of reading the scatter's records: it stages the 12-byte
+// list entries and prefetches the positions one chunk ahead like the scatter; no record traffic.
+int gather_rc_smem_bytes(int tile) { return stage_bytes<StageS>() + walk_span(tile) * walk_span(tile) * 8; }
+
+__global__ void __launch_bounds__(kTileThreads) k_gather_walk_rc(DenArgs a) {
+  griddep_wait();
+  extern __shared__ __align__(16) unsigned char dsm[];
+  StageS &st = *reinterpret_cast<StageS *>(dsm);
+  float2 *s_xi = reinterpret_cast<float2 *>(dsm + stage_bytes<StageS>());
+  const int P = walk_span(a.tile);
+  const int span = a.tile + 2 * kMargin;
+  Walker w;
+  if (threadIdx.x == 0) {
+    if (blockIdx.x == 0) {   // the scatter has completed: its stray count decides the next sort
+      a.sortctl[1] = a.sortctl[2];
+      a.sortctl[2] = 0;
+    }
+    walk_start(a, w, st);
+  }
+  __syncthreads();   // barriers initialised, first descriptors visible
+  int cur_tile = -1, tox = 0, toy = 0;
+  unsigned xi_phase = 0;
+  const float area = (float)(a.bx * a.by);
+  const float lam = a.lambda_dev ? __ldg(a.lambda_dev) : a.lambda;
+  WalkChunk cc = walk_next(a, w, st, 0);
+  ScatterIn in = {0, make_float2(0.f, 0.f), 0.f, 0.f};
+  scatter_fetch(a, st, 0, cc, in);
+  for (int c = 0; cc.begin < cc.end; c++) {
+    const int n = cc.end - cc.begin;
+    if (cc.tile != cur_tile) {   // uniform; load_xi_tile's barrier waits until every warp left the old tile
+      load_xi_tile(a, st, s_xi, cc.tile, xi_phase);
+      xi_phase ^= 1u;
+      cur_tile = cc.tile;
+      tox = (cur_tile / a.tiles_y) * a.tile - kMargin;
+      toy = (cur_tile % a.tiles_y) * a.tile - kMargin;
+    }
+    const int b1 = (c + 1) % kStages;   // chunk c + 1: entries and positions fetched ahead
+    mbar_wait(&st.bar[b1], ((c + 1) / kStages) & 1);
+    const WalkChunk cn = st.ch[b1];
+    ScatterIn nx = in;
+    scatter_fetch(a, st, b1, cn, nx);
+    if ((int)threadIdx.x < n) {
+      const FootRec fr = make_rec(a, in, tox, toy, span);
+      const float2 fs = fr.ok ? field_sum(a, s_xi, P, fr.q, fr.stray, fr.i0, fr.j0) : make_float2(0.f, 0.f);
+      gather_out(a, in.cell, lam, area, fr.rr, fs.x, fs.y);
+    }
+    walk_release(st, c);
+    cc = walk_next(a, w, st, c + 1);
+    in = nx;
   }
 }
 
@@ -848,7 +960,13 @@ __global__ void __launch_bounds__(256) k_gather_large(DenArgs a) {
     }
     const double area = a.bx * a.by;   // overlaps above are in bin units
     const float2 v = make_float2((float)(-(double)f.r * area * tx), (float)(-(double)f.r * area * ty));
-    if (a.gxo) {
+    if (a.gxf) {
+      const float lam = a.lambda_dev ? __ldg(a.lambda_dev) : a.lambda;
+      const int gc = a.cell_begin + i;
+      const float2 g = a.g2f[gc];
+      a.gxf[gc] = fmaf(lam, v.x, g.x);
+      a.gyf[gc] = fmaf(lam, v.y, g.y);
+    } else if (a.gxo) {
       const float lam = a.lambda_dev ? __ldg(a.lambda_dev) : a.lambda;
       red_f32(a.gxo + a.cell_begin + i, lam * v.x);
       red_f32(a.gyo + a.cell_begin + i, lam * v.y);
@@ -935,12 +1053,16 @@ DenArgs make_args(const Ctx &c, const float *x, const float *y) {
   a.rec_wh = c.d_rec_wh;
   a.sortctl = c.d_sortctl;
   a.force_sort = c.reuse_sort ? 0 : 1;
+  a.write_rec = c.gather_rc ? 0 : 1;
   a.resort_thr = c.resort_thr;
   a.rho = c.d_rho;
   a.xi = c.d_xi;
   a.force = c.d_force;
   a.gxo = c.direct_gx;
   a.gyo = c.direct_gy;
+  a.gxf = c.fused_gx;
+  a.gyf = c.fused_gy;
+  a.g2f = c.d_g2;
   a.lambda = c.direct_lambda;
   a.lambda_dev = c.lambda_dev;
   a.large = c.d_large;
@@ -976,6 +1098,8 @@ cudaError_t density_configure(int ntiles, int tile) {
   e = cudaFuncSetAttribute(k_place<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, place_smem_bytes(ntiles));
   if (e != cudaSuccess) return e;
   e = cudaFuncSetAttribute(k_scatter_walk, cudaFuncAttributeMaxDynamicSharedMemorySize, scatter_smem_bytes(tile));
+  if (e != cudaSuccess) return e;
+  e = cudaFuncSetAttribute(k_gather_walk_rc, cudaFuncAttributeMaxDynamicSharedMemorySize, gather_rc_smem_bytes(tile));
   if (e != cudaSuccess) return e;
   return cudaFuncSetAttribute(k_gather_walk, cudaFuncAttributeMaxDynamicSharedMemorySize, walk_smem_bytes(tile));
 }
@@ -1117,7 +1241,10 @@ void launch_density_gather(const Ctx &c, const float *x, const float *y, cudaStr
     k_gather_large<<<a.n_large, 256, 0, aux>>>(a);
     cudaEventRecord(c.ev_aux_b, aux);
   }
-  if (c.n_own > 0) launch_chain(c.pdl, k_gather_walk, c.walk_grid, kTileThreads, walk_smem_bytes(c.tile), s, a);
+  if (c.n_own > 0 && c.gather_rc)
+    launch_chain(c.pdl, k_gather_walk_rc, c.walk_grid, kTileThreads, gather_rc_smem_bytes(c.tile), s, a);
+  else if (c.n_own > 0)
+    launch_chain(c.pdl, k_gather_walk, c.walk_grid, kTileThreads, walk_smem_bytes(c.tile), s, a);
   if (side)
     cudaStreamWaitEvent(s, c.ev_aux_b, 0);
   else if (a.n_large > 0)

@@ -534,6 +534,10 @@ dp_status build_density(Ctx &c, const dp_netlist *nl) {
     c.reuse_sort = e ? std::atoi(e) != 0 : c.n_own >= (1 << 19);
     // DP_SORT_COND=1: the sort kernels inside a graph IF node instead of returning early (measured
     // equal at bigblue4, ~7 us slower per GP iteration at adaptec1)
+    const char *ge = std::getenv("DP_GATHER_RC");
+    c.gather_rc = ge && std::atoi(ge) != 0;
+    const char *fe = std::getenv("DP_FUSE_COMBINE");
+    c.fuse_combine = fe && std::atoi(fe) != 0;
     const char *ce = std::getenv("DP_SORT_COND");
     c.sort_cond = ce && std::atoi(ce) != 0;
     // re-sort once more than this share of the small cells has left its tile (DP_RESORT_PCT,
@@ -815,6 +819,7 @@ dp_status create(const dp_netlist *nl, const dp_grid *grid, int device, int rank
   const int wa_k = (c->n_chunks + c->n_big > 0) ? 1 : 0;   // one kernel: big nets, warp nets, chunks
   c->launches_eval = wa_k + density_launches(*c) + ((c->fft_cta || c->fft_hybrid) ? 3 : c->fused_t2 ? 3 : 4) /* P1 P2 P3, T1 P2 T3 or T1 T2a T2b T3 */ + 2 /* combine, finalize */;
   if (c->wa_split && wa_k) c->launches_eval += 1;   // the WA kernel in two launches
+  if (c->fuse_combine && !c->dist) c->launches_eval -= 1;   // no combine pass (default configuration)
   c->launches_eval_hpwl = c->launches_eval;
   if (c->dist && nccl_id) {
     if ((st = nccl_init(*c, nccl_id)) != DP_OK) return bail(st);
@@ -888,12 +893,13 @@ dp_status sharded_fields(Ctx &c, cudaStream_t s) {
   return nccl_all_gather_bytes(c, c.d_xi, nb / G * sizeof(float2), s);
 }
 
-dp_status density_chain_pass(Ctx &c, const float *x, const float *y);
+dp_status density_chain_pass(Ctx &c, const float *x, const float *y, bool with_gather = true);
 
 // the density chain; with fence regions (NEXT-4, reading A38) one pass per region, each with its
-// own map (from the region's blockage map), Poisson solve (its own energy slots) and gather
-dp_status density_chain(Ctx &c, const float *x, const float *y) {
-  if (c.n_regions == 0) return density_chain_pass(c, x, y);
+// own map (from the region's blockage map), Poisson solve (its own energy slots) and gather.
+// with_gather = false (fused combine): map and fields only, the caller launches the gather
+dp_status density_chain(Ctx &c, const float *x, const float *y, bool with_gather = true) {
+  if (c.n_regions == 0) return density_chain_pass(c, x, y, with_gather);
   for (int r = 0; r <= c.n_regions; r++) {
     c.cur_region = r;
     const dp_status st = density_chain_pass(c, x, y);
@@ -903,7 +909,7 @@ dp_status density_chain(Ctx &c, const float *x, const float *y) {
   return DP_OK;
 }
 
-dp_status density_chain_pass(Ctx &c, const float *x, const float *y) {
+dp_status density_chain_pass(Ctx &c, const float *x, const float *y, bool with_gather) {
   {
     StageMark m(c, DP_STAGE_MAP, c.s_den);
     launch_density_map(c, x, y, c.s_den, c.s_aux);
@@ -926,6 +932,7 @@ dp_status density_chain_pass(Ctx &c, const float *x, const float *y) {
     }
   }
   if (c.wa_split) DP_CUDA(cudaEventRecord(c.ev_fields, c.s_den));
+  if (!with_gather) return DP_OK;
   StageMark m(c, DP_STAGE_GATHER, c.s_den);
   launch_density_gather(c, x, y, c.s_den, c.s_aux);
   return DP_OK;
@@ -1044,6 +1051,13 @@ dp_status eval_body(Ctx &c, const float *x, const float *y, float gamma, float l
   c.direct_gx = direct ? gx : nullptr;
   c.direct_gy = direct ? gy : nullptr;
   c.direct_lambda = lambda;
+  // fused combine (DP_FUSE_COMBINE=1): the gather waits for the WA stream and writes gx, gy itself
+  const bool fused = c.fuse_combine && !direct && do_wa && do_den && !c.deterministic && !c.dist && !c.has_fixed &&
+                     c.n_regions == 0 && !c.wa_split;
+  struct FusedReset {
+    Ctx &c;
+    ~FusedReset() { c.fused_gx = c.fused_gy = nullptr; }
+  } fused_reset{c};
   const size_t gbytes = sizeof(float) * (size_t)c.num_cells;
   DP_CUDA(cudaEventRecord(c.ev_fork, s));
   if (do_den) {
@@ -1052,9 +1066,9 @@ dp_status eval_body(Ctx &c, const float *x, const float *y, float gamma, float l
       DP_CUDA(cudaMemsetAsync(gx, 0, gbytes, c.s_den));
       DP_CUDA(cudaMemsetAsync(gy, 0, gbytes, c.s_den));
     }
-    dp_status st = density_chain(c, x, y);
+    dp_status st = density_chain(c, x, y, !fused);
     if (st != DP_OK) return st;
-    DP_CUDA(cudaEventRecord(c.ev_den, c.s_den));
+    if (!fused) DP_CUDA(cudaEventRecord(c.ev_den, c.s_den));
   }
   if (do_wa) {
     DP_CUDA(cudaStreamWaitEvent(
@@ -1096,6 +1110,17 @@ dp_status eval_body(Ctx &c, const float *x, const float *y, float gamma, float l
     }
     DP_CUDA(cudaEventRecord(c.ev_wa, c.s_wa));
   }
+  if (fused) {   // the gather after the fields and the complete WA accumulator
+    DP_CUDA(cudaStreamWaitEvent(c.s_den, c.ev_wa, 0));
+    c.fused_gx = gx;
+    c.fused_gy = gy;
+    {
+      StageMark m(c, DP_STAGE_GATHER, c.s_den);
+      launch_density_gather(c, x, y, c.s_den, c.s_aux);
+    }
+    c.fused_gx = c.fused_gy = nullptr;
+    DP_CUDA(cudaEventRecord(c.ev_den, c.s_den));
+  }
   if (do_wa) DP_CUDA(cudaStreamWaitEvent(s, c.ev_wa, 0));
   if (do_den) DP_CUDA(cudaStreamWaitEvent(s, c.ev_den, 0));
   {
@@ -1111,7 +1136,7 @@ dp_status eval_body(Ctx &c, const float *x, const float *y, float gamma, float l
           finalize(c, lambda, do_wa, do_den, do_wa && d_hpwl != nullptr, d_obj, d_wl, d_energy, d_hpwl, c.s_aux);
       if (st != DP_OK) return st;
       DP_CUDA(cudaEventRecord(c.ev_fin, c.s_aux));
-      if (!direct) launch_combine(c, do_den ? lambda : 0.f, gx, gy, do_wa, do_den, s);
+      if (!direct && !fused) launch_combine(c, do_den ? lambda : 0.f, gx, gy, do_wa, do_den, s);
       DP_CUDA(cudaStreamWaitEvent(s, c.ev_fin, 0));
     }
   }

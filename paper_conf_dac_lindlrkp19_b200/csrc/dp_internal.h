@@ -195,6 +195,7 @@ struct Ctx {
   int32_t *d_sortctl = nullptr;
   int32_t resort_thr = 0;
   bool reuse_sort = true;             // DP_REUSE_SORT=0/1 (default: >= 2^19 own cells): keep the list between sorts
+  bool gather_rc = false;             // DP_GATHER_RC=1: the gather recomputes footprints (no records)
   bool sort_cond = false;             // DP_SORT_COND=1: the sort in an IF node of captured evaluations (A/B)
   cudaStream_t s_body = nullptr;      // captures the body of the sort's IF node
   bool serial = false;
@@ -208,6 +209,8 @@ struct Ctx {
   bool pdl = true;                // programmatic dependent launch along the density chain (DP_PDL=0: off)
   bool direct = false;            // DP_DIRECT=1: WA and gather add into the caller's gx, gy (no combine pass)
   float *direct_gx = nullptr, *direct_gy = nullptr;   // set for the duration of one eval_body
+  bool fuse_combine = false;      // DP_FUSE_COMBINE=1: the gather waits for WA and writes gx, gy (no combine pass)
+  float *fused_gx = nullptr, *fused_gy = nullptr;     // set for the duration of one eval_body
   float direct_lambda = 0.f;
   int det_frac = 30;              // its units 2^-det_frac (>= every chunk's slot scale in practice: exact shifts)
   long long *d_g2i = nullptr;     // [2 num_cells] int64 WA gradient (allocated on first enable)

@@ -328,7 +328,9 @@ def test_eval_full_size(name):
     check_vector("gy", to_np(out["gy"]), ref["gy"])
 
 
-@pytest.mark.parametrize("env", [{"DP_WA_SPLIT": "50"}, {"DP_FFT": "2"}, {"DP_FFT": "1"}])
+@pytest.mark.parametrize("env", [{"DP_WA_SPLIT": "50"}, {"DP_FFT": "2"}, {"DP_FFT": "1"}, {"DP_FUSE_COMBINE": "1"},
+                                 {"DP_FUSE_COMBINE": "1", "DP_REUSE_SORT": "1"}, {"DP_GATHER_RC": "1"},
+                                 {"DP_GATHER_RC": "1", "DP_REUSE_SORT": "1", "DP_FUSE_COMBINE": "1"}])
 def test_schedule_switches_match(env):
     """The measured-and-off A/B switches of the evaluation schedule compute the
     same evaluation: the WA launch split around the transforms (the same work units and partial

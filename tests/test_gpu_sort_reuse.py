@@ -78,13 +78,14 @@ def _moves(nl, x, y, kind, seed=7):
 
 @pytest.mark.parametrize("name", ["tiny", "adaptec1"])
 @pytest.mark.parametrize("kind", ["jitter", "drift", "reshuffle", "collapse", "outside"])
-@pytest.mark.parametrize("cond", [0, 1])
-def test_stale_list_bit_identical(name, kind, cond):
-    """cond = 1: the sort kernels inside a graph IF node (DP_SORT_COND=1), else early returns."""
+@pytest.mark.parametrize("cond,rc", [(0, 0), (1, 0), (0, 1)])
+def test_stale_list_bit_identical(name, kind, cond, rc):
+    """cond = 1: the sort kernels inside a graph IF node (DP_SORT_COND=1), else early returns;
+    rc = 1: the gather recomputes the footprints instead of reading the scatter's records."""
     nl = make_netlist(name)
     x0, y0 = make_positions(nl)
     x1, y1 = _moves(nl, x0, y0, kind)
-    reuse = _ctx(nl, DP_REUSE_SORT=1, DP_RESORT_PCT=100, DP_SORT_COND=cond)   # keeps the list of x0
+    reuse = _ctx(nl, DP_REUSE_SORT=1, DP_RESORT_PCT=100, DP_SORT_COND=cond, DP_GATHER_RC=rc)   # keeps the list of x0
     fresh = _ctx(nl, DP_REUSE_SORT=0)
     _eval(reuse, x0, y0, nl)
     st0 = dp.dp_debug_sort_stats(reuse)

@@ -186,3 +186,26 @@ def test_reuse_default_by_size():
     for _ in range(3):
         ctx.eval(_t(x), _t(y), nl.bin_w, 1.0)
     assert dp.dp_debug_sort_stats(ctx)["sorts"] == 3
+
+
+@pytest.mark.parametrize("name,iters", [("adaptec1", 300)])
+def test_gp_trajectory_bitwise_with_reuse(name, iters):
+    """The GP loop (NEXT-1) over the kept list: from the P:153 start, where the clump spreads and
+    the list goes stale, the deterministic-mode trajectory (history and positions) is bit-identical
+    to the one that sorts every evaluation; the reusing run sorted fewer times."""
+    nl = make_netlist(name)
+    x, y = make_positions(nl, "initial")
+    runs = []
+    for env in ({"DP_REUSE_SORT": 1}, {"DP_REUSE_SORT": 0}):
+        ctx = _ctx(nl, **env)
+        loop = dp.GpLoop(ctx)
+        loop.init(_t(x), _t(y))
+        loop.run(iters)
+        h = loop.history()
+        ux, uy = loop.positions()
+        runs.append((h, ux.cpu().numpy(), uy.cpu().numpy(), dp.dp_debug_sort_stats(ctx)["sorts"]))
+        loop.close()
+    (h0, x0, y0, s0), (h1, x1, y1, s1) = runs
+    assert h0 == h1
+    assert np.array_equal(x0, x1) and np.array_equal(y0, y1)
+    assert s0 < s1

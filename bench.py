@@ -225,10 +225,24 @@ def run_reference(args, rank, world):
     budget = 150.0
     full = per_eval * (args.steps + args.warmup) <= budget
     frac = 1.0 if full else max(1e-3, budget / max(1, args.steps + args.warmup) / per_eval)
+    # the positions walk like our arm's (a seeded random walk of walk_sigma bins per axis and step,
+    # clamped to the region; the oracle's cost does not depend on them)
+    import numpy as np
+    rng = np.random.default_rng(3000)
+    pos = {"x": x.astype(np.float32), "y": y.astype(np.float32)}
+
+    def walk():
+        if args.walk_sigma > 0:
+            pos["x"] = np.minimum(np.maximum(pos["x"] + rng.normal(0, args.walk_sigma * nl.bin_w, nl.num_cells),
+                                             nl.xl), nl.xh - nl.cell_w).astype(np.float32)
+            pos["y"] = np.minimum(np.maximum(pos["y"] + rng.normal(0, args.walk_sigma * nl.bin_h, nl.num_cells),
+                                             nl.yl), nl.yh - nl.cell_h).astype(np.float32)
+        return pos["x"], pos["y"]
+
     if full:
-        step = lambda: timed_oracle_eval(nl, x, y, gamma, lam, nproc)   # noqa: E731
+        step = lambda: timed_oracle_eval(nl, *walk(), gamma, lam, nproc)   # noqa: E731
     else:
-        step = lambda: oracle_sample(nl, x, y, frac, gamma, lam)         # noqa: E731
+        step = lambda: oracle_sample(nl, *walk(), frac, gamma, lam)         # noqa: E731
     for _ in range(args.warmup):
         step()
     t0 = time.perf_counter()
@@ -243,7 +257,11 @@ def run_reference(args, rank, world):
     out = {"metric": METRIC, "value": value, "unit": UNIT, "impl": "reference", "n_gpus": args.gpus,
            "steps": args.steps, "warmup": args.warmup, "ms_per_step": dt / args.steps * 1e3,
            "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
-           "dtype": "f64", "data": "synthetic", "config": workload_config(nl, args.dist, 1),
+           "dtype": "f64", "data": "synthetic",
+           "config": dict(workload_config(nl, args.dist, 1),
+                          trajectory={"start": args.dist, "step_sigma_bins_per_axis": args.walk_sigma,
+                                      "note": "the same random walk recipe as our arm (numpy generator); "
+                                              "the oracle sorts nothing, its cost does not depend on it"}),
            "cpu_baseline": {"value": value, "unit": UNIT, "kind": "oracle", "cores": nproc, "sample": sample},
            "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(out), flush=True)

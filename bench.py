@@ -48,6 +48,8 @@ def parse():
     ap.add_argument("--e2e-steps", type=int, default=200)
     ap.add_argument("--walk-sigma", type=float, default=0.13,
                     help="random-walk step per axis in bins (GP-like motion, DESIGN.md §7); 0 = fixed positions")
+    ap.add_argument("--no-sort-every", action="store_true",
+                    help="skip the sort-every-evaluation comparison context (launch lists / ncu runs)")
     ap.add_argument("--skip-next", action="store_true",
                     help="skip the NEXT-row secondaries (LSE, deterministic, GP loop): profiling runs")
     return ap.parse_args()
@@ -418,7 +420,7 @@ def run_ours(args, rank, world, local_rank):
     fixed_ms = sum(cold_steps(min(K, 200), step)) / min(K, 200)
     # secondary: sorting on every evaluation (DP_REUSE_SORT=0 context), the same walk, L2-cold
     sort_every_ms = None
-    if world == 1:
+    if world == 1 and not args.no_sort_every:
         os.environ["DP_REUSE_SORT"] = "0"
         try:
             ctx_s = dp.dp_create(nl, local_rank)

@@ -39,7 +39,7 @@ namespace dp {
 
 namespace {
 
-constexpr int kTileThreads = 512;   // scatter / gather CTA size (smem-bound at 2 CTAs per SM)
+constexpr int kTileThreads = DP_WALK_THREADS;   // scatter / gather CTA size (smem-bound at 2 CTAs per SM)
 
 struct DenArgs {
   const float *x, *y;   // global cell arrays

@@ -63,7 +63,10 @@ constexpr int kHalo = 2;              // small-cell footprints extend <= 2 bins 
 #define DP_MARGIN 2   // -DDP_MARGIN=m: A/B builds (0 / 2 / 4 measured)
 #endif
 constexpr int kMargin = DP_MARGIN;
-constexpr int kStageRecs = 512;       // records per staging buffer of the scatter/gather walkers
+#ifndef DP_WALK_THREADS
+#define DP_WALK_THREADS 512   // -DDP_WALK_THREADS=256: A/B builds
+#endif
+constexpr int kStageRecs = DP_WALK_THREADS;   // records per staging buffer of the scatter/gather walkers (one per thread)
 // Tile bins accumulate each contribution v in (0, 1] as u = floor(v 2^29) in one native 32-bit
 // shared atomic (modulo 2^32; the thread whose add wraps carries 2^32 units to the int64 map).
 constexpr int kRhoScaleLog2 = 29;   // global bin map: int64 units of 2^-29

@@ -986,6 +986,16 @@ __global__ void __launch_bounds__(kWaThreads, 2) k_wa_chunks(const WaArgs a0) {
   __syncthreads();   // barrier initialised before anyone waits on it
   mbar_wait(bar, 0);
   // far cells: positions gathered once per chunk
+#ifndef DP_WA_FAR_LDG
+  // 4-byte cp.async global -> shared (no register round trip), completed before the barrier
+  // (the register path below, -DDP_WA_FAR_LDG: 5047-5055 vs 5064-5065 evals/s)
+  for (int f = tid; f < ch.far_n; f += kWaThreads) {
+    const int c = s_far[f];
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(smem_u32(s_px + kWaWindow + f)), "l"(a.x + c) : "memory");
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(smem_u32(s_py + kWaWindow + f)), "l"(a.y + c) : "memory");
+  }
+  asm volatile("cp.async.wait_all;" ::: "memory");
+#else
   for (int f0 = tid; f0 < ch.far_n; f0 += 4 * kWaThreads) {   // 8 loads in flight per thread
     float fx[4], fy[4];
 #pragma unroll
@@ -1004,6 +1014,7 @@ __global__ void __launch_bounds__(kWaThreads, 2) k_wa_chunks(const WaArgs a0) {
       }
     }
   }
+#endif
   mbar_wait(bar + 1, 0);
   __syncthreads();
 

@@ -61,6 +61,7 @@ struct DenArgs {
   // strays of this one (scatter), [3] sorts performed.  The sort kernels run when force_sort,
   // [0] or [1] > resort_thr, and return at once otherwise
   int *sortctl;
+  int *host_ctl;   // mapped pinned host word: the gather publishes the last evaluation's strays to the host
   int force_sort, resort_thr;
   int write_rec;   // the scatter writes footprint records (the gather reads them; 0: it recomputes)
   unsigned long long *rho;   // int64 fixed point, 2^-kRhoScaleLog2 units
@@ -817,8 +818,10 @@ __global__ void __launch_bounds__(kTileThreads) k_gather_walk(DenArgs a) {
   Walker w;
   if (threadIdx.x == 0) {
     if (blockIdx.x == 0) {   // the scatter has completed: its stray count decides the next sort
-      a.sortctl[1] = a.sortctl[2];
+      const int strays = a.sortctl[2];
+      a.sortctl[1] = strays;
       a.sortctl[2] = 0;
+      if (a.host_ctl) *(volatile int *)a.host_ctl = strays;   // the host's view (graph choice, §5.5)
     }
     walk_start(a, w, st);
   }
@@ -866,8 +869,10 @@ __global__ void __launch_bounds__(kTileThreads) k_gather_walk_rc(DenArgs a) {
   Walker w;
   if (threadIdx.x == 0) {
     if (blockIdx.x == 0) {   // the scatter has completed: its stray count decides the next sort
-      a.sortctl[1] = a.sortctl[2];
+      const int strays = a.sortctl[2];
+      a.sortctl[1] = strays;
       a.sortctl[2] = 0;
+      if (a.host_ctl) *(volatile int *)a.host_ctl = strays;   // the host's view (graph choice, §5.5)
     }
     walk_start(a, w, st);
   }
@@ -1052,6 +1057,7 @@ DenArgs make_args(const Ctx &c, const float *x, const float *y) {
   a.rec_cell = c.d_rec_cell;
   a.rec_wh = c.d_rec_wh;
   a.sortctl = c.d_sortctl;
+  a.host_ctl = c.h_ctl_dev;
   a.force_sort = c.reuse_sort ? 0 : 1;
   a.write_rec = c.gather_rc ? 0 : 1;
   a.resort_thr = c.resort_thr;
@@ -1166,7 +1172,8 @@ void launch_density_map(const Ctx &c, const float *x, const float *y, cudaStream
   // k_map_init: no launches at all when the list is kept (DP_SORT_COND=0: the kernels return early)
   cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
   cudaStreamIsCapturing(s, &cs);
-  const bool cond = nblk > 0 && !a.force_sort && c.sort_cond && c.s_body && cs == cudaStreamCaptureStatusActive;
+  const bool cond = nblk > 0 && !a.force_sort && !c.omit_sort && c.sort_cond && c.s_body &&
+                    cs == cudaStreamCaptureStatusActive;
   cudaStream_t ss = s;   // stream of D1-D3
   if (cond) {
     cudaGraph_t g = nullptr;
@@ -1199,7 +1206,10 @@ void launch_density_map(const Ctx &c, const float *x, const float *y, cudaStream
     k_scatter_large<<<a.n_large, 256, 0, aux>>>(a);
     cudaEventRecord(c.ev_aux_b, aux);
   }
-  if (nblk > 0) {
+  if (nblk > 0 && c.omit_sort && !a.force_sort) {   // captured while the list is kept: no sort kernels (§5.5)
+    if (c.sched == 2 || c.sched == 3) cudaEventRecord(c.ev_sched, s);
+    launch_chain(c.pdl, k_scatter_walk, c.walk_grid, kTileThreads, scatter_smem_bytes(c.tile), s, a);
+  } else if (nblk > 0) {
     const int cgrid = std::min(nblk, c.count_grid > 0 ? c.count_grid : nblk);
     if (a.fixed)
       launch_chain(c.pdl, k_count<true>, cgrid, kCountThreads, ntiles * 4, ss, a);

@@ -534,6 +534,13 @@ dp_status build_density(Ctx &c, const dp_netlist *nl) {
     c.reuse_sort = e ? std::atoi(e) != 0 : c.n_own >= (1 << 19);
     // DP_SORT_COND=1: the sort kernels inside a graph IF node instead of returning early (measured
     // equal at bigblue4, ~7 us slower per GP iteration at adaptec1)
+    const char *he = std::getenv("DP_SORT_HOST");
+    c.sort_host = !(he && std::atoi(he) == 0);
+    const char *se = std::getenv("DP_SORT_EVERY");
+    c.sort_every = se ? std::max(1, std::atoi(se)) : 8;
+    DP_CUDA(cudaHostAlloc(&c.h_ctl, sizeof(int32_t), cudaHostAllocMapped));
+    *c.h_ctl = 0;
+    DP_CUDA(cudaHostGetDevicePointer(reinterpret_cast<void **>(&c.h_ctl_dev), c.h_ctl, 0));
     const char *ge = std::getenv("DP_GATHER_RC");
     c.gather_rc = ge && std::atoi(ge) != 0;
     const char *fe = std::getenv("DP_FUSE_COMBINE");
@@ -625,7 +632,9 @@ void destroy(Ctx *c) {
   }
   if (c->s_h2d) cudaStreamDestroy(c->s_h2d);
   if (c->s_d2h) cudaStreamDestroy(c->s_d2h);
-  if (c->gexec) cudaGraphExecDestroy(c->gexec);
+  for (int v = 0; v < 2; v++)
+    if (c->gexec_v[v]) cudaGraphExecDestroy(c->gexec_v[v]);
+  if (c->h_ctl) cudaFreeHost(c->h_ctl);
   if (c->s_cap) cudaStreamDestroy(c->s_cap);
   if (c->s_wa) cudaStreamDestroy(c->s_wa);
   if (c->s_den) cudaStreamDestroy(c->s_den);
@@ -984,41 +993,51 @@ dp_status eval_body(Ctx &c, const float *x, const float *y, float gamma, float l
 dp_status eval_graph(Ctx &c, const float *x, const float *y, float gamma, float lambda, float *gx, float *gy,
                      double *d_obj, double *d_wl, double *d_energy, double *d_hpwl, cudaStream_t s, bool do_wa,
                      bool do_den) {
+  // the sort kernels are left out of the captured evaluation while the host's (possibly a few
+  // evaluations old) view of the stray count is below the re-sort threshold, except on every
+  // sort_every-th call (the device decides there); strays are handled exactly either way, so a
+  // late view only delays a sort
+  const int v = c.sort_variant();
+  const bool with_sort = v == 1;
   const GraphKey key{x, y, gx, gy, d_obj, d_wl, d_energy, d_hpwl, gamma, lambda, do_wa, do_den, c.wl_model,
-                     c.deterministic};
-  if (!(c.gexec && key == c.gkey)) {
+                     c.deterministic, with_sort};
+  cudaGraphExec_t &gexec = c.gexec_v[v];
+  if (!(gexec && key == c.gkey_v[v])) {
     cudaGraph_t g = nullptr;
     DP_CUDA(cudaStreamBeginCapture(c.s_cap, cudaStreamCaptureModeThreadLocal));
+    c.omit_sort = !with_sort;
     dp_status st = eval_body(c, x, y, gamma, lambda, gx, gy, d_obj, d_wl, d_energy, d_hpwl, c.s_cap, do_wa, do_den);
+    c.omit_sort = false;
     const cudaError_t ce = cudaStreamEndCapture(c.s_cap, &g);
     if (st != DP_OK) {
       if (g) cudaGraphDestroy(g);
       return st;
     }
     if (ce != cudaSuccess) return cuda_fail(ce, "cudaStreamEndCapture");
-    if (c.gexec) {
+    if (gexec) {
       cudaGraphExecUpdateResultInfo info;
-      if (cudaGraphExecUpdate(c.gexec, g, &info) != cudaSuccess) {
+      if (cudaGraphExecUpdate(gexec, g, &info) != cudaSuccess) {
         cudaGetLastError();
-        cudaGraphExecDestroy(c.gexec);
-        c.gexec = nullptr;
+        cudaGraphExecDestroy(gexec);
+        gexec = nullptr;
       }
     }
-    if (!c.gexec) {
+    if (!gexec) {
       // honour the captured stream priorities (density chain first), as in a stream launch
-      const cudaError_t ie = cudaGraphInstantiateWithFlags(&c.gexec, g, cudaGraphInstantiateFlagUseNodePriority);
+      const cudaError_t ie = cudaGraphInstantiateWithFlags(&gexec, g, cudaGraphInstantiateFlagUseNodePriority);
       if (ie != cudaSuccess) {
         cudaGraphDestroy(g);
-        c.gexec = nullptr;
+        gexec = nullptr;
         return cuda_fail(ie, "cudaGraphInstantiate");
       }
     }
     cudaGraphDestroy(g);
-    c.gkey = key;
+    c.gkey_v[v] = key;
   }
   dp_status st0 = call_begin(c, s);
   if (st0 != DP_OK) return st0;
-  DP_CUDA(cudaGraphLaunch(c.gexec, s));
+  DP_CUDA(cudaGraphLaunch(gexec, s));
+  if (with_sort && do_den) c.sorted_once = true;
   return call_end(c, s);
 }
 
@@ -1153,6 +1172,7 @@ dp_status eval_body_ext(Ctx &c, const float *x, const float *y, float gamma, flo
   return eval_body(c, x, y, gamma, lambda, gx, gy, d_obj, d_wl, d_energy, d_hpwl, s, do_wa, do_den);
 }
 dp_status request_sort(Ctx &c, cudaStream_t s) {
+  c.sorted_once = false;   // the next captured evaluation carries the sort kernels
   DP_CUDA(cudaMemsetAsync(c.d_sortctl, 0x01, sizeof(int32_t), s));   // word 0 != 0: sort requested
   return DP_OK;
 }
@@ -1276,12 +1296,13 @@ dp_status dp_set_fixed(dp_ctx *ctx, const uint8_t *h_fixed, const float *x, cons
   cudaStream_t s = (cudaStream_t)stream;
   dp_status st = dp::call_begin(*c, s);
   if (st != DP_OK) return st;
-  if (c->gexec) {   // the captured evaluation changes (map initialisation, masks): re-capture
-    DP_CUDA(cudaStreamSynchronize(s));
-    cudaGraphExecDestroy(c->gexec);
-    c->gexec = nullptr;
-    c->gkey = dp::GraphKey{};
-  }
+  DP_CUDA(cudaStreamSynchronize(s));   // the captured evaluation changes (map initialisation, masks): re-capture
+  for (int v = 0; v < 2; v++)
+    if (c->gexec_v[v]) {
+      cudaGraphExecDestroy(c->gexec_v[v]);
+      c->gexec_v[v] = nullptr;
+      c->gkey_v[v] = dp::GraphKey{};
+    }
   if (!h_fixed) {
     c->has_fixed = false;
     if ((st = dp::request_sort(*c, s)) != DP_OK) return st;   // the list lacks the formerly fixed cells
@@ -1340,11 +1361,12 @@ dp_status dp_set_regions(dp_ctx *ctx, int32_t n_regions, const double *h_boxes, 
   dp::DeviceGuard g(c->device);
   DP_CUDA(cudaDeviceSynchronize());
   c->config_gen++;
-  if (c->gexec) {   // the captured evaluation changes: re-capture
-    cudaGraphExecDestroy(c->gexec);
-    c->gexec = nullptr;
-    c->gkey = dp::GraphKey{};
-  }
+  for (int v = 0; v < 2; v++)   // the captured evaluation changes: re-capture
+    if (c->gexec_v[v]) {
+      cudaGraphExecDestroy(c->gexec_v[v]);
+      c->gexec_v[v] = nullptr;
+      c->gkey_v[v] = dp::GraphKey{};
+    }
   c->n_regions = 0;
   {   // the list was built for one region pass: the next evaluation sorts
     dp_status rs = dp::request_sort(*c, nullptr);

@@ -112,10 +112,11 @@ struct GraphKey {
   bool wa = false, den = false;
   int wl_model = 0;
   bool det = false;
+  bool sort = true;   // the sort kernels are in the graph
   bool operator==(const GraphKey &o) const {
     return x == o.x && y == o.y && gx == o.gx && gy == o.gy && obj == o.obj && wl == o.wl && en == o.en &&
            hpwl == o.hpwl && gamma == o.gamma && lambda == o.lambda && wa == o.wa && den == o.den &&
-           wl_model == o.wl_model && det == o.det;
+           wl_model == o.wl_model && det == o.det && sort == o.sort;
   }
 };
 
@@ -199,13 +200,28 @@ struct Ctx {
   int32_t resort_thr = 0;
   bool reuse_sort = true;             // DP_REUSE_SORT=0/1 (default: >= 2^19 own cells): keep the list between sorts
   bool gather_rc = false;             // DP_GATHER_RC=1: the gather recomputes footprints (no records)
-  bool sort_cond = false;             // DP_SORT_COND=1: the sort in an IF node of captured evaluations (A/B)
+  bool sort_cond = false;
+  bool sort_host = true;              // DP_SORT_HOST=0: every captured evaluation carries the sort kernels
+  bool sorted_once = false;           // a graph with the sort kernels has run since the last sort request
+  int32_t *h_ctl = nullptr;           // mapped pinned host word: strays of the last evaluation (the gather writes it)
+  int32_t *h_ctl_dev = nullptr;       // its device address
+  int32_t sort_every = 8;             // DP_SORT_EVERY: every k-th captured evaluation carries the sort kernels anyway
+  int64_t sort_tick = 0;
+  // the graph variant of the next captured evaluation (or GP iteration): 1 = with the sort kernels
+  int sort_variant() {
+    const bool kept = sort_host && sorted_once && reuse_sort && n_regions == 0 && h_ctl &&
+                      *reinterpret_cast<volatile int32_t *>(h_ctl) <= resort_thr;
+    return (!kept || ++sort_tick % sort_every == 0) ? 1 : 0;
+  }
+  mutable bool omit_sort = false;     // set while capturing a graph without the sort kernels             // DP_SORT_COND=1: the sort in an IF node of captured evaluations (A/B)
   cudaStream_t s_body = nullptr;      // captures the body of the sort's IF node
   bool serial = false;
   bool use_graph = true;   // DP_GRAPH=0 disables the captured-graph evaluation path
   cudaStream_t s_cap = nullptr;
-  cudaGraphExec_t gexec = nullptr;
-  GraphKey gkey;
+  // captured evaluations: [1] with the sort kernels (they return at once unless a sort is due),
+  // [0] without them (the host saw few strays in the last evaluations)
+  cudaGraphExec_t gexec_v[2] = {nullptr, nullptr};
+  GraphKey gkey_v[2];
   int wl_model = 0;        // DP_WL_WA / DP_WL_LSE (dp_set_wl_model)
   bool deterministic = false;     // dp_set_deterministic (NEXT-2): WA gradient as exact int64 sums
   bool hpwl_fast = false;         // GP loop: HPWL from fp32 pin positions fused into the fast WA path (A37)

@@ -350,8 +350,8 @@ struct Gp {
   GpDev *dev = nullptr;
   double *out = nullptr;     // {obj, wl, energy, hpwl}
   cudaStream_t s_cap = nullptr;
-  cudaGraphExec_t gexec = nullptr;
-  int64_t gexec_gen = -1;    // Ctx::config_gen the iteration graph was captured with
+  cudaGraphExec_t gexec_v[2] = {nullptr, nullptr};   // captured iterations without / with the sort kernels
+  int64_t gexec_gen_v[2] = {-1, -1};   // Ctx::config_gen the iteration graphs were captured with
   int64_t gen = -1;          // Ctx::config_gen of the last gp_refresh
   double *region_ovf_buf = nullptr;   // fence regions: overflow partials of the density passes
   size_t region_ovf_cap = 0;
@@ -374,7 +374,8 @@ dp_status gp_alloc(Gp &g, T **p, size_t n) {
 
 void gp_free(Gp *g) {
   if (!g) return;
-  if (g->gexec) cudaGraphExecDestroy(g->gexec);
+  for (int v = 0; v < 2; v++)
+    if (g->gexec_v[v]) cudaGraphExecDestroy(g->gexec_v[v]);
   if (g->s_cap) cudaStreamDestroy(g->s_cap);
   for (void *q : g->allocs) cudaFree(q);
   delete g;
@@ -634,31 +635,42 @@ dp_status dp_gp_run(dp_gp *gp, int32_t iterations, dp_stream_t stream) {
       if ((st = dp::gp_iteration(*g, s)) != DP_OK) return st;
     return dp::ctx_call_end(c, s);
   }
-  if (g->gexec && g->gexec_gen != c.config_gen) {   // dp_set_* since the capture: the body changed
-    cudaGraphExecDestroy(g->gexec);
-    g->gexec = nullptr;
-  }
-  if (!g->gexec) {   // capture one iteration once; replay it per iteration
+  for (int v = 0; v < 2; v++)
+    if (g->gexec_v[v] && g->gexec_gen_v[v] != c.config_gen) {   // dp_set_* since the capture: the body changed
+      cudaGraphExecDestroy(g->gexec_v[v]);
+      g->gexec_v[v] = nullptr;
+    }
+  // two captured iterations: [1] with the density sort kernels, [0] without (the list is kept;
+  // chosen per iteration like the evaluation graphs)
+  auto capture = [&](int v) -> dp_status {
     cudaGraph_t graph = nullptr;
     DP_CUDA(cudaStreamBeginCapture(g->s_cap, cudaStreamCaptureModeThreadLocal));
+    c.omit_sort = v == 0;
     dp_status st = dp::gp_iteration(*g, g->s_cap);
+    c.omit_sort = false;
     const cudaError_t ce = cudaStreamEndCapture(g->s_cap, &graph);
     if (st != DP_OK) {
       if (graph) cudaGraphDestroy(graph);
       return st;
     }
     if (ce != cudaSuccess) return dp::cuda_fail(ce, "cudaStreamEndCapture (gp)");
-    const cudaError_t ie = cudaGraphInstantiateWithFlags(&g->gexec, graph, cudaGraphInstantiateFlagUseNodePriority);
+    const cudaError_t ie = cudaGraphInstantiateWithFlags(&g->gexec_v[v], graph, cudaGraphInstantiateFlagUseNodePriority);
     cudaGraphDestroy(graph);
     if (ie != cudaSuccess) {
-      g->gexec = nullptr;
+      g->gexec_v[v] = nullptr;
       return dp::cuda_fail(ie, "cudaGraphInstantiate (gp)");
     }
-    g->gexec_gen = c.config_gen;
-  }
+    g->gexec_gen_v[v] = c.config_gen;
+    return DP_OK;
+  };
   dp_status st = dp::ctx_call_begin(c, s);
   if (st != DP_OK) return st;
-  for (int it = 0; it < iterations; it++) DP_CUDA(cudaGraphLaunch(g->gexec, s));
+  for (int it = 0; it < iterations; it++) {
+    const int v = c.sort_variant();
+    if (!g->gexec_v[v] && (st = capture(v)) != DP_OK) return st;
+    DP_CUDA(cudaGraphLaunch(g->gexec_v[v], s));
+    if (v == 1) c.sorted_once = true;
+  }
   return dp::ctx_call_end(c, s);
 }
 

@@ -63,6 +63,9 @@ struct DenArgs {
   int *sortctl;
   int *host_ctl;   // mapped pinned host word: the gather publishes the last evaluation's strays to the host
   int force_sort, resort_thr;
+  int early_gather;   // (gather) the ring starts before griddepcontrol.wait (DP_EARLY_GATHER=0: at the top)
+  int early;       // (scatter) the predecessor writes only the map: ring start, list copies and the first
+                   // position loads run before griddepcontrol.wait
   int write_rec;   // the scatter writes footprint records (the gather reads them; 0: it recomputes)
   unsigned long long *rho;   // int64 fixed point, 2^-kRhoScaleLog2 units
   const float2 *xi;
@@ -620,7 +623,7 @@ __device__ __forceinline__ FootRec make_rec(const DenArgs &a, const ScatterIn &i
 }
 
 __global__ void __launch_bounds__(kTileThreads) k_scatter_walk(DenArgs a) {
-  griddep_wait();
+  if (!a.early) griddep_wait();
   extern __shared__ __align__(16) unsigned char dsm[];
   StageS &st = *reinterpret_cast<StageS *>(dsm);
   unsigned *s_acc = reinterpret_cast<unsigned *>(dsm + stage_bytes<StageS>());   // 2^-29 units, mod 2^32
@@ -640,6 +643,7 @@ __global__ void __launch_bounds__(kTileThreads) k_scatter_walk(DenArgs a) {
   WalkChunk cc = walk_next(a, w, st, 0);
   ScatterIn in = {0, make_float2(0.f, 0.f), 0.f, 0.f};
   scatter_fetch(a, st, 0, cc, in);
+  if (a.early) griddep_wait();   // the map is zeroed: from here on it is written
   for (int c = 0; cc.begin < cc.end; c++) {
     const int n = cc.end - cc.begin;
     if (cc.tile != cur_tile) {   // uniform: every warp sees the same chunks
@@ -810,7 +814,9 @@ __device__ __forceinline__ void load_xi_tile(const DenArgs &a, St &st, float2 *s
 }
 
 __global__ void __launch_bounds__(kTileThreads) k_gather_walk(DenArgs a) {
-  griddep_wait();
+  if (!a.early_gather) griddep_wait();
+  // the records were written by the scatter, which completed before the transforms began: the ring
+  // starts before griddepcontrol.wait, which only the field (the predecessor's output) needs
   extern __shared__ __align__(16) unsigned char dsm[];
   StageG &st = *reinterpret_cast<StageG *>(dsm);
   float2 *s_xi = reinterpret_cast<float2 *>(dsm + stage_bytes<StageG>());
@@ -826,6 +832,7 @@ __global__ void __launch_bounds__(kTileThreads) k_gather_walk(DenArgs a) {
     walk_start(a, w, st);
   }
   __syncthreads();   // barriers initialised, first descriptors visible
+  if (a.early_gather) griddep_wait();   // the field of the transform pass before this kernel
   int cur_tile = -1;
   unsigned xi_phase = 0;
   const float area = (float)(a.bx * a.by);
@@ -860,7 +867,7 @@ __global__ void __launch_bounds__(kTileThreads) k_gather_walk(DenArgs a) {
 int gather_rc_smem_bytes(int tile) { return stage_bytes<StageS>() + walk_span(tile) * walk_span(tile) * 8; }
 
 __global__ void __launch_bounds__(kTileThreads) k_gather_walk_rc(DenArgs a) {
-  griddep_wait();
+  if (!a.early_gather) griddep_wait();
   extern __shared__ __align__(16) unsigned char dsm[];
   StageS &st = *reinterpret_cast<StageS *>(dsm);
   float2 *s_xi = reinterpret_cast<float2 *>(dsm + stage_bytes<StageS>());
@@ -877,6 +884,7 @@ __global__ void __launch_bounds__(kTileThreads) k_gather_walk_rc(DenArgs a) {
     walk_start(a, w, st);
   }
   __syncthreads();   // barriers initialised, first descriptors visible
+  if (a.early_gather) griddep_wait();   // the field of the transform pass before this kernel
   int cur_tile = -1, tox = 0, toy = 0;
   unsigned xi_phase = 0;
   const float area = (float)(a.bx * a.by);
@@ -1003,6 +1011,15 @@ __global__ void __launch_bounds__(256) k_region_overflow(const unsigned long lon
   }
 }
 
+// rho <- 0 as a kernel (not a memset node), so that the scatter walker can follow it with a
+// programmatic dependency and run its prologue while the map is cleared
+__global__ void __launch_bounds__(256) k_zero_map(unsigned long long *rho, long long nbins) {
+  ulonglong2 *d = reinterpret_cast<ulonglong2 *>(rho);
+  const long long n2 = nbins >> 1;   // maps are even-sized
+  for (long long i = blockIdx.x * 256ll + threadIdx.x; i < n2; i += (long long)gridDim.x * 256)
+    d[i] = make_ulonglong2(0ull, 0ull);
+}
+
 // Start of the map in a captured evaluation: rho <- src (the fixed-charge map) or 0, and the
 // graph's IF node around D1-D3 is set to "sort needed" (sort reuse: the count, scan and place
 // launches are skipped altogether when the list is kept).
@@ -1060,6 +1077,8 @@ DenArgs make_args(const Ctx &c, const float *x, const float *y) {
   a.host_ctl = c.h_ctl_dev;
   a.force_sort = c.reuse_sort ? 0 : 1;
   a.write_rec = c.gather_rc ? 0 : 1;
+  a.early = 0;
+  a.early_gather = c.early_gather ? 1 : 0;
   a.resort_thr = c.resort_thr;
   a.rho = c.d_rho;
   a.xi = c.d_xi;
@@ -1175,6 +1194,9 @@ void launch_density_map(const Ctx &c, const float *x, const float *y, cudaStream
   const bool cond = nblk > 0 && !a.force_sort && !c.omit_sort && c.sort_cond && c.s_body &&
                     cs == cudaStreamCaptureStatusActive;
   cudaStream_t ss = s;   // stream of D1-D3
+  // the graph variant without the sort kernels: the scatter follows a zeroing kernel
+  // programmatically and starts its prologue early (DP_EARLY=0: memset and a plain dependency)
+  const bool early = nblk > 0 && c.omit_sort && !a.force_sort && !cond && c.pdl && c.early_scatter;
   if (cond) {
     cudaGraph_t g = nullptr;
     const cudaGraphNode_t *deps = nullptr;
@@ -1196,6 +1218,8 @@ void launch_density_map(const Ctx &c, const float *x, const float *y, cudaStream
     ss = c.s_body;
   } else if (src) {
     cudaMemcpyAsync(c.d_rho, src, sizeof(unsigned long long) * nb, cudaMemcpyDeviceToDevice, s);
+  } else if (early) {
+    k_zero_map<<<2 * c.num_sms, 256, 0, s>>>(c.d_rho, (long long)nb);
   } else {
     cudaMemsetAsync(c.d_rho, 0, sizeof(unsigned long long) * nb, s);
   }
@@ -1208,6 +1232,7 @@ void launch_density_map(const Ctx &c, const float *x, const float *y, cudaStream
   }
   if (nblk > 0 && c.omit_sort && !a.force_sort) {   // captured while the list is kept: no sort kernels (§5.5)
     if (c.sched == 2 || c.sched == 3) cudaEventRecord(c.ev_sched, s);
+    a.early = early && !src ? 1 : 0;
     launch_chain(c.pdl, k_scatter_walk, c.walk_grid, kTileThreads, scatter_smem_bytes(c.tile), s, a);
   } else if (nblk > 0) {
     const int cgrid = std::min(nblk, c.count_grid > 0 ? c.count_grid : nblk);

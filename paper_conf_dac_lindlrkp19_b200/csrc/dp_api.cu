@@ -536,6 +536,10 @@ dp_status build_density(Ctx &c, const dp_netlist *nl) {
     // equal at bigblue4, ~7 us slower per GP iteration at adaptec1)
     const char *he = std::getenv("DP_SORT_HOST");
     c.sort_host = !(he && std::atoi(he) == 0);
+    const char *eg = std::getenv("DP_EARLY_GATHER");
+    c.early_gather = !(eg && std::atoi(eg) == 0);
+    const char *ee = std::getenv("DP_EARLY");
+    c.early_scatter = !(ee && std::atoi(ee) == 0);
     const char *se = std::getenv("DP_SORT_EVERY");
     c.sort_every = se ? std::max(1, std::atoi(se)) : 8;
     DP_CUDA(cudaHostAlloc(&c.h_ctl, sizeof(int32_t), cudaHostAllocMapped));

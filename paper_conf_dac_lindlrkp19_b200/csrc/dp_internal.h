@@ -201,6 +201,8 @@ struct Ctx {
   bool reuse_sort = true;             // DP_REUSE_SORT=0/1 (default: >= 2^19 own cells): keep the list between sorts
   bool gather_rc = false;             // DP_GATHER_RC=1: the gather recomputes footprints (no records)
   bool sort_cond = false;
+  bool early_gather = true;           // DP_EARLY_GATHER=0: the gather waits for its predecessor at the top
+  bool early_scatter = true;          // DP_EARLY=0: the no-sort variant keeps the memset and a plain dependency
   bool sort_host = true;              // DP_SORT_HOST=0: every captured evaluation carries the sort kernels
   bool sorted_once = false;           // a graph with the sort kernels has run since the last sort request
   int32_t *h_ctl = nullptr;           // mapped pinned host word: strays of the last evaluation (the gather writes it)

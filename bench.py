@@ -641,8 +641,8 @@ def run_ours(args, rank, world, local_rank):
                 "synchronous_dp_eval_host_per_s": e2e_sync_per_s},
         "secondary": secondary,
         # the captured evaluation leaves out the three sort kernels while the list is kept, except on
-        # every 8th call (contexts of >= 2^19 own cells)
-        "gpu_launches": (info.launches_eval * K if (world > 1 or nl.num_cells < (1 << 19))
+        # every 8th call (single-GPU contexts)
+        "gpu_launches": (info.launches_eval * K if world > 1
                          else (info.launches_eval - 3) * K + 3 * ((K + 7) // 8)),
         "clocks": clocks,
     }

@@ -527,11 +527,12 @@ dp_status build_density(Ctx &c, const dp_netlist *nl) {
   {
     const int32_t ctl[4] = {1, 0, 0, 0};   // the first evaluation sorts
     DP_CUDA(cudaMemcpy(c.d_sortctl, ctl, sizeof(ctl), cudaMemcpyHostToDevice));
-    // DP_REUSE_SORT: 1 / 0 force; unset: reuse for contexts of >= 2^19 own cells.  Measured on the
-    // GP trajectory from the P:153 start: bigblue4 (2.18M cells) 418 -> 364 us per
-    // iteration with reuse, adaptec1 (211K cells, whose sort costs ~10 us) 114 -> 120 us
+    // DP_REUSE_SORT=0: sort on every evaluation.  Reuse is the default at every size since the
+    // sort kernels are left out of the captured graph: adaptec1 13210 -> 15350
+    // evals/s on the walk, GP 113 -> 112 us per iteration (with the kernels returning early instead,
+    // reuse had measured slower there: 114 -> 120 us)
     const char *e = std::getenv("DP_REUSE_SORT");
-    c.reuse_sort = e ? std::atoi(e) != 0 : c.n_own >= (1 << 19);
+    c.reuse_sort = e ? std::atoi(e) != 0 : true;
     // DP_SORT_COND=1: the sort kernels inside a graph IF node instead of returning early (measured
     // equal at bigblue4, ~7 us slower per GP iteration at adaptec1)
     const char *he = std::getenv("DP_SORT_HOST");

@@ -198,7 +198,7 @@ struct Ctx {
   // strays (cells outside the tile they were listed in) exceed resort_thr
   int32_t *d_sortctl = nullptr;
   int32_t resort_thr = 0;
-  bool reuse_sort = true;             // DP_REUSE_SORT=0/1 (default: >= 2^19 own cells): keep the list between sorts
+  bool reuse_sort = true;             // DP_REUSE_SORT=0: sort on every evaluation (default: keep the list between sorts)
   bool gather_rc = false;             // DP_GATHER_RC=1: the gather recomputes footprints (no records)
   bool sort_cond = false;
   bool early_gather = true;           // DP_EARLY_GATHER=0: the gather waits for its predecessor at the top

@@ -66,6 +66,7 @@ struct DenArgs {
   int early_gather;   // (gather) the ring starts before griddepcontrol.wait (DP_EARLY_GATHER=0: at the top)
   int early;       // (scatter) the predecessor writes only the map: ring start, list copies and the first
                    // position loads run before griddepcontrol.wait
+  int rec_hint;    // DP_REC_HINT=1: records stored evict-last by the scatter, read evict-first by the gather
   int write_rec;   // the scatter writes footprint records (the gather reads them; 0: it recomputes)
   unsigned long long *rho;   // int64 fixed point, 2^-kRhoScaleLog2 units
   const float2 *xi;
@@ -402,8 +403,14 @@ int walk_smem_bytes(int tile) { return stage_bytes<StageG>() + walk_span(tile) *
 
 __device__ __forceinline__ unsigned issue_copies(const DenArgs &a, RecBufG &B, int b0, int n, uint64_t *bar) {
   if (n > 0) {
-    bulk_g2s(B.rec, a.rec + b0, 16u * n, bar);
-    bulk_g2s(B.rc, a.rec_rc + b0, 8u * n, bar);
+    if (a.rec_hint) {   // the records' last use: evict-first
+      const uint64_t pol = l2_evict_first_policy();
+      bulk_g2s_hint(B.rec, a.rec + b0, 16u * n, bar, pol);
+      bulk_g2s_hint(B.rc, a.rec_rc + b0, 8u * n, bar, pol);
+    } else {
+      bulk_g2s(B.rec, a.rec + b0, 16u * n, bar);
+      bulk_g2s(B.rc, a.rec_rc + b0, 8u * n, bar);
+    }
     bulk_g2s(B.cell, a.rec_cell + b0, 4u * n, bar);
   }
   return 28u;
@@ -637,6 +644,8 @@ __global__ void __launch_bounds__(kTileThreads) k_scatter_walk(DenArgs a) {
   for (int k = threadIdx.x; k < P * P; k += blockDim.x) s_acc[k] = 0u;
   __syncthreads();
   const float scale_fx = (float)(1u << kRhoScaleLog2);
+  uint64_t pol_last = 0;
+  if (a.rec_hint) asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol_last));
   int cur_tile = -1;
   int tox = 0, toy = 0;   // origin of the shared tile (first bin of the tile - kMargin)
   unsigned strays = 0;
@@ -717,8 +726,17 @@ __global__ void __launch_bounds__(kTileThreads) k_scatter_walk(DenArgs a) {
         }
       }
       if (a.write_rec) {   // the records of the record-reading gather
-        a.rec[cc.begin + threadIdx.x] = q;
-        a.rec_rc[cc.begin + threadIdx.x] = rc;
+        if (a.rec_hint) {   // kept in L2 for the gather (evict-last)
+          asm volatile("st.global.L2::cache_hint.v4.f32 [%0], {%1, %2, %3, %4}, %5;" ::"l"(a.rec + cc.begin + threadIdx.x),
+                       "f"(q.x), "f"(q.y), "f"(q.z), "f"(q.w), "l"(pol_last)
+                       : "memory");
+          asm volatile("st.global.L2::cache_hint.v2.s32 [%0], {%1, %2}, %3;" ::"l"(a.rec_rc + cc.begin + threadIdx.x),
+                       "r"(rc.x), "r"(rc.y), "l"(pol_last)
+                       : "memory");
+        } else {
+          a.rec[cc.begin + threadIdx.x] = q;
+          a.rec_rc[cc.begin + threadIdx.x] = rc;
+        }
       }
     }
     walk_release(st, c);
@@ -1077,6 +1095,7 @@ DenArgs make_args(const Ctx &c, const float *x, const float *y) {
   a.host_ctl = c.h_ctl_dev;
   a.force_sort = c.reuse_sort ? 0 : 1;
   a.write_rec = c.gather_rc ? 0 : 1;
+  a.rec_hint = c.rec_hint ? 1 : 0;
   a.early = 0;
   a.early_gather = c.early_gather ? 1 : 0;
   a.resort_thr = c.resort_thr;

@@ -537,6 +537,8 @@ dp_status build_density(Ctx &c, const dp_netlist *nl) {
     // equal at bigblue4, ~7 us slower per GP iteration at adaptec1)
     const char *he = std::getenv("DP_SORT_HOST");
     c.sort_host = !(he && std::atoi(he) == 0);
+    const char *rh = std::getenv("DP_REC_HINT");
+    c.rec_hint = rh && std::atoi(rh) != 0;
     const char *eg = std::getenv("DP_EARLY_GATHER");
     c.early_gather = !(eg && std::atoi(eg) == 0);
     const char *ee = std::getenv("DP_EARLY");

@@ -66,6 +66,7 @@ struct DenArgs {
   int early_gather;   // (gather) the ring starts before griddepcontrol.wait (DP_EARLY_GATHER=0: at the top)
   int early;       // (scatter) the predecessor writes only the map: ring start, list copies and the first
                    // position loads run before griddepcontrol.wait
+  int merge;       // walker slices per CTA (the scatter with DP_SCATTER_MERGE = 2: one CTA per SM)
   int rec_hint;    // DP_REC_HINT=1: records stored evict-last by the scatter, read evict-first by the gather
   int write_rec;   // the scatter writes footprint records (the gather reads them; 0: it recomputes)
   unsigned long long *rho;   // int64 fixed point, 2^-kRhoScaleLog2 units
@@ -430,14 +431,15 @@ struct Walker {
 };
 
 __device__ __forceinline__ void walk_init(const DenArgs &a, Walker &w) {
+  // a CTA covers a.merge consecutive walker slices (the scatter with DP_SCATTER_MERGE; else 1)
   const int N = a.tile_off[a.ntiles];
-  const int G = gridDim.x;
-  w.cur = (int)(((long long)N * blockIdx.x) / G);
-  w.re = (int)(((long long)N * (blockIdx.x + 1)) / G);
+  const int m = a.merge, G = gridDim.x * m, g0 = blockIdx.x * m;
+  w.cur = (int)(((long long)N * g0) / G);
+  w.re = (int)(((long long)N * (g0 + m)) / G);
   w.t = 0;
   w.tend = 0;
   if (w.cur >= w.re) return;
-  w.t = a.walk_tile[blockIdx.x];   // from D2: tile_off[t] <= cur < tile_off[t + 1]
+  w.t = a.walk_tile[g0];   // from D2: tile_off[t] <= cur < tile_off[t + 1]
   w.tend = a.tile_off[w.t + 1];
 }
 
@@ -1096,6 +1098,7 @@ DenArgs make_args(const Ctx &c, const float *x, const float *y) {
   a.force_sort = c.reuse_sort ? 0 : 1;
   a.write_rec = c.gather_rc ? 0 : 1;
   a.rec_hint = c.rec_hint ? 1 : 0;
+  a.merge = 1;
   a.early = 0;
   a.early_gather = c.early_gather ? 1 : 0;
   a.resort_thr = c.resort_thr;
@@ -1252,7 +1255,8 @@ void launch_density_map(const Ctx &c, const float *x, const float *y, cudaStream
   if (nblk > 0 && c.omit_sort && !a.force_sort) {   // captured while the list is kept: no sort kernels (§5.5)
     if (c.sched == 2 || c.sched == 3) cudaEventRecord(c.ev_sched, s);
     a.early = early && !src ? 1 : 0;
-    launch_chain(c.pdl, k_scatter_walk, c.walk_grid, kTileThreads, scatter_smem_bytes(c.tile), s, a);
+    a.merge = c.scatter_merge;
+    launch_chain(c.pdl, k_scatter_walk, c.walk_grid / c.scatter_merge, kTileThreads, scatter_smem_bytes(c.tile), s, a);
   } else if (nblk > 0) {
     const int cgrid = std::min(nblk, c.count_grid > 0 ? c.count_grid : nblk);
     if (a.fixed)
@@ -1278,7 +1282,8 @@ void launch_density_map(const Ctx &c, const float *x, const float *y, cudaStream
     }
     if (c.sched == 2 || (c.sched == 3 && cond)) cudaEventRecord(c.ev_sched, s);   // DP_SCHED=2: WA starts after the placement
     // after the IF node the walker is an ordinary dependent (programmatic edges join kernel nodes)
-    launch_chain(c.pdl && !cond, k_scatter_walk, c.walk_grid, kTileThreads, scatter_smem_bytes(c.tile), s, a);
+    a.merge = c.scatter_merge;
+    launch_chain(c.pdl && !cond, k_scatter_walk, c.walk_grid / c.scatter_merge, kTileThreads, scatter_smem_bytes(c.tile), s, a);
   }
   if (side)
     cudaStreamWaitEvent(s, c.ev_aux_b, 0);

@@ -537,6 +537,8 @@ dp_status build_density(Ctx &c, const dp_netlist *nl) {
     // equal at bigblue4, ~7 us slower per GP iteration at adaptec1)
     const char *he = std::getenv("DP_SORT_HOST");
     c.sort_host = !(he && std::atoi(he) == 0);
+    const char *sm = std::getenv("DP_SCATTER_MERGE");
+    c.scatter_merge = sm && std::atoi(sm) == 2 ? 2 : 1;
     const char *rh = std::getenv("DP_REC_HINT");
     c.rec_hint = rh && std::atoi(rh) != 0;
     const char *eg = std::getenv("DP_EARLY_GATHER");
@@ -615,6 +617,7 @@ dp_status build_density(Ctx &c, const dp_netlist *nl) {
     const int k = e ? std::max(1, std::atoi(e)) : 1;
     c.walk_grid *= k;
   }
+  if (c.walk_grid % c.scatter_merge) c.scatter_merge = 1;   // merged scatter slices need an even grid
   if ((st = dev_alloc(c, &c.d_walk_tile, c.walk_grid)) != DP_OK) return st;
   DP_CUDA(cudaMemset(c.d_walk_tile, 0, sizeof(int32_t) * c.walk_grid));
   return DP_OK;

@@ -201,6 +201,7 @@ struct Ctx {
   bool reuse_sort = true;             // DP_REUSE_SORT=0: sort on every evaluation (default: keep the list between sorts)
   bool gather_rc = false;             // DP_GATHER_RC=1: the gather recomputes footprints (no records)
   bool sort_cond = false;
+  int scatter_merge = 1;              // DP_SCATTER_MERGE=2: the scatter runs one CTA per two walker slices (A/B)
   bool rec_hint = false;              // DP_REC_HINT=1: L2 evict-last records (scatter) / evict-first reads (gather)
   bool early_gather = true;           // DP_EARLY_GATHER=0: the gather waits for its predecessor at the top
   bool early_scatter = true;          // DP_EARLY=0: the no-sort variant keeps the memset and a plain dependency

@@ -1060,8 +1060,14 @@ dp_status eval_impl(Ctx &c, const float *x, const float *y, float gamma, float l
     return eval_graph(c, x, y, gamma, lambda, gx, gy, d_obj, d_wl, d_energy, d_hpwl, s, do_wa, do_den);
   dp_status st0 = call_begin(c, s);
   if (st0 != DP_OK) return st0;
+  // direct launches (profiling, DP_GRAPH=0, multi-GPU contexts) choose the sort variant per call
+  // like the captured graphs (§5.5); a caller's own capture always carries the sort kernels
+  const int v = cs == cudaStreamCaptureStatusNone ? c.sort_variant() : 1;
+  c.omit_sort = v == 0;
   st0 = eval_body(c, x, y, gamma, lambda, gx, gy, d_obj, d_wl, d_energy, d_hpwl, s, do_wa, do_den);
+  c.omit_sort = false;
   if (st0 != DP_OK) return st0;
+  if (v == 1 && do_den) c.sorted_once = true;
   return call_end(c, s);
 }
 
